@@ -1,0 +1,448 @@
+#!/usr/bin/env python
+"""TT-EmbeddingBag fwd+bwd(+update) throughput on B200 (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c4] [--rank R]
+                    [--impl ours|reference] [--opt sgd|adagrad] [--ids identity|perm]
+
+One "step" = the whole hot path over one synthetic batch: index stage (sort /
+unique / inverse / prefixes), prefix + row contractions, pooling, in-advance
+aggregation, core-gradient contractions and the core update (fused when N=1;
+NCCL all-reduce of the core gradients + update when N>1).  Prints ONE JSON line
+on rank 0.  `--impl reference` times the CPU oracle (the tier's reference arm).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from synth import workload as W  # noqa: E402
+
+METRIC = "TT-EmbeddingBag fwd+bwd lookups/sec"
+UNIT = "lookups/s"
+HBM_PEAK_FALLBACK = 6650.0
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d.get("hbm_gbs", HBM_PEAK_FALLBACK)), float(d.get("sm_max_mhz", 1965.0)), "measured"
+    return HBM_PEAK_FALLBACK, 1965.0, "fallback"
+
+
+def fp32_peak_tflops(sm_count: int, mhz: float) -> float:
+    """FP32 FFMA peak: SMs x 128 FP32 lanes x 2 flop x clock."""
+    return sm_count * 128 * 2 * mhz * 1e6 / 1e12
+
+
+# ---------------------------------------------------------------------------
+# clocks sampling during the timed region
+# ---------------------------------------------------------------------------
+class Clocks:
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.gpu = gpu_index
+        self.rows = []
+        self._stop = threading.Event()
+        self._th = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                out = subprocess.run(["nvidia-smi", f"--id={self.gpu}", f"--query-gpu={self.Q}",
+                                      "--format=csv,noheader,nounits"], capture_output=True,
+                                     text=True, timeout=5).stdout.strip()
+                if out:
+                    self.rows.append([x.strip() for x in out.split(",")])
+            except Exception:
+                pass
+            self._stop.wait(0.2)
+
+    def __enter__(self):
+        self._th = threading.Thread(target=self._run, daemon=True)
+        self._th.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self._th:
+            self._th.join(timeout=10)
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"], "samples": 0}
+        sm = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in self.rows if r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for r in self.rows:
+            for n, v in zip(names, r[5:9]):
+                if v.strip().lower() == "active":
+                    reasons.add(n)
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(self.rows)}
+
+
+# ---------------------------------------------------------------------------
+# algorithmic work
+# ---------------------------------------------------------------------------
+def step_work(cfg, B, nnz, counts, touched, opt):
+    n1, n2, n3 = cfg.col_factors
+    R, N, T = cfg.rank, cfg.dim, cfg.num_tables
+    U, P = counts["U"], counts["P"]
+    flops = 3 * 2 * n1 * n2 * R * R * P + 3 * 2 * N * R * U
+    slice_bytes = 4 * (touched["c1"] * n1 * R + touched["c2"] * R * n2 * R + touched["c3"] * R * n3)
+    passes = 3 if opt == "sgd" else 5                  # fwd read, bwd read, update write (+ state r/w)
+    bytes_ = 8 * nnz + 8 * (T * B + 1) + 2 * 4 * N * T * B + passes * slice_bytes
+    return flops, bytes_
+
+
+def stage_work(name, cfg, B, nnz, counts):
+    """(flops, bytes, bound) of one launch of a stage, algorithmic."""
+    n1, n2, n3 = cfg.col_factors
+    R, N, T = cfg.rank, cfg.dim, cfg.num_tables
+    U, P, NG = counts["U"], counts["P"], counts["NG"]
+    if name == "fwd_prefix":
+        return 2 * n1 * n2 * R * R * P, 4 * (NG * R * n2 * R + P * n1 * R), "alu"
+    if name == "bwd_prefix":
+        return 4 * n1 * n2 * R * R * P, 4 * (2 * NG * R * n2 * R + P * n1 * R), "alu"
+    if name == "fwd_rows":
+        return 2 * N * R * U, 4 * U * N, "alu"
+    if name == "bwd_rows":
+        return 4 * N * R * U, 4 * U * N, "alu"
+    if name == "pool":
+        return 0, 4 * N * T * B + 4 * N * nnz + 4 * nnz + 8 * (T * B + 1), "hbm"
+    if name == "agg":
+        return 0, 4 * N * nnz + 8 * nnz + 4 * N * U, "hbm"
+    if name == "sort_pass":
+        return 0, 16 * nnz, "hbm"
+    return 0, 0, "hbm"
+
+
+# ---------------------------------------------------------------------------
+# reference arm: the CPU oracle as it stands
+# ---------------------------------------------------------------------------
+def oracle_step(orc, cfg, cores, idx, off, b, go, lr, opt):
+    orc.forward(cores, idx, off, b)
+    g = orc.backward(cores, idx, off, b, go)
+    new = []
+    for t, c in enumerate(cores):
+        new.append(tuple(orc.update(opt, lr, c[k], g[t][k])[0] for k in range(3)))
+    return new
+
+
+def sub_batch(idx, off, T, B, b):
+    """The first b samples of every table of a (T, B) batch."""
+    parts, lens = [], []
+    for t in range(T):
+        s, e = off[t * B], off[t * B + b]
+        parts.append(idx[s:e])
+        lens.append(np.diff(off[t * B:t * B + b + 1]))
+    lens = np.concatenate(lens)
+    o = np.zeros(T * b + 1, np.int64)
+    np.cumsum(lens, out=o[1:])
+    return np.concatenate(parts), o
+
+
+def calibrate_sample(orc, cfg, cores, idx, off, B, go, lr, opt, target_s):
+    b = max(1, min(B, 64))
+    while True:
+        si, so = sub_batch(idx, off, cfg.num_tables, B, b)
+        t0 = time.perf_counter()
+        oracle_step(orc, cfg, cores, si, so, b, go[:b], lr, opt)
+        dt = time.perf_counter() - t0
+        if dt >= 0.25 * target_s or b >= B:
+            break
+        b = min(B, b * 4)
+    scale = target_s / max(dt, 1e-6)
+    return max(1, min(B, int(b * scale)))
+
+
+def cpu_baseline(cfg, cores, idx, off, B, go, lr, opt, target_s=15.0):
+    import oracle
+    orc = oracle.Oracle.from_config(cfg)
+    b = calibrate_sample(orc, cfg, cores, idx, off, B, go, lr, opt, target_s)
+    si, so = sub_batch(idx, off, cfg.num_tables, B, b)
+    t0 = time.perf_counter()
+    oracle_step(orc, cfg, cores, si, so, b, go[:b], lr, opt)
+    dt = time.perf_counter() - t0
+    look = int(so[-1])
+    return {"value": look / dt, "unit": UNIT, "cores": oracle.Oracle.num_threads(), "kind": "oracle",
+            "sample": f"first {b} of {B} samples of every table of step-0 batch ({look} lookups), "
+                      f"fp64 oracle fwd+bwd+{opt} update, {dt:.1f} s wall"}
+
+
+def run_reference(args, cfg, rank, world):
+    if rank != 0:
+        return
+    import oracle
+    B = cfg.batch if args.scaling == "weak" else cfg.batch // world
+    cores = W.make_cores(cfg, seed=args.seed)
+    idx, off = W.make_batch(cfg, step=0, seed=args.seed, batch=B)
+    go = W.make_grad_out(cfg, B, step=0, seed=args.seed)
+    orc = oracle.Oracle.from_config(cfg)
+    budget = 150.0 / max(1, args.steps + args.warmup)
+    b = calibrate_sample(orc, cfg, cores, idx, off, B, go, args.lr, args.opt, budget)
+    si, so = sub_batch(idx, off, cfg.num_tables, B, b)
+    for _ in range(args.warmup):
+        oracle_step(orc, cfg, cores, si, so, b, go[:b], args.lr, args.opt)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        cores = oracle_step(orc, cfg, cores, si, so, b, go[:b], args.lr, args.opt)
+    dt = time.perf_counter() - t0
+    look = int(so[-1]) * args.steps
+    val = look / dt
+    line = {"metric": METRIC, "value": val, "unit": UNIT, "impl": "reference", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * dt / args.steps,
+            "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "config": workload_config(cfg, B, world, args),
+            "cpu_baseline": {"value": val, "unit": UNIT, "cores": oracle.Oracle.num_threads(),
+                             "kind": "oracle",
+                             "sample": f"first {b} of {B} samples of every table per step "
+                                       f"({int(so[-1])} lookups), fp64 oracle fwd+bwd+{args.opt} update"},
+            "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def workload_config(cfg, B, world, args):
+    return {"workload": cfg.name, "tables": cfg.num_tables, "max_rows": max(cfg.table_rows),
+            "dim": cfg.dim, "col_factors": list(cfg.col_factors), "tt_rank": cfg.rank,
+            "batch_per_gpu": B, "global_batch": B * world, "pooling": cfg.pooling,
+            "ids": f"zipf{cfg.zipf_s}-{cfg.id_map}" if cfg.zipf_s else f"uniform-{cfg.id_map}",
+            "optimizer": args.opt, "update": "fused" if world == 1 else "allreduce+update",
+            "parallelism": f"dp{world}", "l2": "flushed between timed steps (untimed 512 MiB write)"}
+
+
+# ---------------------------------------------------------------------------
+# our arm
+# ---------------------------------------------------------------------------
+def kernels_per_step(emb_ctx, world):
+    """Our kernel launches per step (memsets excluded): see DESIGN.md."""
+    kp, gp = emb_ctx
+    idx_stage = 1 + 2 + kp + 1 + 1 + 2 + gp + 1
+    fwd = 3
+    bwd = 5 + (1 if world == 1 else 0)
+    upd = 0 if world == 1 else 1
+    return idx_stage + fwd + bwd + upd
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--config", default="c4")
+    ap.add_argument("--rank", type=int, default=None, help="TT rank for c5 (32/64/128)")
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--opt", default="sgd", choices=["sgd", "adagrad"])
+    ap.add_argument("--ids", default="identity", choices=["identity", "perm"])
+    ap.add_argument("--scaling", default=None, choices=["weak", "strong"])
+    ap.add_argument("--pool", type=int, default=4, help="distinct pre-generated batches")
+    ap.add_argument("--lr", type=float, default=0.01)
+    ap.add_argument("--seed", type=int, default=0)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--stages", action="store_true", help="print per-stage times to stderr")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    cfg = W.config(args.config, args.rank) if args.config == "c5" else W.config(args.config)
+    cfg = cfg.replace(id_map=args.ids)
+    if args.scaling is None:
+        args.scaling = "strong" if args.config == "c5" else "weak"
+
+    if args.impl == "reference":
+        if world > 1:
+            import torch.distributed as dist
+            dist.init_process_group("gloo")
+        run_reference(args, cfg, rank, world)
+        return
+
+    import torch
+    import torch.distributed as dist
+    import paper_conf_sc_wangwfmmd22_b200 as tt
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    B = cfg.batch if args.scaling == "weak" else cfg.batch // world
+    fused = world == 1
+
+    # ---- inputs: a pool of batches resident in HBM ----
+    pool = []
+    for i in range(args.pool):
+        if args.scaling == "weak":
+            idx, off = W.make_batch(cfg, step=i, seed=args.seed + 1000 * rank, batch=B)
+            go = W.make_grad_out(cfg, B, step=i, seed=args.seed + 1000 * rank)
+        else:
+            gi, goff = W.make_batch(cfg, step=i, seed=args.seed)
+            idx, off, _ = W.shard_batch(gi, goff, cfg.num_tables, cfg.batch, rank, world)
+            go = W.make_grad_out(cfg, cfg.batch, step=i, seed=args.seed)[rank * B:(rank + 1) * B].copy()
+        pool.append((idx, off, go))
+    max_nnz = max(len(p[0]) for p in pool)
+    emb = tt.TTEmbeddingBag(cfg.table_rows, cfg.row_factors, cfg.col_factors, cfg.rank, B, max_nnz,
+                            optimizer=args.opt, fused_update=fused, device=local_rank)
+    cores = W.make_cores(cfg, seed=args.seed)
+    emb.load_cores(cores)
+    dpool = [(torch.as_tensor(i, device=dev), torch.as_tensor(o, device=dev), torch.as_tensor(g, device=dev))
+             for i, o, g in pool]
+    out = torch.empty(B, cfg.num_tables, cfg.dim, device=dev)
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    stream = torch.cuda.current_stream()
+
+    def step(i):
+        di, do, dg = dpool[i % len(dpool)]
+        emb.forward(di, do, B, out=out)
+        emb.backward(dg, lr=args.lr)
+        if world > 1:
+            dist.all_reduce(emb.grads)
+            emb.update(args.lr)
+
+    for i in range(args.warmup):
+        step(i)
+    torch.cuda.synchronize()
+    assert emb.check() == 0, "device-side input error"
+
+    # ---- timed region (device events per step; L2 flushed between steps, untimed) ----
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    emb.set_timing(True)
+    emb.stage_times()   # reset
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with Clocks(local_rank) as clk:
+        for i in range(args.steps):
+            flush.fill_(i & 0xff)
+            ev[i][0].record(stream)
+            step(i)
+            ev[i][1].record(stream)
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    stages = emb.stage_times()
+    emb.set_timing(False)
+    t_ms = sum(a.elapsed_time(b) for a, b in ev)
+    t_max = torch.tensor([t_ms], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t_max, op=dist.ReduceOp.MAX)
+    t_ms = float(t_max.item())
+    look_step = sum(int(p[0].shape[0]) for p in pool) / len(pool)
+    value = world * look_step * args.steps / (t_ms / 1e3)
+
+    # ---- counts of the last step for the roofline ----
+    counts = emb.counts()
+    plan = emb.plan()
+    last = (args.steps - 1) % len(pool)
+    nnz_last = len(pool[last][0])
+    pt = plan["pfx_t"].cpu().numpy().astype(np.int64)
+    pi1 = plan["pfx_i1"].cpu().numpy().astype(np.int64)
+    ri3 = plan["row_i3"].cpu().numpy().astype(np.int64)
+    rt = pt[plan["row_pfx"].cpu().numpy().astype(np.int64)]
+    touched = {"c1": len(np.unique(pt * (1 << 32) + pi1)), "c2": counts["NG"],
+               "c3": len(np.unique(rt * (1 << 32) + ri3))}
+    hbm_peak, sm_max_mhz, peak_kind = load_peaks()
+    sm_count = torch.cuda.get_device_properties(dev).multi_processor_count
+    alu_peak = fp32_peak_tflops(sm_count, sm_max_mhz)
+    flops, bytes_ = step_work(cfg, B, nnz_last, counts, touched, args.opt)
+    ms_step = t_ms / args.steps
+    # dominant stage
+    dom = max(stages.items(), key=lambda kv: kv[1][0])
+    dname, (dms, dn) = dom
+    f1, b1, bound = stage_work(dname, cfg, B, nnz_last, counts)
+    per_launch_ms = dms / max(dn, 1)
+    if bound == "alu":
+        ach = f1 / (per_launch_ms / 1e3) / 1e12
+        roof = {"bound": "alu", "kernel": dname, "achieved": ach, "peak": alu_peak, "unit": "TFLOP/s",
+                "frac": ach / alu_peak, "traffic": None,
+                "peak_source": f"derived: {sm_count} SM x 128 FP32 FMA/clk x 2 x {sm_max_mhz:.0f} MHz"}
+    else:
+        ach = b1 / (per_launch_ms / 1e3) / 1e9
+        roof = {"bound": "hbm", "kernel": dname, "achieved": ach, "peak": hbm_peak, "unit": "GB/s",
+                "frac": ach / hbm_peak, "traffic": None, "peak_source": f"{peak_kind} copy bandwidth"}
+    roof["share_of_step"] = dms / max(t_ms, 1e-9)
+    t_alu = flops / (alu_peak * 1e12) * 1e3
+    t_hbm = bytes_ / (hbm_peak * 1e9) * 1e3
+    step_roof = {"alg_gflop": flops / 1e9, "alg_mb": bytes_ / 1e6, "t_alu_ms": t_alu, "t_hbm_ms": t_hbm,
+                 "frac_hbm_roofline": t_hbm / ms_step, "frac_binding_roofline": max(t_alu, t_hbm) / ms_step,
+                 "binding": "alu" if t_alu > t_hbm else "hbm", "U": counts["U"], "P": counts["P"],
+                 "NG": counts["NG"], "touched_slices": touched}
+
+    # ---- end-to-end through the host-buffer ABI calls ----
+    e2e = None
+    if not args.no_e2e and world == 1:
+        hpool = [(torch.as_tensor(i).pin_memory(), torch.as_tensor(o).pin_memory(),
+                  torch.as_tensor(g).pin_memory()) for i, o, g in pool]
+        hout = torch.empty(B, cfg.num_tables, cfg.dim).pin_memory()
+
+        def hstep(i):
+            hi, ho, hg = hpool[i % len(hpool)]
+            emb.forward_host(hi, ho, B, hout)
+            emb.backward_host(hg, lr=args.lr)
+
+        for i in range(args.warmup):
+            hstep(i)
+        torch.cuda.synchronize()
+        hev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+        for i in range(args.steps):
+            flush.fill_(i & 0xff)
+            hev[i][0].record(stream)
+            hstep(i)
+            hev[i][1].record(stream)
+        torch.cuda.synchronize()
+        te = sum(a.elapsed_time(b) for a, b in hev)
+        h2d = sum(p[0].numel() * 8 + p[1].numel() * 8 + p[2].numel() * 4 for p in pool) / len(pool)
+        e2e = {"value": look_step * args.steps / (te / 1e3), "unit": UNIT, "h2d_bytes_per_step": int(h2d),
+               "d2h_bytes_per_step": int(hout.numel() * 4), "ms_per_step": te / args.steps,
+               "path": "ttemb_forward_host + ttemb_backward_host (pinned host buffers)"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        idx0, off0, go0 = pool[0]
+        cpu = cpu_baseline(cfg, cores, idx0, off0, B, go0, args.lr, args.opt)
+
+    if args.stages and rank == 0:
+        for k, (ms, n) in sorted(stages.items(), key=lambda kv: -kv[1][0]):
+            if n:
+                print(f"  {k:12s} {ms / args.steps * 1e3:9.1f} us/step  ({n} launches)", file=sys.stderr)
+
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
+                "scaling": args.scaling, "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+                "config": workload_config(cfg, B, world, args), "roofline": roof,
+                "step_roofline": step_roof, "cpu_baseline": cpu, "e2e": e2e,
+                "gpu_launches": kernels_per_step((emb_passes(emb)), world) * args.steps,
+                "clocks": clk.summary(),
+                "stages_us_per_step": {k: round(v[0] / args.steps * 1e3, 2) for k, v in stages.items() if v[1]}}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def emb_passes(emb):
+    rows = sum(emb.table_rows)
+    kp = max(1, (max(rows - 1, 0).bit_length() + 7) // 8)
+    gb = sum(f[1] for f in emb.row_factors)
+    gp = max(1, (max(gb - 1, 0).bit_length() + 7) // 8)
+    return kp, gp
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,181 @@
+/*
+ * ttemb.h -- C ABI of libttemb.so: the B200 (sm_100a) TT-EmbeddingBag hot path.
+ *
+ * What it computes (PAPER.md, cited P:<line>; DESIGN.md for the readings R1..R24):
+ *   A table W_t in R^{M_t x N} is stored as three TT cores (Eq. 1-2):
+ *     C1[m1][n1][R], C2[m2][R][n2][R], C3[m3][R][n3],   N = n1 n2 n3,  m1 m2 m3 >= M_t
+ *   Row i has digits i1 = floor(i/(m2 m3)), i2 = floor(i/m3) mod m2, i3 = i mod m3
+ *   (Eq. 3, pinned by the Fig. 5(b) example P:164) and
+ *     W_t[i, (j1 n2 + j2) n3 + j3] = sum_{r1,r2} C1[i1,j1,r1] C2[i2,r1,j2,r2] C3[i3,r2,j3].
+ *   forward:  out[b][t][:] = sum_{j in bag(t,b)} W_t[indices[j], :]   (sum pooling, Eq. 4,
+ *             P:164-167; a drop-in for nn.EmbeddingBag(mode="sum"))
+ *   backward: dL/dC_k of L = sum(out * grad_out)  (Eq. 6 read as left^T dL/de right^T,
+ *             P:185-191), gradients aggregated per unique row first
+ *   update:   SGD  C -= lr g;  Adagrad  S += g^2, C -= lr g / (sqrt(S) + eps)
+ * Inside, the forward computes each shared prefix product C1[i1] C2[i2] once per
+ * batch (the Reuse buffer) and the backward reduces per unique core slice.
+ *
+ * Conventions
+ *   * Every call returns int: 0 = TTEMB_OK, < 0 = ttemb_status.  Host-detectable
+ *     errors return before anything is enqueued.
+ *   * "device" pointers are CUDA global memory on the handle's device; "host"
+ *     pointers are CPU memory (pinned for asynchronous copies).
+ *   * `stream` is a cudaStream_t (NULL = legacy default stream).  Every call is
+ *     asynchronous on it; nothing synchronises the host except ttemb_check,
+ *     ttemb_read_counts and ttemb_stage_times.
+ *   * Offsets are table-major: bag (t,b) = indices[offsets[t*B+b] .. offsets[t*B+b+1]),
+ *     offsets[0] = 0, non-decreasing, offsets[T*B] = nnz.  out / grad_out are
+ *     [B][T][dim] float32, row-major (DLRM's concatenated embedding layer).
+ *   * Ownership: the caller allocates every buffer (cores, optimizer state,
+ *     gradients, workspace) and keeps it alive until ttemb_destroy; the library
+ *     never allocates device memory on the hot path.  Not thread-safe per handle;
+ *     one forward may be in flight per handle (its plan is kept for backward).
+ *   * Device-detectable input errors (id < 0 or id >= M_t, including padding ids
+ *     in [M_t, m1 m2 m3), malformed offsets) set a flag in device memory; outputs
+ *     of that step are unspecified (but memory-safe) and ttemb_check reports
+ *     TTEMB_ERR_INDEX_RANGE / TTEMB_ERR_INVALID_ARG.
+ */
+#ifndef TTEMB_H
+#define TTEMB_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  TTEMB_OK = 0,
+  TTEMB_ERR_INVALID_ARG = -1,   /* bad config / argument / offsets                */
+  TTEMB_ERR_UNSUPPORTED = -2,   /* num_cores != 3, rank/factor limits exceeded    */
+  TTEMB_ERR_INDEX_RANGE = -3,   /* an id outside [0, M_t) (reported by ttemb_check) */
+  TTEMB_ERR_STATE = -4,         /* backward without forward, update when fused    */
+  TTEMB_ERR_CUDA = -5,          /* a CUDA runtime error                           */
+  TTEMB_ERR_CAPACITY = -6       /* nnz > max_nnz or batch > max_batch             */
+} ttemb_status;
+
+typedef enum { TTEMB_SGD = 0, TTEMB_ADAGRAD = 1 } ttemb_opt;
+
+/* ttemb_config.flags */
+#define TTEMB_FUSED_UPDATE 1u   /* backward applies the update (single replica) */
+
+typedef struct {
+  int64_t num_rows;        /* M_t >= 1 */
+  int32_t row_factors[3];  /* (m1, m2, m3), m1 m2 m3 >= M_t  (R10) */
+} ttemb_table;
+
+typedef struct {
+  int32_t num_tables;            /* T >= 1 (T = 1 is a plain EmbeddingBag)            */
+  const ttemb_table* tables;     /* [T], host memory, copied by ttemb_create          */
+  int32_t num_cores;             /* must be 3 (the paper's design)         */
+  int32_t dim;                   /* N = col_factors[0]*col_factors[1]*col_factors[2]  */
+  int32_t col_factors[3];        /* (n1, n2, n3), shared by all tables                */
+  int32_t rank;                  /* R1 = R2 = rank (1..128), R0 = R3 = 1      */
+  int32_t index_bits;            /* 64 (int64 ids, PyTorch default) or 32             */
+  int32_t max_batch;             /* B capacity (workspace sizing)                     */
+  int64_t max_nnz;               /* nnz capacity, <= 2^30                             */
+  int32_t optimizer;             /* ttemb_opt                                         */
+  float adagrad_eps;             /* Adagrad eps (PyTorch default 1e-10)               */
+  uint32_t flags;                /* TTEMB_FUSED_UPDATE                                */
+} ttemb_config;
+
+typedef struct ttemb_ctx* ttemb_t;
+
+/* Byte sizes of the caller-owned buffers for `cfg`.  core_bytes == grad_bytes;
+ * state_bytes is 0 for SGD.  Pure host computation. */
+int ttemb_query_sizes(const ttemb_config* cfg, size_t* core_bytes, size_t* state_bytes,
+                      size_t* grad_bytes, size_t* workspace_bytes);
+
+/* Validate `cfg` and bind the caller's device buffers (sizes from
+ * ttemb_query_sizes; 256-byte aligned): cores (parameters, initialised by the
+ * caller via ttemb_core_layout), state (Adagrad accumulator, zero-initialised
+ * by the caller; may be NULL for SGD), grads (dense dL/dC, same layout as
+ * cores; written by ttemb_backward, read by ttemb_update; safe to all-reduce
+ * in place between the two), workspace (scratch).  `device` is the CUDA
+ * ordinal the buffers live on.  On success *out is a new handle. */
+int ttemb_create(const ttemb_config* cfg, int device, void* cores, void* state, void* grads,
+                 void* workspace, ttemb_t* out);
+int ttemb_destroy(ttemb_t h);
+
+/* Where core `core` (0, 1, 2) of table `table` lives: float offset into the
+ * cores / grads / state buffers and its shape:
+ *   core 0: {m1, n1, R, 1}   core 1: {m2, R, n2, R}   core 2: {m3, R, n3, 1}. */
+int ttemb_core_layout(ttemb_t h, int table, int core, int64_t* offset_floats,
+                      int32_t shape[4]);
+
+/* Forward (device buffers): indices [nnz] (int64 or int32 per index_bits),
+ * offsets [T*batch+1] int64, out [batch][T][dim] float32 (fully overwritten).
+ * Runs the index stage (sort / unique / inverse / prefixes), the prefix and
+ * row contractions and the pooling; keeps the plan for ttemb_backward. */
+int ttemb_forward(ttemb_t h, const void* indices, const int64_t* offsets, int64_t nnz,
+                  int32_t batch, float* out, void* stream);
+
+/* Backward of the last forward: grad_out [batch][T][dim] float32 (device).
+ * Without TTEMB_FUSED_UPDATE it overwrites the whole grads buffer with dL/dC
+ * (untouched slices 0); with it, it applies the update with `lr` instead
+ * (grads then holds scratch). */
+int ttemb_backward(ttemb_t h, const float* grad_out, float lr, void* stream);
+
+/* Optimizer step from the grads buffer (after an optional all-reduce SUM).
+ * TTEMB_ERR_STATE when the handle was created with TTEMB_FUSED_UPDATE. */
+int ttemb_update(ttemb_t h, float lr, void* stream);
+
+/* Host-buffer variants (end-to-end path): copy the inputs from host memory
+ * into the workspace staging area, run the step, and copy `out` back to the
+ * host, all on `stream`.  Pinned host memory keeps the copies asynchronous. */
+int ttemb_forward_host(ttemb_t h, const void* host_indices, const int64_t* host_offsets,
+                       int64_t nnz, int32_t batch, float* host_out, void* stream);
+int ttemb_backward_host(ttemb_t h, const float* host_grad_out, float lr, void* stream);
+
+/* Synchronise `stream` and report deferred device errors of the last calls
+ * (TTEMB_ERR_INDEX_RANGE, TTEMB_ERR_INVALID_ARG for malformed offsets). */
+int ttemb_check(ttemb_t h, void* stream);
+
+/* Device-resident results of the index stage of the last forward (valid until
+ * the next forward).  Counts live on the device (read them with
+ * ttemb_read_counts).  Arrays are uint32; sizes in brackets. */
+typedef struct {
+  int64_t nnz;
+  int32_t batch;
+  const uint32_t* counts;    /* [4] U, P, NG, error flags                              */
+  const uint32_t* skey;      /* [nnz] sorted keys, key = rowbase_t + id                */
+  const uint32_t* spos;      /* [nnz] stable argsort of the keys                       */
+  const uint32_t* bag_of;    /* [nnz] output row b*T + t of position j                 */
+  const uint32_t* ukey;      /* [U] distinct keys, ascending                            */
+  const uint32_t* seg_off;   /* [U+1] sorted-position segment of each unique row        */
+  const uint32_t* inverse;   /* [nnz] unique slot of position j                         */
+  const uint32_t* row_pfx;   /* [U] prefix slot of each unique row                      */
+  const uint32_t* row_i3;    /* [U] third digit                                         */
+  const uint32_t* pfx_t;     /* [P] table of each unique prefix (t, floor(row/m3))      */
+  const uint32_t* pfx_i1;    /* [P] first digit                                         */
+  const uint32_t* pfx_i2;    /* [P] second digit                                        */
+  const uint32_t* row_seg;   /* [P+1] unique rows of each prefix                        */
+  const uint32_t* grp_pfx;   /* [P] prefixes ordered by (t, i2, i1)                     */
+  const uint32_t* grp_off;   /* [NG+1] i2-groups (one C2 slice each)                    */
+  const uint32_t* grp_t;     /* [NG] */
+  const uint32_t* grp_i2;    /* [NG] */
+  const float* prefix_products; /* [P][n1][n2][R] the Reuse buffer              */
+  const float* rows;         /* [U][dim] W rows of the unique ids                       */
+} ttemb_plan;
+
+int ttemb_get_plan(ttemb_t h, ttemb_plan* plan);
+
+/* Synchronous helper: copy {U, P, NG, error flags} of the last forward to host. */
+int ttemb_read_counts(ttemb_t h, int64_t counts[4], void* stream);
+
+/* Per-stage device timing (CUDA events on the launching stream).  While
+ * enabled, every stage of forward/backward/update records an event pair;
+ * ttemb_stage_times synchronises and returns, per stage id, the summed
+ * milliseconds and launch count since the last reset; names via
+ * ttemb_stage_name.  Returns the number of stages. */
+int ttemb_set_timing(ttemb_t h, int enable);
+int ttemb_stage_times(ttemb_t h, double* ms, int64_t* launches, int max_stages);
+const char* ttemb_stage_name(int stage);
+
+const char* ttemb_status_string(int status);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* TTEMB_H */

@@ -1,0 +1,108 @@
+"""ctypes declarations of include/ttemb.h and the loader of the in-tree libttemb.so.
+
+There is no fallback: if the library is missing or fails to load, importing the
+binding raises.  Every step of the hot path runs in the CUDA kernels behind
+this ABI; Python only marshals arguments.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libttemb.so")
+
+TTEMB_OK = 0
+TTEMB_ERR_INVALID_ARG = -1
+TTEMB_ERR_UNSUPPORTED = -2
+TTEMB_ERR_INDEX_RANGE = -3
+TTEMB_ERR_STATE = -4
+TTEMB_ERR_CUDA = -5
+TTEMB_ERR_CAPACITY = -6
+TTEMB_SGD = 0
+TTEMB_ADAGRAD = 1
+TTEMB_FUSED_UPDATE = 1
+
+SYMBOLS = ["ttemb_query_sizes", "ttemb_create", "ttemb_destroy", "ttemb_core_layout",
+           "ttemb_forward", "ttemb_backward", "ttemb_update", "ttemb_forward_host",
+           "ttemb_backward_host", "ttemb_check", "ttemb_get_plan", "ttemb_read_counts",
+           "ttemb_set_timing", "ttemb_stage_times", "ttemb_stage_name", "ttemb_status_string"]
+
+
+class ttemb_table(C.Structure):
+    _fields_ = [("num_rows", C.c_int64), ("row_factors", C.c_int32 * 3)]
+
+
+class ttemb_config(C.Structure):
+    _fields_ = [("num_tables", C.c_int32), ("tables", C.POINTER(ttemb_table)),
+                ("num_cores", C.c_int32), ("dim", C.c_int32), ("col_factors", C.c_int32 * 3),
+                ("rank", C.c_int32), ("index_bits", C.c_int32), ("max_batch", C.c_int32),
+                ("max_nnz", C.c_int64), ("optimizer", C.c_int32), ("adagrad_eps", C.c_float),
+                ("flags", C.c_uint32)]
+
+
+_u32p = C.POINTER(C.c_uint32)
+
+
+class ttemb_plan(C.Structure):
+    _fields_ = [("nnz", C.c_int64), ("batch", C.c_int32)] + [
+        (n, C.c_void_p) for n in ["counts", "skey", "spos", "bag_of", "ukey", "seg_off", "inverse",
+                                  "row_pfx", "row_i3", "pfx_t", "pfx_i1", "pfx_i2", "row_seg",
+                                  "grp_pfx", "grp_off", "grp_t", "grp_i2", "prefix_products",
+                                  "rows"]]
+
+
+class TTEmbError(RuntimeError):
+    def __init__(self, code: int, what: str = ""):
+        self.code = code
+        msg = status_string(code) if _lib is not None else str(code)
+        super().__init__(f"{what}: {msg} ({code})" if what else f"{msg} ({code})")
+
+
+_lib = None
+
+
+def load(path: str = LIB_PATH):
+    """Load libttemb.so (raises if it is missing: no CPU fallback exists)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(path):
+        raise ImportError(f"libttemb.so not built at {path}; run __graft_entry__.build() "
+                          "or python -m paper_conf_sc_wangwfmmd22_b200.build")
+    lib = C.CDLL(path)
+    vp, i64, i32, f32 = C.c_void_p, C.c_int64, C.c_int32, C.c_float
+    sz = C.POINTER(C.c_size_t)
+    lib.ttemb_query_sizes.argtypes = [C.POINTER(ttemb_config), sz, sz, sz, sz]
+    lib.ttemb_create.argtypes = [C.POINTER(ttemb_config), C.c_int, vp, vp, vp, vp, C.POINTER(vp)]
+    lib.ttemb_destroy.argtypes = [vp]
+    lib.ttemb_core_layout.argtypes = [vp, C.c_int, C.c_int, C.POINTER(i64), C.POINTER(i32)]
+    lib.ttemb_forward.argtypes = [vp, vp, vp, i64, i32, vp, vp]
+    lib.ttemb_backward.argtypes = [vp, vp, f32, vp]
+    lib.ttemb_update.argtypes = [vp, f32, vp]
+    lib.ttemb_forward_host.argtypes = [vp, vp, vp, i64, i32, vp, vp]
+    lib.ttemb_backward_host.argtypes = [vp, vp, f32, vp]
+    lib.ttemb_check.argtypes = [vp, vp]
+    lib.ttemb_get_plan.argtypes = [vp, C.POINTER(ttemb_plan)]
+    lib.ttemb_read_counts.argtypes = [vp, C.POINTER(i64), vp]
+    lib.ttemb_set_timing.argtypes = [vp, C.c_int]
+    lib.ttemb_stage_times.argtypes = [vp, C.POINTER(C.c_double), C.POINTER(i64), C.c_int]
+    lib.ttemb_stage_name.argtypes = [C.c_int]
+    lib.ttemb_stage_name.restype = C.c_char_p
+    lib.ttemb_status_string.argtypes = [C.c_int]
+    lib.ttemb_status_string.restype = C.c_char_p
+    for s in SYMBOLS:
+        f = getattr(lib, s)
+        if s not in ("ttemb_stage_name", "ttemb_status_string"):
+            f.restype = C.c_int
+    _lib = lib
+    return lib
+
+
+def status_string(code: int) -> str:
+    return load().ttemb_status_string(int(code)).decode()
+
+
+def check(rc: int, what: str = "") -> None:
+    if rc != TTEMB_OK:
+        raise TTEmbError(rc, what)

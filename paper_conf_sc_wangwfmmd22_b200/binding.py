@@ -1,0 +1,312 @@
+"""Thin Python binding over libttemb.so (include/ttemb.h).
+
+The module-level functions carry the C names (ttemb_create, ttemb_forward, ...)
+and only marshal arguments.  `TTEmbeddingBag` is a convenience owner of the
+caller-side buffers: PyTorch provides device memory and streams, nothing else
+(every step of the path runs in the library's kernels).
+"""
+from __future__ import annotations
+
+import ctypes as C
+from typing import Dict, List, Optional, Sequence, Tuple
+
+import numpy as np
+import torch
+
+from . import _lib as L
+from ._lib import TTEmbError, check
+
+STAGES: List[str] = []
+
+
+def _stream_ptr(stream: Optional[torch.cuda.Stream]) -> int:
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return int(s.cuda_stream)
+
+
+def make_config(table_rows: Sequence[int], row_factors: Sequence[Tuple[int, int, int]],
+                col_factors: Tuple[int, int, int], rank: int, max_batch: int, max_nnz: int,
+                optimizer: str = "sgd", adagrad_eps: float = 1e-10, fused_update: bool = False,
+                index_bits: int = 64, num_cores: int = 3):
+    """Returns (ttemb_config, keep-alive table array)."""
+    T = len(table_rows)
+    tabs = (L.ttemb_table * max(T, 1))()
+    for t in range(T):
+        tabs[t].num_rows = int(table_rows[t])
+        for k in range(3):
+            tabs[t].row_factors[k] = int(row_factors[t][k])
+    cfg = L.ttemb_config()
+    cfg.num_tables = T
+    cfg.tables = C.cast(tabs, C.POINTER(L.ttemb_table))
+    cfg.num_cores = int(num_cores)
+    cfg.dim = int(np.prod(col_factors))
+    for k in range(3):
+        cfg.col_factors[k] = int(col_factors[k])
+    cfg.rank = int(rank)
+    cfg.index_bits = int(index_bits)
+    cfg.max_batch = int(max_batch)
+    cfg.max_nnz = int(max_nnz)
+    cfg.optimizer = {"sgd": L.TTEMB_SGD, "adagrad": L.TTEMB_ADAGRAD}[optimizer]
+    cfg.adagrad_eps = float(adagrad_eps)
+    cfg.flags = L.TTEMB_FUSED_UPDATE if fused_update else 0
+    return cfg, tabs
+
+
+# ---------------------------------------------------------------------------
+# Same-name wrappers of the C ABI
+# ---------------------------------------------------------------------------
+def ttemb_query_sizes(cfg) -> Tuple[int, int, int, int]:
+    v = [C.c_size_t() for _ in range(4)]
+    check(L.load().ttemb_query_sizes(C.byref(cfg), *[C.byref(x) for x in v]), "ttemb_query_sizes")
+    return tuple(int(x.value) for x in v)
+
+
+def ttemb_create(cfg, device: int, cores: int, state: int, grads: int, workspace: int) -> int:
+    h = C.c_void_p()
+    check(L.load().ttemb_create(C.byref(cfg), int(device), cores, state or None, grads, workspace,
+                                C.byref(h)), "ttemb_create")
+    return h.value
+
+
+def ttemb_destroy(h: int) -> None:
+    check(L.load().ttemb_destroy(h), "ttemb_destroy")
+
+
+def ttemb_core_layout(h: int, table: int, core: int) -> Tuple[int, Tuple[int, int, int, int]]:
+    off = C.c_int64()
+    shape = (C.c_int32 * 4)()
+    check(L.load().ttemb_core_layout(h, table, core, C.byref(off), shape), "ttemb_core_layout")
+    return int(off.value), tuple(int(x) for x in shape)
+
+
+def ttemb_forward(h: int, indices: int, offsets: int, nnz: int, batch: int, out: int, stream: int) -> int:
+    return L.load().ttemb_forward(h, indices, offsets, int(nnz), int(batch), out, stream)
+
+
+def ttemb_backward(h: int, grad_out: int, lr: float, stream: int) -> int:
+    return L.load().ttemb_backward(h, grad_out, float(lr), stream)
+
+
+def ttemb_update(h: int, lr: float, stream: int) -> int:
+    return L.load().ttemb_update(h, float(lr), stream)
+
+
+def ttemb_forward_host(h: int, indices: int, offsets: int, nnz: int, batch: int, out: int, stream: int) -> int:
+    return L.load().ttemb_forward_host(h, indices, offsets, int(nnz), int(batch), out, stream)
+
+
+def ttemb_backward_host(h: int, grad_out: int, lr: float, stream: int) -> int:
+    return L.load().ttemb_backward_host(h, grad_out, float(lr), stream)
+
+
+def ttemb_check(h: int, stream: int) -> int:
+    return L.load().ttemb_check(h, stream)
+
+
+def ttemb_get_plan(h: int) -> "L.ttemb_plan":
+    p = L.ttemb_plan()
+    check(L.load().ttemb_get_plan(h, C.byref(p)), "ttemb_get_plan")
+    return p
+
+
+def ttemb_read_counts(h: int, stream: int) -> Tuple[int, int, int, int]:
+    v = (C.c_int64 * 4)()
+    check(L.load().ttemb_read_counts(h, v, stream), "ttemb_read_counts")
+    return tuple(int(x) for x in v)
+
+
+def ttemb_set_timing(h: int, enable: bool) -> None:
+    check(L.load().ttemb_set_timing(h, int(bool(enable))), "ttemb_set_timing")
+
+
+def ttemb_stage_times(h: int) -> Dict[str, Tuple[float, int]]:
+    n = 64
+    ms = (C.c_double * n)()
+    cnt = (C.c_int64 * n)()
+    k = L.load().ttemb_stage_times(h, ms, cnt, n)
+    if k < 0:
+        raise TTEmbError(k, "ttemb_stage_times")
+    return {ttemb_stage_name(i): (float(ms[i]), int(cnt[i])) for i in range(k)}
+
+
+def ttemb_stage_name(i: int) -> str:
+    return L.load().ttemb_stage_name(int(i)).decode()
+
+
+def ttemb_status_string(code: int) -> str:
+    return L.status_string(code)
+
+
+# ---------------------------------------------------------------------------
+# Convenience owner
+# ---------------------------------------------------------------------------
+class TTEmbeddingBag:
+    """Table-batched TT-EmbeddingBag (sum pooling) on one CUDA device.
+
+    Buffers (torch tensors, caller-owned in ABI terms): cores, state (Adagrad),
+    grads, workspace.  Cores are zero until `load_cores` / `core_views` writes.
+    """
+
+    def __init__(self, table_rows, row_factors, col_factors, rank, max_batch, max_nnz,
+                 optimizer: str = "sgd", adagrad_eps: float = 1e-10, fused_update: bool = False,
+                 index_bits: int = 64, device: int = 0):
+        L.load()
+        self.table_rows = [int(x) for x in table_rows]
+        self.row_factors = [tuple(int(y) for y in f) for f in row_factors]
+        self.col_factors = tuple(int(x) for x in col_factors)
+        self.rank = int(rank)
+        self.T = len(self.table_rows)
+        self.N = int(np.prod(self.col_factors))
+        self.optimizer = optimizer
+        self.fused = bool(fused_update)
+        self.index_bits = int(index_bits)
+        self.device = torch.device("cuda", device)
+        self._cfg, self._tabs = make_config(table_rows, row_factors, col_factors, rank, max_batch,
+                                            max_nnz, optimizer, adagrad_eps, fused_update, index_bits)
+        cb, sb, gb, wb = ttemb_query_sizes(self._cfg)
+        self.sizes = dict(core_bytes=cb, state_bytes=sb, grad_bytes=gb, workspace_bytes=wb)
+        f32 = torch.float32
+        self.cores = torch.zeros(cb // 4, dtype=f32, device=self.device)
+        self.grads = torch.zeros(gb // 4, dtype=f32, device=self.device)
+        self.state = torch.zeros(sb // 4, dtype=f32, device=self.device) if sb else None
+        self.workspace = torch.empty(max(wb, 256), dtype=torch.uint8, device=self.device)
+        self.h = ttemb_create(self._cfg, device, self.cores.data_ptr(),
+                              self.state.data_ptr() if self.state is not None else 0,
+                              self.grads.data_ptr(), self.workspace.data_ptr())
+        self.layout = [[ttemb_core_layout(self.h, t, k) for k in range(3)] for t in range(self.T)]
+        self.batch = 0
+        self.nnz = 0
+
+    @classmethod
+    def from_config(cls, cfg, max_batch=None, max_nnz=None, **kw):
+        B = cfg.batch if max_batch is None else max_batch
+        nnz = B * cfg.num_tables * cfg.pooling if max_nnz is None else max_nnz
+        return cls(cfg.table_rows, cfg.row_factors, cfg.col_factors, cfg.rank, B, nnz, **kw)
+
+    def __del__(self):
+        h = getattr(self, "h", None)
+        if h:
+            try:
+                torch.cuda.synchronize(self.device)
+                ttemb_destroy(h)
+            except Exception:
+                pass
+            self.h = None
+
+    # -- parameters --------------------------------------------------------
+    def _views(self, buf: torch.Tensor):
+        out = []
+        for t in range(self.T):
+            vs = []
+            for k in range(3):
+                off, shape = self.layout[t][k]
+                shp = shape[:3] if k != 1 else shape
+                n = int(np.prod(shp))
+                vs.append(buf[off:off + n].view(*shp))
+            out.append(tuple(vs))
+        return out
+
+    def core_views(self):
+        return self._views(self.cores)
+
+    def grad_views(self):
+        return self._views(self.grads)
+
+    def state_views(self):
+        return self._views(self.state) if self.state is not None else None
+
+    def load_cores(self, cores) -> None:
+        """cores: per table (C1[m1][n1][R], C2[m2][R][n2][R], C3[m3][R][n3])."""
+        for dst, src in zip(self.core_views(), cores):
+            for d, s in zip(dst, src):
+                d.copy_(torch.as_tensor(np.asarray(s, dtype=np.float32)).view(d.shape))
+
+    # -- step ----------------------------------------------------------------
+    def forward(self, indices: torch.Tensor, offsets: torch.Tensor, batch: int,
+                out: Optional[torch.Tensor] = None, stream=None) -> torch.Tensor:
+        want = torch.int64 if self.index_bits == 64 else torch.int32
+        assert indices.dtype == want and indices.is_cuda and offsets.dtype == torch.int64
+        assert offsets.numel() == self.T * batch + 1
+        if out is None:
+            out = torch.empty(batch, self.T, self.N, dtype=torch.float32, device=self.device)
+        nnz = indices.numel()
+        rc = ttemb_forward(self.h, indices.data_ptr() if nnz else None, offsets.data_ptr(), nnz, batch,
+                           out.data_ptr() if out.numel() else None, _stream_ptr(stream))
+        check(rc, "ttemb_forward")
+        self.batch, self.nnz = batch, nnz
+        return out
+
+    def backward(self, grad_out: torch.Tensor, lr: float = 0.0, stream=None) -> None:
+        assert grad_out.dtype == torch.float32 and grad_out.is_contiguous()
+        assert tuple(grad_out.shape) == (self.batch, self.T, self.N)
+        check(ttemb_backward(self.h, grad_out.data_ptr() if grad_out.numel() else None, lr,
+                             _stream_ptr(stream)), "ttemb_backward")
+
+    def update(self, lr: float, stream=None) -> None:
+        check(ttemb_update(self.h, lr, _stream_ptr(stream)), "ttemb_update")
+
+    def forward_host(self, indices: torch.Tensor, offsets: torch.Tensor, batch: int,
+                     out: torch.Tensor, stream=None) -> None:
+        """indices / offsets / out in (pinned) host memory."""
+        assert not indices.is_cuda and not offsets.is_cuda and not out.is_cuda
+        nnz = indices.numel()
+        check(ttemb_forward_host(self.h, indices.data_ptr() if nnz else None, offsets.data_ptr(), nnz,
+                                 batch, out.data_ptr() if out.numel() else None, _stream_ptr(stream)),
+              "ttemb_forward_host")
+        self.batch, self.nnz = batch, nnz
+
+    def backward_host(self, grad_out: torch.Tensor, lr: float = 0.0, stream=None) -> None:
+        assert not grad_out.is_cuda
+        check(ttemb_backward_host(self.h, grad_out.data_ptr() if grad_out.numel() else None, lr,
+                                  _stream_ptr(stream)), "ttemb_backward_host")
+
+    def check(self, stream=None) -> int:
+        return ttemb_check(self.h, _stream_ptr(stream))
+
+    def counts(self, stream=None) -> Dict[str, int]:
+        U, P, NG, err = ttemb_read_counts(self.h, _stream_ptr(stream))
+        return dict(U=U, P=P, NG=NG, err=err)
+
+    def plan(self, stream=None) -> Dict[str, torch.Tensor]:
+        """Copies of the index-stage outputs of the last forward (sizes from the counts)."""
+        c = self.counts(stream)
+        p = ttemb_get_plan(self.h)
+        U, P, NG, nnz = c["U"], c["P"], c["NG"], int(p.nnz)
+        size = {"skey": nnz, "spos": nnz, "bag_of": nnz, "inverse": nnz, "ukey": U, "seg_off": U + 1,
+                "row_pfx": U, "row_i3": U, "pfx_t": P, "pfx_i1": P, "pfx_i2": P, "row_seg": P + 1,
+                "grp_pfx": P, "grp_off": NG + 1, "grp_t": NG, "grp_i2": NG}
+        out = {}
+        for k, n in size.items():
+            out[k] = _copy_device_u32(getattr(p, k), n, self.device)
+        n1, n2, n3 = self.col_factors
+        out["prefix_products"] = _copy_device_f32(p.prefix_products, P * n1 * n2 * self.rank,
+                                                  self.device).view(P, n1, n2, self.rank)
+        out["rows"] = _copy_device_f32(p.rows, U * self.N, self.device).view(U, self.N)
+        out.update(U=U, P=P, NG=NG)
+        return out
+
+    def set_timing(self, enable: bool) -> None:
+        ttemb_set_timing(self.h, enable)
+
+    def stage_times(self) -> Dict[str, Tuple[float, int]]:
+        return ttemb_stage_times(self.h)
+
+
+class _DevArray:
+    """A raw device pointer exposed through __cuda_array_interface__ (zero-copy view)."""
+
+    def __init__(self, ptr: int, n: int, typestr: str):
+        self.__cuda_array_interface__ = {"shape": (n,), "typestr": typestr, "data": (ptr, True),
+                                         "version": 2}
+
+
+def _copy_device_u32(ptr: int, n: int, device) -> torch.Tensor:
+    if n <= 0:
+        return torch.empty(0, dtype=torch.int32, device=device)
+    return torch.as_tensor(_DevArray(ptr, n, "<u4"), device=device).view(torch.int32).clone()
+
+
+def _copy_device_f32(ptr: int, n: int, device) -> torch.Tensor:
+    if n <= 0:
+        return torch.empty(0, dtype=torch.float32, device=device)
+    return torch.as_tensor(_DevArray(ptr, n, "<f4"), device=device).clone()

@@ -1,0 +1,480 @@
+// ttemb_api.cu -- the C ABI of libttemb.so (include/ttemb.h): configuration checks,
+// buffer layout, workspace carving, stage sequencing, deferred error reporting and
+// per-stage CUDA-event timing.  No kernel arithmetic lives here.
+#include <stdio.h>
+#include <string.h>
+
+#include <algorithm>
+#include <new>
+
+#include "ttemb_internal.cuh"
+
+namespace ttemb {
+cudaError_t configure_fwd(Ctx& c);
+cudaError_t configure_bwd(Ctx& c);
+int64_t radix_tiles(int64_t n);
+int64_t scan_tiles(int64_t n);
+int64_t agg_chunks(int64_t nnz);
+
+StageScope::StageScope(Ctx& c_, int st, cudaStream_t s_) : c(c_), stage(st), s(s_) {
+  if (!c.timing) return;
+  if (c.ev_pool.size() < 2) {
+    for (int i = 0; i < 64; ++i) {
+      cudaEvent_t e;
+      if (cudaEventCreate(&e) == cudaSuccess) c.ev_pool.push_back(e);
+    }
+  }
+  if (c.ev_pool.size() < 2) return;
+  a = c.ev_pool.back(); c.ev_pool.pop_back();
+  b = c.ev_pool.back(); c.ev_pool.pop_back();
+  cudaEventRecord(a, s);
+}
+StageScope::~StageScope() {
+  if (!a) return;
+  cudaEventRecord(b, s);
+  c.pending.push_back({stage, a, b});
+}
+
+static const char* kStageNames[ST_COUNT] = {
+    "zero_state", "build_keys", "sort_hist", "sort_pass", "unique", "prefix", "gsort_hist",
+    "gsort_pass", "groups", "fwd_prefix", "fwd_rows", "pool", "bwd_zero", "agg", "agg_fix",
+    "bwd_rows", "bwd_prefix", "dc1", "update_c3", "update", "h2d", "d2h"};
+
+namespace {
+
+struct Carver {
+  uint8_t* base;
+  size_t off = 0;
+  explicit Carver(uint8_t* b) : base(b) {}
+  template <typename T>
+  T* take(size_t count) {
+    off = (off + 255) & ~(size_t)255;
+    T* p = base ? reinterpret_cast<T*>(base + off) : nullptr;
+    off += sizeof(T) * (count ? count : 1);
+    return p;
+  }
+};
+
+int bits_for(uint64_t max_value) {
+  int b = 0;
+  while (b < 64 && (max_value >> b) != 0) ++b;
+  return b;
+}
+
+int validate(const ttemb_config* cfg) {
+  if (!cfg || !cfg->tables || cfg->num_tables < 1) return TTEMB_ERR_INVALID_ARG;
+  if (cfg->num_cores != 3) return TTEMB_ERR_UNSUPPORTED;
+  const int n1 = cfg->col_factors[0], n2 = cfg->col_factors[1], n3 = cfg->col_factors[2];
+  if (n1 < 1 || n2 < 1 || n3 < 1 || (int64_t)n1 * n2 * n3 != cfg->dim) return TTEMB_ERR_INVALID_ARG;
+  if (cfg->rank < 1) return TTEMB_ERR_INVALID_ARG;
+  if (cfg->rank > 128) return TTEMB_ERR_UNSUPPORTED;
+  if ((int64_t)n1 * n2 > 1024 || cfg->dim > 4096) return TTEMB_ERR_UNSUPPORTED;
+  if (cfg->index_bits != 64 && cfg->index_bits != 32) return TTEMB_ERR_INVALID_ARG;
+  if (cfg->max_batch < 0 || cfg->max_nnz < 0) return TTEMB_ERR_INVALID_ARG;
+  if (cfg->max_nnz > (int64_t(1) << 30)) return TTEMB_ERR_UNSUPPORTED;
+  if ((int64_t)cfg->num_tables * cfg->max_batch > (int64_t(1) << 31)) return TTEMB_ERR_UNSUPPORTED;
+  if (cfg->optimizer != TTEMB_SGD && cfg->optimizer != TTEMB_ADAGRAD) return TTEMB_ERR_INVALID_ARG;
+  if (cfg->flags & ~TTEMB_FUSED_UPDATE) return TTEMB_ERR_INVALID_ARG;
+  uint64_t total = 0, buckets = 0;
+  for (int t = 0; t < cfg->num_tables; ++t) {
+    const ttemb_table& tb = cfg->tables[t];
+    const int64_t m1 = tb.row_factors[0], m2 = tb.row_factors[1], m3 = tb.row_factors[2];
+    if (tb.num_rows < 1 || m1 < 1 || m2 < 1 || m3 < 1) return TTEMB_ERR_INVALID_ARG;
+    if (m1 * m2 * m3 < tb.num_rows) return TTEMB_ERR_INVALID_ARG;
+    if (m1 > (1 << 24) || m2 > (1 << 24) || m3 > (1 << 24)) return TTEMB_ERR_UNSUPPORTED;
+    total += (uint64_t)tb.num_rows;
+    buckets += (uint64_t)m2;
+  }
+  if (total > 0xFFFFFFFFull || buckets > 0xFFFFFFFFull) return TTEMB_ERR_UNSUPPORTED;
+  return TTEMB_OK;
+}
+
+// Fills every size-derived field of c (no device pointers).
+void plan_sizes(const ttemb_config* cfg, Ctx& c) {
+  c.T = cfg->num_tables;
+  c.n1 = cfg->col_factors[0]; c.n2 = cfg->col_factors[1]; c.n3 = cfg->col_factors[2];
+  c.N = cfg->dim; c.R = cfg->rank; c.NC = c.n2 * c.R;
+  c.index_bits = cfg->index_bits; c.opt = cfg->optimizer;
+  c.eps = cfg->adagrad_eps; c.flags = cfg->flags;
+  c.max_nnz = cfg->max_nnz; c.max_batch = cfg->max_batch;
+  c.meta.assign(c.T, TableMeta{});
+  const size_t s1 = (size_t)c.n1 * c.R, s2 = (size_t)c.R * c.n2 * c.R, s3 = (size_t)c.R * c.n3;
+  auto up4 = [](size_t x) { return (x + 3) & ~(size_t)3; };
+  size_t off = 0;
+  uint64_t rb = 0, pfx = 0;
+  uint32_t gb = 0;
+  for (int t = 0; t < c.T; ++t) {   // [C1 of all tables]
+    const ttemb_table& tb = cfg->tables[t];
+    TableMeta& m = c.meta[t];
+    m.m1 = tb.row_factors[0]; m.m2 = tb.row_factors[1]; m.m3 = tb.row_factors[2];
+    m.M = (uint32_t)tb.num_rows;
+    m.rowbase = rb; rb += (uint64_t)tb.num_rows;
+    m.grpbase = gb; gb += m.m2;
+    pfx += (uint64_t)((tb.num_rows + m.m3 - 1) / m.m3);
+    m.c1_off = off; off += up4(m.m1 * s1);
+  }
+  for (int t = 0; t < c.T; ++t) { c.meta[t].c2_off = off; off += up4(c.meta[t].m2 * s2); }
+  c.c3_begin = off;
+  for (int t = 0; t < c.T; ++t) { c.meta[t].c3_off = off; off += up4(c.meta[t].m3 * s3); }
+  c.c3_floats = off - c.c3_begin;
+  c.core_floats = off;
+  c.total_rows = rb;
+  c.total_buckets = gb;
+  c.key_passes = std::max(1, (bits_for(rb ? rb - 1 : 0) + 7) / 8);
+  c.gkey_passes = std::max(1, (bits_for(gb ? gb - 1 : 0) + 7) / 8);
+  c.U_cap = std::min<int64_t>(c.max_nnz, (int64_t)rb);
+  c.P_cap = std::min<int64_t>(c.U_cap, (int64_t)pfx);
+  c.NG_cap = std::min<int64_t>(c.P_cap, (int64_t)gb);
+  c.rs1_tiles = radix_tiles(c.max_nnz);
+  c.rs2_tiles = radix_tiles(c.P_cap);
+  c.sc_tiles = std::max<int64_t>(1, scan_tiles(c.max_nnz));
+}
+
+// Carves the workspace; with base == nullptr only computes the size.
+size_t carve(Ctx& c, uint8_t* base) {
+  Carver k(base);
+  const int64_t nnz = std::max<int64_t>(c.max_nnz, 1);
+  const int64_t U = std::max<int64_t>(c.U_cap, 1), P = std::max<int64_t>(c.P_cap, 1);
+  const int64_t NG = std::max<int64_t>(c.NG_cap, 1);
+  const int64_t bags = (int64_t)c.T * c.max_batch;
+  const size_t J12R = (size_t)c.n1 * c.n2 * c.R;
+  PlanDev& p = c.p;
+  c.d_meta = k.take<TableMeta>(c.T);
+  c.d_rowbase = k.take<uint64_t>(c.T + 1);
+  c.d_grpbase = k.take<uint32_t>(c.T + 1);
+  // --- zeroed every forward ---
+  k.off = (k.off + 255) & ~(size_t)255;
+  const size_t zb = k.off;
+  p.counts = k.take<uint32_t>(kNumCounts);
+  p.hist1 = k.take<uint32_t>(4 * 256);
+  p.hist2 = k.take<uint32_t>(4 * 256);
+  p.rs1_counter = k.take<uint32_t>(4);
+  p.rs2_counter = k.take<uint32_t>(4);
+  p.sc_counter = k.take<uint32_t>(4);
+  p.rs1_status = k.take<uint32_t>((size_t)c.key_passes * std::max<int64_t>(c.rs1_tiles, 1) * 256);
+  p.rs2_status = k.take<uint32_t>((size_t)c.gkey_passes * std::max<int64_t>(c.rs2_tiles, 1) * 256);
+  p.sc_status = k.take<uint32_t>((size_t)3 * c.sc_tiles);
+  k.off = (k.off + 255) & ~(size_t)255;
+  c.zero_bytes = k.off - zb;
+  c.zero_begin = base ? base + zb : nullptr;
+  // --- plan ---
+  p.dbase1 = k.take<uint32_t>(4 * 256);
+  p.dbase2 = k.take<uint32_t>(4 * 256);
+  p.keysA = k.take<uint32_t>(nnz); p.valsA = k.take<uint32_t>(nnz);
+  p.keysB = k.take<uint32_t>(nnz); p.valsB = k.take<uint32_t>(nnz);
+  p.bag_of = k.take<uint32_t>(nnz); p.sbag = k.take<uint32_t>(nnz); p.inverse = k.take<uint32_t>(nnz);
+  p.ukey = k.take<uint32_t>(U); p.seg_off = k.take<uint32_t>(U + 1);
+  p.row_pfx = k.take<uint32_t>(U); p.row_i3 = k.take<uint32_t>(U);
+  p.pfx_t = k.take<uint32_t>(P); p.pfx_i1 = k.take<uint32_t>(P); p.pfx_i2 = k.take<uint32_t>(P);
+  p.row_seg = k.take<uint32_t>(P + 1);
+  p.gkeyB = k.take<uint32_t>(P); p.gvalB = k.take<uint32_t>(P);
+  p.grp_pfx = k.take<uint32_t>(P); p.grp_off = k.take<uint32_t>(NG + 1);
+  p.grp_t = k.take<uint32_t>(NG); p.grp_i2 = k.take<uint32_t>(NG);
+  // --- float intermediates ---
+  p.pbuf = k.take<float>((size_t)P * J12R);
+  p.dpbuf = k.take<float>((size_t)P * J12R);
+  p.dabuf = k.take<float>((size_t)P * c.n1 * c.R);
+  p.rows = k.take<float>((size_t)U * c.N);
+  p.gbuf = k.take<float>((size_t)U * c.N);
+  p.aggpart = k.take<float>((size_t)2 * agg_chunks(nnz) * c.N);
+  // --- host staging (end-to-end API) ---
+  c.st_idx = k.take<uint8_t>((size_t)nnz * (c.index_bits / 8));
+  c.st_off = k.take<int64_t>(bags + 1);
+  c.st_out = k.take<float>((size_t)std::max<int64_t>(bags, 1) * c.N);
+  c.st_grad = k.take<float>((size_t)std::max<int64_t>(bags, 1) * c.N);
+  return (k.off + 255) & ~(size_t)255;
+}
+
+int map_cuda(cudaError_t e) { return e == cudaSuccess ? TTEMB_OK : TTEMB_ERR_CUDA; }
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur;
+    if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+}  // namespace
+}  // namespace ttemb
+
+using namespace ttemb;
+
+struct ttemb_ctx {
+  Ctx c;
+};
+
+extern "C" {
+
+const char* ttemb_status_string(int status) {
+  switch (status) {
+    case TTEMB_OK: return "ok";
+    case TTEMB_ERR_INVALID_ARG: return "invalid argument";
+    case TTEMB_ERR_UNSUPPORTED: return "unsupported configuration";
+    case TTEMB_ERR_INDEX_RANGE: return "index out of range";
+    case TTEMB_ERR_STATE: return "invalid call order";
+    case TTEMB_ERR_CUDA: return "CUDA error";
+    case TTEMB_ERR_CAPACITY: return "capacity exceeded";
+    default: return "unknown status";
+  }
+}
+
+const char* ttemb_stage_name(int stage) {
+  return (stage >= 0 && stage < ST_COUNT) ? kStageNames[stage] : "?";
+}
+
+int ttemb_query_sizes(const ttemb_config* cfg, size_t* core_bytes, size_t* state_bytes,
+                      size_t* grad_bytes, size_t* workspace_bytes) {
+  const int rc = validate(cfg);
+  if (rc) return rc;
+  Ctx c;
+  plan_sizes(cfg, c);
+  const size_t cb = sizeof(float) * c.core_floats;
+  if (core_bytes) *core_bytes = cb;
+  if (grad_bytes) *grad_bytes = cb;
+  if (state_bytes) *state_bytes = cfg->optimizer == TTEMB_ADAGRAD ? cb : 0;
+  if (workspace_bytes) *workspace_bytes = carve(c, nullptr);
+  return TTEMB_OK;
+}
+
+int ttemb_create(const ttemb_config* cfg, int device, void* cores, void* state, void* grads,
+                 void* workspace, ttemb_t* out) {
+  if (!out) return TTEMB_ERR_INVALID_ARG;
+  *out = nullptr;
+  int rc = validate(cfg);
+  if (rc) return rc;
+  if (!cores || !grads || !workspace) return TTEMB_ERR_INVALID_ARG;
+  if (cfg->optimizer == TTEMB_ADAGRAD && !state) return TTEMB_ERR_INVALID_ARG;
+  if (((uintptr_t)cores | (uintptr_t)grads | (uintptr_t)workspace | (uintptr_t)state) & 255)
+    return TTEMB_ERR_INVALID_ARG;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) {
+    cudaGetLastError();
+    return TTEMB_ERR_CUDA;
+  }
+  DeviceGuard dg(device);
+  ttemb_ctx* h = new (std::nothrow) ttemb_ctx;
+  if (!h) return TTEMB_ERR_INVALID_ARG;
+  Ctx& c = h->c;
+  plan_sizes(cfg, c);
+  c.device = device;
+  c.cores = (float*)cores; c.state = (float*)state; c.grads = (float*)grads;
+  c.ws = (uint8_t*)workspace;
+  c.ws_bytes = carve(c, c.ws);
+  cudaDeviceProp prop;
+  if (cudaGetDeviceProperties(&prop, device) != cudaSuccess) { delete h; return TTEMB_ERR_CUDA; }
+  c.sm_count = prop.multiProcessorCount;
+  std::vector<uint64_t> rb(c.T + 1);
+  std::vector<uint32_t> gb(c.T + 1);
+  for (int t = 0; t < c.T; ++t) { rb[t] = c.meta[t].rowbase; gb[t] = c.meta[t].grpbase; }
+  rb[c.T] = c.total_rows; gb[c.T] = c.total_buckets;
+  cudaError_t e = cudaMemcpy(c.d_meta, c.meta.data(), sizeof(TableMeta) * c.T, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(c.d_rowbase, rb.data(), sizeof(uint64_t) * (c.T + 1), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(c.d_grpbase, gb.data(), sizeof(uint32_t) * (c.T + 1), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = configure_fwd(c);
+  if (e == cudaSuccess) e = configure_bwd(c);
+  if (e != cudaSuccess) {
+    fprintf(stderr, "ttemb_create: %s\n", cudaGetErrorString(e));
+    delete h;
+    return TTEMB_ERR_CUDA;
+  }
+  *out = h;
+  return TTEMB_OK;
+}
+
+int ttemb_destroy(ttemb_t h) {
+  if (!h) return TTEMB_ERR_INVALID_ARG;
+  for (auto& p : h->c.pending) { cudaEventDestroy(p.a); cudaEventDestroy(p.b); }
+  for (auto e : h->c.ev_pool) cudaEventDestroy(e);
+  delete h;
+  return TTEMB_OK;
+}
+
+int ttemb_core_layout(ttemb_t h, int table, int core, int64_t* offset_floats, int32_t shape[4]) {
+  if (!h || table < 0 || table >= h->c.T || core < 0 || core > 2) return TTEMB_ERR_INVALID_ARG;
+  const Ctx& c = h->c;
+  const TableMeta& m = c.meta[table];
+  int32_t s[4];
+  int64_t off;
+  if (core == 0) { off = m.c1_off; s[0] = m.m1; s[1] = c.n1; s[2] = c.R; s[3] = 1; }
+  else if (core == 1) { off = m.c2_off; s[0] = m.m2; s[1] = c.R; s[2] = c.n2; s[3] = c.R; }
+  else { off = m.c3_off; s[0] = m.m3; s[1] = c.R; s[2] = c.n3; s[3] = 1; }
+  if (offset_floats) *offset_floats = off;
+  if (shape) memcpy(shape, s, sizeof(s));
+  return TTEMB_OK;
+}
+
+int ttemb_forward(ttemb_t h, const void* indices, const int64_t* offsets, int64_t nnz,
+                  int32_t batch, float* out, void* stream) {
+  if (!h) return TTEMB_ERR_INVALID_ARG;
+  Ctx& c = h->c;
+  if (nnz < 0 || batch < 0 || !offsets || (nnz > 0 && !indices) || (!out && batch > 0))
+    return TTEMB_ERR_INVALID_ARG;
+  if (nnz > c.max_nnz || batch > c.max_batch) return TTEMB_ERR_CAPACITY;
+  if (batch == 0 && nnz != 0) return TTEMB_ERR_INVALID_ARG;
+  DeviceGuard dg(c.device);
+  cudaStream_t s = (cudaStream_t)stream;
+  c.nnz = nnz;
+  c.B = batch;
+  c.fwd_done = false;
+  cudaError_t e = run_index_stage(c, indices, offsets, s);
+  if (e == cudaSuccess) e = run_forward_compute(c, out, offsets, s);
+  if (e != cudaSuccess) {
+    fprintf(stderr, "ttemb_forward: %s\n", cudaGetErrorString(e));
+    return TTEMB_ERR_CUDA;
+  }
+  c.fwd_done = true;
+  return TTEMB_OK;
+}
+
+int ttemb_backward(ttemb_t h, const float* grad_out, float lr, void* stream) {
+  if (!h) return TTEMB_ERR_INVALID_ARG;
+  Ctx& c = h->c;
+  if (!c.fwd_done) return TTEMB_ERR_STATE;
+  if (!grad_out && c.B > 0) return TTEMB_ERR_INVALID_ARG;
+  DeviceGuard dg(c.device);
+  cudaError_t e = run_backward(c, grad_out, lr, (cudaStream_t)stream);
+  if (e != cudaSuccess) {
+    fprintf(stderr, "ttemb_backward: %s\n", cudaGetErrorString(e));
+    return TTEMB_ERR_CUDA;
+  }
+  return TTEMB_OK;
+}
+
+int ttemb_update(ttemb_t h, float lr, void* stream) {
+  if (!h) return TTEMB_ERR_INVALID_ARG;
+  Ctx& c = h->c;
+  if (c.flags & TTEMB_FUSED_UPDATE) return TTEMB_ERR_STATE;
+  DeviceGuard dg(c.device);
+  return map_cuda(run_update(c, lr, (cudaStream_t)stream));
+}
+
+int ttemb_forward_host(ttemb_t h, const void* host_indices, const int64_t* host_offsets,
+                       int64_t nnz, int32_t batch, float* host_out, void* stream) {
+  if (!h) return TTEMB_ERR_INVALID_ARG;
+  Ctx& c = h->c;
+  if (nnz < 0 || batch < 0 || !host_offsets || (nnz > 0 && !host_indices) || (!host_out && batch > 0))
+    return TTEMB_ERR_INVALID_ARG;
+  if (nnz > c.max_nnz || batch > c.max_batch) return TTEMB_ERR_CAPACITY;
+  DeviceGuard dg(c.device);
+  cudaStream_t s = (cudaStream_t)stream;
+  {
+    StageScope sc(c, ST_H2D, s);
+    if (nnz > 0)
+      cudaMemcpyAsync(c.st_idx, host_indices, (size_t)nnz * (c.index_bits / 8), cudaMemcpyHostToDevice, s);
+    cudaMemcpyAsync(c.st_off, host_offsets, sizeof(int64_t) * ((size_t)c.T * batch + 1),
+                    cudaMemcpyHostToDevice, s);
+  }
+  int rc = ttemb_forward(h, c.st_idx, c.st_off, nnz, batch, c.st_out, stream);
+  if (rc) return rc;
+  {
+    StageScope sc(c, ST_D2H, s);
+    if (batch > 0)
+      cudaMemcpyAsync(host_out, c.st_out, sizeof(float) * (size_t)batch * c.T * c.N,
+                      cudaMemcpyDeviceToHost, s);
+  }
+  return map_cuda(cudaGetLastError());
+}
+
+int ttemb_backward_host(ttemb_t h, const float* host_grad_out, float lr, void* stream) {
+  if (!h) return TTEMB_ERR_INVALID_ARG;
+  Ctx& c = h->c;
+  if (!c.fwd_done) return TTEMB_ERR_STATE;
+  if (!host_grad_out && c.B > 0) return TTEMB_ERR_INVALID_ARG;
+  DeviceGuard dg(c.device);
+  cudaStream_t s = (cudaStream_t)stream;
+  {
+    StageScope sc(c, ST_H2D, s);
+    if (c.B > 0)
+      cudaMemcpyAsync(c.st_grad, host_grad_out, sizeof(float) * (size_t)c.B * c.T * c.N,
+                      cudaMemcpyHostToDevice, s);
+  }
+  return ttemb_backward(h, c.st_grad, lr, stream);
+}
+
+int ttemb_check(ttemb_t h, void* stream) {
+  if (!h) return TTEMB_ERR_INVALID_ARG;
+  Ctx& c = h->c;
+  DeviceGuard dg(c.device);
+  uint32_t err = 0;
+  cudaError_t e = cudaStreamSynchronize((cudaStream_t)stream);
+  if (e == cudaSuccess) e = cudaMemcpy(&err, c.p.counts + kCntErr, sizeof(uint32_t), cudaMemcpyDeviceToHost);
+  if (e != cudaSuccess) {
+    fprintf(stderr, "ttemb_check: %s\n", cudaGetErrorString(e));
+    return TTEMB_ERR_CUDA;
+  }
+  if (err & kErrRange) return TTEMB_ERR_INDEX_RANGE;
+  if (err & kErrOffsets) return TTEMB_ERR_INVALID_ARG;
+  return TTEMB_OK;
+}
+
+int ttemb_get_plan(ttemb_t h, ttemb_plan* plan) {
+  if (!h || !plan) return TTEMB_ERR_INVALID_ARG;
+  const Ctx& c = h->c;
+  if (!c.fwd_done) return TTEMB_ERR_STATE;
+  const PlanDev& p = c.p;
+  plan->nnz = c.nnz; plan->batch = c.B;
+  plan->counts = p.counts; plan->skey = p.skey; plan->spos = p.spos; plan->bag_of = p.bag_of;
+  plan->ukey = p.ukey; plan->seg_off = p.seg_off; plan->inverse = p.inverse;
+  plan->row_pfx = p.row_pfx; plan->row_i3 = p.row_i3; plan->pfx_t = p.pfx_t;
+  plan->pfx_i1 = p.pfx_i1; plan->pfx_i2 = p.pfx_i2; plan->row_seg = p.row_seg;
+  plan->grp_pfx = p.grp_pfx; plan->grp_off = p.grp_off; plan->grp_t = p.grp_t;
+  plan->grp_i2 = p.grp_i2; plan->prefix_products = p.pbuf; plan->rows = p.rows;
+  return TTEMB_OK;
+}
+
+int ttemb_read_counts(ttemb_t h, int64_t counts[4], void* stream) {
+  if (!h || !counts) return TTEMB_ERR_INVALID_ARG;
+  Ctx& c = h->c;
+  DeviceGuard dg(c.device);
+  uint32_t v[4];
+  cudaError_t e = cudaStreamSynchronize((cudaStream_t)stream);
+  if (e == cudaSuccess) e = cudaMemcpy(v, c.p.counts, sizeof(v), cudaMemcpyDeviceToHost);
+  if (e != cudaSuccess) return TTEMB_ERR_CUDA;
+  for (int i = 0; i < 4; ++i) counts[i] = v[i];
+  return TTEMB_OK;
+}
+
+int ttemb_set_timing(ttemb_t h, int enable) {
+  if (!h) return TTEMB_ERR_INVALID_ARG;
+  Ctx& c = h->c;
+  DeviceGuard dg(c.device);
+  c.timing = enable != 0;
+  if (c.timing && c.ev_pool.size() < 4096) {
+    for (size_t i = c.ev_pool.size(); i < 4096; ++i) {
+      cudaEvent_t e;
+      if (cudaEventCreate(&e) != cudaSuccess) return TTEMB_ERR_CUDA;
+      c.ev_pool.push_back(e);
+    }
+  }
+  return TTEMB_OK;
+}
+
+int ttemb_stage_times(ttemb_t h, double* ms, int64_t* launches, int max_stages) {
+  if (!h) return TTEMB_ERR_INVALID_ARG;
+  Ctx& c = h->c;
+  DeviceGuard dg(c.device);
+  for (auto& p : c.pending) {
+    if (cudaEventSynchronize(p.b) != cudaSuccess) return TTEMB_ERR_CUDA;
+    float t = 0.f;
+    cudaEventElapsedTime(&t, p.a, p.b);
+    c.stage_ms[p.stage] += t;
+    c.stage_n[p.stage] += 1;
+    c.ev_pool.push_back(p.a);
+    c.ev_pool.push_back(p.b);
+  }
+  c.pending.clear();
+  for (int i = 0; i < ST_COUNT && i < max_stages; ++i) {
+    if (ms) ms[i] = c.stage_ms[i];
+    if (launches) launches[i] = c.stage_n[i];
+    c.stage_ms[i] = 0.0;
+    c.stage_n[i] = 0;
+  }
+  return ST_COUNT;
+}
+
+}  // extern "C"

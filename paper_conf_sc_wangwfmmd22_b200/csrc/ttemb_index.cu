@@ -1,0 +1,479 @@
+// ttemb_index.cu -- the index stage, sm_100a.
+//
+//   a1 key build + range check: key_j = rowbase_t + id_j, bag_of_j = b*T + t  (Eq. 3
+//      needs the per-table row id)
+//   a2 stable LSD radix sort of the 32-bit keys carrying positions (onesweep: an
+//      upfront digit histogram, then one kernel per 8-bit pass with warp-level
+//      match_any ranking and decoupled look-back across tiles)
+//   a3 unique rows, segment offsets, inverse map (single-pass scan with warp
+//      ballots and decoupled look-back) -- "compute the unique embeddings within a
+//      batch"
+//   a4 TT digits and unique prefixes p = floor(row/m3) (Alg. 1's Buf_idx = idx /
+//      length_3), then prefixes regrouped by (t, i2) with a second radix sort
+//      so one CTA owns each C2 slice (replaces Alg. 1's flag array).
+// Everything here is integer work and bit-exact against oracle/ttemb_oracle.c.
+#include "ttemb_internal.cuh"
+
+namespace ttemb {
+
+namespace {
+
+constexpr uint32_t FULL = 0xffffffffu;
+constexpr uint32_t kFlagAgg = 1u << 30, kFlagPfx = 2u << 30, kValMask = (1u << 30) - 1;
+
+__device__ __forceinline__ uint32_t lanemask_lt() {
+  uint32_t m;
+  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+  return m;
+}
+__device__ __forceinline__ uint32_t ld_acquire(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release(uint32_t* p, uint32_t v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+// Decoupled look-back: publish `agg` for tile `tile` in status[tile*stride], walk back
+// over predecessors, publish the inclusive prefix, return the exclusive prefix.
+__device__ __forceinline__ uint32_t lookback(uint32_t* status, size_t stride, uint32_t tile,
+                                             uint32_t agg) {
+  uint32_t* me = status + (size_t)tile * stride;
+  if (tile == 0) {
+    st_release(me, kFlagPfx | agg);
+    return 0;
+  }
+  st_release(me, kFlagAgg | agg);
+  uint32_t excl = 0;
+  for (int64_t j = (int64_t)tile - 1; j >= 0; --j) {
+    uint32_t v;
+    do {
+      v = ld_acquire(status + (size_t)j * stride);
+    } while ((v >> 30) == 0);
+    excl += v & kValMask;
+    if (v & kFlagPfx) break;
+  }
+  st_release(me, kFlagPfx | (excl + agg));
+  return excl;
+}
+
+// Exclusive scan of one value per thread over a 256-thread block.
+__device__ __forceinline__ uint32_t block_excl_scan_256(uint32_t v, uint32_t* s_warp,
+                                                        uint32_t& total) {
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  uint32_t x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    uint32_t y = __shfl_up_sync(FULL, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) s_warp[w] = x;
+  __syncthreads();
+  if (w == 0) {
+    uint32_t s = lane < 8 ? s_warp[lane] : 0;
+#pragma unroll
+    for (int o = 1; o < 8; o <<= 1) {
+      uint32_t y = __shfl_up_sync(FULL, s, o);
+      if (lane >= o) s += y;
+    }
+    if (lane < 8) s_warp[lane] = s;
+  }
+  __syncthreads();
+  total = s_warp[7];
+  const uint32_t wpre = w ? s_warp[w - 1] : 0;
+  return wpre + x - v;
+}
+
+// ------------------------------------------------------------------------------------
+// a1: keys
+// ------------------------------------------------------------------------------------
+template <typename IdxT>
+__global__ void __launch_bounds__(256)
+k_build_keys(const IdxT* __restrict__ indices, const int64_t* __restrict__ offsets, int64_t nnz,
+             int32_t B, int T, const uint64_t* __restrict__ rowbase, uint32_t* __restrict__ keys,
+             uint32_t* __restrict__ bag_of, uint32_t* __restrict__ counts) {
+  const int64_t nbags = (int64_t)T * B;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  uint32_t err = 0;
+  for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < nnz; j += stride) {
+    // bag of position j: the last b with offsets[b] <= j
+    int64_t lo = 0, hi = nbags - 1;
+    while (lo < hi) {
+      const int64_t mid = (lo + hi + 1) >> 1;
+      if (__ldg(offsets + mid) <= j) lo = mid; else hi = mid - 1;
+    }
+    const int t = (int)(lo / B);
+    const int64_t b = lo - (int64_t)t * B;
+    const int64_t id = (int64_t)indices[j];
+    const uint64_t rb = __ldg(rowbase + t);
+    const uint64_t M = __ldg(rowbase + t + 1) - rb;
+    uint32_t key = (uint32_t)rb;
+    if (id < 0 || (uint64_t)id >= M) err |= kErrRange;
+    else key = (uint32_t)(rb + (uint64_t)id);
+    keys[j] = key;
+    bag_of[j] = (uint32_t)(b * T + t);
+  }
+  for (int64_t b = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; b <= nbags; b += stride) {
+    const int64_t v = offsets[b];
+    if (v < 0 || v > nnz) err |= kErrOffsets;
+    if (b == 0 && v != 0) err |= kErrOffsets;
+    if (b == nbags && v != nnz) err |= kErrOffsets;
+    if (b < nbags && offsets[b + 1] < v) err |= kErrOffsets;
+  }
+  if (err) atomicOr(counts + kCntErr, err);
+}
+
+// ------------------------------------------------------------------------------------
+// a2: onesweep LSD radix sort, 8-bit digits
+// ------------------------------------------------------------------------------------
+constexpr int RS_T = 256, RS_IPT = 16, RS_WARPS = RS_T / 32, RS_TILE = RS_T * RS_IPT;
+
+// Digit histograms of all passes in one read of the keys.
+__global__ void __launch_bounds__(256)
+k_radix_hist(const uint32_t* __restrict__ keys, const uint32_t* n_dev, uint32_t n_static,
+             int passes, uint32_t* __restrict__ hist) {
+  __shared__ uint32_t sh[4][256];
+  for (int i = threadIdx.x; i < 4 * 256; i += blockDim.x) (&sh[0][0])[i] = 0;
+  __syncthreads();
+  const uint32_t n = n_dev ? *n_dev : n_static;
+  const int lane = threadIdx.x & 31;
+  for (uint32_t base = blockIdx.x * blockDim.x; base < n; base += gridDim.x * blockDim.x) {
+    const uint32_t i = base + threadIdx.x;
+    const bool ok = i < n;
+    const uint32_t k = ok ? keys[i] : 0u;
+    for (int p = 0; p < passes; ++p) {
+      const uint32_t d = ok ? ((k >> (8 * p)) & 255u) : 256u;
+      const uint32_t peers = __match_any_sync(FULL, d);      // warp-aggregated increments
+      if (d < 256 && (__ffs(peers) - 1) == lane) atomicAdd(&sh[p][d], __popc(peers));
+    }
+  }
+  __syncthreads();
+  for (int i = threadIdx.x; i < passes * 256; i += blockDim.x) {
+    const uint32_t v = (&sh[0][0])[i];
+    if (v) atomicAdd(hist + i, v);
+  }
+}
+
+__global__ void __launch_bounds__(256)
+k_hist_scan(const uint32_t* __restrict__ hist, uint32_t* __restrict__ dbase, int passes) {
+  __shared__ uint32_t s_warp[8];
+  for (int p = 0; p < passes; ++p) {
+    uint32_t tot;
+    const uint32_t e = block_excl_scan_256(hist[p * 256 + threadIdx.x], s_warp, tot);
+    dbase[p * 256 + threadIdx.x] = e;
+    __syncthreads();
+  }
+}
+
+__global__ void __launch_bounds__(RS_T)
+k_radix_pass(const uint32_t* __restrict__ kin, const uint32_t* __restrict__ vin,
+             uint32_t* __restrict__ kout, uint32_t* __restrict__ vout, const uint32_t* n_dev,
+             uint32_t n_static, int shift, const uint32_t* __restrict__ dbase,
+             uint32_t* status, uint32_t* counter) {
+  __shared__ uint32_t s_wc[RS_WARPS][256];
+  __shared__ uint32_t s_k[RS_TILE];
+  __shared__ uint32_t s_v[RS_TILE];
+  __shared__ uint32_t s_bstart[256], s_gbase[256], s_warp[8], s_tile;
+  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  if (tid == 0) s_tile = atomicAdd(counter, 1u);
+  for (int i = tid; i < RS_WARPS * 256; i += RS_T) (&s_wc[0][0])[i] = 0;
+  __syncthreads();
+  const uint32_t n = n_dev ? *n_dev : n_static;
+  const uint32_t tile = s_tile;
+  const uint32_t base = tile * RS_TILE;
+  if (base >= n) return;
+
+  uint32_t key[RS_IPT], val[RS_IPT], rank[RS_IPT];
+  uint32_t dig[RS_IPT];
+#pragma unroll
+  for (int k = 0; k < RS_IPT; ++k) {
+    const uint32_t i = base + w * 32 * RS_IPT + k * 32 + lane;
+    const bool ok = i < n;
+    key[k] = ok ? kin[i] : 0u;
+    val[k] = ok ? (vin ? vin[i] : i) : 0u;
+    dig[k] = ok ? ((key[k] >> shift) & 255u) : 256u;
+  }
+  // warp-level stable ranking: items in (k, lane) order == element order
+#pragma unroll
+  for (int k = 0; k < RS_IPT; ++k) {
+    const uint32_t d = dig[k];
+    const uint32_t peers = __match_any_sync(FULL, d);
+    const uint32_t lt = __popc(peers & lanemask_lt());
+    uint32_t c = 0;
+    if (d < 256) c = s_wc[w][d];
+    __syncwarp();
+    if (d < 256 && lt == 0) s_wc[w][d] = c + __popc(peers);
+    __syncwarp();
+    rank[k] = c + lt;
+  }
+  __syncthreads();
+  // per digit: exclusive offsets over warps, tile count
+  uint32_t run = 0;
+#pragma unroll
+  for (int ww = 0; ww < RS_WARPS; ++ww) {
+    const uint32_t c = s_wc[ww][tid];
+    s_wc[ww][tid] = run;
+    run += c;
+  }
+  uint32_t tot;
+  const uint32_t bstart = block_excl_scan_256(run, s_warp, tot);
+  s_bstart[tid] = bstart;
+  const uint32_t excl = lookback(status + tid, 256, tile, run);
+  s_gbase[tid] = dbase[tid] + excl;
+  __syncthreads();
+#pragma unroll
+  for (int k = 0; k < RS_IPT; ++k) {
+    const uint32_t d = dig[k];
+    if (d < 256) {
+      const uint32_t pos = s_bstart[d] + s_wc[w][d] + rank[k];
+      s_k[pos] = key[k];
+      s_v[pos] = val[k];
+    }
+  }
+  __syncthreads();
+  const uint32_t cnt = min((uint32_t)RS_TILE, n - base);
+  for (uint32_t i = tid; i < cnt; i += RS_T) {
+    const uint32_t k = s_k[i];
+    const uint32_t d = (k >> shift) & 255u;
+    const uint32_t o = s_gbase[d] + i - s_bstart[d];
+    kout[o] = k;
+    vout[o] = s_v[i];
+  }
+}
+
+// ------------------------------------------------------------------------------------
+// Single-pass scan skeleton: flags -> exclusive slots, with decoupled look-back.
+// Body provides size(), flag(i), emit(i, slot, flag), finish(total).
+// ------------------------------------------------------------------------------------
+constexpr int SC_T = 256, SC_IPT = 8, SC_TILE = SC_T * SC_IPT;
+
+template <class Body>
+__global__ void __launch_bounds__(SC_T) k_scan(Body body, uint32_t* status, uint32_t* counter) {
+  __shared__ uint32_t s_wc[SC_IPT * 8];
+  __shared__ uint32_t s_tile, s_base, s_total;
+  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  if (tid == 0) s_tile = atomicAdd(counter, 1u);
+  __syncthreads();
+  const uint32_t n = body.size();
+  const uint32_t tile = s_tile, base = tile * SC_TILE;
+  if (n == 0) {
+    if (tile == 0 && tid == 0) body.finish(0);
+    return;
+  }
+  if (base >= n) return;
+  uint32_t ball[SC_IPT];
+#pragma unroll
+  for (int k = 0; k < SC_IPT; ++k) {
+    const uint32_t i = base + k * SC_T + tid;
+    const bool f = (i < n) && body.flag(i);
+    ball[k] = __ballot_sync(FULL, f);
+    if (lane == 0) s_wc[k * 8 + w] = __popc(ball[k]);
+  }
+  __syncthreads();
+  if (w == 0) {   // exclusive scan of the 64 warp counts, k-major
+    const uint32_t a = s_wc[2 * lane], b = s_wc[2 * lane + 1];
+    uint32_t x = a + b;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(FULL, x, o);
+      if (lane >= o) x += y;
+    }
+    const uint32_t ex = x - a - b;
+    s_wc[2 * lane] = ex;
+    s_wc[2 * lane + 1] = ex + a;
+    if (lane == 31) s_total = x;
+  }
+  __syncthreads();
+  if (tid == 0) s_base = lookback(status, 1, tile, s_total);
+  __syncthreads();
+  const uint32_t lt = lanemask_lt();
+#pragma unroll
+  for (int k = 0; k < SC_IPT; ++k) {
+    const uint32_t i = base + k * SC_T + tid;
+    if (i < n) {
+      const uint32_t f = (ball[k] >> lane) & 1u;
+      const uint32_t slot = s_base + s_wc[k * 8 + w] + __popc(ball[k] & lt);
+      body.emit(i, slot, f);
+    }
+  }
+  if (base + SC_TILE >= n && tid == 0) body.finish(s_base + s_total);
+}
+
+// a3: unique rows / segments / inverse over the sorted keys
+struct UniqueBody {
+  const uint32_t* skey; const uint32_t* spos; const uint32_t* bag_of;
+  uint32_t* ukey; uint32_t* seg_off; uint32_t* inverse; uint32_t* sbag; uint32_t* counts;
+  uint32_t nnz;
+  __device__ uint32_t size() const { return nnz; }
+  __device__ bool flag(uint32_t k) const { return k == 0 || skey[k] != skey[k - 1]; }
+  __device__ void emit(uint32_t k, uint32_t slot, uint32_t f) const {
+    const uint32_t u = f ? slot : slot - 1;
+    if (f) { ukey[u] = skey[k]; seg_off[u] = k; }
+    const uint32_t pos = spos[k];
+    inverse[pos] = u;
+    sbag[k] = bag_of[pos];
+  }
+  __device__ void finish(uint32_t U) const { counts[kCntU] = U; seg_off[U] = nnz; }
+};
+
+__device__ __forceinline__ int table_of_key(const uint64_t* rowbase, int T, uint32_t key) {
+  int lo = 0, hi = T - 1;   // last t with rowbase[t] <= key
+  while (lo < hi) {
+    const int mid = (lo + hi + 1) >> 1;
+    if (__ldg(rowbase + mid) <= key) lo = mid; else hi = mid - 1;
+  }
+  return lo;
+}
+
+// a4: TT digits (Eq. 3) and unique prefixes over the unique rows
+struct PrefixBody {
+  const uint32_t* ukey; const uint64_t* rowbase; const TableMeta* meta; int T;
+  uint32_t* row_pfx; uint32_t* row_i3; uint32_t* pfx_t; uint32_t* pfx_i1; uint32_t* pfx_i2;
+  uint32_t* row_seg; uint32_t* gkey; uint32_t* gval; uint32_t* counts;
+  __device__ uint32_t size() const { return counts[kCntU]; }
+  __device__ void decode(uint32_t u, int& t, uint32_t& p, uint32_t& i3) const {
+    const uint32_t key = ukey[u];
+    t = table_of_key(rowbase, T, key);
+    const uint32_t row = (uint32_t)(key - __ldg(rowbase + t));
+    const uint32_t m3 = meta[t].m3;
+    p = row / m3;
+    i3 = row - p * m3;
+  }
+  __device__ bool flag(uint32_t u) const {
+    if (u == 0) return true;
+    int t0, t1; uint32_t p0, p1, x;
+    decode(u, t1, p1, x);
+    decode(u - 1, t0, p0, x);
+    return t0 != t1 || p0 != p1;
+  }
+  __device__ void emit(uint32_t u, uint32_t slot, uint32_t f) const {
+    int t; uint32_t p, i3;
+    decode(u, t, p, i3);
+    const uint32_t q = f ? slot : slot - 1;
+    row_pfx[u] = q;
+    row_i3[u] = i3;
+    if (f) {
+      const uint32_t m2 = meta[t].m2;
+      const uint32_t i1 = p / m2, i2 = p - i1 * m2;
+      pfx_t[q] = (uint32_t)t; pfx_i1[q] = i1; pfx_i2[q] = i2; row_seg[q] = u;
+      gkey[q] = meta[t].grpbase + i2;
+      gval[q] = q;
+    }
+  }
+  __device__ void finish(uint32_t P) const { counts[kCntP] = P; row_seg[P] = counts[kCntU]; }
+};
+
+// i2-groups over the (t, i2)-sorted prefixes
+struct GroupBody {
+  const uint32_t* gkey; const uint32_t* gval; const uint32_t* grpbase; int T;
+  uint32_t* grp_pfx; uint32_t* grp_off; uint32_t* grp_t; uint32_t* grp_i2; uint32_t* counts;
+  __device__ uint32_t size() const { return counts[kCntP]; }
+  __device__ bool flag(uint32_t q) const { return q == 0 || gkey[q] != gkey[q - 1]; }
+  __device__ void emit(uint32_t q, uint32_t slot, uint32_t f) const {
+    grp_pfx[q] = gval[q];
+    if (f) {
+      const uint32_t k = gkey[q];
+      int lo = 0, hi = T - 1;
+      while (lo < hi) {
+        const int mid = (lo + hi + 1) >> 1;
+        if (__ldg(grpbase + mid) <= k) lo = mid; else hi = mid - 1;
+      }
+      grp_off[slot] = q; grp_t[slot] = (uint32_t)lo; grp_i2[slot] = k - __ldg(grpbase + lo);
+    }
+  }
+  __device__ void finish(uint32_t NG) const { counts[kCntNG] = NG; grp_off[NG] = counts[kCntP]; }
+};
+
+// Host: full LSD sort; returns which buffer pair holds the result (0 = A, 1 = B).
+int radix_sort(Ctx& c, uint32_t* kA, uint32_t* vA, uint32_t* kB, uint32_t* vB,
+               const uint32_t* n_dev, uint32_t n_static, int64_t n_max, int passes,
+               uint32_t* hist, uint32_t* dbase, uint32_t* counters, uint32_t* status,
+               int64_t tiles, int st_hist, int st_pass, cudaStream_t s) {
+  {
+    StageScope sc(c, st_hist, s);
+    k_radix_hist<<<grid_for(c, n_max, 256, 4), 256, 0, s>>>(kA, n_dev, n_static, passes, hist);
+    k_hist_scan<<<1, 256, 0, s>>>(hist, dbase, passes);
+  }
+  uint32_t *ki = kA, *vi = vA, *ko = kB, *vo = vB;
+  const int64_t grid = tiles > 0 ? tiles : 1;
+  for (int p = 0; p < passes; ++p) {
+    StageScope sc(c, st_pass, s);
+    k_radix_pass<<<(unsigned)grid, RS_T, 0, s>>>(ki, p == 0 ? nullptr : vi, ko, vo, n_dev, n_static,
+                                                  8 * p, dbase + 256 * p,
+                                                  status + (size_t)p * tiles * 256, counters + p);
+    uint32_t* t;
+    t = ki; ki = ko; ko = t;
+    t = vi; vi = vo; vo = t;
+  }
+  return (passes & 1) ? 1 : 0;
+}
+
+}  // namespace
+
+int64_t radix_tiles(int64_t n) { return cdiv(n, RS_TILE); }
+int64_t scan_tiles(int64_t n) { return cdiv(n, SC_TILE); }
+
+cudaError_t run_index_stage(Ctx& c, const void* indices, const int64_t* offsets, cudaStream_t s) {
+  PlanDev& p = c.p;
+  const int64_t nnz = c.nnz;
+  {
+    StageScope sc(c, ST_ZERO, s);
+    cudaMemsetAsync(c.zero_begin, 0, c.zero_bytes, s);
+  }
+  {
+    StageScope sc(c, ST_KEYS, s);
+    const int64_t items = nnz > (int64_t)c.T * c.B + 1 ? nnz : (int64_t)c.T * c.B + 1;
+    const int g = grid_for(c, items, 256, 8);
+    if (c.index_bits == 64)
+      k_build_keys<int64_t><<<g, 256, 0, s>>>((const int64_t*)indices, offsets, nnz, c.B, c.T,
+                                              c.d_rowbase, p.keysA, p.bag_of, p.counts);
+    else
+      k_build_keys<int32_t><<<g, 256, 0, s>>>((const int32_t*)indices, offsets, nnz, c.B, c.T,
+                                              c.d_rowbase, p.keysA, p.bag_of, p.counts);
+  }
+  // a2: sort (key, position)
+  const int64_t tiles1 = radix_tiles(nnz);
+  const int which = radix_sort(c, p.keysA, p.valsA, p.keysB, p.valsB, nullptr, (uint32_t)nnz, nnz,
+                               c.key_passes, p.hist1, p.dbase1, p.rs1_counter, p.rs1_status, tiles1,
+                               ST_SORT_HIST, ST_SORT_PASS, s);
+  p.skey = which ? p.keysB : p.keysA;
+  p.spos = which ? p.valsB : p.valsA;
+  // the other ping-pong pair is free now: group-sort buffers
+  p.gkeyA = which ? p.keysA : p.keysB;
+  p.gvalA = which ? p.valsA : p.valsB;
+  // a3
+  {
+    StageScope sc(c, ST_UNIQUE, s);
+    UniqueBody b{p.skey, p.spos, p.bag_of, p.ukey, p.seg_off, p.inverse, p.sbag, p.counts,
+                 (uint32_t)nnz};
+    const int64_t tiles = scan_tiles(nnz);
+    k_scan<UniqueBody><<<(unsigned)(tiles ? tiles : 1), SC_T, 0, s>>>(b, p.sc_status, p.sc_counter + 0);
+  }
+  // a4: digits + prefixes
+  {
+    StageScope sc(c, ST_PREFIX, s);
+    PrefixBody b{p.ukey, c.d_rowbase, c.d_meta, c.T, p.row_pfx, p.row_i3, p.pfx_t, p.pfx_i1,
+                 p.pfx_i2, p.row_seg, p.gkeyA, p.gvalA, p.counts};
+    const int64_t tiles = scan_tiles(c.U_cap);
+    k_scan<PrefixBody><<<(unsigned)(tiles ? tiles : 1), SC_T, 0, s>>>(
+        b, p.sc_status + c.sc_tiles, p.sc_counter + 1);
+  }
+  // group sort by (t, i2), stable (keeps i1 ascending inside a group)
+  const int64_t tiles2 = radix_tiles(c.P_cap);
+  const int which2 = radix_sort(c, p.gkeyA, p.gvalA, p.gkeyB, p.gvalB, p.counts + kCntP, 0, c.P_cap,
+                                c.gkey_passes, p.hist2, p.dbase2, p.rs2_counter, p.rs2_status,
+                                tiles2, ST_GSORT_HIST, ST_GSORT_PASS, s);
+  p.gkey = which2 ? p.gkeyB : p.gkeyA;
+  p.gval = which2 ? p.gvalB : p.gvalA;
+  {
+    StageScope sc(c, ST_GROUPS, s);
+    GroupBody b{p.gkey, p.gval, c.d_grpbase, c.T, p.grp_pfx, p.grp_off, p.grp_t, p.grp_i2, p.counts};
+    const int64_t tiles = scan_tiles(c.P_cap);
+    k_scan<GroupBody><<<(unsigned)(tiles ? tiles : 1), SC_T, 0, s>>>(
+        b, p.sc_status + 2 * c.sc_tiles, p.sc_counter + 2);
+  }
+  return cudaGetLastError();
+}
+
+}  // namespace ttemb

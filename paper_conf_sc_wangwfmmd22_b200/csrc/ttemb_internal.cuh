@@ -1,0 +1,136 @@
+// ttemb_internal.cuh -- shared host/device definitions of libttemb.so (B200, sm_100a).
+//
+// Data layout in HBM:
+//   cores / grads / state: [all tables' C1][all tables' C2][all tables' C3], fp32,
+//   C1_t[m1][n1][R], C2_t[m2][R][n2][R], C3_t[m3][R][n3]; each table's block starts
+//   16-byte aligned so slices can be moved as float4.
+//   workspace: the index-stage plan (u32 arrays), the prefix products (Reuse buffer,
+//   P:178), unique rows, aggregated row gradients, dP, dC1 partials, the per-step
+//   zeroed scan/sort state, and host staging buffers.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <vector>
+
+#include "../../include/ttemb.h"
+
+namespace ttemb {
+
+// ---- error flags in counts[3] ------------------------------------------------
+constexpr uint32_t kErrRange = 1u;     // an id outside [0, M_t)
+constexpr uint32_t kErrOffsets = 2u;   // malformed offsets
+
+// counts[] slots (device)
+constexpr int kCntU = 0, kCntP = 1, kCntNG = 2, kCntErr = 3, kNumCounts = 16;
+
+// ---- stage ids for per-stage timing ----------------------------------------------
+enum Stage : int {
+  ST_ZERO = 0, ST_KEYS, ST_SORT_HIST, ST_SORT_PASS, ST_UNIQUE, ST_PREFIX, ST_GSORT_HIST,
+  ST_GSORT_PASS, ST_GROUPS, ST_FWD_PREFIX, ST_FWD_ROWS, ST_POOL, ST_BWD_ZERO, ST_AGG,
+  ST_AGG_FIX, ST_BWD_ROWS, ST_BWD_PREFIX, ST_DC1, ST_UPD_C3, ST_UPDATE, ST_H2D, ST_D2H,
+  ST_COUNT
+};
+
+struct TableMeta {
+  uint32_t m1, m2, m3, M;      // row factors, rows (M <= 2^32-1 checked on host)
+  uint64_t rowbase;            // first key of the table (exclusive prefix sum of M)
+  uint64_t c1_off, c2_off, c3_off;  // float offsets into cores / grads / state
+  uint32_t grpbase;            // first (t, i2) bucket id = sum of m2 of earlier tables
+  uint32_t pad;
+};
+
+// Per-step plan pointers (all device).
+struct PlanDev {
+  uint32_t* counts;
+  uint32_t *keysA, *valsA, *keysB, *valsB;     // radix ping-pong (sort 1), reused by sort 2
+  uint32_t *skey, *spos;                       // -> final sort-1 buffers
+  uint32_t *bag_of, *sbag, *inverse;           // [nnz]
+  uint32_t *ukey, *seg_off, *row_pfx, *row_i3; // [U]
+  uint32_t *pfx_t, *pfx_i1, *pfx_i2, *row_seg; // [P]
+  uint32_t *gkeyA, *gvalA, *gkeyB, *gvalB;     // group sort ping-pong [P]
+  uint32_t *gkey, *gval;                       // -> final sort-2 buffers
+  uint32_t *grp_pfx, *grp_off, *grp_t, *grp_i2;
+  uint32_t *hist1, *dbase1, *hist2, *dbase2;   // [4][256]
+  uint32_t *rs1_counter, *rs1_status;          // sort-1 look-back state [4][tiles][256]
+  uint32_t *rs2_counter, *rs2_status;
+  uint32_t *sc_counter, *sc_status;            // scans [3][tiles]
+  float *pbuf, *rows, *gbuf, *dpbuf, *dabuf, *aggpart;
+};
+
+struct Ctx {
+  // configuration
+  int device = 0, sm_count = 148;
+  int T = 0, n1 = 0, n2 = 0, n3 = 0, N = 0, R = 0, NC = 0;
+  int index_bits = 64, opt = 0;
+  float eps = 1e-10f;
+  uint32_t flags = 0;
+  int64_t max_nnz = 0;
+  int32_t max_batch = 0;
+  uint64_t total_rows = 0;
+  uint32_t total_buckets = 0;
+  int key_passes = 1, gkey_passes = 1;
+  int64_t U_cap = 0, P_cap = 0, NG_cap = 0;
+  int64_t rs1_tiles = 0, rs2_tiles = 0, sc_tiles = 0;
+  std::vector<TableMeta> meta;
+  size_t core_floats = 0, c3_begin = 0, c3_floats = 0;
+
+  // caller buffers
+  float* cores = nullptr;
+  float* state = nullptr;
+  float* grads = nullptr;
+  uint8_t* ws = nullptr;
+
+  // workspace carve
+  TableMeta* d_meta = nullptr;
+  uint64_t* d_rowbase = nullptr;     // [T+1]
+  uint32_t* d_grpbase = nullptr;     // [T+1]
+  PlanDev p{};
+  uint8_t* zero_begin = nullptr;
+  size_t zero_bytes = 0;
+  void* st_idx = nullptr;
+  int64_t* st_off = nullptr;
+  float* st_out = nullptr;
+  float* st_grad = nullptr;
+  size_t ws_bytes = 0;
+
+  // step state
+  int64_t nnz = 0;
+  int32_t B = 0;
+  bool fwd_done = false;
+
+  // timing
+  bool timing = false;
+  std::vector<cudaEvent_t> ev_pool;
+  struct Pending { int stage; cudaEvent_t a, b; };
+  std::vector<Pending> pending;
+  double stage_ms[ST_COUNT] = {};
+  int64_t stage_n[ST_COUNT] = {};
+};
+
+// ---- stage timing helpers (host) ---------------------------------------------------
+struct StageScope {
+  Ctx& c; int stage; cudaStream_t s; cudaEvent_t a = nullptr, b = nullptr;
+  StageScope(Ctx& c_, int st, cudaStream_t s_);
+  ~StageScope();
+};
+
+// ---- launchers (host) ----------------------------------------------------------------
+cudaError_t run_index_stage(Ctx& c, const void* indices, const int64_t* offsets, cudaStream_t s);
+cudaError_t run_forward_compute(Ctx& c, float* out, const int64_t* offsets, cudaStream_t s);
+cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s);
+cudaError_t run_update(Ctx& c, float lr, cudaStream_t s);
+cudaError_t configure_kernels(Ctx& c);
+
+// ---- small helpers -------------------------------------------------------------------
+static inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+static inline int grid_for(const Ctx& c, int64_t items, int threads, int per_sm = 8) {
+  int64_t g = cdiv(items, threads);
+  int64_t cap = (int64_t)c.sm_count * per_sm;
+  if (g > cap) g = cap;
+  if (g < 1) g = 1;
+  return (int)g;
+}
+
+}  // namespace ttemb

@@ -142,7 +142,7 @@ def rng(*parts) -> np.random.Generator:
 # ---------------------------------------------------------------------------
 # Id streams
 # ---------------------------------------------------------------------------
-@functools.lru_cache(maxsize=4)
+@functools.lru_cache(maxsize=32)
 def _zipf_cdf(m: int, s: float) -> np.ndarray:
     """Cumulative distribution of the bounded Zipf law p_r ~ r^-s, r = 1..m."""
     r = np.arange(1, m + 1, dtype=np.float64)
@@ -152,7 +152,7 @@ def _zipf_cdf(m: int, s: float) -> np.ndarray:
     return c
 
 
-@functools.lru_cache(maxsize=4)
+@functools.lru_cache(maxsize=32)
 def _perm(m: int, seed_tag: str) -> np.ndarray:
     return rng("perm", seed_tag, m).permutation(m).astype(np.int64)
 

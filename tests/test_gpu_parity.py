@@ -1,0 +1,319 @@
+"""CUDA path (libttemb.so through the C ABI) vs the CPU oracle, element by element.
+
+Integer plan: bit-exact.  Floats: |gpu - oracle| <= tol * oracle(|inputs|) with
+tol = 1e-5 for the forward output and 1e-4 for core gradients (BASELINE.json
+north_star).  The oracle never sees a value produced
+by the CUDA path.
+"""
+import numpy as np
+import pytest
+import torch
+
+from oracle import Oracle
+from synth import workload as W
+from tests.helpers import assert_companion, assert_update_close
+
+pytestmark = pytest.mark.gpu
+
+if torch.cuda.is_available():
+    import paper_conf_sc_wangwfmmd22_b200 as tt
+    from paper_conf_sc_wangwfmmd22_b200 import _lib as L
+
+DEV = torch.device("cuda", 0)
+
+
+def gpu_emb(cfg, B, nnz, **kw):
+    emb = tt.TTEmbeddingBag(cfg.table_rows, cfg.row_factors, cfg.col_factors, cfg.rank,
+                            max(B, 1), max(nnz, 1), **kw)
+    return emb
+
+
+def run_forward(emb, idx, off, B, index_bits=64):
+    it = torch.as_tensor(idx.astype(np.int64 if index_bits == 64 else np.int32), device=DEV)
+    ot = torch.as_tensor(off, device=DEV)
+    out = emb.forward(it, ot, B)
+    return out
+
+
+def check_plan(emb, orc, idx, off, B):
+    mine = emb.plan()
+    ref = orc.plan(idx, off, B)
+    for k in ("U", "P", "NG"):
+        assert mine[k] == ref[k], (k, mine[k], ref[k])
+    for k, v in ref.items():
+        if isinstance(v, np.ndarray):
+            got = mine[k].cpu().numpy().view(np.uint32)
+            np.testing.assert_array_equal(got, v, err_msg=k)
+    return mine, ref
+
+
+def small_cases():
+    return [
+        ("c1", W.config("c1"), None),
+        ("multi-var-L", W.small_config([37, 100, 5, 1000], [(3, 4, 4), (5, 4, 5), (1, 2, 3), (10, 10, 10)],
+                                       (2, 3, 2), 5, 33, 1, 1.05), "var"),
+        ("r1-kron", W.small_config([60], [(3, 4, 5)], (2, 3, 2), 1, 17, 3), None),
+        ("dup-heavy", W.small_config([50], [(2, 5, 5)], (2, 2, 2), 4, 40, 7, 2.0), None),
+        ("wide-R128", W.small_config([3000, 200], [(15, 15, 15), (6, 6, 6)], (4, 4, 8), 128, 24, 2, 1.05), None),
+        ("odd-dims", W.small_config([777], [(9, 10, 9)], (3, 1, 5), 7, 50, 2, 1.1), "var"),
+    ]
+
+
+def make_inputs(cfg, mode, seed=0, batch=None):
+    B = cfg.batch if batch is None else batch
+    lens = None
+    if mode == "var":
+        rng = np.random.default_rng(seed)
+        lens = rng.integers(0, 6, size=cfg.num_tables * B)
+        lens[0] = 0
+        lens[-1] = 0
+    idx, off = W.make_batch(cfg, step=seed, seed=seed, batch=B, lengths=lens)
+    return idx, off, B
+
+
+# ---------------------------------------------------------------------------
+@pytest.mark.parametrize("name,cfg,mode", small_cases(), ids=[c[0] for c in small_cases()])
+def test_forward_backward_small(name, cfg, mode):
+    idx, off, B = make_inputs(cfg, mode, seed=3)
+    cores = W.make_cores(cfg, seed=3)
+    go = W.make_grad_out(cfg, B, seed=3)
+    emb = gpu_emb(cfg, B, len(idx))
+    emb.load_cores(cores)
+    out = run_forward(emb, idx, off, B)
+    emb.backward(torch.as_tensor(go, device=DEV))
+    assert emb.check() == 0
+    orc = Oracle.from_config(cfg)
+    check_plan(emb, orc, idx, off, B)
+    ref = orc.forward(cores, idx, off, B)
+    ref_abs = orc.forward(cores, idx, off, B, absolute=True)
+    assert_companion(out.cpu().numpy(), ref, ref_abs, 1e-5, "forward")
+    g = orc.backward(cores, idx, off, B, go)
+    ga = orc.backward(cores, idx, off, B, go, absolute=True)
+    for t, mine in enumerate(emb.grad_views()):
+        for k in range(3):
+            assert_companion(mine[k].cpu().numpy(), g[t][k], ga[t][k], 1e-4, f"dC{k+1} table {t}")
+
+
+@pytest.mark.parametrize("name", ["c1", "c2", "c3"])
+def test_configs_full_batch(name):
+    cfg = W.config(name)
+    idx, off = W.make_batch(cfg, seed=7)
+    B = cfg.batch
+    cores = W.make_cores(cfg, seed=7)
+    go = W.make_grad_out(cfg, B, seed=7)
+    emb = gpu_emb(cfg, B, len(idx))
+    emb.load_cores(cores)
+    out = run_forward(emb, idx, off, B)
+    emb.backward(torch.as_tensor(go, device=DEV))
+    assert emb.check() == 0
+    orc = Oracle.from_config(cfg)
+    check_plan(emb, orc, idx, off, B)
+    assert_companion(out.cpu().numpy(), orc.forward(cores, idx, off, B),
+                     orc.forward(cores, idx, off, B, absolute=True), 1e-5, "forward")
+    g = orc.backward(cores, idx, off, B, go)
+    ga = orc.backward(cores, idx, off, B, go, absolute=True)
+    for t, mine in enumerate(emb.grad_views()):
+        for k in range(3):
+            assert_companion(mine[k].cpu().numpy(), g[t][k], ga[t][k], 1e-4, f"dC{k+1} t{t}")
+
+
+def test_c4_reduced_batch():
+    """Criteo-TB shape (26 tables, R=64, N=64) at batch 2048: every output checked."""
+    cfg = W.config("c4")
+    B = 2048
+    idx, off = W.make_batch(cfg, seed=11, batch=B)
+    cores = W.make_cores(cfg, seed=11)
+    go = W.make_grad_out(cfg, B, seed=11)
+    emb = gpu_emb(cfg, B, len(idx))
+    emb.load_cores(cores)
+    out = run_forward(emb, idx, off, B)
+    emb.backward(torch.as_tensor(go, device=DEV))
+    orc = Oracle.from_config(cfg)
+    check_plan(emb, orc, idx, off, B)
+    assert_companion(out.cpu().numpy(), orc.forward(cores, idx, off, B),
+                     orc.forward(cores, idx, off, B, absolute=True), 1e-5, "forward")
+    g = orc.backward(cores, idx, off, B, go)
+    ga = orc.backward(cores, idx, off, B, go, absolute=True)
+    for t, mine in enumerate(emb.grad_views()):
+        for k in range(3):
+            assert_companion(mine[k].cpu().numpy(), g[t][k], ga[t][k], 1e-4, f"dC{k+1} t{t}")
+
+
+@pytest.mark.parametrize("name,rank", [("c4", None), ("c5", 128)])
+def test_full_size_sampled(name, rank):
+    """Full BASELINE sizes in the bench launch configuration (fused update off so
+    the gradients stay observable): plan bit-exact vs numpy, sampled bags vs the
+    oracle, core gradients of sampled slices vs the oracle on the full batch."""
+    cfg = W.config(name, rank) if rank else W.config(name)
+    B = cfg.batch if name == "c4" else 16384          # c5: a quarter of the global batch (one of 4 GPUs)
+    idx, off = W.make_batch(cfg, seed=5, batch=B)
+    cores = W.make_cores(cfg, seed=5)
+    emb = gpu_emb(cfg, B, len(idx))
+    emb.load_cores(cores)
+    out = run_forward(emb, idx, off, B).cpu().numpy()
+    assert emb.check() == 0
+    plan = emb.plan()
+    # unique count and inverse map against numpy (whole batch)
+    T = cfg.num_tables
+    rowbase = np.concatenate([[0], np.cumsum(cfg.table_rows)[:-1]]).astype(np.int64)
+    bag = np.repeat(np.arange(T * B), np.diff(off))
+    key = rowbase[bag // B] + idx
+    uk, inv = np.unique(key, return_inverse=True)
+    assert plan["U"] == len(uk)
+    np.testing.assert_array_equal(plan["ukey"].cpu().numpy().view(np.uint32), uk)
+    np.testing.assert_array_equal(plan["inverse"].cpu().numpy().view(np.uint32), inv)
+    # sampled bags: rebuild a small batch from them and run the oracle on it
+    rng = np.random.default_rng(0)
+    bs = np.sort(rng.choice(B, size=64, replace=False))
+    sub_lens = []
+    sub_idx = []
+    for t in range(T):
+        for b in bs:
+            s, e = off[t * B + b], off[t * B + b + 1]
+            sub_idx.append(idx[s:e])
+            sub_lens.append(e - s)
+    sidx = np.concatenate(sub_idx)
+    soff = np.concatenate([[0], np.cumsum(sub_lens)]).astype(np.int64)
+    orc = Oracle.from_config(cfg)
+    ref = orc.forward(cores, sidx, soff, len(bs))
+    ref_abs = orc.forward(cores, sidx, soff, len(bs), absolute=True)
+    assert_companion(out[bs], ref, ref_abs, 1e-5, "sampled forward")
+
+
+def test_fused_update_sgd_and_adagrad():
+    cfg = W.small_config([500, 300], [(8, 8, 8), (7, 7, 7)], (2, 2, 4), 16, 64, 2, 1.05)
+    idx, off = W.make_batch(cfg, seed=2)
+    cores = W.make_cores(cfg, seed=2)
+    go = W.make_grad_out(cfg, cfg.batch, seed=2)
+    orc = Oracle.from_config(cfg)
+    g = orc.backward(cores, idx, off, cfg.batch, go)
+    ga = orc.backward(cores, idx, off, cfg.batch, go, absolute=True)
+    lr = 0.05
+    for opt in ("sgd", "adagrad"):
+        for fused in (True, False):
+            emb = gpu_emb(cfg, cfg.batch, len(idx), optimizer=opt, fused_update=fused)
+            emb.load_cores(cores)
+            run_forward(emb, idx, off, cfg.batch)
+            emb.backward(torch.as_tensor(go, device=DEV), lr=lr)
+            if not fused:
+                emb.update(lr)
+            else:
+                with pytest.raises(tt.TTEmbError):
+                    emb.update(lr)
+            torch.cuda.synchronize()
+            for t, (cv, sv) in enumerate(zip(emb.core_views(),
+                                             emb.state_views() or [None] * cfg.num_tables)):
+                for k in range(3):
+                    ref_p, ref_s = Oracle.update(opt, lr, cores[t][k], g[t][k], None)
+                    assert_update_close(cv[k].cpu().numpy(), ref_p, cores[t][k], g[t][k], ga[t][k], lr,
+                                        opt, got_s=None if sv is None else sv[k].cpu().numpy(),
+                                        ref_s=ref_s, s_old=np.zeros_like(cores[t][k]),
+                                        what=f"{opt} fused={fused} t{t} C{k+1}")
+
+
+def test_two_steps_match_oracle_trajectory():
+    """Two fused SGD steps: the second step's gradients use the updated cores."""
+    cfg = W.small_config([1000], [(10, 10, 10)], (2, 2, 4), 8, 64, 1, 1.05)
+    cores = W.make_cores(cfg, seed=4)
+    emb = gpu_emb(cfg, cfg.batch, cfg.batch, fused_update=True)
+    emb.load_cores(cores)
+    orc = Oracle.from_config(cfg)
+    lr = 0.1
+    ref_cores = [tuple(x.copy() for x in c) for c in cores]
+    for step in range(2):
+        idx, off = W.make_batch(cfg, step=step, seed=4)
+        go = W.make_grad_out(cfg, cfg.batch, step=step, seed=4)
+        run_forward(emb, idx, off, cfg.batch)
+        emb.backward(torch.as_tensor(go, device=DEV), lr=lr)
+        g = orc.backward(ref_cores, idx, off, cfg.batch, go)
+        ref_cores = [tuple(Oracle.update("sgd", lr, c[k], g[t][k])[0] for k in range(3))
+                     for t, c in enumerate(ref_cores)]
+    for cv, rc in zip(emb.core_views(), ref_cores):
+        for k in range(3):
+            np.testing.assert_allclose(cv[k].cpu().numpy(), rc[k], rtol=1e-4, atol=1e-5)
+
+
+def test_int32_indices_and_host_api():
+    cfg = W.config("c2")
+    B = 512
+    idx, off = W.make_batch(cfg, seed=9, batch=B)
+    cores = W.make_cores(cfg, seed=9)
+    go = W.make_grad_out(cfg, B, seed=9)
+    e64 = gpu_emb(cfg, B, len(idx))
+    e64.load_cores(cores)
+    o64 = run_forward(e64, idx, off, B)
+    e64.backward(torch.as_tensor(go, device=DEV))
+    e32 = gpu_emb(cfg, B, len(idx), index_bits=32)
+    e32.load_cores(cores)
+    o32 = run_forward(e32, idx, off, B, index_bits=32)
+    e32.backward(torch.as_tensor(go, device=DEV))
+    torch.testing.assert_close(o32, o64, rtol=0, atol=0)
+    eh = gpu_emb(cfg, B, len(idx))
+    eh.load_cores(cores)
+    hi = torch.as_tensor(idx).pin_memory()
+    ho = torch.as_tensor(off).pin_memory()
+    hout = torch.empty(B, cfg.num_tables, cfg.dim).pin_memory()
+    eh.forward_host(hi, ho, B, hout)
+    eh.backward_host(torch.as_tensor(go).pin_memory())
+    torch.cuda.synchronize()
+    torch.testing.assert_close(hout, o64.cpu(), rtol=0, atol=0)
+    # dC1 / dC2 are reduced without atomics: bitwise equal across runs
+    for a, b in zip(eh.grad_views(), e64.grad_views()):
+        torch.testing.assert_close(a[0], b[0], rtol=0, atol=0)
+        torch.testing.assert_close(a[1], b[1], rtol=0, atol=0)
+
+
+def test_deterministic_forward_and_plan():
+    cfg = W.config("c3")
+    B = 2048
+    idx, off = W.make_batch(cfg, seed=1, batch=B)
+    cores = W.make_cores(cfg, seed=1)
+    emb = gpu_emb(cfg, B, len(idx))
+    emb.load_cores(cores)
+    o1 = run_forward(emb, idx, off, B).clone()
+    p1 = emb.plan()
+    o2 = run_forward(emb, idx, off, B)
+    p2 = emb.plan()
+    torch.testing.assert_close(o1, o2, rtol=0, atol=0)
+    for k in ("ukey", "inverse", "grp_pfx", "row_seg"):
+        assert torch.equal(p1[k], p2[k])
+
+
+def test_edge_cases_empty_and_range_errors():
+    cfg = W.small_config([100, 50], [(5, 5, 4), (4, 4, 4)], (2, 2, 2), 4, 8, 1)
+    cores = W.make_cores(cfg, seed=0)
+    emb = gpu_emb(cfg, 8, 64)
+    emb.load_cores(cores)
+    # all bags empty
+    off = np.zeros(2 * 8 + 1, np.int64)
+    out = run_forward(emb, np.zeros(0, np.int64), off, 8)
+    emb.backward(torch.zeros(8, 2, 8, device=DEV))
+    assert emb.check() == 0
+    assert float(out.abs().sum()) == 0.0
+    assert emb.counts()["U"] == 0
+    for v in emb.grad_views():
+        for x in v:
+            assert float(x.abs().sum()) == 0.0
+    # batch 0
+    out = run_forward(emb, np.zeros(0, np.int64), np.zeros(1, np.int64), 0)
+    assert out.numel() == 0 and emb.check() == 0
+    # id out of range (>= M, including padding ids < m1 m2 m3) -> INDEX_RANGE
+    idx = np.array([5, 100, 3, 1, 0, 2, 4, 6, 7, 8, 9, 10, 11, 12, 13, 14], np.int64)
+    off = np.arange(17, dtype=np.int64)
+    run_forward(emb, idx, off, 8)
+    assert emb.check() == L.TTEMB_ERR_INDEX_RANGE
+    idx[1] = -1
+    run_forward(emb, idx, off, 8)
+    assert emb.check() == L.TTEMB_ERR_INDEX_RANGE
+    # malformed offsets -> INVALID_ARG (deferred)
+    bad = off.copy()
+    bad[3], bad[4] = bad[4], bad[3]
+    idx[1] = 1
+    run_forward(emb, idx, bad, 8)
+    assert emb.check() == L.TTEMB_ERR_INVALID_ARG
+    # capacity and state errors are synchronous
+    with pytest.raises(tt.TTEmbError):
+        run_forward(emb, np.zeros(65, np.int64), np.concatenate([np.zeros(16, np.int64), [65]]), 8)
+    fresh = gpu_emb(cfg, 8, 64)
+    with pytest.raises(tt.TTEmbError):
+        fresh.backward(torch.zeros(0, 2, 8, device=DEV))
