@@ -407,7 +407,7 @@ def main():
             hev[i][1].record(stream)
         torch.cuda.synchronize()
         te = sum(a.elapsed_time(b) for a, b in hev)
-        h2d = sum(p[0].numel() * 8 + p[1].numel() * 8 + p[2].numel() * 4 for p in pool) / len(pool)
+        h2d = sum(p[0].size * 8 + p[1].size * 8 + p[2].size * 4 for p in pool) / len(pool)
         e2e = {"value": look_step * args.steps / (te / 1e3), "unit": UNIT, "h2d_bytes_per_step": int(h2d),
                "d2h_bytes_per_step": int(hout.numel() * 4), "ms_per_step": te / args.steps,
                "path": "ttemb_forward_host + ttemb_backward_host (pinned host buffers)"}

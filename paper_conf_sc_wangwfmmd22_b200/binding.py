@@ -296,7 +296,7 @@ class _DevArray:
     """A raw device pointer exposed through __cuda_array_interface__ (zero-copy view)."""
 
     def __init__(self, ptr: int, n: int, typestr: str):
-        self.__cuda_array_interface__ = {"shape": (n,), "typestr": typestr, "data": (ptr, True),
+        self.__cuda_array_interface__ = {"shape": (n,), "typestr": typestr, "data": (ptr, False),
                                          "version": 2}
 
 
