@@ -59,6 +59,7 @@ typedef enum { TTEMB_SGD = 0, TTEMB_ADAGRAD = 1 } ttemb_opt;
 
 /* ttemb_config.flags */
 #define TTEMB_FUSED_UPDATE 1u   /* backward applies the update (single replica) */
+#define TTEMB_FP32_CORES 2u     /* force the FP32 CUDA-core contraction path (no tcgen05) */
 
 typedef struct {
   int64_t num_rows;        /* M_t >= 1 */
@@ -77,7 +78,7 @@ typedef struct {
   int64_t max_nnz;               /* nnz capacity, <= 2^30                             */
   int32_t optimizer;             /* ttemb_opt                                         */
   float adagrad_eps;             /* Adagrad eps (PyTorch default 1e-10)               */
-  uint32_t flags;                /* TTEMB_FUSED_UPDATE                                */
+  uint32_t flags;                /* TTEMB_FUSED_UPDATE | TTEMB_FP32_CORES             */
 } ttemb_config;
 
 typedef struct ttemb_ctx* ttemb_t;
@@ -155,7 +156,6 @@ typedef struct {
   const uint32_t* grp_off;   /* [NG+1] i2-groups (one C2 slice each)                    */
   const uint32_t* grp_t;     /* [NG] */
   const uint32_t* grp_i2;    /* [NG] */
-  const float* prefix_products; /* [P][n1][n2][R] the Reuse buffer              */
   const float* rows;         /* [U][dim] W rows of the unique ids                       */
 } ttemb_plan;
 

@@ -22,6 +22,7 @@ TTEMB_ERR_CAPACITY = -6
 TTEMB_SGD = 0
 TTEMB_ADAGRAD = 1
 TTEMB_FUSED_UPDATE = 1
+TTEMB_FP32_CORES = 2
 
 SYMBOLS = ["ttemb_query_sizes", "ttemb_create", "ttemb_destroy", "ttemb_core_layout",
            "ttemb_forward", "ttemb_backward", "ttemb_update", "ttemb_forward_host",
@@ -48,8 +49,7 @@ class ttemb_plan(C.Structure):
     _fields_ = [("nnz", C.c_int64), ("batch", C.c_int32)] + [
         (n, C.c_void_p) for n in ["counts", "skey", "spos", "bag_of", "ukey", "seg_off", "inverse",
                                   "row_pfx", "row_i3", "pfx_t", "pfx_i1", "pfx_i2", "row_seg",
-                                  "grp_pfx", "grp_off", "grp_t", "grp_i2", "prefix_products",
-                                  "rows"]]
+                                  "grp_pfx", "grp_off", "grp_t", "grp_i2", "rows"]]
 
 
 class TTEmbError(RuntimeError):

@@ -27,7 +27,7 @@ def _stream_ptr(stream: Optional[torch.cuda.Stream]) -> int:
 def make_config(table_rows: Sequence[int], row_factors: Sequence[Tuple[int, int, int]],
                 col_factors: Tuple[int, int, int], rank: int, max_batch: int, max_nnz: int,
                 optimizer: str = "sgd", adagrad_eps: float = 1e-10, fused_update: bool = False,
-                index_bits: int = 64, num_cores: int = 3):
+                index_bits: int = 64, num_cores: int = 3, fp32_cores: bool = False):
     """Returns (ttemb_config, keep-alive table array)."""
     T = len(table_rows)
     tabs = (L.ttemb_table * max(T, 1))()
@@ -48,7 +48,7 @@ def make_config(table_rows: Sequence[int], row_factors: Sequence[Tuple[int, int,
     cfg.max_nnz = int(max_nnz)
     cfg.optimizer = {"sgd": L.TTEMB_SGD, "adagrad": L.TTEMB_ADAGRAD}[optimizer]
     cfg.adagrad_eps = float(adagrad_eps)
-    cfg.flags = L.TTEMB_FUSED_UPDATE if fused_update else 0
+    cfg.flags = (L.TTEMB_FUSED_UPDATE if fused_update else 0) | (L.TTEMB_FP32_CORES if fp32_cores else 0)
     return cfg, tabs
 
 
@@ -149,7 +149,7 @@ class TTEmbeddingBag:
 
     def __init__(self, table_rows, row_factors, col_factors, rank, max_batch, max_nnz,
                  optimizer: str = "sgd", adagrad_eps: float = 1e-10, fused_update: bool = False,
-                 index_bits: int = 64, device: int = 0):
+                 index_bits: int = 64, device: int = 0, fp32_cores: bool = False):
         L.load()
         self.table_rows = [int(x) for x in table_rows]
         self.row_factors = [tuple(int(y) for y in f) for f in row_factors]
@@ -162,7 +162,8 @@ class TTEmbeddingBag:
         self.index_bits = int(index_bits)
         self.device = torch.device("cuda", device)
         self._cfg, self._tabs = make_config(table_rows, row_factors, col_factors, rank, max_batch,
-                                            max_nnz, optimizer, adagrad_eps, fused_update, index_bits)
+                                            max_nnz, optimizer, adagrad_eps, fused_update, index_bits,
+                                            fp32_cores=fp32_cores)
         cb, sb, gb, wb = ttemb_query_sizes(self._cfg)
         self.sizes = dict(core_bytes=cb, state_bytes=sb, grad_bytes=gb, workspace_bytes=wb)
         f32 = torch.float32
@@ -279,8 +280,6 @@ class TTEmbeddingBag:
         for k, n in size.items():
             out[k] = _copy_device_u32(getattr(p, k), n, self.device)
         n1, n2, n3 = self.col_factors
-        out["prefix_products"] = _copy_device_f32(p.prefix_products, P * n1 * n2 * self.rank,
-                                                  self.device).view(P, n1, n2, self.rank)
         out["rows"] = _copy_device_f32(p.rows, U * self.N, self.device).view(U, self.N)
         out.update(U=U, P=P, NG=NG)
         return out

@@ -10,11 +10,10 @@
 #include "ttemb_internal.cuh"
 
 namespace ttemb {
-cudaError_t configure_fwd(Ctx& c);
-cudaError_t configure_bwd(Ctx& c);
 int64_t radix_tiles(int64_t n);
 int64_t scan_tiles(int64_t n);
 int64_t agg_chunks(int64_t nnz);
+int64_t dc1_chunks(int64_t P);
 
 StageScope::StageScope(Ctx& c_, int st, cudaStream_t s_) : c(c_), stage(st), s(s_) {
   if (!c.timing) return;
@@ -68,13 +67,13 @@ int validate(const ttemb_config* cfg) {
   if (n1 < 1 || n2 < 1 || n3 < 1 || (int64_t)n1 * n2 * n3 != cfg->dim) return TTEMB_ERR_INVALID_ARG;
   if (cfg->rank < 1) return TTEMB_ERR_INVALID_ARG;
   if (cfg->rank > 128) return TTEMB_ERR_UNSUPPORTED;
-  if ((int64_t)n1 * n2 > 1024 || cfg->dim > 4096) return TTEMB_ERR_UNSUPPORTED;
+  if (n1 > 8 || n3 > 8 || cfg->dim > 4096) return TTEMB_ERR_UNSUPPORTED;
   if (cfg->index_bits != 64 && cfg->index_bits != 32) return TTEMB_ERR_INVALID_ARG;
   if (cfg->max_batch < 0 || cfg->max_nnz < 0) return TTEMB_ERR_INVALID_ARG;
   if (cfg->max_nnz > (int64_t(1) << 30)) return TTEMB_ERR_UNSUPPORTED;
   if ((int64_t)cfg->num_tables * cfg->max_batch > (int64_t(1) << 31)) return TTEMB_ERR_UNSUPPORTED;
   if (cfg->optimizer != TTEMB_SGD && cfg->optimizer != TTEMB_ADAGRAD) return TTEMB_ERR_INVALID_ARG;
-  if (cfg->flags & ~TTEMB_FUSED_UPDATE) return TTEMB_ERR_INVALID_ARG;
+  if (cfg->flags & ~(TTEMB_FUSED_UPDATE | TTEMB_FP32_CORES)) return TTEMB_ERR_INVALID_ARG;
   uint64_t total = 0, buckets = 0;
   for (int t = 0; t < cfg->num_tables; ++t) {
     const ttemb_table& tb = cfg->tables[t];
@@ -137,7 +136,6 @@ size_t carve(Ctx& c, uint8_t* base) {
   const int64_t U = std::max<int64_t>(c.U_cap, 1), P = std::max<int64_t>(c.P_cap, 1);
   const int64_t NG = std::max<int64_t>(c.NG_cap, 1);
   const int64_t bags = (int64_t)c.T * c.max_batch;
-  const size_t J12R = (size_t)c.n1 * c.n2 * c.R;
   PlanDev& p = c.p;
   c.d_meta = k.take<TableMeta>(c.T);
   c.d_rowbase = k.take<uint64_t>(c.T + 1);
@@ -151,6 +149,7 @@ size_t carve(Ctx& c, uint8_t* base) {
   p.rs1_counter = k.take<uint32_t>(4);
   p.rs2_counter = k.take<uint32_t>(4);
   p.sc_counter = k.take<uint32_t>(4);
+  p.work = k.take<uint32_t>(4);
   p.rs1_status = k.take<uint32_t>((size_t)c.key_passes * std::max<int64_t>(c.rs1_tiles, 1) * 256);
   p.rs2_status = k.take<uint32_t>((size_t)c.gkey_passes * std::max<int64_t>(c.rs2_tiles, 1) * 256);
   p.sc_status = k.take<uint32_t>((size_t)3 * c.sc_tiles);
@@ -171,12 +170,11 @@ size_t carve(Ctx& c, uint8_t* base) {
   p.grp_pfx = k.take<uint32_t>(P); p.grp_off = k.take<uint32_t>(NG + 1);
   p.grp_t = k.take<uint32_t>(NG); p.grp_i2 = k.take<uint32_t>(NG);
   // --- float intermediates ---
-  p.pbuf = k.take<float>((size_t)P * J12R);
-  p.dpbuf = k.take<float>((size_t)P * J12R);
   p.dabuf = k.take<float>((size_t)P * c.n1 * c.R);
   p.rows = k.take<float>((size_t)U * c.N);
   p.gbuf = k.take<float>((size_t)U * c.N);
-  p.aggpart = k.take<float>((size_t)2 * agg_chunks(nnz) * c.N);
+  p.aggpart = k.take<float>(std::max<size_t>((size_t)2 * agg_chunks(nnz) * c.N,
+                                              (size_t)2 * dc1_chunks(P) * c.n1 * c.R));
   // --- host staging (end-to-end API) ---
   c.st_idx = k.take<uint8_t>((size_t)nnz * (c.index_bits / 8));
   c.st_off = k.take<int64_t>(bags + 1);
@@ -275,8 +273,7 @@ int ttemb_create(const ttemb_config* cfg, int device, void* cores, void* state, 
   cudaError_t e = cudaMemcpy(c.d_meta, c.meta.data(), sizeof(TableMeta) * c.T, cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(c.d_rowbase, rb.data(), sizeof(uint64_t) * (c.T + 1), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(c.d_grpbase, gb.data(), sizeof(uint32_t) * (c.T + 1), cudaMemcpyHostToDevice);
-  if (e == cudaSuccess) e = configure_fwd(c);
-  if (e == cudaSuccess) e = configure_bwd(c);
+  if (e == cudaSuccess) e = configure_group(c);
   if (e != cudaSuccess) {
     fprintf(stderr, "ttemb_create: %s\n", cudaGetErrorString(e));
     delete h;
@@ -423,7 +420,7 @@ int ttemb_get_plan(ttemb_t h, ttemb_plan* plan) {
   plan->row_pfx = p.row_pfx; plan->row_i3 = p.row_i3; plan->pfx_t = p.pfx_t;
   plan->pfx_i1 = p.pfx_i1; plan->pfx_i2 = p.pfx_i2; plan->row_seg = p.row_seg;
   plan->grp_pfx = p.grp_pfx; plan->grp_off = p.grp_off; plan->grp_t = p.grp_t;
-  plan->grp_i2 = p.grp_i2; plan->prefix_products = p.pbuf; plan->rows = p.rows;
+  plan->grp_i2 = p.grp_i2; plan->rows = p.rows;
   return TTEMB_OK;
 }
 

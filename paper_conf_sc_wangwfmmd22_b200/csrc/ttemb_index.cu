@@ -36,9 +36,12 @@ __device__ __forceinline__ void st_release(uint32_t* p, uint32_t v) {
 }
 
 // Decoupled look-back: publish `agg` for tile `tile` in status[tile*stride], walk back
-// over predecessors, publish the inclusive prefix, return the exclusive prefix.
+// over predecessors in windows of 8 independent acquire loads (so a walk over many
+// not-yet-inclusive predecessors costs ~n/8 round trips), publish the inclusive prefix,
+// return the exclusive prefix.
 __device__ __forceinline__ uint32_t lookback(uint32_t* status, size_t stride, uint32_t tile,
                                              uint32_t agg) {
+  constexpr int W = 8;
   uint32_t* me = status + (size_t)tile * stride;
   if (tile == 0) {
     st_release(me, kFlagPfx | agg);
@@ -46,13 +49,22 @@ __device__ __forceinline__ uint32_t lookback(uint32_t* status, size_t stride, ui
   }
   st_release(me, kFlagAgg | agg);
   uint32_t excl = 0;
-  for (int64_t j = (int64_t)tile - 1; j >= 0; --j) {
-    uint32_t v;
-    do {
-      v = ld_acquire(status + (size_t)j * stride);
-    } while ((v >> 30) == 0);
-    excl += v & kValMask;
-    if (v & kFlagPfx) break;
+  int64_t j = (int64_t)tile - 1;
+  bool done = false;
+  while (!done) {
+    uint32_t v[W];
+#pragma unroll
+    for (int i = 0; i < W; ++i)
+      v[i] = (j - i >= 0) ? ld_acquire(status + (size_t)(j - i) * stride) : kFlagPfx;
+#pragma unroll
+    for (int i = 0; i < W; ++i) {
+      if (!done) {
+        while ((v[i] >> 30) == 0) v[i] = ld_acquire(status + (size_t)(j - i) * stride);
+        excl += v[i] & kValMask;
+        if (v[i] & kFlagPfx) done = true;
+      }
+    }
+    j -= W;
   }
   st_release(me, kFlagPfx | (excl + agg));
   return excl;

@@ -56,7 +56,8 @@ struct PlanDev {
   uint32_t *rs1_counter, *rs1_status;          // sort-1 look-back state [4][tiles][256]
   uint32_t *rs2_counter, *rs2_status;
   uint32_t *sc_counter, *sc_status;            // scans [3][tiles]
-  float *pbuf, *rows, *gbuf, *dpbuf, *dabuf, *aggpart;
+  uint32_t* work;                              // dynamic group schedulers [2]
+  float *rows, *gbuf, *dabuf, *aggpart;
 };
 
 struct Ctx {
@@ -121,7 +122,7 @@ cudaError_t run_index_stage(Ctx& c, const void* indices, const int64_t* offsets,
 cudaError_t run_forward_compute(Ctx& c, float* out, const int64_t* offsets, cudaStream_t s);
 cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s);
 cudaError_t run_update(Ctx& c, float lr, cudaStream_t s);
-cudaError_t configure_kernels(Ctx& c);
+cudaError_t configure_group(Ctx& c);
 
 // ---- small helpers -------------------------------------------------------------------
 static inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }

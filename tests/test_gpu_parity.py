@@ -56,13 +56,18 @@ def small_cases():
         ("dup-heavy", W.small_config([50], [(2, 5, 5)], (2, 2, 2), 4, 40, 7, 2.0), None),
         ("wide-R128", W.small_config([3000, 200], [(15, 15, 15), (6, 6, 6)], (4, 4, 8), 128, 24, 2, 1.05), None),
         ("odd-dims", W.small_config([777], [(9, 10, 9)], (3, 1, 5), 7, 50, 2, 1.1), "var"),
+        # R = 64 (tensor-core path): n1 = 2 / 4 / 8, n3 = 4 / 8, hot groups spanning m-tiles
+        ("tc-n1-2", W.small_config([20000, 300], [(28, 28, 26), (7, 7, 7)], (2, 2, 4), 64, 96, 3, 1.05), "var"),
+        ("tc-n1-8-n3-8", W.small_config([5000], [(18, 18, 16)], (8, 1, 8), 64, 64, 2, 1.2), None),
+        ("tc-multitile", W.small_config([400000], [(74, 74, 74)], (4, 4, 8), 64, 512, 4, 0.6), None),
+        ("tc-mixedmag", W.small_config([3000, 900], [(15, 15, 14), (10, 10, 9)], (4, 2, 4), 64, 80, 2, 1.05), "mixed"),
     ]
 
 
 def make_inputs(cfg, mode, seed=0, batch=None):
     B = cfg.batch if batch is None else batch
     lens = None
-    if mode == "var":
+    if mode == "var" or mode == "mixed":
         rng = np.random.default_rng(seed)
         lens = rng.integers(0, 6, size=cfg.num_tables * B)
         lens[0] = 0
@@ -75,7 +80,7 @@ def make_inputs(cfg, mode, seed=0, batch=None):
 @pytest.mark.parametrize("name,cfg,mode", small_cases(), ids=[c[0] for c in small_cases()])
 def test_forward_backward_small(name, cfg, mode):
     idx, off, B = make_inputs(cfg, mode, seed=3)
-    cores = W.make_cores(cfg, seed=3)
+    cores = W.make_cores(cfg, seed=3, mixed_magnitude=(mode == "mixed"))
     go = W.make_grad_out(cfg, B, seed=3)
     emb = gpu_emb(cfg, B, len(idx))
     emb.load_cores(cores)
@@ -117,14 +122,16 @@ def test_configs_full_batch(name):
             assert_companion(mine[k].cpu().numpy(), g[t][k], ga[t][k], 1e-4, f"dC{k+1} t{t}")
 
 
-def test_c4_reduced_batch():
-    """Criteo-TB shape (26 tables, R=64, N=64) at batch 2048: every output checked."""
+@pytest.mark.parametrize("fp32_cores", [False, True], ids=["tcgen05", "fp32-cores"])
+def test_c4_reduced_batch(fp32_cores):
+    """Criteo-TB shape (26 tables, R=64, N=64) at batch 2048: every output checked, on the
+    tensor-core (3xTF32) path and on the FP32 CUDA-core path."""
     cfg = W.config("c4")
     B = 2048
     idx, off = W.make_batch(cfg, seed=11, batch=B)
     cores = W.make_cores(cfg, seed=11)
     go = W.make_grad_out(cfg, B, seed=11)
-    emb = gpu_emb(cfg, B, len(idx))
+    emb = gpu_emb(cfg, B, len(idx), fp32_cores=fp32_cores)
     emb.load_cores(cores)
     out = run_forward(emb, idx, off, B)
     emb.backward(torch.as_tensor(go, device=DEV))
@@ -139,7 +146,7 @@ def test_c4_reduced_batch():
             assert_companion(mine[k].cpu().numpy(), g[t][k], ga[t][k], 1e-4, f"dC{k+1} t{t}")
 
 
-@pytest.mark.parametrize("name,rank", [("c4", None), ("c5", 128)])
+@pytest.mark.parametrize("name,rank", [("c4", None), ("c5", 64), ("c5", 128)])
 def test_full_size_sampled(name, rank):
     """Full BASELINE sizes in the bench launch configuration (fused update off so
     the gradients stay observable): plan bit-exact vs numpy, sampled bags vs the
