@@ -171,6 +171,9 @@ size_t carve(Ctx& c, uint8_t* base) {
   p.grp_t = k.take<uint32_t>(NG); p.grp_i2 = k.take<uint32_t>(NG);
   // --- float intermediates ---
   p.dabuf = k.take<float>((size_t)P * c.n1 * c.R);
+  const size_t pf = tc_eligible(c) ? (size_t)P * c.n1 * c.NC : 1;
+  p.pbuf = k.take<float>(pf);
+  p.dpbuf = k.take<float>(pf);
   p.rows = k.take<float>((size_t)U * c.N);
   p.gbuf = k.take<float>((size_t)U * c.N);
   p.aggpart = k.take<float>(std::max<size_t>((size_t)2 * agg_chunks(nnz) * c.N,
@@ -274,6 +277,7 @@ int ttemb_create(const ttemb_config* cfg, int device, void* cores, void* state, 
   if (e == cudaSuccess) e = cudaMemcpy(c.d_rowbase, rb.data(), sizeof(uint64_t) * (c.T + 1), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(c.d_grpbase, gb.data(), sizeof(uint32_t) * (c.T + 1), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = configure_group(c);
+  if (e == cudaSuccess) e = configure_tc(c);
   if (e != cudaSuccess) {
     fprintf(stderr, "ttemb_create: %s\n", cudaGetErrorString(e));
     delete h;

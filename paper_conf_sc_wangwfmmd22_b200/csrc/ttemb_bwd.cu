@@ -221,7 +221,7 @@ cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s
   a.n1 = c.n1; a.N = c.N; a.R = c.R;
   a.lr = lr; a.eps = c.eps; a.opt = c.opt; a.fused = fused ? 1 : 0;
   if (c.nnz > 0) {
-    cudaError_t e = run_group_bwd(c, lr, s);
+    cudaError_t e = tc_eligible(c) ? run_tc_bwd(c, lr, s) : run_group_bwd(c, lr, s);
     if (e != cudaSuccess) return e;
     {
       StageScope sc(c, ST_DC1, s);

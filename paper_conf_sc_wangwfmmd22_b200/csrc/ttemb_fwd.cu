@@ -20,7 +20,9 @@ namespace {
 template <int VW>
 __global__ void __launch_bounds__(256)
 k_pool(const float* __restrict__ rows, const uint32_t* __restrict__ inverse,
-       const int64_t* __restrict__ offsets, int64_t nnz, int T, int B, int N, float* __restrict__ out) {
+       const int64_t* __restrict__ offsets, int64_t nnz, int T, int B, int N, float* __restrict__ out,
+       const uint32_t* __restrict__ counts, int skip_single) {
+  if (skip_single && counts[kCntMulti] == 0) return;   // one id per bag: written directly
   const int NV = N / VW;
   const int64_t total = (int64_t)T * B * NV;
   for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < total;
@@ -54,8 +56,9 @@ cudaError_t run_group_fwd(Ctx& c, cudaStream_t s);
 
 cudaError_t run_forward_compute(Ctx& c, float* out, const int64_t* offsets, cudaStream_t s) {
   const PlanDev& p = c.p;
+  const bool tc = tc_eligible(c);
   if (c.nnz > 0) {
-    cudaError_t e = run_group_fwd(c, s);
+    cudaError_t e = tc ? run_tc_fwd(c, out, s) : run_group_fwd(c, s);
     if (e != cudaSuccess) return e;
   }
   {
@@ -64,10 +67,10 @@ cudaError_t run_forward_compute(Ctx& c, float* out, const int64_t* offsets, cuda
     if (total > 0) {
       if (c.N % 4 == 0)
         k_pool<4><<<grid_for(c, total / 4, 256, 8), 256, 0, s>>>(p.rows, p.inverse, offsets, c.nnz,
-                                                                 c.T, c.B, c.N, out);
+                                                                 c.T, c.B, c.N, out, p.counts, 0);
       else
         k_pool<1><<<grid_for(c, total, 256, 8), 256, 0, s>>>(p.rows, p.inverse, offsets, c.nnz, c.T,
-                                                             c.B, c.N, out);
+                                                             c.B, c.N, out, p.counts, 0);
     }
   }
   return cudaGetLastError();

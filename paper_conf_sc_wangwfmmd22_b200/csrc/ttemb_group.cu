@@ -21,7 +21,6 @@
 #include <algorithm>
 
 #include "ttemb_internal.cuh"
-#include "tc.cuh"
 
 namespace ttemb {
 
@@ -577,558 +576,6 @@ __global__ void __launch_bounds__(256) k_group_bwd(GroupArgs a) {
   }
 }
 
-// ====================================================================================
-// Tensor-core path (R == 64): the three rank-R contractions on tcgen05 (kind::tf32,
-// 3xTF32 split, fp32 accumulate in TMEM), operands staged as K-major CM matrices
-// (tc.cuh).  Tile: 64 rows (q, j1) x one j2 block (64 columns of C2) x K = 64.
-//   GEMM1  P   [m][c]  = A1 (m x r1) . X1^T       A1 = CM(m, r1), X1 = CM(c, r1)
-//   GEMM3  dA^T[r1][m] = X2 (r1 x c) . D1^T       X2 = CM(r1, c), D1 = CM(m, c)
-//   GEMM2  dC2 [r1][c] += A2 (r1 x m) . D2^T      A2 = CM(r1, m), D2 = CM(c, m)
-// Loop order per group: m-tile (outer) x j2 chunk (inner); dA accumulates over chunks
-// and dC2[chunk] over m-tiles in TMEM.  The next chunk's C2 values are prefetched into
-// registers while the current chunk computes (the next group is claimed one ahead).
-// Accumulators (M = 64): row i lives in TMEM lane (i % 16) + 32 (i / 16).
-// ====================================================================================
-constexpr int TR = 64, TMT = 64, TCW = 64, TNRB = 8, TNT = 256, TRSL = 8;
-constexpr uint32_t TCM = 64 * 64 * 4;           // bytes of one 64x64 fp32 CM matrix
-constexpr int TCWP = TCW + 4;                   // fp32 P tile row stride
-
-struct TcSmem {
-  float *x1h, *x1l, *x2h, *x2l, *a1h, *a1l, *a2h, *a2l, *d1h, *d1l, *d2h, *d2l;
-  float* sP;
-  uint32_t *rs, *rc, *sl, *pf, *misc;
-  uint64_t* mbar;
-};
-
-__host__ __device__ inline size_t tc_smem_bytes(bool bwd) {
-  const size_t mats = bwd ? 12 : 4;
-  return mats * TCM + (size_t)TMT * TCWP * 4 + 5 * 80 * 4 + 64;
-}
-
-__device__ __forceinline__ TcSmem tc_carve(float* base, bool bwd) {
-  TcSmem t;
-  char* p = reinterpret_cast<char*>(base);
-  auto take = [&](size_t bytes) { char* q = p; p += bytes; return reinterpret_cast<float*>(q); };
-  t.x1h = take(TCM); t.x1l = take(TCM);
-  t.a1h = take(TCM); t.a1l = take(TCM);
-  if (bwd) {
-    t.x2h = take(TCM); t.x2l = take(TCM); t.a2h = take(TCM); t.a2l = take(TCM);
-    t.d1h = take(TCM); t.d1l = take(TCM); t.d2h = take(TCM); t.d2l = take(TCM);
-  } else {
-    t.x2h = t.x2l = t.a2h = t.a2l = t.d1h = t.d1l = t.d2h = t.d2l = nullptr;
-  }
-  t.sP = take((size_t)TMT * TCWP * 4);
-  t.rs = reinterpret_cast<uint32_t*>(take(80 * 4));
-  t.rc = reinterpret_cast<uint32_t*>(take(80 * 4));
-  t.sl = reinterpret_cast<uint32_t*>(take(80 * 4));
-  t.pf = reinterpret_cast<uint32_t*>(take(80 * 4));
-  t.misc = reinterpret_cast<uint32_t*>(take(80 * 4));
-  t.mbar = reinterpret_cast<uint64_t*>(take(64));
-  return t;
-}
-
-__device__ __forceinline__ void st_split4(float* hi, float* lo, uint32_t off, float4 v) {
-  float4 h = make_float4(tc::tf32_hi(v.x), tc::tf32_hi(v.y), tc::tf32_hi(v.z), tc::tf32_hi(v.w));
-  float4 l = make_float4(v.x - h.x, v.y - h.y, v.z - h.z, v.w - h.w);
-  *reinterpret_cast<float4*>(reinterpret_cast<char*>(hi) + off) = h;
-  *reinterpret_cast<float4*>(reinterpret_cast<char*>(lo) + off) = l;
-}
-__device__ __forceinline__ void st_split1(float* hi, float* lo, uint32_t off, float v) {
-  const float h = tc::tf32_hi(v);
-  *reinterpret_cast<float*>(reinterpret_cast<char*>(hi) + off) = h;
-  *reinterpret_cast<float*>(reinterpret_cast<char*>(lo) + off) = v - h;
-}
-__device__ __forceinline__ float* fat(float* base, uint32_t off) {
-  return reinterpret_cast<float*>(reinterpret_cast<char*>(base) + off);
-}
-
-// Register prefetch of one C2 chunk [r1][c0 .. c0+64): X1 pattern (4 r1 of one c) and
-// X2 pattern (4 c of one r1); all loads are issued before any is consumed.
-struct C2Pref {
-  float4 x1[4];
-  float4 x2[4];
-};
-
-__device__ __forceinline__ void c2_prefetch(C2Pref& pf, const float* C2s, int NC, int c0, bool want_x2) {
-#pragma unroll
-  for (int k = 0; k < 4; ++k) {
-    const int e = threadIdx.x + TNT * k;
-    const int c = e & 63, rq = e >> 6;
-    const float* p = C2s + (size_t)(4 * rq) * NC + c0 + c;
-    pf.x1[k].x = __ldg(p);
-    pf.x1[k].y = __ldg(p + NC);
-    pf.x1[k].z = __ldg(p + 2 * NC);
-    pf.x1[k].w = __ldg(p + 3 * NC);
-  }
-  if (want_x2) {
-#pragma unroll
-    for (int k = 0; k < 4; ++k) {
-      const int e = threadIdx.x + TNT * k;
-      const int r = e & 63, cq = e >> 6;
-      pf.x2[k] = __ldg(reinterpret_cast<const float4*>(C2s + (size_t)r * NC + c0 + 4 * cq));
-    }
-  }
-}
-
-__device__ __forceinline__ void c2_store(const TcSmem& t, const C2Pref& pf, bool want_x2) {
-#pragma unroll
-  for (int k = 0; k < 4; ++k) {
-    const int e = threadIdx.x + TNT * k;
-    st_split4(t.x1h, t.x1l, tc::cm_off(e & 63, 4 * (e >> 6), TNRB), pf.x1[k]);
-  }
-  if (want_x2) {
-#pragma unroll
-    for (int k = 0; k < 4; ++k) {
-      const int e = threadIdx.x + TNT * k;
-      st_split4(t.x2h, t.x2l, tc::cm_off(e & 63, 4 * (e >> 6), TNRB), pf.x2[k]);
-    }
-  }
-}
-
-// Prefix / row / dP-slice lists of the m-tile and A1 = CM(m, r1) (+ A2 = CM(r1, m)).
-// Rows >= npq*n1 are zero.  Ends with a barrier after the lists; A stores follow.
-__device__ __forceinline__ void tc_stage_tile(const GroupArgs& a, const TcSmem& t,
-                                              const float* C1t, uint32_t qa, int npq, bool bwd) {
-  const int tid = threadIdx.x;
-  if (tid < npq) {
-    const uint32_t p = a.grp_pfx[qa + tid];
-    t.pf[tid] = p;
-    t.misc[8 + tid] = a.pfx_i1[p];
-    const uint32_t r0 = a.row_seg[p], r1 = a.row_seg[p + 1];
-    t.rs[tid] = r0;
-    t.rc[tid] = r1 - r0;
-  }
-  __syncthreads();
-  if (tid < 32) {   // exclusive scans of row counts and dP slice counts (npq <= 64)
-    const uint32_t v0 = tid < npq ? t.rc[tid] : 0, v1 = tid + 32 < npq ? t.rc[tid + 32] : 0;
-    const uint32_t w0 = (v0 + TRSL - 1) / TRSL, w1 = (v1 + TRSL - 1) / TRSL;
-    uint32_t x0 = v0, x1 = v1, y0 = w0, y1 = w1;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const uint32_t a0 = __shfl_up_sync(0xffffffffu, x0, o), a1 = __shfl_up_sync(0xffffffffu, x1, o);
-      const uint32_t b0 = __shfl_up_sync(0xffffffffu, y0, o), b1 = __shfl_up_sync(0xffffffffu, y1, o);
-      if (tid >= o) { x0 += a0; x1 += a1; y0 += b0; y1 += b1; }
-    }
-    const uint32_t tx = __shfl_sync(0xffffffffu, x0, 31), ty = __shfl_sync(0xffffffffu, y0, 31);
-    if (tid < npq) { t.rc[tid] = x0 - v0; t.sl[tid] = y0 - w0; }
-    if (tid + 32 < npq) { t.rc[tid + 32] = tx + x1 - v1; t.sl[tid + 32] = ty + y1 - w1; }
-    if (tid == 31) { t.rc[npq] = tx + x1; t.sl[npq] = ty + y1; }
-  }
-  const int rows = npq * a.n1;
-  float4 va[4];
-#pragma unroll
-  for (int k = 0; k < 4; ++k) {                                     // A1: 4 r1 of one m
-    const int e = tid + TNT * k;
-    const int m = e & 63, kq = e >> 6;
-    va[k] = make_float4(0.f, 0.f, 0.f, 0.f);
-    if (m < rows) {
-      const uint32_t i1 = a.pfx_i1[a.grp_pfx[qa + m / a.n1]];
-      va[k] = __ldg(reinterpret_cast<const float4*>(C1t + ((size_t)i1 * a.n1 + (m % a.n1)) * TR + 4 * kq));
-    }
-  }
-  float vb[4][4];
-  if (bwd) {
-#pragma unroll
-    for (int k = 0; k < 4; ++k) {                                   // A2: 4 m of one r1
-      const int e = tid + TNT * k;
-      const int r = e & 63, mq = e >> 6;
-#pragma unroll
-      for (int i = 0; i < 4; ++i) {
-        const int m = 4 * mq + i;
-        vb[k][i] = 0.f;
-        if (m < rows) {
-          const uint32_t i1 = a.pfx_i1[a.grp_pfx[qa + m / a.n1]];
-          vb[k][i] = __ldg(C1t + ((size_t)i1 * a.n1 + (m % a.n1)) * TR + r);
-        }
-      }
-    }
-  }
-#pragma unroll
-  for (int k = 0; k < 4; ++k) {
-    const int e = tid + TNT * k;
-    st_split4(t.a1h, t.a1l, tc::cm_off(e & 63, 4 * (e >> 6), TNRB), va[k]);
-    if (bwd)
-      st_split4(t.a2h, t.a2l, tc::cm_off(e & 63, 4 * (e >> 6), TNRB),
-                make_float4(vb[k][0], vb[k][1], vb[k][2], vb[k][3]));
-  }
-}
-
-// 3xTF32 64x64 (K = 64) product of two K-major CM matrices into TMEM column base d.
-__device__ __forceinline__ void tc_mma3(uint32_t d, const float* ah, const float* al,
-                                        const float* bh, const float* bl, bool accumulate) {
-  const uint32_t id = tc::idesc_tf32(64, 64, false, false);
-  const uint32_t sah = tc::smem_u32(ah), sal = tc::smem_u32(al);
-  const uint32_t sbh = tc::smem_u32(bh), sbl = tc::smem_u32(bl);
-#pragma unroll
-  for (int kk = 0; kk < 8; ++kk) {
-    const uint32_t o = kk * 2 * TNRB * 128;
-    const uint64_t dah = tc::sdesc(sah + o, TNRB * 128, 128), dal = tc::sdesc(sal + o, TNRB * 128, 128);
-    const uint64_t dbh = tc::sdesc(sbh + o, TNRB * 128, 128), dbl = tc::sdesc(sbl + o, TNRB * 128, 128);
-    tc::mma_tf32(d, dah, dbh, id, (accumulate || kk > 0) ? 1u : 0u);
-    tc::mma_tf32(d, dah, dbl, id, 1u);
-    tc::mma_tf32(d, dal, dbh, id, 1u);
-  }
-}
-
-__device__ __forceinline__ void tc_wait(const TcSmem& t, uint32_t& phase) {
-  tc::mbar_wait(t.mbar, phase);
-  phase ^= 1u;
-  tc::fence_after();
-}
-
-// Barrier that publishes generic-proxy smem writes to the tensor core.
-__device__ __forceinline__ void tc_publish() {
-  tc::fence_async_smem();
-  tc::fence_before();
-  __syncthreads();
-  tc::fence_after();
-}
-
-// TMEM accumulator (M = 64 rows x 64 cols at column base) -> fp32 rows of sP.
-__device__ __forceinline__ void tc_tmem_to_sP(const TcSmem& t, uint32_t tbase) {
-  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int q = w & 3, half = w >> 2;
-  float v[32];
-  tc::tmem_ld32(tc::taddr(tbase, 32 * q, 32 * half), v);
-  if (lane < 16) {
-    float* dst = t.sP + (16 * q + lane) * TCWP + 32 * half;
-#pragma unroll
-    for (int j = 0; j < 32; j += 4) *reinterpret_cast<float4*>(dst + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
-  }
-}
-
-// Forward row stage on the P tile: E_u[j1][j2][:] for every row u of the tile (R = 64).
-template <int MN1, int MN3>
-__device__ __forceinline__ void tc_fwd_rows(const GroupArgs& a, const TcSmem& t, const float* C3t,
-                                            int npq, int j2) {
-  const uint32_t nr = t.rc[npq];
-  const int n1 = a.n1, n3 = a.n3;
-  for (uint32_t ri = threadIdx.x; ri < nr; ri += TNT) {
-    const int ql = find_prefix(t.rc, npq, ri);
-    const uint32_t u = t.rs[ql] + (ri - t.rc[ql]);
-    const float* c3 = C3t + (size_t)a.row_i3[u] * TR * n3;
-    float acc[MN1][MN3];
-#pragma unroll
-    for (int i = 0; i < MN1; ++i)
-#pragma unroll
-      for (int j = 0; j < MN3; ++j) acc[i][j] = 0.f;
-    const float* pr = t.sP + (size_t)(ql * n1) * TCWP;
-#pragma unroll 4
-    for (int r = 0; r < TR; r += 4) {
-      float cv[4][MN3];
-#pragma unroll
-      for (int i = 0; i < 4; ++i)
-#pragma unroll
-        for (int j = 0; j < MN3; j += 4) {
-          const float4 t4 = __ldg(reinterpret_cast<const float4*>(c3 + (r + i) * n3 + j));
-          cv[i][j] = t4.x; cv[i][j + 1] = t4.y; cv[i][j + 2] = t4.z; cv[i][j + 3] = t4.w;
-        }
-#pragma unroll
-      for (int j1 = 0; j1 < MN1; ++j1) {
-        if (j1 < n1) {
-          const float4 p4 = *reinterpret_cast<const float4*>(pr + j1 * TCWP + r);
-          const float pv[4] = {p4.x, p4.y, p4.z, p4.w};
-#pragma unroll
-          for (int i = 0; i < 4; ++i)
-#pragma unroll
-            for (int j = 0; j < MN3; ++j) acc[j1][j] = fmaf(pv[i], cv[i][j], acc[j1][j]);
-        }
-      }
-    }
-    float* dst = a.rows + (size_t)u * a.N;
-#pragma unroll
-    for (int j1 = 0; j1 < MN1; ++j1) {
-      if (j1 >= n1) continue;
-      float* d = dst + (j1 * a.n2 + j2) * n3;
-#pragma unroll
-      for (int j = 0; j < MN3; j += 4)
-        *reinterpret_cast<float4*>(d + j) = make_float4(acc[j1][j], acc[j1][j + 1], acc[j1][j + 2], acc[j1][j + 3]);
-    }
-  }
-}
-
-template <int MN1, int MN3>
-__global__ void __launch_bounds__(TNT, 2) k_tc_fwd(GroupArgs a) {
-  extern __shared__ __align__(128) float smem[];
-  const TcSmem t = tc_carve(smem, false);
-  __shared__ uint32_t s_tmem;
-  const int tid = threadIdx.x;
-  if (tid == 0) {
-    tc::mbar_init(t.mbar, 1);
-    tc::fence_mbar_init();
-    t.misc[0] = atomicAdd(a.work, 1u);
-    t.misc[1] = atomicAdd(a.work, 1u);
-  }
-  if (tid < 32) tc::tmem_alloc(&s_tmem, 64);
-  tc::fence_before();
-  __syncthreads();
-  tc::fence_after();
-  const uint32_t tP = s_tmem;
-  uint32_t phase = 0;
-  const uint32_t NG = a.counts[kCntNG];
-  const int PPT = TMT / a.n1, NCH = a.NC / TCW;
-  uint32_t g = t.misc[0], gnext = t.misc[1];
-  C2Pref pf;
-  auto c2_of = [&](uint32_t gg) {
-    return a.cores + a.meta[a.grp_t[gg]].c2_off + (size_t)a.grp_i2[gg] * TR * a.NC;
-  };
-  if (g < NG) c2_prefetch(pf, c2_of(g), a.NC, 0, false);
-  while (g < NG) {
-    const uint32_t tt = a.grp_t[g];
-    const uint32_t q0 = a.grp_off[g], q1 = a.grp_off[g + 1];
-    const TableMeta tm = a.meta[tt];
-    const float* C2s = c2_of(g);
-    const float* C1t = a.cores + tm.c1_off;
-    const float* C3t = a.cores + tm.c3_off;
-    const uint32_t nmt = (q1 - q0 + PPT - 1) / PPT;
-    for (uint32_t mt = 0; mt < nmt; ++mt) {
-      const uint32_t qa = q0 + mt * PPT;
-      const int npq = (int)min((uint32_t)PPT, q1 - qa);
-      __syncthreads();
-      tc_stage_tile(a, t, C1t, qa, npq, false);
-      for (int k = 0; k < NCH; ++k) {
-        if (k > 0) __syncthreads();
-        c2_store(t, pf, false);
-        if (k + 1 < NCH) c2_prefetch(pf, C2s, a.NC, (k + 1) * TCW, false);
-        else if (mt + 1 < nmt) c2_prefetch(pf, C2s, a.NC, 0, false);
-        else if (gnext < NG) c2_prefetch(pf, c2_of(gnext), a.NC, 0, false);
-        tc_publish();
-        if (tid == 0) {
-          tc_mma3(tP, t.a1h, t.a1l, t.x1h, t.x1l, false);
-          tc::commit(t.mbar);
-        }
-        __syncwarp();
-        tc_wait(t, phase);
-        tc_tmem_to_sP(t, tP);
-        tc::fence_before();
-        __syncthreads();
-        tc_fwd_rows<MN1, MN3>(a, t, C3t, npq, k);
-      }
-    }
-    __syncthreads();
-    if (tid == 0) t.misc[1] = atomicAdd(a.work, 1u);
-    __syncthreads();
-    g = gnext;
-    gnext = t.misc[1];
-  }
-  tc::fence_before();
-  __syncthreads();
-  tc::fence_after();
-  if (tid < 32) tc::tmem_dealloc(tP, 64);
-}
-
-// dP of the tile (this chunk's j2), accumulated in fp32 into D1h (CM(m, c) positions) with
-// shared atomics.  Item = (slice of <= TRSL rows of one prefix, r-block of 4) so hot
-// prefixes with hundreds of rows are spread over many threads.
-template <int MN1, int MN3>
-__device__ __forceinline__ void tc_bwd_dp(const GroupArgs& a, const TcSmem& t, const float* C3t,
-                                          int npq, int j2) {
-  const int n1 = a.n1, n3 = a.n3;
-  const uint32_t nsl = t.sl[npq];
-  for (uint32_t it = threadIdx.x; it < nsl * 16; it += TNT) {
-    const uint32_t sli = it >> 4;
-    const int r0 = (int)(it & 15) * 4;
-    const int ql = find_prefix(t.sl, npq, sli);
-    const uint32_t cnt = t.rc[ql + 1] - t.rc[ql];
-    const uint32_t k0 = (sli - t.sl[ql]) * TRSL, k1 = min(k0 + TRSL, cnt);
-    float acc[MN1][4];
-#pragma unroll
-    for (int i = 0; i < MN1; ++i)
-#pragma unroll
-      for (int j = 0; j < 4; ++j) acc[i][j] = 0.f;
-    for (uint32_t k = k0; k < k1; ++k) {
-      const uint32_t u = t.rs[ql] + k;
-      const float* c3 = C3t + (size_t)a.row_i3[u] * TR * n3 + (size_t)r0 * n3;
-      const float* gu = a.gbuf + (size_t)u * a.N + j2 * n3;
-      float cv[4][MN3];
-#pragma unroll
-      for (int i = 0; i < 4; ++i)
-#pragma unroll
-        for (int j = 0; j < MN3; j += 4) {
-          const float4 t4 = __ldg(reinterpret_cast<const float4*>(c3 + i * n3 + j));
-          cv[i][j] = t4.x; cv[i][j + 1] = t4.y; cv[i][j + 2] = t4.z; cv[i][j + 3] = t4.w;
-        }
-#pragma unroll
-      for (int j1 = 0; j1 < MN1; ++j1) {
-        if (j1 >= n1) continue;
-        float gv[MN3];
-#pragma unroll
-        for (int j = 0; j < MN3; j += 4) {
-          const float4 t4 = __ldg(reinterpret_cast<const float4*>(gu + j1 * a.n2 * n3 + j));
-          gv[j] = t4.x; gv[j + 1] = t4.y; gv[j + 2] = t4.z; gv[j + 3] = t4.w;
-        }
-#pragma unroll
-        for (int i = 0; i < 4; ++i)
-#pragma unroll
-          for (int j = 0; j < MN3; ++j) acc[j1][i] = fmaf(gv[j], cv[i][j], acc[j1][i]);
-      }
-    }
-#pragma unroll
-    for (int j1 = 0; j1 < MN1; ++j1) {
-      if (j1 >= n1) continue;
-      const int m = ql * n1 + j1;
-#pragma unroll
-      for (int i = 0; i < 4; ++i) atomicAdd(fat(t.d1h, tc::cm_off(m, r0 + i, TNRB)), acc[j1][i]);
-    }
-  }
-}
-
-// fp32 dP in D1h -> D1 (hi/lo, CM(m, c)) and D2 (hi/lo, CM(c, m)).
-__device__ __forceinline__ void tc_split_dp(const TcSmem& t) {
-#pragma unroll
-  for (int k = 0; k < 4; ++k) {
-    const int f = threadIdx.x + TNT * k;
-    const int m = f & 63, cq = f >> 6;
-    const uint32_t off = tc::cm_off(m, 4 * cq, TNRB);
-    const float4 v = *reinterpret_cast<const float4*>(fat(t.d1h, off));
-    st_split4(t.d1h, t.d1l, off, v);
-    st_split1(t.d2h, t.d2l, tc::cm_off(4 * cq + 0, m, TNRB), v.x);
-    st_split1(t.d2h, t.d2l, tc::cm_off(4 * cq + 1, m, TNRB), v.y);
-    st_split1(t.d2h, t.d2l, tc::cm_off(4 * cq + 2, m, TNRB), v.z);
-    st_split1(t.d2h, t.d2l, tc::cm_off(4 * cq + 3, m, TNRB), v.w);
-  }
-}
-
-template <int MN1, int MN3>
-__global__ void __launch_bounds__(TNT, 1) k_tc_bwd(GroupArgs a) {
-  extern __shared__ __align__(128) float smem[];
-  const TcSmem t = tc_carve(smem, true);
-  __shared__ uint32_t s_tmem;
-  const int tid = threadIdx.x;
-  const int w = tid >> 5, lane = tid & 31, q4 = w & 3, half = w >> 2;
-  if (tid == 0) {
-    tc::mbar_init(t.mbar, 1);
-    tc::fence_mbar_init();
-    t.misc[0] = atomicAdd(a.work, 1u);
-    t.misc[1] = atomicAdd(a.work, 1u);
-  }
-  if (tid < 32) tc::tmem_alloc(&s_tmem, 512);
-  tc::fence_before();
-  __syncthreads();
-  tc::fence_after();
-  const uint32_t tP = s_tmem, tDA = s_tmem + 64, tDC2 = s_tmem + 128;
-  uint32_t phase = 0;
-  const uint32_t NG = a.counts[kCntNG];
-  const int PPT = TMT / a.n1, NCH = a.NC / TCW;
-  Smem s{};
-  s.sP = t.sP; s.rs = t.rs; s.rc = t.rc; s.pf = t.pf;
-  GroupArgs b = a;
-  b.CWp = TCWP;
-  uint32_t g = t.misc[0], gnext = t.misc[1];
-  C2Pref pf;
-  auto c2_of = [&](uint32_t gg) {
-    return a.cores + a.meta[a.grp_t[gg]].c2_off + (size_t)a.grp_i2[gg] * TR * a.NC;
-  };
-  if (g < NG) c2_prefetch(pf, c2_of(g), a.NC, 0, true);
-  while (g < NG) {
-    const uint32_t tt = a.grp_t[g], i2 = a.grp_i2[g];
-    const uint32_t q0 = a.grp_off[g], q1 = a.grp_off[g + 1];
-    const TableMeta tm = a.meta[tt];
-    const size_t c2o = tm.c2_off + (size_t)i2 * TR * a.NC;
-    const float* C2s = a.cores + c2o;
-    const float* C1t = a.cores + tm.c1_off;
-    const float* C3t = a.cores + tm.c3_off;
-    const uint32_t nmt = (q1 - q0 + PPT - 1) / PPT;
-    for (uint32_t mt = 0; mt < nmt; ++mt) {
-      const uint32_t qa = q0 + mt * PPT;
-      const int npq = (int)min((uint32_t)PPT, q1 - qa);
-      const int rows = npq * a.n1;
-      __syncthreads();
-      tc_stage_tile(a, t, C1t, qa, npq, true);
-      for (int k = 0; k < NCH; ++k) {
-        if (k > 0) __syncthreads();
-        c2_store(t, pf, true);
-        if (k + 1 < NCH) c2_prefetch(pf, C2s, a.NC, (k + 1) * TCW, true);
-        else if (mt + 1 < nmt) c2_prefetch(pf, C2s, a.NC, 0, true);
-        else if (gnext < NG) c2_prefetch(pf, c2_of(gnext), a.NC, 0, true);
-#pragma unroll
-        for (int z = 0; z < 4; ++z)   // fp32 dP accumulator (D1h) <- 0
-          *reinterpret_cast<float4*>(t.d1h + 4 * (tid + TNT * z)) = make_float4(0.f, 0.f, 0.f, 0.f);
-        tc_publish();
-        if (tid == 0) {                                      // GEMM1: P recompute
-          tc_mma3(tP, t.a1h, t.a1l, t.x1h, t.x1l, false);
-          tc::commit(t.mbar);
-        }
-        __syncwarp();
-        tc_wait(t, phase);
-        tc_tmem_to_sP(t, tP);
-        tc::fence_before();
-        __syncthreads();
-        tc_bwd_dp<MN1, MN3>(a, t, C3t, npq, k);               // dP -> D1h (fp32)
-        bwd_dc3<MN1, MN3, true>(b, s, tm.c3_off, npq, k, 1);   // dC3 += P^T G (atomics)
-        __syncthreads();
-        tc_split_dp(t);
-        tc_publish();
-        if (tid == 0) {
-          tc_mma3(tDA, t.x2h, t.x2l, t.d1h, t.d1l, k > 0);                 // GEMM3: dA^T
-          tc_mma3(tDC2 + 64 * k, t.a2h, t.a2l, t.d2h, t.d2l, mt > 0);       // GEMM2: dC2 += A^T dP
-          tc::commit(t.mbar);
-        }
-        __syncwarp();
-        tc_wait(t, phase);
-      }
-      {   // dA^T [r1][m] -> dabuf[(p, j1)][r1]
-        float v[32];
-        tc::tmem_ld32(tc::taddr(tDA, 32 * q4, 32 * half), v);
-        if (lane < 16) {
-          const int r1 = 16 * q4 + lane;
-#pragma unroll
-          for (int j = 0; j < 32; ++j) {
-            const int m = 32 * half + j;
-            if (m < rows) a.dabuf[((size_t)t.pf[m / a.n1] * a.n1 + (m % a.n1)) * TR + r1] = v[j];
-          }
-        }
-        tc::fence_before();
-      }
-    }
-    // dC2: this CTA owns C2[t][i2]; gradient or fused update, chunk by chunk
-    for (int k = 0; k < NCH; ++k) {
-      float v[32];
-      tc::tmem_ld32(tc::taddr(tDC2 + 64 * k, 32 * q4, 32 * half), v);
-      if (lane < 16) {
-        const int r1 = 16 * q4 + lane;
-        const size_t base = c2o + (size_t)r1 * a.NC + k * TCW + 32 * half;
-        if (a.fused) {
-          float x[32];
-#pragma unroll
-          for (int j = 0; j < 32; j += 4) {
-            const float4 x4 = *reinterpret_cast<const float4*>(a.cores + base + j);
-            x[j] = x4.x; x[j + 1] = x4.y; x[j + 2] = x4.z; x[j + 3] = x4.w;
-          }
-          if (a.opt == TTEMB_SGD) {
-#pragma unroll
-            for (int j = 0; j < 32; j += 4)
-              *reinterpret_cast<float4*>(a.cores + base + j) =
-                  make_float4(x[j] - a.lr * v[j], x[j + 1] - a.lr * v[j + 1], x[j + 2] - a.lr * v[j + 2],
-                              x[j + 3] - a.lr * v[j + 3]);
-          } else {
-#pragma unroll
-            for (int j = 0; j < 32; ++j) {
-              const float sv = a.state[base + j] + v[j] * v[j];
-              a.state[base + j] = sv;
-              a.cores[base + j] = x[j] - a.lr * v[j] / (sqrtf(sv) + a.eps);
-            }
-          }
-        } else {
-#pragma unroll
-          for (int j = 0; j < 32; j += 4)
-            *reinterpret_cast<float4*>(a.grads + base + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
-        }
-      }
-    }
-    tc::fence_before();
-    __syncthreads();
-    if (tid == 0) t.misc[1] = atomicAdd(a.work, 1u);
-    __syncthreads();
-    g = gnext;
-    gnext = t.misc[1];
-  }
-  tc::fence_before();
-  __syncthreads();
-  tc::fence_after();
-  if (tid < 32) tc::tmem_dealloc(tP, 512);
-}
-
 template <int MN1, int MN3, bool VEC>
 cudaError_t set_attrs(size_t fwd_bytes, size_t bwd_bytes) {
   cudaError_t e = cudaFuncSetAttribute(k_group_fwd<MN1, MN3, VEC>,
@@ -1202,47 +649,10 @@ size_t group_smem_bytes(const Ctx& c, bool bwd) {
   return sizeof(float) * smem_floats(c.R, sh.CW, sh.MT, sh.PPT, bwd);
 }
 
-bool use_tc(const Ctx& c) {
-  return !(c.flags & TTEMB_FP32_CORES) && c.R == TR && (c.n3 % 4 == 0) && c.n3 <= 8 &&
-         (c.n1 == 1 || c.n1 == 2 || c.n1 == 4 || c.n1 == 8) && c.n2 <= 6;
-}
-
-template <int MN1, int MN3>
-cudaError_t tc_attrs() {
-  cudaError_t e = cudaFuncSetAttribute(k_tc_fwd<MN1, MN3>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)tc_smem_bytes(false));
-  if (e != cudaSuccess) return e;
-  return cudaFuncSetAttribute(k_tc_bwd<MN1, MN3>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                              (int)tc_smem_bytes(true));
-}
-
-template <int MN1, int MN3>
-void tc_launch(bool bwd, int grid, const GroupArgs& a, cudaStream_t s) {
-  if (bwd) k_tc_bwd<MN1, MN3><<<grid, 256, tc_smem_bytes(true), s>>>(a);
-  else k_tc_fwd<MN1, MN3><<<grid, 256, tc_smem_bytes(false), s>>>(a);
-}
-
-cudaError_t tc_dispatch_attrs(int mn1, int mn3) {
-  if (mn1 <= 2) return mn3 == 4 ? tc_attrs<2, 4>() : tc_attrs<2, 8>();
-  if (mn1 == 4) return mn3 == 4 ? tc_attrs<4, 4>() : tc_attrs<4, 8>();
-  return mn3 == 4 ? tc_attrs<8, 4>() : tc_attrs<8, 8>();
-}
-
-void tc_dispatch_launch(int mn1, int mn3, bool bwd, int grid, const GroupArgs& a, cudaStream_t s) {
-  if (mn1 <= 2) return mn3 == 4 ? tc_launch<2, 4>(bwd, grid, a, s) : tc_launch<2, 8>(bwd, grid, a, s);
-  if (mn1 == 4) return mn3 == 4 ? tc_launch<4, 4>(bwd, grid, a, s) : tc_launch<4, 8>(bwd, grid, a, s);
-  return mn3 == 4 ? tc_launch<8, 4>(bwd, grid, a, s) : tc_launch<8, 8>(bwd, grid, a, s);
-}
-
 }  // namespace
 
 cudaError_t configure_group(Ctx& c) {
   const Shape sh = shape_of(c);
-  if (use_tc(c)) {
-    const int mn3 = c.n3 <= 4 ? 4 : 8;
-    cudaError_t e = tc_dispatch_attrs(sh.mn1, mn3);
-    if (e != cudaSuccess) return e;
-  }
   const size_t fb = group_smem_bytes(c, false), bb = group_smem_bytes(c, true);
   if (bb > 227 * 1024) return cudaErrorInvalidConfiguration;
   return sh.vec ? dispatch_attrs<true>(sh.mn1, sh.mn3, fb, bb)
@@ -1253,11 +663,6 @@ cudaError_t run_group_fwd(Ctx& c, cudaStream_t s) {
   const Shape sh = shape_of(c);
   GroupArgs a = make_args(c, 0.f, c.p.work + 0);
   StageScope sc(c, ST_FWD_PREFIX, s);
-  if (use_tc(c)) {
-    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(c.NG_cap, (int64_t)c.sm_count * 2));
-    tc_dispatch_launch(sh.mn1, c.n3 <= 4 ? 4 : 8, false, grid, a, s);
-    return cudaGetLastError();
-  }
   const size_t bytes = group_smem_bytes(c, false);
   const int per_sm = bytes > 110 * 1024 ? 1 : 2;
   const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(c.NG_cap, (int64_t)c.sm_count * per_sm));
@@ -1270,11 +675,6 @@ cudaError_t run_group_bwd(Ctx& c, float lr, cudaStream_t s) {
   const Shape sh = shape_of(c);
   GroupArgs a = make_args(c, lr, c.p.work + 1);
   StageScope sc(c, ST_BWD_PREFIX, s);
-  if (use_tc(c)) {
-    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(c.NG_cap, (int64_t)c.sm_count));
-    tc_dispatch_launch(sh.mn1, c.n3 <= 4 ? 4 : 8, true, grid, a, s);
-    return cudaGetLastError();
-  }
   const size_t bytes = group_smem_bytes(c, true);
   const int per_sm = bytes > 110 * 1024 ? 1 : 2;
   const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(c.NG_cap, (int64_t)c.sm_count * per_sm));

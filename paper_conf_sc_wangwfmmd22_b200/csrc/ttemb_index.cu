@@ -107,7 +107,7 @@ k_build_keys(const IdxT* __restrict__ indices, const int64_t* __restrict__ offse
              uint32_t* __restrict__ bag_of, uint32_t* __restrict__ counts) {
   const int64_t nbags = (int64_t)T * B;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-  uint32_t err = 0;
+  uint32_t err = 0, multi = 0;
   for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < nnz; j += stride) {
     // bag of position j: the last b with offsets[b] <= j
     int64_t lo = 0, hi = nbags - 1;
@@ -132,8 +132,10 @@ k_build_keys(const IdxT* __restrict__ indices, const int64_t* __restrict__ offse
     if (b == 0 && v != 0) err |= kErrOffsets;
     if (b == nbags && v != nnz) err |= kErrOffsets;
     if (b < nbags && offsets[b + 1] < v) err |= kErrOffsets;
+    if (b < nbags && offsets[b + 1] - v != 1) multi = 1u;
   }
   if (err) atomicOr(counts + kCntErr, err);
+  if (multi) atomicOr(counts + kCntMulti, 1u);
 }
 
 // ------------------------------------------------------------------------------------

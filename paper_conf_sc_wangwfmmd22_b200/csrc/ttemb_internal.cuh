@@ -23,7 +23,7 @@ constexpr uint32_t kErrRange = 1u;     // an id outside [0, M_t)
 constexpr uint32_t kErrOffsets = 2u;   // malformed offsets
 
 // counts[] slots (device)
-constexpr int kCntU = 0, kCntP = 1, kCntNG = 2, kCntErr = 3, kNumCounts = 16;
+constexpr int kCntU = 0, kCntP = 1, kCntNG = 2, kCntErr = 3, kCntMulti = 4, kNumCounts = 16;
 
 // ---- stage ids for per-stage timing ----------------------------------------------
 enum Stage : int {
@@ -58,6 +58,7 @@ struct PlanDev {
   uint32_t *sc_counter, *sc_status;            // scans [3][tiles]
   uint32_t* work;                              // dynamic group schedulers [2]
   float *rows, *gbuf, *dabuf, *aggpart;
+  float *pbuf, *dpbuf;                         // tensor-core path: P and dL/dP per prefix
 };
 
 struct Ctx {
@@ -123,6 +124,10 @@ cudaError_t run_forward_compute(Ctx& c, float* out, const int64_t* offsets, cuda
 cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s);
 cudaError_t run_update(Ctx& c, float lr, cudaStream_t s);
 cudaError_t configure_group(Ctx& c);
+cudaError_t configure_tc(Ctx& c);
+bool tc_eligible(const Ctx& c);
+cudaError_t run_tc_fwd(Ctx& c, float* out, cudaStream_t s);
+cudaError_t run_tc_bwd(Ctx& c, float lr, cudaStream_t s);
 
 // ---- small helpers -------------------------------------------------------------------
 static inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }

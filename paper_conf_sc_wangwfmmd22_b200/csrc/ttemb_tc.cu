@@ -1,0 +1,687 @@
+// ttemb_tc.cu -- rank-64 tensor-core path (sm_100a): the rank-R contractions on tcgen05
+// (kind::tf32, 3xTF32 split, fp32 accumulate in TMEM) and the row stages as
+// high-occupancy warp-per-row-chunk kernels.  SURVEY 8(a) rows a5, a6, a9, a10, a12.
+//
+//   forward   k_tc_p      P_tile = A1 . X1^T           (Reuse buffer) -> Pbuf
+//             k_rows_fwd  E_u = P_q . C3[i3_u]         (Eq. 2)  -> out (one id per bag)
+//                                                               or rows[u] (pooled later)
+//   backward  k_rows_bwd  dP_q += G_u . C3[i3_u]^T     (Eq. 6)    -> dPbuf
+//                         dC3[i3_u] += P_q^T G_u       (red.global.add.v4, L2-resident)
+//             k_tc_bwd2   dC2[i2] += A2 . D2^T,  dA^T = X2 . D1^T  per i2-group
+//                         (dC2 reduced in TMEM over the whole group, no atomics; fused
+//                          SGD/Adagrad update of the C2 slice the CTA owns)
+// Operands are staged as K-major "CM" core-matrix layouts (tc.cuh):
+//   A1 = CM(m, r1)  X1 = CM(c, r1)  X2 = CM(r1, c)  A2 = CM(r1, m)  D1 = CM(m, c)  D2 = CM(c, m)
+// Tiles: 64 rows (q, j1) x one j2 block (64 columns of C2) x K = 64.  The next chunk's
+// operands are prefetched into registers while the current chunk's MMAs run, and the
+// next group is claimed one ahead.  The row kernels walk 16 consecutive unique rows per
+// warp, so Zipf-hot prefixes (hundreds of rows) spread over many warps.
+#include <algorithm>
+
+#include "tc.cuh"
+#include "ttemb_internal.cuh"
+
+namespace ttemb {
+
+namespace {
+
+constexpr int TR = 64, TMT = 64, TCW = 64, TNRB = 8, TNT = 256;
+constexpr uint32_t TCM = 64 * 64 * 4;          // bytes of one 64x64 fp32 CM matrix
+constexpr int RCH = 16;                        // unique rows per warp item
+constexpr int SPS = TR + 4;                    // smem P row stride (floats)
+
+struct TcArgs {
+  float* cores;
+  float* grads;
+  float* state;
+  const TableMeta* meta;
+  const uint32_t *counts, *grp_off, *grp_t, *grp_i2, *grp_pfx, *pfx_i1, *pfx_t, *row_seg, *row_i3,
+      *row_pfx, *seg_off, *sbag;
+  float* pbuf;          // [P][n1][NC]  prefix products (Reuse buffer)
+  float* dpbuf;         // [P][n1][NC]  dL/dP per prefix
+  float* rows;          // [U][N]
+  const float* gbuf;    // [U][N]  aggregated row gradients
+  float* dabuf;         // [P][n1][R] dC1 partials
+  float* out;           // [B][T][N]
+  uint32_t* work;
+  int n1, n2, n3, N, NC, n1s;
+  float lr, eps;
+  int opt, fused;
+};
+
+__device__ __forceinline__ float* fat(float* base, uint32_t off) {
+  return reinterpret_cast<float*>(reinterpret_cast<char*>(base) + off);
+}
+__device__ __forceinline__ void st_split4(float* hi, float* lo, uint32_t off, float4 v) {
+  const float4 h = make_float4(tc::tf32_hi(v.x), tc::tf32_hi(v.y), tc::tf32_hi(v.z), tc::tf32_hi(v.w));
+  *reinterpret_cast<float4*>(fat(hi, off)) = h;
+  *reinterpret_cast<float4*>(fat(lo, off)) = make_float4(v.x - h.x, v.y - h.y, v.z - h.z, v.w - h.w);
+}
+__device__ __forceinline__ void red_add_v4(float* addr, float4 v) {
+  asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(addr), "f"(v.x), "f"(v.y),
+               "f"(v.z), "f"(v.w)
+               : "memory");
+}
+
+// 3xTF32 64x64 (K = 64) product of two K-major CM matrices into TMEM column base d.
+__device__ __forceinline__ void mma3(uint32_t d, const float* ah, const float* al, const float* bh,
+                                     const float* bl, bool accumulate) {
+  const uint32_t id = tc::idesc_tf32(64, 64, false, false);
+  const uint32_t sah = tc::smem_u32(ah), sal = tc::smem_u32(al);
+  const uint32_t sbh = tc::smem_u32(bh), sbl = tc::smem_u32(bl);
+#pragma unroll
+  for (int kk = 0; kk < 8; ++kk) {
+    const uint32_t o = kk * 2 * TNRB * 128;
+    const uint64_t dah = tc::sdesc(sah + o, TNRB * 128, 128), dal = tc::sdesc(sal + o, TNRB * 128, 128);
+    const uint64_t dbh = tc::sdesc(sbh + o, TNRB * 128, 128), dbl = tc::sdesc(sbl + o, TNRB * 128, 128);
+    tc::mma_tf32(d, dah, dbh, id, (accumulate || kk > 0) ? 1u : 0u);
+    tc::mma_tf32(d, dah, dbl, id, 1u);
+    tc::mma_tf32(d, dal, dbh, id, 1u);
+  }
+}
+
+__device__ __forceinline__ void publish() {   // generic smem writes -> tensor-core reads
+  tc::fence_async_smem();
+  tc::fence_before();
+  __syncthreads();
+  tc::fence_after();
+}
+
+// Float4 "pattern" loads of a 64x64 tile of a row-major matrix (row stride ld) at
+// (row0, col0): ROWQ = 4 rows of one column (for CM(col, row)), COLQ = 4 columns of one row
+// (for CM(row, col)).  Element e = tid + 256 k, k < 4.
+__device__ __forceinline__ void load_rowq(float4 (&v)[4], const float* base, size_t ld, int nrows) {
+#pragma unroll
+  for (int k = 0; k < 4; ++k) {
+    const int e = threadIdx.x + TNT * k;
+    const int c = e & 63, rq = e >> 6;
+    float x[4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) x[i] = (4 * rq + i < nrows) ? __ldg(base + (size_t)(4 * rq + i) * ld + c) : 0.f;
+    v[k] = make_float4(x[0], x[1], x[2], x[3]);
+  }
+}
+__device__ __forceinline__ void load_colq(float4 (&v)[4], const float* base, size_t ld, int nrows) {
+#pragma unroll
+  for (int k = 0; k < 4; ++k) {
+    const int e = threadIdx.x + TNT * k;
+    const int r = e & 63, cq = e >> 6;
+    v[k] = r < nrows ? __ldg(reinterpret_cast<const float4*>(base + (size_t)r * ld + 4 * cq))
+                     : make_float4(0.f, 0.f, 0.f, 0.f);
+  }
+}
+// Store a pattern into its CM layout: rowq -> CM(col, 4 rows), colq -> CM(row, 4 cols).
+__device__ __forceinline__ void store_pat(float* hi, float* lo, const float4 (&v)[4]) {
+#pragma unroll
+  for (int k = 0; k < 4; ++k) {
+    const int e = threadIdx.x + TNT * k;
+    st_split4(hi, lo, tc::cm_off(e & 63, 4 * (e >> 6), TNRB), v[k]);
+  }
+}
+
+// Per-m-tile row table in shared memory: for tile row m = (q, j1):
+//   rowp[m] = p * n1 + j1      (row of pbuf / dpbuf / dabuf)
+//   rowa[m] = i1_p * n1 + j1   (row of C1)        -- 0xffffffff past the tile
+__device__ __forceinline__ void fill_table(const TcArgs& a, uint32_t* rowp, uint32_t* rowa,
+                                           uint32_t qa, int npq) {
+  const int m = threadIdx.x;
+  if (m < 64) {
+    const int rows = npq << a.n1s;
+    uint32_t vp = 0xffffffffu, va = 0xffffffffu;
+    if (m < rows) {
+      const uint32_t p = a.grp_pfx[qa + (m >> a.n1s)];
+      const uint32_t j1 = m & ((1 << a.n1s) - 1);
+      vp = (p << a.n1s) + j1;
+      va = (a.pfx_i1[p] << a.n1s) + j1;
+    }
+    rowp[m] = vp;
+    rowa[m] = va;
+  }
+}
+
+// Tile matrix X[m][col] with row m at src + tab[m] * ld (rows with tab == ~0 read as 0):
+// ROWQ = 4 consecutive m of one column (for CM(col, m)), COLQ = 4 columns of one m (CM(m, col)).
+__device__ __forceinline__ void load_tab(float4 (&v)[4], const float* src, size_t ld, const uint32_t* tab,
+                                         bool rowq) {
+#pragma unroll
+  for (int k = 0; k < 4; ++k) {
+    const int e = threadIdx.x + TNT * k;
+    if (rowq) {
+      const int c = e & 63, mq = e >> 6;
+      float x[4];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const uint32_t r = tab[4 * mq + i];
+        x[i] = r != 0xffffffffu ? __ldg(src + (size_t)r * ld + c) : 0.f;
+      }
+      v[k] = make_float4(x[0], x[1], x[2], x[3]);
+    } else {
+      const int m = e & 63, cq = e >> 6;
+      const uint32_t r = tab[m];
+      v[k] = r != 0xffffffffu ? __ldg(reinterpret_cast<const float4*>(src + (size_t)r * ld + 4 * cq))
+                              : make_float4(0.f, 0.f, 0.f, 0.f);
+    }
+  }
+}
+
+__device__ __forceinline__ const float* c2_slice(const TcArgs& a, uint32_t g) {
+  return a.cores + a.meta[a.grp_t[g]].c2_off + (size_t)a.grp_i2[g] * TR * a.NC;
+}
+
+// ------------------------------------------------------------------------------------
+// Forward GEMM: P = A1 . X1^T for every group, written to pbuf
+// ------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(TNT, 2) k_tc_p(TcArgs a) {
+  extern __shared__ __align__(128) char smem[];
+  float* x1h = reinterpret_cast<float*>(smem);
+  float* x1l = x1h + TCM / 4;
+  float* a1h = x1l + TCM / 4;
+  float* a1l = a1h + TCM / 4;
+  __shared__ uint64_t mbar;
+  __shared__ uint32_t s_tmem, s_g[2], s_rowp[2][64], s_rowa[2][64];
+  const int tid = threadIdx.x, w = tid >> 5, lane = tid & 31, q4 = w & 3, half = w >> 2;
+  if (tid == 0) {
+    tc::mbar_init(&mbar, 1);
+    tc::fence_mbar_init();
+    s_g[0] = atomicAdd(a.work, 1u);
+    s_g[1] = atomicAdd(a.work, 1u);
+  }
+  if (tid < 32) tc::tmem_alloc(&s_tmem, 64);
+  tc::fence_before();
+  __syncthreads();
+  tc::fence_after();
+  const uint32_t tP = s_tmem;
+  uint32_t phase = 0;
+  const uint32_t NG = a.counts[kCntNG];
+  const int PPT = TMT >> a.n1s, NCH = a.NC / TCW;
+  uint32_t g = s_g[0], gnext = s_g[1];
+  int tb = 0;
+  float4 px[4], pa[4];
+  if (g < NG) {
+    fill_table(a, s_rowp[0], s_rowa[0], a.grp_off[g], (int)min((uint32_t)PPT, a.grp_off[g + 1] - a.grp_off[g]));
+    __syncthreads();
+    load_rowq(px, c2_slice(a, g), a.NC, TR);
+    load_tab(pa, a.cores + a.meta[a.grp_t[g]].c1_off, TR, s_rowa[0], false);
+  }
+  while (g < NG) {
+    const uint32_t q0 = a.grp_off[g], q1 = a.grp_off[g + 1];
+    const float* C2s = c2_slice(a, g);
+    const uint32_t nmt = (q1 - q0 + PPT - 1) / PPT;
+    for (uint32_t mt = 0; mt < nmt; ++mt) {
+      __syncthreads();
+      store_pat(a1h, a1l, pa);                              // A1 = CM(m, r1)
+      for (int k = 0; k < NCH; ++k) {
+        if (k > 0) __syncthreads();
+        store_pat(x1h, x1l, px);                            // X1 = CM(c, r1)
+        if (k + 1 < NCH) {
+          load_rowq(px, C2s + (k + 1) * TCW, a.NC, TR);
+        } else {                                            // next tile (or group): table + prefetch
+          uint32_t ng = g, nqa = q0 + (mt + 1) * PPT;
+          if (mt + 1 >= nmt) { ng = gnext; nqa = ng < NG ? a.grp_off[ng] : 0; }
+          if (ng < NG) {
+            fill_table(a, s_rowp[tb ^ 1], s_rowa[tb ^ 1], nqa, (int)min((uint32_t)PPT, a.grp_off[ng + 1] - nqa));
+            __syncthreads();
+            load_rowq(px, c2_slice(a, ng), a.NC, TR);
+            load_tab(pa, a.cores + a.meta[a.grp_t[ng]].c1_off, TR, s_rowa[tb ^ 1], false);
+          }
+        }
+        publish();
+        if (tid == 0) {
+          mma3(tP, a1h, a1l, x1h, x1l, false);
+          tc::commit(&mbar);
+        }
+        __syncwarp();
+        tc::mbar_wait(&mbar, phase);
+        phase ^= 1u;
+        tc::fence_after();
+        float v[32];
+        tc::tmem_ld32(tc::taddr(tP, 32 * q4, 32 * half), v);
+        if (lane < 16) {
+          const uint32_t r = s_rowp[tb][16 * q4 + lane];
+          if (r != 0xffffffffu) {
+            float* dst = a.pbuf + (size_t)r * a.NC + k * TCW + 32 * half;
+#pragma unroll
+            for (int j = 0; j < 32; j += 4)
+              *reinterpret_cast<float4*>(dst + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
+          }
+        }
+        tc::fence_before();
+      }
+      tb ^= 1;
+    }
+    __syncthreads();
+    if (tid == 0) s_g[1] = atomicAdd(a.work, 1u);
+    __syncthreads();
+    g = gnext;
+    gnext = s_g[1];
+  }
+  tc::fence_before();
+  __syncthreads();
+  tc::fence_after();
+  if (tid < 32) tc::tmem_dealloc(tP, 64);
+}
+
+// ------------------------------------------------------------------------------------
+// Row stages: one warp per chunk of RCH consecutive unique rows; the next row's C3 slice,
+// G row and (on a prefix change) P_q are prefetched into registers while the current row
+// computes from shared memory.
+// ------------------------------------------------------------------------------------
+struct WarpSmem {
+  float sP[16 * SPS];      // P_q rows j12 < 16, r < 64
+  float sC3[TR * 8];       // C3[i3_u] : [r][j3], n3 <= 8
+  float sG[128];           // G_u : [j12][j3]
+};
+
+template <int N3>
+struct RowPref {
+  static constexpr int C3L = TR * N3 / 4 / 32;   // float4 of a C3 slice per lane
+  float4 c3[C3L];
+  float4 p[8];                                  // P_q: J12 * 16 float4 <= 256
+  float4 g;                                     // G_u: J12 * N3 / 4 <= 32 float4
+  uint32_t q;
+};
+
+template <int N3>
+__device__ __forceinline__ void row_prefetch(RowPref<N3>& f, const TcArgs& a, uint32_t u, int J12,
+                                             bool load_p, bool load_g, uint32_t cur) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t q = a.row_pfx[u];
+  const float4* c3 = reinterpret_cast<const float4*>(a.cores + a.meta[a.pfx_t[q]].c3_off +
+                                                     (size_t)a.row_i3[u] * TR * N3);
+#pragma unroll
+  for (int i = 0; i < RowPref<N3>::C3L; ++i) f.c3[i] = __ldg(c3 + lane + 32 * i);
+  if (load_p && q != cur) {
+    const float4* src = reinterpret_cast<const float4*>(a.pbuf + (size_t)q * J12 * TR);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      const int e = lane + 32 * i;
+      if (e < J12 * (TR / 4)) f.p[i] = __ldg(src + e);
+    }
+  }
+  if (load_g && lane < J12 * N3 / 4) f.g = __ldg(reinterpret_cast<const float4*>(a.gbuf + (size_t)u * a.N) + lane);
+  f.q = q;
+}
+
+template <int N3>
+__device__ __forceinline__ void row_stage(WarpSmem& ws, const RowPref<N3>& f, int J12, bool store_p,
+                                          bool store_g) {
+  const int lane = threadIdx.x & 31;
+#pragma unroll
+  for (int i = 0; i < RowPref<N3>::C3L; ++i) reinterpret_cast<float4*>(ws.sC3)[lane + 32 * i] = f.c3[i];
+  if (store_p) {
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      const int e = lane + 32 * i;
+      if (e < J12 * (TR / 4)) {
+        const int j = e >> 4, r4 = e & 15;
+        *reinterpret_cast<float4*>(ws.sP + j * SPS + 4 * r4) = f.p[i];
+      }
+    }
+  }
+  if (store_g && lane < J12 * N3 / 4) reinterpret_cast<float4*>(ws.sG)[lane] = f.g;
+}
+
+// forward: E_u[j12][j3] = sum_r P_q[j12][r] C3_u[r][j3]; lane = (j12 = lane / 2, r half)
+template <int N3>
+__global__ void __launch_bounds__(128) k_rows_fwd(TcArgs a) {
+  __shared__ __align__(16) WarpSmem ws_all[4];
+  WarpSmem& ws = ws_all[threadIdx.x >> 5];
+  const int lane = threadIdx.x & 31, J12 = a.n1 * a.n2;
+  const uint32_t U = a.counts[kCntU];
+  const int j12 = lane >> 1, rh = lane & 1;
+  const int64_t nch = (U + RCH - 1) / RCH;
+  for (int64_t ch = (int64_t)blockIdx.x * 4 + (threadIdx.x >> 5); ch < nch; ch += (int64_t)gridDim.x * 4) {
+    const uint32_t u0 = (uint32_t)ch * RCH, u1 = min(u0 + RCH, U);
+    RowPref<N3> f;
+    uint32_t cur = 0xffffffffu;
+    row_prefetch<N3>(f, a, u0, J12, true, false, cur);
+    for (uint32_t u = u0; u < u1; ++u) {
+      const bool newp = f.q != cur;
+      __syncwarp();
+      row_stage<N3>(ws, f, J12, newp, false);
+      cur = f.q;
+      __syncwarp();
+      if (u + 1 < u1) row_prefetch<N3>(f, a, u + 1, J12, true, false, cur);
+      float acc[N3];
+#pragma unroll
+      for (int j = 0; j < N3; ++j) acc[j] = 0.f;
+      if (j12 < J12) {
+        const float* pr = ws.sP + j12 * SPS + 32 * rh;
+        const float* c3 = ws.sC3 + 32 * rh * N3;
+#pragma unroll 8
+        for (int r = 0; r < 32; r += 4) {
+          const float4 p4 = *reinterpret_cast<const float4*>(pr + r);
+          const float pv[4] = {p4.x, p4.y, p4.z, p4.w};
+#pragma unroll
+          for (int i = 0; i < 4; ++i)
+#pragma unroll
+            for (int j = 0; j < N3; j += 4) {
+              const float4 c4 = *reinterpret_cast<const float4*>(c3 + (r + i) * N3 + j);
+              acc[j] = fmaf(pv[i], c4.x, acc[j]);
+              acc[j + 1] = fmaf(pv[i], c4.y, acc[j + 1]);
+              acc[j + 2] = fmaf(pv[i], c4.z, acc[j + 2]);
+              acc[j + 3] = fmaf(pv[i], c4.w, acc[j + 3]);
+            }
+        }
+      }
+#pragma unroll
+      for (int j = 0; j < N3; ++j) acc[j] += __shfl_xor_sync(0xffffffffu, acc[j], 1);
+      if (rh == 0 && j12 < J12) {
+        float* d = a.rows + (size_t)u * a.N + j12 * N3;
+#pragma unroll
+        for (int j = 0; j < N3; j += 4) *reinterpret_cast<float4*>(d + j) = make_float4(acc[j], acc[j + 1], acc[j + 2], acc[j + 3]);
+      }
+    }
+  }
+}
+
+// dPbuf rows of prefixes whose rows straddle a chunk boundary are accumulated with atomics:
+// zero them first.
+__global__ void __launch_bounds__(256) k_dp_zero(TcArgs a) {
+  const uint32_t P = a.counts[kCntP];
+  const int J12R = a.n1 * a.n2 * TR;
+  const int lane = threadIdx.x & 31;
+  for (uint32_t q = blockIdx.x * 8 + (threadIdx.x >> 5); q < P; q += gridDim.x * 8) {
+    const uint32_t r0 = a.row_seg[q], r1 = a.row_seg[q + 1];
+    if (r0 / RCH == (r1 - 1) / RCH) continue;
+    float4* d = reinterpret_cast<float4*>(a.dpbuf + (size_t)q * J12R);
+    for (int f = lane; f < J12R / 4; f += 32) d[f] = make_float4(0.f, 0.f, 0.f, 0.f);
+  }
+}
+
+// backward row stage: dP_q[j12][r] += sum_j3 G_u[j12][j3] C3_u[r][j3]   (lane = j12, r half)
+//                     dC3[i3][r][j3] += sum_j12 P_q[j12][r] G_u[j12][j3] (lane = r pair)
+template <int N3>
+__global__ void __launch_bounds__(128) k_rows_bwd(TcArgs a) {
+  __shared__ __align__(16) WarpSmem ws_all[4];
+  WarpSmem& ws = ws_all[threadIdx.x >> 5];
+  const int lane = threadIdx.x & 31, J12 = a.n1 * a.n2;
+  const uint32_t U = a.counts[kCntU];
+  const int j12 = lane >> 1, rh = lane & 1;
+  const int64_t nch = (U + RCH - 1) / RCH;
+  for (int64_t ch = (int64_t)blockIdx.x * 4 + (threadIdx.x >> 5); ch < nch; ch += (int64_t)gridDim.x * 4) {
+    const uint32_t u0 = (uint32_t)ch * RCH, u1 = min(u0 + RCH, U);
+    uint32_t cur = 0xffffffffu;
+    float dp[32];
+#pragma unroll
+    for (int i = 0; i < 32; ++i) dp[i] = 0.f;
+    auto flush = [&](uint32_t q) {
+      if (j12 >= J12) return;
+      const uint32_t r0 = a.row_seg[q], r1 = a.row_seg[q + 1];
+      float* d = a.dpbuf + ((size_t)q * J12 + j12) * TR + 32 * rh;
+      const bool whole = (r0 / RCH == (r1 - 1) / RCH);
+#pragma unroll
+      for (int i = 0; i < 32; i += 4) {
+        const float4 v = make_float4(dp[i], dp[i + 1], dp[i + 2], dp[i + 3]);
+        if (whole) *reinterpret_cast<float4*>(d + i) = v;
+        else red_add_v4(d + i, v);
+      }
+#pragma unroll
+      for (int i = 0; i < 32; ++i) dp[i] = 0.f;
+    };
+    RowPref<N3> f;
+    row_prefetch<N3>(f, a, u0, J12, true, true, cur);
+    for (uint32_t u = u0; u < u1; ++u) {
+      const uint32_t q = f.q;
+      const size_t c3o = a.meta[a.pfx_t[q]].c3_off + (size_t)a.row_i3[u] * TR * N3;
+      if (q != cur && cur != 0xffffffffu) flush(cur);
+      const bool newp = q != cur;
+      __syncwarp();
+      row_stage<N3>(ws, f, J12, newp, true);
+      cur = q;
+      __syncwarp();
+      if (u + 1 < u1) row_prefetch<N3>(f, a, u + 1, J12, true, true, cur);
+      if (j12 < J12) {     // dP: 32 r of this lane's half
+        float gg[N3];
+#pragma unroll
+        for (int j = 0; j < N3; j += 4) {
+          const float4 g4 = *reinterpret_cast<const float4*>(ws.sG + j12 * N3 + j);
+          gg[j] = g4.x; gg[j + 1] = g4.y; gg[j + 2] = g4.z; gg[j + 3] = g4.w;
+        }
+        const float* c3 = ws.sC3 + 32 * rh * N3;
+#pragma unroll
+        for (int i = 0; i < 32; ++i) {
+#pragma unroll
+          for (int j = 0; j < N3; j += 4) {
+            const float4 c4 = *reinterpret_cast<const float4*>(c3 + i * N3 + j);
+            dp[i] = fmaf(gg[j], c4.x, dp[i]);
+            dp[i] = fmaf(gg[j + 1], c4.y, dp[i]);
+            dp[i] = fmaf(gg[j + 2], c4.z, dp[i]);
+            dp[i] = fmaf(gg[j + 3], c4.w, dp[i]);
+          }
+        }
+      }
+      {                    // dC3: r = 2 lane, 2 lane + 1
+        float acc[2][N3];
+#pragma unroll
+        for (int i = 0; i < 2; ++i)
+#pragma unroll
+          for (int j = 0; j < N3; ++j) acc[i][j] = 0.f;
+        for (int jj = 0; jj < J12; ++jj) {
+          const float2 p2 = *reinterpret_cast<const float2*>(ws.sP + jj * SPS + 2 * lane);
+#pragma unroll
+          for (int j = 0; j < N3; j += 4) {
+            const float4 g4 = *reinterpret_cast<const float4*>(ws.sG + jj * N3 + j);
+            acc[0][j] = fmaf(p2.x, g4.x, acc[0][j]); acc[0][j + 1] = fmaf(p2.x, g4.y, acc[0][j + 1]);
+            acc[0][j + 2] = fmaf(p2.x, g4.z, acc[0][j + 2]); acc[0][j + 3] = fmaf(p2.x, g4.w, acc[0][j + 3]);
+            acc[1][j] = fmaf(p2.y, g4.x, acc[1][j]); acc[1][j + 1] = fmaf(p2.y, g4.y, acc[1][j + 1]);
+            acc[1][j + 2] = fmaf(p2.y, g4.z, acc[1][j + 2]); acc[1][j + 3] = fmaf(p2.y, g4.w, acc[1][j + 3]);
+          }
+        }
+        float* d = a.grads + c3o + (size_t)(2 * lane) * N3;
+#pragma unroll
+        for (int i = 0; i < 2; ++i)
+#pragma unroll
+          for (int j = 0; j < N3; j += 4)
+            red_add_v4(d + i * N3 + j, make_float4(acc[i][j], acc[i][j + 1], acc[i][j + 2], acc[i][j + 3]));
+      }
+    }
+    if (cur != 0xffffffffu) flush(cur);
+  }
+}
+
+// ------------------------------------------------------------------------------------
+// Backward GEMMs per i2-group: dA^T = X2 . D1^T (TMEM, accumulated over chunks) and
+// dC2[chunk] += A2 . D2^T (TMEM, accumulated over m-tiles)
+// ------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(TNT, 1) k_tc_bwd2(TcArgs a) {
+  extern __shared__ __align__(128) char smem[];
+  float* base = reinterpret_cast<float*>(smem);
+  float *x2h = base, *x2l = x2h + TCM / 4, *a2h = x2l + TCM / 4, *a2l = a2h + TCM / 4;
+  float *d1h = a2l + TCM / 4, *d1l = d1h + TCM / 4, *d2h = d1l + TCM / 4, *d2l = d2h + TCM / 4;
+  __shared__ uint64_t mbar;
+  __shared__ uint32_t s_tmem, s_g[2], s_rowp[2][64], s_rowa[2][64];
+  const int tid = threadIdx.x, w = tid >> 5, lane = tid & 31, q4 = w & 3, half = w >> 2;
+  if (tid == 0) {
+    tc::mbar_init(&mbar, 1);
+    tc::fence_mbar_init();
+    s_g[0] = atomicAdd(a.work, 1u);
+    s_g[1] = atomicAdd(a.work, 1u);
+  }
+  if (tid < 32) tc::tmem_alloc(&s_tmem, 512);
+  tc::fence_before();
+  __syncthreads();
+  tc::fence_after();
+  const uint32_t tDA = s_tmem, tDC2 = s_tmem + 64;
+  uint32_t phase = 0;
+  const uint32_t NG = a.counts[kCntNG];
+  const int PPT = TMT >> a.n1s, NCH = a.NC / TCW;
+  uint32_t g = s_g[0], gnext = s_g[1];
+  int tb = 0;
+  float4 px[4], pd1[4], pd2[4], pa[4];
+  if (g < NG) {
+    fill_table(a, s_rowp[0], s_rowa[0], a.grp_off[g], (int)min((uint32_t)PPT, a.grp_off[g + 1] - a.grp_off[g]));
+    __syncthreads();
+    load_colq(px, c2_slice(a, g), a.NC, TR);
+    load_tab(pd1, a.dpbuf, a.NC, s_rowp[0], false);
+    load_tab(pd2, a.dpbuf, a.NC, s_rowp[0], true);
+    load_tab(pa, a.cores + a.meta[a.grp_t[g]].c1_off, TR, s_rowa[0], true);
+  }
+  while (g < NG) {
+    const uint32_t i2 = a.grp_i2[g];
+    const uint32_t q0 = a.grp_off[g], q1 = a.grp_off[g + 1];
+    const size_t c2o = a.meta[a.grp_t[g]].c2_off + (size_t)i2 * TR * a.NC;
+    const float* C2s = a.cores + c2o;
+    const uint32_t nmt = (q1 - q0 + PPT - 1) / PPT;
+    for (uint32_t mt = 0; mt < nmt; ++mt) {
+      __syncthreads();
+      store_pat(a2h, a2l, pa);                               // A2 = CM(r1, m)
+      for (int k = 0; k < NCH; ++k) {
+        if (k > 0) __syncthreads();
+        store_pat(x2h, x2l, px);                             // X2 = CM(r1, c)
+        store_pat(d1h, d1l, pd1);                            // D1 = CM(m, c)
+        store_pat(d2h, d2l, pd2);                            // D2 = CM(c, m)
+        if (k + 1 < NCH) {
+          load_colq(px, C2s + (k + 1) * TCW, a.NC, TR);
+          load_tab(pd1, a.dpbuf + (k + 1) * TCW, a.NC, s_rowp[tb], false);
+          load_tab(pd2, a.dpbuf + (k + 1) * TCW, a.NC, s_rowp[tb], true);
+        } else {                                             // next tile (or group)
+          uint32_t ng = g, nqa = q0 + (mt + 1) * PPT;
+          if (mt + 1 >= nmt) { ng = gnext; nqa = ng < NG ? a.grp_off[ng] : 0; }
+          if (ng < NG) {
+            fill_table(a, s_rowp[tb ^ 1], s_rowa[tb ^ 1], nqa, (int)min((uint32_t)PPT, a.grp_off[ng + 1] - nqa));
+            __syncthreads();
+            load_colq(px, c2_slice(a, ng), a.NC, TR);
+            load_tab(pd1, a.dpbuf, a.NC, s_rowp[tb ^ 1], false);
+            load_tab(pd2, a.dpbuf, a.NC, s_rowp[tb ^ 1], true);
+            load_tab(pa, a.cores + a.meta[a.grp_t[ng]].c1_off, TR, s_rowa[tb ^ 1], true);
+          }
+        }
+        publish();
+        if (tid == 0) {
+          mma3(tDA, x2h, x2l, d1h, d1l, k > 0);              // dA^T [r1][m]
+          mma3(tDC2 + 64 * k, a2h, a2l, d2h, d2l, mt > 0);   // dC2  [r1][c]
+          tc::commit(&mbar);
+        }
+        __syncwarp();
+        tc::mbar_wait(&mbar, phase);
+        phase ^= 1u;
+        tc::fence_after();
+      }
+      {   // dA^T -> dabuf[(p, j1)][r1]
+        float v[32];
+        tc::tmem_ld32(tc::taddr(tDA, 32 * q4, 32 * half), v);
+        if (lane < 16) {
+          const int r1 = 16 * q4 + lane;
+#pragma unroll
+          for (int j = 0; j < 32; ++j) {
+            const uint32_t r = s_rowp[tb][32 * half + j];
+            if (r != 0xffffffffu) a.dabuf[(size_t)r * TR + r1] = v[j];
+          }
+        }
+        tc::fence_before();
+      }
+      tb ^= 1;
+    }
+    for (int k = 0; k < NCH; ++k) {   // this CTA owns C2[t][i2]: gradient or fused update
+      float v[32];
+      tc::tmem_ld32(tc::taddr(tDC2 + 64 * k, 32 * q4, 32 * half), v);
+      if (lane < 16) {
+        const int r1 = 16 * q4 + lane;
+        const size_t b0 = c2o + (size_t)r1 * a.NC + k * TCW + 32 * half;
+        if (a.fused) {
+          if (a.opt == TTEMB_SGD) {
+            float4 x[8];
+#pragma unroll
+            for (int j = 0; j < 8; ++j) x[j] = *reinterpret_cast<const float4*>(a.cores + b0 + 4 * j);
+#pragma unroll
+            for (int j = 0; j < 8; ++j)
+              *reinterpret_cast<float4*>(a.cores + b0 + 4 * j) =
+                  make_float4(x[j].x - a.lr * v[4 * j], x[j].y - a.lr * v[4 * j + 1],
+                              x[j].z - a.lr * v[4 * j + 2], x[j].w - a.lr * v[4 * j + 3]);
+          } else {
+#pragma unroll
+            for (int j = 0; j < 32; ++j) {
+              const float sv = a.state[b0 + j] + v[j] * v[j];
+              a.state[b0 + j] = sv;
+              a.cores[b0 + j] = a.cores[b0 + j] - a.lr * v[j] / (sqrtf(sv) + a.eps);
+            }
+          }
+        } else {
+#pragma unroll
+          for (int j = 0; j < 32; j += 4)
+            *reinterpret_cast<float4*>(a.grads + b0 + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
+        }
+      }
+    }
+    tc::fence_before();
+    __syncthreads();
+    if (tid == 0) s_g[1] = atomicAdd(a.work, 1u);
+    __syncthreads();
+    g = gnext;
+    gnext = s_g[1];
+  }
+  tc::fence_before();
+  __syncthreads();
+  tc::fence_after();
+  if (tid < 32) tc::tmem_dealloc(tDA, 512);
+}
+
+TcArgs make_tc_args(Ctx& c, float lr, uint32_t* work, float* out) {
+  const PlanDev& p = c.p;
+  TcArgs a;
+  a.cores = c.cores; a.grads = c.grads; a.state = c.state; a.meta = c.d_meta;
+  a.counts = p.counts; a.grp_off = p.grp_off; a.grp_t = p.grp_t; a.grp_i2 = p.grp_i2;
+  a.grp_pfx = p.grp_pfx; a.pfx_i1 = p.pfx_i1; a.pfx_t = p.pfx_t; a.row_seg = p.row_seg;
+  a.row_i3 = p.row_i3; a.row_pfx = p.row_pfx; a.seg_off = p.seg_off; a.sbag = p.sbag;
+  a.pbuf = p.pbuf; a.dpbuf = p.dpbuf; a.rows = p.rows; a.gbuf = p.gbuf; a.dabuf = p.dabuf;
+  a.out = out; a.work = work;
+  a.n1 = c.n1; a.n2 = c.n2; a.n3 = c.n3; a.N = c.N; a.NC = c.NC;
+  a.n1s = c.n1 == 1 ? 0 : c.n1 == 2 ? 1 : c.n1 == 4 ? 2 : 3;
+  a.lr = lr; a.eps = c.eps; a.opt = c.opt; a.fused = (c.flags & TTEMB_FUSED_UPDATE) ? 1 : 0;
+  return a;
+}
+
+constexpr size_t kTcPSmem = 4 * TCM;
+constexpr size_t kTcBwdSmem = 8 * TCM;
+
+}  // namespace
+
+bool tc_eligible(const Ctx& c) {
+  return !(c.flags & TTEMB_FP32_CORES) && c.R == TR && (c.n3 == 4 || c.n3 == 8) &&
+         (c.n1 == 1 || c.n1 == 2 || c.n1 == 4 || c.n1 == 8) && c.n1 * c.n2 <= 16 && c.n2 <= 7;
+}
+
+cudaError_t configure_tc(Ctx& c) {
+  if (!tc_eligible(c)) return cudaSuccess;
+  cudaError_t e = cudaFuncSetAttribute(k_tc_p, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kTcPSmem);
+  if (e != cudaSuccess) return e;
+  return cudaFuncSetAttribute(k_tc_bwd2, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kTcBwdSmem);
+}
+
+// Forward contractions: P (tcgen05) then rows / direct output.
+cudaError_t run_tc_fwd(Ctx& c, float* out, cudaStream_t s) {
+  TcArgs a = make_tc_args(c, 0.f, c.p.work + 0, out);
+  {
+    StageScope sc(c, ST_FWD_PREFIX, s);
+    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(c.NG_cap, (int64_t)c.sm_count * 2));
+    k_tc_p<<<grid, TNT, kTcPSmem, s>>>(a);
+  }
+  {
+    StageScope sc(c, ST_FWD_ROWS, s);
+    const int grid = grid_for(c, cdiv(c.U_cap, RCH), 4, 8);
+    if (c.n3 == 4) k_rows_fwd<4><<<grid, 128, 0, s>>>(a);
+    else k_rows_fwd<8><<<grid, 128, 0, s>>>(a);
+  }
+  return cudaGetLastError();
+}
+
+// Backward contractions: dP / dC3 row stage, then the group GEMMs (dC2, dA).
+cudaError_t run_tc_bwd(Ctx& c, float lr, cudaStream_t s) {
+  TcArgs a = make_tc_args(c, lr, c.p.work + 1, nullptr);
+  {
+    StageScope sc(c, ST_BWD_ROWS, s);
+    k_dp_zero<<<grid_for(c, c.P_cap, 8, 8), 256, 0, s>>>(a);
+    const int grid = grid_for(c, cdiv(c.U_cap, RCH), 4, 8);
+    if (c.n3 == 4) k_rows_bwd<4><<<grid, 128, 0, s>>>(a);
+    else k_rows_bwd<8><<<grid, 128, 0, s>>>(a);
+  }
+  {
+    StageScope sc(c, ST_BWD_PREFIX, s);
+    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(c.NG_cap, (int64_t)c.sm_count));
+    k_tc_bwd2<<<grid, TNT, kTcBwdSmem, s>>>(a);
+  }
+  return cudaGetLastError();
+}
+
+}  // namespace ttemb
