@@ -171,27 +171,32 @@ __device__ __forceinline__ const float* c2_slice(const TcArgs& a, uint32_t g) {
 // ------------------------------------------------------------------------------------
 // Forward GEMM: P = A1 . X1^T for every group, written to pbuf
 // ------------------------------------------------------------------------------------
+// Forward GEMM: P = A1 . X1^T for every group, written to pbuf.  X1 and the TMEM
+// accumulator are double-buffered: MMA(k) runs while chunk k-1's accumulator is drained
+// to pbuf and chunk k+1 is staged.
 __global__ void __launch_bounds__(TNT, 2) k_tc_p(TcArgs a) {
   extern __shared__ __align__(128) char smem[];
-  float* x1h = reinterpret_cast<float*>(smem);
-  float* x1l = x1h + TCM / 4;
-  float* a1h = x1l + TCM / 4;
+  float* const xb = reinterpret_cast<float*>(smem);          // X1 buffer b: hi at xb + 2b*TCM/4
+  auto x1h = [&](int b) { return xb + (2 * b) * (TCM / 4); };
+  auto x1l = [&](int b) { return xb + (2 * b + 1) * (TCM / 4); };
+  float* a1h = xb + 4 * (TCM / 4);
   float* a1l = a1h + TCM / 4;
-  __shared__ uint64_t mbar;
+  __shared__ uint64_t mbar[2];
   __shared__ uint32_t s_tmem, s_g[2], s_rowp[2][64], s_rowa[2][64];
   const int tid = threadIdx.x, w = tid >> 5, lane = tid & 31, q4 = w & 3, half = w >> 2;
   if (tid == 0) {
-    tc::mbar_init(&mbar, 1);
+    tc::mbar_init(&mbar[0], 1);
+    tc::mbar_init(&mbar[1], 1);
     tc::fence_mbar_init();
     s_g[0] = atomicAdd(a.work, 1u);
     s_g[1] = atomicAdd(a.work, 1u);
   }
-  if (tid < 32) tc::tmem_alloc(&s_tmem, 64);
+  if (tid < 32) tc::tmem_alloc(&s_tmem, 128);
   tc::fence_before();
   __syncthreads();
   tc::fence_after();
-  const uint32_t tP = s_tmem;
-  uint32_t phase = 0;
+  const uint32_t tP0 = s_tmem;
+  uint32_t ph0 = 0u, ph1 = 0u;
   const uint32_t NG = a.counts[kCntNG];
   const int PPT = TMT >> a.n1s, NCH = a.NC / TCW;
   uint32_t g = s_g[0], gnext = s_g[1];
@@ -203,6 +208,24 @@ __global__ void __launch_bounds__(TNT, 2) k_tc_p(TcArgs a) {
     load_rowq(px, c2_slice(a, g), a.NC, TR);
     load_tab(pa, a.cores + a.meta[a.grp_t[g]].c1_off, TR, s_rowa[0], false);
   }
+  // drain the accumulator of chunk kc (buffer b) into pbuf rows of table tbl
+  auto drain = [&](int b, int kc, const uint32_t* tbl) {
+    tc::mbar_wait(&mbar[b], b == 0 ? ph0 : ph1);
+    if (b == 0) ph0 ^= 1u; else ph1 ^= 1u;
+    tc::fence_after();
+    float v[32];
+    tc::tmem_ld32(tc::taddr(tP0 + 64 * b, 32 * q4, 32 * half), v);
+    if (lane < 16) {
+      const uint32_t r = tbl[16 * q4 + lane];
+      if (r != 0xffffffffu) {
+        float* dst = a.pbuf + (size_t)r * a.NC + kc * TCW + 32 * half;
+#pragma unroll
+        for (int j = 0; j < 32; j += 4)
+          *reinterpret_cast<float4*>(dst + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
+      }
+    }
+    tc::fence_before();
+  };
   while (g < NG) {
     const uint32_t q0 = a.grp_off[g], q1 = a.grp_off[g + 1];
     const float* C2s = c2_slice(a, g);
@@ -211,8 +234,9 @@ __global__ void __launch_bounds__(TNT, 2) k_tc_p(TcArgs a) {
       __syncthreads();
       store_pat(a1h, a1l, pa);                              // A1 = CM(m, r1)
       for (int k = 0; k < NCH; ++k) {
-        if (k > 0) __syncthreads();
-        store_pat(x1h, x1l, px);                            // X1 = CM(c, r1)
+        const int b = k & 1;
+        __syncthreads();                                    // X1[b] readers (MMA k-2) drained below
+        store_pat(x1h(b), x1l(b), px);                      // X1 = CM(c, r1)
         if (k + 1 < NCH) {
           load_rowq(px, C2s + (k + 1) * TCW, a.NC, TR);
         } else {                                            // next tile (or group): table + prefetch
@@ -227,26 +251,13 @@ __global__ void __launch_bounds__(TNT, 2) k_tc_p(TcArgs a) {
         }
         publish();
         if (tid == 0) {
-          mma3(tP, a1h, a1l, x1h, x1l, false);
-          tc::commit(&mbar);
+          mma3(tP0 + 64 * b, a1h, a1l, x1h(b), x1l(b), false);
+          tc::commit(&mbar[b]);
         }
         __syncwarp();
-        tc::mbar_wait(&mbar, phase);
-        phase ^= 1u;
-        tc::fence_after();
-        float v[32];
-        tc::tmem_ld32(tc::taddr(tP, 32 * q4, 32 * half), v);
-        if (lane < 16) {
-          const uint32_t r = s_rowp[tb][16 * q4 + lane];
-          if (r != 0xffffffffu) {
-            float* dst = a.pbuf + (size_t)r * a.NC + k * TCW + 32 * half;
-#pragma unroll
-            for (int j = 0; j < 32; j += 4)
-              *reinterpret_cast<float4*>(dst + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
-          }
-        }
-        tc::fence_before();
+        if (k > 0) drain(b ^ 1, k - 1, s_rowp[tb]);        // overlaps MMA(k)
       }
+      drain((NCH - 1) & 1, NCH - 1, s_rowp[tb]);
       tb ^= 1;
     }
     __syncthreads();
@@ -258,7 +269,7 @@ __global__ void __launch_bounds__(TNT, 2) k_tc_p(TcArgs a) {
   tc::fence_before();
   __syncthreads();
   tc::fence_after();
-  if (tid < 32) tc::tmem_dealloc(tP, 64);
+  if (tid < 32) tc::tmem_dealloc(tP0, 128);
 }
 
 // ------------------------------------------------------------------------------------
@@ -480,20 +491,29 @@ __global__ void __launch_bounds__(128) k_rows_bwd(TcArgs a) {
   }
 }
 
-// ------------------------------------------------------------------------------------
 // Backward GEMMs per i2-group: dA^T = X2 . D1^T (TMEM, accumulated over chunks) and
-// dC2[chunk] += A2 . D2^T (TMEM, accumulated over m-tiles)
-// ------------------------------------------------------------------------------------
+// dC2[chunk] += A2 . D2^T (TMEM, accumulated over m-tiles).  X2 / D1 / D2 are
+// double-buffered so MMA(k) overlaps the staging of chunk k+1; in the group's last m-tile
+// the finished dC2 chunk k-2 is applied (fused update) from the staged X2 copy
+// (C2 = X2_hi + X2_lo exactly) before its buffer is reused.
 __global__ void __launch_bounds__(TNT, 1) k_tc_bwd2(TcArgs a) {
   extern __shared__ __align__(128) char smem[];
-  float* base = reinterpret_cast<float*>(smem);
-  float *x2h = base, *x2l = x2h + TCM / 4, *a2h = x2l + TCM / 4, *a2l = a2h + TCM / 4;
-  float *d1h = a2l + TCM / 4, *d1l = d1h + TCM / 4, *d2h = d1l + TCM / 4, *d2l = d2h + TCM / 4;
-  __shared__ uint64_t mbar;
+  float* const base = reinterpret_cast<float*>(smem);     // buffer b: 6 matrices at base + 6b*TCM/4
+  constexpr int MF = TCM / 4;
+  auto x2h = [&](int b) { return base + (6 * b + 0) * MF; };
+  auto x2l = [&](int b) { return base + (6 * b + 1) * MF; };
+  auto d1h = [&](int b) { return base + (6 * b + 2) * MF; };
+  auto d1l = [&](int b) { return base + (6 * b + 3) * MF; };
+  auto d2h = [&](int b) { return base + (6 * b + 4) * MF; };
+  auto d2l = [&](int b) { return base + (6 * b + 5) * MF; };
+  float* a2h = base + 12 * MF;
+  float* a2l = base + 13 * MF;
+  __shared__ uint64_t mbar[2];
   __shared__ uint32_t s_tmem, s_g[2], s_rowp[2][64], s_rowa[2][64];
   const int tid = threadIdx.x, w = tid >> 5, lane = tid & 31, q4 = w & 3, half = w >> 2;
   if (tid == 0) {
-    tc::mbar_init(&mbar, 1);
+    tc::mbar_init(&mbar[0], 1);
+    tc::mbar_init(&mbar[1], 1);
     tc::fence_mbar_init();
     s_g[0] = atomicAdd(a.work, 1u);
     s_g[1] = atomicAdd(a.work, 1u);
@@ -503,7 +523,8 @@ __global__ void __launch_bounds__(TNT, 1) k_tc_bwd2(TcArgs a) {
   __syncthreads();
   tc::fence_after();
   const uint32_t tDA = s_tmem, tDC2 = s_tmem + 64;
-  uint32_t phase = 0;
+  uint32_t ph0 = 0u, ph1 = 0u;
+  int pend0 = 0, pend1 = 0;
   const uint32_t NG = a.counts[kCntNG];
   const int PPT = TMT >> a.n1s, NCH = a.NC / TCW;
   uint32_t g = s_g[0], gnext = s_g[1];
@@ -517,6 +538,55 @@ __global__ void __launch_bounds__(TNT, 1) k_tc_bwd2(TcArgs a) {
     load_tab(pd2, a.dpbuf, a.NC, s_rowp[0], true);
     load_tab(pa, a.cores + a.meta[a.grp_t[g]].c1_off, TR, s_rowa[0], true);
   }
+  auto wait_buf = [&](int b) {
+    if (b == 0 ? pend0 : pend1) {
+      tc::mbar_wait(&mbar[b], b == 0 ? ph0 : ph1);
+      if (b == 0) { ph0 ^= 1u; pend0 = 0; } else { ph1 ^= 1u; pend1 = 0; }
+      tc::fence_after();
+    }
+  };
+  // final dC2 of chunk kc (MMAs done): gradient or fused update, C2 read from X2[b]
+  auto finish_chunk = [&](int kc, int b, size_t c2o) {
+    float v[32];
+    tc::tmem_ld32(tc::taddr(tDC2 + 64 * kc, 32 * q4, 32 * half), v);
+    if (lane < 16) {
+      const int r1 = 16 * q4 + lane;
+      const size_t b0 = c2o + (size_t)r1 * a.NC + kc * TCW + 32 * half;
+      if (a.fused) {
+        float x[32];
+#pragma unroll
+        for (int j = 0; j < 32; j += 4) {
+          const uint32_t off = tc::cm_off(r1, 32 * half + j, TNRB);
+          const float4 h = *reinterpret_cast<const float4*>(fat(x2h(b), off));
+          const float4 l = *reinterpret_cast<const float4*>(fat(x2l(b), off));
+          x[j] = h.x + l.x; x[j + 1] = h.y + l.y; x[j + 2] = h.z + l.z; x[j + 3] = h.w + l.w;
+        }
+        if (a.opt == TTEMB_SGD) {
+#pragma unroll
+          for (int j = 0; j < 32; j += 4)
+            *reinterpret_cast<float4*>(a.cores + b0 + j) =
+                make_float4(x[j] - a.lr * v[j], x[j + 1] - a.lr * v[j + 1], x[j + 2] - a.lr * v[j + 2],
+                            x[j + 3] - a.lr * v[j + 3]);
+        } else {
+#pragma unroll
+          for (int j = 0; j < 32; j += 4) {
+            const float4 s4 = *reinterpret_cast<const float4*>(a.state + b0 + j);
+            const float s0 = s4.x + v[j] * v[j], s1 = s4.y + v[j + 1] * v[j + 1];
+            const float s2 = s4.z + v[j + 2] * v[j + 2], s3 = s4.w + v[j + 3] * v[j + 3];
+            *reinterpret_cast<float4*>(a.state + b0 + j) = make_float4(s0, s1, s2, s3);
+            *reinterpret_cast<float4*>(a.cores + b0 + j) =
+                make_float4(x[j] - a.lr * v[j] / (sqrtf(s0) + a.eps), x[j + 1] - a.lr * v[j + 1] / (sqrtf(s1) + a.eps),
+                            x[j + 2] - a.lr * v[j + 2] / (sqrtf(s2) + a.eps), x[j + 3] - a.lr * v[j + 3] / (sqrtf(s3) + a.eps));
+          }
+        }
+      } else {
+#pragma unroll
+        for (int j = 0; j < 32; j += 4)
+          *reinterpret_cast<float4*>(a.grads + b0 + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
+      }
+    }
+    tc::fence_before();
+  };
   while (g < NG) {
     const uint32_t i2 = a.grp_i2[g];
     const uint32_t q0 = a.grp_off[g], q1 = a.grp_off[g + 1];
@@ -524,13 +594,19 @@ __global__ void __launch_bounds__(TNT, 1) k_tc_bwd2(TcArgs a) {
     const float* C2s = a.cores + c2o;
     const uint32_t nmt = (q1 - q0 + PPT - 1) / PPT;
     for (uint32_t mt = 0; mt < nmt; ++mt) {
+      const bool last_tile = (mt + 1 == nmt);
+      wait_buf(0);
+      wait_buf(1);
       __syncthreads();
       store_pat(a2h, a2l, pa);                               // A2 = CM(r1, m)
       for (int k = 0; k < NCH; ++k) {
-        if (k > 0) __syncthreads();
-        store_pat(x2h, x2l, px);                             // X2 = CM(r1, c)
-        store_pat(d1h, d1l, pd1);                            // D1 = CM(m, c)
-        store_pat(d2h, d2l, pd2);                            // D2 = CM(c, m)
+        const int b = k & 1;
+        wait_buf(b);                                         // MMA(k-2) done: buffer b free
+        if (last_tile && k >= 2) finish_chunk(k - 2, b, c2o);
+        __syncthreads();
+        store_pat(x2h(b), x2l(b), px);                       // X2 = CM(r1, c)
+        store_pat(d1h(b), d1l(b), pd1);                      // D1 = CM(m, c)
+        store_pat(d2h(b), d2l(b), pd2);                      // D2 = CM(c, m)
         if (k + 1 < NCH) {
           load_colq(px, C2s + (k + 1) * TCW, a.NC, TR);
           load_tab(pd1, a.dpbuf + (k + 1) * TCW, a.NC, s_rowp[tb], false);
@@ -549,14 +625,16 @@ __global__ void __launch_bounds__(TNT, 1) k_tc_bwd2(TcArgs a) {
         }
         publish();
         if (tid == 0) {
-          mma3(tDA, x2h, x2l, d1h, d1l, k > 0);              // dA^T [r1][m]
-          mma3(tDC2 + 64 * k, a2h, a2l, d2h, d2l, mt > 0);   // dC2  [r1][c]
-          tc::commit(&mbar);
+          mma3(tDA, x2h(b), x2l(b), d1h(b), d1l(b), k > 0);          // dA^T [r1][m]
+          mma3(tDC2 + 64 * k, a2h, a2l, d2h(b), d2l(b), mt > 0);      // dC2  [r1][c]
+          tc::commit(&mbar[b]);
         }
         __syncwarp();
-        tc::mbar_wait(&mbar, phase);
-        phase ^= 1u;
-        tc::fence_after();
+        if (b == 0) pend0 = 1; else pend1 = 1;
+      }
+      for (int kc = (NCH >= 2 ? NCH - 2 : 0); kc < NCH; ++kc) {   // drain the last two chunks
+        wait_buf(kc & 1);
+        if (last_tile) finish_chunk(kc, kc & 1, c2o);
       }
       {   // dA^T -> dabuf[(p, j1)][r1]
         float v[32];
@@ -573,38 +651,6 @@ __global__ void __launch_bounds__(TNT, 1) k_tc_bwd2(TcArgs a) {
       }
       tb ^= 1;
     }
-    for (int k = 0; k < NCH; ++k) {   // this CTA owns C2[t][i2]: gradient or fused update
-      float v[32];
-      tc::tmem_ld32(tc::taddr(tDC2 + 64 * k, 32 * q4, 32 * half), v);
-      if (lane < 16) {
-        const int r1 = 16 * q4 + lane;
-        const size_t b0 = c2o + (size_t)r1 * a.NC + k * TCW + 32 * half;
-        if (a.fused) {
-          if (a.opt == TTEMB_SGD) {
-            float4 x[8];
-#pragma unroll
-            for (int j = 0; j < 8; ++j) x[j] = *reinterpret_cast<const float4*>(a.cores + b0 + 4 * j);
-#pragma unroll
-            for (int j = 0; j < 8; ++j)
-              *reinterpret_cast<float4*>(a.cores + b0 + 4 * j) =
-                  make_float4(x[j].x - a.lr * v[4 * j], x[j].y - a.lr * v[4 * j + 1],
-                              x[j].z - a.lr * v[4 * j + 2], x[j].w - a.lr * v[4 * j + 3]);
-          } else {
-#pragma unroll
-            for (int j = 0; j < 32; ++j) {
-              const float sv = a.state[b0 + j] + v[j] * v[j];
-              a.state[b0 + j] = sv;
-              a.cores[b0 + j] = a.cores[b0 + j] - a.lr * v[j] / (sqrtf(sv) + a.eps);
-            }
-          }
-        } else {
-#pragma unroll
-          for (int j = 0; j < 32; j += 4)
-            *reinterpret_cast<float4*>(a.grads + b0 + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
-        }
-      }
-    }
-    tc::fence_before();
     __syncthreads();
     if (tid == 0) s_g[1] = atomicAdd(a.work, 1u);
     __syncthreads();
@@ -632,8 +678,8 @@ TcArgs make_tc_args(Ctx& c, float lr, uint32_t* work, float* out) {
   return a;
 }
 
-constexpr size_t kTcPSmem = 4 * TCM;
-constexpr size_t kTcBwdSmem = 8 * TCM;
+constexpr size_t kTcPSmem = 6 * TCM;
+constexpr size_t kTcBwdSmem = 14 * TCM;
 
 }  // namespace
 
