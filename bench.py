@@ -36,8 +36,9 @@ def load_peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
         d = json.load(open(p))
-        return float(d.get("hbm_gbs", HBM_PEAK_FALLBACK)), float(d.get("sm_max_mhz", 1965.0)), "measured"
-    return HBM_PEAK_FALLBACK, 1965.0, "fallback"
+        return (float(d.get("hbm_gbs", HBM_PEAK_FALLBACK)), float(d.get("sm_max_mhz", 1965.0)),
+                float(d.get("bf16_tflops", 1590.0)), "measured")
+    return HBM_PEAK_FALLBACK, 1965.0, 1590.0, "fallback"
 
 
 def fp32_peak_tflops(sm_count: int, mhz: float) -> float:
@@ -110,15 +111,16 @@ def step_work(cfg, B, nnz, counts, touched, opt):
     return flops, bytes_
 
 
-def stage_work(name, cfg, B, nnz, counts):
-    """(flops, bytes, bound) of one launch of a stage, algorithmic."""
+def stage_work(name, cfg, B, nnz, counts, tc=False):
+    """(flops, bytes, bound) of one launch of a stage, algorithmic.  On the tcgen05 path the
+    rank-R contractions are bound by the tensor pipe ("tensor"), else by FP32 FFMA ("alu")."""
     n1, n2, n3 = cfg.col_factors
     R, N, T = cfg.rank, cfg.dim, cfg.num_tables
     U, P, NG = counts["U"], counts["P"], counts["NG"]
     if name == "fwd_prefix":
-        return 2 * n1 * n2 * R * R * P, 4 * (NG * R * n2 * R + P * n1 * R), "alu"
+        return 2 * n1 * n2 * R * R * P, 4 * (NG * R * n2 * R + P * n1 * R), "tensor" if tc else "alu"
     if name == "bwd_prefix":
-        return 4 * n1 * n2 * R * R * P, 4 * (2 * NG * R * n2 * R + P * n1 * R), "alu"
+        return 4 * n1 * n2 * R * R * P, 4 * (2 * NG * R * n2 * R + P * n1 * R), "tensor" if tc else "alu"
     if name == "fwd_rows":
         return 2 * N * R * U, 4 * U * N, "alu"
     if name == "bwd_rows":
@@ -229,14 +231,16 @@ def workload_config(cfg, B, world, args):
 # ---------------------------------------------------------------------------
 # our arm
 # ---------------------------------------------------------------------------
-def kernels_per_step(emb_ctx, world):
-    """Our kernel launches per step (memsets excluded): see DESIGN.md."""
+def kernels_per_step(emb_ctx, world, tc=True):
+    """Our kernel launches per step (cudaMemsetAsync excluded), matching the ncu launch list:
+    index stage = build_keys + hist_scan + kp passes + unique + prefix + (radix_hist +
+    hist_scan) + gp passes + groups; forward = contraction kernels + pool; backward = agg,
+    agg_fix, contraction kernels, dc1, dc1_fix (+ update_c3 fused / update after all-reduce)."""
     kp, gp = emb_ctx
-    idx_stage = 1 + 2 + kp + 1 + 1 + 2 + gp + 1
-    fwd = 3
-    bwd = 5 + (1 if world == 1 else 0)
-    upd = 0 if world == 1 else 1
-    return idx_stage + fwd + bwd + upd
+    idx_stage = 1 + 1 + kp + 1 + 1 + 2 + gp + 1
+    fwd = (2 if tc else 1) + 1
+    bwd = 2 + (3 if tc else 1) + 2 + 1
+    return idx_stage + fwd + bwd
 
 
 def main():
@@ -256,6 +260,7 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--stages", action="store_true", help="print per-stage times to stderr")
+    ap.add_argument("--fp32-cores", action="store_true", help="force the FFMA contraction path (no tcgen05)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
@@ -277,6 +282,7 @@ def main():
     import torch
     import torch.distributed as dist
     import paper_conf_sc_wangwfmmd22_b200 as tt
+    from paper_conf_sc_wangwfmmd22_b200 import parallel
 
     torch.cuda.set_device(local_rank)
     dev = torch.device("cuda", local_rank)
@@ -293,12 +299,13 @@ def main():
             go = W.make_grad_out(cfg, B, step=i, seed=args.seed + 1000 * rank)
         else:
             gi, goff = W.make_batch(cfg, step=i, seed=args.seed)
-            idx, off, _ = W.shard_batch(gi, goff, cfg.num_tables, cfg.batch, rank, world)
+            idx, off, _ = parallel.shard_bags(gi, goff, cfg.num_tables, cfg.batch, rank, world)
             go = W.make_grad_out(cfg, cfg.batch, step=i, seed=args.seed)[rank * B:(rank + 1) * B].copy()
         pool.append((idx, off, go))
     max_nnz = max(len(p[0]) for p in pool)
     emb = tt.TTEmbeddingBag(cfg.table_rows, cfg.row_factors, cfg.col_factors, cfg.rank, B, max_nnz,
-                            optimizer=args.opt, fused_update=fused, device=local_rank)
+                            optimizer=args.opt, fused_update=fused, device=local_rank,
+                            fp32_cores=args.fp32_cores)
     cores = W.make_cores(cfg, seed=args.seed)
     emb.load_cores(cores)
     dpool = [(torch.as_tensor(i, device=dev), torch.as_tensor(o, device=dev), torch.as_tensor(g, device=dev))
@@ -312,7 +319,7 @@ def main():
         emb.forward(di, do, B, out=out)
         emb.backward(dg, lr=args.lr)
         if world > 1:
-            dist.all_reduce(emb.grads)
+            parallel.allreduce_grads(emb.grads)
             emb.update(args.lr)
 
     for i in range(args.warmup):
@@ -357,7 +364,8 @@ def main():
     rt = pt[plan["row_pfx"].cpu().numpy().astype(np.int64)]
     touched = {"c1": len(np.unique(pt * (1 << 32) + pi1)), "c2": counts["NG"],
                "c3": len(np.unique(rt * (1 << 32) + ri3))}
-    hbm_peak, sm_max_mhz, peak_kind = load_peaks()
+    hbm_peak, sm_max_mhz, bf16_peak, peak_kind = load_peaks()
+    on_tc = tc_path(cfg, args)
     sm_count = torch.cuda.get_device_properties(dev).multi_processor_count
     alu_peak = fp32_peak_tflops(sm_count, sm_max_mhz)
     flops, bytes_ = step_work(cfg, B, nnz_last, counts, touched, args.opt)
@@ -365,9 +373,17 @@ def main():
     # dominant stage
     dom = max(stages.items(), key=lambda kv: kv[1][0])
     dname, (dms, dn) = dom
-    f1, b1, bound = stage_work(dname, cfg, B, nnz_last, counts)
+    f1, b1, bound = stage_work(dname, cfg, B, nnz_last, counts, tc=on_tc)
     per_launch_ms = dms / max(dn, 1)
-    if bound == "alu":
+    if bound == "tensor":
+        # 3xTF32: each fp32 product costs 3 TF32 MMAs; TF32 dense = bf16 / 2 (nominal ratio)
+        tpk = bf16_peak / 2.0 / 3.0
+        ach = f1 / (per_launch_ms / 1e3) / 1e12
+        roof = {"bound": "tensor", "kernel": dname, "achieved": ach, "peak": tpk, "unit": "TFLOP/s",
+                "frac": ach / tpk, "traffic": None,
+                "peak_source": f"{peak_kind} bf16 {bf16_peak:.0f} TFLOP/s x 1/2 (tf32) x 1/3 (3xTF32), "
+                               "fp32-equivalent algorithmic FLOPs"}
+    elif bound == "alu":
         ach = f1 / (per_launch_ms / 1e3) / 1e12
         roof = {"bound": "alu", "kernel": dname, "achieved": ach, "peak": alu_peak, "unit": "TFLOP/s",
                 "frac": ach / alu_peak, "traffic": None,
@@ -428,12 +444,18 @@ def main():
                 "scaling": args.scaling, "vs_baseline": None, "dtype": "f32", "data": "synthetic",
                 "config": workload_config(cfg, B, world, args), "roofline": roof,
                 "step_roofline": step_roof, "cpu_baseline": cpu, "e2e": e2e,
-                "gpu_launches": kernels_per_step((emb_passes(emb)), world) * args.steps,
+                "gpu_launches": kernels_per_step(emb_passes(emb), world, tc=tc_path(cfg, args)) * args.steps,
                 "clocks": clk.summary(),
                 "stages_us_per_step": {k: round(v[0] / args.steps * 1e3, 2) for k, v in stages.items() if v[1]}}
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
+
+
+def tc_path(cfg, args):
+    n1, n2, n3 = cfg.col_factors
+    return (not args.fp32_cores) and cfg.rank == 64 and n3 in (4, 8) and n1 in (1, 2, 4, 8) \
+        and n1 * n2 <= 16 and n2 <= 7
 
 
 def emb_passes(emb):

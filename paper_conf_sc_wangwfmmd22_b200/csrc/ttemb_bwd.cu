@@ -40,11 +40,10 @@ k_agg(const float* __restrict__ grad_out, const uint32_t* __restrict__ skey,
       int N, float* __restrict__ gbuf, float* __restrict__ part) {
   using V = typename std::conditional<VW == 4, float4, float>::type;
   const int NV = N / VW;
-  const int64_t nchunks = (nnz + AGG_CS - 1) / AGG_CS;
-  const int64_t total = nchunks * NV;
-  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < total;
-       e += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t ch = e / NV;
+  const uint32_t nchunks = (uint32_t)((nnz + AGG_CS - 1) / AGG_CS);
+  const uint32_t total = nchunks * NV;
+  for (uint32_t e = blockIdx.x * blockDim.x + threadIdx.x; e < total; e += gridDim.x * blockDim.x) {
+    const uint32_t ch = e / NV;
     const int col = (int)(e - ch * NV) * VW;
     const int64_t k0 = ch * AGG_CS, k1 = min(k0 + AGG_CS, nnz);
     V acc = V{};
@@ -68,7 +67,9 @@ k_agg(const float* __restrict__ grad_out, const uint32_t* __restrict__ skey,
 }
 
 // a8 part 2: a row whose segment spans chunks c0..c1 is finished by the warp of chunk c1
-// (the chunk where it ends): G = tail(c0) + heads(c0+1..c1), lanes over columns.
+// (the chunk where it ends): G = tail(c0) + heads(c0+1..c1).  Lanes split the chunk range
+// (fixed strided partition + butterfly), so Zipf-hot rows spanning hundreds of chunks
+// stay cheap; the summation order is fixed, hence deterministic.
 __global__ void __launch_bounds__(256)
 k_agg_fix(const uint32_t* __restrict__ skey, const uint32_t* __restrict__ spos,
           const uint32_t* __restrict__ inverse, const uint32_t* __restrict__ seg_off, int64_t nnz,
@@ -83,10 +84,38 @@ k_agg_fix(const uint32_t* __restrict__ skey, const uint32_t* __restrict__ spos,
     const uint32_t u = inverse[spos[k]];
     const int64_t c0 = seg_off[u] / AGG_CS, c1 = (seg_off[u + 1] - 1) / AGG_CS;
     if (c1 != ch) continue;                                // not the segment's last chunk
-    for (int col = lane; col < N; col += 32) {
-      float acc = part[((size_t)c0 * 2 + 1) * N + col];
-      for (int64_t c = c0 + 1; c <= c1; ++c) acc += part[((size_t)c * 2 + 0) * N + col];
-      gbuf[(size_t)u * N + col] = acc;
+    // G = tail(c0) + heads(c0+1 .. c1).  N % 4 == 0: lanes = (float4 column group cq < 16,
+    // half h of the chunk range); 4 independent accumulators each; one shuffle joins halves.
+    if ((N & 3) == 0) {
+      const int cq = lane & 15, h = lane >> 4;
+      for (int c4 = cq; c4 < N / 4; c4 += 16) {
+        float4 acc[4];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) acc[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (h == 0) acc[0] = *reinterpret_cast<const float4*>(part + ((size_t)c0 * 2 + 1) * N + 4 * c4);
+        int64_t c = c0 + 1 + h;
+        int i = 0;
+        for (; c <= c1; c += 2, i = (i + 1) & 3) {
+          const float4 v = *reinterpret_cast<const float4*>(part + ((size_t)c * 2) * N + 4 * c4);
+          acc[i].x += v.x; acc[i].y += v.y; acc[i].z += v.z; acc[i].w += v.w;
+        }
+        float4 r;
+        r.x = (acc[0].x + acc[1].x) + (acc[2].x + acc[3].x);
+        r.y = (acc[0].y + acc[1].y) + (acc[2].y + acc[3].y);
+        r.z = (acc[0].z + acc[1].z) + (acc[2].z + acc[3].z);
+        r.w = (acc[0].w + acc[1].w) + (acc[2].w + acc[3].w);
+        r.x += __shfl_xor_sync(0xffffffffu, r.x, 16);
+        r.y += __shfl_xor_sync(0xffffffffu, r.y, 16);
+        r.z += __shfl_xor_sync(0xffffffffu, r.z, 16);
+        r.w += __shfl_xor_sync(0xffffffffu, r.w, 16);
+        if (h == 0) *reinterpret_cast<float4*>(gbuf + (size_t)u * N + 4 * c4) = r;
+      }
+    } else {
+      for (int col = lane; col < N; col += 32) {
+        float acc = part[((size_t)c0 * 2 + 1) * N + col];
+        for (int64_t c = c0 + 1; c <= c1; ++c) acc += part[((size_t)c * 2) * N + col];
+        gbuf[(size_t)u * N + col] = acc;
+      }
     }
   }
 }
@@ -166,6 +195,7 @@ __global__ void __launch_bounds__(256) k_dc1_fix(BwdArgs a, const float* __restr
            same_run(a, (uint32_t)(c0 * DC1_CS), (uint32_t)(c0 * DC1_CS) - 1))
       --c0;
     float g = part[((size_t)c0 * 2 + 1) * S1 + k];
+#pragma unroll 8
     for (int64_t c = c0 + 1; c <= ch; ++c) g += part[((size_t)c * 2 + 0) * S1 + k];
     dc1_finish(a, p0, k, g);
   }
@@ -201,16 +231,16 @@ cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s
     StageScope sc(c, ST_AGG, s);
     const int64_t total = agg_chunks(c.nnz) * c.N;
     if (c.N % 4 == 0)
-      k_agg<4><<<grid_for(c, total / 4, 256, 8), 256, 0, s>>>(grad_out, p.skey, p.sbag, p.spos,
+      k_agg<4><<<grid_for(c, total / 4, 256, 32), 256, 0, s>>>(grad_out, p.skey, p.sbag, p.spos,
                                                               p.inverse, p.seg_off, c.nnz, c.N,
                                                               p.gbuf, p.aggpart);
     else
-      k_agg<1><<<grid_for(c, total, 256, 8), 256, 0, s>>>(grad_out, p.skey, p.sbag, p.spos, p.inverse,
+      k_agg<1><<<grid_for(c, total, 256, 32), 256, 0, s>>>(grad_out, p.skey, p.sbag, p.spos, p.inverse,
                                                           p.seg_off, c.nnz, c.N, p.gbuf, p.aggpart);
   }
   if (c.nnz > 0) {
     StageScope sc(c, ST_AGG_FIX, s);
-    k_agg_fix<<<grid_for(c, agg_chunks(c.nnz) * 32, 256, 8), 256, 0, s>>>(
+    k_agg_fix<<<grid_for(c, agg_chunks(c.nnz) * 32, 256, 32), 256, 0, s>>>(
         p.skey, p.spos, p.inverse, p.seg_off, c.nnz, c.N, p.aggpart, p.gbuf);
   }
   BwdArgs a;
@@ -226,13 +256,13 @@ cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s
     {
       StageScope sc(c, ST_DC1, s);
       const int64_t items = cdiv(c.P_cap, DC1_CS) * c.n1 * c.R;
-      k_dc1<<<grid_for(c, items, 256, 8), 256, 0, s>>>(a, p.aggpart);
-      k_dc1_fix<<<grid_for(c, items, 256, 8), 256, 0, s>>>(a, p.aggpart);
+      k_dc1<<<grid_for(c, items, 256, 32), 256, 0, s>>>(a, p.aggpart);
+      k_dc1_fix<<<grid_for(c, items, 256, 32), 256, 0, s>>>(a, p.aggpart);
     }
   }
   if (fused) {
     StageScope sc(c, ST_UPD_C3, s);
-    k_update<<<grid_for(c, (int64_t)c.c3_floats, 256, 8), 256, 0, s>>>(
+    k_update<<<grid_for(c, (int64_t)c.c3_floats, 256, 32), 256, 0, s>>>(
         c.cores, c.state, c.grads, c.c3_begin, c.c3_floats, lr, c.eps, c.opt);
   }
   return cudaGetLastError();
@@ -240,7 +270,7 @@ cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s
 
 cudaError_t run_update(Ctx& c, float lr, cudaStream_t s) {
   StageScope sc(c, ST_UPDATE, s);
-  k_update<<<grid_for(c, (int64_t)c.core_floats, 256, 8), 256, 0, s>>>(
+  k_update<<<grid_for(c, (int64_t)c.core_floats, 256, 32), 256, 0, s>>>(
       c.cores, c.state, c.grads, 0, c.core_floats, lr, c.eps, c.opt);
   return cudaGetLastError();
 }

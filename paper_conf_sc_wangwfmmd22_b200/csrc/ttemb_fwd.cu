@@ -9,6 +9,8 @@
 //   a7 sum pooling out[b][t] = sum_{j in bag} E_{inverse[j]}     (Eq. 4, P:164 step 4)
 // FP32 FFMA on CUDA cores (tensor cores only where ncu shows the rank-R
 // contraction is the bottleneck).
+#include <type_traits>
+
 #include "ttemb_internal.cuh"
 
 namespace ttemb {
@@ -16,36 +18,49 @@ namespace ttemb {
 namespace {
 
 // a7: out[b][t][:] = sum over the bag's positions (index order); empty bag -> 0.
-// Thread = (bag, VW-wide column group); VW = 4 when N % 4 == 0 (float4 traffic).
+// Thread = (bag, VW-wide column group); 4 independent items per thread are processed
+// together so their index -> row loads overlap.
 template <int VW>
 __global__ void __launch_bounds__(256)
 k_pool(const float* __restrict__ rows, const uint32_t* __restrict__ inverse,
        const int64_t* __restrict__ offsets, int64_t nnz, int T, int B, int N, float* __restrict__ out,
        const uint32_t* __restrict__ counts, int skip_single) {
   if (skip_single && counts[kCntMulti] == 0) return;   // one id per bag: written directly
-  const int NV = N / VW;
-  const int64_t total = (int64_t)T * B * NV;
-  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < total;
-       e += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t bag = e / NV;
-    const int col = (int)(e - bag * NV) * VW;
-    const int t = (int)(bag / B);
-    const int64_t b = bag - (int64_t)t * B;
-    int64_t s = __ldg(offsets + bag), f = __ldg(offsets + bag + 1);
-    s = s < 0 ? 0 : (s > nnz ? nnz : s);
-    f = f < s ? s : (f > nnz ? nnz : f);
-    float* dst = out + ((size_t)b * T + t) * N + col;
-    if constexpr (VW == 4) {
-      float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
-      for (int64_t j = s; j < f; ++j) {
-        const float4 v = __ldg(reinterpret_cast<const float4*>(rows + (size_t)__ldg(inverse + j) * N + col));
-        acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
+  using V = typename std::conditional<VW == 4, float4, float>::type;
+  const uint32_t NV = (uint32_t)(N / VW);
+  const uint32_t total = (uint32_t)T * (uint32_t)B * NV;
+  const uint32_t stride = gridDim.x * blockDim.x;
+  for (uint32_t e0 = blockIdx.x * blockDim.x + threadIdx.x; e0 < total; e0 += 4 * stride) {
+    int64_t s[4], f[4];
+    uint32_t bag[4], col[4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const uint32_t e = e0 + i * stride;
+      bag[i] = e / NV;
+      col[i] = (e - bag[i] * NV) * VW;
+      s[i] = f[i] = 0;
+      if (e < total) {
+        s[i] = __ldg(offsets + bag[i]);
+        f[i] = __ldg(offsets + bag[i] + 1);
+        s[i] = s[i] < 0 ? 0 : (s[i] > nnz ? nnz : s[i]);
+        f[i] = f[i] < s[i] ? s[i] : (f[i] > nnz ? nnz : f[i]);
       }
-      *reinterpret_cast<float4*>(dst) = acc;
-    } else {
-      float acc = 0.f;
-      for (int64_t j = s; j < f; ++j) acc += __ldg(rows + (size_t)__ldg(inverse + j) * N + col);
-      *dst = acc;
+    }
+    V acc[4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      acc[i] = V{};
+      for (int64_t j = s[i]; j < f[i]; ++j) {
+        const V v = __ldg(reinterpret_cast<const V*>(rows + (size_t)__ldg(inverse + j) * N + col[i]));
+        if constexpr (VW == 4) { acc[i].x += v.x; acc[i].y += v.y; acc[i].z += v.z; acc[i].w += v.w; }
+        else acc[i] += v;
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      if (e0 + i * stride >= total) continue;
+      const uint32_t t = bag[i] / (uint32_t)B, b = bag[i] - t * (uint32_t)B;
+      *reinterpret_cast<V*>(out + ((size_t)b * T + t) * N + col[i]) = acc[i];
     }
   }
 }
@@ -66,10 +81,10 @@ cudaError_t run_forward_compute(Ctx& c, float* out, const int64_t* offsets, cuda
     const int64_t total = (int64_t)c.T * c.B * c.N;
     if (total > 0) {
       if (c.N % 4 == 0)
-        k_pool<4><<<grid_for(c, total / 4, 256, 8), 256, 0, s>>>(p.rows, p.inverse, offsets, c.nnz,
+        k_pool<4><<<grid_for(c, total / 16, 256, 32), 256, 0, s>>>(p.rows, p.inverse, offsets, c.nnz,
                                                                  c.T, c.B, c.N, out, p.counts, 0);
       else
-        k_pool<1><<<grid_for(c, total, 256, 8), 256, 0, s>>>(p.rows, p.inverse, offsets, c.nnz, c.T,
+        k_pool<1><<<grid_for(c, total / 4, 256, 32), 256, 0, s>>>(p.rows, p.inverse, offsets, c.nnz, c.T,
                                                              c.B, c.N, out, p.counts, 0);
     }
   }

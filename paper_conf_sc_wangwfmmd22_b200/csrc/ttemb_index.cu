@@ -35,13 +35,13 @@ __device__ __forceinline__ void st_release(uint32_t* p, uint32_t v) {
   asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
 
-// Decoupled look-back: publish `agg` for tile `tile` in status[tile*stride], walk back
-// over predecessors in windows of 8 independent acquire loads (so a walk over many
-// not-yet-inclusive predecessors costs ~n/8 round trips), publish the inclusive prefix,
-// return the exclusive prefix.
+// Decoupled look-back (one thread per status word): publish `agg` for tile `tile` in
+// status[tile*stride], walk back over predecessors in windows of W independent acquire
+// loads, publish the inclusive prefix, return the exclusive prefix.  When all tiles run
+// concurrently the inclusive prefixes propagate ~W tiles per round trip.
+template <int W>
 __device__ __forceinline__ uint32_t lookback(uint32_t* status, size_t stride, uint32_t tile,
                                              uint32_t agg) {
-  constexpr int W = 8;
   uint32_t* me = status + (size_t)tile * stride;
   if (tile == 0) {
     st_release(me, kFlagPfx | agg);
@@ -67,6 +67,36 @@ __device__ __forceinline__ uint32_t lookback(uint32_t* status, size_t stride, ui
     j -= W;
   }
   st_release(me, kFlagPfx | (excl + agg));
+  return excl;
+}
+
+// Warp-wide look-back for a single status word per tile (call with the whole warp):
+// each round reads 32 predecessors in parallel.
+__device__ __forceinline__ uint32_t lookback_warp(uint32_t* status, uint32_t tile, uint32_t agg) {
+  const int lane = threadIdx.x & 31;
+  if (tile == 0) {
+    if (lane == 0) st_release(status, kFlagPfx | agg);
+    return 0;
+  }
+  if (lane == 0) st_release(status + tile, kFlagAgg | agg);
+  uint32_t excl = 0;
+  int64_t j = (int64_t)tile - 1;
+  for (;;) {
+    const int64_t idx = j - lane;
+    uint32_t v = idx >= 0 ? ld_acquire(status + idx) : kFlagPfx;
+    while (__any_sync(FULL, (v >> 30) == 0)) {
+      if ((v >> 30) == 0) v = ld_acquire(status + idx);
+    }
+    const uint32_t pfx = __ballot_sync(FULL, (v & kFlagPfx) != 0);
+    const int stop = pfx ? __ffs(pfx) - 1 : 31;          // nearest inclusive prefix
+    uint32_t x = lane <= stop ? (v & kValMask) : 0u;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(FULL, x, o);
+    excl += x;
+    if (pfx) break;
+    j -= 32;
+  }
+  if (lane == 0) st_release(status + tile, kFlagPfx | (excl + agg));
   return excl;
 }
 
@@ -100,42 +130,50 @@ __device__ __forceinline__ uint32_t block_excl_scan_256(uint32_t v, uint32_t* s_
 // ------------------------------------------------------------------------------------
 // a1: keys
 // ------------------------------------------------------------------------------------
+// Bag-parallel: thread per bag writes the keys / bag ids of its positions and counts the
+// radix digits of every pass (the sort's upfront histogram, fused here).  keys / bag_of
+// are zeroed beforehand so malformed offsets (flagged) leave only in-range values.
 template <typename IdxT>
 __global__ void __launch_bounds__(256)
 k_build_keys(const IdxT* __restrict__ indices, const int64_t* __restrict__ offsets, int64_t nnz,
              int32_t B, int T, const uint64_t* __restrict__ rowbase, uint32_t* __restrict__ keys,
-             uint32_t* __restrict__ bag_of, uint32_t* __restrict__ counts) {
+             uint32_t* __restrict__ bag_of, uint32_t* __restrict__ counts, int passes,
+             uint32_t* __restrict__ hist) {
+  __shared__ uint32_t sh[4][256];
+  for (int i = threadIdx.x; i < 4 * 256; i += blockDim.x) (&sh[0][0])[i] = 0;
+  __syncthreads();
   const int64_t nbags = (int64_t)T * B;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   uint32_t err = 0, multi = 0;
-  for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < nnz; j += stride) {
-    // bag of position j: the last b with offsets[b] <= j
-    int64_t lo = 0, hi = nbags - 1;
-    while (lo < hi) {
-      const int64_t mid = (lo + hi + 1) >> 1;
-      if (__ldg(offsets + mid) <= j) lo = mid; else hi = mid - 1;
-    }
-    const int t = (int)(lo / B);
-    const int64_t b = lo - (int64_t)t * B;
-    const int64_t id = (int64_t)indices[j];
+  for (int64_t b = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; b < nbags; b += stride) {
+    int64_t s = __ldg(offsets + b), e = __ldg(offsets + b + 1);
+    if (s < 0 || e > nnz || e < s) { err |= kErrOffsets; s = 0; e = 0; }
+    if (b == 0 && s != 0) err |= kErrOffsets;
+    if (b == nbags - 1 && e != nnz) err |= kErrOffsets;
+    if (e - s != 1) multi = 1u;
+    const int t = (int)(b / B);
+    const int64_t bb = b - (int64_t)t * B;
     const uint64_t rb = __ldg(rowbase + t);
     const uint64_t M = __ldg(rowbase + t + 1) - rb;
-    uint32_t key = (uint32_t)rb;
-    if (id < 0 || (uint64_t)id >= M) err |= kErrRange;
-    else key = (uint32_t)(rb + (uint64_t)id);
-    keys[j] = key;
-    bag_of[j] = (uint32_t)(b * T + t);
+    const uint32_t bo = (uint32_t)(bb * T + t);
+    for (int64_t j = s; j < e; ++j) {
+      const int64_t id = (int64_t)indices[j];
+      uint32_t key = (uint32_t)rb;
+      if (id < 0 || (uint64_t)id >= M) err |= kErrRange;
+      else key = (uint32_t)(rb + (uint64_t)id);
+      keys[j] = key;
+      bag_of[j] = bo;
+      for (int p = 0; p < passes; ++p) atomicAdd(&sh[p][(key >> (8 * p)) & 255u], 1u);
+    }
   }
-  for (int64_t b = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; b <= nbags; b += stride) {
-    const int64_t v = offsets[b];
-    if (v < 0 || v > nnz) err |= kErrOffsets;
-    if (b == 0 && v != 0) err |= kErrOffsets;
-    if (b == nbags && v != nnz) err |= kErrOffsets;
-    if (b < nbags && offsets[b + 1] < v) err |= kErrOffsets;
-    if (b < nbags && offsets[b + 1] - v != 1) multi = 1u;
-  }
+  if (nbags == 0 && nnz != 0 && blockIdx.x == 0 && threadIdx.x == 0) err |= kErrOffsets;
   if (err) atomicOr(counts + kCntErr, err);
   if (multi) atomicOr(counts + kCntMulti, 1u);
+  __syncthreads();
+  for (int i = threadIdx.x; i < passes * 256; i += blockDim.x) {
+    const uint32_t v = (&sh[0][0])[i];
+    if (v) atomicAdd(hist + i, v);
+  }
 }
 
 // ------------------------------------------------------------------------------------
@@ -233,7 +271,7 @@ k_radix_pass(const uint32_t* __restrict__ kin, const uint32_t* __restrict__ vin,
   uint32_t tot;
   const uint32_t bstart = block_excl_scan_256(run, s_warp, tot);
   s_bstart[tid] = bstart;
-  const uint32_t excl = lookback(status + tid, 256, tile, run);
+  const uint32_t excl = lookback<16>(status + tid, 256, tile, run);
   s_gbase[tid] = dbase[tid] + excl;
   __syncthreads();
 #pragma unroll
@@ -260,7 +298,7 @@ k_radix_pass(const uint32_t* __restrict__ kin, const uint32_t* __restrict__ vin,
 // Single-pass scan skeleton: flags -> exclusive slots, with decoupled look-back.
 // Body provides size(), flag(i), emit(i, slot, flag), finish(total).
 // ------------------------------------------------------------------------------------
-constexpr int SC_T = 256, SC_IPT = 8, SC_TILE = SC_T * SC_IPT;
+constexpr int SC_T = 256, SC_IPT = 8, SC_TILE = SC_T * SC_IPT;   // SC_IPT * 8 == 64 warp counts
 
 template <class Body>
 __global__ void __launch_bounds__(SC_T) k_scan(Body body, uint32_t* status, uint32_t* counter) {
@@ -299,7 +337,10 @@ __global__ void __launch_bounds__(SC_T) k_scan(Body body, uint32_t* status, uint
     if (lane == 31) s_total = x;
   }
   __syncthreads();
-  if (tid == 0) s_base = lookback(status, 1, tile, s_total);
+  if (w == 0) {
+    const uint32_t b = lookback_warp(status, tile, s_total);
+    if (lane == 0) s_base = b;
+  }
   __syncthreads();
   const uint32_t lt = lanemask_lt();
 #pragma unroll
@@ -403,10 +444,11 @@ struct GroupBody {
 int radix_sort(Ctx& c, uint32_t* kA, uint32_t* vA, uint32_t* kB, uint32_t* vB,
                const uint32_t* n_dev, uint32_t n_static, int64_t n_max, int passes,
                uint32_t* hist, uint32_t* dbase, uint32_t* counters, uint32_t* status,
-               int64_t tiles, int st_hist, int st_pass, cudaStream_t s) {
+               int64_t tiles, int st_hist, int st_pass, cudaStream_t s, bool have_hist = false) {
   {
     StageScope sc(c, st_hist, s);
-    k_radix_hist<<<grid_for(c, n_max, 256, 4), 256, 0, s>>>(kA, n_dev, n_static, passes, hist);
+    if (!have_hist)
+      k_radix_hist<<<grid_for(c, n_max, 256, 4), 256, 0, s>>>(kA, n_dev, n_static, passes, hist);
     k_hist_scan<<<1, 256, 0, s>>>(hist, dbase, passes);
   }
   uint32_t *ki = kA, *vi = vA, *ko = kB, *vo = vB;
@@ -437,20 +479,26 @@ cudaError_t run_index_stage(Ctx& c, const void* indices, const int64_t* offsets,
   }
   {
     StageScope sc(c, ST_KEYS, s);
-    const int64_t items = nnz > (int64_t)c.T * c.B + 1 ? nnz : (int64_t)c.T * c.B + 1;
-    const int g = grid_for(c, items, 256, 8);
+    if (nnz > 0) {
+      cudaMemsetAsync(p.keysA, 0, sizeof(uint32_t) * nnz, s);
+      cudaMemsetAsync(p.bag_of, 0, sizeof(uint32_t) * nnz, s);
+    }
+    const int64_t bags = (int64_t)c.T * c.B;
+    const int g = grid_for(c, bags > 0 ? bags : 1, 256, 32);
     if (c.index_bits == 64)
       k_build_keys<int64_t><<<g, 256, 0, s>>>((const int64_t*)indices, offsets, nnz, c.B, c.T,
-                                              c.d_rowbase, p.keysA, p.bag_of, p.counts);
+                                              c.d_rowbase, p.keysA, p.bag_of, p.counts,
+                                              c.key_passes, p.hist1);
     else
       k_build_keys<int32_t><<<g, 256, 0, s>>>((const int32_t*)indices, offsets, nnz, c.B, c.T,
-                                              c.d_rowbase, p.keysA, p.bag_of, p.counts);
+                                              c.d_rowbase, p.keysA, p.bag_of, p.counts,
+                                              c.key_passes, p.hist1);
   }
   // a2: sort (key, position)
   const int64_t tiles1 = radix_tiles(nnz);
   const int which = radix_sort(c, p.keysA, p.valsA, p.keysB, p.valsB, nullptr, (uint32_t)nnz, nnz,
                                c.key_passes, p.hist1, p.dbase1, p.rs1_counter, p.rs1_status, tiles1,
-                               ST_SORT_HIST, ST_SORT_PASS, s);
+                               ST_SORT_HIST, ST_SORT_PASS, s, /*have_hist=*/true);
   p.skey = which ? p.keysB : p.keysA;
   p.spos = which ? p.valsB : p.valsA;
   // the other ping-pong pair is free now: group-sort buffers

@@ -131,7 +131,7 @@ cudaError_t run_tc_bwd(Ctx& c, float lr, cudaStream_t s);
 
 // ---- small helpers -------------------------------------------------------------------
 static inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
-static inline int grid_for(const Ctx& c, int64_t items, int threads, int per_sm = 8) {
+static inline int grid_for(const Ctx& c, int64_t items, int threads, int per_sm = 32) {
   int64_t g = cdiv(items, threads);
   int64_t cap = (int64_t)c.sm_count * per_sm;
   if (g > cap) g = cap;

@@ -16,7 +16,11 @@
 // operands are prefetched into registers while the current chunk's MMAs run, and the
 // next group is claimed one ahead.  The row kernels walk 16 consecutive unique rows per
 // warp, so Zipf-hot prefixes (hundreds of rows) spread over many warps.
+#include <stdio.h>
+#include <stdlib.h>
+
 #include <algorithm>
+#include <vector>
 
 #include "tc.cuh"
 #include "ttemb_internal.cuh"
@@ -44,6 +48,7 @@ struct TcArgs {
   float* dabuf;         // [P][n1][R] dC1 partials
   float* out;           // [B][T][N]
   uint32_t* work;
+  unsigned long long* trace;   // optional per-phase cycle counters (TTEMB_TRACE)
   int n1, n2, n3, N, NC, n1s;
   float lr, eps;
   int opt, fused;
@@ -601,12 +606,15 @@ __global__ void __launch_bounds__(TNT, 1) k_tc_bwd2(TcArgs a) {
       store_pat(a2h, a2l, pa);                               // A2 = CM(r1, m)
       for (int k = 0; k < NCH; ++k) {
         const int b = k & 1;
+        long long tt0 = clock64();
         wait_buf(b);                                         // MMA(k-2) done: buffer b free
         if (last_tile && k >= 2) finish_chunk(k - 2, b, c2o);
+        long long tt1 = clock64();
         __syncthreads();
         store_pat(x2h(b), x2l(b), px);                       // X2 = CM(r1, c)
         store_pat(d1h(b), d1l(b), pd1);                      // D1 = CM(m, c)
         store_pat(d2h(b), d2l(b), pd2);                      // D2 = CM(c, m)
+        long long tt2 = clock64();
         if (k + 1 < NCH) {
           load_colq(px, C2s + (k + 1) * TCW, a.NC, TR);
           load_tab(pd1, a.dpbuf + (k + 1) * TCW, a.NC, s_rowp[tb], false);
@@ -623,15 +631,27 @@ __global__ void __launch_bounds__(TNT, 1) k_tc_bwd2(TcArgs a) {
             load_tab(pa, a.cores + a.meta[a.grp_t[ng]].c1_off, TR, s_rowa[tb ^ 1], true);
           }
         }
+        long long tt3 = clock64();
         publish();
+        long long tt4 = clock64();
         if (tid == 0) {
           mma3(tDA, x2h(b), x2l(b), d1h(b), d1l(b), k > 0);          // dA^T [r1][m]
           mma3(tDC2 + 64 * k, a2h, a2l, d2h(b), d2l(b), mt > 0);      // dC2  [r1][c]
           tc::commit(&mbar[b]);
         }
         __syncwarp();
+        long long tt5 = clock64();
+        if (a.trace && tid == 0) {
+          unsigned long long* tr = a.trace + 8 * blockIdx.x;
+          tr[0] += tt1 - tt0; tr[1] += tt2 - tt1; tr[2] += tt3 - tt2; tr[3] += tt4 - tt3; tr[4] += tt5 - tt4; tr[7] += 1;
+        }
+        if (a.trace && tid == 32) {
+          unsigned long long* tr = a.trace + 8 * blockIdx.x;
+          tr[5] += tt5 - tt4;
+        }
         if (b == 0) pend0 = 1; else pend1 = 1;
       }
+      long long te0 = clock64();
       for (int kc = (NCH >= 2 ? NCH - 2 : 0); kc < NCH; ++kc) {   // drain the last two chunks
         wait_buf(kc & 1);
         if (last_tile) finish_chunk(kc, kc & 1, c2o);
@@ -649,6 +669,7 @@ __global__ void __launch_bounds__(TNT, 1) k_tc_bwd2(TcArgs a) {
         }
         tc::fence_before();
       }
+      if (a.trace && tid == 0) a.trace[8 * blockIdx.x + 6] += clock64() - te0;
       tb ^= 1;
     }
     __syncthreads();
@@ -671,7 +692,7 @@ TcArgs make_tc_args(Ctx& c, float lr, uint32_t* work, float* out) {
   a.grp_pfx = p.grp_pfx; a.pfx_i1 = p.pfx_i1; a.pfx_t = p.pfx_t; a.row_seg = p.row_seg;
   a.row_i3 = p.row_i3; a.row_pfx = p.row_pfx; a.seg_off = p.seg_off; a.sbag = p.sbag;
   a.pbuf = p.pbuf; a.dpbuf = p.dpbuf; a.rows = p.rows; a.gbuf = p.gbuf; a.dabuf = p.dabuf;
-  a.out = out; a.work = work;
+  a.out = out; a.work = work; a.trace = nullptr;
   a.n1 = c.n1; a.n2 = c.n2; a.n3 = c.n3; a.N = c.N; a.NC = c.NC;
   a.n1s = c.n1 == 1 ? 0 : c.n1 == 2 ? 1 : c.n1 == 4 ? 2 : 3;
   a.lr = lr; a.eps = c.eps; a.opt = c.opt; a.fused = (c.flags & TTEMB_FUSED_UPDATE) ? 1 : 0;
@@ -725,7 +746,22 @@ cudaError_t run_tc_bwd(Ctx& c, float lr, cudaStream_t s) {
   {
     StageScope sc(c, ST_BWD_PREFIX, s);
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(c.NG_cap, (int64_t)c.sm_count));
+    static unsigned long long* trace = nullptr;
+    if (getenv("TTEMB_TRACE")) {
+      if (!trace) cudaMalloc(&trace, sizeof(unsigned long long) * 8 * grid);
+      cudaMemsetAsync(trace, 0, sizeof(unsigned long long) * 8 * grid, s);
+      a.trace = trace;
+    }
     k_tc_bwd2<<<grid, TNT, kTcBwdSmem, s>>>(a);
+    if (trace) {
+      std::vector<unsigned long long> h(8 * grid);
+      cudaMemcpyAsync(h.data(), trace, h.size() * 8, cudaMemcpyDeviceToHost, s);
+      cudaStreamSynchronize(s);
+      double sum[8] = {};
+      for (int b = 0; b < grid; ++b) for (int i = 0; i < 8; ++i) sum[i] += h[8 * b + i];
+      fprintf(stderr, "[trace bwd2] steps/CTA %.1f | cycles/CTA: wait+finish %.0f store %.0f prefetch %.0f publish %.0f mma_issue(t0) %.0f mma(t32) %.0f tile_end %.0f\n",
+              sum[7] / grid, sum[0] / grid, sum[1] / grid, sum[2] / grid, sum[3] / grid, sum[4] / grid, sum[5] / grid, sum[6] / grid);
+    }
   }
   return cudaGetLastError();
 }

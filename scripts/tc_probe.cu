@@ -100,7 +100,9 @@ __global__ void probe(int mode, int M, int N, int K, const float* a_src, const f
   if (threadIdx.x < 32) tc::tmem_dealloc(tb, 256);
 }
 
-int main() {
+int timing_main();
+int main(int argc, char** argv) {
+  if (argc > 1) return timing_main();
   struct Case { int mode, M, N, K; };
   Case cases[] = {{1, 128, 64, 64}, {1, 128, 64, 8}, {1, 128, 48, 32}, {2, 64, 128, 64},
                   {2, 128, 128, 64}, {2, 64, 128, 8}, {3, 64, 64, 128}, {3, 128, 48, 128},
@@ -154,4 +156,75 @@ int main() {
   }
   printf(fails ? "TC PROBE FAILED\n" : "TC PROBE OK\n");
   return fails ? 1 : 0;
+}
+
+// ---- timing microbenchmark: NM back-to-back 3xTF32 K=64 products (24 MMAs each) ----
+__global__ void mma_timing(int M, int N, int reps, int precomp, long long* cycles) {
+  extern __shared__ __align__(1024) float sm[];
+  __shared__ uint64_t mbar;
+  __shared__ uint32_t tmem_base;
+  for (int i = threadIdx.x; i < 4 * 64 * 64 * 2; i += blockDim.x) sm[i] = 0.001f * (i % 97);
+  if (threadIdx.x == 0) { tc::mbar_init(&mbar, 1); tc::fence_mbar_init(); }
+  if (threadIdx.x < 32) tc::tmem_alloc(&tmem_base, 256);
+  tc::fence_async_smem();
+  tc::fence_before();
+  __syncthreads();
+  tc::fence_after();
+  const uint32_t tb = tmem_base;
+  long long t0 = 0, t1 = 0;
+  if (threadIdx.x == 0) {
+    const int MR = M / 8;    // row blocks of A (M rows), B has N rows
+    const uint32_t id = tc::idesc_tf32(M, N, false, false);
+    const uint32_t ah = tc::smem_u32(sm), al = ah + M * 64 * 4, bh = al + M * 64 * 4, bl = bh + N * 64 * 4;
+    t0 = clock64();
+    for (int rep = 0; rep < reps; ++rep) {
+      if (precomp) {
+        const uint64_t dah = tc::sdesc(ah, MR * 128, 128), dal = tc::sdesc(al, MR * 128, 128);
+        const uint64_t dbh = tc::sdesc(bh, (N / 8) * 128, 128), dbl = tc::sdesc(bl, (N / 8) * 128, 128);
+#pragma unroll
+        for (int kk = 0; kk < 8; ++kk) {
+          const uint64_t oa = (uint64_t)((kk * 2 * MR * 128) >> 4), ob = (uint64_t)((kk * 2 * (N / 8) * 128) >> 4);
+          tc::mma_tf32(tb, dah + oa, dbh + ob, id, (rep > 0 || kk > 0) ? 1u : 0u);
+          tc::mma_tf32(tb, dah + oa, dbl + ob, id, 1u);
+          tc::mma_tf32(tb, dal + oa, dbh + ob, id, 1u);
+        }
+      } else {
+#pragma unroll
+        for (int kk = 0; kk < 8; ++kk) {
+          const uint32_t oa = kk * 2 * MR * 128, ob = kk * 2 * (N / 8) * 128;
+          const uint64_t dah = tc::sdesc(ah + oa, MR * 128, 128), dal = tc::sdesc(al + oa, MR * 128, 128);
+          const uint64_t dbh = tc::sdesc(bh + ob, (N / 8) * 128, 128), dbl = tc::sdesc(bl + ob, (N / 8) * 128, 128);
+          tc::mma_tf32(tb, dah, dbh, id, (rep > 0 || kk > 0) ? 1u : 0u);
+          tc::mma_tf32(tb, dah, dbl, id, 1u);
+          tc::mma_tf32(tb, dal, dbh, id, 1u);
+        }
+      }
+    }
+    t1 = clock64();
+    tc::commit(&mbar);
+  }
+  tc::mbar_wait(&mbar, 0);
+  if (threadIdx.x == 0) { cycles[0] = t1 - t0; cycles[1] = clock64() - t0; }
+  tc::fence_before();
+  __syncthreads();
+  if (threadIdx.x < 32) tc::tmem_dealloc(tb, 256);
+}
+
+int timing_main() {
+  long long* d;
+  cudaMalloc(&d, 16);
+  cudaFuncSetAttribute(mma_timing, cudaFuncAttributeMaxDynamicSharedMemorySize, 4 * 64 * 64 * 4 * 2 + 1024);
+  int shapes[][2] = {{64, 64}, {128, 64}, {64, 128}, {128, 128}, {64, 256}, {128, 256}};
+  for (auto& sh : shapes)
+    for (int pre = 0; pre < 2; ++pre) {
+      const int reps = 50;
+      mma_timing<<<1, 128, 4 * 64 * 64 * 4 * 2 + 1024>>>(sh[0], sh[1], reps, pre, d);
+      cudaError_t e = cudaDeviceSynchronize();
+      long long h[2];
+      cudaMemcpy(h, d, 16, cudaMemcpyDeviceToHost);
+      const double n = reps * 24.0;
+      printf("M=%3d N=%3d precomp=%d: issue %.1f cyc/MMA, complete %.1f cyc/MMA (%.0f MAC/cyc) %s\n", sh[0], sh[1], pre,
+             h[0] / n, h[1] / n, (double)sh[0] * sh[1] * 8 / (h[1] / n), e == cudaSuccess ? "" : cudaGetErrorString(e));
+    }
+  return 0;
 }
