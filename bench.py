@@ -393,6 +393,13 @@ def main():
         roof = {"bound": "hbm", "kernel": dname, "achieved": ach, "peak": hbm_peak, "unit": "GB/s",
                 "frac": ach / hbm_peak, "traffic": None, "peak_source": f"{peak_kind} copy bandwidth"}
     roof["share_of_step"] = dms / max(t_ms, 1e-9)
+    tr_path = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tr_path):      # DRAM bytes per launch from the committed ncu --set full capture
+        tr = json.load(open(tr_path))
+        if dname in tr.get("dram_bytes_per_launch", {}):
+            roof["traffic"] = tr["dram_bytes_per_launch"][dname]
+            roof["traffic_source"] = tr.get("source")
+            roof["alg_bytes_per_launch"] = b1
     t_alu = flops / (alu_peak * 1e12) * 1e3
     t_hbm = bytes_ / (hbm_peak * 1e9) * 1e3
     step_roof = {"alg_gflop": flops / 1e9, "alg_mb": bytes_ / 1e6, "t_alu_ms": t_alu, "t_hbm_ms": t_hbm,
