@@ -48,7 +48,6 @@ struct TcArgs {
   float* dabuf;         // [P][n1][R] dC1 partials
   float* out;           // [B][T][N]
   uint32_t* work;
-  unsigned long long* trace;   // optional per-phase cycle counters (TTEMB_TRACE)
   int n1, n2, n3, N, NC, n1s;
   float lr, eps;
   int opt, fused;
@@ -496,14 +495,19 @@ __global__ void __launch_bounds__(128) k_rows_bwd(TcArgs a) {
   }
 }
 
-// Backward GEMMs per i2-group: dA^T = X2 . D1^T (TMEM, accumulated over chunks) and
-// dC2[chunk] += A2 . D2^T (TMEM, accumulated over m-tiles).  X2 / D1 / D2 are
-// double-buffered so MMA(k) overlaps the staging of chunk k+1; in the group's last m-tile
-// the finished dC2 chunk k-2 is applied (fused update) from the staged X2 copy
-// (C2 = X2_hi + X2_lo exactly) before its buffer is reused.
-__global__ void __launch_bounds__(TNT, 1) k_tc_bwd2(TcArgs a) {
+// Backward GEMMs per i2-group, warp-specialised: warps 0-7 (256 threads) stage operands,
+// run the epilogues and the fused C2 update; warp 8 issues the tcgen05 MMAs.
+//   dA^T [r1][m]  = X2 . D1^T   (TMEM, accumulated over the tile's chunks)
+//   dC2  [r1][c] += A2 . D2^T   (TMEM per chunk, accumulated over the group's m-tiles)
+// X2 / D1 / D2 are double-buffered; full[b] (one arrival per producer thread) hands a staged step
+// to the MMA warp together with a small command word, empty[b] (tcgen05.commit) hands the
+// buffer back.  Row addresses of a tile are computed once per tile, so the per-chunk
+// prefetch is a plain burst of loads.
+constexpr int WS_PROD = 256, WS_ALL = 288;
+
+__global__ void __launch_bounds__(WS_ALL, 1) k_tc_bwd2(TcArgs a) {
   extern __shared__ __align__(128) char smem[];
-  float* const base = reinterpret_cast<float*>(smem);     // buffer b: 6 matrices at base + 6b*TCM/4
+  float* const base = reinterpret_cast<float*>(smem);
   constexpr int MF = TCM / 4;
   auto x2h = [&](int b) { return base + (6 * b + 0) * MF; };
   auto x2l = [&](int b) { return base + (6 * b + 1) * MF; };
@@ -513,175 +517,229 @@ __global__ void __launch_bounds__(TNT, 1) k_tc_bwd2(TcArgs a) {
   auto d2l = [&](int b) { return base + (6 * b + 5) * MF; };
   float* a2h = base + 12 * MF;
   float* a2l = base + 13 * MF;
-  __shared__ uint64_t mbar[2];
+  __shared__ uint64_t full[2], empty[2];
+  __shared__ uint32_t cmd[2][2];
   __shared__ uint32_t s_tmem, s_g[2], s_rowp[2][64], s_rowa[2][64];
-  const int tid = threadIdx.x, w = tid >> 5, lane = tid & 31, q4 = w & 3, half = w >> 2;
+  const int tid = threadIdx.x, w = tid >> 5, lane = tid & 31;
   if (tid == 0) {
-    tc::mbar_init(&mbar[0], 1);
-    tc::mbar_init(&mbar[1], 1);
+    for (int b = 0; b < 2; ++b) {
+      tc::mbar_init(&full[b], WS_PROD);
+      tc::mbar_init(&empty[b], 1);
+    }
     tc::fence_mbar_init();
     s_g[0] = atomicAdd(a.work, 1u);
     s_g[1] = atomicAdd(a.work, 1u);
   }
-  if (tid < 32) tc::tmem_alloc(&s_tmem, 512);
+  if (w == 0) tc::tmem_alloc(&s_tmem, 512);
   tc::fence_before();
   __syncthreads();
   tc::fence_after();
   const uint32_t tDA = s_tmem, tDC2 = s_tmem + 64;
-  uint32_t ph0 = 0u, ph1 = 0u;
-  int pend0 = 0, pend1 = 0;
   const uint32_t NG = a.counts[kCntNG];
   const int PPT = TMT >> a.n1s, NCH = a.NC / TCW;
-  uint32_t g = s_g[0], gnext = s_g[1];
-  int tb = 0;
-  float4 px[4], pd1[4], pd2[4], pa[4];
-  if (g < NG) {
-    fill_table(a, s_rowp[0], s_rowa[0], a.grp_off[g], (int)min((uint32_t)PPT, a.grp_off[g + 1] - a.grp_off[g]));
-    __syncthreads();
-    load_colq(px, c2_slice(a, g), a.NC, TR);
-    load_tab(pd1, a.dpbuf, a.NC, s_rowp[0], false);
-    load_tab(pd2, a.dpbuf, a.NC, s_rowp[0], true);
-    load_tab(pa, a.cores + a.meta[a.grp_t[g]].c1_off, TR, s_rowa[0], true);
-  }
-  auto wait_buf = [&](int b) {
-    if (b == 0 ? pend0 : pend1) {
-      tc::mbar_wait(&mbar[b], b == 0 ? ph0 : ph1);
-      if (b == 0) { ph0 ^= 1u; pend0 = 0; } else { ph1 ^= 1u; pend1 = 0; }
+
+  if (w == 8) {
+    // ------------------------------ MMA issuer ------------------------------
+    uint32_t fph0 = 0, fph1 = 0;
+    for (uint32_t s = 0;; ++s) {
+      const int b = s & 1;
+      tc::mbar_wait(&full[b], b ? fph1 : fph0);
+      if (b) fph1 ^= 1u; else fph0 ^= 1u;
       tc::fence_after();
+      const uint32_t c0 = cmd[b][0], c1 = cmd[b][1];
+      if (c0 == 0xffffffffu) break;
+      if (lane == 0) {
+        const int k = (int)c0;
+        mma3(tDA, x2h(b), x2l(b), d1h(b), d1l(b), k > 0);               // dA^T [r1][m]
+        mma3(tDC2 + 64 * k, a2h, a2l, d2h(b), d2l(b), c1 != 0);          // dC2  [r1][c]
+        tc::commit(&empty[b]);
+      }
+      __syncwarp();
     }
-  };
-  // final dC2 of chunk kc (MMAs done): gradient or fused update, C2 read from X2[b]
-  auto finish_chunk = [&](int kc, int b, size_t c2o) {
-    float v[32];
-    tc::tmem_ld32(tc::taddr(tDC2 + 64 * kc, 32 * q4, 32 * half), v);
-    if (lane < 16) {
-      const int r1 = 16 * q4 + lane;
-      const size_t b0 = c2o + (size_t)r1 * a.NC + kc * TCW + 32 * half;
-      if (a.fused) {
-        float x[32];
-#pragma unroll
-        for (int j = 0; j < 32; j += 4) {
-          const uint32_t off = tc::cm_off(r1, 32 * half + j, TNRB);
-          const float4 h = *reinterpret_cast<const float4*>(fat(x2h(b), off));
-          const float4 l = *reinterpret_cast<const float4*>(fat(x2l(b), off));
-          x[j] = h.x + l.x; x[j + 1] = h.y + l.y; x[j + 2] = h.z + l.z; x[j + 3] = h.w + l.w;
-        }
-        if (a.opt == TTEMB_SGD) {
-#pragma unroll
-          for (int j = 0; j < 32; j += 4)
-            *reinterpret_cast<float4*>(a.cores + b0 + j) =
-                make_float4(x[j] - a.lr * v[j], x[j + 1] - a.lr * v[j + 1], x[j + 2] - a.lr * v[j + 2],
-                            x[j + 3] - a.lr * v[j + 3]);
-        } else {
+  } else {
+    // --------------------------- producers / epilogue ---------------------------
+    const int q4 = w & 3, half = w >> 2;
+    uint32_t eph0 = 0, eph1 = 0;
+    int pend0 = 0, pend1 = 0;
+    auto wait_buf = [&](int b) {
+      if (b == 0 ? pend0 : pend1) {
+        tc::mbar_wait(&empty[b], b == 0 ? eph0 : eph1);
+        if (b == 0) { eph0 ^= 1u; pend0 = 0; } else { eph1 ^= 1u; pend1 = 0; }
+        tc::fence_after();
+      }
+    };
+    auto finish_chunk = [&](int kc, int b, size_t c2o) {
+      float v[32];
+      tc::tmem_ld32(tc::taddr(tDC2 + 64 * kc, 32 * q4, 32 * half), v);
+      if (lane < 16) {
+        const int r1 = 16 * q4 + lane;
+        const size_t b0 = c2o + (size_t)r1 * a.NC + kc * TCW + 32 * half;
+        if (a.fused) {
+          float x[32];
 #pragma unroll
           for (int j = 0; j < 32; j += 4) {
-            const float4 s4 = *reinterpret_cast<const float4*>(a.state + b0 + j);
-            const float s0 = s4.x + v[j] * v[j], s1 = s4.y + v[j + 1] * v[j + 1];
-            const float s2 = s4.z + v[j + 2] * v[j + 2], s3 = s4.w + v[j + 3] * v[j + 3];
-            *reinterpret_cast<float4*>(a.state + b0 + j) = make_float4(s0, s1, s2, s3);
-            *reinterpret_cast<float4*>(a.cores + b0 + j) =
-                make_float4(x[j] - a.lr * v[j] / (sqrtf(s0) + a.eps), x[j + 1] - a.lr * v[j + 1] / (sqrtf(s1) + a.eps),
-                            x[j + 2] - a.lr * v[j + 2] / (sqrtf(s2) + a.eps), x[j + 3] - a.lr * v[j + 3] / (sqrtf(s3) + a.eps));
+            const uint32_t off = tc::cm_off(r1, 32 * half + j, TNRB);
+            const float4 h = *reinterpret_cast<const float4*>(fat(x2h(b), off));
+            const float4 l = *reinterpret_cast<const float4*>(fat(x2l(b), off));
+            x[j] = h.x + l.x; x[j + 1] = h.y + l.y; x[j + 2] = h.z + l.z; x[j + 3] = h.w + l.w;
           }
-        }
-      } else {
+          if (a.opt == TTEMB_SGD) {
 #pragma unroll
-        for (int j = 0; j < 32; j += 4)
-          *reinterpret_cast<float4*>(a.grads + b0 + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
-      }
-    }
-    tc::fence_before();
-  };
-  while (g < NG) {
-    const uint32_t i2 = a.grp_i2[g];
-    const uint32_t q0 = a.grp_off[g], q1 = a.grp_off[g + 1];
-    const size_t c2o = a.meta[a.grp_t[g]].c2_off + (size_t)i2 * TR * a.NC;
-    const float* C2s = a.cores + c2o;
-    const uint32_t nmt = (q1 - q0 + PPT - 1) / PPT;
-    for (uint32_t mt = 0; mt < nmt; ++mt) {
-      const bool last_tile = (mt + 1 == nmt);
-      wait_buf(0);
-      wait_buf(1);
-      __syncthreads();
-      store_pat(a2h, a2l, pa);                               // A2 = CM(r1, m)
-      for (int k = 0; k < NCH; ++k) {
-        const int b = k & 1;
-        long long tt0 = clock64();
-        wait_buf(b);                                         // MMA(k-2) done: buffer b free
-        if (last_tile && k >= 2) finish_chunk(k - 2, b, c2o);
-        long long tt1 = clock64();
-        __syncthreads();
-        store_pat(x2h(b), x2l(b), px);                       // X2 = CM(r1, c)
-        store_pat(d1h(b), d1l(b), pd1);                      // D1 = CM(m, c)
-        store_pat(d2h(b), d2l(b), pd2);                      // D2 = CM(c, m)
-        long long tt2 = clock64();
-        if (k + 1 < NCH) {
-          load_colq(px, C2s + (k + 1) * TCW, a.NC, TR);
-          load_tab(pd1, a.dpbuf + (k + 1) * TCW, a.NC, s_rowp[tb], false);
-          load_tab(pd2, a.dpbuf + (k + 1) * TCW, a.NC, s_rowp[tb], true);
-        } else {                                             // next tile (or group)
-          uint32_t ng = g, nqa = q0 + (mt + 1) * PPT;
-          if (mt + 1 >= nmt) { ng = gnext; nqa = ng < NG ? a.grp_off[ng] : 0; }
-          if (ng < NG) {
-            fill_table(a, s_rowp[tb ^ 1], s_rowa[tb ^ 1], nqa, (int)min((uint32_t)PPT, a.grp_off[ng + 1] - nqa));
-            __syncthreads();
-            load_colq(px, c2_slice(a, ng), a.NC, TR);
-            load_tab(pd1, a.dpbuf, a.NC, s_rowp[tb ^ 1], false);
-            load_tab(pd2, a.dpbuf, a.NC, s_rowp[tb ^ 1], true);
-            load_tab(pa, a.cores + a.meta[a.grp_t[ng]].c1_off, TR, s_rowa[tb ^ 1], true);
-          }
-        }
-        long long tt3 = clock64();
-        publish();
-        long long tt4 = clock64();
-        if (tid == 0) {
-          mma3(tDA, x2h(b), x2l(b), d1h(b), d1l(b), k > 0);          // dA^T [r1][m]
-          mma3(tDC2 + 64 * k, a2h, a2l, d2h(b), d2l(b), mt > 0);      // dC2  [r1][c]
-          tc::commit(&mbar[b]);
-        }
-        __syncwarp();
-        long long tt5 = clock64();
-        if (a.trace && tid == 0) {
-          unsigned long long* tr = a.trace + 8 * blockIdx.x;
-          tr[0] += tt1 - tt0; tr[1] += tt2 - tt1; tr[2] += tt3 - tt2; tr[3] += tt4 - tt3; tr[4] += tt5 - tt4; tr[7] += 1;
-        }
-        if (a.trace && tid == 32) {
-          unsigned long long* tr = a.trace + 8 * blockIdx.x;
-          tr[5] += tt5 - tt4;
-        }
-        if (b == 0) pend0 = 1; else pend1 = 1;
-      }
-      long long te0 = clock64();
-      for (int kc = (NCH >= 2 ? NCH - 2 : 0); kc < NCH; ++kc) {   // drain the last two chunks
-        wait_buf(kc & 1);
-        if (last_tile) finish_chunk(kc, kc & 1, c2o);
-      }
-      {   // dA^T -> dabuf[(p, j1)][r1]
-        float v[32];
-        tc::tmem_ld32(tc::taddr(tDA, 32 * q4, 32 * half), v);
-        if (lane < 16) {
-          const int r1 = 16 * q4 + lane;
+            for (int j = 0; j < 32; j += 4)
+              *reinterpret_cast<float4*>(a.cores + b0 + j) =
+                  make_float4(x[j] - a.lr * v[j], x[j + 1] - a.lr * v[j + 1], x[j + 2] - a.lr * v[j + 2],
+                              x[j + 3] - a.lr * v[j + 3]);
+          } else {
 #pragma unroll
-          for (int j = 0; j < 32; ++j) {
-            const uint32_t r = s_rowp[tb][32 * half + j];
-            if (r != 0xffffffffu) a.dabuf[(size_t)r * TR + r1] = v[j];
+            for (int j = 0; j < 32; j += 4) {
+              const float4 s4 = *reinterpret_cast<const float4*>(a.state + b0 + j);
+              const float s0 = s4.x + v[j] * v[j], s1 = s4.y + v[j + 1] * v[j + 1];
+              const float s2 = s4.z + v[j + 2] * v[j + 2], s3 = s4.w + v[j + 3] * v[j + 3];
+              *reinterpret_cast<float4*>(a.state + b0 + j) = make_float4(s0, s1, s2, s3);
+              *reinterpret_cast<float4*>(a.cores + b0 + j) =
+                  make_float4(x[j] - a.lr * v[j] / (sqrtf(s0) + a.eps), x[j + 1] - a.lr * v[j + 1] / (sqrtf(s1) + a.eps),
+                              x[j + 2] - a.lr * v[j + 2] / (sqrtf(s2) + a.eps), x[j + 3] - a.lr * v[j + 3] / (sqrtf(s3) + a.eps));
+            }
+          }
+        } else {
+#pragma unroll
+          for (int j = 0; j < 32; j += 4)
+            *reinterpret_cast<float4*>(a.grads + b0 + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
+        }
+      }
+      tc::fence_before();
+    };
+    // hand step (buffer b) to the MMA warp
+    auto post = [&](int b, uint32_t c0, uint32_t c1) {
+      tc::fence_async_smem();
+      tc::fence_before();
+      if (tid == 0) { cmd[b][0] = c0; cmd[b][1] = c1; }
+      tc::mbar_arrive(&full[b]);
+    };
+    // per-tile row offsets: COLQ row (one per thread), ROWQ rows (4 per k)
+    uint32_t rcol = 0, racol = 0;
+    uint32_t rrow[16];
+    auto tile_rows = [&](int tbuf) {
+      rcol = s_rowp[tbuf][tid & 63];
+      racol = s_rowa[tbuf][tid & 63];
+#pragma unroll
+      for (int k = 0; k < 4; ++k)
+#pragma unroll
+        for (int i = 0; i < 4; ++i) rrow[4 * k + i] = s_rowp[tbuf][4 * ((tid >> 6) + 4 * k) + i];
+    };
+    auto load_d = [&](float4 (&p1)[4], float4 (&p2)[4], int c0) {
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        const int cq = (tid >> 6) + 4 * k;
+        p1[k] = rcol != 0xffffffffu ? __ldg(reinterpret_cast<const float4*>(a.dpbuf + (size_t)rcol * a.NC + c0 + 4 * cq))
+                                   : make_float4(0.f, 0.f, 0.f, 0.f);
+        float x[4];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const uint32_t r = rrow[4 * k + i];
+          x[i] = r != 0xffffffffu ? __ldg(a.dpbuf + (size_t)r * a.NC + c0 + (tid & 63)) : 0.f;
+        }
+        p2[k] = make_float4(x[0], x[1], x[2], x[3]);
+      }
+    };
+    auto load_a2 = [&](float4 (&p)[4], const float* C1t, int tbuf) {   // A2 = CM(r1, m): 4 m of one r1
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        float x[4];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const uint32_t r = s_rowa[tbuf][4 * ((tid >> 6) + 4 * k) + i];
+          x[i] = r != 0xffffffffu ? __ldg(C1t + (size_t)r * TR + (tid & 63)) : 0.f;
+        }
+        p[k] = make_float4(x[0], x[1], x[2], x[3]);
+      }
+    };
+    uint32_t g = s_g[0], gnext = s_g[1];
+    int tb = 0;
+    uint32_t s = 0;
+    float4 px[4], pd1[4], pd2[4], pa[4];
+    if (g < NG) {
+      if (tid < 64) fill_table(a, s_rowp[0], s_rowa[0], a.grp_off[g], (int)min((uint32_t)PPT, a.grp_off[g + 1] - a.grp_off[g]));
+      tc::named_sync(1, WS_PROD);
+      tile_rows(0);
+      load_colq(px, c2_slice(a, g), a.NC, TR);
+      load_d(pd1, pd2, 0);
+      load_a2(pa, a.cores + a.meta[a.grp_t[g]].c1_off, 0);
+    }
+    while (g < NG) {
+      const uint32_t i2 = a.grp_i2[g];
+      const uint32_t q0 = a.grp_off[g], q1 = a.grp_off[g + 1];
+      const size_t c2o = a.meta[a.grp_t[g]].c2_off + (size_t)i2 * TR * a.NC;
+      const float* C2s = a.cores + c2o;
+      const uint32_t nmt = (q1 - q0 + PPT - 1) / PPT;
+      for (uint32_t mt = 0; mt < nmt; ++mt) {
+        const bool last_tile = (mt + 1 == nmt);
+        wait_buf(0);
+        wait_buf(1);
+        tc::named_sync(1, WS_PROD);                            // previous tile's epilogue done
+        store_pat(a2h, a2l, pa);                               // A2 = CM(r1, m)
+        const uint32_t s0 = s;
+        for (int k = 0; k < NCH; ++k, ++s) {
+          const int b = s & 1;
+          wait_buf(b);                                         // MMA(s-2) done: buffer b free
+          if (last_tile && k >= 2) finish_chunk(k - 2, b, c2o);
+          store_pat(x2h(b), x2l(b), px);                       // X2 = CM(r1, c)
+          store_pat(d1h(b), d1l(b), pd1);                      // D1 = CM(m, c)
+          store_pat(d2h(b), d2l(b), pd2);                      // D2 = CM(c, m)
+          post(b, (uint32_t)k, mt > 0 ? 1u : 0u);
+          if (b == 0) pend0 = 1; else pend1 = 1;
+          if (k + 1 < NCH) {                                   // prefetch the next step
+            load_colq(px, C2s + (k + 1) * TCW, a.NC, TR);
+            load_d(pd1, pd2, (k + 1) * TCW);
+          } else {
+            uint32_t ng = g, nqa = q0 + (mt + 1) * PPT;
+            if (mt + 1 >= nmt) { ng = gnext; nqa = ng < NG ? a.grp_off[ng] : 0; }
+            if (ng < NG) {
+              if (tid < 64) fill_table(a, s_rowp[tb ^ 1], s_rowa[tb ^ 1], nqa, (int)min((uint32_t)PPT, a.grp_off[ng + 1] - nqa));
+              tc::named_sync(1, WS_PROD);
+              tile_rows(tb ^ 1);
+              load_colq(px, c2_slice(a, ng), a.NC, TR);
+              load_d(pd1, pd2, 0);
+              load_a2(pa, a.cores + a.meta[a.grp_t[ng]].c1_off, tb ^ 1);
+            }
           }
         }
-        tc::fence_before();
+        // drain the tile: last two steps (their buffers hold chunks NCH-2, NCH-1)
+        for (int kc = (NCH >= 2 ? NCH - 2 : 0); kc < NCH; ++kc) {
+          const int b = (int)((s0 + kc) & 1);
+          wait_buf(b);
+          if (last_tile) finish_chunk(kc, b, c2o);
+        }
+        {   // dA^T -> dabuf[(p, j1)][r1]
+          float v[32];
+          tc::tmem_ld32(tc::taddr(tDA, 32 * q4, 32 * half), v);
+          if (lane < 16) {
+            const int r1 = 16 * q4 + lane;
+#pragma unroll
+            for (int j = 0; j < 32; ++j) {
+              const uint32_t r = s_rowp[tb][32 * half + j];
+              if (r != 0xffffffffu) a.dabuf[(size_t)r * TR + r1] = v[j];
+            }
+          }
+          tc::fence_before();
+        }
+        tb ^= 1;
       }
-      if (a.trace && tid == 0) a.trace[8 * blockIdx.x + 6] += clock64() - te0;
-      tb ^= 1;
+      tc::named_sync(1, WS_PROD);
+      if (tid == 0) s_g[1] = atomicAdd(a.work, 1u);
+      tc::named_sync(1, WS_PROD);
+      g = gnext;
+      gnext = s_g[1];
     }
-    __syncthreads();
-    if (tid == 0) s_g[1] = atomicAdd(a.work, 1u);
-    __syncthreads();
-    g = gnext;
-    gnext = s_g[1];
+    const int b = s & 1;                                       // tell the MMA warp to stop
+    wait_buf(b);
+    post(b, 0xffffffffu, 0u);
+    wait_buf(b ^ 1);
   }
   tc::fence_before();
   __syncthreads();
   tc::fence_after();
-  if (tid < 32) tc::tmem_dealloc(tDA, 512);
+  if (w == 0) tc::tmem_dealloc(tDA, 512);
 }
 
 TcArgs make_tc_args(Ctx& c, float lr, uint32_t* work, float* out) {
@@ -692,7 +750,7 @@ TcArgs make_tc_args(Ctx& c, float lr, uint32_t* work, float* out) {
   a.grp_pfx = p.grp_pfx; a.pfx_i1 = p.pfx_i1; a.pfx_t = p.pfx_t; a.row_seg = p.row_seg;
   a.row_i3 = p.row_i3; a.row_pfx = p.row_pfx; a.seg_off = p.seg_off; a.sbag = p.sbag;
   a.pbuf = p.pbuf; a.dpbuf = p.dpbuf; a.rows = p.rows; a.gbuf = p.gbuf; a.dabuf = p.dabuf;
-  a.out = out; a.work = work; a.trace = nullptr;
+  a.out = out; a.work = work;
   a.n1 = c.n1; a.n2 = c.n2; a.n3 = c.n3; a.N = c.N; a.NC = c.NC;
   a.n1s = c.n1 == 1 ? 0 : c.n1 == 2 ? 1 : c.n1 == 4 ? 2 : 3;
   a.lr = lr; a.eps = c.eps; a.opt = c.opt; a.fused = (c.flags & TTEMB_FUSED_UPDATE) ? 1 : 0;
@@ -746,22 +804,7 @@ cudaError_t run_tc_bwd(Ctx& c, float lr, cudaStream_t s) {
   {
     StageScope sc(c, ST_BWD_PREFIX, s);
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(c.NG_cap, (int64_t)c.sm_count));
-    static unsigned long long* trace = nullptr;
-    if (getenv("TTEMB_TRACE")) {
-      if (!trace) cudaMalloc(&trace, sizeof(unsigned long long) * 8 * grid);
-      cudaMemsetAsync(trace, 0, sizeof(unsigned long long) * 8 * grid, s);
-      a.trace = trace;
-    }
-    k_tc_bwd2<<<grid, TNT, kTcBwdSmem, s>>>(a);
-    if (trace) {
-      std::vector<unsigned long long> h(8 * grid);
-      cudaMemcpyAsync(h.data(), trace, h.size() * 8, cudaMemcpyDeviceToHost, s);
-      cudaStreamSynchronize(s);
-      double sum[8] = {};
-      for (int b = 0; b < grid; ++b) for (int i = 0; i < 8; ++i) sum[i] += h[8 * b + i];
-      fprintf(stderr, "[trace bwd2] steps/CTA %.1f | cycles/CTA: wait+finish %.0f store %.0f prefetch %.0f publish %.0f mma_issue(t0) %.0f mma(t32) %.0f tile_end %.0f\n",
-              sum[7] / grid, sum[0] / grid, sum[1] / grid, sum[2] / grid, sum[3] / grid, sum[4] / grid, sum[5] / grid, sum[6] / grid);
-    }
+    k_tc_bwd2<<<grid, WS_ALL, kTcBwdSmem, s>>>(a);
   }
   return cudaGetLastError();
 }
