@@ -5,13 +5,17 @@
 // Operand layout in shared memory ("CM layout", SWIZZLE_NONE / interleaved canonical):
 //   a matrix X[r][c] is stored as 8x4 core matrices (8 rows of 16 B = 4 fp32 along c),
 //   128 contiguous bytes each; core (rb, cb) lives at byte (cb * NRB + rb) * 128 where
-//   NRB = rows / 8.  The same bytes describe X as
-//     K-major  with rows = M/N, c = K : SBO = 128,        LBO = NRB*128, K-step(8) = +2*NRB*128
-//     MN-major with c = M/N,  rows = K : SBO = NRB*128,    LBO = 128,     K-step(8) = +128
-//   so one staged copy serves a matrix and its transpose in different MMAs.
+//   NRB = rows / 8.  Used K-major only (rows = M/N, c = K):
+//     SBO = 128, LBO = NRB*128, K-step(8) = +2*NRB*128.
+// MN-major operands (tf32 accepts only SWIZZLE_128B_BASE32B, measured with
+// scripts/tc_probe2.cu): K rows of 128 B = 32 consecutive M/N elements, 4 K rows per 512 B
+// atom, 32 B granule g stored at g ^ (k % 4); LBO = stride between 32-element M/N atoms,
+// SBO = stride between 4-row K groups, K-step(8) = +2*SBO (see mn32_off).
 // TF32 MMA: K = 8 per instruction; fp32 accumulate in TMEM.  fp32 accuracy is recovered
-// with the 3xTF32 split x = hi + lo (hi = cvt.rna.tf32(x), lo = x - hi):
-//   A B ~= A_hi B_hi + A_hi B_lo + A_lo B_hi.
+// with the 3xTF32 split A B ~= A_hi B_hi + A_hi B_lo + A_lo B_hi.  The tensor core reads an
+// fp32 operand as tf32 by truncation (measured), so the raw fp32 copy serves as "hi" and
+// only lo = x - trunc_tf32(x) is stored separately; the older staging path rounds
+// (hi = cvt.rna.tf32(x), lo = x - hi), which is equally exact.
 #pragma once
 
 #include <stdint.h>
@@ -45,6 +49,37 @@ __device__ __forceinline__ uint64_t sdesc(uint32_t saddr, uint32_t lbo, uint32_t
   return d;
 }
 
+// Shared-memory matrix descriptor with an explicit layout type (0 none, 1 128B_BASE32B,
+// 2 128B, 4 64B, 6 32B).
+__device__ __forceinline__ uint64_t sdesc_l(uint32_t saddr, uint32_t lbo, uint32_t sbo, uint32_t layout) {
+  return sdesc(saddr, lbo, sbo) | ((uint64_t)layout << 61);
+}
+
+// Byte offset of (mn, k) in an MN-major SWIZZLE_128B_BASE32B operand whose M/N extent is
+// mnx (multiple of 32), K groups outermost: LBO = 512, SBO = (mnx / 32) * 512.
+__device__ __forceinline__ uint32_t mn32_off(int mn, int k, int mnx) {
+  return (uint32_t)((((k >> 2) * (mnx >> 5) + (mn >> 5)) << 9) + ((k & 3) << 7) +
+                    ((((mn & 31) >> 3) ^ (k & 3)) << 5) + ((mn & 7) << 2));
+}
+
+__device__ __forceinline__ float tf32_trunc(float x) { return __uint_as_float(__float_as_uint(x) & 0xffffe000u); }
+
+// 16-byte global -> shared async copy (L2 only) and its group bookkeeping.
+__device__ __forceinline__ void cp_async16(uint32_t dst, const void* src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+
+// 1-D bulk (TMA engine) global -> shared copy completing `bytes` transactions on mbar.
+// dst, src and bytes must be multiples of 16.
+__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t bytes, uint64_t* mbar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
+               "l"(src), "r"(bytes), "r"(smem_u32(mbar))
+               : "memory");
+}
+
 // Instruction descriptor: kind::tf32, fp32 accumulate.
 __device__ __forceinline__ uint32_t idesc_tf32(int M, int N, bool a_mn_major, bool b_mn_major) {
   uint32_t d = 0;
@@ -76,18 +111,42 @@ __device__ __forceinline__ void mbar_init(uint64_t* mbar, uint32_t count) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(mbar)), "r"(count) : "memory");
 }
 
-__device__ __forceinline__ void mbar_wait(uint64_t* mbar, uint32_t phase) {
+__device__ __forceinline__ bool mbar_try(uint64_t* mbar, uint32_t phase) {
+  uint32_t ok;
   asm volatile(
       "{\n\t.reg .pred P1;\n\t"
-      "WAIT_%=:\n\t"
-      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1, %2;\n\t"
-      "@P1 bra DONE_%=;\n\t"
-      "bra WAIT_%=;\n\t"
-      "DONE_%=:\n\t}\n" ::"r"(smem_u32(mbar)), "r"(phase), "r"(0x989680u) : "memory");
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%1], %2, %3;\n\t"
+      "selp.u32 %0, 1, 0, P1;\n\t}\n"
+      : "=r"(ok)
+      : "r"(smem_u32(mbar)), "r"(phase), "r"(0x989680u)
+      : "memory");
+  return ok != 0;
+}
+
+__device__ __forceinline__ uint64_t globaltimer_ns() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+
+// Wait for the phase with the given parity to complete.  A wait that exceeds 5 s traps
+// (the launch fails with an error instead of hanging the device on a pipeline bug).
+__device__ __forceinline__ void mbar_wait(uint64_t* mbar, uint32_t phase) {
+  if (mbar_try(mbar, phase)) return;
+  const uint64_t t0 = globaltimer_ns();
+  while (!mbar_try(mbar, phase))
+    if (globaltimer_ns() - t0 > 5000000000ull) __trap();
 }
 
 __device__ __forceinline__ void mbar_arrive(uint64_t* mbar) {
   asm volatile("{\n\t.reg .b64 st;\n\tmbarrier.arrive.shared::cta.b64 st, [%0];\n\t}" ::"r"(smem_u32(mbar))
+               : "memory");
+}
+
+// Arrive and add `bytes` to the transaction count the current phase waits for.
+__device__ __forceinline__ void mbar_arrive_tx(uint64_t* mbar, uint32_t bytes) {
+  asm volatile("{\n\t.reg .b64 st;\n\tmbarrier.arrive.expect_tx.shared::cta.b64 st, [%0], %1;\n\t}" ::"r"(smem_u32(mbar)),
+               "r"(bytes)
                : "memory");
 }
 

@@ -59,6 +59,8 @@ struct PlanDev {
   uint32_t* work;                              // dynamic group schedulers [2]
   float *rows, *gbuf, *dabuf, *aggpart;
   float *pbuf, *dpbuf;                         // tensor-core path: P and dL/dP per prefix
+  uint32_t* grp_arow;                          // [P]  C1 row (float offset / R) of sorted prefix q, j1 = 0
+  unsigned long long* grp_c2;                  // [NG] float offset of the C2 slice of group g
 };
 
 struct Ctx {

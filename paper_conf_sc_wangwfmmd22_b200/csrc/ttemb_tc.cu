@@ -2,7 +2,7 @@
 // (kind::tf32, 3xTF32 split, fp32 accumulate in TMEM) and the row stages as
 // high-occupancy warp-per-row-chunk kernels.  SURVEY 8(a) rows a5, a6, a9, a10, a12.
 //
-//   forward   k_tc_p      P_tile = A1 . X1^T           (Reuse buffer) -> Pbuf
+//   forward   k_tc_fwd    P^T = C2^T . A1^T per group  (Reuse buffer) -> Pbuf
 //             k_rows_fwd  E_u = P_q . C3[i3_u]         (Eq. 2)  -> out (one id per bag)
 //                                                               or rows[u] (pooled later)
 //   backward  k_rows_bwd  dP_q += G_u . C3[i3_u]^T     (Eq. 6)    -> dPbuf
@@ -41,6 +41,8 @@ struct TcArgs {
   const TableMeta* meta;
   const uint32_t *counts, *grp_off, *grp_t, *grp_i2, *grp_pfx, *pfx_i1, *pfx_t, *row_seg, *row_i3,
       *row_pfx, *seg_off, *sbag;
+  uint32_t* grp_arow;   // [P]  C1 row index (floats / R) of sorted prefix q at j1 = 0
+  unsigned long long* grp_c2;   // [NG] float offset of group g's C2 slice
   float* pbuf;          // [P][n1][NC]  prefix products (Reuse buffer)
   float* dpbuf;         // [P][n1][NC]  dL/dP per prefix
   float* rows;          // [U][N]
@@ -49,6 +51,9 @@ struct TcArgs {
   float* out;           // [B][T][N]
   uint32_t* work;
   int n1, n2, n3, N, NC, n1s;
+  unsigned long long* trace;   // optional per-CTA role timers (TTEMB_TRACE), 16 slots per CTA
+  int dbg;                     // TTEMB_DBG bit mask (timing experiments only; results invalid)
+  int f_nmb, f_trm, f_nst;   // forward GEMM geometry (k_tc_fwd): M blocks, tile rows, raw slots
   float lr, eps;
   int opt, fused;
 };
@@ -173,107 +178,280 @@ __device__ __forceinline__ const float* c2_slice(const TcArgs& a, uint32_t g) {
 }
 
 // ------------------------------------------------------------------------------------
-// Forward GEMM: P = A1 . X1^T for every group, written to pbuf
+// Forward GEMM, transposed so the prefix rows are the MMA N dimension:
+//   P^T[c][m] = sum_r1 C2[i2][r1][c] . C1[i1_m][j1_m][r1]      (Reuse buffer)
+// M = c (blocks of 128, MN-major operand straight from the row-major C2 slice),
+// N = tile rows rounded up to 16 (K-major C1 rows), K = r1 in stages of 16.
+// Warp roles (288 threads): warps 0-3 load stages with cp.async (no register staging)
+// and write the 3xTF32 "lo" copies; warp 8 issues the MMAs; warps 4-7 drain the TMEM
+// accumulator (double-buffered across tiles) into pbuf[(p, j1)][c] with coalesced stores.
+// Rows of a tile are whole prefixes of one i2-group (up to fg.trm rows).
 // ------------------------------------------------------------------------------------
-// Forward GEMM: P = A1 . X1^T for every group, written to pbuf.  X1 and the TMEM
-// accumulator are double-buffered: MMA(k) runs while chunk k-1's accumulator is drained
-// to pbuf and chunk k+1 is staged.
-__global__ void __launch_bounds__(TNT, 2) k_tc_p(TcArgs a) {
-  extern __shared__ __align__(128) char smem[];
-  float* const xb = reinterpret_cast<float*>(smem);          // X1 buffer b: hi at xb + 2b*TCM/4
-  auto x1h = [&](int b) { return xb + (2 * b) * (TCM / 4); };
-  auto x1l = [&](int b) { return xb + (2 * b + 1) * (TCM / 4); };
-  float* a1h = xb + 4 * (TCM / 4);
-  float* a1l = a1h + TCM / 4;
-  __shared__ uint64_t mbar[2];
-  __shared__ uint32_t s_tmem, s_g[2], s_rowp[2][64], s_rowa[2][64];
-  const int tid = threadIdx.x, w = tid >> 5, lane = tid & 31, q4 = w & 3, half = w >> 2;
-  if (tid == 0) {
-    tc::mbar_init(&mbar[0], 1);
-    tc::mbar_init(&mbar[1], 1);
-    tc::fence_mbar_init();
-    s_g[0] = atomicAdd(a.work, 1u);
-    s_g[1] = atomicAdd(a.work, 1u);
+constexpr int F_LOAD = 128, F_THREADS = 288, F_KS = 16, F_MAXNS = 8;
+
+// Per-step gather tables for the group GEMMs: C1 row of every sorted prefix and the C2
+// slice offset of every group (one level of indirection for the pipelined loaders).
+__global__ void k_tc_prep(TcArgs a) {
+  const uint32_t P = a.counts[kCntP], NG = a.counts[kCntNG];
+  for (uint32_t q = blockIdx.x * blockDim.x + threadIdx.x; q < max(P, NG); q += gridDim.x * blockDim.x) {
+    if (q < P) {
+      const uint32_t p = a.grp_pfx[q];
+      a.grp_arow[q] = (uint32_t)(a.meta[a.pfx_t[p]].c1_off / TR) + (a.pfx_i1[p] << a.n1s);
+    }
+    if (q < NG) a.grp_c2[q] = a.meta[a.grp_t[q]].c2_off + (unsigned long long)a.grp_i2[q] * TR * a.NC;
   }
-  if (tid < 32) tc::tmem_alloc(&s_tmem, 128);
+}
+
+// TTEMB_TRACE instrumentation: clock64 intervals accumulated in registers (trc[k]) and
+// written by each role's leader thread at kernel end to trace[16 * blockIdx.x + k].
+#define TT_T0(v) long long v = a.trace ? clock64() : 0
+#define TT_ADD(k, v, cond)                                                        \
+  do {                                                                            \
+    if (a.trace) {                                                                \
+      const long long _n = clock64();                                             \
+      trc[k] += (unsigned long long)(_n - (v));                                   \
+      v = _n;                                                                     \
+    }                                                                             \
+  } while (0)
+
+struct FwdSmemCtl {
+  uint64_t landed[F_MAXNS], full[2], empty[2], accfull[2], accempty[2], tfull[4], tempty[4];
+  uint32_t cmd[8][4];        // per stage (s & 7): acc slot, k-stage, N, flags (1 last, 2 done)
+  uint32_t srows[8];         // per stage (s & 7): tile rows
+  uint32_t tinfo[4][2];      // tile ring (loaders -> epilogue): first prefix, rows (~0 = done)
+  uint32_t tmem;
+  uint32_t rowp[2][128];     // per accumulator slot: pbuf row of each tile row (epilogue-built)
+};
+
+// Shared memory: NS linear staging slots filled by the bulk-copy (TMA) engine -- stage =
+// 16 consecutive r1 rows of the C2 slice (one contiguous 16*NC*4-byte copy) + 16 r1 of
+// every tile row's C1 row (one 64-byte copy per row) -- then 2 converted slots of "hi"
+// (raw fp32 in MMA layouts: C2 part MN-major mn32_off, C1 part K-major CM) and 2 of "lo"
+// (x - trunc_tf32(x), same layouts).  The loaders convert stage s - LAG while up to LAG
+// newer stages are in flight; the MMA warp consumes converted stages.
+__global__ void __launch_bounds__(F_THREADS, 1) k_tc_fwd(TcArgs a) {
+  extern __shared__ __align__(1024) char smem_raw[];
+  __shared__ FwdSmemCtl ctl;
+  char* const smem = smem_raw + ((1024u - (tc::smem_u32(smem_raw) & 1023u)) & 1023u);   // swizzle atoms
+  const int tid = threadIdx.x, w = tid >> 5, lane = tid & 31;
+  const int NS = a.f_nst, TRM = a.f_trm, MNX = a.f_nmb * 128;
+  const uint32_t SS = 64u * (a.NC + TRM);            // staging bytes per stage (C2 rows, C1 rows)
+  const uint32_t SC = 64u * (MNX + TRM);             // converted bytes per stage (hi or lo)
+  const uint32_t C1OFF = 64u * MNX;                  // C1 part offset inside a converted stage
+  const uint32_t HIB = (uint32_t)NS * SS, LOB = HIB + 2 * SC;
+  if (tid == 0) {
+    for (int b = 0; b < NS; ++b) tc::mbar_init(&ctl.landed[b], 1);
+    for (int b = 0; b < 2; ++b) { tc::mbar_init(&ctl.full[b], F_LOAD); tc::mbar_init(&ctl.empty[b], 1); }
+    for (int s = 0; s < 2; ++s) { tc::mbar_init(&ctl.accfull[s], 1); tc::mbar_init(&ctl.accempty[s], 128); }
+    for (int s = 0; s < 4; ++s) { tc::mbar_init(&ctl.tfull[s], 1); tc::mbar_init(&ctl.tempty[s], 128); }
+    tc::fence_mbar_init();
+  }
+  if (w == 8) tc::tmem_alloc(&ctl.tmem, 512);
   tc::fence_before();
   __syncthreads();
   tc::fence_after();
-  const uint32_t tP0 = s_tmem;
-  uint32_t ph0 = 0u, ph1 = 0u;
+  const uint32_t sbase = tc::smem_u32(smem);
   const uint32_t NG = a.counts[kCntNG];
-  const int PPT = TMT >> a.n1s, NCH = a.NC / TCW;
-  uint32_t g = s_g[0], gnext = s_g[1];
-  int tb = 0;
-  float4 px[4], pa[4];
-  if (g < NG) {
-    fill_table(a, s_rowp[0], s_rowa[0], a.grp_off[g], (int)min((uint32_t)PPT, a.grp_off[g + 1] - a.grp_off[g]));
-    __syncthreads();
-    load_rowq(px, c2_slice(a, g), a.NC, TR);
-    load_tab(pa, a.cores + a.meta[a.grp_t[g]].c1_off, TR, s_rowa[0], false);
-  }
-  // drain the accumulator of chunk kc (buffer b) into pbuf rows of table tbl
-  auto drain = [&](int b, int kc, const uint32_t* tbl) {
-    tc::mbar_wait(&mbar[b], b == 0 ? ph0 : ph1);
-    if (b == 0) ph0 ^= 1u; else ph1 ^= 1u;
-    tc::fence_after();
-    float v[32];
-    tc::tmem_ld32(tc::taddr(tP0 + 64 * b, 32 * q4, 32 * half), v);
-    if (lane < 16) {
-      const uint32_t r = tbl[16 * q4 + lane];
-      if (r != 0xffffffffu) {
-        float* dst = a.pbuf + (size_t)r * a.NC + kc * TCW + 32 * half;
+  const int TPP = TRM >> a.n1s;                        // prefixes per tile
+  unsigned long long trc[14];
 #pragma unroll
-        for (int j = 0; j < 32; j += 4)
-          *reinterpret_cast<float4*>(dst + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
-      }
-    }
-    tc::fence_before();
-  };
-  while (g < NG) {
-    const uint32_t q0 = a.grp_off[g], q1 = a.grp_off[g + 1];
-    const float* C2s = c2_slice(a, g);
-    const uint32_t nmt = (q1 - q0 + PPT - 1) / PPT;
-    for (uint32_t mt = 0; mt < nmt; ++mt) {
-      __syncthreads();
-      store_pat(a1h, a1l, pa);                              // A1 = CM(m, r1)
-      for (int k = 0; k < NCH; ++k) {
-        const int b = k & 1;
-        __syncthreads();                                    // X1[b] readers (MMA k-2) drained below
-        store_pat(x1h(b), x1l(b), px);                      // X1 = CM(c, r1)
-        if (k + 1 < NCH) {
-          load_rowq(px, C2s + (k + 1) * TCW, a.NC, TR);
-        } else {                                            // next tile (or group): table + prefetch
-          uint32_t ng = g, nqa = q0 + (mt + 1) * PPT;
-          if (mt + 1 >= nmt) { ng = gnext; nqa = ng < NG ? a.grp_off[ng] : 0; }
-          if (ng < NG) {
-            fill_table(a, s_rowp[tb ^ 1], s_rowa[tb ^ 1], nqa, (int)min((uint32_t)PPT, a.grp_off[ng + 1] - nqa));
-            __syncthreads();
-            load_rowq(px, c2_slice(a, ng), a.NC, TR);
-            load_tab(pa, a.cores + a.meta[a.grp_t[ng]].c1_off, TR, s_rowa[tb ^ 1], false);
+  for (int k = 0; k < 14; ++k) trc[k] = 0;
+  const long long t_start = a.trace ? clock64() : 0;
+
+  if (w < 4) {
+    // ------------------------------- loaders -------------------------------
+    const int t = tid;
+    const uint32_t LAG = (uint32_t)NS - 2;             // stages in flight behind the newest
+    uint32_t s = 0, i = 0;
+    auto convert = [&](uint32_t sf) {                  // staging -> hi / lo MMA layouts
+      const uint32_t b = sf % NS, l = sf & 1;
+      TT_T0(tt);
+      tc::named_sync(1, F_LOAD);                       // previous convert done (staging reuse)
+      tc::mbar_wait(&ctl.landed[b], (sf / NS) & 1);
+      TT_ADD(2, tt, t == 0);
+      tc::mbar_wait(&ctl.empty[l], ((sf >> 1) & 1) ^ 1);
+      TT_ADD(3, tt, t == 0);
+      const char* st = smem + (size_t)b * SS;
+      char* hi = smem + HIB + (size_t)l * SC;
+      char* lo = smem + LOB + (size_t)l * SC;
+      if (!(a.dbg & 2)) {
+        const int cpr = a.NC >> 2;
+        for (int e = t; e < F_KS * cpr; e += F_LOAD) {
+          const int k = e / cpr, c4 = e - k * cpr;
+          const float4 x = *reinterpret_cast<const float4*>(st + 16 * e);
+          const uint32_t off = tc::mn32_off(4 * c4, k, MNX);
+          *reinterpret_cast<float4*>(hi + off) = x;
+          *reinterpret_cast<float4*>(lo + off) =
+              make_float4(x.x - tc::tf32_trunc(x.x), x.y - tc::tf32_trunc(x.y), x.z - tc::tf32_trunc(x.z),
+                          x.w - tc::tf32_trunc(x.w));
+        }
+        if (t < (int)ctl.srows[sf & 7]) {
+#pragma unroll
+          for (int u = 0; u < F_KS / 4; ++u) {
+            const float4 x = *reinterpret_cast<const float4*>(st + 64 * a.NC + 64 * t + 16 * u);
+            const uint32_t off = C1OFF + tc::cm_off(t, 4 * u, TRM >> 3);
+            *reinterpret_cast<float4*>(hi + off) = x;
+            *reinterpret_cast<float4*>(lo + off) =
+                make_float4(x.x - tc::tf32_trunc(x.x), x.y - tc::tf32_trunc(x.y), x.z - tc::tf32_trunc(x.z),
+                            x.w - tc::tf32_trunc(x.w));
           }
         }
-        publish();
-        if (tid == 0) {
-          mma3(tP0 + 64 * b, a1h, a1l, x1h(b), x1l(b), false);
-          tc::commit(&mbar[b]);
-        }
-        __syncwarp();
-        if (k > 0) drain(b ^ 1, k - 1, s_rowp[tb]);        // overlaps MMA(k)
       }
-      drain((NCH - 1) & 1, NCH - 1, s_rowp[tb]);
-      tb ^= 1;
+      tc::fence_async_smem();
+      tc::mbar_arrive(&ctl.full[l]);
+      TT_ADD(4, tt, t == 0);
+    };
+    // Static round-robin group schedule; the next tile's metadata is loaded two stages
+    // ahead of its use so no dependent global-load chain sits between tiles.
+    const uint32_t j1 = t & ((1u << a.n1s) - 1);
+    uint32_t g = blockIdx.x, q0 = 0, q1 = 0, qa = 0;
+    unsigned long long c2o = 0;
+    uint32_t arow = 0;                                 // C1 row index of this thread's tile row
+    if (g < NG) {
+      q0 = a.grp_off[g]; q1 = a.grp_off[g + 1]; c2o = a.grp_c2[g]; qa = q0;
+      if ((int)t < (int)(min((uint32_t)TPP, q1 - qa) << a.n1s)) arow = a.grp_arow[qa + (t >> a.n1s)] + j1;
     }
-    __syncthreads();
-    if (tid == 0) s_g[1] = atomicAdd(a.work, 1u);
-    __syncthreads();
-    g = gnext;
-    gnext = s_g[1];
+    while (g < NG) {
+      const int rows = (int)min((uint32_t)TPP, q1 - qa) << a.n1s;
+      const int n16 = (rows + 15) & ~15;
+      const uint32_t slot = i & 1;
+      if (t == 0) {                                    // tile ring entry for the epilogue
+        tc::mbar_wait(&ctl.tempty[i & 3], ((i >> 2) & 1) ^ 1);
+        ctl.tinfo[i & 3][0] = qa; ctl.tinfo[i & 3][1] = (uint32_t)rows;
+        tc::mbar_arrive(&ctl.tfull[i & 3]);
+      }
+      const float* C2s = a.cores + c2o;
+      const float* A1r = a.cores + (size_t)arow * TR;
+      // next tile
+      const bool same = qa + TPP < q1;
+      const uint32_t ng = same ? g : g + gridDim.x;
+      uint32_t nq0 = q0, nq1 = q1, narow = 0;
+      unsigned long long nc2 = c2o;
+#pragma unroll 1
+      for (int ks = 0; ks < TR / F_KS; ++ks, ++s) {
+        const uint32_t b = s % NS;
+        TT_T0(tt);
+        if (t == 0) {
+          ctl.cmd[s & 7][0] = slot; ctl.cmd[s & 7][1] = (uint32_t)ks; ctl.cmd[s & 7][2] = (uint32_t)n16;
+          ctl.cmd[s & 7][3] = ks == TR / F_KS - 1 ? 1u : 0u;
+          ctl.srows[s & 7] = (uint32_t)rows;
+          tc::mbar_arrive_tx(&ctl.landed[b], 64u * (a.NC + rows));
+          if (!(a.dbg & 4)) tc::bulk_g2s(sbase + b * SS, C2s + (size_t)ks * F_KS * a.NC, 64u * a.NC, &ctl.landed[b]);
+          else tc::bulk_g2s(sbase + b * SS, C2s, 64u * a.NC, &ctl.landed[b]);
+        }
+        if (t < rows) tc::bulk_g2s(sbase + b * SS + 64u * a.NC + 64u * t, A1r + ks * F_KS, 64u, &ctl.landed[b]);
+        TT_ADD(0, tt, t == 0);
+        if (ks == 0 && !same && ng < NG) { nq0 = a.grp_off[ng]; nq1 = a.grp_off[ng + 1]; nc2 = a.grp_c2[ng]; }
+        if (ks == 2 && ng < NG) {
+          const uint32_t nqa = same ? qa + TPP : nq0;
+          if ((int)t < (int)(min((uint32_t)TPP, nq1 - nqa) << a.n1s)) narow = a.grp_arow[nqa + (t >> a.n1s)] + j1;
+        }
+        TT_ADD(1, tt, t == 0);
+        if (s >= LAG) convert(s - LAG);
+      }
+      ++i;
+      if (same) { qa += TPP; }
+      else { g = ng; q0 = nq0; q1 = nq1; qa = nq0; c2o = nc2; }
+      arow = narow;
+    }
+    for (uint32_t sf = s >= LAG ? s - LAG : 0; sf < s; ++sf) convert(sf);
+    // termination: a "done" tile for the epilogue, a done command for the MMA warp
+    if (t == 0) {
+      tc::mbar_wait(&ctl.tempty[i & 3], ((i >> 2) & 1) ^ 1);
+      ctl.tinfo[i & 3][1] = 0xffffffffu;
+      tc::mbar_arrive(&ctl.tfull[i & 3]);
+    }
+    tc::mbar_wait(&ctl.empty[s & 1], ((s >> 1) & 1) ^ 1);
+    if (t == 0) ctl.cmd[s & 7][3] = 2u;
+    tc::mbar_arrive(&ctl.full[s & 1]);
+  } else if (w == 8) {
+    // ------------------------------- MMA issuer -------------------------------
+    const uint32_t tacc = ctl.tmem;
+    uint32_t i = 0;
+    for (uint32_t s = 0;; ++s) {
+      const uint32_t l = s & 1;
+      TT_T0(tt);
+      tc::mbar_wait(&ctl.full[l], (s >> 1) & 1);
+      TT_ADD(6, tt, lane == 0);
+      tc::fence_after();
+      const uint32_t slot = ctl.cmd[s & 7][0], ks = ctl.cmd[s & 7][1], n16 = ctl.cmd[s & 7][2], fl = ctl.cmd[s & 7][3];
+      if (fl & 2u) break;
+      if (ks == 0) { tc::mbar_wait(&ctl.accempty[slot], ((i >> 1) & 1) ^ 1); tc::fence_after(); }
+      TT_ADD(7, tt, lane == 0);
+      if (lane == 0 && !(a.dbg & 8)) {
+        const uint32_t id = tc::idesc_tf32(128, (int)n16, true, false);
+        const uint32_t rh = sbase + HIB + l * SC, rl = sbase + LOB + l * SC;
+        const uint32_t sboA = (uint32_t)(MNX >> 5) * 512, lboB = (uint32_t)(TRM >> 3) * 128;
+#pragma unroll
+        for (int kk = 0; kk < F_KS / 8; ++kk) {
+          const uint32_t ao = kk * 2 * sboA, bo = C1OFF + kk * 2 * lboB;
+          const uint64_t bh = tc::sdesc(rh + bo, lboB, 128), bl = tc::sdesc(rl + bo, lboB, 128);
+          for (int mb = 0; mb < a.f_nmb; ++mb) {
+            const uint64_t ah = tc::sdesc_l(rh + ao + mb * 2048, 512, sboA, 1);
+            const uint64_t al = tc::sdesc_l(rl + ao + mb * 2048, 512, sboA, 1);
+            const uint32_t d = tacc + slot * 256 + mb * TRM;
+            tc::mma_tf32(d, ah, bh, id, (ks > 0 || kk > 0) ? 1u : 0u);
+            tc::mma_tf32(d, ah, bl, id, 1u);
+            tc::mma_tf32(d, al, bh, id, 1u);
+          }
+        }
+      }
+      if (lane == 0) {
+        tc::commit(&ctl.empty[l]);
+        if (fl & 1u) tc::commit(&ctl.accfull[slot]);
+      }
+      __syncwarp();
+      TT_ADD(8, tt, lane == 0);
+      if (fl & 1u) ++i;
+    }
+  } else {
+    // ------------------------------- epilogue -------------------------------
+    const uint32_t tacc = ctl.tmem;
+    const int q = w & 3;
+    const int et = tid - 128;
+    for (uint32_t i = 0;; ++i) {
+      const uint32_t slot = i & 1;
+      TT_T0(tt);
+      tc::mbar_wait(&ctl.tfull[i & 3], (i >> 2) & 1);
+      TT_ADD(9, tt, et == 0);
+      const uint32_t qa = ctl.tinfo[i & 3][0], rows = ctl.tinfo[i & 3][1];
+      tc::mbar_arrive(&ctl.tempty[i & 3]);
+      if (rows == 0xffffffffu) break;
+      if (et < (int)rows) ctl.rowp[slot][et] = (a.grp_pfx[qa + (et >> a.n1s)] << a.n1s) + (et & ((1 << a.n1s) - 1));
+      tc::named_sync(2, 128);
+      TT_ADD(10, tt, et == 0);
+      tc::mbar_wait(&ctl.accfull[slot], (i >> 1) & 1);
+      TT_ADD(11, tt, et == 0);
+      tc::fence_after();
+      for (int mb = 0; mb < a.f_nmb; ++mb) {
+        const int c = mb * 128 + 32 * q + lane;
+        for (int j0 = 0; j0 < (int)rows; j0 += 32) {
+          float v[32];
+          tc::tmem_ld32(tc::taddr(tacc + slot * 256 + mb * TRM + j0, 32 * q, 0), v);
+          if (c < a.NC && !(a.dbg & 1)) {
+#pragma unroll
+            for (int j = 0; j < 32; ++j)
+              if (j0 + j < (int)rows) a.pbuf[(size_t)ctl.rowp[slot][j0 + j] * a.NC + c] = v[j];
+          }
+        }
+      }
+      tc::fence_before();
+      tc::mbar_arrive(&ctl.accempty[slot]);
+      TT_ADD(12, tt, et == 0);
+      if (a.trace) trc[13] += 1;
+    }
+  }
+  if (a.trace) {
+    const bool lead = tid == 0 || tid == 256 || tid == 128;
+    if (lead)
+      for (int k = 0; k < 14; ++k)
+        if (trc[k]) a.trace[16 * blockIdx.x + k] = trc[k];
+    if (tid == 0) a.trace[16 * blockIdx.x + 14] = (unsigned long long)(clock64() - t_start);
   }
   tc::fence_before();
   __syncthreads();
   tc::fence_after();
-  if (tid < 32) tc::tmem_dealloc(tP0, 128);
+  if (w == 8) tc::tmem_dealloc(ctl.tmem, 512);
 }
 
 // ------------------------------------------------------------------------------------
@@ -749,15 +927,25 @@ TcArgs make_tc_args(Ctx& c, float lr, uint32_t* work, float* out) {
   a.counts = p.counts; a.grp_off = p.grp_off; a.grp_t = p.grp_t; a.grp_i2 = p.grp_i2;
   a.grp_pfx = p.grp_pfx; a.pfx_i1 = p.pfx_i1; a.pfx_t = p.pfx_t; a.row_seg = p.row_seg;
   a.row_i3 = p.row_i3; a.row_pfx = p.row_pfx; a.seg_off = p.seg_off; a.sbag = p.sbag;
+  a.grp_arow = p.grp_arow; a.grp_c2 = p.grp_c2;
   a.pbuf = p.pbuf; a.dpbuf = p.dpbuf; a.rows = p.rows; a.gbuf = p.gbuf; a.dabuf = p.dabuf;
-  a.out = out; a.work = work;
+  a.out = out; a.work = work; a.trace = nullptr;
+  a.dbg = getenv("TTEMB_DBG") ? atoi(getenv("TTEMB_DBG")) : 0;
   a.n1 = c.n1; a.n2 = c.n2; a.n3 = c.n3; a.N = c.N; a.NC = c.NC;
   a.n1s = c.n1 == 1 ? 0 : c.n1 == 2 ? 1 : c.n1 == 4 ? 2 : 3;
+  a.f_nmb = (c.NC + 127) / 128;
+  a.f_trm = a.f_nmb <= 2 ? 128 : a.f_nmb == 3 ? 80 : 64;
+  {   // staging slots: NS * 64 (NC + TRM) + 4 * 64 (MNX + TRM) bytes <= 220 KB
+    const size_t sc = 64u * (a.f_nmb * 128 + a.f_trm), ss = 64u * (c.NC + a.f_trm);
+    a.f_nst = (int)std::min<size_t>(F_MAXNS, (220 * 1024 - 4 * sc) / ss);
+  }
   a.lr = lr; a.eps = c.eps; a.opt = c.opt; a.fused = (c.flags & TTEMB_FUSED_UPDATE) ? 1 : 0;
   return a;
 }
 
-constexpr size_t kTcPSmem = 6 * TCM;
+size_t fwd_smem(const TcArgs& a) {
+  return (size_t)a.f_nst * 64u * (a.NC + a.f_trm) + 4u * 64u * (a.f_nmb * 128 + a.f_trm) + 1024;
+}
 constexpr size_t kTcBwdSmem = 14 * TCM;
 
 }  // namespace
@@ -769,7 +957,7 @@ bool tc_eligible(const Ctx& c) {
 
 cudaError_t configure_tc(Ctx& c) {
   if (!tc_eligible(c)) return cudaSuccess;
-  cudaError_t e = cudaFuncSetAttribute(k_tc_p, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kTcPSmem);
+  cudaError_t e = cudaFuncSetAttribute(k_tc_fwd, cudaFuncAttributeMaxDynamicSharedMemorySize, 222 * 1024);
   if (e != cudaSuccess) return e;
   return cudaFuncSetAttribute(k_tc_bwd2, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kTcBwdSmem);
 }
@@ -779,8 +967,25 @@ cudaError_t run_tc_fwd(Ctx& c, float* out, cudaStream_t s) {
   TcArgs a = make_tc_args(c, 0.f, c.p.work + 0, out);
   {
     StageScope sc(c, ST_FWD_PREFIX, s);
-    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(c.NG_cap, (int64_t)c.sm_count * 2));
-    k_tc_p<<<grid, TNT, kTcPSmem, s>>>(a);
+    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(c.NG_cap, (int64_t)c.sm_count));
+    static unsigned long long* trace = nullptr;
+    if (getenv("TTEMB_TRACE")) {
+      if (!trace) cudaMalloc(&trace, sizeof(unsigned long long) * 16 * grid);
+      cudaMemsetAsync(trace, 0, sizeof(unsigned long long) * 16 * grid, s);
+      a.trace = trace;
+    }
+    k_tc_prep<<<grid_for(c, std::max(c.P_cap, c.NG_cap), 256, 4), 256, 0, s>>>(a);
+    k_tc_fwd<<<grid, F_THREADS, fwd_smem(a), s>>>(a);
+    if (a.trace) {
+      std::vector<unsigned long long> h(16 * grid);
+      cudaMemcpyAsync(h.data(), trace, h.size() * 8, cudaMemcpyDeviceToHost, s);
+      cudaStreamSynchronize(s);
+      double m[16] = {};
+      for (int b = 0; b < grid; ++b) for (int k = 0; k < 16; ++k) m[k] += (double)h[16 * b + k] / grid;
+      fprintf(stderr, "[trace fwd] tiles/CTA %.1f loader-total %.0f | loader: issue %.0f prefetch %.0f landed %.0f empty %.0f convert %.0f -"
+              " | mma: full %.0f accempty %.0f issue %.0f | epi: tinfo %.0f table %.0f accfull %.0f drain %.0f (cycles/CTA)\n",
+              m[13], m[14], m[0], m[1], m[2], m[3], m[4], m[5], m[6], m[7], m[8], m[9], m[10], m[11], m[12]);
+    }
   }
   {
     StageScope sc(c, ST_FWD_ROWS, s);

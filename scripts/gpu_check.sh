@@ -1,5 +1,5 @@
 # GPU round check: parity tests, smoke, short bench (used via gpurun)
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv,noheader
-timeout 1500 python -m pytest tests -m gpu -q --timeout 900 -p no:cacheprovider -x 2>&1 | tail -30
+timeout 600 python -m pytest tests -m gpu -q --timeout 300 -p no:cacheprovider -x 2>&1 | tail -30
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" 2>&1 | tail -3
-timeout 900 python bench.py --steps 10 --warmup 3 --stages ${BENCH_ARGS} > gpurun_out/bench.json 2> gpurun_out/bench.err; tail -25 gpurun_out/bench.err; cat gpurun_out/bench.json
+timeout 300 python bench.py --steps 10 --warmup 3 --stages ${BENCH_ARGS} > gpurun_out/bench.json 2> gpurun_out/bench.err; tail -25 gpurun_out/bench.err; cat gpurun_out/bench.json
