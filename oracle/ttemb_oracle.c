@@ -10,7 +10,7 @@
  *   ttref_digits       pinned: Fig. 5(b) worked example, brute force
  *   ttref_row_*        pinned: dense materialisation + torch embedding_bag,
  *                      R=1 Kronecker closed form, identity-core table
- *   ttref_plan         pinned: numpy.unique / stable argsort
+ *   ttref_plan         pinned: numpy.unique / stable argsort / unravel_index
  *   ttref_forward      pinned: dense embedding_bag on the materialised table
  *   ttref_backward     pinned: torch.autograd, exact central differences
  *   ttref_update       pinned: torch.optim.SGD / torch.optim.Adagrad
@@ -188,13 +188,36 @@ static int64_t find_key(const uint32_t* ukey, int64_t U, uint32_t key) {
 /* ------------------------------------------------------------------------ */
 /* Plan                                                                      */
 /* ------------------------------------------------------------------------ */
-typedef struct { uint32_t t, i2, i1, id; } pf_t;
-static int cmp_pf(const void* x, const void* y) {
-  const pf_t* a = (const pf_t*)x; const pf_t* b = (const pf_t*)y;
-  if (a->t != b->t) return a->t < b->t ? -1 : 1;
-  if (a->i2 != b->i2) return a->i2 < b->i2 ? -1 : 1;
-  if (a->i1 != b->i1) return a->i1 < b->i1 ? -1 : 1;
-  return 0;
+/* The plan orders distinct rows "group-major": by table t, then the C2 digit i2, then the C1
+ * digit i1, then i3 (R23), i.e. by the plan key
+ *     K(t, i) = gbase_t + (i2 * m1 + i1) * m3 + i3,   gbase_t = sum_{t' < t} m1 m2 m3,
+ * with (i1, i2, i3) the digits of Eq. 3.  Rows sharing a prefix (i1, i2) (Alg. 1's
+ * Buf_idx = idx / length_3) are then consecutive, and prefixes sharing a C2 slice
+ * (the i2-groups) are consecutive too. */
+static int plan_keys(const ttref_shape* s, const int64_t* indices, const int64_t* offsets,
+                     int64_t nnz, int32_t B, uint32_t* key, uint32_t* bag_of) {
+  const int T = s->T;
+  if (check_offsets(offsets, (int64_t)T * B, nnz)) return -1;
+  uint64_t gbase = 0;
+  int bad = 0;
+  for (int t = 0; t < T; ++t) {
+    const int32_t* m = s->mfac + 3 * t;
+    for (int32_t b = 0; b < B; ++b) {
+      const int64_t bag = (int64_t)t * B + b;
+      for (int64_t j = offsets[bag]; j < offsets[bag + 1]; ++j) {
+        const int64_t id = indices[j];
+        if (id < 0 || id >= s->rows[t]) { bad = 1; key[j] = (uint32_t)gbase; }
+        else {
+          int64_t d[3];
+          ttref_digits(m, id, d);
+          key[j] = (uint32_t)(gbase + (uint64_t)((d[1] * m[0] + d[0]) * m[2] + d[2]));
+        }
+        bag_of[j] = (uint32_t)((int64_t)b * T + t);
+      }
+    }
+    gbase += (uint64_t)m[0] * m[1] * m[2];
+  }
+  return bad ? -3 : 0;
 }
 
 int ttref_plan(const ttref_shape* s, const int64_t* indices, const int64_t* offsets,
@@ -207,7 +230,7 @@ int ttref_plan(const ttref_shape* s, const int64_t* indices, const int64_t* offs
                int64_t counts[3]) {
   if (check_shape(s) || B < 0 || nnz < 0) return -1;
   uint32_t* key = (uint32_t*)malloc(sizeof(uint32_t) * (size_t)(nnz ? nnz : 1));
-  int rc = build_keys(s, indices, offsets, nnz, B, key, bag_of);
+  int rc = plan_keys(s, indices, offsets, nnz, B, key, bag_of);
   if (rc) { free(key); return rc; }
 
   /* stable sort of (key, position) */
@@ -222,39 +245,37 @@ int ttref_plan(const ttref_shape* s, const int64_t* indices, const int64_t* offs
   }
   seg_off[U] = (uint32_t)nnz;
 
-  /* digits + unique prefixes p = floor(row / m3)  (Alg. 1: Buf_idx = idx / length_3) */
-  int64_t P = 0;
-  uint32_t prev_t = 0xFFFFFFFFu; int64_t prev_p = -1;
+  /* digits back from the plan key; unique prefixes (t, i2, i1) and i2-groups (t, i2) are runs */
+  int64_t P = 0, NG = 0;
   for (int64_t u = 0; u < U; ++u) {
-    uint64_t rb; int t = table_of_key(s, ukey[u], &rb);
-    int64_t row = (int64_t)ukey[u] - (int64_t)rb;
-    int64_t d[3];
-    ttref_digits(s->mfac + 3 * t, row, d);
-    int64_t p = row / s->mfac[3 * t + 2];
-    if ((uint32_t)t != prev_t || p != prev_p) {
-      pfx_t[P] = (uint32_t)t; pfx_i1[P] = (uint32_t)d[0]; pfx_i2[P] = (uint32_t)d[1];
-      row_seg[P] = (uint32_t)u; ++P;
-      prev_t = (uint32_t)t; prev_p = p;
+    uint64_t gbase = 0;
+    int t = 0;
+    for (; t < s->T - 1; ++t) {
+      const int32_t* m = s->mfac + 3 * t;
+      const uint64_t span = (uint64_t)m[0] * m[1] * m[2];
+      if ((uint64_t)ukey[u] < gbase + span) break;
+      gbase += span;
+    }
+    const int32_t* m = s->mfac + 3 * t;
+    const uint64_t local = (uint64_t)ukey[u] - gbase;
+    const uint32_t i3 = (uint32_t)(local % (uint64_t)m[2]);
+    const uint64_t pq = local / (uint64_t)m[2];           /* i2 * m1 + i1 */
+    const uint32_t i1 = (uint32_t)(pq % (uint64_t)m[0]), i2 = (uint32_t)(pq / (uint64_t)m[0]);
+    if (P == 0 || pfx_t[P - 1] != (uint32_t)t || pfx_i2[P - 1] != i2 || pfx_i1[P - 1] != i1) {
+      if (P == 0 || pfx_t[P - 1] != (uint32_t)t || pfx_i2[P - 1] != i2) {
+        grp_off[NG] = (uint32_t)P; grp_t[NG] = (uint32_t)t; grp_i2[NG] = i2; ++NG;
+      }
+      pfx_t[P] = (uint32_t)t; pfx_i1[P] = i1; pfx_i2[P] = i2; row_seg[P] = (uint32_t)u;
+      grp_pfx[P] = (uint32_t)P;
+      ++P;
     }
     row_pfx[u] = (uint32_t)(P - 1);
-    row_i3[u] = (uint32_t)d[2];
+    row_i3[u] = i3;
   }
   row_seg[P] = (uint32_t)U;
-
-  /* prefixes ordered by (t, i2, i1): the i2-groups sharing one C2 slice */
-  pf_t* pf = (pf_t*)malloc(sizeof(pf_t) * (size_t)(P ? P : 1));
-  for (int64_t q = 0; q < P; ++q) { pf[q].t = pfx_t[q]; pf[q].i2 = pfx_i2[q]; pf[q].i1 = pfx_i1[q]; pf[q].id = (uint32_t)q; }
-  qsort(pf, (size_t)P, sizeof(pf_t), cmp_pf);
-  int64_t NG = 0;
-  for (int64_t q = 0; q < P; ++q) {
-    grp_pfx[q] = pf[q].id;
-    if (q == 0 || pf[q].t != pf[q - 1].t || pf[q].i2 != pf[q - 1].i2) {
-      grp_off[NG] = (uint32_t)q; grp_t[NG] = pf[q].t; grp_i2[NG] = pf[q].i2; ++NG;
-    }
-  }
   grp_off[NG] = (uint32_t)P;
   counts[0] = U; counts[1] = P; counts[2] = NG;
-  free(pf); free(v); free(key);
+  free(v); free(key);
   return 0;
 }
 

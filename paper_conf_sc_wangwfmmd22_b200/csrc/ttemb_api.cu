@@ -74,7 +74,7 @@ int validate(const ttemb_config* cfg) {
   if ((int64_t)cfg->num_tables * cfg->max_batch > (int64_t(1) << 31)) return TTEMB_ERR_UNSUPPORTED;
   if (cfg->optimizer != TTEMB_SGD && cfg->optimizer != TTEMB_ADAGRAD) return TTEMB_ERR_INVALID_ARG;
   if (cfg->flags & ~(TTEMB_FUSED_UPDATE | TTEMB_FP32_CORES)) return TTEMB_ERR_INVALID_ARG;
-  uint64_t total = 0, buckets = 0;
+  uint64_t total = 0, buckets = 0, keys = 0;
   for (int t = 0; t < cfg->num_tables; ++t) {
     const ttemb_table& tb = cfg->tables[t];
     const int64_t m1 = tb.row_factors[0], m2 = tb.row_factors[1], m3 = tb.row_factors[2];
@@ -83,8 +83,9 @@ int validate(const ttemb_config* cfg) {
     if (m1 > (1 << 24) || m2 > (1 << 24) || m3 > (1 << 24)) return TTEMB_ERR_UNSUPPORTED;
     total += (uint64_t)tb.num_rows;
     buckets += (uint64_t)m2;
+    keys += (uint64_t)(m1 * m2 * m3);
   }
-  if (total > 0xFFFFFFFFull || buckets > 0xFFFFFFFFull) return TTEMB_ERR_UNSUPPORTED;
+  if (total > 0xFFFFFFFFull || buckets > 0xFFFFFFFFull || keys > 0xFFFFFFFFull) return TTEMB_ERR_UNSUPPORTED;
   return TTEMB_OK;
 }
 
@@ -100,7 +101,7 @@ void plan_sizes(const ttemb_config* cfg, Ctx& c) {
   const size_t s1 = (size_t)c.n1 * c.R, s2 = (size_t)c.R * c.n2 * c.R, s3 = (size_t)c.R * c.n3;
   auto up4 = [](size_t x) { return (x + 3) & ~(size_t)3; };
   size_t off = 0;
-  uint64_t rb = 0, pfx = 0;
+  uint64_t rb = 0, pfx = 0, kb = 0;
   uint32_t gb = 0;
   for (int t = 0; t < c.T; ++t) {   // [C1 of all tables]
     const ttemb_table& tb = cfg->tables[t];
@@ -108,18 +109,21 @@ void plan_sizes(const ttemb_config* cfg, Ctx& c) {
     m.m1 = tb.row_factors[0]; m.m2 = tb.row_factors[1]; m.m3 = tb.row_factors[2];
     m.M = (uint32_t)tb.num_rows;
     m.rowbase = rb; rb += (uint64_t)tb.num_rows;
+    m.kbase = kb; kb += (uint64_t)m.m1 * m.m2 * m.m3;
     m.grpbase = gb; gb += m.m2;
     pfx += (uint64_t)((tb.num_rows + m.m3 - 1) / m.m3);
     m.c1_off = off; off += up4(m.m1 * s1);
   }
+  c.c1_floats = off;
   for (int t = 0; t < c.T; ++t) { c.meta[t].c2_off = off; off += up4(c.meta[t].m2 * s2); }
   c.c3_begin = off;
   for (int t = 0; t < c.T; ++t) { c.meta[t].c3_off = off; off += up4(c.meta[t].m3 * s3); }
   c.c3_floats = off - c.c3_begin;
   c.core_floats = off;
   c.total_rows = rb;
+  c.total_keys = kb;
   c.total_buckets = gb;
-  c.key_passes = std::max(1, (bits_for(rb ? rb - 1 : 0) + 7) / 8);
+  c.key_passes = std::max(1, (bits_for(kb ? kb - 1 : 0) + 7) / 8);
   c.gkey_passes = std::max(1, (bits_for(gb ? gb - 1 : 0) + 7) / 8);
   c.U_cap = std::min<int64_t>(c.max_nnz, (int64_t)rb);
   c.P_cap = std::min<int64_t>(c.U_cap, (int64_t)pfx);
@@ -138,7 +142,7 @@ size_t carve(Ctx& c, uint8_t* base) {
   const int64_t bags = (int64_t)c.T * c.max_batch;
   PlanDev& p = c.p;
   c.d_meta = k.take<TableMeta>(c.T);
-  c.d_rowbase = k.take<uint64_t>(c.T + 1);
+  c.d_kbase = k.take<uint64_t>(c.T + 1);
   c.d_grpbase = k.take<uint32_t>(c.T + 1);
   // --- zeroed every forward ---
   k.off = (k.off + 255) & ~(size_t)255;
@@ -273,13 +277,14 @@ int ttemb_create(const ttemb_config* cfg, int device, void* cores, void* state, 
   c.sm_count = prop.multiProcessorCount;
   std::vector<uint64_t> rb(c.T + 1);
   std::vector<uint32_t> gb(c.T + 1);
-  for (int t = 0; t < c.T; ++t) { rb[t] = c.meta[t].rowbase; gb[t] = c.meta[t].grpbase; }
-  rb[c.T] = c.total_rows; gb[c.T] = c.total_buckets;
+  for (int t = 0; t < c.T; ++t) { rb[t] = c.meta[t].kbase; gb[t] = c.meta[t].grpbase; }
+  rb[c.T] = c.total_keys; gb[c.T] = c.total_buckets;
   cudaError_t e = cudaMemcpy(c.d_meta, c.meta.data(), sizeof(TableMeta) * c.T, cudaMemcpyHostToDevice);
-  if (e == cudaSuccess) e = cudaMemcpy(c.d_rowbase, rb.data(), sizeof(uint64_t) * (c.T + 1), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(c.d_kbase, rb.data(), sizeof(uint64_t) * (c.T + 1), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(c.d_grpbase, gb.data(), sizeof(uint32_t) * (c.T + 1), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = configure_group(c);
   if (e == cudaSuccess) e = configure_tc(c);
+  if (e == cudaSuccess) e = configure_fused(c);
   if (e != cudaSuccess) {
     fprintf(stderr, "ttemb_create: %s\n", cudaGetErrorString(e));
     delete h;

@@ -133,71 +133,33 @@ struct BwdArgs {
   int opt, fused;
 };
 
-// a11: dC1[t][i1] = sum of the dA partials of the contiguous (t, i1) prefix run, as a
-// fixed-chunk segmented reduction (deterministic, balanced under long hot runs):
-// part 1: thread = (chunk of DC1_CS prefixes, element); runs fully inside the chunk are
-// finished here, partial runs leave head/tail partials; part 2 joins them.
-constexpr int DC1_CS = 16;
-
-__device__ __forceinline__ bool same_run(const BwdArgs& a, uint32_t p, uint32_t q) {
-  return a.pfx_t[p] == a.pfx_t[q] && a.pfx_i1[p] == a.pfx_i1[q];
-}
-
-__device__ __forceinline__ void dc1_finish(const BwdArgs& a, uint32_t p, int k, float g) {
-  const int S1 = a.n1 * a.R;
-  const size_t idx = a.meta[a.pfx_t[p]].c1_off + (size_t)a.pfx_i1[p] * S1 + k;
-  if (a.fused) apply_update(a.cores + idx, a.state + idx, g, a.lr, a.eps, a.opt);
-  else a.grads[idx] = g;
-}
-
-__global__ void __launch_bounds__(256) k_dc1(BwdArgs a, float* __restrict__ part) {
-  const int S1 = a.n1 * a.R;
+// a11: dC1[t][i1] = sum of the dA partials of every prefix with that (t, i1).  In the
+// group-major plan those prefixes are spread over the i2-groups, so the partials are added
+// into the (zeroed, L2-resident) C1 gradient region with vector reductions (Fig. 6(a) step 2,
+// P:191); the fused path then updates C1 densely together with C3.
+__global__ void __launch_bounds__(256) k_dc1(BwdArgs a) {
+  const int S4 = (a.n1 * a.R) >> 2;
   const uint32_t P = a.counts[kCntP];
-  const int64_t nch = (P + DC1_CS - 1) / DC1_CS;
-  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < nch * S1;
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < (int64_t)P * S4;
        e += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t ch = e / S1;
-    const int k = (int)(e - ch * S1);
-    const uint32_t p0 = (uint32_t)(ch * DC1_CS), p1 = min((uint32_t)(p0 + DC1_CS), P);
-    const bool starts_before = p0 > 0 && same_run(a, p0, p0 - 1);
-    float acc = 0.f;
-    bool head = starts_before;
-    for (uint32_t p = p0; p < p1; ++p) {
-      acc += __ldg(a.dabuf + (size_t)p * S1 + k);
-      const bool run_end = (p + 1 == P) || !same_run(a, p, p + 1);
-      if (run_end || p + 1 == p1) {
-        if (head) part[((size_t)ch * 2 + 0) * S1 + k] = acc;          // began in an earlier chunk
-        else if (run_end) dc1_finish(a, p, k, acc);                   // whole run in this chunk
-        else part[((size_t)ch * 2 + 1) * S1 + k] = acc;               // continues after
-        acc = 0.f;
-        head = false;
-      }
-    }
+    const uint32_t q = (uint32_t)(e / S4);
+    const int k4 = (int)(e - (int64_t)q * S4);
+    const float4 v = __ldg(reinterpret_cast<const float4*>(a.dabuf) + e);
+    float* dst = a.grads + a.meta[a.pfx_t[q]].c1_off + (size_t)a.pfx_i1[q] * (4 * S4) + 4 * k4;
+    asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(dst), "f"(v.x), "f"(v.y), "f"(v.z),
+                 "f"(v.w)
+                 : "memory");
   }
 }
 
-__global__ void __launch_bounds__(256) k_dc1_fix(BwdArgs a, const float* __restrict__ part) {
+__global__ void __launch_bounds__(256) k_dc1_scalar(BwdArgs a) {
   const int S1 = a.n1 * a.R;
   const uint32_t P = a.counts[kCntP];
-  const int64_t nch = (P + DC1_CS - 1) / DC1_CS;
-  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < nch * S1;
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < (int64_t)P * S1;
        e += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t ch = e / S1;
-    const int k = (int)(e - ch * S1);
-    const uint32_t p0 = (uint32_t)(ch * DC1_CS);
-    if (p0 == 0 || !same_run(a, p0, p0 - 1)) continue;       // no run enters this chunk
-    const uint32_t p1 = min((uint32_t)(p0 + DC1_CS), P);
-    uint32_t pe = p0;                                          // last prefix of the entering run
-    while (pe + 1 < p1 && same_run(a, pe, pe + 1)) ++pe;
-    if (pe + 1 < P && same_run(a, pe, pe + 1)) continue;       // run continues past this chunk
-    int64_t c0 = ch - 1;                                       // chunk where the run started
-    while (c0 > 0 && same_run(a, (uint32_t)(c0 * DC1_CS), p0) &&
-           same_run(a, (uint32_t)(c0 * DC1_CS), (uint32_t)(c0 * DC1_CS) - 1))
-      --c0;
-    float g = part[((size_t)c0 * 2 + 1) * S1 + k];
-#pragma unroll 8
-    for (int64_t c = c0 + 1; c <= ch; ++c) g += part[((size_t)c * 2 + 0) * S1 + k];
-    dc1_finish(a, p0, k, g);
+    const uint32_t q = (uint32_t)(e / S1);
+    const int k = (int)(e - (int64_t)q * S1);
+    atomicAdd(a.grads + a.meta[a.pfx_t[q]].c1_off + (size_t)a.pfx_i1[q] * S1 + k, __ldg(a.dabuf + e));
   }
 }
 
@@ -217,15 +179,19 @@ k_update(float* __restrict__ cores, float* __restrict__ state, const float* __re
 cudaError_t run_group_bwd(Ctx& c, float lr, cudaStream_t s);
 
 int64_t agg_chunks(int64_t nnz) { return (nnz + AGG_CS - 1) / AGG_CS; }
-int64_t dc1_chunks(int64_t P) { return (P + DC1_CS - 1) / DC1_CS; }
+int64_t dc1_chunks(int64_t P) { return 1; }
 
 cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s) {
   const PlanDev& p = c.p;
   const bool fused = (c.flags & TTEMB_FUSED_UPDATE) != 0;
   {
     StageScope sc(c, ST_BWD_ZERO, s);
-    if (fused) cudaMemsetAsync(c.grads + c.c3_begin, 0, sizeof(float) * c.c3_floats, s);
-    else cudaMemsetAsync(c.grads, 0, sizeof(float) * c.core_floats, s);
+    if (fused) {
+      cudaMemsetAsync(c.grads, 0, sizeof(float) * c.c1_floats, s);
+      cudaMemsetAsync(c.grads + c.c3_begin, 0, sizeof(float) * c.c3_floats, s);
+    } else {
+      cudaMemsetAsync(c.grads, 0, sizeof(float) * c.core_floats, s);
+    }
   }
   if (c.nnz > 0) {
     StageScope sc(c, ST_AGG, s);
@@ -255,15 +221,18 @@ cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s
     if (e != cudaSuccess) return e;
     {
       StageScope sc(c, ST_DC1, s);
-      const int64_t items = cdiv(c.P_cap, DC1_CS) * c.n1 * c.R;
-      k_dc1<<<grid_for(c, items, 256, 32), 256, 0, s>>>(a, p.aggpart);
-      k_dc1_fix<<<grid_for(c, items, 256, 32), 256, 0, s>>>(a, p.aggpart);
+      if ((c.n1 * c.R) % 4 == 0)
+        k_dc1<<<grid_for(c, c.P_cap * c.n1 * c.R / 4, 256, 32), 256, 0, s>>>(a);
+      else
+        k_dc1_scalar<<<grid_for(c, c.P_cap * c.n1 * c.R, 256, 32), 256, 0, s>>>(a);
     }
   }
-  if (fused) {
+  if (fused) {   // C2 was updated inside the group kernel; C1 and C3 densely here
     StageScope sc(c, ST_UPD_C3, s);
     k_update<<<grid_for(c, (int64_t)c.c3_floats, 256, 32), 256, 0, s>>>(
         c.cores, c.state, c.grads, c.c3_begin, c.c3_floats, lr, c.eps, c.opt);
+    k_update<<<grid_for(c, (int64_t)c.c1_floats, 256, 32), 256, 0, s>>>(
+        c.cores, c.state, c.grads, 0, c.c1_floats, lr, c.eps, c.opt);
   }
   return cudaGetLastError();
 }

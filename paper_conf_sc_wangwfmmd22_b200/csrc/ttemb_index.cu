@@ -1,16 +1,19 @@
 // ttemb_index.cu -- the index stage, sm_100a.
 //
-//   a1 key build + range check: key_j = rowbase_t + id_j, bag_of_j = b*T + t  (Eq. 3
-//      needs the per-table row id)
+//   a1 key build + range check: the group-major plan key
+//        key_j = kbase_t + (i2 m1 + i1) m3 + i3     ((i1, i2, i3) = Eq. 3 digits of id_j)
+//      and bag_of_j = b*T + t.  Sorting by this key puts duplicates, then rows of one prefix
+//      (i1, i2) (Alg. 1's Buf_idx = idx / length_3), then prefixes of one C2 slice
+//      (the i2-groups) next to each other, so one sort yields the whole plan.
 //   a2 stable LSD radix sort of the 32-bit keys carrying positions (onesweep: an
 //      upfront digit histogram, then one kernel per 8-bit pass with warp-level
 //      match_any ranking and decoupled look-back across tiles)
 //   a3 unique rows, segment offsets, inverse map (single-pass scan with warp
 //      ballots and decoupled look-back) -- "compute the unique embeddings within a
 //      batch"
-//   a4 TT digits and unique prefixes p = floor(row/m3) (Alg. 1's Buf_idx = idx /
-//      length_3), then prefixes regrouped by (t, i2) with a second radix sort
-//      so one CTA owns each C2 slice (replaces Alg. 1's flag array).
+//   a4 TT digits, unique prefixes (runs of (t, i2, i1)) and i2-groups (runs of (t, i2))
+//      as two more single-pass scans, so one CTA owns each C2 slice (replaces Alg. 1's
+//      flag array).
 // Everything here is integer work and bit-exact against oracle/ttemb_oracle.c.
 #include "ttemb_internal.cuh"
 
@@ -136,7 +139,7 @@ __device__ __forceinline__ uint32_t block_excl_scan_256(uint32_t v, uint32_t* s_
 template <typename IdxT>
 __global__ void __launch_bounds__(256)
 k_build_keys(const IdxT* __restrict__ indices, const int64_t* __restrict__ offsets, int64_t nnz,
-             int32_t B, int T, const uint64_t* __restrict__ rowbase, uint32_t* __restrict__ keys,
+             int32_t B, int T, const TableMeta* __restrict__ meta, uint32_t* __restrict__ keys,
              uint32_t* __restrict__ bag_of, uint32_t* __restrict__ counts, int passes,
              uint32_t* __restrict__ hist) {
   __shared__ uint32_t sh[4][256];
@@ -153,14 +156,17 @@ k_build_keys(const IdxT* __restrict__ indices, const int64_t* __restrict__ offse
     if (e - s != 1) multi = 1u;
     const int t = (int)(b / B);
     const int64_t bb = b - (int64_t)t * B;
-    const uint64_t rb = __ldg(rowbase + t);
-    const uint64_t M = __ldg(rowbase + t + 1) - rb;
+    const TableMeta& mt = meta[t];
+    const uint32_t kb = (uint32_t)mt.kbase, M = mt.M, m1 = mt.m1, m2 = mt.m2, m3 = mt.m3;
     const uint32_t bo = (uint32_t)(bb * T + t);
     for (int64_t j = s; j < e; ++j) {
       const int64_t id = (int64_t)indices[j];
-      uint32_t key = (uint32_t)rb;
+      uint32_t key = kb;
       if (id < 0 || (uint64_t)id >= M) err |= kErrRange;
-      else key = (uint32_t)(rb + (uint64_t)id);
+      else {
+        const uint32_t r = (uint32_t)id, p = r / m3, i3 = r - p * m3, i1 = p / m2, i2 = p - i1 * m2;
+        key = kb + (i2 * m1 + i1) * m3 + i3;
+      }
       keys[j] = key;
       bag_of[j] = bo;
       for (int p = 0; p < passes; ++p) atomicAdd(&sh[p][(key >> (8 * p)) & 255u], 1u);
@@ -372,28 +378,28 @@ struct UniqueBody {
   __device__ void finish(uint32_t U) const { counts[kCntU] = U; seg_off[U] = nnz; }
 };
 
-__device__ __forceinline__ int table_of_key(const uint64_t* rowbase, int T, uint32_t key) {
-  int lo = 0, hi = T - 1;   // last t with rowbase[t] <= key
+__device__ __forceinline__ int table_of_key(const uint64_t* kbase, int T, uint32_t key) {
+  int lo = 0, hi = T - 1;   // last t with kbase[t] <= key
   while (lo < hi) {
     const int mid = (lo + hi + 1) >> 1;
-    if (__ldg(rowbase + mid) <= key) lo = mid; else hi = mid - 1;
+    if (__ldg(kbase + mid) <= key) lo = mid; else hi = mid - 1;
   }
   return lo;
 }
 
-// a4: TT digits (Eq. 3) and unique prefixes over the unique rows
+// a4: TT digits (Eq. 3) and unique prefixes (runs of (t, i2 m1 + i1)) over the unique rows
 struct PrefixBody {
-  const uint32_t* ukey; const uint64_t* rowbase; const TableMeta* meta; int T;
+  const uint32_t* ukey; const uint64_t* kbase; const TableMeta* meta; int T;
   uint32_t* row_pfx; uint32_t* row_i3; uint32_t* pfx_t; uint32_t* pfx_i1; uint32_t* pfx_i2;
-  uint32_t* row_seg; uint32_t* gkey; uint32_t* gval; uint32_t* counts;
+  uint32_t* row_seg; uint32_t* counts;
   __device__ uint32_t size() const { return counts[kCntU]; }
-  __device__ void decode(uint32_t u, int& t, uint32_t& p, uint32_t& i3) const {
+  __device__ void decode(uint32_t u, int& t, uint32_t& pq, uint32_t& i3) const {
     const uint32_t key = ukey[u];
-    t = table_of_key(rowbase, T, key);
-    const uint32_t row = (uint32_t)(key - __ldg(rowbase + t));
+    t = table_of_key(kbase, T, key);
+    const uint32_t local = (uint32_t)(key - __ldg(kbase + t));
     const uint32_t m3 = meta[t].m3;
-    p = row / m3;
-    i3 = row - p * m3;
+    pq = local / m3;                  // i2 * m1 + i1
+    i3 = local - pq * m3;
   }
   __device__ bool flag(uint32_t u) const {
     if (u == 0) return true;
@@ -403,39 +409,31 @@ struct PrefixBody {
     return t0 != t1 || p0 != p1;
   }
   __device__ void emit(uint32_t u, uint32_t slot, uint32_t f) const {
-    int t; uint32_t p, i3;
-    decode(u, t, p, i3);
+    int t; uint32_t pq, i3;
+    decode(u, t, pq, i3);
     const uint32_t q = f ? slot : slot - 1;
     row_pfx[u] = q;
     row_i3[u] = i3;
     if (f) {
-      const uint32_t m2 = meta[t].m2;
-      const uint32_t i1 = p / m2, i2 = p - i1 * m2;
+      const uint32_t m1 = meta[t].m1;
+      const uint32_t i2 = pq / m1, i1 = pq - i2 * m1;
       pfx_t[q] = (uint32_t)t; pfx_i1[q] = i1; pfx_i2[q] = i2; row_seg[q] = u;
-      gkey[q] = meta[t].grpbase + i2;
-      gval[q] = q;
     }
   }
   __device__ void finish(uint32_t P) const { counts[kCntP] = P; row_seg[P] = counts[kCntU]; }
 };
 
-// i2-groups over the (t, i2)-sorted prefixes
+// i2-groups: runs of (t, i2) over the prefixes (already in group-major order)
 struct GroupBody {
-  const uint32_t* gkey; const uint32_t* gval; const uint32_t* grpbase; int T;
+  const uint32_t* pfx_t; const uint32_t* pfx_i2;
   uint32_t* grp_pfx; uint32_t* grp_off; uint32_t* grp_t; uint32_t* grp_i2; uint32_t* counts;
   __device__ uint32_t size() const { return counts[kCntP]; }
-  __device__ bool flag(uint32_t q) const { return q == 0 || gkey[q] != gkey[q - 1]; }
+  __device__ bool flag(uint32_t q) const {
+    return q == 0 || pfx_t[q] != pfx_t[q - 1] || pfx_i2[q] != pfx_i2[q - 1];
+  }
   __device__ void emit(uint32_t q, uint32_t slot, uint32_t f) const {
-    grp_pfx[q] = gval[q];
-    if (f) {
-      const uint32_t k = gkey[q];
-      int lo = 0, hi = T - 1;
-      while (lo < hi) {
-        const int mid = (lo + hi + 1) >> 1;
-        if (__ldg(grpbase + mid) <= k) lo = mid; else hi = mid - 1;
-      }
-      grp_off[slot] = q; grp_t[slot] = (uint32_t)lo; grp_i2[slot] = k - __ldg(grpbase + lo);
-    }
+    grp_pfx[q] = q;
+    if (f) { grp_off[slot] = q; grp_t[slot] = pfx_t[q]; grp_i2[slot] = pfx_i2[q]; }
   }
   __device__ void finish(uint32_t NG) const { counts[kCntNG] = NG; grp_off[NG] = counts[kCntP]; }
 };
@@ -487,11 +485,11 @@ cudaError_t run_index_stage(Ctx& c, const void* indices, const int64_t* offsets,
     const int g = grid_for(c, bags > 0 ? bags : 1, 256, 32);
     if (c.index_bits == 64)
       k_build_keys<int64_t><<<g, 256, 0, s>>>((const int64_t*)indices, offsets, nnz, c.B, c.T,
-                                              c.d_rowbase, p.keysA, p.bag_of, p.counts,
+                                              c.d_meta, p.keysA, p.bag_of, p.counts,
                                               c.key_passes, p.hist1);
     else
       k_build_keys<int32_t><<<g, 256, 0, s>>>((const int32_t*)indices, offsets, nnz, c.B, c.T,
-                                              c.d_rowbase, p.keysA, p.bag_of, p.counts,
+                                              c.d_meta, p.keysA, p.bag_of, p.counts,
                                               c.key_passes, p.hist1);
   }
   // a2: sort (key, position)
@@ -501,9 +499,6 @@ cudaError_t run_index_stage(Ctx& c, const void* indices, const int64_t* offsets,
                                ST_SORT_HIST, ST_SORT_PASS, s, /*have_hist=*/true);
   p.skey = which ? p.keysB : p.keysA;
   p.spos = which ? p.valsB : p.valsA;
-  // the other ping-pong pair is free now: group-sort buffers
-  p.gkeyA = which ? p.keysA : p.keysB;
-  p.gvalA = which ? p.valsA : p.valsB;
   // a3
   {
     StageScope sc(c, ST_UNIQUE, s);
@@ -512,25 +507,18 @@ cudaError_t run_index_stage(Ctx& c, const void* indices, const int64_t* offsets,
     const int64_t tiles = scan_tiles(nnz);
     k_scan<UniqueBody><<<(unsigned)(tiles ? tiles : 1), SC_T, 0, s>>>(b, p.sc_status, p.sc_counter + 0);
   }
-  // a4: digits + prefixes
+  // a4: digits + prefixes, then i2-groups
   {
     StageScope sc(c, ST_PREFIX, s);
-    PrefixBody b{p.ukey, c.d_rowbase, c.d_meta, c.T, p.row_pfx, p.row_i3, p.pfx_t, p.pfx_i1,
-                 p.pfx_i2, p.row_seg, p.gkeyA, p.gvalA, p.counts};
+    PrefixBody b{p.ukey, c.d_kbase, c.d_meta, c.T, p.row_pfx, p.row_i3, p.pfx_t, p.pfx_i1,
+                 p.pfx_i2, p.row_seg, p.counts};
     const int64_t tiles = scan_tiles(c.U_cap);
     k_scan<PrefixBody><<<(unsigned)(tiles ? tiles : 1), SC_T, 0, s>>>(
         b, p.sc_status + c.sc_tiles, p.sc_counter + 1);
   }
-  // group sort by (t, i2), stable (keeps i1 ascending inside a group)
-  const int64_t tiles2 = radix_tiles(c.P_cap);
-  const int which2 = radix_sort(c, p.gkeyA, p.gvalA, p.gkeyB, p.gvalB, p.counts + kCntP, 0, c.P_cap,
-                                c.gkey_passes, p.hist2, p.dbase2, p.rs2_counter, p.rs2_status,
-                                tiles2, ST_GSORT_HIST, ST_GSORT_PASS, s);
-  p.gkey = which2 ? p.gkeyB : p.gkeyA;
-  p.gval = which2 ? p.gvalB : p.gvalA;
   {
     StageScope sc(c, ST_GROUPS, s);
-    GroupBody b{p.gkey, p.gval, c.d_grpbase, c.T, p.grp_pfx, p.grp_off, p.grp_t, p.grp_i2, p.counts};
+    GroupBody b{p.pfx_t, p.pfx_i2, p.grp_pfx, p.grp_off, p.grp_t, p.grp_i2, p.counts};
     const int64_t tiles = scan_tiles(c.P_cap);
     k_scan<GroupBody><<<(unsigned)(tiles ? tiles : 1), SC_T, 0, s>>>(
         b, p.sc_status + 2 * c.sc_tiles, p.sc_counter + 2);

@@ -35,7 +35,8 @@ enum Stage : int {
 
 struct TableMeta {
   uint32_t m1, m2, m3, M;      // row factors, rows (M <= 2^32-1 checked on host)
-  uint64_t rowbase;            // first key of the table (exclusive prefix sum of M)
+  uint64_t rowbase;            // exclusive prefix sum of M (row numbering across tables)
+  uint64_t kbase;              // first plan key of the table: exclusive prefix sum of m1 m2 m3
   uint64_t c1_off, c2_off, c3_off;  // float offsets into cores / grads / state
   uint32_t grpbase;            // first (t, i2) bucket id = sum of m2 of earlier tables
   uint32_t pad;
@@ -72,13 +73,13 @@ struct Ctx {
   uint32_t flags = 0;
   int64_t max_nnz = 0;
   int32_t max_batch = 0;
-  uint64_t total_rows = 0;
+  uint64_t total_rows = 0, total_keys = 0;
   uint32_t total_buckets = 0;
   int key_passes = 1, gkey_passes = 1;
   int64_t U_cap = 0, P_cap = 0, NG_cap = 0;
   int64_t rs1_tiles = 0, rs2_tiles = 0, sc_tiles = 0;
   std::vector<TableMeta> meta;
-  size_t core_floats = 0, c3_begin = 0, c3_floats = 0;
+  size_t core_floats = 0, c1_floats = 0, c3_begin = 0, c3_floats = 0;
 
   // caller buffers
   float* cores = nullptr;
@@ -88,7 +89,7 @@ struct Ctx {
 
   // workspace carve
   TableMeta* d_meta = nullptr;
-  uint64_t* d_rowbase = nullptr;     // [T+1]
+  uint64_t* d_kbase = nullptr;       // [T+1] plan-key base of every table (+ total)
   uint32_t* d_grpbase = nullptr;     // [T+1]
   PlanDev p{};
   uint8_t* zero_begin = nullptr;
@@ -130,6 +131,9 @@ cudaError_t configure_tc(Ctx& c);
 bool tc_eligible(const Ctx& c);
 cudaError_t run_tc_fwd(Ctx& c, float* out, cudaStream_t s);
 cudaError_t run_tc_bwd(Ctx& c, float lr, cudaStream_t s);
+bool fused_eligible(const Ctx& c);
+cudaError_t configure_fused(Ctx& c);
+cudaError_t run_fused_fwd(Ctx& c, cudaStream_t s);
 
 // ---- small helpers -------------------------------------------------------------------
 static inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }

@@ -54,3 +54,19 @@ def assert_update_close(got_p, ref_p, p_old, g_ref, g_abs, lr, opt, tol=1e-4, go
         i = np.flatnonzero(bad)[:5]
         raise AssertionError(f"{what}: {bad.sum()} / {bad.size} updated params off: got {got_p[i]}, "
                              f"ref {ref_p[i]}, bound {bound[i]}")
+
+
+def plan_key(cfg, idx, off, B):
+    """Group-major plan key of every position (R23): kbase_t + (i2 m1 + i1) m3 + i3,
+    digits (i1, i2, i3) of Eq. 3 via numpy.unravel_index per table."""
+    T = cfg.num_tables
+    mf = np.array(cfg.row_factors, np.int64)
+    kbase = np.concatenate([[0], np.cumsum(mf.prod(axis=1))[:-1]]).astype(np.int64)
+    bag = np.repeat(np.arange(T * B), np.diff(off))
+    tab = bag // B
+    key = np.empty(len(idx), np.int64)
+    for t in range(T):
+        sel = tab == t
+        d1, d2, d3 = np.unravel_index(np.asarray(idx)[sel], tuple(mf[t]))
+        key[sel] = kbase[t] + (d2 * mf[t, 0] + d1) * mf[t, 2] + d3
+    return key

@@ -11,7 +11,7 @@ import torch
 
 from oracle import Oracle
 from synth import workload as W
-from tests.helpers import assert_companion, assert_update_close
+from tests.helpers import assert_companion, assert_update_close, plan_key
 
 pytestmark = pytest.mark.gpu
 
@@ -162,9 +162,7 @@ def test_full_size_sampled(name, rank):
     plan = emb.plan()
     # unique count and inverse map against numpy (whole batch)
     T = cfg.num_tables
-    rowbase = np.concatenate([[0], np.cumsum(cfg.table_rows)[:-1]]).astype(np.int64)
-    bag = np.repeat(np.arange(T * B), np.diff(off))
-    key = rowbase[bag // B] + idx
+    key = plan_key(cfg, idx, off, B)
     uk, inv = np.unique(key, return_inverse=True)
     assert plan["U"] == len(uk)
     np.testing.assert_array_equal(plan["ukey"].cpu().numpy().view(np.uint32), uk)
@@ -264,9 +262,10 @@ def test_int32_indices_and_host_api():
     eh.backward_host(torch.as_tensor(go).pin_memory())
     torch.cuda.synchronize()
     torch.testing.assert_close(hout, o64.cpu(), rtol=0, atol=0)
-    # dC1 / dC2 are reduced without atomics: bitwise equal across runs
+    # dC2 is reduced without atomics: bitwise equal across runs; dC1 is summed with vector
+    # reductions in arrival order (R19 / Q19): equal up to fp32 reassociation
     for a, b in zip(eh.grad_views(), e64.grad_views()):
-        torch.testing.assert_close(a[0], b[0], rtol=0, atol=0)
+        torch.testing.assert_close(a[0], b[0], rtol=1e-5, atol=1e-6)
         torch.testing.assert_close(a[1], b[1], rtol=0, atol=0)
 
 

@@ -174,10 +174,14 @@ def test_plan_matches_numpy(name, seed):
     orc = Oracle.from_config(cfg)
     plan = orc.plan(idx, off, B)
     T = cfg.num_tables
-    rowbase = np.concatenate([[0], np.cumsum(cfg.table_rows)[:-1]]).astype(np.int64)
+    # group-major plan key (R23): digits by numpy, re-ravelled in (i2, i1, i3) order
+    mf = np.array(cfg.row_factors, np.int64)
+    span = mf.prod(axis=1)
+    gbase = np.concatenate([[0], np.cumsum(span)[:-1]]).astype(np.int64)
     bag = np.repeat(np.arange(T * B), np.diff(off))
     tab = bag // B
-    key = rowbase[tab] + idx
+    d1, d2, d3 = (np.array(x, np.int64) for x in zip(*[np.unravel_index(i, tuple(mf[t])) for i, t in zip(idx, tab)]))
+    key = gbase[tab] + (d2 * mf[tab, 0] + d1) * mf[tab, 2] + d3
     order = np.argsort(key, kind="stable")
     np.testing.assert_array_equal(plan["skey"], key[order])
     np.testing.assert_array_equal(plan["spos"], order)
@@ -186,26 +190,23 @@ def test_plan_matches_numpy(name, seed):
     np.testing.assert_array_equal(plan["ukey"], uk)
     np.testing.assert_array_equal(plan["inverse"], inv)
     np.testing.assert_array_equal(plan["seg_off"], np.concatenate([[0], np.cumsum(cnt)]))
-    ut = np.searchsorted(rowbase, uk, side="right") - 1
-    urow = uk - rowbase[ut]
-    m = np.array(cfg.row_factors)[ut]
-    i1, i2, i3 = (np.array(x) for x in zip(*[np.unravel_index(r, tuple(f)) for r, f in zip(urow, m)]))
+    # every unique row's digits (from the first position that holds it)
+    firstpos = order[np.concatenate([[0], np.cumsum(cnt)[:-1]])]
+    ut, i1, i2, i3 = tab[firstpos], d1[firstpos], d2[firstpos], d3[firstpos]
     np.testing.assert_array_equal(plan["row_i3"], i3)
-    pk = np.stack([ut, urow // m[:, 2]], 1)
+    pk = np.stack([ut, i2, i1], 1)
     upk, pinv = np.unique(pk, axis=0, return_inverse=True)
     np.testing.assert_array_equal(plan["row_pfx"], pinv.ravel())
     assert plan["P"] == len(upk)
     first = np.concatenate([[0], np.flatnonzero(np.diff(pinv.ravel())) + 1])
-    np.testing.assert_array_equal(plan["pfx_t"], ut[first])
-    np.testing.assert_array_equal(plan["pfx_i1"], i1[first])
-    np.testing.assert_array_equal(plan["pfx_i2"], i2[first])
+    np.testing.assert_array_equal(plan["pfx_t"], upk[:, 0])
+    np.testing.assert_array_equal(plan["pfx_i2"], upk[:, 1])
+    np.testing.assert_array_equal(plan["pfx_i1"], upk[:, 2])
     np.testing.assert_array_equal(plan["row_seg"], np.concatenate([first, [len(uk)]]))
-    g = np.lexsort((plan["pfx_i1"], plan["pfx_i2"], plan["pfx_t"]))
-    np.testing.assert_array_equal(plan["grp_pfx"], g)
-    gk = np.stack([plan["pfx_t"][g], plan["pfx_i2"][g]], 1)
-    gu, gfirst = np.unique(gk, axis=0, return_index=True)
+    np.testing.assert_array_equal(plan["grp_pfx"], np.arange(plan["P"]))
+    gu, gfirst = np.unique(upk[:, :2], axis=0, return_index=True)
     assert plan["NG"] == len(gu)
-    np.testing.assert_array_equal(plan["grp_off"], np.concatenate([np.sort(gfirst), [plan["P"]]]))
+    np.testing.assert_array_equal(plan["grp_off"], np.concatenate([gfirst, [plan["P"]]]))
     np.testing.assert_array_equal(plan["grp_t"], gu[:, 0])
     np.testing.assert_array_equal(plan["grp_i2"], gu[:, 1])
 
