@@ -31,7 +31,7 @@ namespace {
 
 constexpr int XR = 64;                         // TT rank = K of the prefix GEMM
 constexpr int XT = 64;                         // tile rows (prefix, j1) = MMA N (max)
-constexpr int X_LW = 8, X_RW = 7;   // 16 warps total: 128 registers per thread
+constexpr int X_LW = 8, X_RW = 4;   // loaders, epilogue warps
 constexpr int X_THREADS = (X_LW + 1 + X_RW) * 32;
 constexpr int X_MMA_W = X_LW, X_ROW_W0 = X_LW + 1;
 constexpr int XPSTR = 256;                     // P_s row stride (floats); columns XOR-swizzled
@@ -86,15 +86,12 @@ __global__ void k_fused_prep(XArgs a) {
 
 __device__ __forceinline__ float tf32_lo(float x) { return x - tc::tf32_trunc(x); }
 
-template <int N3>
-__global__ void __launch_bounds__(X_THREADS, 1) k_fused_fwd(XArgs a) {
+__global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
   extern __shared__ __align__(128) char smem_raw[];
   __shared__ XCtl ctl;
   char* const smem = smem_raw + ((128u - (tc::smem_u32(smem_raw) & 127u)) & 127u);
   float* const raw = reinterpret_cast<float*>(smem);
   char* const bbuf = smem + X_RAW_BYTES;
-  float* const ps = reinterpret_cast<float*>(smem + X_RAW_BYTES + 2 * XB_SLOT);
-  float* const c3s = ps + XT * XPSTR;
   const int tid = threadIdx.x, w = tid >> 5, lane = tid & 31;
   const uint32_t NG = a.counts[kCntNG];
   const uint32_t raw_bytes = (uint32_t)XR * a.NC * 4u;
@@ -108,7 +105,7 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_fused_fwd(XArgs a) {
       tc::mbar_init(&ctl.d_full[s], 1);
       tc::mbar_init(&ctl.d_free[s], X_RW * 32);
     }
-    for (int s = 0; s < 4; ++s) { tc::mbar_init(&ctl.u_full[s], 1); tc::mbar_init(&ctl.u_empty[s], 2); }
+    for (int s = 0; s < 4; ++s) { tc::mbar_init(&ctl.u_full[s], 1); tc::mbar_init(&ctl.u_empty[s], 1 + X_RW); }
     tc::fence_mbar_init();
   }
   if (w == X_MMA_W) tc::tmem_alloc(&ctl.tmem, 512);
@@ -121,6 +118,7 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_fused_fwd(XArgs a) {
   const int tpp = a.tpp;
   unsigned long long trc[10] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
   const long long t_start = a.trace ? clock64() : 0;
+  const unsigned long long g_start = a.trace ? tc::globaltimer_ns() : 0;
 
   if (w < X_LW) {
     // ------------------------------- loaders -------------------------------
@@ -213,16 +211,6 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_fused_fwd(XArgs a) {
           tc::mbar_arrive(&ctl.b_full[s]);
           XTA(4);
         }
-        {   // L2 prefetch of the tile's C3 slices (the row warps read them about two tiles later);
-            // the tile's unique rows are one contiguous range (group-major plan)
-          const float* c3base = a.cores + a.meta[a.grp_t[cur]].c3_off;
-          const uint32_t u0 = a.row_seg[qa], u1 = a.row_seg[qa + np];
-          for (uint32_t u = u0 + tid; u < u1; u += X_LW * 32) {
-            const char* p3 = reinterpret_cast<const char*>(c3base + (size_t)__ldg(a.row_i3 + u) * XR * N3);
-#pragma unroll
-            for (int l = 0; l < XR * N3 * 4 / 128; ++l) asm volatile("prefetch.global.L2 [%0];" ::"l"(p3 + 128 * l));
-          }
-        }
       }
       XT0();
       // next group: registers <- raw (nxt); raw <- the group after (claimed now)
@@ -293,147 +281,41 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_fused_fwd(XArgs a) {
       if (fl & 2u) ++gs;
     }
   } else {
-    // ------------------------------- row warps -------------------------------
-    constexpr int C3L = XR * N3 / 4 / 32;        // float4 of a C3 slice per lane
-    constexpr int NSL = N3 == 4 ? 3 : 2;         // per-warp C3 ring slots (cp.async)
-    const int rw = w - X_ROW_W0, rtid = tid - X_ROW_W0 * 32;
+    // ------------------------- epilogue: TMEM -> P stash -------------------------
+    // warp w drains lane quarter Q = w % 4 of every c-block: thread = column c, 32 tile rows
+    // per tcgen05.ld; pbuf[(q n1 + j1)][c] rows of one tile are contiguous (group-major plan)
     const int Q = w & 3;
-    // drain assignment: (c-block, lane quarter) pairs; warps rw 0-3 take block 0 (quarters
-    // 1,2,3,0), rw 4-6 block 1 (quarters 1,2,3), rw 3 (quarter 0) also block 1
-    const int blk0 = rw < 4 ? 0 : 1, blk_step = rw == 3 ? 1 : 2;
-    const uint32_t ring3 = tc::smem_u32(c3s + rw * (NSL * XR * N3));
-    const float* ring3p = c3s + rw * (NSL * XR * N3);
-    const int J12 = a.n1 * a.n2;
-    const int j12 = lane >> 1, h = lane & 1;
-    const int j1 = j12 / a.n2, j2 = j12 - j1 * a.n2;
-    const bool jval = j12 < J12;
-    // P_s(m, c) lives at m * XPSTR + (c ^ 4 ((c >> 5) & 7)): conflict-free for the drain (32
-    // consecutive c per warp store) and for the row loads (8 column blocks per LDS.128 phase).
-    const int pb = (j2 * XR + 32 * h) >> 5;
-    const int pxor = pb & 7;
     for (uint32_t ui = 0;; ++ui) {
       XT0();
       tc::mbar_wait(&ctl.u_full[ui & 3], (ui >> 2) & 1);
       XTA(0);
-      const uint32_t g = ctl.ring[ui & 3][0], qa = ctl.ring[ui & 3][1];
-      const uint32_t np = ctl.ring[ui & 3][2], fl = ctl.ring[ui & 3][3];
-      const uint32_t u0 = ctl.ring[ui & 3][4], u1 = ctl.ring[ui & 3][5];
+      const uint32_t qa = ctl.ring[ui & 3][1], np = ctl.ring[ui & 3][2], fl = ctl.ring[ui & 3][3];
+      __syncwarp();
       if (fl & 4u) break;
       const int rows = (int)np << a.n1s;
       const uint32_t s = ui & 1;
-      const uint32_t Rt = u1 - u0;
-      const float* c3base = a.cores + a.meta[a.grp_t[g]].c3_off;
-      // ---- drain D[s]: this warp's c-block quarter -> P_s ----
-      XTA(1);
       tc::mbar_wait(&ctl.d_full[s], (ui >> 1) & 1);
-      XTA(2);
+      XTA(1);
       tc::fence_after();
-      XTA(7);
-      for (int blk = blk0; blk < a.nblk; blk += blk_step) {
+      float* dst = a.pbuf + (size_t)qa * a.n1 * a.NC;
+      for (int blk = 0; blk < a.nblk; ++blk) {
         const int c = blk * 128 + Q * 32 + lane;
-        const int dcol = c ^ (4 * ((c >> 5) & 7));
         for (int j0 = 0; j0 < rows; j0 += 32) {
           float v[32];
           tc::tmem_ld32(tc::taddr(tm + 256 + s * 128 + blk * 64 + j0, 32 * Q, 0), v);
+          const int lim = min(32, rows - j0);
           if (c < a.NC) {
-            float* dst = ps + j0 * XPSTR + dcol;
+            float* d = dst + (size_t)j0 * a.NC + c;
 #pragma unroll
-            for (int j = 0; j < 32; ++j) dst[j * XPSTR] = v[j];
+            for (int j = 0; j < 32; ++j)
+              if (j < lim) d[(size_t)j * a.NC] = v[j];
           }
         }
       }
-      XTA(9);
       tc::fence_before();
       tc::mbar_arrive(&ctl.d_free[s]);
-      XTA(3);
-      tc::named_sync(2, X_RW * 32);
-      XTA(4);
-      // ---- P stash for the backward row stage: pbuf[q][j1][c] <- P_s (float4); the tile's
-      //      prefixes qa .. qa+np-1 are consecutive, so this is one contiguous block ----
-      if (a.pbuf) {
-        const int nc4 = a.NC >> 2, tot = rows * nc4;
-        float* dst = a.pbuf + (size_t)qa * a.n1 * a.NC;
-        for (int f = rtid; f < tot; f += X_RW * 32) {
-          const int mm = f / nc4, c4 = (f - mm * nc4) * 4;
-          *reinterpret_cast<float4*>(dst + (size_t)mm * a.NC + c4) =
-              *reinterpret_cast<const float4*>(ps + mm * XPSTR + (c4 ^ (4 * ((c4 >> 5) & 7))));
-        }
-      }
-      // ---- rows: this warp's share [r0, r1) of the tile's Rt unique rows u0 .. u1-1 ----
-      const uint32_t r0 = (uint32_t)(((uint64_t)Rt * rw) / X_RW), r1 = (uint32_t)(((uint64_t)Rt * (rw + 1)) / X_RW);
-      int curk = -1;
-      float4 pv[8];
-      for (uint32_t rb = r0; rb < r1; rb += 32) {
-        const int nr = (int)min(32u, r1 - rb);
-        // lane-parallel: row u0 + rb + lane -> (tile prefix k, i3)
-        const uint32_t ul = u0 + rb + lane;
-        int kl = 0;
-        uint32_t i3l = 0;
-        if (lane < nr) {
-          kl = (int)(__ldg(a.row_pfx + ul) - qa);
-          i3l = __ldg(a.row_i3 + ul);
-        }
-        auto issue = [&](int j) {   // C3 slice of row rb + j -> ring slot j % NSL
-          const uint32_t i3 = __shfl_sync(0xffffffffu, i3l, j);
-          const float4* src = reinterpret_cast<const float4*>(c3base + (size_t)i3 * XR * N3);
-          const uint32_t dst = ring3 + (uint32_t)((j % NSL) * XR * N3 * 4);
-#pragma unroll
-          for (int i = 0; i < C3L; ++i) tc::cp_async16(dst + 16u * (lane + 32 * i), src + lane + 32 * i);
-        };
-#pragma unroll
-        for (int j = 0; j < NSL - 1; ++j) {
-          if (j < nr) issue(j);
-          tc::cp_commit();
-        }
-        for (int j = 0; j < nr; ++j) {
-          tc::cp_wait<NSL - 2>();
-          __syncwarp();
-          const int k = __shfl_sync(0xffffffffu, kl, j);
-          const uint32_t u = u0 + rb + j;
-          if (k != curk) {
-            const float* prow = ps + ((k << a.n1s) + j1) * XPSTR + 32 * pb;
-#pragma unroll
-            for (int i = 0; i < 8; ++i)
-              pv[i] = jval ? *reinterpret_cast<const float4*>(prow + 4 * (i ^ pxor)) : make_float4(0.f, 0.f, 0.f, 0.f);
-            curk = k;
-          }
-          float acc[N3];
-#pragma unroll
-          for (int q = 0; q < N3; ++q) acc[q] = 0.f;
-          const float* c3 = ring3p + (j % NSL) * XR * N3 + 32 * h * N3;
-#pragma unroll
-          for (int i = 0; i < 8; ++i) {
-            const float pr[4] = {pv[i].x, pv[i].y, pv[i].z, pv[i].w};
-#pragma unroll
-            for (int e = 0; e < 4; ++e)
-#pragma unroll
-              for (int q = 0; q < N3; q += 4) {
-                const float4 c4 = *reinterpret_cast<const float4*>(c3 + (4 * i + e) * N3 + q);
-                acc[q] = fmaf(pr[e], c4.x, acc[q]);
-                acc[q + 1] = fmaf(pr[e], c4.y, acc[q + 1]);
-                acc[q + 2] = fmaf(pr[e], c4.z, acc[q + 2]);
-                acc[q + 3] = fmaf(pr[e], c4.w, acc[q + 3]);
-              }
-          }
-          __syncwarp();
-          if (j + NSL - 1 < nr) issue(j + NSL - 1);
-          tc::cp_commit();
-#pragma unroll
-          for (int q = 0; q < N3; ++q) acc[q] += __shfl_xor_sync(0xffffffffu, acc[q], 1);
-          if (h == 0 && jval) {
-            float* d = a.rows + (size_t)u * a.N + j12 * N3;
-#pragma unroll
-            for (int q = 0; q < N3; q += 4) *reinterpret_cast<float4*>(d + q) = make_float4(acc[q], acc[q + 1], acc[q + 2], acc[q + 3]);
-          }
-        }
-        tc::cp_wait<0>();
-        __syncwarp();
-      }
-      XTA(5);
-      tc::named_sync(2, X_RW * 32);      // P_s free for the next tile's drain
-      XTA(6);
-      trc[8] += Rt;
-      if (rtid == 0) tc::mbar_arrive(&ctl.u_empty[ui & 3]);
+      XTA(2);
+      if (lane == 0) tc::mbar_arrive(&ctl.u_empty[ui & 3]);
     }
   }
   if (a.trace) {
@@ -441,6 +323,10 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_fused_fwd(XArgs a) {
     if (role >= 0)
       for (int k = 0; k < 10; ++k) a.trace[32 * blockIdx.x + 10 * role + k] = trc[k];
     if (tid == 0) a.trace[32 * blockIdx.x + 30] = (unsigned long long)(clock64() - t_start);
+    if (tid == X_ROW_W0 * 32) {
+      a.trace[32 * blockIdx.x + 31] = tc::globaltimer_ns();
+      a.trace[32 * blockIdx.x + 29] = g_start;
+    }
   }
   tc::fence_before();
   __syncthreads();
@@ -448,9 +334,138 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_fused_fwd(XArgs a) {
   if (w == X_MMA_W) tc::tmem_dealloc(tm, 512);
 }
 
-size_t fused_smem(int n3) {
-  return 128 + X_RAW_BYTES + 2 * XB_SLOT + (size_t)XT * XPSTR * 4 + (size_t)X_RW * (n3 == 4 ? 3 : 2) * XR * n3 * 4;
+constexpr size_t kPrefixSmem = 128 + X_RAW_BYTES + 2 * XB_SLOT;
+
+// ------------------------------------------------------------------------------------
+// Row contraction a6 (Eq. 2, Fig. 5(b) step 3): E_u = P_q (n1 n2 x R) . C3[i3_u] (R x n3)
+// on FFMA, high occupancy (8 warps per CTA, 4 CTAs per SM).  A warp owns RCH consecutive
+// unique rows (rows of one prefix are consecutive, so P_q is reloaded only at prefix
+// changes).  Lane map: jq = lane >> 3 owns j12 = 4 jq .. 4 jq + 3, rp = lane & 7 owns
+// r = 8 rp .. 8 rp + 7 (P_q slice in 32 registers); the C3 slice of each row is streamed
+// into a per-warp 3-slot shared-memory ring by cp.async two rows ahead, with rows skewed by
+// 4 floats per 8 so the 8 rp lanes of an LDS.128 phase hit distinct banks; the 4 j12 x n3
+// partial sums are reduced over rp by recursive halving (3 shuffle levels) and each lane
+// stores n3/2 consecutive outputs.
+// ------------------------------------------------------------------------------------
+constexpr int RW_WARPS = 8, RW_RCH = 16, RW_NSL = 3;
+
+struct RowArgs {
+  const float* cores;
+  const TableMeta* meta;
+  const uint32_t *counts, *row_pfx, *row_i3, *pfx_t;
+  const float* pbuf;          // [P][n1][NC]
+  float* rows;                // [U][N]
+  int n1, n1s, n2, N, NC;
+};
+
+template <int N3>
+__global__ void __launch_bounds__(RW_WARPS * 32, 3) k_rows_fwd2(RowArgs a) {
+  constexpr int SLOT = XR * N3 + 32;
+  constexpr int C3L = XR * N3 / 4 / 32;
+  extern __shared__ __align__(16) float rw_smem[];
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  float* const ringp = rw_smem + w * (RW_NSL * SLOT);
+  const uint32_t ring = tc::smem_u32(ringp);
+  const uint32_t U = a.counts[kCntU];
+  const int J12 = a.n1 * a.n2;
+  const int jq = lane >> 3, rp = lane & 7;
+  // per-lane P offsets inside a prefix block [n1][NC] for e = 0..3 (j12 = 4 jq + e)
+  int poff[4];
+#pragma unroll
+  for (int e = 0; e < 4; ++e) {
+    const int j12 = 4 * jq + e, j1 = j12 / a.n2, j2 = j12 - j1 * a.n2;
+    poff[e] = j12 < J12 ? j1 * a.NC + j2 * XR + 8 * rp : -1;
+  }
+  const int64_t nch = ((int64_t)U + RW_RCH - 1) / RW_RCH;
+  const int64_t gw = (int64_t)blockIdx.x * RW_WARPS + w, nw = (int64_t)gridDim.x * RW_WARPS;
+  for (int64_t ch = gw; ch < nch; ch += nw) {
+    const uint32_t u0 = (uint32_t)ch * RW_RCH;
+    const int nr = (int)min((uint32_t)RW_RCH, U - u0);
+    uint32_t ql = 0;
+    unsigned long long o3l = 0;
+    if (lane < nr) {
+      ql = __ldg(a.row_pfx + u0 + lane);
+      o3l = a.meta[__ldg(a.pfx_t + ql)].c3_off + (unsigned long long)__ldg(a.row_i3 + u0 + lane) * XR * N3;
+    }
+    auto issue = [&](int j) {
+      const unsigned long long o3 = __shfl_sync(0xffffffffu, o3l, j);
+      const float4* src = reinterpret_cast<const float4*>(a.cores + o3);
+      const uint32_t dst = ring + (uint32_t)((j % RW_NSL) * SLOT * 4);
+#pragma unroll
+      for (int i = 0; i < C3L; ++i) {
+        const int f = lane + 32 * i, r = f / (N3 / 4);
+        tc::cp_async16(dst + 4u * (uint32_t)(4 * f + 4 * ((r >> 3) & 7)), src + f);
+      }
+    };
+#pragma unroll
+    for (int j = 0; j < RW_NSL - 1; ++j) {
+      if (j < nr) issue(j);
+      tc::cp_commit();
+    }
+    uint32_t curq = 0xffffffffu;
+    float pr[4][8];
+    for (int j = 0; j < nr; ++j) {
+      const uint32_t q = __shfl_sync(0xffffffffu, ql, j);
+      if (q != curq) {
+        const float* pq = a.pbuf + (size_t)q * a.n1 * a.NC;
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          float4 x0 = make_float4(0.f, 0.f, 0.f, 0.f), x1 = x0;
+          if (poff[e] >= 0) {
+            x0 = __ldg(reinterpret_cast<const float4*>(pq + poff[e]));
+            x1 = __ldg(reinterpret_cast<const float4*>(pq + poff[e] + 4));
+          }
+          pr[e][0] = x0.x; pr[e][1] = x0.y; pr[e][2] = x0.z; pr[e][3] = x0.w;
+          pr[e][4] = x1.x; pr[e][5] = x1.y; pr[e][6] = x1.z; pr[e][7] = x1.w;
+        }
+        curq = q;
+      }
+      tc::cp_wait<RW_NSL - 2>();
+      __syncwarp();
+      float acc[4 * N3];
+#pragma unroll
+      for (int i = 0; i < 4 * N3; ++i) acc[i] = 0.f;
+      const float* c3 = ringp + (j % RW_NSL) * SLOT + (8 * rp) * N3 + 4 * rp;
+#pragma unroll
+      for (int x = 0; x < 8; ++x) {
+        float cv[N3];
+#pragma unroll
+        for (int b = 0; b < N3; b += 4) {
+          const float4 t4 = *reinterpret_cast<const float4*>(c3 + x * N3 + b);
+          cv[b] = t4.x; cv[b + 1] = t4.y; cv[b + 2] = t4.z; cv[b + 3] = t4.w;
+        }
+#pragma unroll
+        for (int e = 0; e < 4; ++e)
+#pragma unroll
+          for (int b = 0; b < N3; ++b) acc[e * N3 + b] = fmaf(pr[e][x], cv[b], acc[e * N3 + b]);
+      }
+      __syncwarp();
+      if (j + RW_NSL - 1 < nr) issue(j + RW_NSL - 1);
+      tc::cp_commit();
+#pragma unroll
+      for (int lv = 0; lv < 3; ++lv) {
+        const int mask = 4 >> lv, half = (4 * N3) >> (lv + 1);
+        const bool hi = (lane & mask) != 0;
+#pragma unroll
+        for (int i = 0; i < half; ++i) {
+          const float snd = hi ? acc[i] : acc[i + half];
+          const float kp = hi ? acc[i + half] : acc[i];
+          acc[i] = kp + __shfl_xor_sync(0xffffffffu, snd, mask);
+        }
+      }
+      // this lane holds E[j12 = 4 jq + rp / 2][j3 = (rp & 1) n3/2 .. + n3/2 - 1]
+      if (4 * jq + (rp >> 1) < J12) {
+        float* d = a.rows + (size_t)(u0 + j) * a.N + (4 * jq) * N3 + rp * (N3 / 2);
+        if (N3 == 4) *reinterpret_cast<float2*>(d) = make_float2(acc[0], acc[1]);
+        else *reinterpret_cast<float4*>(d) = make_float4(acc[0], acc[1], acc[2], acc[3]);
+      }
+    }
+    tc::cp_wait<0>();
+    __syncwarp();
+  }
 }
+
+size_t rows_smem(int n3) { return (size_t)RW_WARPS * RW_NSL * (XR * n3 + 32) * 4; }
 
 }  // namespace
 
@@ -461,9 +476,11 @@ bool fused_eligible(const Ctx& c) {
 
 cudaError_t configure_fused(Ctx& c) {
   if (!fused_eligible(c)) return cudaSuccess;
-  cudaError_t e = cudaFuncSetAttribute(k_fused_fwd<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fused_smem(4));
+  cudaError_t e = cudaFuncSetAttribute(k_prefix_fwd, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kPrefixSmem);
   if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(k_fused_fwd<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fused_smem(8));
+    e = cudaFuncSetAttribute(k_rows_fwd2<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)rows_smem(4));
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(k_rows_fwd2<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)rows_smem(8));
   return e;
 }
 
@@ -488,20 +505,38 @@ cudaError_t run_fused_fwd(Ctx& c, cudaStream_t s) {
       cudaMemsetAsync(trace, 0, sizeof(unsigned long long) * 32 * grid, s);
       a.trace = trace;
     }
-    if (c.n3 == 4) k_fused_fwd<4><<<grid, X_THREADS, fused_smem(4), s>>>(a);
-    else k_fused_fwd<8><<<grid, X_THREADS, fused_smem(8), s>>>(a);
+    k_prefix_fwd<<<grid, X_THREADS, kPrefixSmem, s>>>(a);
     if (a.trace) {
       std::vector<unsigned long long> hb(32 * grid);
       cudaMemcpyAsync(hb.data(), trace, hb.size() * 8, cudaMemcpyDeviceToHost, s);
       cudaStreamSynchronize(s);
       double m[32] = {};
-      for (int b = 0; b < grid; ++b) for (int k = 0; k < 32; ++k) m[k] += (double)hb[32 * b + k] / grid;
+      for (int b = 0; b < grid; ++b) for (int k = 0; k < 29; ++k) m[k] += (double)hb[32 * b + k] / grid;
+      unsigned long long s0 = ~0ull, s1 = ~0ull, e0 = 0, e1 = ~0ull;
+      double tmax = 0;
+      for (int b = 0; b < grid; ++b) {
+        s0 = std::min(s0, hb[32 * b + 29]); s1 = s1 == ~0ull ? hb[32 * b + 29] : std::max(s1, hb[32 * b + 29]);
+        e0 = std::max(e0, hb[32 * b + 31]); e1 = std::min(e1, hb[32 * b + 31]);
+        tmax = std::max(tmax, (double)hb[32 * b + 30]);
+      }
+      fprintf(stderr, "[trace fused] span: first start -> last start %.1f us, first end %.1f us, last end %.1f us; max CTA cycles %.0f\n",
+              (s1 - s0) * 1e-3, (e1 - s0) * 1e-3, (e0 - s0) * 1e-3, tmax);
       fprintf(stderr, "[trace fused] total %.0f | loader: ring+bload %.0f a_free %.0f a_store %.0f b_free %.0f b_store %.0f "
               "raw_wait %.0f raw_sync %.0f | mma: u_full %.0f a_full %.0f b_full %.0f d_free %.0f issue %.0f units %.1f | "
               "rows: u_full %.0f plist %.0f d_full %.0f [fa %.0f loop %.0f] fb+arrive %.0f sync1 %.0f rows %.0f sync2 %.0f nrows %.0f (cycles/CTA)\n",
               m[30], m[0], m[1], m[2], m[3], m[4], m[5], m[6], m[10], m[11], m[12], m[13], m[14], m[19], m[20], m[21],
               m[22], m[27], m[29], m[23], m[24], m[25], m[26], m[28]);
     }
+  }
+  {
+    StageScope sc(c, ST_FWD_ROWS, s);
+    RowArgs r;
+    r.cores = c.cores; r.meta = c.d_meta; r.counts = p.counts; r.row_pfx = p.row_pfx; r.row_i3 = p.row_i3;
+    r.pfx_t = p.pfx_t; r.pbuf = p.pbuf; r.rows = p.rows;
+    r.n1 = c.n1; r.n1s = a.n1s; r.n2 = c.n2; r.N = c.N; r.NC = c.NC;
+    const int grid = grid_for(c, cdiv(c.U_cap, RW_RCH), RW_WARPS, 4);
+    if (c.n3 == 4) k_rows_fwd2<4><<<grid, RW_WARPS * 32, rows_smem(4), s>>>(r);
+    else k_rows_fwd2<8><<<grid, RW_WARPS * 32, rows_smem(8), s>>>(r);
   }
   return cudaGetLastError();
 }
