@@ -467,6 +467,188 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 3) k_rows_fwd2(RowArgs a) {
 
 size_t rows_smem(int n3) { return (size_t)RW_WARPS * RW_NSL * (XR * n3 + 32) * 4; }
 
+// ------------------------------------------------------------------------------------
+// Row backward a9 (Eq. 6 read as left^T . dL/de . right^T), same lane map and
+// C3 ring as k_rows_fwd2, with the aggregated row gradient G_u (a8) staged next to C3:
+//   dP_q[j12][r] += sum_j3 G_u[j12][j3] C3_u[r][j3]   registers (4 j12 x 8 r per lane),
+//                                                     flushed to dpbuf at prefix changes
+//   dC3[i3_u][r][j3] += sum_j12 P_q[j12][r] G_u[j12][j3]  partial over the lane's 4 j12,
+//                    reduced over jq (2 shuffle levels), red.global.add.v4 (L2-resident)
+// dP of a prefix whose rows straddle a chunk boundary is accumulated with vector reductions
+// into rows zeroed by k_dp_zero2; prefixes inside one chunk are stored directly.
+// ------------------------------------------------------------------------------------
+struct RowBwdArgs {
+  const float* cores;
+  float* grads;
+  const TableMeta* meta;
+  const uint32_t *counts, *row_pfx, *row_i3, *pfx_t, *row_seg;
+  const float* pbuf;          // [P][n1][NC]
+  const float* gbuf;          // [U][N]
+  float* dpbuf;               // [P][n1][NC]
+  int n1, n2, N, NC;
+};
+
+__global__ void __launch_bounds__(256) k_dp_zero2(RowBwdArgs a) {
+  const uint32_t P = a.counts[kCntP];
+  const int blk = a.n1 * a.NC / 4;
+  const int lane = threadIdx.x & 31;
+  for (uint32_t q = blockIdx.x * 8 + (threadIdx.x >> 5); q < P; q += gridDim.x * 8) {
+    const uint32_t r0 = a.row_seg[q], r1 = a.row_seg[q + 1];
+    if (r0 / RW_RCH == (r1 - 1) / RW_RCH) continue;
+    float4* d = reinterpret_cast<float4*>(a.dpbuf + (size_t)q * a.n1 * a.NC);
+    for (int f = lane; f < blk; f += 32) d[f] = make_float4(0.f, 0.f, 0.f, 0.f);
+  }
+}
+
+__device__ __forceinline__ void red_v4(float* addr, float4 v) {
+  asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(addr), "f"(v.x), "f"(v.y), "f"(v.z), "f"(v.w)
+               : "memory");
+}
+
+template <int N3>
+__global__ void __launch_bounds__(RW_WARPS * 32, 2) k_rows_bwd2(RowBwdArgs a) {
+  constexpr int C3S = XR * N3 + 32;             // skewed C3 part of a slot
+  constexpr int SLOT = C3S + 16 * N3;           // + G_u (N <= 16 n3)
+  constexpr int C3L = XR * N3 / 4 / 32;
+  extern __shared__ __align__(16) float rw_smem[];
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  float* const ringp = rw_smem + w * (RW_NSL * SLOT);
+  const uint32_t ring = tc::smem_u32(ringp);
+  const uint32_t U = a.counts[kCntU];
+  const int J12 = a.n1 * a.n2;
+  const int jq = lane >> 3, rp = lane & 7;
+  int poff[4];
+#pragma unroll
+  for (int e = 0; e < 4; ++e) {
+    const int j12 = 4 * jq + e, j1 = j12 / a.n2, j2 = j12 - j1 * a.n2;
+    poff[e] = j12 < J12 ? j1 * a.NC + j2 * XR + 8 * rp : -1;
+  }
+  const int64_t nch = ((int64_t)U + RW_RCH - 1) / RW_RCH;
+  const int64_t gw = (int64_t)blockIdx.x * RW_WARPS + w, nw = (int64_t)gridDim.x * RW_WARPS;
+  for (int64_t ch = gw; ch < nch; ch += nw) {
+    const uint32_t u0 = (uint32_t)ch * RW_RCH;
+    const int nr = (int)min((uint32_t)RW_RCH, U - u0);
+    uint32_t ql = 0;
+    unsigned long long o3l = 0;
+    if (lane < nr) {
+      ql = __ldg(a.row_pfx + u0 + lane);
+      o3l = a.meta[__ldg(a.pfx_t + ql)].c3_off + (unsigned long long)__ldg(a.row_i3 + u0 + lane) * XR * N3;
+    }
+    const uint32_t prevq = u0 > 0 ? __ldg(a.row_pfx + u0 - 1) : 0xffffffffu;
+    const uint32_t nextq = u0 + nr < U ? __ldg(a.row_pfx + u0 + nr) : 0xffffffffu;
+    auto issue = [&](int j) {
+      const unsigned long long o3 = __shfl_sync(0xffffffffu, o3l, j);
+      const float4* src = reinterpret_cast<const float4*>(a.cores + o3);
+      const uint32_t dst = ring + (uint32_t)((j % RW_NSL) * SLOT * 4);
+#pragma unroll
+      for (int i = 0; i < C3L; ++i) {
+        const int f = lane + 32 * i, r = f / (N3 / 4);
+        tc::cp_async16(dst + 4u * (uint32_t)(4 * f + 4 * ((r >> 3) & 7)), src + f);
+      }
+      if (lane < a.N / 4)
+        tc::cp_async16(dst + 4u * (uint32_t)(C3S + 4 * lane),
+                       reinterpret_cast<const float4*>(a.gbuf + (size_t)(u0 + j) * a.N) + lane);
+    };
+#pragma unroll
+    for (int j = 0; j < RW_NSL - 1; ++j) {
+      if (j < nr) issue(j);
+      tc::cp_commit();
+    }
+    uint32_t curq = 0xffffffffu;
+    float pr[4][8], dp[4][8];
+    auto flush = [&]() {
+      const bool red = curq == prevq || curq == nextq;
+      float* d = a.dpbuf + (size_t)curq * a.n1 * a.NC;
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        if (poff[e] < 0) continue;
+        const float4 v0 = make_float4(dp[e][0], dp[e][1], dp[e][2], dp[e][3]);
+        const float4 v1 = make_float4(dp[e][4], dp[e][5], dp[e][6], dp[e][7]);
+        if (red) { red_v4(d + poff[e], v0); red_v4(d + poff[e] + 4, v1); }
+        else {
+          *reinterpret_cast<float4*>(d + poff[e]) = v0;
+          *reinterpret_cast<float4*>(d + poff[e] + 4) = v1;
+        }
+      }
+    };
+    for (int j = 0; j < nr; ++j) {
+      const uint32_t q = __shfl_sync(0xffffffffu, ql, j);
+      if (q != curq) {
+        if (curq != 0xffffffffu) flush();
+        const float* pq = a.pbuf + (size_t)q * a.n1 * a.NC;
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          float4 x0 = make_float4(0.f, 0.f, 0.f, 0.f), x1 = x0;
+          if (poff[e] >= 0) {
+            x0 = __ldg(reinterpret_cast<const float4*>(pq + poff[e]));
+            x1 = __ldg(reinterpret_cast<const float4*>(pq + poff[e] + 4));
+          }
+          pr[e][0] = x0.x; pr[e][1] = x0.y; pr[e][2] = x0.z; pr[e][3] = x0.w;
+          pr[e][4] = x1.x; pr[e][5] = x1.y; pr[e][6] = x1.z; pr[e][7] = x1.w;
+#pragma unroll
+          for (int x = 0; x < 8; ++x) dp[e][x] = 0.f;
+        }
+        curq = q;
+      }
+      tc::cp_wait<RW_NSL - 2>();
+      __syncwarp();
+      const float* slot = ringp + (j % RW_NSL) * SLOT;
+      float g[4][N3];
+#pragma unroll
+      for (int e = 0; e < 4; ++e)
+#pragma unroll
+        for (int b = 0; b < N3; b += 4) {
+          const float4 t4 = *reinterpret_cast<const float4*>(slot + C3S + (4 * jq + e) * N3 + b);
+          g[e][b] = t4.x; g[e][b + 1] = t4.y; g[e][b + 2] = t4.z; g[e][b + 3] = t4.w;
+        }
+      float dc[8 * N3];
+      const float* c3 = slot + (8 * rp) * N3 + 4 * rp;
+#pragma unroll
+      for (int x = 0; x < 8; ++x) {
+        float cv[N3];
+#pragma unroll
+        for (int b = 0; b < N3; b += 4) {
+          const float4 t4 = *reinterpret_cast<const float4*>(c3 + x * N3 + b);
+          cv[b] = t4.x; cv[b + 1] = t4.y; cv[b + 2] = t4.z; cv[b + 3] = t4.w;
+        }
+#pragma unroll
+        for (int b = 0; b < N3; ++b) dc[x * N3 + b] = 0.f;
+#pragma unroll
+        for (int e = 0; e < 4; ++e)
+#pragma unroll
+          for (int b = 0; b < N3; ++b) {
+            dp[e][x] = fmaf(g[e][b], cv[b], dp[e][x]);
+            dc[x * N3 + b] = fmaf(pr[e][x], g[e][b], dc[x * N3 + b]);
+          }
+      }
+      __syncwarp();
+      if (j + RW_NSL - 1 < nr) issue(j + RW_NSL - 1);
+      tc::cp_commit();
+      // dC3: reduce over jq (lane bits 4, 3); lane keeps r = 8 rp + 2 jq + {0, 1}, all j3
+#pragma unroll
+      for (int lv = 0; lv < 2; ++lv) {
+        const int mask = 16 >> lv, half = (8 * N3) >> (lv + 1);
+        const bool hi = (lane & mask) != 0;
+#pragma unroll
+        for (int i = 0; i < half; ++i) {
+          const float snd = hi ? dc[i] : dc[i + half];
+          const float kp = hi ? dc[i + half] : dc[i];
+          dc[i] = kp + __shfl_xor_sync(0xffffffffu, snd, mask);
+        }
+      }
+      const unsigned long long o3 = __shfl_sync(0xffffffffu, o3l, j);
+      float* d3 = a.grads + o3 + (size_t)(8 * rp + 2 * jq) * N3;
+#pragma unroll
+      for (int i = 0; i < 2 * N3; i += 4) red_v4(d3 + i, make_float4(dc[i], dc[i + 1], dc[i + 2], dc[i + 3]));
+    }
+    if (curq != 0xffffffffu) flush();
+    tc::cp_wait<0>();
+    __syncwarp();
+  }
+}
+
+size_t rows_bwd_smem(int n3) { return (size_t)RW_WARPS * RW_NSL * (XR * n3 + 32 + 16 * n3) * 4; }
+
 }  // namespace
 
 bool fused_eligible(const Ctx& c) {
@@ -481,6 +663,10 @@ cudaError_t configure_fused(Ctx& c) {
     e = cudaFuncSetAttribute(k_rows_fwd2<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)rows_smem(4));
   if (e == cudaSuccess)
     e = cudaFuncSetAttribute(k_rows_fwd2<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)rows_smem(8));
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(k_rows_bwd2<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)rows_bwd_smem(4));
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(k_rows_bwd2<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)rows_bwd_smem(8));
   return e;
 }
 
@@ -538,6 +724,20 @@ cudaError_t run_fused_fwd(Ctx& c, cudaStream_t s) {
     if (c.n3 == 4) k_rows_fwd2<4><<<grid, RW_WARPS * 32, rows_smem(4), s>>>(r);
     else k_rows_fwd2<8><<<grid, RW_WARPS * 32, rows_smem(8), s>>>(r);
   }
+  return cudaGetLastError();
+}
+
+// Backward row stage (dP stash + dC3) for the fused-eligible shapes.
+cudaError_t run_rows_bwd2(Ctx& c, cudaStream_t s) {
+  const PlanDev& p = c.p;
+  RowBwdArgs r;
+  r.cores = c.cores; r.grads = c.grads; r.meta = c.d_meta; r.counts = p.counts; r.row_pfx = p.row_pfx;
+  r.row_i3 = p.row_i3; r.pfx_t = p.pfx_t; r.row_seg = p.row_seg; r.pbuf = p.pbuf; r.gbuf = p.gbuf;
+  r.dpbuf = p.dpbuf; r.n1 = c.n1; r.n2 = c.n2; r.N = c.N; r.NC = c.NC;
+  k_dp_zero2<<<grid_for(c, c.P_cap, 8, 8), 256, 0, s>>>(r);
+  const int grid = grid_for(c, cdiv(c.U_cap, RW_RCH), RW_WARPS, 2);
+  if (c.n3 == 4) k_rows_bwd2<4><<<grid, RW_WARPS * 32, rows_bwd_smem(4), s>>>(r);
+  else k_rows_bwd2<8><<<grid, RW_WARPS * 32, rows_bwd_smem(8), s>>>(r);
   return cudaGetLastError();
 }
 

@@ -1002,10 +1002,15 @@ cudaError_t run_tc_bwd(Ctx& c, float lr, cudaStream_t s) {
   TcArgs a = make_tc_args(c, lr, c.p.work + 1, nullptr);
   {
     StageScope sc(c, ST_BWD_ROWS, s);
+    if (fused_eligible(c)) {
+      cudaError_t e = run_rows_bwd2(c, s);
+      if (e != cudaSuccess) return e;
+    } else {
     k_dp_zero<<<grid_for(c, c.P_cap, 8, 8), 256, 0, s>>>(a);
     const int grid = grid_for(c, cdiv(c.U_cap, RCH), 4, 8);
     if (c.n3 == 4) k_rows_bwd<4><<<grid, 128, 0, s>>>(a);
     else k_rows_bwd<8><<<grid, 128, 0, s>>>(a);
+    }
   }
   {
     StageScope sc(c, ST_BWD_PREFIX, s);
