@@ -285,6 +285,7 @@ int ttemb_create(const ttemb_config* cfg, int device, void* cores, void* state, 
   if (e == cudaSuccess) e = configure_group(c);
   if (e == cudaSuccess) e = configure_tc(c);
   if (e == cudaSuccess) e = configure_fused(c);
+  if (e == cudaSuccess) e = configure_bwdtc(c);
   if (e != cudaSuccess) {
     fprintf(stderr, "ttemb_create: %s\n", cudaGetErrorString(e));
     delete h;

@@ -219,7 +219,7 @@ cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s
   if (c.nnz > 0) {
     cudaError_t e = tc_eligible(c) ? run_tc_bwd(c, lr, s) : run_group_bwd(c, lr, s);
     if (e != cudaSuccess) return e;
-    {
+    if (!fused_eligible(c)) {   // (the tcgen05 prefix-backward kernel adds dA into dC1 itself)
       StageScope sc(c, ST_DC1, s);
       if ((c.n1 * c.R) % 4 == 0)
         k_dc1<<<grid_for(c, c.P_cap * c.n1 * c.R / 4, 256, 32), 256, 0, s>>>(a);

@@ -1,0 +1,420 @@
+// ttemb_bwdtc.cu -- prefix backward on tcgen05, sm_100a.
+//
+// One persistent CTA per SM walks the i2-groups g = (t, i2) (static round robin).  Per tile
+// of <= 64 rows m = (prefix q, j1) of the group, with dP = dL/dP from the row stage (dpbuf):
+//   dC2[i2]^T[c][r1] += sum_m dP[m][c] . C1[i1_m][j1_m][r1]      (Eq. 6 read as left^T . dL/de
+//                       . right^T; the left factor of C2 is the C1 slice)
+//       M = 128 c per block, N = 64 r1, K = 64 m: A = dP^T held in TENSOR MEMORY (lane = c,
+//       column = m, written by the loader threads), B = C1^T rows in shared memory;
+//       accumulated in TMEM over all tiles of the group (no atomics, no partial buffers).
+//   dA[m][r1] = sum_c dP[m][c] . C2[i2][r1][c]                  (the C1 gradient partials)
+//       M = 128 = the tile's dP rows stacked as [dP_hi; dP_lo], N = 64 r1, K = c in chunks of
+//       64 staged in shared memory (double-buffered); two MMAs per K step (B = C2_hi, C2_lo)
+//       give A_hi B_hi + A_lo B_hi + A_hi B_lo, i.e. 3xTF32 with two M = 128 instructions.
+//       The epilogue adds dA straight into the C1 gradient (red.global.add.v4, L2-resident).
+// At the group's last tile the dC2 accumulator is drained and, with TTEMB_FUSED_UPDATE, the
+// C2 slice is updated in place (SGD / Adagrad, the paper's fused TT core update);
+// the slice has no other reader in this kernel once its last tile's MMAs completed.
+// fp32 accuracy: 3xTF32 (hi = raw fp32, read by the tensor core with truncation; lo =
+// x - trunc_tf32(x)); scripts/tc_probe3.cu measures the TMEM-A form.
+//
+// Warp roles (416 threads): 0-7 loaders (cp.async chunk staging, lo split, dP^T -> TMEM),
+// 8 MMA issuer, 9-12 epilogue (dA -> dC1 reductions, dC2 -> gradient / fused update).
+#include <stdio.h>
+#include <stdlib.h>
+
+#include <algorithm>
+
+#include "tc.cuh"
+#include "ttemb_internal.cuh"
+
+namespace ttemb {
+
+namespace {
+
+constexpr int YR = 64, YT = 64;                 // rank; tile rows (prefix, j1)
+constexpr int Y_LW = 8, Y_EW = 4;
+constexpr int Y_THREADS = (Y_LW + 1 + Y_EW) * 32;
+constexpr int Y_MMA_W = Y_LW;
+constexpr uint32_t Y_B1 = 2u * YR * YT * 4;     // C1^T hi + lo (CM(r1, m)), 32 KB
+constexpr uint32_t Y_A2LBO = 16 * 128 + 16;    // CM(128 rows, 64 c); +16 B per core column keeps
+                                                // the column-wise dP^T extraction conflict-free
+constexpr uint32_t Y_A2 = 16 * Y_A2LBO;         // [dP_hi; dP_lo] chunk (~32 KB)
+constexpr uint32_t Y_B2 = 2u * YR * 64 * 4;     // C2 chunk hi + lo, CM(r1, 64 c), 32 KB
+constexpr uint32_t Y_STAGE = Y_A2 + Y_B2;
+constexpr int Y_NST = 3;                        // chunk stages (cp.async, two in flight)
+constexpr size_t kBwdSmem = 128 + Y_B1 + Y_NST * Y_STAGE;
+
+struct YArgs {
+  float* cores;
+  float* grads;
+  float* state;
+  const TableMeta* meta;
+  const uint32_t *counts, *grp_off, *grp_t, *pfx_i1, *pfx_t;
+  const uint32_t* grp_arow;               // [P]  C1 row index (floats / R) of prefix q, j1 = 0
+  const unsigned long long* grp_c2;       // [NG] float offset of the group's C2 slice
+  const float* dpbuf;                     // [P][n1][NC]
+  uint32_t* work;
+  int n1, n1s, NC, nblk, tpp, nchunk;
+  float lr, eps;
+  int opt, fused;
+};
+
+struct YCtl {
+  uint64_t a1_full, a1_free;              // dP^T in TMEM + C1^T in smem (per tile)
+  uint64_t s_full[Y_NST], s_free[Y_NST];  // K-chunk stages
+  uint64_t d1_full, d1_free;              // dC2 accumulator (per group)
+  uint64_t d2_full, d2_free;              // dA accumulator (per tile)
+  uint64_t u_full[4], u_empty[4];
+  uint32_t ring[4][4];                    // group, first prefix, #prefixes, flags (1 first, 2 last, 4 done)
+  uint32_t claim[2];
+  uint32_t tmem;
+};
+
+__device__ __forceinline__ float lo32(float x) { return x - tc::tf32_trunc(x); }
+
+__global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
+  extern __shared__ __align__(128) char smem_raw[];
+  __shared__ YCtl ctl;
+  char* const smem = smem_raw + ((128u - (tc::smem_u32(smem_raw) & 127u)) & 127u);
+  char* const b1 = smem;                                 // C1^T hi | lo
+  char* const stg = smem + Y_B1;                         // stages: [A2 | B2 hi | B2 lo]
+  const int tid = threadIdx.x, w = tid >> 5, lane = tid & 31;
+  const uint32_t NG = a.counts[kCntNG];
+  if (tid == 0) {
+    tc::mbar_init(&ctl.a1_full, Y_LW * 32);
+    tc::mbar_init(&ctl.a1_free, 1);
+    for (int s = 0; s < Y_NST; ++s) { tc::mbar_init(&ctl.s_full[s], Y_LW * 32); tc::mbar_init(&ctl.s_free[s], 1); }
+    tc::mbar_init(&ctl.d1_full, 1);
+    tc::mbar_init(&ctl.d1_free, Y_EW * 32);
+    tc::mbar_init(&ctl.d2_full, 1);
+    tc::mbar_init(&ctl.d2_free, Y_EW * 32);
+    for (int s = 0; s < 4; ++s) { tc::mbar_init(&ctl.u_full[s], 1); tc::mbar_init(&ctl.u_empty[s], 1 + Y_EW); }
+    tc::fence_mbar_init();
+  }
+  if (w == Y_MMA_W) tc::tmem_alloc(&ctl.tmem, 512);
+  tc::fence_before();
+  __syncthreads();
+  tc::fence_after();
+  const uint32_t tm = ctl.tmem;
+  // TMEM columns: [0,128) dP^T hi (64 per c-block), [128,256) lo, [256,384) dC2^T (64 per
+  // c-block), [384,448) dA pass B = C2_hi, [448,512) dA pass B = C2_lo.
+  const int tpp = a.tpp, NC = a.NC;
+
+  if (w < Y_LW) {
+    // ------------------------------- loaders -------------------------------
+    // Jobs = (group, tile, K-chunk) in a static round-robin group order, so the issue side can
+    // run two chunks ahead across tile and group boundaries.  A chunk is copied with cp.async
+    // straight into its MMA layout (dP rows -> A2 rows 0..63, C2 rows -> B2 hi); each thread
+    // then writes the lo parts of the 16-byte pieces it copied, and the warps owning the
+    // chunk's TMEM lane quarters extract dP^T (hi, lo) from A2 into TMEM for the dC2 GEMM.
+    struct Job { uint32_t g, q1, qa; int ck; };
+    const uint32_t G0 = blockIdx.x, GS = gridDim.x;
+    auto start = [&](Job& j, uint32_t g) {
+      j.g = g; j.ck = 0;
+      if (g < NG) { j.qa = a.grp_off[g]; j.q1 = a.grp_off[g + 1]; }
+    };
+    auto advance = [&](Job& j) {
+      if (++j.ck < a.nchunk) return;
+      j.ck = 0;
+      j.qa += tpp;
+      if (j.qa >= j.q1) start(j, j.g + GS);
+    };
+    const int mb = tid & 63;                  // copy map: row mb, float4 columns (tid >> 6) + 4 k
+    auto issue = [&](const Job& j, uint32_t sidx) {
+      const uint32_t rows = min((uint32_t)tpp, j.q1 - j.qa) << a.n1s;
+      const float* dps = a.dpbuf + (size_t)j.qa * a.n1 * NC + j.ck * 64;
+      const float* c2 = a.cores + a.grp_c2[j.g] + j.ck * 64;
+      const uint32_t a2 = tc::smem_u32(stg + (sidx % Y_NST) * Y_STAGE), b2 = a2 + Y_A2;
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        const int c4 = 4 * ((tid >> 6) + 4 * k);
+        const uint32_t oa = (uint32_t)((c4 >> 2) * Y_A2LBO + (mb >> 3) * 128 + (mb & 7) * 16);
+        tc::cp_async16_z(a2 + oa, dps + (size_t)(mb < (int)rows ? mb : 0) * NC + c4, mb < (int)rows);
+        tc::cp_async16(b2 + tc::cm_off(mb, c4, 8), c2 + (size_t)mb * NC + c4);
+      }
+    };
+    uint32_t ui = 0, si = 0, sp = 0;          // tile counter, issued / processed chunk counters
+    Job P, I;
+    start(P, G0);
+    I = P;
+    for (int d = 0; d < Y_NST - 1; ++d) {
+      if (I.g < NG) {
+        tc::mbar_wait(&ctl.s_free[si % Y_NST], ((si / Y_NST) & 1) ^ 1);
+        issue(I, si);
+        advance(I);
+        ++si;
+      }
+      tc::cp_commit();
+    }
+    while (P.g < NG) {
+      const uint32_t np = min((uint32_t)tpp, P.q1 - P.qa);
+      const int rows = (int)np << a.n1s;
+      if (P.ck == 0) {
+        const uint32_t q0 = a.grp_off[P.g];
+        const uint32_t fl = (P.qa == q0 ? 1u : 0u) | (P.qa + tpp >= P.q1 ? 2u : 0u);
+        if (tid == 0) {
+          tc::mbar_wait(&ctl.u_empty[ui & 3], ((ui >> 2) & 1) ^ 1);
+          ctl.ring[ui & 3][0] = P.g; ctl.ring[ui & 3][1] = P.qa; ctl.ring[ui & 3][2] = np; ctl.ring[ui & 3][3] = fl;
+          tc::mbar_arrive(&ctl.u_full[ui & 3]);
+        }
+        // C1^T -> B1 = CM(r1, m) hi | lo (element (r1, m) = C1 row m, column r1); zero past the tile
+        float4 cv[4];
+        const bool ok = mb < rows;
+        const uint32_t arow = ok ? a.grp_arow[P.qa + (mb >> a.n1s)] + (mb & ((1 << a.n1s) - 1)) : 0u;
+        const float4* src = reinterpret_cast<const float4*>(a.cores + (size_t)arow * YR);
+#pragma unroll
+        for (int k = 0; k < 4; ++k) cv[k] = ok ? __ldg(src + (tid >> 6) + 4 * k) : make_float4(0.f, 0.f, 0.f, 0.f);
+        tc::mbar_wait(&ctl.a1_free, (ui & 1) ^ 1);      // previous tile's dC2 GEMM done
+        tc::fence_after();
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          const int r0 = 4 * ((tid >> 6) + 4 * k);
+          const float v[4] = {cv[k].x, cv[k].y, cv[k].z, cv[k].w};
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            const uint32_t off = tc::cm_off(r0 + i, mb, YR / 8);
+            *reinterpret_cast<float*>(b1 + off) = v[i];
+            *reinterpret_cast<float*>(b1 + Y_B1 / 2 + off) = lo32(v[i]);
+          }
+        }
+      }
+      // chunk P landed (one newer chunk may still be in flight)
+      tc::cp_wait<Y_NST - 2>();
+      const uint32_t sidx = sp % Y_NST;
+      char* a2 = stg + sidx * Y_STAGE;
+      char* b2h = a2 + Y_A2;
+      char* b2l = b2h + Y_B2 / 2;
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        const int c4 = 4 * ((tid >> 6) + 4 * k);
+        const uint32_t oa = (uint32_t)((c4 >> 2) * Y_A2LBO + (mb >> 3) * 128 + (mb & 7) * 16);
+        const uint32_t ol = (uint32_t)((c4 >> 2) * Y_A2LBO + ((64 + mb) >> 3) * 128 + (mb & 7) * 16);
+        const float4 p = *reinterpret_cast<const float4*>(a2 + oa);
+        *reinterpret_cast<float4*>(a2 + ol) = make_float4(lo32(p.x), lo32(p.y), lo32(p.z), lo32(p.w));
+        const uint32_t ob = tc::cm_off(mb, c4, 8);
+        const float4 q = *reinterpret_cast<const float4*>(b2h + ob);
+        *reinterpret_cast<float4*>(b2l + ob) = make_float4(lo32(q.x), lo32(q.y), lo32(q.z), lo32(q.w));
+      }
+      tc::named_sync(1, Y_LW * 32);                     // whole chunk (hi and lo) visible
+      {   // dP^T of this chunk -> TMEM: chunk ck covers c-block ck / 2, lane quarters 2 (ck & 1) + {0, 1}
+        const int blk = P.ck >> 1, Q = w & 3;
+        if ((Q >> 1) == (P.ck & 1) && blk < a.nblk) {
+          const int cc = 32 * (Q & 1) + lane;             // column inside the chunk
+          const int m0 = 32 * (w >> 2);                    // warps 0-3: rows 0..31, 4-7: 32..63
+          float xh[32], xl[32];
+#pragma unroll
+          for (int i = 0; i < 32; ++i) {
+            const int m = m0 + i;
+            const uint32_t base = (uint32_t)((cc >> 2) * Y_A2LBO + (m & 7) * 16 + (cc & 3) * 4);
+            xh[i] = *reinterpret_cast<const float*>(a2 + base + (m >> 3) * 128);
+            xl[i] = *reinterpret_cast<const float*>(a2 + base + ((64 + m) >> 3) * 128);
+          }
+          tc::tmem_st32(tc::taddr(tm + blk * 64 + m0, 32 * Q, 0), xh);
+          tc::tmem_st32(tc::taddr(tm + 128 + blk * 64 + m0, 32 * Q, 0), xl);
+          tc::tmem_wait_st();
+        }
+      }
+      tc::fence_async_smem();
+      tc::fence_before();
+      tc::mbar_arrive(&ctl.s_full[sidx]);
+      if (P.ck == a.nchunk - 1) {
+        tc::mbar_arrive(&ctl.a1_full);
+        ++ui;
+      }
+      ++sp;
+      advance(P);
+      // refill: the chunk two ahead
+      if (I.g < NG) {
+        tc::mbar_wait(&ctl.s_free[si % Y_NST], ((si / Y_NST) & 1) ^ 1);
+        issue(I, si);
+        advance(I);
+        ++si;
+      }
+      tc::cp_commit();
+    }
+    tc::cp_wait<0>();
+    if (tid == 0) {
+      tc::mbar_wait(&ctl.u_empty[ui & 3], ((ui >> 2) & 1) ^ 1);
+      ctl.ring[ui & 3][3] = 4u;
+      tc::mbar_arrive(&ctl.u_full[ui & 3]);
+    }
+  } else if (w == Y_MMA_W) {
+    // ------------------------------- MMA issuer -------------------------------
+    uint32_t sk = 0, gs = 0;
+    for (uint32_t ui = 0;; ++ui) {
+      tc::mbar_wait(&ctl.u_full[ui & 3], (ui >> 2) & 1);
+      const uint32_t fl = ctl.ring[ui & 3][3];
+      __syncwarp();
+      if (lane == 0) tc::mbar_arrive(&ctl.u_empty[ui & 3]);
+      if (fl & 4u) break;
+      // dA = [dP_hi; dP_lo] . C2_{hi,lo}^T over the K chunks (as they land)
+      tc::mbar_wait(&ctl.d2_free, (ui & 1) ^ 1);
+      tc::fence_after();
+      for (int ck = 0; ck < a.nchunk; ++ck, ++sk) {
+        const uint32_t s = sk % Y_NST;
+        tc::mbar_wait(&ctl.s_full[s], (sk / Y_NST) & 1);
+        tc::fence_after();
+        if (lane == 0) {
+          const uint32_t id = tc::idesc_tf32(128, 64, false, false);
+          const uint32_t a2 = tc::smem_u32(stg + s * Y_STAGE), b2h = a2 + Y_A2, b2l = b2h + Y_B2 / 2;
+#pragma unroll
+          for (int kk = 0; kk < 8; ++kk) {
+            const uint64_t da = tc::sdesc(a2 + kk * 2 * Y_A2LBO, Y_A2LBO, 128);
+            const uint64_t dbh = tc::sdesc(b2h + kk * 2 * 8 * 128, 8 * 128, 128);
+            const uint64_t dbl = tc::sdesc(b2l + kk * 2 * 8 * 128, 8 * 128, 128);
+            const uint32_t acc = (ck > 0 || kk > 0) ? 1u : 0u;
+            tc::mma_tf32(tm + 384, da, dbh, id, acc);
+            tc::mma_tf32(tm + 448, da, dbl, id, acc);
+          }
+          tc::commit(&ctl.s_free[s]);
+          if (ck + 1 == a.nchunk) tc::commit(&ctl.d2_full);
+        }
+        __syncwarp();
+      }
+      // dC2^T += dP^T . C1  (K = 64 tile rows), after the whole tile's dP^T reached TMEM
+      tc::mbar_wait(&ctl.a1_full, ui & 1);
+      if (fl & 1u) tc::mbar_wait(&ctl.d1_free, (gs & 1) ^ 1);
+      tc::fence_after();
+      if (lane == 0) {
+        const uint32_t id = tc::idesc_tf32(128, 64, false, false);
+        const uint32_t bh = tc::smem_u32(b1), bl = bh + Y_B1 / 2;
+        for (int blk = 0; blk < a.nblk; ++blk) {
+          const uint32_t d = tm + 256 + blk * 64;
+#pragma unroll
+          for (int kk = 0; kk < YT / 8; ++kk) {
+            const uint32_t o = kk * 2 * (YR / 8) * 128;
+            const uint64_t dbh = tc::sdesc(bh + o, (YR / 8) * 128, 128);
+            const uint64_t dbl = tc::sdesc(bl + o, (YR / 8) * 128, 128);
+            const uint32_t ah = tm + blk * 64 + kk * 8, al = tm + 128 + blk * 64 + kk * 8;
+            tc::mma_tf32_ts(d, ah, dbh, id, ((fl & 1u) && kk == 0) ? 0u : 1u);
+            tc::mma_tf32_ts(d, ah, dbl, id, 1u);
+            tc::mma_tf32_ts(d, al, dbh, id, 1u);
+          }
+        }
+        tc::commit(&ctl.a1_free);
+        if (fl & 2u) tc::commit(&ctl.d1_full);
+      }
+      __syncwarp();
+      if (fl & 2u) ++gs;
+    }
+  } else {
+    // ------------------------------- epilogue -------------------------------
+    const int Q = w & 3;
+    uint32_t gs = 0;
+    for (uint32_t ui = 0;; ++ui) {
+      tc::mbar_wait(&ctl.u_full[ui & 3], (ui >> 2) & 1);
+      const uint32_t g = ctl.ring[ui & 3][0], qa = ctl.ring[ui & 3][1];
+      const uint32_t np = ctl.ring[ui & 3][2], fl = ctl.ring[ui & 3][3];
+      __syncwarp();
+      if (fl & 4u) break;
+      const int rows = (int)np << a.n1s;
+      // dA: lanes 0..63 hold dP_hi rows (both passes), lanes 64..127 dP_lo rows (pass C2_hi)
+      tc::mbar_wait(&ctl.d2_full, ui & 1);
+      tc::fence_after();
+      {
+        const int m = (Q & 1) * 32 + lane;               // tile row of this lane
+        float v[32], x[32];
+        float* dst = nullptr;
+        if (m < rows) {
+          const uint32_t q = qa + (m >> a.n1s);
+          const uint32_t t = a.pfx_t[q];
+          dst = a.grads + a.meta[t].c1_off + ((size_t)(a.pfx_i1[q] << a.n1s) + (m & ((1 << a.n1s) - 1))) * YR;
+        }
+        for (int h = 0; h < 2; ++h) {
+          tc::tmem_ld32(tc::taddr(tm + 384 + 32 * h, 32 * Q, 0), v);
+          if (Q < 2) {
+            tc::tmem_ld32(tc::taddr(tm + 448 + 32 * h, 32 * Q, 0), x);
+#pragma unroll
+            for (int i = 0; i < 32; ++i) v[i] += x[i];
+          }
+          if (dst) {
+#pragma unroll
+            for (int i = 0; i < 32; i += 4)
+              asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(dst + 32 * h + i), "f"(v[i]),
+                           "f"(v[i + 1]), "f"(v[i + 2]), "f"(v[i + 3])
+                           : "memory");
+          }
+        }
+      }
+      tc::fence_before();
+      tc::mbar_arrive(&ctl.d2_free);
+      if (fl & 2u) {
+        // group complete: dC2^T [c][r1] -> gradient or fused C2 update (this CTA owns the slice)
+        tc::mbar_wait(&ctl.d1_full, gs & 1);
+        tc::fence_after();
+        const unsigned long long so = a.grp_c2[g];
+        for (int blk = 0; blk < a.nblk; ++blk) {
+          const int c = blk * 128 + Q * 32 + lane;
+          for (int h = 0; h < 2; ++h) {
+            float v[32];
+            tc::tmem_ld32(tc::taddr(tm + 256 + blk * 64 + 32 * h, 32 * Q, 0), v);
+            if (c < NC) {
+              const size_t base = so + (size_t)(32 * h) * NC + c;
+              if (!a.fused) {
+#pragma unroll
+                for (int i = 0; i < 32; ++i) a.grads[base + (size_t)i * NC] = v[i];
+              } else if (a.opt == TTEMB_SGD) {
+                float old[32];
+#pragma unroll
+                for (int i = 0; i < 32; ++i) old[i] = a.cores[base + (size_t)i * NC];
+#pragma unroll
+                for (int i = 0; i < 32; ++i) a.cores[base + (size_t)i * NC] = old[i] - a.lr * v[i];
+              } else {
+#pragma unroll
+                for (int h2 = 0; h2 < 32; h2 += 16) {
+                  float old[16], st[16];
+#pragma unroll
+                  for (int i = 0; i < 16; ++i) {
+                    old[i] = a.cores[base + (size_t)(h2 + i) * NC];
+                    st[i] = a.state[base + (size_t)(h2 + i) * NC];
+                  }
+#pragma unroll
+                  for (int i = 0; i < 16; ++i) {
+                    const float gr = v[h2 + i], sn = st[i] + gr * gr;
+                    a.state[base + (size_t)(h2 + i) * NC] = sn;
+                    a.cores[base + (size_t)(h2 + i) * NC] = old[i] - a.lr * gr / (sqrtf(sn) + a.eps);
+                  }
+                }
+              }
+            }
+          }
+        }
+        tc::fence_before();
+        tc::mbar_arrive(&ctl.d1_free);
+        ++gs;
+      }
+      if (lane == 0) tc::mbar_arrive(&ctl.u_empty[ui & 3]);
+    }
+  }
+  tc::fence_before();
+  __syncthreads();
+  tc::fence_after();
+  if (w == Y_MMA_W) tc::tmem_dealloc(tm, 512);
+}
+
+}  // namespace
+
+cudaError_t configure_bwdtc(Ctx& c) {
+  if (!fused_eligible(c)) return cudaSuccess;
+  return cudaFuncSetAttribute(k_prefix_bwd, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBwdSmem);
+}
+
+// dC2 (fused update) and dC1 partials from the dP stash; requires run_fused_fwd's per-step
+// tables (grp_arow, grp_c2).
+cudaError_t run_prefix_bwd(Ctx& c, float lr, cudaStream_t s) {
+  const PlanDev& p = c.p;
+  YArgs a;
+  a.cores = c.cores; a.grads = c.grads; a.state = c.state; a.meta = c.d_meta; a.counts = p.counts;
+  a.grp_off = p.grp_off; a.grp_t = p.grp_t; a.pfx_i1 = p.pfx_i1; a.pfx_t = p.pfx_t; a.grp_arow = p.grp_arow;
+  a.grp_c2 = p.grp_c2; a.dpbuf = p.dpbuf; a.work = p.work + 2;
+  a.n1 = c.n1; a.n1s = c.n1 == 1 ? 0 : c.n1 == 2 ? 1 : c.n1 == 4 ? 2 : 3;
+  a.NC = c.NC; a.nblk = (c.NC + 127) / 128; a.tpp = YT / c.n1; a.nchunk = (c.NC + 63) / 64;
+  a.lr = lr; a.eps = c.eps; a.opt = c.opt; a.fused = (c.flags & TTEMB_FUSED_UPDATE) ? 1 : 0;
+  StageScope sc(c, ST_BWD_PREFIX, s);
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(c.NG_cap, (int64_t)c.sm_count));
+  k_prefix_bwd<<<grid, Y_THREADS, kBwdSmem, s>>>(a);
+  return cudaGetLastError();
+}
+
+}  // namespace ttemb

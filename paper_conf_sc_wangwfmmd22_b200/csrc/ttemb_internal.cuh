@@ -135,6 +135,8 @@ bool fused_eligible(const Ctx& c);
 cudaError_t configure_fused(Ctx& c);
 cudaError_t run_fused_fwd(Ctx& c, cudaStream_t s);
 cudaError_t run_rows_bwd2(Ctx& c, cudaStream_t s);
+cudaError_t configure_bwdtc(Ctx& c);
+cudaError_t run_prefix_bwd(Ctx& c, float lr, cudaStream_t s);
 
 // ---- small helpers -------------------------------------------------------------------
 static inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }

@@ -999,18 +999,22 @@ cudaError_t run_tc_fwd(Ctx& c, float* out, cudaStream_t s) {
 
 // Backward contractions: dP / dC3 row stage, then the group GEMMs (dC2, dA).
 cudaError_t run_tc_bwd(Ctx& c, float lr, cudaStream_t s) {
+  if (fused_eligible(c)) {
+    cudaError_t e;
+    {
+      StageScope sc(c, ST_BWD_ROWS, s);
+      e = run_rows_bwd2(c, s);
+    }
+    if (e == cudaSuccess) e = run_prefix_bwd(c, lr, s);
+    return e;
+  }
   TcArgs a = make_tc_args(c, lr, c.p.work + 1, nullptr);
   {
     StageScope sc(c, ST_BWD_ROWS, s);
-    if (fused_eligible(c)) {
-      cudaError_t e = run_rows_bwd2(c, s);
-      if (e != cudaSuccess) return e;
-    } else {
     k_dp_zero<<<grid_for(c, c.P_cap, 8, 8), 256, 0, s>>>(a);
     const int grid = grid_for(c, cdiv(c.U_cap, RCH), 4, 8);
     if (c.n3 == 4) k_rows_bwd<4><<<grid, 128, 0, s>>>(a);
     else k_rows_bwd<8><<<grid, 128, 0, s>>>(a);
-    }
   }
   {
     StageScope sc(c, ST_BWD_PREFIX, s);
