@@ -120,6 +120,59 @@ k_agg_fix(const uint32_t* __restrict__ skey, const uint32_t* __restrict__ spos,
   }
 }
 
+
+// a8 (in-advance gradient aggregation): G_u = sum of grad_out over the occurrences of
+// unique row u.  Warp = 32 consecutive sorted occurrences; each half-warp walks every other
+// occurrence (lanes = float4 columns) and adds its running sum into G_u with one vector
+// reduction per (half-warp, segment piece).  Zipf-hot rows (thousands of occurrences) are
+// spread over many warps; G is zeroed first (rows [0, U) only).
+__global__ void __launch_bounds__(256) k_zero_rows(float* __restrict__ buf, const uint32_t* __restrict__ counts, int N) {
+  const int64_t n4 = (int64_t)counts[kCntU] * N / 4;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += (int64_t)gridDim.x * blockDim.x)
+    reinterpret_cast<float4*>(buf)[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+}
+
+__global__ void __launch_bounds__(256)
+k_agg_scatter(const float* __restrict__ grad_out, const uint32_t* __restrict__ sbag,
+              const uint32_t* __restrict__ spos, const uint32_t* __restrict__ inverse, int64_t nnz, int N,
+              float* __restrict__ gbuf) {
+  const int lane = threadIdx.x & 31;
+  const int NV = N >> 2, P = 32 / NV;            // float4 columns; occurrences in flight per step
+  const int f = lane % NV, p = lane / NV;
+  const int64_t nch = (nnz + 31) / 32;
+  const int64_t nw = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t ch = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); ch < nch; ch += nw) {
+    const int64_t k0 = ch * 32;
+    const int cnt = (int)min((int64_t)32, nnz - k0);
+    uint32_t bl = 0, ul = 0xffffffffu;
+    if (lane < cnt) {
+      bl = __ldg(sbag + k0 + lane);
+      ul = __ldg(inverse + __ldg(spos + k0 + lane));
+    }
+    float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+    uint32_t cur = 0xffffffffu;
+    for (int i0 = 0; i0 < cnt; i0 += P) {
+      const int i = i0 + p;
+      const uint32_t bag = __shfl_sync(0xffffffffu, bl, i & 31);
+      const uint32_t u = __shfl_sync(0xffffffffu, ul, i & 31);
+      if (i < cnt) {
+        if (u != cur) {
+          if (cur != 0xffffffffu)
+            asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(gbuf + (size_t)cur * N + 4 * f),
+                         "f"(acc.x), "f"(acc.y), "f"(acc.z), "f"(acc.w) : "memory");
+          acc = make_float4(0.f, 0.f, 0.f, 0.f);
+          cur = u;
+        }
+        const float4 v = __ldg(reinterpret_cast<const float4*>(grad_out + (size_t)bag * N) + f);
+        acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
+      }
+    }
+    if (cur != 0xffffffffu)
+      asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(gbuf + (size_t)cur * N + 4 * f),
+                   "f"(acc.x), "f"(acc.y), "f"(acc.z), "f"(acc.w) : "memory");
+  }
+}
+
 struct BwdArgs {
   float* cores;
   float* grads;
@@ -195,19 +248,22 @@ cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s
   }
   if (c.nnz > 0) {
     StageScope sc(c, ST_AGG, s);
-    const int64_t total = agg_chunks(c.nnz) * c.N;
-    if (c.N % 4 == 0)
-      k_agg<4><<<grid_for(c, total / 4, 256, 32), 256, 0, s>>>(grad_out, p.skey, p.sbag, p.spos,
-                                                              p.inverse, p.seg_off, c.nnz, c.N,
-                                                              p.gbuf, p.aggpart);
-    else
-      k_agg<1><<<grid_for(c, total, 256, 32), 256, 0, s>>>(grad_out, p.skey, p.sbag, p.spos, p.inverse,
-                                                          p.seg_off, c.nnz, c.N, p.gbuf, p.aggpart);
-  }
-  if (c.nnz > 0) {
-    StageScope sc(c, ST_AGG_FIX, s);
-    k_agg_fix<<<grid_for(c, agg_chunks(c.nnz) * 32, 256, 32), 256, 0, s>>>(
-        p.skey, p.spos, p.inverse, p.seg_off, c.nnz, c.N, p.aggpart, p.gbuf);
+    if (c.N % 4 == 0 && c.N <= 128 && (128 % c.N) == 0) {
+      k_zero_rows<<<grid_for(c, c.U_cap * c.N / 4, 256, 8), 256, 0, s>>>(p.gbuf, p.counts, c.N);
+      k_agg_scatter<<<grid_for(c, cdiv(c.nnz, 32), 8, 32), 256, 0, s>>>(grad_out, p.sbag, p.spos, p.inverse,
+                                                                         c.nnz, c.N, p.gbuf);
+    } else {
+      const int64_t total = agg_chunks(c.nnz) * c.N;
+      if (c.N % 4 == 0)
+        k_agg<4><<<grid_for(c, total / 4, 256, 32), 256, 0, s>>>(grad_out, p.skey, p.sbag, p.spos,
+                                                                p.inverse, p.seg_off, c.nnz, c.N,
+                                                                p.gbuf, p.aggpart);
+      else
+        k_agg<1><<<grid_for(c, total, 256, 32), 256, 0, s>>>(grad_out, p.skey, p.sbag, p.spos, p.inverse,
+                                                            p.seg_off, c.nnz, c.N, p.gbuf, p.aggpart);
+      k_agg_fix<<<grid_for(c, agg_chunks(c.nnz) * 32, 256, 32), 256, 0, s>>>(
+          p.skey, p.spos, p.inverse, p.seg_off, c.nnz, c.N, p.aggpart, p.gbuf);
+    }
   }
   BwdArgs a;
   a.cores = c.cores; a.grads = c.grads; a.state = c.state; a.meta = c.d_meta;

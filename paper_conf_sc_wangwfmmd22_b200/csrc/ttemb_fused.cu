@@ -352,9 +352,10 @@ constexpr int RW_WARPS = 8, RW_RCH = 16, RW_NSL = 3;
 struct RowArgs {
   const float* cores;
   const TableMeta* meta;
-  const uint32_t *counts, *row_pfx, *row_i3, *pfx_t;
+  const uint32_t *counts, *row_pfx, *row_i3, *pfx_t, *seg_off, *sbag;
   const float* pbuf;          // [P][n1][NC]
   float* rows;                // [U][N]
+  float* out;                 // [B][T][N]: written directly when every bag holds one id (a7)
   int n1, n1s, n2, N, NC;
 };
 
@@ -670,7 +671,7 @@ cudaError_t configure_fused(Ctx& c) {
   return e;
 }
 
-cudaError_t run_fused_fwd(Ctx& c, cudaStream_t s) {
+cudaError_t run_fused_fwd(Ctx& c, float* out, cudaStream_t s) {
   const PlanDev& p = c.p;
   XArgs a;
   a.cores = c.cores; a.meta = c.d_meta; a.counts = p.counts; a.grp_off = p.grp_off; a.grp_t = p.grp_t;
@@ -718,7 +719,7 @@ cudaError_t run_fused_fwd(Ctx& c, cudaStream_t s) {
     StageScope sc(c, ST_FWD_ROWS, s);
     RowArgs r;
     r.cores = c.cores; r.meta = c.d_meta; r.counts = p.counts; r.row_pfx = p.row_pfx; r.row_i3 = p.row_i3;
-    r.pfx_t = p.pfx_t; r.pbuf = p.pbuf; r.rows = p.rows;
+    r.pfx_t = p.pfx_t; r.pbuf = p.pbuf; r.rows = p.rows; r.seg_off = p.seg_off; r.sbag = p.sbag; r.out = out;
     r.n1 = c.n1; r.n1s = a.n1s; r.n2 = c.n2; r.N = c.N; r.NC = c.NC;
     const int grid = grid_for(c, cdiv(c.U_cap, RW_RCH), RW_WARPS, 4);
     if (c.n3 == 4) k_rows_fwd2<4><<<grid, RW_WARPS * 32, rows_smem(4), s>>>(r);

@@ -65,6 +65,35 @@ k_pool(const float* __restrict__ rows, const uint32_t* __restrict__ inverse,
   }
 }
 
+// a7 when every bag holds exactly one id (the one-hot configs): out[bag_of[j]] = E_{inverse[j]}
+// -- thread = (position, float4 column), four independent items per thread.
+__global__ void __launch_bounds__(256)
+k_pool_single(const float* __restrict__ rows, const uint32_t* __restrict__ inverse,
+              const uint32_t* __restrict__ bag_of, int64_t nnz, int N, float* __restrict__ out,
+              const uint32_t* __restrict__ counts) {
+  if (counts[kCntMulti] != 0) return;
+  const int NV = N >> 2;
+  const int64_t total = nnz * NV, stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t e0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e0 < total; e0 += 4 * stride) {
+    float4 v[4];
+    int64_t dst[4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const int64_t e = e0 + i * stride;
+      dst[i] = -1;
+      if (e < total) {
+        const int64_t j = e / NV;
+        const int f = (int)(e - j * NV);
+        v[i] = __ldg(reinterpret_cast<const float4*>(rows + (size_t)__ldg(inverse + j) * N) + f);
+        dst[i] = (int64_t)__ldg(bag_of + j) * NV + f;
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+      if (dst[i] >= 0) reinterpret_cast<float4*>(out)[dst[i]] = v[i];
+  }
+}
+
 }  // namespace
 
 cudaError_t run_group_fwd(Ctx& c, cudaStream_t s);
@@ -80,9 +109,14 @@ cudaError_t run_forward_compute(Ctx& c, float* out, const int64_t* offsets, cuda
     StageScope sc(c, ST_POOL, s);
     const int64_t total = (int64_t)c.T * c.B * c.N;
     if (total > 0) {
-      if (c.N % 4 == 0)
+      if (c.N % 4 == 0) {
+        // one id per bag (device flag): a position-parallel copy; otherwise the bag-parallel sum
+        if (c.nnz > 0)
+          k_pool_single<<<grid_for(c, c.nnz * c.N / 16, 256, 32), 256, 0, s>>>(p.rows, p.inverse, p.bag_of,
+                                                                              c.nnz, c.N, out, p.counts);
         k_pool<4><<<grid_for(c, total / 16, 256, 32), 256, 0, s>>>(p.rows, p.inverse, offsets, c.nnz,
-                                                                 c.T, c.B, c.N, out, p.counts, 0);
+                                                                 c.T, c.B, c.N, out, p.counts, 1);
+      }
       else
         k_pool<1><<<grid_for(c, total / 4, 256, 32), 256, 0, s>>>(p.rows, p.inverse, offsets, c.nnz, c.T,
                                                              c.B, c.N, out, p.counts, 0);

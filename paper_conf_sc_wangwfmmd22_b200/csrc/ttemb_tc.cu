@@ -964,7 +964,7 @@ cudaError_t configure_tc(Ctx& c) {
 
 // Forward contractions: P (tcgen05) then rows / direct output.
 cudaError_t run_tc_fwd(Ctx& c, float* out, cudaStream_t s) {
-  if (fused_eligible(c)) return run_fused_fwd(c, s);
+  if (fused_eligible(c)) return run_fused_fwd(c, out, s);
   TcArgs a = make_tc_args(c, 0.f, c.p.work + 0, out);
   {
     StageScope sc(c, ST_FWD_PREFIX, s);

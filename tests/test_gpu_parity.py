@@ -262,11 +262,11 @@ def test_int32_indices_and_host_api():
     eh.backward_host(torch.as_tensor(go).pin_memory())
     torch.cuda.synchronize()
     torch.testing.assert_close(hout, o64.cpu(), rtol=0, atol=0)
-    # dC2 is reduced without atomics: bitwise equal across runs; dC1 is summed with vector
-    # reductions in arrival order (R19 / Q19): equal up to fp32 reassociation
+    # the aggregated row gradients and dC1 are summed with vector reductions in arrival order
+    # (R19 / Q19): runs agree up to fp32 reassociation
     for a, b in zip(eh.grad_views(), e64.grad_views()):
-        torch.testing.assert_close(a[0], b[0], rtol=1e-5, atol=1e-6)
-        torch.testing.assert_close(a[1], b[1], rtol=0, atol=0)
+        for k in range(3):
+            torch.testing.assert_close(a[k], b[k], rtol=1e-5, atol=1e-5 * float(b[k].abs().max()))
 
 
 def test_deterministic_forward_and_plan():
