@@ -231,15 +231,20 @@ def workload_config(cfg, B, world, args):
 # ---------------------------------------------------------------------------
 # our arm
 # ---------------------------------------------------------------------------
-def kernels_per_step(emb_ctx, world, tc=True):
-    """Our kernel launches per step (cudaMemsetAsync excluded), matching the ncu launch list:
-    index stage = build_keys + hist_scan + kp passes + unique + prefix + (radix_hist +
-    hist_scan) + gp passes + groups; forward = contraction kernels + pool; backward = agg,
-    agg_fix, contraction kernels, dc1, dc1_fix (+ update_c3 fused / update after all-reduce)."""
-    kp, gp = emb_ctx
-    idx_stage = 1 + 1 + kp + 1 + 1 + 2 + gp + 1
-    fwd = (2 if tc else 1) + 1
-    bwd = 2 + (3 if tc else 1) + 2 + 1
+def kernels_per_step(emb_ctx, world, fused=True, cfg=None):
+    """Our kernel launches per step (cudaMemsetAsync excluded), matching the ncu launch list.
+    tcgen05 path: index stage = build_keys + hist_scan + kp radix passes + unique / prefix /
+    group scans; forward = prep + prefix GEMM + rows + pool (single + multi, one exits early);
+    backward = zero_rows + agg + dp_zero + rows_bwd + prefix GEMM bwd (+ 2 dense C1/C3 updates
+    when fused, + 1 update after the all-reduce otherwise)."""
+    kp, _ = emb_ctx
+    idx_stage = 1 + 1 + kp + 3
+    if fused:
+        fwd = 4
+        bwd = 5 + (2 if world == 1 else 1)
+    else:
+        fwd = 2
+        bwd = 2 + 1 + 1 + (1 if world == 1 else 1)
     return idx_stage + fwd + bwd
 
 
@@ -261,6 +266,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--stages", action="store_true", help="print per-stage times to stderr")
     ap.add_argument("--fp32-cores", action="store_true", help="force the FFMA contraction path (no tcgen05)")
+    ap.add_argument("--no-graph", dest="graph", action="store_false",
+                    help="launch every step eagerly instead of replaying a captured CUDA graph")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
@@ -327,10 +334,29 @@ def main():
     torch.cuda.synchronize()
     assert emb.check() == 0, "device-side input error"
 
+    # ---- optional CUDA graphs: one captured step per pool batch (same kernels, no launch gaps) ----
+    graphs = None
+    if args.graph and world == 1:
+        torch.cuda.synchronize()
+        graphs = []
+        for i in range(len(dpool)):
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g):
+                step(i)
+            graphs.append(g)
+        for i in range(len(graphs)):
+            graphs[i].replay()
+        torch.cuda.synchronize()
+        assert emb.check() == 0, "device-side input error (graph replay)"
+
+    def run(i):
+        if graphs is not None:
+            graphs[i % len(graphs)].replay()
+        else:
+            step(i)
+
     # ---- timed region (device events per step; L2 flushed between steps, untimed) ----
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-    emb.set_timing(True)
-    emb.stage_times()   # reset
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
@@ -338,13 +364,11 @@ def main():
         for i in range(args.steps):
             flush.fill_(i & 0xff)
             ev[i][0].record(stream)
-            step(i)
+            run(i)
             ev[i][1].record(stream)
         torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
-    stages = emb.stage_times()
-    emb.set_timing(False)
     t_ms = sum(a.elapsed_time(b) for a, b in ev)
     t_max = torch.tensor([t_ms], dtype=torch.float64, device=dev)
     if world > 1:
@@ -352,6 +376,18 @@ def main():
     t_ms = float(t_max.item())
     look_step = sum(int(p[0].shape[0]) for p in pool) / len(pool)
     value = world * look_step * args.steps / (t_ms / 1e3)
+
+    # ---- per-stage breakdown: a separate eager pass with CUDA events around every stage on the
+    #      launching stream (kept out of the timed region so the events do not perturb it) ----
+    emb.set_timing(True)
+    emb.stage_times()   # reset
+    for i in range(args.steps):
+        flush.fill_(i & 0xff)
+        step(i)
+    torch.cuda.synchronize()
+    stages = emb.stage_times()
+    emb.set_timing(False)
+    stage_total_ms = sum(v[0] for v in stages.values())
 
     # ---- counts of the last step for the roofline ----
     counts = emb.counts()
@@ -392,7 +428,7 @@ def main():
         ach = b1 / (per_launch_ms / 1e3) / 1e9
         roof = {"bound": "hbm", "kernel": dname, "achieved": ach, "peak": hbm_peak, "unit": "GB/s",
                 "frac": ach / hbm_peak, "traffic": None, "peak_source": f"{peak_kind} copy bandwidth"}
-    roof["share_of_step"] = dms / max(t_ms, 1e-9)
+    roof["share_of_step"] = dms / max(stage_total_ms, 1e-9)
     tr_path = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tr_path):      # DRAM bytes per launch from the committed ncu --set full capture
         tr = json.load(open(tr_path))
@@ -451,7 +487,8 @@ def main():
                 "scaling": args.scaling, "vs_baseline": None, "dtype": "f32", "data": "synthetic",
                 "config": workload_config(cfg, B, world, args), "roofline": roof,
                 "step_roofline": step_roof, "cpu_baseline": cpu, "e2e": e2e,
-                "gpu_launches": kernels_per_step(emb_passes(emb), world, tc=tc_path(cfg, args)) * args.steps,
+                "gpu_launches": kernels_per_step(emb_passes(emb), world, fused=tc_path(cfg, args)) * args.steps,
+                "graph": bool(graphs is not None),
                 "clocks": clk.summary(),
                 "stages_us_per_step": {k: round(v[0] / args.steps * 1e3, 2) for k, v in stages.items() if v[1]}}
         print(json.dumps(line), flush=True)
@@ -460,14 +497,15 @@ def main():
 
 
 def tc_path(cfg, args):
+    """The tcgen05 path (R = 64, n2 R <= 256, n3 in {4, 8}, n1 a power of two <= 8)."""
     n1, n2, n3 = cfg.col_factors
     return (not args.fp32_cores) and cfg.rank == 64 and n3 in (4, 8) and n1 in (1, 2, 4, 8) \
-        and n1 * n2 <= 16 and n2 <= 7
+        and n1 * n2 <= 16 and n2 * cfg.rank <= 256
 
 
 def emb_passes(emb):
-    rows = sum(emb.table_rows)
-    kp = max(1, (max(rows - 1, 0).bit_length() + 7) // 8)
+    keys = sum(int(f[0]) * int(f[1]) * int(f[2]) for f in emb.row_factors)   # group-major plan keys
+    kp = max(1, (max(keys - 1, 0).bit_length() + 7) // 8)
     gb = sum(f[1] for f in emb.row_factors)
     gp = max(1, (max(gb - 1, 0).bit_length() + 7) // 8)
     return kp, gp
