@@ -219,19 +219,78 @@ def run_reference(args, cfg, rank, world):
     print(json.dumps(line), flush=True)
 
 
+def run_paper(args, cfg, rank, world):
+    """--impl paper: the paper's own GPU design (Alg. 1 reuse buffer + cuBLAS batched GEMMs,
+    aggregation by index_add; comparators/paper_design.py) on the same workload and GPU,
+    timed like our arm (device events, L2 flushed between steps).  SURVEY.md 8(f1)."""
+    import torch
+    from comparators.paper_design import PaperDesignTT
+    torch.backends.cuda.matmul.allow_tf32 = False
+    if world > 1 and rank != 0:
+        return
+    dev = torch.device("cuda", int(os.environ.get("LOCAL_RANK", "0")))
+    torch.cuda.set_device(dev)
+    B = cfg.batch
+    pool = []
+    for i in range(min(args.pool, 2)):
+        idx, off = W.make_batch(cfg, step=i, seed=args.seed, batch=B)
+        go = W.make_grad_out(cfg, B, step=i, seed=args.seed)
+        pool.append((torch.as_tensor(idx, device=dev), torch.as_tensor(off, device=dev),
+                     torch.as_tensor(go, device=dev)))
+    m = PaperDesignTT(cfg.table_rows, cfg.row_factors, cfg.col_factors, cfg.rank, dev)
+    m.load_cores(W.make_cores(cfg, seed=args.seed))
+    offs_host = [p[1].cpu() for p in pool]
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+
+    def step(i):
+        di, do, dg = pool[i % len(pool)]
+        m.forward(di, offs_host[i % len(pool)], B)
+        m.backward(dg)
+        m.update_sgd(args.lr)
+
+    for i in range(args.warmup):
+        step(i)
+    torch.cuda.synchronize()
+    stream = torch.cuda.current_stream()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    with Clocks(dev.index) as clk:
+        for i in range(args.steps):
+            flush.fill_(i & 0xff)
+            ev[i][0].record(stream)
+            step(i)
+            ev[i][1].record(stream)
+        torch.cuda.synchronize()
+    t_ms = sum(a.elapsed_time(b) for a, b in ev)
+    look = sum(int(p[0].shape[0]) for p in pool) / len(pool)
+    val = look * args.steps / (t_ms / 1e3)
+    line = {"metric": METRIC, "value": val, "unit": UNIT, "impl": "paper-design", "n_gpus": 1,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": t_ms / args.steps,
+            "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None, "dtype": "f32",
+            "data": "synthetic", "config": workload_config(cfg, B, 1, args),
+            "design": "Alg. 1 reuse buffer (torch.unique owners) + cuBLAS batched GEMM stages, index_add "
+                      "aggregation / pooling / core-gradient reduction, unfused SGD (P:178-196, P:346)",
+            "clocks": clk.summary()}
+    line["config"]["update"] = "unfused"
+    print(json.dumps(line), flush=True)
+
+
 def workload_config(cfg, B, world, args):
     return {"workload": cfg.name, "tables": cfg.num_tables, "max_rows": max(cfg.table_rows),
             "dim": cfg.dim, "col_factors": list(cfg.col_factors), "tt_rank": cfg.rank,
             "batch_per_gpu": B, "global_batch": B * world, "pooling": cfg.pooling,
             "ids": f"zipf{cfg.zipf_s}-{cfg.id_map}" if cfg.zipf_s else f"uniform-{cfg.id_map}",
-            "optimizer": args.opt, "update": "fused" if world == 1 else "allreduce+update",
-            "parallelism": f"dp{world}", "l2": "flushed between timed steps (untimed 512 MiB write)"}
+            "optimizer": args.opt,
+            "update": ("fused" if world == 1 and not getattr(args, "unfused", False)
+                       else "allreduce+update" if world > 1 else "unfused"),
+            "parallelism": f"dp{world}", "l2": "flushed between timed steps (untimed 512 MiB write)",
+            **({"ablation": [k for k in ("no_reuse", "no_agg", "unfused") if getattr(args, k, False)]}
+               if any(getattr(args, k, False) for k in ("no_reuse", "no_agg", "unfused")) else {})}
 
 
 # ---------------------------------------------------------------------------
 # our arm
 # ---------------------------------------------------------------------------
-def kernels_per_step(emb_ctx, world, fused=True, cfg=None):
+def kernels_per_step(emb_ctx, world, fused=True, cfg=None, fused_update=None):
     """Our kernel launches per step (cudaMemsetAsync excluded), matching the ncu launch list.
     tcgen05 path: index stage = build_keys + hist_scan + kp radix passes + unique / prefix /
     group scans; forward = prep + prefix GEMM + rows + pool (single + multi, one exits early);
@@ -239,9 +298,11 @@ def kernels_per_step(emb_ctx, world, fused=True, cfg=None):
     when fused, + 1 update after the all-reduce otherwise)."""
     kp, _ = emb_ctx
     idx_stage = 1 + 1 + kp + 3
+    if fused_update is None:
+        fused_update = world == 1
     if fused:
         fwd = 4
-        bwd = 5 + (2 if world == 1 else 1)
+        bwd = 5 + (2 if fused_update else 1)
     else:
         fwd = 2
         bwd = 2 + 1 + 1 + (1 if world == 1 else 1)
@@ -255,7 +316,8 @@ def main():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--config", default="c4")
     ap.add_argument("--rank", type=int, default=None, help="TT rank for c5 (32/64/128)")
-    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference", "paper"],
+                    help="reference = the CPU oracle; paper = the paper's design in torch/cuBLAS")
     ap.add_argument("--opt", default="sgd", choices=["sgd", "adagrad"])
     ap.add_argument("--ids", default="identity", choices=["identity", "perm"])
     ap.add_argument("--scaling", default=None, choices=["weak", "strong"])
@@ -266,6 +328,12 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--stages", action="store_true", help="print per-stage times to stderr")
     ap.add_argument("--fp32-cores", action="store_true", help="force the FFMA contraction path (no tcgen05)")
+    ap.add_argument("--no-reuse", action="store_true",
+                    help="ablation: no batch-level prefix reuse (TTEMB_NO_PREFIX_REUSE, P:419)")
+    ap.add_argument("--no-agg", action="store_true",
+                    help="ablation: no row dedup / in-advance gradient aggregation (TTEMB_NO_AGGREGATION, P:416)")
+    ap.add_argument("--unfused", action="store_true",
+                    help="ablation: backward writes dense core grads, separate update (P:421)")
     ap.add_argument("--no-graph", dest="graph", action="store_false",
                     help="launch every step eagerly instead of replaying a captured CUDA graph")
     args = ap.parse_args()
@@ -285,6 +353,9 @@ def main():
             dist.init_process_group("gloo")
         run_reference(args, cfg, rank, world)
         return
+    if args.impl == "paper":
+        run_paper(args, cfg, rank, world)
+        return
 
     import torch
     import torch.distributed as dist
@@ -296,7 +367,7 @@ def main():
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
     B = cfg.batch if args.scaling == "weak" else cfg.batch // world
-    fused = world == 1
+    fused = world == 1 and not args.unfused
 
     # ---- inputs: a pool of batches resident in HBM ----
     pool = []
@@ -312,7 +383,8 @@ def main():
     max_nnz = max(len(p[0]) for p in pool)
     emb = tt.TTEmbeddingBag(cfg.table_rows, cfg.row_factors, cfg.col_factors, cfg.rank, B, max_nnz,
                             optimizer=args.opt, fused_update=fused, device=local_rank,
-                            fp32_cores=args.fp32_cores)
+                            fp32_cores=args.fp32_cores, prefix_reuse=not args.no_reuse,
+                            aggregation=not args.no_agg)
     cores = W.make_cores(cfg, seed=args.seed)
     emb.load_cores(cores)
     dpool = [(torch.as_tensor(i, device=dev), torch.as_tensor(o, device=dev), torch.as_tensor(g, device=dev))
@@ -327,6 +399,7 @@ def main():
         emb.backward(dg, lr=args.lr)
         if world > 1:
             parallel.allreduce_grads(emb.grads)
+        if not fused:
             emb.update(args.lr)
 
     for i in range(args.warmup):
@@ -487,7 +560,8 @@ def main():
                 "scaling": args.scaling, "vs_baseline": None, "dtype": "f32", "data": "synthetic",
                 "config": workload_config(cfg, B, world, args), "roofline": roof,
                 "step_roofline": step_roof, "cpu_baseline": cpu, "e2e": e2e,
-                "gpu_launches": kernels_per_step(emb_passes(emb), world, fused=tc_path(cfg, args)) * args.steps,
+                "gpu_launches": kernels_per_step(emb_passes(emb), world, fused=tc_path(cfg, args),
+                                                 fused_update=fused) * args.steps,
                 "graph": bool(graphs is not None),
                 "clocks": clk.summary(),
                 "stages_us_per_step": {k: round(v[0] / args.steps * 1e3, 2) for k, v in stages.items() if v[1]}}

@@ -60,6 +60,14 @@ typedef enum { TTEMB_SGD = 0, TTEMB_ADAGRAD = 1 } ttemb_opt;
 /* ttemb_config.flags */
 #define TTEMB_FUSED_UPDATE 1u   /* backward applies the update (single replica) */
 #define TTEMB_FP32_CORES 2u     /* force the FP32 CUDA-core contraction path (no tcgen05) */
+/* Ablation switches (Fig. 14 / 17 / 18 of the paper).  Results are unchanged
+ * (same outputs and gradients up to fp32 rounding order); only the amount of work grows. */
+#define TTEMB_NO_PREFIX_REUSE 4u  /* every unique row computes its own prefix product
+                                     C1[i1] C2[i2] (disables batch-level intermediate-result
+                                     reuse) */
+#define TTEMB_NO_AGGREGATION 8u   /* every lookup occurrence is its own row in forward and
+                                     backward (disables row dedup and the in-advance gradient
+                                     aggregation) */
 
 typedef struct {
   int64_t num_rows;        /* M_t >= 1 */
@@ -78,7 +86,7 @@ typedef struct {
   int64_t max_nnz;               /* nnz capacity, <= 2^30                             */
   int32_t optimizer;             /* ttemb_opt                                         */
   float adagrad_eps;             /* Adagrad eps (PyTorch default 1e-10)               */
-  uint32_t flags;                /* TTEMB_FUSED_UPDATE | TTEMB_FP32_CORES             */
+  uint32_t flags;                /* TTEMB_FUSED_UPDATE | TTEMB_FP32_CORES | ablations */
 } ttemb_config;
 
 typedef struct ttemb_ctx* ttemb_t;

@@ -23,6 +23,8 @@ TTEMB_SGD = 0
 TTEMB_ADAGRAD = 1
 TTEMB_FUSED_UPDATE = 1
 TTEMB_FP32_CORES = 2
+TTEMB_NO_PREFIX_REUSE = 4
+TTEMB_NO_AGGREGATION = 8
 
 SYMBOLS = ["ttemb_query_sizes", "ttemb_create", "ttemb_destroy", "ttemb_core_layout",
            "ttemb_forward", "ttemb_backward", "ttemb_update", "ttemb_forward_host",

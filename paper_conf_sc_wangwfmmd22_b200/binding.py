@@ -27,8 +27,10 @@ def _stream_ptr(stream: Optional[torch.cuda.Stream]) -> int:
 def make_config(table_rows: Sequence[int], row_factors: Sequence[Tuple[int, int, int]],
                 col_factors: Tuple[int, int, int], rank: int, max_batch: int, max_nnz: int,
                 optimizer: str = "sgd", adagrad_eps: float = 1e-10, fused_update: bool = False,
-                index_bits: int = 64, num_cores: int = 3, fp32_cores: bool = False):
-    """Returns (ttemb_config, keep-alive table array)."""
+                index_bits: int = 64, num_cores: int = 3, fp32_cores: bool = False,
+                prefix_reuse: bool = True, aggregation: bool = True):
+    """Returns (ttemb_config, keep-alive table array).  prefix_reuse / aggregation = False set the
+    ablation flags TTEMB_NO_PREFIX_REUSE / TTEMB_NO_AGGREGATION."""
     T = len(table_rows)
     tabs = (L.ttemb_table * max(T, 1))()
     for t in range(T):
@@ -48,7 +50,9 @@ def make_config(table_rows: Sequence[int], row_factors: Sequence[Tuple[int, int,
     cfg.max_nnz = int(max_nnz)
     cfg.optimizer = {"sgd": L.TTEMB_SGD, "adagrad": L.TTEMB_ADAGRAD}[optimizer]
     cfg.adagrad_eps = float(adagrad_eps)
-    cfg.flags = (L.TTEMB_FUSED_UPDATE if fused_update else 0) | (L.TTEMB_FP32_CORES if fp32_cores else 0)
+    cfg.flags = ((L.TTEMB_FUSED_UPDATE if fused_update else 0) | (L.TTEMB_FP32_CORES if fp32_cores else 0)
+                 | (0 if prefix_reuse else L.TTEMB_NO_PREFIX_REUSE)
+                 | (0 if aggregation else L.TTEMB_NO_AGGREGATION))
     return cfg, tabs
 
 
@@ -149,7 +153,8 @@ class TTEmbeddingBag:
 
     def __init__(self, table_rows, row_factors, col_factors, rank, max_batch, max_nnz,
                  optimizer: str = "sgd", adagrad_eps: float = 1e-10, fused_update: bool = False,
-                 index_bits: int = 64, device: int = 0, fp32_cores: bool = False):
+                 index_bits: int = 64, device: int = 0, fp32_cores: bool = False,
+                 prefix_reuse: bool = True, aggregation: bool = True):
         L.load()
         self.table_rows = [int(x) for x in table_rows]
         self.row_factors = [tuple(int(y) for y in f) for f in row_factors]
@@ -163,7 +168,8 @@ class TTEmbeddingBag:
         self.device = torch.device("cuda", device)
         self._cfg, self._tabs = make_config(table_rows, row_factors, col_factors, rank, max_batch,
                                             max_nnz, optimizer, adagrad_eps, fused_update, index_bits,
-                                            fp32_cores=fp32_cores)
+                                            fp32_cores=fp32_cores, prefix_reuse=prefix_reuse,
+                                            aggregation=aggregation)
         cb, sb, gb, wb = ttemb_query_sizes(self._cfg)
         self.sizes = dict(core_bytes=cb, state_bytes=sb, grad_bytes=gb, workspace_bytes=wb)
         f32 = torch.float32

@@ -73,7 +73,8 @@ int validate(const ttemb_config* cfg) {
   if (cfg->max_nnz > (int64_t(1) << 30)) return TTEMB_ERR_UNSUPPORTED;
   if ((int64_t)cfg->num_tables * cfg->max_batch > (int64_t(1) << 31)) return TTEMB_ERR_UNSUPPORTED;
   if (cfg->optimizer != TTEMB_SGD && cfg->optimizer != TTEMB_ADAGRAD) return TTEMB_ERR_INVALID_ARG;
-  if (cfg->flags & ~(TTEMB_FUSED_UPDATE | TTEMB_FP32_CORES)) return TTEMB_ERR_INVALID_ARG;
+  if (cfg->flags & ~(TTEMB_FUSED_UPDATE | TTEMB_FP32_CORES | TTEMB_NO_PREFIX_REUSE | TTEMB_NO_AGGREGATION))
+    return TTEMB_ERR_INVALID_ARG;
   uint64_t total = 0, buckets = 0, keys = 0;
   for (int t = 0; t < cfg->num_tables; ++t) {
     const ttemb_table& tb = cfg->tables[t];
@@ -125,8 +126,9 @@ void plan_sizes(const ttemb_config* cfg, Ctx& c) {
   c.total_buckets = gb;
   c.key_passes = std::max(1, (bits_for(kb ? kb - 1 : 0) + 7) / 8);
   c.gkey_passes = std::max(1, (bits_for(gb ? gb - 1 : 0) + 7) / 8);
-  c.U_cap = std::min<int64_t>(c.max_nnz, (int64_t)rb);
-  c.P_cap = std::min<int64_t>(c.U_cap, (int64_t)pfx);
+  // Ablations (TTEMB_NO_*): every occurrence a row / every row a prefix.
+  c.U_cap = (c.flags & TTEMB_NO_AGGREGATION) ? c.max_nnz : std::min<int64_t>(c.max_nnz, (int64_t)rb);
+  c.P_cap = (c.flags & TTEMB_NO_PREFIX_REUSE) ? c.U_cap : std::min<int64_t>(c.U_cap, (int64_t)pfx);
   c.NG_cap = std::min<int64_t>(c.P_cap, (int64_t)gb);
   c.rs1_tiles = radix_tiles(c.max_nnz);
   c.rs2_tiles = radix_tiles(c.P_cap);

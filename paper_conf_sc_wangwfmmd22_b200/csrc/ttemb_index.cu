@@ -369,8 +369,9 @@ struct UniqueBody {
   const uint32_t* skey; const uint32_t* spos; const uint32_t* bag_of;
   uint32_t* ukey; uint32_t* seg_off; uint32_t* inverse; uint32_t* sbag; uint32_t* counts;
   uint32_t nnz;
+  uint32_t every;   // TTEMB_NO_AGGREGATION: each occurrence is its own row
   __device__ uint32_t size() const { return nnz; }
-  __device__ bool flag(uint32_t k) const { return k == 0 || skey[k] != skey[k - 1]; }
+  __device__ bool flag(uint32_t k) const { return every || k == 0 || skey[k] != skey[k - 1]; }
   __device__ void emit(uint32_t k, uint32_t slot, uint32_t f) const {
     const uint32_t u = f ? slot : slot - 1;
     if (f) { ukey[u] = skey[k]; seg_off[u] = k; }
@@ -395,6 +396,7 @@ struct PrefixBody {
   const uint32_t* ukey; const uint64_t* kbase; const TableMeta* meta; int T;
   uint32_t* row_pfx; uint32_t* row_i3; uint32_t* pfx_t; uint32_t* pfx_i1; uint32_t* pfx_i2;
   uint32_t* row_seg; uint32_t* counts;
+  uint32_t every;   // TTEMB_NO_PREFIX_REUSE: each row is its own prefix
   __device__ uint32_t size() const { return counts[kCntU]; }
   __device__ void decode(uint32_t u, int& t, uint32_t& pq, uint32_t& i3) const {
     const uint32_t key = ukey[u];
@@ -405,7 +407,7 @@ struct PrefixBody {
     i3 = local - pq * m3;
   }
   __device__ bool flag(uint32_t u) const {
-    if (u == 0) return true;
+    if (u == 0 || every) return true;
     int t0, t1; uint32_t p0, p1, x;
     decode(u, t1, p1, x);
     decode(u - 1, t0, p0, x);
@@ -506,7 +508,7 @@ cudaError_t run_index_stage(Ctx& c, const void* indices, const int64_t* offsets,
   {
     StageScope sc(c, ST_UNIQUE, s);
     UniqueBody b{p.skey, p.spos, p.bag_of, p.ukey, p.seg_off, p.inverse, p.sbag, p.counts,
-                 (uint32_t)nnz};
+                 (uint32_t)nnz, (c.flags & TTEMB_NO_AGGREGATION) ? 1u : 0u};
     const int64_t tiles = scan_tiles(nnz);
     k_scan<UniqueBody><<<(unsigned)(tiles ? tiles : 1), SC_T, 0, s>>>(b, p.sc_status, p.sc_counter + 0);
   }
@@ -514,7 +516,7 @@ cudaError_t run_index_stage(Ctx& c, const void* indices, const int64_t* offsets,
   {
     StageScope sc(c, ST_PREFIX, s);
     PrefixBody b{p.ukey, c.d_kbase, c.d_meta, c.T, p.row_pfx, p.row_i3, p.pfx_t, p.pfx_i1,
-                 p.pfx_i2, p.row_seg, p.counts};
+                 p.pfx_i2, p.row_seg, p.counts, (c.flags & TTEMB_NO_PREFIX_REUSE) ? 1u : 0u};
     const int64_t tiles = scan_tiles(c.U_cap);
     k_scan<PrefixBody><<<(unsigned)(tiles ? tiles : 1), SC_T, 0, s>>>(
         b, p.sc_status + c.sc_tiles, p.sc_counter + 1);

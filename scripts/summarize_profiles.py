@@ -18,7 +18,10 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 OUT = os.path.join(ROOT, "gpurun_out")
 PROF = os.path.join(ROOT, "profiles")
 STAGE_OF = {"k_tc_bwd2": "bwd_prefix", "k_tc_p": "fwd_prefix", "k_rows_bwd": "bwd_rows",
-            "k_rows_fwd": "fwd_rows", "k_group_bwd": "bwd_prefix", "k_group_fwd": "fwd_prefix"}
+            "k_rows_fwd": "fwd_rows", "k_group_bwd": "bwd_prefix", "k_group_fwd": "fwd_prefix",
+            "k_prefix_bwd": "bwd_prefix", "k_prefix_fwd": "fwd_prefix", "k_rows_fwd2": "fwd_rows",
+            "k_rows_bwd2": "bwd_rows", "k_agg_scatter": "agg", "k_pool": "pool",
+            "k_build_keys": "build_keys"}
 
 
 def short(name):
@@ -40,6 +43,8 @@ def launches(tag):
             continue
         if h and len(r) == len(h):
             n = short(r[h.index("Kernel Name")])
+            if n.startswith("at::"):      # bench.py's untimed L2 flush (torch fill), not our kernels
+                continue
             v = float(r[h.index("Metric Value")].replace(",", ""))
             if n not in agg:
                 agg[n] = [0.0, 0]
@@ -48,7 +53,8 @@ def launches(tag):
             agg[n][1] += 1
     tot = sum(v[0] for v in agg.values())
     lines = [f"# {tag}: ncu launch list (gpu__time_duration.sum, --clock-control none)", "",
-             "Cold-cache, serialised replay of one bench step (c4); compare shares, not absolutes.", "",
+             "Cold-cache, serialised replay of one bench step (c4); compare shares, not absolutes.",
+             "The bench's untimed L2-flush fill (at::FillFunctor) is excluded.", "",
              "| kernel | launches | us / launch | share |", "|---|---|---|---|"]
     for n in sorted(order, key=lambda k: -agg[k][0]):
         v, c = agg[n]
@@ -57,18 +63,42 @@ def launches(tag):
     open(os.path.join(PROF, f"{tag}_launches.md"), "w").write("\n".join(lines) + "\n")
 
 
+def ncu_rows():
+    """Rows of every prof_top*.ncu-rep (first launch of each kernel name wins)."""
+    h = units = None
+    out, seen = [], set()
+    for f in sorted(os.listdir(OUT)):
+        if not (f.startswith("prof_top") and f.endswith(".ncu-rep")):
+            continue
+        raw = subprocess.run(["ncu", "-i", os.path.join(OUT, f), "--page", "raw", "--csv"],
+                             capture_output=True, text=True).stdout
+        rows = list(csv.reader(io.StringIO(raw)))
+        if len(rows) < 3:
+            continue
+        hh = rows[0]
+        if h is None:
+            h, units = hh, rows[1]
+        for r in rows[2:]:
+            d = dict(zip(hh, r))
+            n = short(d["Kernel Name"])
+            if n in seen:
+                continue
+            seen.add(n)
+            out.append([d.get(k, "") for k in h])
+    return h, units, out
+
+
 def ncu_top(tag):
-    rep = os.path.join(OUT, "prof_top.ncu-rep")
-    if not os.path.exists(rep):
+    h, units, body = ncu_rows()
+    if h is None:
         return
-    raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
-    rows = list(csv.reader(io.StringIO(raw)))
-    h, units = rows[0], rows[1]
+    rows = [h, units] + body
     want = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
             "sm__throughput.avg.pct_of_peak_sustained_elapsed",
             "gpu__compute_memory_throughput.avg.pct_of_peak_sustained_elapsed",
             "dram__throughput.avg.pct_of_peak_sustained_elapsed",
             "sm__pipe_tensor_cycles_active_realtime.avg.pct_of_peak_sustained_elapsed",
+            "sm__inst_executed_pipe_tc.avg.pct_of_peak_sustained_active",
             "sm__inst_executed_pipe_fma.avg.pct_of_peak_sustained_active",
             "smsp__warps_active.avg.pct_of_peak_sustained_active",
             "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum.pct_of_peak_sustained_elapsed",

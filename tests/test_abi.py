@@ -106,3 +106,17 @@ def test_create_rejects_null_buffers():
     h = C.c_void_p()
     rc = L.load().ttemb_create(C.byref(cfg), 0, None, None, None, None, C.byref(h))
     assert rc == L.TTEMB_ERR_INVALID_ARG and not h.value
+
+
+def test_ablation_flags_accepted_and_size_the_workspace():
+    """TTEMB_NO_PREFIX_REUSE / TTEMB_NO_AGGREGATION are valid flags; they only grow
+    the workspace (U capacity = nnz, P capacity = U); unknown flag bits are rejected."""
+    base = tt.ttemb_query_sizes(_cfg()[0])
+    for kw in (dict(prefix_reuse=False), dict(aggregation=False), dict(prefix_reuse=False, aggregation=False)):
+        cfg, keep = _cfg(**kw)
+        core, state, grad, ws = tt.ttemb_query_sizes(cfg)
+        assert (core, state, grad) == base[:3] and ws >= base[3]
+    cfg, keep = _cfg()
+    cfg.flags = 1 << 7
+    v = [C.c_size_t() for _ in range(4)]
+    assert L.load().ttemb_query_sizes(C.byref(cfg), *[C.byref(x) for x in v]) == L.TTEMB_ERR_INVALID_ARG

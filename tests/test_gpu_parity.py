@@ -323,3 +323,45 @@ def test_edge_cases_empty_and_range_errors():
     fresh = gpu_emb(cfg, 8, 64)
     with pytest.raises(tt.TTEmbError):
         fresh.backward(torch.zeros(0, 2, 8, device=DEV))
+
+
+ABLATIONS = [dict(prefix_reuse=False), dict(aggregation=False), dict(prefix_reuse=False, aggregation=False)]
+
+
+@pytest.mark.parametrize("abl", ABLATIONS, ids=["no-reuse", "no-agg", "no-reuse-no-agg"])
+@pytest.mark.parametrize("case", ["dup-heavy", "tc-multitile", "c4-b1024", "c4-b1024-fp32"])
+def test_ablation_switches(case, abl):
+    """TTEMB_NO_PREFIX_REUSE / TTEMB_NO_AGGREGATION (the paper's Fig. 14/17/18 toggles)
+    change only the amount of work: outputs and core gradients still match the oracle, and the
+    plan counts become U = nnz (no dedup / aggregation) and P = U (no prefix reuse)."""
+    kw = {}
+    if case.startswith("c4"):
+        cfg, mode, B = W.config("c4"), None, 1024
+        kw["fp32_cores"] = case.endswith("fp32")
+    else:
+        cfg, mode = {c[0]: (c[1], c[2]) for c in small_cases()}[case]
+        B = None
+    idx, off, B = make_inputs(cfg, mode, seed=5, batch=B)
+    cores = W.make_cores(cfg, seed=5)
+    go = W.make_grad_out(cfg, B, seed=5)
+    emb = gpu_emb(cfg, B, len(idx), **kw, **abl)
+    emb.load_cores(cores)
+    out = run_forward(emb, idx, off, B)
+    emb.backward(torch.as_tensor(go, device=DEV))
+    assert emb.check() == 0
+    orc = Oracle.from_config(cfg)
+    ref_plan = orc.plan(idx, off, B)
+    cnt = emb.counts()
+    U = len(idx) if abl.get("aggregation") is False else ref_plan["U"]
+    assert cnt["U"] == U
+    if abl.get("prefix_reuse") is False:
+        assert cnt["P"] == U
+    elif abl.get("aggregation") is False:
+        assert cnt["P"] == ref_plan["P"]   # duplicates share their prefix run
+    assert_companion(out.cpu().numpy(), orc.forward(cores, idx, off, B),
+                     orc.forward(cores, idx, off, B, absolute=True), 1e-5, "forward")
+    g = orc.backward(cores, idx, off, B, go)
+    ga = orc.backward(cores, idx, off, B, go, absolute=True)
+    for t, mine in enumerate(emb.grad_views()):
+        for k in range(3):
+            assert_companion(mine[k].cpu().numpy(), g[t][k], ga[t][k], 1e-4, f"dC{k+1} t{t}")
