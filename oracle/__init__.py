@@ -58,6 +58,8 @@ def lib():
                                          C.POINTER(C.c_float), C.c_int64, C.POINTER(C.c_double)]
         _lib.ttref_row_literal.argtypes = _lib.ttref_row_chain.argtypes
         _lib.ttref_num_threads.restype = C.c_int
+        _lib.ttref_apply_bijection.argtypes = [C.POINTER(_Shape), C.c_void_p, i64p, i64p, C.c_int64,
+                                               C.c_int32, i64p]
     return _lib
 
 
@@ -116,6 +118,19 @@ class Oracle:
     def _ids(indices, offsets):
         return (np.ascontiguousarray(indices, dtype=np.int64),
                 np.ascontiguousarray(offsets, dtype=np.int64))
+
+    def apply_bijection(self, bijection, indices, offsets, batch: int) -> np.ndarray:
+        """New_Batch = { index_t(i_j) }; bijection: per table an int array [M_t]."""
+        idx, off = self._ids(indices, offsets)
+        maps = [np.ascontiguousarray(b, dtype=np.int64) for b in bijection]
+        assert len(maps) == self.T
+        ptrs = (C.c_void_p * self.T)(*[m.ctypes.data for m in maps])
+        out = np.zeros(max(len(idx), 1), np.int64)
+        rc = lib().ttref_apply_bijection(C.byref(self._shape), ptrs, _p(idx, C.c_int64),
+                                         _p(off, C.c_int64), len(idx), int(batch), _p(out, C.c_int64))
+        if rc:
+            raise OracleError(rc)
+        return out[:len(idx)]
 
     # -- plan --------------------------------------------------------------
     def plan(self, indices, offsets, batch: int) -> dict:

@@ -282,6 +282,29 @@ int ttref_plan(const ttref_shape* s, const int64_t* indices, const int64_t* offs
 /* ------------------------------------------------------------------------ */
 /* Forward (Eq. 2-4)                                                         */
 /* ------------------------------------------------------------------------ */
+/* the lookup uses New_Batch = { index(i_j) } instead of the raw ids. */
+int ttref_apply_bijection(const ttref_shape* s, const int64_t* const* bij, const int64_t* indices,
+                          const int64_t* offsets, int64_t nnz, int32_t B, int64_t* out_ids) {
+  if (check_shape(s) || B < 0 || nnz < 0) return -1;
+  const int T = s->T;
+  if (offsets[0] != 0 || offsets[(int64_t)T * B] != nnz) return -1;
+  for (int t = 0; t < T; ++t) {
+    const int64_t M = s->rows[t];
+    for (int32_t b = 0; b < B; ++b) {
+      const int64_t bag = (int64_t)t * B + b;
+      if (offsets[bag + 1] < offsets[bag]) return -1;
+      for (int64_t j = offsets[bag]; j < offsets[bag + 1]; ++j) {
+        const int64_t i = indices[j];
+        if (i < 0 || i >= M) return -3;
+        const int64_t k = bij[t][i];
+        if (k < 0 || k >= M) return -3;
+        out_ids[j] = k;
+      }
+    }
+  }
+  return 0;
+}
+
 int ttref_forward(const ttref_shape* s, const float* const* C1, const float* const* C2,
                   const float* const* C3, const int64_t* indices, const int64_t* offsets,
                   int64_t nnz, int32_t B, int literal, double* out) {

@@ -77,6 +77,13 @@ int ttref_backward(const ttref_shape* s, const float* const* C1, const float* co
 int ttref_update(int opt, double lr, double eps, int64_t n, float* param, float* state,
                  const double* grad);
 
+/* Runtime index bijection (Sec. IV-B): New_Batch = { index_t(i_j) }.
+ * bij[t] is table t's map [M_t] (new id of old id i); out_ids[j] = bij[t][indices[j]]
+ * for every position j of every bag of table t.  -3 if an id or a mapped id is
+ * outside [0, M_t), -1 for malformed offsets. */
+int ttref_apply_bijection(const ttref_shape* s, const int64_t* const* bij, const int64_t* indices,
+                          const int64_t* offsets, int64_t nnz, int32_t B, int64_t* out_ids);
+
 /* Threads the oracle's OpenMP loops use (1 if built without OpenMP). */
 int ttref_num_threads(void);
 

@@ -330,3 +330,40 @@ def test_update_matches_torch_optim(opt):
     p1, _ = Oracle.update(opt, lr, p0, g1, None, eps)
     np.testing.assert_array_equal(p1, pt2.detach().numpy().astype(np.float32))
     assert np.array_equal(p1[::10], p0[::10])      # zero gradient leaves the slice unchanged
+
+
+# ---------------------------------------------------------------------------
+# Runtime index bijection (Sec. IV-B)
+# ---------------------------------------------------------------------------
+def test_bijection_is_a_row_permutation_of_the_dense_table():
+    """New_Batch = {index(i_j)}: looking up i through the bijection reads row index(i) of
+    the TT table, i.e. the bag sums of the dense table with rows permuted, W'[i] = W[index(i)]
+    (numpy fancy indexing + torch embedding_bag; an inverse-map or per-table mix-up fails)."""
+    cfg = W.small_config([37, 100, 5], [(3, 4, 4), (5, 4, 5), (1, 2, 3)], (2, 3, 2), 5, 9, 2, 1.05)
+    rng = np.random.default_rng(7)
+    T, B = cfg.num_tables, cfg.batch
+    idx, off = W.make_batch(cfg, step=2, seed=7)
+    cores = W.make_cores(cfg, seed=7)
+    bij = [rng.permutation(M) for M in cfg.table_rows]
+    orc = Oracle.from_config(cfg)
+    out = orc.forward(cores, orc.apply_bijection(bij, idx, off, B), off, B)
+    for t in range(T):
+        Wt = materialise_torch([torch.as_tensor(x, dtype=torch.float64) for x in cores[t]],
+                               cfg.row_factors[t], cfg.col_factors, cfg.table_rows[t])
+        Wp = Wt[torch.as_tensor(bij[t])]
+        o = off[t * B:(t + 1) * B + 1]
+        ref = torch.nn.functional.embedding_bag(torch.as_tensor(idx[o[0]:o[-1]]), Wp,
+                                                torch.as_tensor(o[:-1] - o[0]), mode="sum")
+        np.testing.assert_allclose(out[:, t, :], ref.numpy(), rtol=1e-12, atol=1e-13)
+
+
+def test_bijection_range_errors():
+    orc = Oracle([10], [(2, 2, 3)], (1, 1, 2), 2)
+    with pytest.raises(OracleError) as e:          # mapped id outside [0, M)
+        orc.apply_bijection([np.array([0, 1, 2, 3, 4, 5, 6, 7, 8, 10])], np.array([9]), np.array([0, 1]), 1)
+    assert e.value.code == ERR_INDEX_RANGE
+    with pytest.raises(OracleError) as e:          # raw id outside [0, M)
+        orc.apply_bijection([np.arange(10)], np.array([10]), np.array([0, 1]), 1)
+    assert e.value.code == ERR_INDEX_RANGE
+    np.testing.assert_array_equal(orc.apply_bijection([np.arange(10)[::-1]], np.array([0, 9, 3]),
+                                                      np.array([0, 3]), 1), [9, 0, 6])
