@@ -283,6 +283,8 @@ def workload_config(cfg, B, world, args):
             "update": ("fused" if world == 1 and not getattr(args, "unfused", False)
                        else "allreduce+update" if world > 1 else "unfused"),
             "parallelism": f"dp{world}", "l2": "flushed between timed steps (untimed 512 MiB write)",
+            **({"bijection": f"frequency order (Alg. 2 l.1-4), {args.bijection} history batches"}
+               if getattr(args, "bijection", 0) else {}),
             **({"ablation": [k for k in ("no_reuse", "no_agg", "unfused") if getattr(args, k, False)]}
                if any(getattr(args, k, False) for k in ("no_reuse", "no_agg", "unfused")) else {})}
 
@@ -334,6 +336,9 @@ def main():
                     help="ablation: no row dedup / in-advance gradient aggregation (TTEMB_NO_AGGREGATION, P:416)")
     ap.add_argument("--unfused", action="store_true",
                     help="ablation: backward writes dense core grads, separate update (P:421)")
+    ap.add_argument("--bijection", type=int, default=0, metavar="K",
+                    help="f2: frequency-ordering index bijection (Alg. 2 l.1-4) built offline from K "
+                         "history batches of the stream, applied at run time (P:269)")
     ap.add_argument("--no-graph", dest="graph", action="store_false",
                     help="launch every step eagerly instead of replaying a captured CUDA graph")
     args = ap.parse_args()
@@ -387,6 +392,13 @@ def main():
                             aggregation=not args.no_agg)
     cores = W.make_cores(cfg, seed=args.seed)
     emb.load_cores(cores)
+    bij_t = None
+    if args.bijection:
+        from paper_conf_sc_wangwfmmd22_b200 import reorder
+        hist = (W.make_batch(cfg, step=10_000 + k, seed=args.seed + 1000 * rank, batch=B) + (B,)
+                for k in range(args.bijection))
+        bij_t = torch.as_tensor(reorder.frequency_bijection(cfg.table_rows, hist).view(np.int32), device=dev)
+        emb.set_bijection(bij_t)
     dpool = [(torch.as_tensor(i, device=dev), torch.as_tensor(o, device=dev), torch.as_tensor(g, device=dev))
              for i, o, g in pool]
     out = torch.empty(B, cfg.num_tables, cfg.dim, device=dev)

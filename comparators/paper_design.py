@@ -19,7 +19,7 @@ calls, the way P:346 describes its implementation ("cuBLAS batched GEMM"):
     index_add (Fig. 6(a) step 2), and the SGD update of the touched slices.
 
 fp32 throughout (TF32 disabled), so it is checked against the oracle at the same
-tolerances as the CUDA path (tests/test_gpu_parity.py::test_paper_design_comparator).
+tolerances as the CUDA path (tests/test_paper_comparator.py).
 Everything is torch / cuBLAS: it exists to put a number for "the paper's design on
 this GPU" next to ours, and is imported only by bench.py (--impl paper) and tests.
 """
@@ -56,6 +56,7 @@ class PaperDesignTT:
         n1, n2, n3, R, N, T = self.n1, self.n2, self.n3, self.R, self.N, self.T
         out = torch.zeros(batch, T, N, dtype=torch.float32, device=self.device)
         saved = []
+        offsets = offsets.cpu()            # bag boundaries on the host (slicing); no-op if already there
         for t in range(T):
             m1, m2, m3 = self.row_factors[t]
             lo, hi = int(offsets[t * batch]), int(offsets[(t + 1) * batch])
@@ -63,7 +64,7 @@ class PaperDesignTT:
                 saved.append(None)
                 continue
             idx = indices[lo:hi]
-            lens = offsets[t * batch + 1:(t + 1) * batch + 1] - offsets[t * batch:(t + 1) * batch]
+            lens = (offsets[t * batch + 1:(t + 1) * batch + 1] - offsets[t * batch:(t + 1) * batch]).to(self.device)
             bag = torch.repeat_interleave(torch.arange(batch, device=self.device), lens)
             urow, inv = torch.unique(idx, return_inverse=True)            # unique indices
             pfx = torch.div(urow, m3, rounding_mode="floor")              # Buf_idx = idx / length_3

@@ -169,6 +169,20 @@ typedef struct {
 
 int ttemb_get_plan(ttemb_t h, ttemb_plan* plan);
 
+/* Runtime index bijection (Sec. IV-B: "all indices will first be transformed into
+ * new indices based on the index bijection function ... New_Batch = {index(i_j)}").
+ * `bijection` is a DEVICE array of uint32 with one entry per row of every table,
+ * concatenated in table order (table t occupies [rowbase_t, rowbase_t + M_t), rowbase_t =
+ * M_0 + ... + M_{t-1}; ttemb_total_rows gives the length): every later forward looks up
+ * row bijection[rowbase_t + i] of table t for id i.  The caller owns the buffer and keeps
+ * it alive and unchanged while forwards run; NULL switches the mapping off.  The map must
+ * send [0, M_t) into [0, M_t) (a bijection for the method's purpose); a mapped id >= M_t
+ * raises TTEMB_ERR_INDEX_RANGE through ttemb_check like a raw out-of-range id.  Applied
+ * inside the key-build kernel (no extra pass).  Generate one offline, e.g. with the
+ * frequency ordering of Alg. 2 lines 1-4 (paper_conf_sc_wangwfmmd22_b200/reorder.py). */
+int ttemb_set_bijection(ttemb_t h, const uint32_t* bijection);
+uint64_t ttemb_total_rows(ttemb_t h);   /* sum of M_t (length of a bijection buffer); 0 for NULL */
+
 /* Synchronous helper: copy {U, P, NG, error flags} of the last forward to host. */
 int ttemb_read_counts(ttemb_t h, int64_t counts[4], void* stream);
 

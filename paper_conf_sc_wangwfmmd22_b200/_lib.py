@@ -29,7 +29,8 @@ TTEMB_NO_AGGREGATION = 8
 SYMBOLS = ["ttemb_query_sizes", "ttemb_create", "ttemb_destroy", "ttemb_core_layout",
            "ttemb_forward", "ttemb_backward", "ttemb_update", "ttemb_forward_host",
            "ttemb_backward_host", "ttemb_check", "ttemb_get_plan", "ttemb_read_counts",
-           "ttemb_set_timing", "ttemb_stage_times", "ttemb_stage_name", "ttemb_status_string"]
+           "ttemb_set_timing", "ttemb_stage_times", "ttemb_stage_name", "ttemb_status_string",
+           "ttemb_set_bijection", "ttemb_total_rows"]
 
 
 class ttemb_table(C.Structure):
@@ -93,10 +94,13 @@ def load(path: str = LIB_PATH):
     lib.ttemb_stage_name.restype = C.c_char_p
     lib.ttemb_status_string.argtypes = [C.c_int]
     lib.ttemb_status_string.restype = C.c_char_p
+    lib.ttemb_set_bijection.argtypes = [vp, vp]
+    lib.ttemb_total_rows.argtypes = [vp]
     for s in SYMBOLS:
         f = getattr(lib, s)
-        if s not in ("ttemb_stage_name", "ttemb_status_string"):
+        if s not in ("ttemb_stage_name", "ttemb_status_string", "ttemb_total_rows"):
             f.restype = C.c_int
+    lib.ttemb_total_rows.restype = C.c_uint64
     _lib = lib
     return lib
 

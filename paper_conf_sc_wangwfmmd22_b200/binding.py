@@ -137,6 +137,14 @@ def ttemb_stage_name(i: int) -> str:
     return L.load().ttemb_stage_name(int(i)).decode()
 
 
+def ttemb_set_bijection(h: int, bijection: int) -> None:
+    check(L.load().ttemb_set_bijection(h, bijection or None), "ttemb_set_bijection")
+
+
+def ttemb_total_rows(h: int) -> int:
+    return int(L.load().ttemb_total_rows(h))
+
+
 def ttemb_status_string(code: int) -> str:
     return L.status_string(code)
 
@@ -269,6 +277,19 @@ class TTEmbeddingBag:
 
     def check(self, stream=None) -> int:
         return ttemb_check(self.h, _stream_ptr(stream))
+
+    def set_bijection(self, bijection: Optional[torch.Tensor]) -> None:
+        """Runtime index bijection: a device tensor of sum(M_t) uint32 / int32 entries
+        (table t's map at offset M_0 + ... + M_{t-1}), or None to switch it off.  The tensor is
+        kept alive by this object."""
+        if bijection is None:
+            ttemb_set_bijection(self.h, 0)
+            self._bij = None
+            return
+        assert bijection.is_cuda and bijection.dtype in (torch.int32, torch.uint32)
+        assert bijection.is_contiguous() and bijection.numel() == ttemb_total_rows(self.h)
+        self._bij = bijection
+        ttemb_set_bijection(self.h, bijection.data_ptr())
 
     def counts(self, stream=None) -> Dict[str, int]:
         U, P, NG, err = ttemb_read_counts(self.h, _stream_ptr(stream))

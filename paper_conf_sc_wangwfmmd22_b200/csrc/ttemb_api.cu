@@ -407,6 +407,14 @@ int ttemb_backward_host(ttemb_t h, const float* host_grad_out, float lr, void* s
   return ttemb_backward(h, c.st_grad, lr, stream);
 }
 
+int ttemb_set_bijection(ttemb_t h, const uint32_t* bijection) {
+  if (!h) return TTEMB_ERR_INVALID_ARG;
+  h->c.bij = bijection;
+  return TTEMB_OK;
+}
+
+uint64_t ttemb_total_rows(ttemb_t h) { return h ? h->c.total_rows : 0; }
+
 int ttemb_check(ttemb_t h, void* stream) {
   if (!h) return TTEMB_ERR_INVALID_ARG;
   Ctx& c = h->c;

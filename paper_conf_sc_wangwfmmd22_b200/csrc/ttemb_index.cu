@@ -144,7 +144,7 @@ __global__ void __launch_bounds__(256)
 k_build_keys(const IdxT* __restrict__ indices, const int64_t* __restrict__ offsets, int64_t nnz,
              int32_t B, int T, const TableMeta* __restrict__ meta, uint32_t* __restrict__ keys,
              uint32_t* __restrict__ bag_of, uint32_t* __restrict__ counts, int passes,
-             uint32_t* __restrict__ hist) {
+             uint32_t* __restrict__ hist, const uint32_t* __restrict__ bij) {
   __shared__ uint32_t sh[4][256];
   for (int i = threadIdx.x; i < 4 * 256; i += blockDim.x) (&sh[0][0])[i] = 0;
   __syncthreads();
@@ -162,13 +162,19 @@ k_build_keys(const IdxT* __restrict__ indices, const int64_t* __restrict__ offse
     const TableMeta& mt = meta[t];
     const uint32_t kb = (uint32_t)mt.kbase, M = mt.M, m1 = mt.m1, m2 = mt.m2, m3 = mt.m3;
     const uint32_t bo = (uint32_t)(bb * T + t);
+    const uint32_t* bt = bij ? bij + mt.rowbase : nullptr;   // table t's bijection
     for (int64_t j = s; j < e; ++j) {
       const int64_t id = (int64_t)indices[j];
       uint32_t key = kb;
       if (id < 0 || (uint64_t)id >= M) err |= kErrRange;
       else {
-        const uint32_t r = (uint32_t)id, p = r / m3, i3 = r - p * m3, i1 = p / m2, i2 = p - i1 * m2;
-        key = kb + (i2 * m1 + i1) * m3 + i3;
+        const uint32_t r = bt ? __ldg(bt + id) : (uint32_t)id;   // New_Batch = {index(i_j)}
+        if (r >= M) {
+          err |= kErrRange;
+        } else {
+          const uint32_t p = r / m3, i3 = r - p * m3, i1 = p / m2, i2 = p - i1 * m2;
+          key = kb + (i2 * m1 + i1) * m3 + i3;
+        }
       }
       keys[j] = key;
       bag_of[j] = bo;
@@ -491,11 +497,11 @@ cudaError_t run_index_stage(Ctx& c, const void* indices, const int64_t* offsets,
     if (c.index_bits == 64)
       k_build_keys<int64_t><<<g, 256, 0, s>>>((const int64_t*)indices, offsets, nnz, c.B, c.T,
                                               c.d_meta, p.keysA, p.bag_of, p.counts,
-                                              c.key_passes, p.hist1);
+                                              c.key_passes, p.hist1, c.bij);
     else
       k_build_keys<int32_t><<<g, 256, 0, s>>>((const int32_t*)indices, offsets, nnz, c.B, c.T,
                                               c.d_meta, p.keysA, p.bag_of, p.counts,
-                                              c.key_passes, p.hist1);
+                                              c.key_passes, p.hist1, c.bij);
   }
   // a2: sort (key, position)
   const int64_t tiles1 = radix_tiles(nnz);

@@ -86,6 +86,7 @@ struct Ctx {
   float* state = nullptr;
   float* grads = nullptr;
   uint8_t* ws = nullptr;
+  const uint32_t* bij = nullptr;     // runtime index bijection [sum M_t], or null
 
   // workspace carve
   TableMeta* d_meta = nullptr;

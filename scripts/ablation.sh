@@ -8,6 +8,7 @@ for cfgn in ${ABL_CONFIGS:-c4 c3}; do
   timeout 300 $B --config $cfgn --no-agg > gpurun_out/abl/$cfgn-no_agg.json 2> gpurun_out/abl/$cfgn-no_agg.err
   timeout 300 $B --config $cfgn --unfused > gpurun_out/abl/$cfgn-unfused.json 2> gpurun_out/abl/$cfgn-unfused.err
   timeout 300 $B --config $cfgn --ids perm > gpurun_out/abl/$cfgn-perm.json 2> gpurun_out/abl/$cfgn-perm.err
+  timeout 300 $B --config $cfgn --ids perm --bijection 16 > gpurun_out/abl/$cfgn-perm_bij.json 2> gpurun_out/abl/$cfgn-perm_bij.err
   timeout 600 python bench.py --impl paper --config $cfgn --steps 5 --warmup 3 > gpurun_out/abl/$cfgn-paper.json 2> gpurun_out/abl/$cfgn-paper.err
 done
 for f in gpurun_out/abl/*.json; do echo "$f $(python -c "import json,sys; d=json.load(open('$f')); print(round(d['ms_per_step'],3), 'ms', round(d['value']/1e6,1), 'M/s')" 2>&1 | tail -1)"; done

@@ -17,7 +17,7 @@ HEADER = os.path.join(ROOT, "include", "ttemb.h")
 
 def declared_symbols():
     src = open(HEADER).read()
-    return sorted(set(re.findall(r"^\s*(?:int|const char\*)\s+(ttemb_\w+)\s*\(", src, re.M)))
+    return sorted(set(re.findall(r"^\s*(?:int|uint64_t|const char\*)\s+(ttemb_\w+)\s*\(", src, re.M)))
 
 
 def test_header_symbols_exported():

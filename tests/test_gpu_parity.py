@@ -365,3 +365,54 @@ def test_ablation_switches(case, abl):
     for t, mine in enumerate(emb.grad_views()):
         for k in range(3):
             assert_companion(mine[k].cpu().numpy(), g[t][k], ga[t][k], 1e-4, f"dC{k+1} t{t}")
+
+
+@pytest.mark.parametrize("case", ["multi-var-L", "tc-multitile", "c4-b1024"])
+def test_runtime_bijection(case):
+    """ttemb_set_bijection: the CUDA path looks up New_Batch = {index(i_j)}; outputs and
+    gradients match the oracle applied to the mapped ids; the plan is the plan of the mapped ids."""
+    from paper_conf_sc_wangwfmmd22_b200 import reorder
+    if case.startswith("c4"):
+        cfg, mode, B = W.config("c4").replace(id_map="perm"), None, 1024
+    else:
+        cfg, mode = {c[0]: (c[1], c[2]) for c in small_cases()}[case]
+        B = None
+    idx, off, B = make_inputs(cfg, mode, seed=9, batch=B)
+    hist = [W.make_batch(cfg, step=s, seed=9, batch=B) + (B,) for s in range(1, 4)]
+    bij = reorder.frequency_bijection(cfg.table_rows, hist)
+    maps = reorder.split_bijection(bij, cfg.table_rows)
+    cores = W.make_cores(cfg, seed=9)
+    go = W.make_grad_out(cfg, B, seed=9)
+    emb = gpu_emb(cfg, B, len(idx))
+    emb.load_cores(cores)
+    emb.set_bijection(torch.as_tensor(bij.view(np.int32), device=DEV))
+    out = run_forward(emb, idx, off, B)
+    emb.backward(torch.as_tensor(go, device=DEV))
+    assert emb.check() == 0
+    orc = Oracle.from_config(cfg)
+    mid = orc.apply_bijection(maps, idx, off, B)
+    check_plan(emb, orc, mid, off, B)
+    assert_companion(out.cpu().numpy(), orc.forward(cores, mid, off, B),
+                     orc.forward(cores, mid, off, B, absolute=True), 1e-5, "forward")
+    g = orc.backward(cores, mid, off, B, go)
+    ga = orc.backward(cores, mid, off, B, go, absolute=True)
+    for t, mine in enumerate(emb.grad_views()):
+        for k in range(3):
+            assert_companion(mine[k].cpu().numpy(), g[t][k], ga[t][k], 1e-4, f"dC{k+1} t{t}")
+    # switching it off restores the raw-id lookup
+    emb.set_bijection(None)
+    out2 = run_forward(emb, idx, off, B)
+    emb.backward(torch.as_tensor(go, device=DEV))
+    assert emb.check() == 0
+    check_plan(emb, orc, idx, off, B)
+
+
+def test_bijection_out_of_range_is_reported():
+    cfg = W.config("c1")
+    idx, off = W.make_batch(cfg, seed=1)
+    emb = gpu_emb(cfg, cfg.batch, len(idx))
+    bad = np.arange(cfg.table_rows[0], dtype=np.int32)
+    bad[int(idx[0])] = cfg.table_rows[0]            # maps a used id outside [0, M)
+    emb.set_bijection(torch.as_tensor(bad, device=DEV))
+    run_forward(emb, idx, off, cfg.batch)
+    assert emb.check() == L.TTEMB_ERR_INDEX_RANGE
