@@ -58,6 +58,7 @@ struct YArgs {
   int n1, n1s, NC, nblk, tpp, nchunk;
   float lr, eps;
   int opt, fused;
+  int exp;                                // TTEMB_EXP bits (timing experiments only; results invalid)
 };
 
 struct YCtl {
@@ -190,6 +191,7 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
         const int c4 = 4 * ((tid >> 6) + 4 * k);
         const uint32_t oa = (uint32_t)((c4 >> 2) * Y_A2LBO + (mb >> 3) * 128 + (mb & 7) * 16);
         const uint32_t ol = (uint32_t)((c4 >> 2) * Y_A2LBO + ((64 + mb) >> 3) * 128 + (mb & 7) * 16);
+        if (a.exp & 4) continue;
         const float4 p = *reinterpret_cast<const float4*>(a2 + oa);
         *reinterpret_cast<float4*>(a2 + ol) = make_float4(lo32(p.x), lo32(p.y), lo32(p.z), lo32(p.w));
         const uint32_t ob = tc::cm_off(mb, c4, 8);
@@ -199,7 +201,7 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
       tc::named_sync(1, Y_LW * 32);                     // whole chunk (hi and lo) visible
       {   // dP^T of this chunk -> TMEM: chunk ck covers c-block ck / 2, lane quarters 2 (ck & 1) + {0, 1}
         const int blk = P.ck >> 1, Q = w & 3;
-        if ((Q >> 1) == (P.ck & 1) && blk < a.nblk) {
+        if ((Q >> 1) == (P.ck & 1) && blk < a.nblk && !(a.exp & 8)) {
           const int cc = 32 * (Q & 1) + lane;             // column inside the chunk
           const int m0 = 32 * (w >> 2);                    // warps 0-3: rows 0..31, 4-7: 32..63
           float xh[32], xl[32];
@@ -328,7 +330,7 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
 #pragma unroll
             for (int i = 0; i < 32; ++i) v[i] += x[i];
           }
-          if (dst) {
+          if (dst && !(a.exp & 2)) {
 #pragma unroll
             for (int i = 0; i < 32; i += 4)
               asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(dst + 32 * h + i), "f"(v[i]),
@@ -349,7 +351,7 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
           for (int h = 0; h < 2; ++h) {
             float v[32];
             tc::tmem_ld32(tc::taddr(tm + 256 + blk * 64 + 32 * h, 32 * Q, 0), v);
-            if (c < NC) {
+            if (c < NC && !(a.exp & 1)) {
               const size_t base = so + (size_t)(32 * h) * NC + c;
               if (!a.fused) {
 #pragma unroll
@@ -411,6 +413,7 @@ cudaError_t run_prefix_bwd(Ctx& c, float lr, cudaStream_t s) {
   a.n1 = c.n1; a.n1s = c.n1 == 1 ? 0 : c.n1 == 2 ? 1 : c.n1 == 4 ? 2 : 3;
   a.NC = c.NC; a.nblk = (c.NC + 127) / 128; a.tpp = YT / c.n1; a.nchunk = (c.NC + 63) / 64;
   a.lr = lr; a.eps = c.eps; a.opt = c.opt; a.fused = (c.flags & TTEMB_FUSED_UPDATE) ? 1 : 0;
+  a.exp = exp_bits();
   StageScope sc(c, ST_BWD_PREFIX, s);
   const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(c.NG_cap, (int64_t)c.sm_count));
   k_prefix_bwd<<<grid, Y_THREADS, kBwdSmem, s>>>(a);

@@ -11,6 +11,7 @@
 
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 #include <vector>
 
@@ -32,6 +33,17 @@ enum Stage : int {
   ST_AGG_FIX, ST_BWD_ROWS, ST_BWD_PREFIX, ST_DC1, ST_UPD_C3, ST_UPDATE, ST_H2D, ST_D2H,
   ST_COUNT
 };
+
+// TTEMB_EXP environment bits: switch parts of a kernel off for timing experiments (results
+// are invalid; never set in tests / bench runs that report numbers).
+inline int exp_bits() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("TTEMB_EXP");
+    v = e ? atoi(e) : 0;
+  }
+  return v;
+}
 
 struct TableMeta {
   uint32_t m1, m2, m3, M;      // row factors, rows (M <= 2^32-1 checked on host)
