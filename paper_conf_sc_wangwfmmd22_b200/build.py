@@ -33,7 +33,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
         return LIB
     cmd = [NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2", "-shared",
            "--expt-relaxed-constexpr", "-I", os.path.join(ROOT, "include"),
-           "-o", LIB + ".tmp", *sources()]
+           *os.environ.get("TTEMB_NVCC_FLAGS", "").split(), "-o", LIB + ".tmp", *sources()]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
     subprocess.check_call(cmd, cwd=PKG)

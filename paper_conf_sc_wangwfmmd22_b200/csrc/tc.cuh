@@ -84,6 +84,12 @@ __device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t
                : "memory");
 }
 
+// 1-D bulk prefetch of [src, src + bytes) into L2 (TMA engine, no shared memory, no completion).
+// src and bytes must be multiples of 16.
+__device__ __forceinline__ void bulk_prefetch_l2(const void* src, uint32_t bytes) {
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(src), "r"(bytes) : "memory");
+}
+
 // Instruction descriptor: kind::tf32, fp32 accumulate.
 __device__ __forceinline__ uint32_t idesc_tf32(int M, int N, bool a_mn_major, bool b_mn_major) {
   uint32_t d = 0;

@@ -24,6 +24,7 @@
 #include <stdlib.h>
 
 #include <algorithm>
+#include <vector>
 
 #include "tc.cuh"
 #include "ttemb_internal.cuh"
@@ -40,7 +41,9 @@ constexpr uint32_t Y_B1 = 2u * YR * YT * 4;     // C1^T hi + lo (CM(r1, m)), 32 
 constexpr uint32_t Y_A2LBO = 16 * 128 + 16;    // CM(128 rows, 64 c); +16 B per core column keeps
                                                 // the column-wise dP^T extraction conflict-free
 constexpr uint32_t Y_A2 = 16 * Y_A2LBO;         // [dP_hi; dP_lo] chunk (~32 KB)
-constexpr uint32_t Y_B2 = 2u * YR * 64 * 4;     // C2 chunk hi + lo, CM(r1, 64 c), 32 KB
+constexpr uint32_t Y_B2LBO = 8 * 128 + 16;     // CM(64 r1, 64 c) core-column stride (+16 B: the
+                                                // row-contiguous staging map is conflict-free)
+constexpr uint32_t Y_B2 = 2u * 16 * Y_B2LBO;    // C2 chunk hi + lo (~32.5 KB)
 constexpr uint32_t Y_STAGE = Y_A2 + Y_B2;
 constexpr int Y_NST = 3;                        // chunk stages (cp.async, two in flight)
 constexpr size_t kBwdSmem = 128 + Y_B1 + Y_NST * Y_STAGE;
@@ -58,6 +61,8 @@ struct YArgs {
   int n1, n1s, NC, nblk, tpp, nchunk;
   float lr, eps;
   int opt, fused;
+  unsigned long long* trace;              // TTEMB_TRACE: 32 cycle counters per CTA (timing only)
+  int pf;                                 // L2 prefetch distance in groups (0 = off)
   int exp;                                // TTEMB_EXP bits (timing experiments only; results invalid)
 };
 
@@ -98,6 +103,16 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
   __syncthreads();
   tc::fence_after();
   const uint32_t tm = ctl.tmem;
+#ifdef TTEMB_TRACE_BUILD   // role timers (build with TTEMB_NVCC_FLAGS=-DTTEMB_TRACE_BUILD, run with TTEMB_TRACE=1)
+  unsigned long long trc[32] = {};
+  long long _tt = 0;
+  const long long t_start = a.trace ? clock64() : 0;
+#define YT0() do { if (a.trace) _tt = clock64(); } while (0)
+#define YTA(k) do { if (a.trace) { const long long _n = clock64(); trc[k] += (unsigned long long)(_n - _tt); _tt = _n; } } while (0)
+#else
+#define YT0() do { } while (0)
+#define YTA(k) do { } while (0)
+#endif
   // TMEM columns: [0,128) dP^T hi (64 per c-block), [128,256) lo, [256,384) dC2^T (64 per
   // c-block), [384,448) dA pass B = C2_hi, [448,512) dA pass B = C2_lo.
   const int tpp = a.tpp, NC = a.NC;
@@ -109,11 +124,11 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
     // straight into its MMA layout (dP rows -> A2 rows 0..63, C2 rows -> B2 hi); each thread
     // then writes the lo parts of the 16-byte pieces it copied, and the warps owning the
     // chunk's TMEM lane quarters extract dP^T (hi, lo) from A2 into TMEM for the dC2 GEMM.
-    struct Job { uint32_t g, q1, qa; int ck; };
+    struct Job { uint32_t g, q0, q1, qa; int ck; unsigned long long c2; };
     const uint32_t G0 = blockIdx.x, GS = gridDim.x;
-    auto start = [&](Job& j, uint32_t g) {
+    auto start = [&](Job& j, uint32_t g) {   // group metadata loaded once (three independent loads)
       j.g = g; j.ck = 0;
-      if (g < NG) { j.qa = a.grp_off[g]; j.q1 = a.grp_off[g + 1]; }
+      if (g < NG) { j.q0 = j.qa = a.grp_off[g]; j.q1 = a.grp_off[g + 1]; j.c2 = a.grp_c2[g]; }
     };
     auto advance = [&](Job& j) {
       if (++j.ck < a.nchunk) return;
@@ -121,24 +136,40 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
       j.qa += tpp;
       if (j.qa >= j.q1) start(j, j.g + GS);
     };
-    const int mb = tid & 63;                  // copy map: row mb, float4 columns (tid >> 6) + 4 k
+    const int mb = tid & 63;                  // C1^T staging map: row mb, float4 columns (tid >> 6) + 4 k
+    // chunk copy map: rows (tid >> 4) + 16 k, float4 column 4 (tid & 15): every half-warp reads one
+    // 256-byte row segment (coalesced); the padded core-column strides keep the stores conflict-free
+    const int cr = tid >> 4, cc4 = 4 * (tid & 15);
+    auto a2_off = [&](int r) { return (uint32_t)((cc4 >> 2) * Y_A2LBO + (r >> 3) * 128 + (r & 7) * 16); };
+    auto b2_off = [&](int r) { return (uint32_t)((cc4 >> 2) * Y_B2LBO + (r >> 3) * 128 + (r & 7) * 16); };
     auto issue = [&](const Job& j, uint32_t sidx) {
       const uint32_t rows = min((uint32_t)tpp, j.q1 - j.qa) << a.n1s;
-      const float* dps = a.dpbuf + (size_t)j.qa * a.n1 * NC + j.ck * 64;
-      const float* c2 = a.cores + a.grp_c2[j.g] + j.ck * 64;
+      const float* dps = a.dpbuf + (size_t)j.qa * a.n1 * NC + j.ck * 64 + cc4;
+      const float* c2 = a.cores + j.c2 + j.ck * 64 + cc4;
       const uint32_t a2 = tc::smem_u32(stg + (sidx % Y_NST) * Y_STAGE), b2 = a2 + Y_A2;
 #pragma unroll
       for (int k = 0; k < 4; ++k) {
-        const int c4 = 4 * ((tid >> 6) + 4 * k);
-        const uint32_t oa = (uint32_t)((c4 >> 2) * Y_A2LBO + (mb >> 3) * 128 + (mb & 7) * 16);
-        tc::cp_async16_z(a2 + oa, dps + (size_t)(mb < (int)rows ? mb : 0) * NC + c4, mb < (int)rows);
-        tc::cp_async16(b2 + tc::cm_off(mb, c4, 8), c2 + (size_t)mb * NC + c4);
+        const int r = cr + 16 * k;
+        tc::cp_async16_z(a2 + a2_off(r), dps + (size_t)(r < (int)rows ? r : 0) * NC, r < (int)rows);
+        tc::cp_async16(b2 + b2_off(r), c2 + (size_t)r * NC);
       }
     };
     uint32_t ui = 0, si = 0, sp = 0;          // tile counter, issued / processed chunk counters
     Job P, I;
     start(P, G0);
     I = P;
+    // C1 rows of a tile (row mb of the tile, float4 columns (tid >> 6) + 4 k), loaded one tile
+    // ahead (NT = the next tile of the processing job) so their latency overlaps a whole tile.
+    float4 cvn[4];
+    auto load_c1 = [&](const Job& j, float4* cv) {
+      const uint32_t np = j.g < NG ? min((uint32_t)tpp, j.q1 - j.qa) : 0u;
+      const bool ok = mb < (int)(np << a.n1s) && !(a.exp & 16);
+      const uint32_t arow = ok ? a.grp_arow[j.qa + (mb >> a.n1s)] + (mb & ((1 << a.n1s) - 1)) : 0u;
+      const float4* src = reinterpret_cast<const float4*>(a.cores + (size_t)arow * YR);
+#pragma unroll
+      for (int k = 0; k < 4; ++k) cv[k] = ok ? __ldg(src + (tid >> 6) + 4 * k) : make_float4(0.f, 0.f, 0.f, 0.f);
+    };
+    load_c1(P, cvn);
     for (int d = 0; d < Y_NST - 1; ++d) {
       if (I.g < NG) {
         tc::mbar_wait(&ctl.s_free[si % Y_NST], ((si / Y_NST) & 1) ^ 1);
@@ -149,11 +180,10 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
       tc::cp_commit();
     }
     while (P.g < NG) {
+      YT0();
       const uint32_t np = min((uint32_t)tpp, P.q1 - P.qa);
-      const int rows = (int)np << a.n1s;
       if (P.ck == 0) {
-        const uint32_t q0 = a.grp_off[P.g];
-        const uint32_t fl = (P.qa == q0 ? 1u : 0u) | (P.qa + tpp >= P.q1 ? 2u : 0u);
+        const uint32_t fl = (P.qa == P.q0 ? 1u : 0u) | (P.qa + tpp >= P.q1 ? 2u : 0u);
         if (tid == 0) {
           tc::mbar_wait(&ctl.u_empty[ui & 3], ((ui >> 2) & 1) ^ 1);
           ctl.ring[ui & 3][0] = P.g; ctl.ring[ui & 3][1] = P.qa; ctl.ring[ui & 3][2] = np; ctl.ring[ui & 3][3] = fl;
@@ -161,12 +191,17 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
         }
         // C1^T -> B1 = CM(r1, m) hi | lo (element (r1, m) = C1 row m, column r1); zero past the tile
         float4 cv[4];
-        const bool ok = mb < rows;
-        const uint32_t arow = ok ? a.grp_arow[P.qa + (mb >> a.n1s)] + (mb & ((1 << a.n1s) - 1)) : 0u;
-        const float4* src = reinterpret_cast<const float4*>(a.cores + (size_t)arow * YR);
 #pragma unroll
-        for (int k = 0; k < 4; ++k) cv[k] = ok ? __ldg(src + (tid >> 6) + 4 * k) : make_float4(0.f, 0.f, 0.f, 0.f);
+        for (int k = 0; k < 4; ++k) cv[k] = cvn[k];
+        {   // prefetch the next tile's C1 rows
+          Job NT = P;
+          NT.qa += tpp;
+          if (NT.qa >= NT.q1) start(NT, NT.g + GS);
+          load_c1(NT, cvn);
+        }
+        YTA(0);
         tc::mbar_wait(&ctl.a1_free, (ui & 1) ^ 1);      // previous tile's dC2 GEMM done
+        YTA(1);
         tc::fence_after();
 #pragma unroll
         for (int k = 0; k < 4; ++k) {
@@ -181,24 +216,33 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
         }
       }
       // chunk P landed (one newer chunk may still be in flight)
+      YTA(2);
       tc::cp_wait<Y_NST - 2>();
+      YTA(3);
       const uint32_t sidx = sp % Y_NST;
       char* a2 = stg + sidx * Y_STAGE;
       char* b2h = a2 + Y_A2;
       char* b2l = b2h + Y_B2 / 2;
+      if (!(a.exp & 4)) {
+        float4 p[4], q[4];
 #pragma unroll
-      for (int k = 0; k < 4; ++k) {
-        const int c4 = 4 * ((tid >> 6) + 4 * k);
-        const uint32_t oa = (uint32_t)((c4 >> 2) * Y_A2LBO + (mb >> 3) * 128 + (mb & 7) * 16);
-        const uint32_t ol = (uint32_t)((c4 >> 2) * Y_A2LBO + ((64 + mb) >> 3) * 128 + (mb & 7) * 16);
-        if (a.exp & 4) continue;
-        const float4 p = *reinterpret_cast<const float4*>(a2 + oa);
-        *reinterpret_cast<float4*>(a2 + ol) = make_float4(lo32(p.x), lo32(p.y), lo32(p.z), lo32(p.w));
-        const uint32_t ob = tc::cm_off(mb, c4, 8);
-        const float4 q = *reinterpret_cast<const float4*>(b2h + ob);
-        *reinterpret_cast<float4*>(b2l + ob) = make_float4(lo32(q.x), lo32(q.y), lo32(q.z), lo32(q.w));
+        for (int k = 0; k < 4; ++k) {
+          const int r = cr + 16 * k;
+          p[k] = *reinterpret_cast<const float4*>(a2 + a2_off(r));
+          q[k] = *reinterpret_cast<const float4*>(b2h + b2_off(r));
+        }
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          const int r = cr + 16 * k;
+          *reinterpret_cast<float4*>(a2 + a2_off(64 + r)) =
+              make_float4(lo32(p[k].x), lo32(p[k].y), lo32(p[k].z), lo32(p[k].w));
+          *reinterpret_cast<float4*>(b2l + b2_off(r)) =
+              make_float4(lo32(q[k].x), lo32(q[k].y), lo32(q[k].z), lo32(q[k].w));
+        }
       }
+      YTA(4);
       tc::named_sync(1, Y_LW * 32);                     // whole chunk (hi and lo) visible
+      YTA(5);
       {   // dP^T of this chunk -> TMEM: chunk ck covers c-block ck / 2, lane quarters 2 (ck & 1) + {0, 1}
         const int blk = P.ck >> 1, Q = w & 3;
         if ((Q >> 1) == (P.ck & 1) && blk < a.nblk && !(a.exp & 8)) {
@@ -217,6 +261,7 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
           tc::tmem_wait_st();
         }
       }
+      YTA(6);
       tc::fence_async_smem();
       tc::fence_before();
       tc::mbar_arrive(&ctl.s_full[sidx]);
@@ -228,8 +273,11 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
       advance(P);
       // refill: the chunk two ahead
       if (I.g < NG) {
+        YTA(7);
         tc::mbar_wait(&ctl.s_free[si % Y_NST], ((si / Y_NST) & 1) ^ 1);
+        YTA(8);
         issue(I, si);
+        YTA(9);
         advance(I);
         ++si;
       }
@@ -245,17 +293,22 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
     // ------------------------------- MMA issuer -------------------------------
     uint32_t sk = 0, gs = 0;
     for (uint32_t ui = 0;; ++ui) {
+      YT0();
       tc::mbar_wait(&ctl.u_full[ui & 3], (ui >> 2) & 1);
+      YTA(10);
       const uint32_t fl = ctl.ring[ui & 3][3];
       __syncwarp();
       if (lane == 0) tc::mbar_arrive(&ctl.u_empty[ui & 3]);
       if (fl & 4u) break;
       // dA = [dP_hi; dP_lo] . C2_{hi,lo}^T over the K chunks (as they land)
       tc::mbar_wait(&ctl.d2_free, (ui & 1) ^ 1);
+      YTA(11);
       tc::fence_after();
       for (int ck = 0; ck < a.nchunk; ++ck, ++sk) {
         const uint32_t s = sk % Y_NST;
+        YTA(13);
         tc::mbar_wait(&ctl.s_full[s], (sk / Y_NST) & 1);
+        YTA(12);
         tc::fence_after();
         if (lane == 0) {
           const uint32_t id = tc::idesc_tf32(128, 64, false, false);
@@ -263,11 +316,13 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
 #pragma unroll
           for (int kk = 0; kk < 8; ++kk) {
             const uint64_t da = tc::sdesc(a2 + kk * 2 * Y_A2LBO, Y_A2LBO, 128);
-            const uint64_t dbh = tc::sdesc(b2h + kk * 2 * 8 * 128, 8 * 128, 128);
-            const uint64_t dbl = tc::sdesc(b2l + kk * 2 * 8 * 128, 8 * 128, 128);
+            const uint64_t dbh = tc::sdesc(b2h + kk * 2 * Y_B2LBO, Y_B2LBO, 128);
+            const uint64_t dbl = tc::sdesc(b2l + kk * 2 * Y_B2LBO, Y_B2LBO, 128);
             const uint32_t acc = (ck > 0 || kk > 0) ? 1u : 0u;
-            tc::mma_tf32(tm + 384, da, dbh, id, acc);
-            tc::mma_tf32(tm + 448, da, dbl, id, acc);
+            if (!(a.exp & 32)) {
+              tc::mma_tf32(tm + 384, da, dbh, id, acc);
+              tc::mma_tf32(tm + 448, da, dbl, id, acc);
+            }
           }
           tc::commit(&ctl.s_free[s]);
           if (ck + 1 == a.nchunk) tc::commit(&ctl.d2_full);
@@ -275,7 +330,10 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
         __syncwarp();
       }
       // dC2^T += dP^T . C1  (K = 64 tile rows), after the whole tile's dP^T reached TMEM
+      YTA(13);
       tc::mbar_wait(&ctl.a1_full, ui & 1);
+      YTA(14);
+      YTA(15);
       if (fl & 1u) tc::mbar_wait(&ctl.d1_free, (gs & 1) ^ 1);
       tc::fence_after();
       if (lane == 0) {
@@ -289,6 +347,7 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
             const uint64_t dbh = tc::sdesc(bh + o, (YR / 8) * 128, 128);
             const uint64_t dbl = tc::sdesc(bl + o, (YR / 8) * 128, 128);
             const uint32_t ah = tm + blk * 64 + kk * 8, al = tm + 128 + blk * 64 + kk * 8;
+            if (a.exp & 32) continue;
             tc::mma_tf32_ts(d, ah, dbh, id, ((fl & 1u) && kk == 0) ? 0u : 1u);
             tc::mma_tf32_ts(d, ah, dbl, id, 1u);
             tc::mma_tf32_ts(d, al, dbh, id, 1u);
@@ -298,6 +357,7 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
         if (fl & 2u) tc::commit(&ctl.d1_full);
       }
       __syncwarp();
+      YTA(16);
       if (fl & 2u) ++gs;
     }
   } else {
@@ -305,14 +365,30 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
     const int Q = w & 3;
     uint32_t gs = 0;
     for (uint32_t ui = 0;; ++ui) {
+      YT0();
       tc::mbar_wait(&ctl.u_full[ui & 3], (ui >> 2) & 1);
+      YTA(20);
       const uint32_t g = ctl.ring[ui & 3][0], qa = ctl.ring[ui & 3][1];
       const uint32_t np = ctl.ring[ui & 3][2], fl = ctl.ring[ui & 3][3];
       __syncwarp();
       if (fl & 4u) break;
       const int rows = (int)np << a.n1s;
+      // L2 prefetch of the group PF groups ahead in this CTA's order (dP rows of all its tiles +
+      // its C2 slice: two contiguous ranges), so the loaders' cp.async chunks hit L2.
+      if ((fl & 1u) && w == Y_LW + 1 && lane == 0 && a.pf > 0) {
+        const uint32_t gn = g + (uint32_t)a.pf * gridDim.x;
+        if (gn < NG) {
+          const uint32_t q0 = a.grp_off[gn], q1 = a.grp_off[gn + 1];
+          const size_t fl0 = (size_t)q0 * a.n1 * NC, nfl = (size_t)(q1 - q0) * a.n1 * NC;
+          for (size_t o = 0; o < nfl; o += 16384)
+            tc::bulk_prefetch_l2(a.dpbuf + fl0 + o, (uint32_t)(min((size_t)16384, nfl - o) * 4));
+          tc::bulk_prefetch_l2(a.cores + a.grp_c2[gn], (uint32_t)(YR * NC * 4));
+        }
+      }
       // dA: lanes 0..63 hold dP_hi rows (both passes), lanes 64..127 dP_lo rows (pass C2_hi)
+      YTA(25);
       tc::mbar_wait(&ctl.d2_full, ui & 1);
+      YTA(21);
       tc::fence_after();
       {
         const int m = (Q & 1) * 32 + lane;               // tile row of this lane
@@ -341,9 +417,11 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
       }
       tc::fence_before();
       tc::mbar_arrive(&ctl.d2_free);
+      YTA(22);
       if (fl & 2u) {
         // group complete: dC2^T [c][r1] -> gradient or fused C2 update (this CTA owns the slice)
         tc::mbar_wait(&ctl.d1_full, gs & 1);
+        YTA(23);
         tc::fence_after();
         const unsigned long long so = a.grp_c2[g];
         for (int blk = 0; blk < a.nblk; ++blk) {
@@ -357,11 +435,12 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
 #pragma unroll
                 for (int i = 0; i < 32; ++i) a.grads[base + (size_t)i * NC] = v[i];
               } else if (a.opt == TTEMB_SGD) {
-                float old[32];
+                // C2 -= lr dC2 as fire-and-forget reductions (each warp instruction covers 32
+                // consecutive floats): no read of the old slice, no load latency on this path
 #pragma unroll
-                for (int i = 0; i < 32; ++i) old[i] = a.cores[base + (size_t)i * NC];
-#pragma unroll
-                for (int i = 0; i < 32; ++i) a.cores[base + (size_t)i * NC] = old[i] - a.lr * v[i];
+                for (int i = 0; i < 32; ++i)
+                  asm volatile("red.global.add.f32 [%0], %1;" ::"l"(a.cores + base + (size_t)i * NC),
+                               "f"(-a.lr * v[i]) : "memory");
               } else {
 #pragma unroll
                 for (int h2 = 0; h2 < 32; h2 += 16) {
@@ -384,6 +463,7 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
         }
         tc::fence_before();
         tc::mbar_arrive(&ctl.d1_free);
+        YTA(24);
         ++gs;
       }
       if (lane == 0) tc::mbar_arrive(&ctl.u_empty[ui & 3]);
@@ -393,6 +473,16 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
   __syncthreads();
   tc::fence_after();
   if (w == Y_MMA_W) tc::tmem_dealloc(tm, 512);
+#ifdef TTEMB_TRACE_BUILD
+  if (a.trace) {
+    unsigned long long* tb = a.trace + 32 * blockIdx.x;
+    if (tid == 0) { for (int k = 0; k < 10; ++k) tb[k] = trc[k]; tb[30] = (unsigned long long)(clock64() - t_start); }
+    if (w == Y_MMA_W && lane == 0) for (int k = 10; k < 17; ++k) tb[k] = trc[k];
+    if (w == Y_LW + 1 && lane == 0) for (int k = 20; k < 26; ++k) tb[k] = trc[k];
+  }
+#endif
+#undef YT0
+#undef YTA
 }
 
 }  // namespace
@@ -414,9 +504,30 @@ cudaError_t run_prefix_bwd(Ctx& c, float lr, cudaStream_t s) {
   a.NC = c.NC; a.nblk = (c.NC + 127) / 128; a.tpp = YT / c.n1; a.nchunk = (c.NC + 63) / 64;
   a.lr = lr; a.eps = c.eps; a.opt = c.opt; a.fused = (c.flags & TTEMB_FUSED_UPDATE) ? 1 : 0;
   a.exp = exp_bits();
+  a.pf = env_int("TTEMB_PF_BWD", 0);
   StageScope sc(c, ST_BWD_PREFIX, s);
   const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(c.NG_cap, (int64_t)c.sm_count));
+  static unsigned long long* trace = nullptr;
+  a.trace = nullptr;
+  if (getenv("TTEMB_TRACE")) {
+    if (!trace) cudaMalloc(&trace, sizeof(unsigned long long) * 32 * grid);
+    cudaMemsetAsync(trace, 0, sizeof(unsigned long long) * 32 * grid, s);
+    a.trace = trace;
+  }
   k_prefix_bwd<<<grid, Y_THREADS, kBwdSmem, s>>>(a);
+  if (a.trace) {
+    std::vector<unsigned long long> hb(32 * grid);
+    cudaMemcpyAsync(hb.data(), trace, hb.size() * 8, cudaMemcpyDeviceToHost, s);
+    cudaStreamSynchronize(s);
+    double m[32] = {};
+    for (int b = 0; b < grid; ++b) for (int k = 0; k < 32; ++k) m[k] += (double)hb[32 * b + k] / grid;
+    fprintf(stderr, "[trace bwd] total %.0f | loader: tile-start %.0f a1_free %.0f b1+misc %.0f cp_wait %.0f lo %.0f "
+            "sync %.0f tmem %.0f fence+arrive %.0f s_free %.0f issue %.0f | mma: u_full %.0f d2_free %.0f s_full %.0f "
+            "dA-issue %.0f a1_full %.0f d1_free %.0f dC2-issue %.0f | epi: u_full %.0f d2_full %.0f dA-drain %.0f "
+            "d1_full %.0f dC2-drain %.0f misc %.0f (cycles/CTA)\n",
+            m[30], m[0], m[1], m[2], m[3], m[4], m[5], m[6], m[7], m[8], m[9], m[10], m[11], m[12], m[13], m[14],
+            m[15], m[16], m[20], m[21], m[22], m[23], m[24], m[25]);
+  }
   return cudaGetLastError();
 }
 

@@ -45,6 +45,12 @@ inline int exp_bits() {
   return v;
 }
 
+// Tuning knob from the environment (default when unset).
+inline int env_int(const char* name, int dflt) {
+  const char* e = getenv(name);
+  return e ? atoi(e) : dflt;
+}
+
 struct TableMeta {
   uint32_t m1, m2, m3, M;      // row factors, rows (M <= 2^32-1 checked on host)
   uint64_t rowbase;            // exclusive prefix sum of M (row numbering across tables)
