@@ -51,6 +51,12 @@ def lib():
         _lib.ttref_backward.argtypes = [C.POINTER(_Shape), C.c_void_p, C.c_void_p, C.c_void_p, i64p, i64p,
                                         C.c_int64, C.c_int32, C.POINTER(C.c_float), C.c_int,
                                         C.c_void_p, C.c_void_p, C.c_void_p]
+        _lib.ttref_forward_ex.argtypes = [C.POINTER(_Shape), C.c_void_p, C.c_void_p, C.c_void_p, i64p, i64p,
+                                          C.c_int64, C.c_int32, C.POINTER(C.c_float), C.c_int, C.c_int,
+                                          C.POINTER(C.c_double)]
+        _lib.ttref_backward_ex.argtypes = [C.POINTER(_Shape), C.c_void_p, C.c_void_p, C.c_void_p, i64p, i64p,
+                                           C.c_int64, C.c_int32, C.POINTER(C.c_float), C.c_int,
+                                           C.POINTER(C.c_float), C.c_int, C.c_void_p, C.c_void_p, C.c_void_p]
         _lib.ttref_update.argtypes = [C.c_int, C.c_double, C.c_double, C.c_int64, C.POINTER(C.c_float),
                                       C.POINTER(C.c_float), C.POINTER(C.c_double)]
         _lib.ttref_digits.argtypes = [C.POINTER(C.c_int32), C.c_int64, C.POINTER(C.c_int64)]
@@ -155,28 +161,45 @@ class Oracle:
         return out
 
     # -- forward / backward ------------------------------------------------
+    @staticmethod
+    def _mode(mode: str) -> int:
+        return {"sum": 0, "mean": 1}[mode]
+
     def forward(self, cores, indices, offsets, batch: int, literal: bool = False,
-                absolute: bool = False) -> np.ndarray:
-        """out[B][T][N] fp64.  absolute=True evaluates the |C| companion."""
+                absolute: bool = False, per_sample_weights=None, mode: str = "sum") -> np.ndarray:
+        """out[B][T][N] fp64.  absolute=True evaluates the |C| (and |weights|) companion.
+        mode / per_sample_weights follow nn.EmbeddingBag (weights only with mode="sum")."""
         if absolute:
             cores = [tuple(np.abs(x) for x in c) for c in cores]
         idx, off = self._ids(indices, offsets)
+        psw = None
+        if per_sample_weights is not None:
+            psw = np.ascontiguousarray(per_sample_weights, dtype=np.float32)
+            if absolute:
+                psw = np.abs(psw)
         k1, p1 = self._core_ptrs(cores, 0)
         k2, p2 = self._core_ptrs(cores, 1)
         k3, p3 = self._core_ptrs(cores, 2)
         out = np.zeros((batch, self.T, self.N), np.float64)
-        rc = lib().ttref_forward(C.byref(self._shape), p1, p2, p3, _p(idx, C.c_int64),
-                                 _p(off, C.c_int64), len(idx), int(batch), int(literal),
-                                 _p(out, C.c_double))
+        rc = lib().ttref_forward_ex(C.byref(self._shape), p1, p2, p3, _p(idx, C.c_int64),
+                                    _p(off, C.c_int64), len(idx), int(batch),
+                                    _p(psw, C.c_float) if psw is not None else None, self._mode(mode),
+                                    int(literal), _p(out, C.c_double))
         if rc:
             raise OracleError(rc)
         return out
 
     def backward(self, cores, indices, offsets, batch: int, grad_out, literal: bool = False,
-                 absolute: bool = False) -> List[Tuple[np.ndarray, np.ndarray, np.ndarray]]:
+                 absolute: bool = False, per_sample_weights=None,
+                 mode: str = "sum") -> List[Tuple[np.ndarray, np.ndarray, np.ndarray]]:
         """Core gradients of L = sum(out * grad_out), fp64, per table (dC1, dC2, dC3).
-        absolute=True evaluates the |C|, |grad_out| companion."""
+        absolute=True evaluates the |C|, |grad_out| (|weights|) companion."""
         go = np.ascontiguousarray(grad_out, dtype=np.float32)
+        psw = None
+        if per_sample_weights is not None:
+            psw = np.ascontiguousarray(per_sample_weights, dtype=np.float32)
+            if absolute:
+                psw = np.abs(psw)
         if absolute:
             cores = [tuple(np.abs(x) for x in c) for c in cores]
             go = np.abs(go)
@@ -189,8 +212,9 @@ class Oracle:
         g1 = (C.c_void_p * self.T)(*[g[0].ctypes.data for g in grads])
         g2 = (C.c_void_p * self.T)(*[g[1].ctypes.data for g in grads])
         g3 = (C.c_void_p * self.T)(*[g[2].ctypes.data for g in grads])
-        rc = lib().ttref_backward(C.byref(self._shape), p1, p2, p3, _p(idx, C.c_int64), _p(off, C.c_int64),
-                                  len(idx), int(batch), _p(go, C.c_float), int(literal), g1, g2, g3)
+        rc = lib().ttref_backward_ex(C.byref(self._shape), p1, p2, p3, _p(idx, C.c_int64), _p(off, C.c_int64),
+                                     len(idx), int(batch), _p(psw, C.c_float) if psw is not None else None,
+                                     self._mode(mode), _p(go, C.c_float), int(literal), g1, g2, g3)
         if rc:
             raise OracleError(rc)
         return grads

@@ -146,6 +146,20 @@ static int build_keys(const ttref_shape* s, const int64_t* indices, const int64_
   return bad ? -3 : 0;
 }
 
+/* Weight of position j in its bag (nn.EmbeddingBag semantics, P:48 / P:306 drop-in):
+ * mode 0 (sum): psw[j] if per-sample weights are given, else 1; mode 1 (mean): 1 / |bag|
+ * (PyTorch allows per-sample weights only with sum).  NULL result = all ones. */
+static double* position_weights(const ttref_shape* s, const int64_t* offsets, int64_t nnz, int32_t B,
+                                const float* psw, int mode) {
+  if (!psw && mode == 0) return NULL;
+  double* w = (double*)malloc(sizeof(double) * (size_t)(nnz ? nnz : 1));
+  for (int64_t bag = 0; bag < (int64_t)s->T * B; ++bag) {
+    const int64_t a = offsets[bag], e = offsets[bag + 1];
+    for (int64_t j = a; j < e; ++j) w[j] = mode == 1 ? 1.0 / (double)(e - a) : (double)psw[j];
+  }
+  return w;
+}
+
 static int table_of_key(const ttref_shape* s, uint32_t key, uint64_t* rowbase) {
   uint64_t base = 0;
   for (int t = 0; t < s->T; ++t) {
@@ -308,7 +322,13 @@ int ttref_apply_bijection(const ttref_shape* s, const int64_t* const* bij, const
 int ttref_forward(const ttref_shape* s, const float* const* C1, const float* const* C2,
                   const float* const* C3, const int64_t* indices, const int64_t* offsets,
                   int64_t nnz, int32_t B, int literal, double* out) {
-  if (check_shape(s) || B < 0 || nnz < 0) return -1;
+  return ttref_forward_ex(s, C1, C2, C3, indices, offsets, nnz, B, NULL, 0, literal, out);
+}
+
+int ttref_forward_ex(const ttref_shape* s, const float* const* C1, const float* const* C2,
+                     const float* const* C3, const int64_t* indices, const int64_t* offsets,
+                     int64_t nnz, int32_t B, const float* psw, int mode, int literal, double* out) {
+  if (check_shape(s) || B < 0 || nnz < 0 || mode < 0 || mode > 1 || (psw && mode != 0)) return -1;
   const int T = s->T;
   const int N = s->n[0] * s->n[1] * s->n[2];
   uint32_t* key = (uint32_t*)malloc(sizeof(uint32_t) * (size_t)(nnz ? nnz : 1));
@@ -327,7 +347,9 @@ int ttref_forward(const ttref_shape* s, const float* const* C1, const float* con
     else ttref_row_chain(s, t, C1[t], C2[t], C3[t], row, rows + u * N);
   }
 
-  /* Eq. 4: out[b][t] = sum of the rows of bag (t, b), in index order; empty -> 0 */
+  /* Eq. 4: out[b][t] = sum of the rows of bag (t, b), in index order; empty -> 0.
+   * Weighted / mean bags (nn.EmbeddingBag): out = sum_j w_j row_j */
+  double* w = position_weights(s, offsets, nnz, B, psw, mode);
   memset(out, 0, sizeof(double) * (size_t)B * T * N);
   for (int t = 0; t < T; ++t)
     for (int32_t b = 0; b < B; ++b) {
@@ -335,10 +357,11 @@ int ttref_forward(const ttref_shape* s, const float* const* C1, const float* con
       double* o = out + ((int64_t)b * T + t) * N;
       for (int64_t j = offsets[bag]; j < offsets[bag + 1]; ++j) {
         const double* e = rows + find_key(ukey, U, key[j]) * N;
-        for (int c = 0; c < N; ++c) o[c] += e[c];
+        const double wj = w ? w[j] : 1.0;
+        for (int c = 0; c < N; ++c) o[c] += wj * e[c];
       }
     }
-  free(rows); free(ukey); free(key);
+  free(w); free(rows); free(ukey); free(key);
   return 0;
 }
 
@@ -439,7 +462,15 @@ int ttref_backward(const ttref_shape* s, const float* const* C1, const float* co
                    const float* const* C3, const int64_t* indices, const int64_t* offsets,
                    int64_t nnz, int32_t B, const float* grad_out, int literal,
                    double* const* dC1, double* const* dC2, double* const* dC3) {
-  if (check_shape(s) || B < 0 || nnz < 0) return -1;
+  return ttref_backward_ex(s, C1, C2, C3, indices, offsets, nnz, B, NULL, 0, grad_out, literal,
+                           dC1, dC2, dC3);
+}
+
+int ttref_backward_ex(const ttref_shape* s, const float* const* C1, const float* const* C2,
+                      const float* const* C3, const int64_t* indices, const int64_t* offsets,
+                      int64_t nnz, int32_t B, const float* psw, int mode, const float* grad_out,
+                      int literal, double* const* dC1, double* const* dC2, double* const* dC3) {
+  if (check_shape(s) || B < 0 || nnz < 0 || mode < 0 || mode > 1 || (psw && mode != 0)) return -1;
   const int T = s->T;
   const int n1 = s->n[0], n2 = s->n[1], n3 = s->n[2], R = s->R;
   const int N = n1 * n2 * n3;
@@ -461,11 +492,14 @@ int ttref_backward(const ttref_shape* s, const float* const* C1, const float* co
   /* in-advance aggregation: G[u] = sum over the positions holding row u,
    * ascending position order */
   double* G = (double*)calloc((size_t)(U ? U : 1) * N, sizeof(double));
+  double* w = position_weights(s, offsets, nnz, B, psw, mode);   /* dout/drow_j = w_j */
   for (int64_t j = 0; j < nnz; ++j) {
     double* g = G + find_key(ukey, U, key[j]) * N;
     const float* go = grad_out + (int64_t)bag[j] * N;
-    for (int c = 0; c < N; ++c) g[c] += (double)go[c];
+    const double wj = w ? w[j] : 1.0;
+    for (int c = 0; c < N; ++c) g[c] += wj * (double)go[c];
   }
+  free(w);
 
   /* chunks of unique rows: per-row contributions in parallel, then summed into
    * the core gradients in ascending row order (parallel over slice elements) */

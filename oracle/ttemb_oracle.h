@@ -64,6 +64,13 @@ int ttref_forward(const ttref_shape* s, const float* const* C1, const float* con
                   const float* const* C3, const int64_t* indices, const int64_t* offsets,
                   int64_t nnz, int32_t B, int literal, double* out);
 
+/* nn.EmbeddingBag pooling variants ("drop-in replacement of nn.EmbeddingBag"):
+ * mode 0 = sum (psw = per-sample weights [nnz] or NULL), mode 1 = mean (psw must be NULL,
+ * empty bag -> 0).  out[b][t] = sum_j w_j W_t[idx_j], w_j = psw[j] or 1 or 1/|bag|. */
+int ttref_forward_ex(const ttref_shape* s, const float* const* C1, const float* const* C2,
+                     const float* const* C3, const int64_t* indices, const int64_t* offsets,
+                     int64_t nnz, int32_t B, const float* psw, int mode, int literal, double* out);
+
 /* Backward: dC_k (fp64, same layouts as the cores, overwritten) of
  * L = sum(out * grad_out), grad_out [B][T][N] float32.  literal != 0 uses the
  * 6-deep loop nest per element instead of explicit partial products. */
@@ -71,6 +78,12 @@ int ttref_backward(const ttref_shape* s, const float* const* C1, const float* co
                    const float* const* C3, const int64_t* indices, const int64_t* offsets,
                    int64_t nnz, int32_t B, const float* grad_out, int literal,
                    double* const* dC1, double* const* dC2, double* const* dC3);
+
+/* Backward of the weighted / mean forward (G_u = sum_j w_j grad_out[bag(j)]). */
+int ttref_backward_ex(const ttref_shape* s, const float* const* C1, const float* const* C2,
+                      const float* const* C3, const int64_t* indices, const int64_t* offsets,
+                      int64_t nnz, int32_t B, const float* psw, int mode, const float* grad_out,
+                      int literal, double* const* dC1, double* const* dC2, double* const* dC3);
 
 /* Update (a12): opt 0 = SGD  p -= lr g;  opt 1 = Adagrad (PyTorch semantics):
  * s += g^2; p -= lr g / (sqrt(s) + eps).  fp64 math, rounded to fp32 once. */

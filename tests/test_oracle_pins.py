@@ -367,3 +367,44 @@ def test_bijection_range_errors():
     assert e.value.code == ERR_INDEX_RANGE
     np.testing.assert_array_equal(orc.apply_bijection([np.arange(10)[::-1]], np.array([0, 9, 3]),
                                                       np.array([0, 3]), 1), [9, 0, 6])
+
+
+# ---------------------------------------------------------------------------
+# nn.EmbeddingBag pooling variants (drop-in replacement, P:48 / P:306): mean, per-sample weights
+# ---------------------------------------------------------------------------
+@pytest.mark.parametrize("mode,weighted", [("mean", False), ("sum", True)])
+def test_mean_and_weighted_bags_match_torch_embedding_bag(mode, weighted):
+    """Forward and core gradients of mean / per-sample-weighted bags against
+    torch.nn.functional.embedding_bag(mode, per_sample_weights) on the dense materialised table,
+    differentiated by torch.autograd (variable bag lengths incl. empty bags)."""
+    cfg = W.small_config([200, 64], [(5, 6, 7), (4, 4, 4)], (2, 2, 3), 4, 16, 1, 1.05)
+    rng = np.random.default_rng(11)
+    T, B = cfg.num_tables, cfg.batch
+    lens = rng.integers(0, 6, size=T * B); lens[0] = 0; lens[5] = 0
+    idx, off = W.make_batch(cfg, step=1, seed=11, lengths=lens)
+    psw = rng.uniform(-2, 2, size=len(idx)).astype(np.float32) if weighted else None
+    cores = W.make_cores(cfg, seed=11)
+    go = W.make_grad_out(cfg, B, seed=11)
+    orc = Oracle.from_config(cfg)
+    out = orc.forward(cores, idx, off, B, per_sample_weights=psw, mode=mode)
+    grads = orc.backward(cores, idx, off, B, go, per_sample_weights=psw, mode=mode)
+    for t in range(T):
+        ct = [torch.tensor(x, dtype=torch.float64, requires_grad=True) for x in cores[t]]
+        Wt = materialise_torch(ct, cfg.row_factors[t], cfg.col_factors, cfg.table_rows[t])
+        o = off[t * B:(t + 1) * B + 1]
+        w = torch.as_tensor(psw[o[0]:o[-1]], dtype=torch.float64) if weighted else None
+        ref = torch.nn.functional.embedding_bag(torch.as_tensor(idx[o[0]:o[-1]]), Wt,
+                                                torch.as_tensor(o[:-1] - o[0]), mode=mode,
+                                                per_sample_weights=w)
+        np.testing.assert_allclose(out[:, t, :], ref.detach().numpy(), rtol=1e-12, atol=1e-13)
+        (ref * torch.as_tensor(go[:, t, :], dtype=torch.float64)).sum().backward()
+        for k in range(3):
+            np.testing.assert_allclose(grads[t][k], ct[k].grad.numpy(), rtol=1e-11, atol=1e-12)
+
+
+def test_weights_with_mean_rejected():
+    orc = Oracle([10], [(2, 2, 3)], (1, 1, 2), 2)
+    cores = [(np.ones((2, 1, 2), np.float32), np.ones((2, 2, 1, 2), np.float32), np.ones((3, 2, 2), np.float32))]
+    with pytest.raises(OracleError) as e:
+        orc.forward(cores, np.array([1]), np.array([0, 1]), 1, per_sample_weights=np.ones(1), mode="mean")
+    assert e.value.code == ERR_INVALID
