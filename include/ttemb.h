@@ -65,6 +65,8 @@ typedef enum { TTEMB_SGD = 0, TTEMB_ADAGRAD = 1 } ttemb_opt;
 #define TTEMB_NO_PREFIX_REUSE 4u  /* every unique row computes its own prefix product
                                      C1[i1] C2[i2] (disables batch-level intermediate-result
                                      reuse) */
+#define TTEMB_MEAN_POOLING 16u   /* nn.EmbeddingBag mode="mean": out = sum / |bag| (empty
+                                     bag -> 0); default is mode="sum" (P:48, P:306 drop-in) */
 #define TTEMB_NO_AGGREGATION 8u   /* every lookup occurrence is its own row in forward and
                                      backward (disables row dedup and the in-advance gradient
                                      aggregation) */
@@ -168,6 +170,17 @@ typedef struct {
 } ttemb_plan;
 
 int ttemb_get_plan(ttemb_t h, ttemb_plan* plan);
+
+/* ttemb_forward with per-sample weights (nn.EmbeddingBag(mode="sum") per_sample_weights):
+ * out[b][t] = sum_j w[j] W_t[idx_j]; `per_sample_weights` is a DEVICE float array [nnz]
+ * aligned with `indices` (NULL = all ones, i.e. ttemb_forward).  The weights are copied into
+ * the workspace by the key-build kernel, so the caller may reuse the buffer once the call's
+ * work has run; the following ttemb_backward differentiates the weighted bags
+ * (G_u = sum_j w[j] grad_out[bag(j)]; the weights themselves get no gradient).
+ * TTEMB_ERR_INVALID_ARG with TTEMB_MEAN_POOLING (PyTorch allows weights only with "sum"). */
+int ttemb_forward_weighted(ttemb_t h, const void* indices, const int64_t* offsets,
+                           const float* per_sample_weights, int64_t nnz, int32_t batch, float* out,
+                           void* stream);
 
 /* Runtime index bijection (Sec. IV-B: "all indices will first be transformed into
  * new indices based on the index bijection function ... New_Batch = {index(i_j)}").

@@ -25,12 +25,13 @@ TTEMB_FUSED_UPDATE = 1
 TTEMB_FP32_CORES = 2
 TTEMB_NO_PREFIX_REUSE = 4
 TTEMB_NO_AGGREGATION = 8
+TTEMB_MEAN_POOLING = 16
 
 SYMBOLS = ["ttemb_query_sizes", "ttemb_create", "ttemb_destroy", "ttemb_core_layout",
            "ttemb_forward", "ttemb_backward", "ttemb_update", "ttemb_forward_host",
            "ttemb_backward_host", "ttemb_check", "ttemb_get_plan", "ttemb_read_counts",
            "ttemb_set_timing", "ttemb_stage_times", "ttemb_stage_name", "ttemb_status_string",
-           "ttemb_set_bijection", "ttemb_total_rows"]
+           "ttemb_set_bijection", "ttemb_total_rows", "ttemb_forward_weighted"]
 
 
 class ttemb_table(C.Structure):
@@ -95,6 +96,7 @@ def load(path: str = LIB_PATH):
     lib.ttemb_status_string.argtypes = [C.c_int]
     lib.ttemb_status_string.restype = C.c_char_p
     lib.ttemb_set_bijection.argtypes = [vp, vp]
+    lib.ttemb_forward_weighted.argtypes = [vp, vp, vp, vp, i64, i32, vp, vp]
     lib.ttemb_total_rows.argtypes = [vp]
     for s in SYMBOLS:
         f = getattr(lib, s)

@@ -28,8 +28,8 @@ def make_config(table_rows: Sequence[int], row_factors: Sequence[Tuple[int, int,
                 col_factors: Tuple[int, int, int], rank: int, max_batch: int, max_nnz: int,
                 optimizer: str = "sgd", adagrad_eps: float = 1e-10, fused_update: bool = False,
                 index_bits: int = 64, num_cores: int = 3, fp32_cores: bool = False,
-                prefix_reuse: bool = True, aggregation: bool = True):
-    """Returns (ttemb_config, keep-alive table array).  prefix_reuse / aggregation = False set the
+                prefix_reuse: bool = True, aggregation: bool = True, mode: str = "sum"):
+    """Returns (ttemb_config, keep-alive table array).  mode = "sum" | "mean" (nn.EmbeddingBag).  prefix_reuse / aggregation = False set the
     ablation flags TTEMB_NO_PREFIX_REUSE / TTEMB_NO_AGGREGATION."""
     T = len(table_rows)
     tabs = (L.ttemb_table * max(T, 1))()
@@ -52,7 +52,8 @@ def make_config(table_rows: Sequence[int], row_factors: Sequence[Tuple[int, int,
     cfg.adagrad_eps = float(adagrad_eps)
     cfg.flags = ((L.TTEMB_FUSED_UPDATE if fused_update else 0) | (L.TTEMB_FP32_CORES if fp32_cores else 0)
                  | (0 if prefix_reuse else L.TTEMB_NO_PREFIX_REUSE)
-                 | (0 if aggregation else L.TTEMB_NO_AGGREGATION))
+                 | (0 if aggregation else L.TTEMB_NO_AGGREGATION)
+                 | {"sum": 0, "mean": L.TTEMB_MEAN_POOLING}[mode])
     return cfg, tabs
 
 
@@ -85,6 +86,12 @@ def ttemb_core_layout(h: int, table: int, core: int) -> Tuple[int, Tuple[int, in
 
 def ttemb_forward(h: int, indices: int, offsets: int, nnz: int, batch: int, out: int, stream: int) -> int:
     return L.load().ttemb_forward(h, indices, offsets, int(nnz), int(batch), out, stream)
+
+
+def ttemb_forward_weighted(h: int, indices: int, offsets: int, per_sample_weights: int, nnz: int,
+                           batch: int, out: int, stream: int) -> int:
+    return L.load().ttemb_forward_weighted(h, indices, offsets, per_sample_weights or None, int(nnz),
+                                           int(batch), out, stream)
 
 
 def ttemb_backward(h: int, grad_out: int, lr: float, stream: int) -> int:
@@ -162,8 +169,9 @@ class TTEmbeddingBag:
     def __init__(self, table_rows, row_factors, col_factors, rank, max_batch, max_nnz,
                  optimizer: str = "sgd", adagrad_eps: float = 1e-10, fused_update: bool = False,
                  index_bits: int = 64, device: int = 0, fp32_cores: bool = False,
-                 prefix_reuse: bool = True, aggregation: bool = True):
+                 prefix_reuse: bool = True, aggregation: bool = True, mode: str = "sum"):
         L.load()
+        self.mode = mode
         self.table_rows = [int(x) for x in table_rows]
         self.row_factors = [tuple(int(y) for y in f) for f in row_factors]
         self.col_factors = tuple(int(x) for x in col_factors)
@@ -177,7 +185,7 @@ class TTEmbeddingBag:
         self._cfg, self._tabs = make_config(table_rows, row_factors, col_factors, rank, max_batch,
                                             max_nnz, optimizer, adagrad_eps, fused_update, index_bits,
                                             fp32_cores=fp32_cores, prefix_reuse=prefix_reuse,
-                                            aggregation=aggregation)
+                                            aggregation=aggregation, mode=mode)
         cb, sb, gb, wb = ttemb_query_sizes(self._cfg)
         self.sizes = dict(core_bytes=cb, state_bytes=sb, grad_bytes=gb, workspace_bytes=wb)
         f32 = torch.float32
@@ -238,15 +246,21 @@ class TTEmbeddingBag:
 
     # -- step ----------------------------------------------------------------
     def forward(self, indices: torch.Tensor, offsets: torch.Tensor, batch: int,
-                out: Optional[torch.Tensor] = None, stream=None) -> torch.Tensor:
+                out: Optional[torch.Tensor] = None, stream=None,
+                per_sample_weights: Optional[torch.Tensor] = None) -> torch.Tensor:
         want = torch.int64 if self.index_bits == 64 else torch.int32
         assert indices.dtype == want and indices.is_cuda and offsets.dtype == torch.int64
         assert offsets.numel() == self.T * batch + 1
         if out is None:
             out = torch.empty(batch, self.T, self.N, dtype=torch.float32, device=self.device)
         nnz = indices.numel()
-        rc = ttemb_forward(self.h, indices.data_ptr() if nnz else None, offsets.data_ptr(), nnz, batch,
-                           out.data_ptr() if out.numel() else None, _stream_ptr(stream))
+        psw = 0
+        if per_sample_weights is not None:
+            assert per_sample_weights.dtype == torch.float32 and per_sample_weights.is_cuda
+            assert per_sample_weights.is_contiguous() and per_sample_weights.numel() == nnz
+            psw = per_sample_weights.data_ptr() if nnz else 0
+        rc = ttemb_forward_weighted(self.h, indices.data_ptr() if nnz else None, offsets.data_ptr(), psw,
+                                    nnz, batch, out.data_ptr() if out.numel() else None, _stream_ptr(stream))
         check(rc, "ttemb_forward")
         self.batch, self.nnz = batch, nnz
         return out

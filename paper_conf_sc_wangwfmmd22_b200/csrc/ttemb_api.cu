@@ -73,7 +73,8 @@ int validate(const ttemb_config* cfg) {
   if (cfg->max_nnz > (int64_t(1) << 30)) return TTEMB_ERR_UNSUPPORTED;
   if ((int64_t)cfg->num_tables * cfg->max_batch > (int64_t(1) << 31)) return TTEMB_ERR_UNSUPPORTED;
   if (cfg->optimizer != TTEMB_SGD && cfg->optimizer != TTEMB_ADAGRAD) return TTEMB_ERR_INVALID_ARG;
-  if (cfg->flags & ~(TTEMB_FUSED_UPDATE | TTEMB_FP32_CORES | TTEMB_NO_PREFIX_REUSE | TTEMB_NO_AGGREGATION))
+  if (cfg->flags & ~(TTEMB_FUSED_UPDATE | TTEMB_FP32_CORES | TTEMB_NO_PREFIX_REUSE | TTEMB_NO_AGGREGATION |
+                     TTEMB_MEAN_POOLING))
     return TTEMB_ERR_INVALID_ARG;
   uint64_t total = 0, buckets = 0, keys = 0;
   for (int t = 0; t < cfg->num_tables; ++t) {
@@ -182,6 +183,7 @@ size_t carve(Ctx& c, uint8_t* base) {
   const size_t pf = tc_eligible(c) ? (size_t)P * c.n1 * c.NC : 1;
   p.pbuf = k.take<float>(pf);
   p.dpbuf = k.take<float>(pf);
+  p.wpos = k.take<float>(nnz);
   p.rows = k.take<float>((size_t)U * c.N);
   p.gbuf = k.take<float>((size_t)U * c.N);
   p.aggpart = k.take<float>(std::max<size_t>((size_t)2 * agg_chunks(nnz) * c.N,
@@ -321,8 +323,17 @@ int ttemb_core_layout(ttemb_t h, int table, int core, int64_t* offset_floats, in
 
 int ttemb_forward(ttemb_t h, const void* indices, const int64_t* offsets, int64_t nnz,
                   int32_t batch, float* out, void* stream) {
+  return ttemb_forward_weighted(h, indices, offsets, nullptr, nnz, batch, out, stream);
+}
+
+int ttemb_forward_weighted(ttemb_t h, const void* indices, const int64_t* offsets,
+                           const float* per_sample_weights, int64_t nnz, int32_t batch, float* out,
+                           void* stream) {
   if (!h) return TTEMB_ERR_INVALID_ARG;
   Ctx& c = h->c;
+  if (per_sample_weights && (c.flags & TTEMB_MEAN_POOLING)) return TTEMB_ERR_INVALID_ARG;
+  c.psw = nnz > 0 ? per_sample_weights : nullptr;
+  c.weighted = c.psw != nullptr || (c.flags & TTEMB_MEAN_POOLING) != 0;
   if (nnz < 0 || batch < 0 || !offsets || (nnz > 0 && !indices) || (!out && batch > 0))
     return TTEMB_ERR_INVALID_ARG;
   if (nnz > c.max_nnz || batch > c.max_batch) return TTEMB_ERR_CAPACITY;

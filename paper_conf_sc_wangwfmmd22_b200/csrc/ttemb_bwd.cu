@@ -37,7 +37,7 @@ __global__ void __launch_bounds__(256)
 k_agg(const float* __restrict__ grad_out, const uint32_t* __restrict__ skey,
       const uint32_t* __restrict__ sbag, const uint32_t* __restrict__ spos,
       const uint32_t* __restrict__ inverse, const uint32_t* __restrict__ seg_off, int64_t nnz,
-      int N, float* __restrict__ gbuf, float* __restrict__ part) {
+      int N, float* __restrict__ gbuf, float* __restrict__ part, const float* __restrict__ wpos) {
   using V = typename std::conditional<VW == 4, float4, float>::type;
   const int NV = N / VW;
   const uint32_t nchunks = (uint32_t)((nnz + AGG_CS - 1) / AGG_CS);
@@ -49,8 +49,9 @@ k_agg(const float* __restrict__ grad_out, const uint32_t* __restrict__ skey,
     V acc = V{};
     for (int64_t k = k0; k < k1; ++k) {
       const V v = __ldg(reinterpret_cast<const V*>(grad_out + (size_t)__ldg(sbag + k) * N + col));
-      if constexpr (VW == 4) { acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w; }
-      else acc += v;
+      const float w = wpos ? __ldg(wpos + __ldg(spos + k)) : 1.f;   // d out / d row_j = w_j
+      if constexpr (VW == 4) { acc.x += w * v.x; acc.y += w * v.y; acc.z += w * v.z; acc.w += w * v.w; }
+      else acc += w * v;
       const bool seg_end = (k + 1 == nnz) || __ldg(skey + k + 1) != __ldg(skey + k);
       if (seg_end || k + 1 == k1) {
         const uint32_t u = inverse[spos[k]];
@@ -135,7 +136,7 @@ __global__ void __launch_bounds__(256) k_zero_rows(float* __restrict__ buf, cons
 __global__ void __launch_bounds__(256)
 k_agg_scatter(const float* __restrict__ grad_out, const uint32_t* __restrict__ sbag,
               const uint32_t* __restrict__ spos, const uint32_t* __restrict__ inverse, int64_t nnz, int N,
-              float* __restrict__ gbuf) {
+              float* __restrict__ gbuf, const float* __restrict__ wpos) {
   const int lane = threadIdx.x & 31;
   const int NV = N >> 2, P = 32 / NV;            // float4 columns; occurrences in flight per step
   const int f = lane % NV, p = lane / NV;
@@ -145,9 +146,12 @@ k_agg_scatter(const float* __restrict__ grad_out, const uint32_t* __restrict__ s
     const int64_t k0 = ch * 32;
     const int cnt = (int)min((int64_t)32, nnz - k0);
     uint32_t bl = 0, ul = 0xffffffffu;
+    float wl = 1.f;
     if (lane < cnt) {
       bl = __ldg(sbag + k0 + lane);
-      ul = __ldg(inverse + __ldg(spos + k0 + lane));
+      const uint32_t pos = __ldg(spos + k0 + lane);
+      ul = __ldg(inverse + pos);
+      if (wpos) wl = __ldg(wpos + pos);
     }
     float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
     uint32_t cur = 0xffffffffu;
@@ -155,6 +159,7 @@ k_agg_scatter(const float* __restrict__ grad_out, const uint32_t* __restrict__ s
       const int i = i0 + p;
       const uint32_t bag = __shfl_sync(0xffffffffu, bl, i & 31);
       const uint32_t u = __shfl_sync(0xffffffffu, ul, i & 31);
+      const float w = __shfl_sync(0xffffffffu, wl, i & 31);
       if (i < cnt) {
         if (u != cur) {
           if (cur != 0xffffffffu)
@@ -164,7 +169,7 @@ k_agg_scatter(const float* __restrict__ grad_out, const uint32_t* __restrict__ s
           cur = u;
         }
         const float4 v = __ldg(reinterpret_cast<const float4*>(grad_out + (size_t)bag * N) + f);
-        acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
+        acc.x += w * v.x; acc.y += w * v.y; acc.z += w * v.z; acc.w += w * v.w;
       }
     }
     if (cur != 0xffffffffu)
@@ -251,16 +256,18 @@ cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s
     if (c.N % 4 == 0 && c.N <= 128 && (128 % c.N) == 0) {
       k_zero_rows<<<grid_for(c, c.U_cap * c.N / 4, 256, 8), 256, 0, s>>>(p.gbuf, p.counts, c.N);
       k_agg_scatter<<<grid_for(c, cdiv(c.nnz, 32), 8, 32), 256, 0, s>>>(grad_out, p.sbag, p.spos, p.inverse,
-                                                                         c.nnz, c.N, p.gbuf);
+                                                                         c.nnz, c.N, p.gbuf,
+                                                                         c.weighted ? p.wpos : nullptr);
     } else {
       const int64_t total = agg_chunks(c.nnz) * c.N;
       if (c.N % 4 == 0)
         k_agg<4><<<grid_for(c, total / 4, 256, 32), 256, 0, s>>>(grad_out, p.skey, p.sbag, p.spos,
                                                                 p.inverse, p.seg_off, c.nnz, c.N,
-                                                                p.gbuf, p.aggpart);
+                                                                p.gbuf, p.aggpart, c.weighted ? p.wpos : nullptr);
       else
         k_agg<1><<<grid_for(c, total, 256, 32), 256, 0, s>>>(grad_out, p.skey, p.sbag, p.spos, p.inverse,
-                                                            p.seg_off, c.nnz, c.N, p.gbuf, p.aggpart);
+                                                            p.seg_off, c.nnz, c.N, p.gbuf, p.aggpart,
+                                                            c.weighted ? p.wpos : nullptr);
       k_agg_fix<<<grid_for(c, agg_chunks(c.nnz) * 32, 256, 32), 256, 0, s>>>(
           p.skey, p.spos, p.inverse, p.seg_off, c.nnz, c.N, p.aggpart, p.gbuf);
     }

@@ -24,7 +24,7 @@ template <int VW>
 __global__ void __launch_bounds__(256)
 k_pool(const float* __restrict__ rows, const uint32_t* __restrict__ inverse,
        const int64_t* __restrict__ offsets, int64_t nnz, int T, int B, int N, float* __restrict__ out,
-       const uint32_t* __restrict__ counts, int skip_single) {
+       const uint32_t* __restrict__ counts, int skip_single, const float* __restrict__ wpos) {
   if (skip_single && counts[kCntMulti] == 0) return;   // one id per bag: written directly
   using V = typename std::conditional<VW == 4, float4, float>::type;
   const uint32_t NV = (uint32_t)(N / VW);
@@ -52,8 +52,9 @@ k_pool(const float* __restrict__ rows, const uint32_t* __restrict__ inverse,
       acc[i] = V{};
       for (int64_t j = s[i]; j < f[i]; ++j) {
         const V v = __ldg(reinterpret_cast<const V*>(rows + (size_t)__ldg(inverse + j) * N + col[i]));
-        if constexpr (VW == 4) { acc[i].x += v.x; acc[i].y += v.y; acc[i].z += v.z; acc[i].w += v.w; }
-        else acc[i] += v;
+        const float w = wpos ? __ldg(wpos + j) : 1.f;   // per-sample weight / 1 / |bag|
+        if constexpr (VW == 4) { acc[i].x += w * v.x; acc[i].y += w * v.y; acc[i].z += w * v.z; acc[i].w += w * v.w; }
+        else acc[i] += w * v;
       }
     }
 #pragma unroll
@@ -70,7 +71,7 @@ k_pool(const float* __restrict__ rows, const uint32_t* __restrict__ inverse,
 __global__ void __launch_bounds__(256)
 k_pool_single(const float* __restrict__ rows, const uint32_t* __restrict__ inverse,
               const uint32_t* __restrict__ bag_of, int64_t nnz, int N, float* __restrict__ out,
-              const uint32_t* __restrict__ counts) {
+              const uint32_t* __restrict__ counts, const float* __restrict__ wpos) {
   if (counts[kCntMulti] != 0) return;
   const int NV = N >> 2;
   const int64_t total = nnz * NV, stride = (int64_t)gridDim.x * blockDim.x;
@@ -85,6 +86,10 @@ k_pool_single(const float* __restrict__ rows, const uint32_t* __restrict__ inver
         const int64_t j = e / NV;
         const int f = (int)(e - j * NV);
         v[i] = __ldg(reinterpret_cast<const float4*>(rows + (size_t)__ldg(inverse + j) * N) + f);
+        if (wpos) {
+          const float w = __ldg(wpos + j);
+          v[i].x *= w; v[i].y *= w; v[i].z *= w; v[i].w *= w;
+        }
         dst[i] = (int64_t)__ldg(bag_of + j) * NV + f;
       }
     }
@@ -113,13 +118,16 @@ cudaError_t run_forward_compute(Ctx& c, float* out, const int64_t* offsets, cuda
         // one id per bag (device flag): a position-parallel copy; otherwise the bag-parallel sum
         if (c.nnz > 0)
           k_pool_single<<<grid_for(c, c.nnz * c.N / 16, 256, 32), 256, 0, s>>>(p.rows, p.inverse, p.bag_of,
-                                                                              c.nnz, c.N, out, p.counts);
+                                                                              c.nnz, c.N, out, p.counts,
+                                                                              c.weighted ? p.wpos : nullptr);
         k_pool<4><<<grid_for(c, total / 16, 256, 32), 256, 0, s>>>(p.rows, p.inverse, offsets, c.nnz,
-                                                                 c.T, c.B, c.N, out, p.counts, 1);
+                                                                 c.T, c.B, c.N, out, p.counts, 1,
+                                                                 c.weighted ? p.wpos : nullptr);
       }
       else
         k_pool<1><<<grid_for(c, total / 4, 256, 32), 256, 0, s>>>(p.rows, p.inverse, offsets, c.nnz, c.T,
-                                                             c.B, c.N, out, p.counts, 0);
+                                                             c.B, c.N, out, p.counts, 0,
+                                                             c.weighted ? p.wpos : nullptr);
     }
   }
   return cudaGetLastError();

@@ -144,7 +144,8 @@ __global__ void __launch_bounds__(256)
 k_build_keys(const IdxT* __restrict__ indices, const int64_t* __restrict__ offsets, int64_t nnz,
              int32_t B, int T, const TableMeta* __restrict__ meta, uint32_t* __restrict__ keys,
              uint32_t* __restrict__ bag_of, uint32_t* __restrict__ counts, int passes,
-             uint32_t* __restrict__ hist, const uint32_t* __restrict__ bij) {
+             uint32_t* __restrict__ hist, const uint32_t* __restrict__ bij,
+             const float* __restrict__ psw, int mean, float* __restrict__ wpos) {
   __shared__ uint32_t sh[4][256];
   for (int i = threadIdx.x; i < 4 * 256; i += blockDim.x) (&sh[0][0])[i] = 0;
   __syncthreads();
@@ -163,6 +164,7 @@ k_build_keys(const IdxT* __restrict__ indices, const int64_t* __restrict__ offse
     const uint32_t kb = (uint32_t)mt.kbase, M = mt.M, m1 = mt.m1, m2 = mt.m2, m3 = mt.m3;
     const uint32_t bo = (uint32_t)(bb * T + t);
     const uint32_t* bt = bij ? bij + mt.rowbase : nullptr;   // table t's bijection
+    const float wmean = e > s ? 1.0f / (float)(e - s) : 0.f; // nn.EmbeddingBag mode="mean"
     for (int64_t j = s; j < e; ++j) {
       const int64_t id = (int64_t)indices[j];
       uint32_t key = kb;
@@ -178,6 +180,7 @@ k_build_keys(const IdxT* __restrict__ indices, const int64_t* __restrict__ offse
       }
       keys[j] = key;
       bag_of[j] = bo;
+      if (wpos) wpos[j] = psw ? __ldg(psw + j) : wmean;
       for (int p = 0; p < passes; ++p) atomicAdd(&sh[p][(key >> (8 * p)) & 255u], 1u);
     }
   }
@@ -497,11 +500,15 @@ cudaError_t run_index_stage(Ctx& c, const void* indices, const int64_t* offsets,
     if (c.index_bits == 64)
       k_build_keys<int64_t><<<g, 256, 0, s>>>((const int64_t*)indices, offsets, nnz, c.B, c.T,
                                               c.d_meta, p.keysA, p.bag_of, p.counts,
-                                              c.key_passes, p.hist1, c.bij);
+                                              c.key_passes, p.hist1, c.bij, c.psw,
+                                              (c.flags & TTEMB_MEAN_POOLING) ? 1 : 0,
+                                              c.weighted ? p.wpos : nullptr);
     else
       k_build_keys<int32_t><<<g, 256, 0, s>>>((const int32_t*)indices, offsets, nnz, c.B, c.T,
                                               c.d_meta, p.keysA, p.bag_of, p.counts,
-                                              c.key_passes, p.hist1, c.bij);
+                                              c.key_passes, p.hist1, c.bij, c.psw,
+                                              (c.flags & TTEMB_MEAN_POOLING) ? 1 : 0,
+                                              c.weighted ? p.wpos : nullptr);
   }
   // a2: sort (key, position)
   const int64_t tiles1 = radix_tiles(nnz);

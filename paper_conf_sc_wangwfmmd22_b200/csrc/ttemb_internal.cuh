@@ -77,6 +77,7 @@ struct PlanDev {
   uint32_t *sc_counter, *sc_status;            // scans [3][tiles]
   uint32_t* work;                              // dynamic group schedulers [2]
   float *rows, *gbuf, *dabuf, *aggpart;
+  float* wpos;                                 // [nnz] bag weight of every position (weighted/mean bags)
   float *pbuf, *dpbuf;                         // tensor-core path: P and dL/dP per prefix
   uint32_t* grp_arow;                          // [P]  C1 row (float offset / R) of sorted prefix q, j1 = 0
   unsigned long long* grp_c2;                  // [NG] float offset of the C2 slice of group g
@@ -123,6 +124,8 @@ struct Ctx {
   int64_t nnz = 0;
   int32_t B = 0;
   bool fwd_done = false;
+  const float* psw = nullptr;        // per-sample weights of the current forward (device) or null
+  bool weighted = false;             // this step's bags carry weights (psw or mean): p.wpos valid
 
   // timing
   bool timing = false;

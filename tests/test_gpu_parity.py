@@ -416,3 +416,45 @@ def test_bijection_out_of_range_is_reported():
     emb.set_bijection(torch.as_tensor(bad, device=DEV))
     run_forward(emb, idx, off, cfg.batch)
     assert emb.check() == L.TTEMB_ERR_INDEX_RANGE
+
+
+@pytest.mark.parametrize("mode,weighted", [("mean", False), ("sum", True)], ids=["mean", "weighted"])
+@pytest.mark.parametrize("case", ["multi-var-L", "tc-n1-2", "c4-b1024-var"])
+def test_mean_and_weighted_bags(case, mode, weighted):
+    """nn.EmbeddingBag mode="mean" (TTEMB_MEAN_POOLING) and per-sample weights
+    (ttemb_forward_weighted) vs the oracle's definition (P:48 / P:306 drop-in); variable bag
+    lengths with empty bags; the backward differentiates the weighted bags."""
+    if case.startswith("c4"):
+        cfg, mode_in, B = W.config("c4"), "var", 1024
+    else:
+        cfg, mode_in = {c[0]: (c[1], c[2]) for c in small_cases()}[case]
+        mode_in, B = "var", None
+    idx, off, B = make_inputs(cfg, mode_in, seed=13, batch=B)
+    psw = np.random.default_rng(13).uniform(-2, 2, size=len(idx)).astype(np.float32) if weighted else None
+    cores = W.make_cores(cfg, seed=13)
+    go = W.make_grad_out(cfg, B, seed=13)
+    emb = gpu_emb(cfg, B, len(idx), mode=mode)
+    emb.load_cores(cores)
+    it = torch.as_tensor(idx.astype(np.int64), device=DEV)
+    out = emb.forward(it, torch.as_tensor(off, device=DEV), B,
+                      per_sample_weights=torch.as_tensor(psw, device=DEV) if weighted else None)
+    emb.backward(torch.as_tensor(go, device=DEV))
+    assert emb.check() == 0
+    orc = Oracle.from_config(cfg)
+    kw = dict(per_sample_weights=psw, mode=mode)
+    assert_companion(out.cpu().numpy(), orc.forward(cores, idx, off, B, **kw),
+                     orc.forward(cores, idx, off, B, absolute=True, **kw), 1e-5, "forward")
+    g = orc.backward(cores, idx, off, B, go, **kw)
+    ga = orc.backward(cores, idx, off, B, go, absolute=True, **kw)
+    for t, mine in enumerate(emb.grad_views()):
+        for k in range(3):
+            assert_companion(mine[k].cpu().numpy(), g[t][k], ga[t][k], 1e-4, f"dC{k+1} t{t}")
+
+
+def test_weights_with_mean_rejected_by_the_abi():
+    cfg = W.config("c1")
+    idx, off = W.make_batch(cfg, seed=1)
+    emb = gpu_emb(cfg, cfg.batch, len(idx), mode="mean")
+    with pytest.raises(tt.TTEmbError):
+        emb.forward(torch.as_tensor(idx, device=DEV), torch.as_tensor(off, device=DEV), cfg.batch,
+                    per_sample_weights=torch.ones(len(idx), device=DEV))
