@@ -36,7 +36,7 @@ def build(force: bool = False) -> str:
 
 class _Shape(C.Structure):
     _fields_ = [("T", C.c_int32), ("rows", C.POINTER(C.c_int64)), ("mfac", C.POINTER(C.c_int32)),
-                ("n", C.c_int32 * 3), ("R", C.c_int32)]
+                ("n", C.c_int32 * 3), ("R", C.c_int32), ("dense", C.POINTER(C.c_int32))]
 
 
 def lib():
@@ -83,19 +83,23 @@ class Oracle:
     """fp64 oracle for one table set (shared N = n1 n2 n3 and rank R)."""
 
     def __init__(self, table_rows: Sequence[int], row_factors: Sequence[Tuple[int, int, int]],
-                 col_factors: Tuple[int, int, int], rank: int):
+                 col_factors: Tuple[int, int, int], rank: int, dense: Sequence[bool] = ()):
+        """dense[t] = table t kept uncompressed (hybrid placement): its cores are
+        (W[M][N], empty, empty)."""
         self.rows = np.ascontiguousarray(table_rows, dtype=np.int64)
         self.mfac = np.ascontiguousarray(row_factors, dtype=np.int32).reshape(-1, 3)
         self.n = tuple(int(x) for x in col_factors)
         self.R = int(rank)
         self.T = len(self.rows)
         self.N = self.n[0] * self.n[1] * self.n[2]
+        self.dense = np.ascontiguousarray([1 if d else 0 for d in dense] if len(dense) else [0] * self.T,
+                                          dtype=np.int32)
         self._shape = _Shape(self.T, _p(self.rows, C.c_int64), _p(self.mfac, C.c_int32),
-                             (C.c_int32 * 3)(*self.n), self.R)
+                             (C.c_int32 * 3)(*self.n), self.R, _p(self.dense, C.c_int32))
 
     @classmethod
     def from_config(cls, cfg):
-        return cls(cfg.table_rows, cfg.row_factors, cfg.col_factors, cfg.rank)
+        return cls(cfg.table_rows, cfg.row_factors, cfg.col_factors, cfg.rank, getattr(cfg, "dense", ()))
 
     @staticmethod
     def num_threads() -> int:

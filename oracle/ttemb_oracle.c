@@ -102,14 +102,19 @@ void ttref_row_literal(const ttref_shape* s, int t, const float* C1, const float
 /* ------------------------------------------------------------------------ */
 /* Input validation and keys                                                 */
 /* ------------------------------------------------------------------------ */
+static int is_dense(const ttref_shape* s, int t) { return s->dense && s->dense[t]; }
+
 static int check_shape(const ttref_shape* s) {
   if (!s || s->T < 1 || !s->rows || !s->mfac || s->R < 1) return -1;
   for (int k = 0; k < 3; ++k) if (s->n[k] < 1) return -1;
   uint64_t tot = 0;
   for (int t = 0; t < s->T; ++t) {
     const int32_t* m = s->mfac + 3 * t;
-    if (s->rows[t] < 1 || m[0] < 1 || m[1] < 1 || m[2] < 1) return -1;
-    if ((int64_t)m[0] * m[1] * m[2] < s->rows[t]) return -1;
+    if (s->rows[t] < 1) return -1;
+    if (!is_dense(s, t)) {
+      if (m[0] < 1 || m[1] < 1 || m[2] < 1) return -1;
+      if ((int64_t)m[0] * m[1] * m[2] < s->rows[t]) return -1;
+    }
     tot += (uint64_t)s->rows[t];
   }
   if (tot > 0xFFFFFFFFull) return -1;
@@ -214,23 +219,26 @@ static int plan_keys(const ttref_shape* s, const int64_t* indices, const int64_t
   if (check_offsets(offsets, (int64_t)T * B, nnz)) return -1;
   uint64_t gbase = 0;
   int bad = 0;
-  for (int t = 0; t < T; ++t) {
-    const int32_t* m = s->mfac + 3 * t;
-    for (int32_t b = 0; b < B; ++b) {
-      const int64_t bag = (int64_t)t * B + b;
-      for (int64_t j = offsets[bag]; j < offsets[bag + 1]; ++j) {
-        const int64_t id = indices[j];
-        if (id < 0 || id >= s->rows[t]) { bad = 1; key[j] = (uint32_t)gbase; }
-        else {
-          int64_t d[3];
-          ttref_digits(m, id, d);
-          key[j] = (uint32_t)(gbase + (uint64_t)((d[1] * m[0] + d[0]) * m[2] + d[2]));
+  for (int pass = 0; pass < 2; ++pass)       /* TT tables first, then the dense ones */
+    for (int t = 0; t < T; ++t) {
+      if (is_dense(s, t) != pass) continue;
+      const int32_t* m = s->mfac + 3 * t;
+      for (int32_t b = 0; b < B; ++b) {
+        const int64_t bag = (int64_t)t * B + b;
+        for (int64_t j = offsets[bag]; j < offsets[bag + 1]; ++j) {
+          const int64_t id = indices[j];
+          if (id < 0 || id >= s->rows[t]) { bad = 1; key[j] = (uint32_t)gbase; }
+          else if (pass) key[j] = (uint32_t)(gbase + (uint64_t)id);
+          else {
+            int64_t d[3];
+            ttref_digits(m, id, d);
+            key[j] = (uint32_t)(gbase + (uint64_t)((d[1] * m[0] + d[0]) * m[2] + d[2]));
+          }
+          bag_of[j] = (uint32_t)((int64_t)b * T + t);
         }
-        bag_of[j] = (uint32_t)((int64_t)b * T + t);
       }
+      gbase += pass ? (uint64_t)s->rows[t] : (uint64_t)m[0] * m[1] * m[2];
     }
-    gbase += (uint64_t)m[0] * m[1] * m[2];
-  }
   return bad ? -3 : 0;
 }
 
@@ -260,11 +268,21 @@ int ttref_plan(const ttref_shape* s, const int64_t* indices, const int64_t* offs
   seg_off[U] = (uint32_t)nnz;
 
   /* digits back from the plan key; unique prefixes (t, i2, i1) and i2-groups (t, i2) are runs */
-  int64_t P = 0, NG = 0;
+  int64_t P = 0, NG = 0, Utt = U;
+  uint64_t ttkeys = 0;
+  for (int t = 0; t < s->T; ++t)
+    if (!is_dense(s, t)) ttkeys += (uint64_t)s->mfac[3 * t] * s->mfac[3 * t + 1] * s->mfac[3 * t + 2];
   for (int64_t u = 0; u < U; ++u) {
+    if ((uint64_t)ukey[u] >= ttkeys) {          /* a dense-table row: no TT digits, no prefix */
+      if (Utt == U) Utt = u;
+      row_pfx[u] = 0xFFFFFFFFu;
+      row_i3[u] = 0;
+      continue;
+    }
     uint64_t gbase = 0;
     int t = 0;
     for (; t < s->T - 1; ++t) {
+      if (is_dense(s, t)) continue;
       const int32_t* m = s->mfac + 3 * t;
       const uint64_t span = (uint64_t)m[0] * m[1] * m[2];
       if ((uint64_t)ukey[u] < gbase + span) break;
@@ -286,7 +304,7 @@ int ttref_plan(const ttref_shape* s, const int64_t* indices, const int64_t* offs
     row_pfx[u] = (uint32_t)(P - 1);
     row_i3[u] = i3;
   }
-  row_seg[P] = (uint32_t)U;
+  row_seg[P] = (uint32_t)Utt;
   grp_off[NG] = (uint32_t)P;
   counts[0] = U; counts[1] = P; counts[2] = NG;
   free(v); free(key);
@@ -343,7 +361,9 @@ int ttref_forward_ex(const ttref_shape* s, const float* const* C1, const float* 
   for (int64_t u = 0; u < U; ++u) {
     uint64_t rb; int t = table_of_key(s, ukey[u], &rb);
     int64_t row = (int64_t)ukey[u] - (int64_t)rb;
-    if (literal) ttref_row_literal(s, t, C1[t], C2[t], C3[t], row, rows + u * N);
+    if (is_dense(s, t)) {                       /* uncompressed table: W[row] */
+      for (int c = 0; c < N; ++c) rows[u * N + c] = (double)C1[t][row * N + c];
+    } else if (literal) ttref_row_literal(s, t, C1[t], C2[t], C3[t], row, rows + u * N);
     else ttref_row_chain(s, t, C1[t], C2[t], C3[t], row, rows + u * N);
   }
 
@@ -478,6 +498,10 @@ int ttref_backward_ex(const ttref_shape* s, const float* const* C1, const float*
 
   for (int t = 0; t < T; ++t) {
     const int32_t* m = s->mfac + 3 * t;
+    if (is_dense(s, t)) {                       /* dW of an uncompressed table */
+      memset(dC1[t], 0, sizeof(double) * (size_t)s->rows[t] * N);
+      continue;
+    }
     memset(dC1[t], 0, sizeof(double) * (size_t)m[0] * s1);
     memset(dC2[t], 0, sizeof(double) * (size_t)m[1] * s2);
     memset(dC3[t], 0, sizeof(double) * (size_t)m[2] * s3);
@@ -501,6 +525,14 @@ int ttref_backward_ex(const ttref_shape* s, const float* const* C1, const float*
   }
   free(w);
 
+  /* uncompressed tables: dW[row] = G_u */
+  for (int64_t u = 0; u < U; ++u) {
+    uint64_t rb; int t = table_of_key(s, ukey[u], &rb);
+    if (!is_dense(s, t)) continue;
+    const int64_t row = (int64_t)ukey[u] - (int64_t)rb;
+    for (int c = 0; c < N; ++c) dC1[t][row * N + c] += G[u * N + c];
+  }
+
   /* chunks of unique rows: per-row contributions in parallel, then summed into
    * the core gradients in ascending row order (parallel over slice elements) */
   int64_t per_row = s1 + s2 + s3;
@@ -518,6 +550,7 @@ int ttref_backward_ex(const ttref_shape* s, const float* const* C1, const float*
       for (int64_t u = u0; u < u1; ++u) {
         uint64_t rb; int t = table_of_key(s, ukey[u], &rb);
         int64_t row = (int64_t)ukey[u] - (int64_t)rb;
+        if (is_dense(s, t)) { dig[4 * (u - u0)] = -1; continue; }
         int64_t d[3];
         ttref_digits(s->mfac + 3 * t, row, d);
         int64_t* dg = dig + 4 * (u - u0);
@@ -535,6 +568,7 @@ int ttref_backward_ex(const ttref_shape* s, const float* const* C1, const float*
     for (int64_t e = 0; e < per_row; ++e) {
       for (int64_t u = u0; u < u1; ++u) {
         const int64_t* dg = dig + 4 * (u - u0);
+        if (dg[0] < 0) continue;                  /* dense-table row (done above) */
         const double v = contrib[(u - u0) * per_row + e];
         if (e < s1) dC1[dg[0]][dg[1] * s1 + e] += v;
         else if (e < s1 + s2) dC2[dg[0]][dg[2] * s2 + (e - s1)] += v;

@@ -36,6 +36,9 @@ typedef struct {
   const int32_t* mfac;    /* [T][3] row factors, prod >= M_t */
   int32_t n[3];           /* column factors, N = n1*n2*n3 */
   int32_t R;              /* TT rank, R1 = R2 = R, R0 = R3 = 1 */
+  const int32_t* dense;   /* [T] or NULL: dense[t] != 0 = table t kept uncompressed (hybrid
+                             placement): its "C1" is the plain table W[M][N], C2 / C3 are
+                             absent (NULL), row factors ignored */
 } ttref_shape;
 
 /* Eq. 3 digits of row id i of a table with factors m[3]. */
@@ -49,7 +52,9 @@ void ttref_row_literal(const ttref_shape* s, int t, const float* C1, const float
                        const float* C3, int64_t row, double* e);
 
 /* Integer plan: arrays sized nnz (U, P, NG <= nnz), the
- * *_off / row_seg arrays one more.  counts = {U, P, NG}. */
+ * *_off / row_seg arrays one more.  counts = {U, P, NG}.  Plan keys number the TT tables first
+ * (user order), then the dense tables; dense rows have row_pfx = 0xFFFFFFFF, row_i3 = 0 and no
+ * prefix, so row_seg[P] = number of TT rows. */
 int ttref_plan(const ttref_shape* s, const int64_t* indices, const int64_t* offsets,
                int64_t nnz, int32_t B,
                uint32_t* skey, uint32_t* spos, uint32_t* bag_of,

@@ -80,6 +80,10 @@ class TTConfig:
     pooling: int                    # fixed bag length L (ids per bag)
     zipf_s: Optional[float]         # None -> uniform ids
     id_map: str = "identity"        # "identity" | "perm"
+    dense: Tuple[bool, ...] = ()    # hybrid placement: table kept uncompressed; () = all TT
+
+    def is_dense(self, t: int) -> bool:
+        return bool(self.dense) and bool(self.dense[t])
 
     @property
     def num_tables(self) -> int:
@@ -125,6 +129,14 @@ def config(name: str, rank: Optional[int] = None) -> TTConfig:
 
 
 ALL_CONFIGS = ("c1", "c2", "c3", "c4", "c5")
+
+HYBRID_THRESHOLD = 1_000_000   # "decompose the embedding tables that have more than 1 million rows"
+
+
+def hybrid(cfg: TTConfig, threshold: int = HYBRID_THRESHOLD) -> TTConfig:
+    """The paper's end-to-end placement: tables with more than `threshold` rows are TT
+    compressed, the others stay plain (dense) EmbeddingBag tables."""
+    return cfg.replace(name=cfg.name + "-hybrid", dense=tuple(M <= threshold for M in cfg.table_rows))
 
 
 # ---------------------------------------------------------------------------
@@ -229,7 +241,8 @@ def shard_batch(indices: np.ndarray, offsets: np.ndarray, num_tables: int, batch
 # ---------------------------------------------------------------------------
 def make_cores(cfg: TTConfig, seed: int = 0, mixed_magnitude: bool = False
                ) -> List[Tuple[np.ndarray, np.ndarray, np.ndarray]]:
-    """Per table (C1[m1][n1][R], C2[m2][R][n2][R], C3[m3][R][n3]) float32.
+    """Per table (C1[m1][n1][R], C2[m2][R][n2][R], C3[m3][R][n3]) float32; a dense (hybrid)
+    table is (W[M][N] ~ U(-1/sqrt(N), 1/sqrt(N)), empty, empty).
 
     DESIGN.md R21: C1 ~ U(-1,1), C2, C3 ~ U(-1/sqrt(R), 1/sqrt(R)).
     mixed_magnitude scales a seeded 10% of C2 slices by 1e3 (exercises the
@@ -240,6 +253,12 @@ def make_cores(cfg: TTConfig, seed: int = 0, mixed_magnitude: bool = False
     out = []
     for t, (m1, m2, m3) in enumerate(cfg.row_factors):
         g = rng("cores", cfg.name, seed, t)
+        if cfg.is_dense(t):
+            N = n1 * n2 * n3
+            w = g.uniform(-1.0, 1.0, size=(cfg.table_rows[t], N)) / np.sqrt(N)
+            out.append((w.astype(np.float32), np.zeros((0, R, n2, R), np.float32),
+                        np.zeros((0, R, n3), np.float32)))
+            continue
         c1 = g.uniform(-1.0, 1.0, size=(m1, n1, R)).astype(np.float32)
         c2 = g.uniform(-a, a, size=(m2, R, n2, R)).astype(np.float32)
         c3 = g.uniform(-a, a, size=(m3, R, n3)).astype(np.float32)
@@ -260,8 +279,11 @@ def core_bytes(cfg: TTConfig) -> int:
     n1, n2, n3 = cfg.col_factors
     R = cfg.rank
     tot = 0
-    for m1, m2, m3 in cfg.row_factors:
-        tot += m1 * n1 * R + m2 * R * n2 * R + m3 * R * n3
+    for t, (m1, m2, m3) in enumerate(cfg.row_factors):
+        if cfg.is_dense(t):
+            tot += cfg.table_rows[t] * n1 * n2 * n3
+        else:
+            tot += m1 * n1 * R + m2 * R * n2 * R + m3 * R * n3
     return 4 * tot
 
 

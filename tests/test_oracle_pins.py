@@ -408,3 +408,80 @@ def test_weights_with_mean_rejected():
     with pytest.raises(OracleError) as e:
         orc.forward(cores, np.array([1]), np.array([0, 1]), 1, per_sample_weights=np.ones(1), mode="mean")
     assert e.value.code == ERR_INVALID
+
+
+# ---------------------------------------------------------------------------
+# Hybrid placement: small tables stay plain EmbeddingBag tables
+# ---------------------------------------------------------------------------
+def _hybrid_cfg():
+    base = W.small_config([37, 300, 5, 1000], [(3, 4, 4), (7, 7, 7), (1, 2, 3), (10, 10, 10)],
+                          (2, 3, 2), 4, 24, 1, 1.05)
+    return W.hybrid(base, threshold=100)            # tables 0 and 2 dense, 1 and 3 TT
+
+
+def test_hybrid_forward_and_gradients_match_torch():
+    """Dense tables are plain nn.EmbeddingBag tables (W[M][N]); TT tables as before.  Forward and
+    gradients (dW and dC_k) against torch embedding_bag + autograd on W / the materialised table."""
+    cfg = _hybrid_cfg()
+    assert cfg.dense == (True, False, True, False)
+    rng = np.random.default_rng(21)
+    T, B = cfg.num_tables, cfg.batch
+    lens = rng.integers(0, 5, size=T * B); lens[1] = 0
+    idx, off = W.make_batch(cfg, step=2, seed=21, lengths=lens)
+    cores = W.make_cores(cfg, seed=21)
+    go = W.make_grad_out(cfg, B, seed=21)
+    orc = Oracle.from_config(cfg)
+    out = orc.forward(cores, idx, off, B)
+    grads = orc.backward(cores, idx, off, B, go)
+    for t in range(T):
+        o = off[t * B:(t + 1) * B + 1]
+        if cfg.dense[t]:
+            params = [torch.tensor(cores[t][0], dtype=torch.float64, requires_grad=True)]
+            Wt = params[0]
+        else:
+            params = [torch.tensor(x, dtype=torch.float64, requires_grad=True) for x in cores[t]]
+            Wt = materialise_torch(params, cfg.row_factors[t], cfg.col_factors, cfg.table_rows[t])
+        ref = torch.nn.functional.embedding_bag(torch.as_tensor(idx[o[0]:o[-1]]), Wt,
+                                                torch.as_tensor(o[:-1] - o[0]), mode="sum")
+        np.testing.assert_allclose(out[:, t, :], ref.detach().numpy(), rtol=1e-12, atol=1e-13)
+        (ref * torch.as_tensor(go[:, t, :], dtype=torch.float64)).sum().backward()
+        for k, prm in enumerate(params):
+            np.testing.assert_allclose(grads[t][k], prm.grad.numpy(), rtol=1e-11, atol=1e-12)
+        if cfg.dense[t]:
+            assert grads[t][1].size == 0 and grads[t][2].size == 0
+
+
+def test_hybrid_plan_keys_tt_tables_first():
+    """Plan keys number the TT tables first, then the dense tables (row id order); dense rows have
+    no prefix (row_pfx = 0xFFFFFFFF) and the prefix rows end where the dense rows begin."""
+    cfg = _hybrid_cfg()
+    B = cfg.batch
+    idx, off = W.make_batch(cfg, step=3, seed=22)
+    orc = Oracle.from_config(cfg)
+    plan = orc.plan(idx, off, B)
+    T = cfg.num_tables
+    mf = np.array(cfg.row_factors, np.int64)
+    span = np.where(np.array(cfg.dense), np.array(cfg.table_rows), mf.prod(axis=1))
+    order_t = [t for t in range(T) if not cfg.dense[t]] + [t for t in range(T) if cfg.dense[t]]
+    base = np.zeros(T, np.int64)
+    acc = 0
+    for t in order_t:
+        base[t] = acc
+        acc += span[t]
+    bag = np.repeat(np.arange(T * B), np.diff(off))
+    tab = bag // B
+    key = np.empty(len(idx), np.int64)
+    for j, (i, t) in enumerate(zip(idx, tab)):
+        if cfg.dense[t]:
+            key[j] = base[t] + i
+        else:
+            d1, d2, d3 = np.unravel_index(i, tuple(mf[t]))
+            key[j] = base[t] + (d2 * mf[t, 0] + d1) * mf[t, 2] + d3
+    order = np.argsort(key, kind="stable")
+    np.testing.assert_array_equal(plan["skey"], key[order])
+    uk = np.unique(key)
+    np.testing.assert_array_equal(plan["ukey"], uk)
+    ntt = int(np.sum(uk < sum(span[t] for t in range(T) if not cfg.dense[t])))
+    assert np.all(plan["row_pfx"][ntt:] == 0xFFFFFFFF) and np.all(plan["row_pfx"][:ntt] < plan["P"])
+    assert plan["row_seg"][-1] == ntt
+    assert set(plan["pfx_t"].tolist()) <= {1, 3}
