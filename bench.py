@@ -104,8 +104,10 @@ def step_work(cfg, B, nnz, counts, touched, opt):
     n1, n2, n3 = cfg.col_factors
     R, N, T = cfg.rank, cfg.dim, cfg.num_tables
     U, P = counts["U"], counts["P"]
-    flops = 3 * 2 * n1 * n2 * R * R * P + 3 * 2 * N * R * U
-    slice_bytes = 4 * (touched["c1"] * n1 * R + touched["c2"] * R * n2 * R + touched["c3"] * R * n3)
+    nd = touched.get("dense_rows", 0)                  # hybrid: plain rows (no TT arithmetic)
+    flops = 3 * 2 * n1 * n2 * R * R * P + 3 * 2 * N * R * (U - nd)
+    slice_bytes = 4 * (touched["c1"] * n1 * R + touched["c2"] * R * n2 * R + touched["c3"] * R * n3
+                       + nd * N)
     passes = 3 if opt == "sgd" else 5                  # fwd read, bwd read, update write (+ state r/w)
     bytes_ = 8 * nnz + 8 * (T * B + 1) + 2 * 4 * N * T * B + passes * slice_bytes
     return flops, bytes_
@@ -339,6 +341,8 @@ def main():
     ap.add_argument("--bijection", type=int, default=0, metavar="K",
                     help="f2: frequency-ordering index bijection (Alg. 2 l.1-4) built offline from K "
                          "history batches of the stream, applied at run time (P:269)")
+    ap.add_argument("--hybrid", action="store_true",
+                    help="f3: hybrid placement -- tables with <= 1M rows stay dense (P:310)")
     ap.add_argument("--no-graph", dest="graph", action="store_false",
                     help="launch every step eagerly instead of replaying a captured CUDA graph")
     args = ap.parse_args()
@@ -349,6 +353,8 @@ def main():
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
     cfg = W.config(args.config, args.rank) if args.config == "c5" else W.config(args.config)
     cfg = cfg.replace(id_map=args.ids)
+    if args.hybrid:
+        cfg = W.hybrid(cfg)
     if args.scaling is None:
         args.scaling = "strong" if args.config == "c5" else "weak"
 
@@ -387,6 +393,7 @@ def main():
         pool.append((idx, off, go))
     max_nnz = max(len(p[0]) for p in pool)
     emb = tt.TTEmbeddingBag(cfg.table_rows, cfg.row_factors, cfg.col_factors, cfg.rank, B, max_nnz,
+                            dense=cfg.dense,
                             optimizer=args.opt, fused_update=fused, device=local_rank,
                             fp32_cores=args.fp32_cores, prefix_reuse=not args.no_reuse,
                             aggregation=not args.no_agg)
@@ -481,10 +488,12 @@ def main():
     nnz_last = len(pool[last][0])
     pt = plan["pfx_t"].cpu().numpy().astype(np.int64)
     pi1 = plan["pfx_i1"].cpu().numpy().astype(np.int64)
-    ri3 = plan["row_i3"].cpu().numpy().astype(np.int64)
-    rt = pt[plan["row_pfx"].cpu().numpy().astype(np.int64)]
+    rp = plan["row_pfx"].cpu().numpy().astype(np.int64) & 0xFFFFFFFF
+    tt_row = rp != 0xFFFFFFFF                       # hybrid: dense-table rows have no prefix
+    ri3 = plan["row_i3"].cpu().numpy().astype(np.int64)[tt_row]
+    rt = pt[rp[tt_row]]
     touched = {"c1": len(np.unique(pt * (1 << 32) + pi1)), "c2": counts["NG"],
-               "c3": len(np.unique(rt * (1 << 32) + ri3))}
+               "c3": len(np.unique(rt * (1 << 32) + ri3)), "dense_rows": int((~tt_row).sum())}
     hbm_peak, sm_max_mhz, bf16_peak, peak_kind = load_peaks()
     on_tc = tc_path(cfg, args)
     sm_count = torch.cuda.get_device_properties(dev).multi_processor_count

@@ -73,7 +73,12 @@ typedef enum { TTEMB_SGD = 0, TTEMB_ADAGRAD = 1 } ttemb_opt;
 
 typedef struct {
   int64_t num_rows;        /* M_t >= 1 */
-  int32_t row_factors[3];  /* (m1, m2, m3), m1 m2 m3 >= M_t  (R10) */
+  int32_t row_factors[3];  /* (m1, m2, m3), m1 m2 m3 >= M_t  (R10); ignored if dense */
+  int32_t dense;           /* != 0: hybrid placement (only tables with more than 1 M
+                              rows are TT-compressed) -- the table is a plain EmbeddingBag
+                              table W[M_t][dim] in the cores buffer (ttemb_core_layout core 0,
+                              shape {M_t, dim, 1, 1}; cores 1 and 2 are empty), looked up,
+                              pooled, aggregated and updated by the same call */
 } ttemb_table;
 
 typedef struct {

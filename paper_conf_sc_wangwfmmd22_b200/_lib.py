@@ -35,7 +35,7 @@ SYMBOLS = ["ttemb_query_sizes", "ttemb_create", "ttemb_destroy", "ttemb_core_lay
 
 
 class ttemb_table(C.Structure):
-    _fields_ = [("num_rows", C.c_int64), ("row_factors", C.c_int32 * 3)]
+    _fields_ = [("num_rows", C.c_int64), ("row_factors", C.c_int32 * 3), ("dense", C.c_int32)]
 
 
 class ttemb_config(C.Structure):

@@ -28,13 +28,16 @@ def make_config(table_rows: Sequence[int], row_factors: Sequence[Tuple[int, int,
                 col_factors: Tuple[int, int, int], rank: int, max_batch: int, max_nnz: int,
                 optimizer: str = "sgd", adagrad_eps: float = 1e-10, fused_update: bool = False,
                 index_bits: int = 64, num_cores: int = 3, fp32_cores: bool = False,
-                prefix_reuse: bool = True, aggregation: bool = True, mode: str = "sum"):
-    """Returns (ttemb_config, keep-alive table array).  mode = "sum" | "mean" (nn.EmbeddingBag).  prefix_reuse / aggregation = False set the
+                prefix_reuse: bool = True, aggregation: bool = True, mode: str = "sum",
+                dense: Sequence[bool] = ()):
+    """Returns (ttemb_config, keep-alive table array).  mode = "sum" | "mean" (nn.EmbeddingBag);
+    dense[t] keeps table t uncompressed (hybrid placement).  prefix_reuse / aggregation = False set the
     ablation flags TTEMB_NO_PREFIX_REUSE / TTEMB_NO_AGGREGATION."""
     T = len(table_rows)
     tabs = (L.ttemb_table * max(T, 1))()
     for t in range(T):
         tabs[t].num_rows = int(table_rows[t])
+        tabs[t].dense = 1 if (len(dense) and dense[t]) else 0
         for k in range(3):
             tabs[t].row_factors[k] = int(row_factors[t][k])
     cfg = L.ttemb_config()
@@ -169,9 +172,11 @@ class TTEmbeddingBag:
     def __init__(self, table_rows, row_factors, col_factors, rank, max_batch, max_nnz,
                  optimizer: str = "sgd", adagrad_eps: float = 1e-10, fused_update: bool = False,
                  index_bits: int = 64, device: int = 0, fp32_cores: bool = False,
-                 prefix_reuse: bool = True, aggregation: bool = True, mode: str = "sum"):
+                 prefix_reuse: bool = True, aggregation: bool = True, mode: str = "sum",
+                 dense: Sequence[bool] = ()):
         L.load()
         self.mode = mode
+        self.dense = [bool(dense[t]) if len(dense) else False for t in range(len(table_rows))]
         self.table_rows = [int(x) for x in table_rows]
         self.row_factors = [tuple(int(y) for y in f) for f in row_factors]
         self.col_factors = tuple(int(x) for x in col_factors)
@@ -185,7 +190,7 @@ class TTEmbeddingBag:
         self._cfg, self._tabs = make_config(table_rows, row_factors, col_factors, rank, max_batch,
                                             max_nnz, optimizer, adagrad_eps, fused_update, index_bits,
                                             fp32_cores=fp32_cores, prefix_reuse=prefix_reuse,
-                                            aggregation=aggregation, mode=mode)
+                                            aggregation=aggregation, mode=mode, dense=self.dense)
         cb, sb, gb, wb = ttemb_query_sizes(self._cfg)
         self.sizes = dict(core_bytes=cb, state_bytes=sb, grad_bytes=gb, workspace_bytes=wb)
         f32 = torch.float32
@@ -204,6 +209,7 @@ class TTEmbeddingBag:
     def from_config(cls, cfg, max_batch=None, max_nnz=None, **kw):
         B = cfg.batch if max_batch is None else max_batch
         nnz = B * cfg.num_tables * cfg.pooling if max_nnz is None else max_nnz
+        kw.setdefault("dense", getattr(cfg, "dense", ()))
         return cls(cfg.table_rows, cfg.row_factors, cfg.col_factors, cfg.rank, B, nnz, **kw)
 
     def __del__(self):
@@ -224,6 +230,8 @@ class TTEmbeddingBag:
             for k in range(3):
                 off, shape = self.layout[t][k]
                 shp = shape[:3] if k != 1 else shape
+                if self.dense[t] and k == 0:
+                    shp = shape[:2]            # hybrid: the plain table W[M][N]
                 n = int(np.prod(shp))
                 vs.append(buf[off:off + n].view(*shp))
             out.append(tuple(vs))

@@ -79,6 +79,12 @@ int validate(const ttemb_config* cfg) {
   uint64_t total = 0, buckets = 0, keys = 0;
   for (int t = 0; t < cfg->num_tables; ++t) {
     const ttemb_table& tb = cfg->tables[t];
+    if (tb.dense) {                       // hybrid placement: plain table, factors ignored
+      if (tb.num_rows < 1) return TTEMB_ERR_INVALID_ARG;
+      total += (uint64_t)tb.num_rows;
+      keys += (uint64_t)tb.num_rows;
+      continue;
+    }
     const int64_t m1 = tb.row_factors[0], m2 = tb.row_factors[1], m3 = tb.row_factors[2];
     if (tb.num_rows < 1 || m1 < 1 || m2 < 1 || m3 < 1) return TTEMB_ERR_INVALID_ARG;
     if (m1 * m2 * m3 < tb.num_rows) return TTEMB_ERR_INVALID_ARG;
@@ -105,22 +111,38 @@ void plan_sizes(const ttemb_config* cfg, Ctx& c) {
   size_t off = 0;
   uint64_t rb = 0, pfx = 0, kb = 0;
   uint32_t gb = 0;
-  for (int t = 0; t < c.T; ++t) {   // [C1 of all tables]
+  c.n_dense = 0;
+  for (int t = 0; t < c.T; ++t) {   // [C1 of all TT tables]
     const ttemb_table& tb = cfg->tables[t];
     TableMeta& m = c.meta[t];
-    m.m1 = tb.row_factors[0]; m.m2 = tb.row_factors[1]; m.m3 = tb.row_factors[2];
+    m.dense = tb.dense ? 1u : 0u;
     m.M = (uint32_t)tb.num_rows;
-    m.rowbase = rb; rb += (uint64_t)tb.num_rows;
-    m.kbase = kb; kb += (uint64_t)m.m1 * m.m2 * m.m3;
+    m.rowbase = rb; rb += (uint64_t)tb.num_rows;     // user table order (bijection layout)
+    if (m.dense) {
+      m.m1 = m.m2 = m.m3 = 1;
+      ++c.n_dense;
+      continue;
+    }
+    m.m1 = tb.row_factors[0]; m.m2 = tb.row_factors[1]; m.m3 = tb.row_factors[2];
+    m.kbase = kb; kb += (uint64_t)m.m1 * m.m2 * m.m3;   // plan keys: TT tables first
     m.grpbase = gb; gb += m.m2;
     pfx += (uint64_t)((tb.num_rows + m.m3 - 1) / m.m3);
     m.c1_off = off; off += up4(m.m1 * s1);
   }
+  c.tt_keys = kb;
+  for (int t = 0; t < c.T; ++t)                     // then the dense tables' keys
+    if (c.meta[t].dense) { c.meta[t].kbase = kb; kb += c.meta[t].M; }
   c.c1_floats = off;
-  for (int t = 0; t < c.T; ++t) { c.meta[t].c2_off = off; off += up4(c.meta[t].m2 * s2); }
+  for (int t = 0; t < c.T; ++t)
+    if (!c.meta[t].dense) { c.meta[t].c2_off = off; off += up4(c.meta[t].m2 * s2); }
   c.c3_begin = off;
-  for (int t = 0; t < c.T; ++t) { c.meta[t].c3_off = off; off += up4(c.meta[t].m3 * s3); }
+  for (int t = 0; t < c.T; ++t)
+    if (!c.meta[t].dense) { c.meta[t].c3_off = off; off += up4(c.meta[t].m3 * s3); }
   c.c3_floats = off - c.c3_begin;
+  c.dense_begin = off;                               // [W of the dense tables]
+  for (int t = 0; t < c.T; ++t)
+    if (c.meta[t].dense) { c.meta[t].c1_off = off; c.meta[t].c2_off = c.meta[t].c3_off = 0; off += up4((size_t)c.meta[t].M * c.N); }
+  c.dense_floats = off - c.dense_begin;
   c.core_floats = off;
   c.total_rows = rb;
   c.total_keys = kb;
@@ -147,6 +169,7 @@ size_t carve(Ctx& c, uint8_t* base) {
   c.d_meta = k.take<TableMeta>(c.T);
   c.d_kbase = k.take<uint64_t>(c.T + 1);
   c.d_grpbase = k.take<uint32_t>(c.T + 1);
+  c.d_kmap = k.take<uint32_t>(c.T);
   // --- zeroed every forward ---
   k.off = (k.off + 255) & ~(size_t)255;
   const size_t zb = k.off;
@@ -280,12 +303,19 @@ int ttemb_create(const ttemb_config* cfg, int device, void* cores, void* state, 
   if (cudaGetDeviceProperties(&prop, device) != cudaSuccess) { delete h; return TTEMB_ERR_CUDA; }
   c.sm_count = prop.multiProcessorCount;
   std::vector<uint64_t> rb(c.T + 1);
-  std::vector<uint32_t> gb(c.T + 1);
-  for (int t = 0; t < c.T; ++t) { rb[t] = c.meta[t].kbase; gb[t] = c.meta[t].grpbase; }
+  std::vector<uint32_t> gb(c.T + 1), km(c.T);
+  {   // key ranges in key order (TT tables, then dense tables) -> user table
+    int i = 0;
+    for (int pass = 0; pass < 2; ++pass)
+      for (int t = 0; t < c.T; ++t)
+        if ((int)c.meta[t].dense == pass) { rb[i] = c.meta[t].kbase; km[i] = (uint32_t)t; ++i; }
+  }
+  for (int t = 0; t < c.T; ++t) gb[t] = c.meta[t].grpbase;
   rb[c.T] = c.total_keys; gb[c.T] = c.total_buckets;
   cudaError_t e = cudaMemcpy(c.d_meta, c.meta.data(), sizeof(TableMeta) * c.T, cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(c.d_kbase, rb.data(), sizeof(uint64_t) * (c.T + 1), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(c.d_grpbase, gb.data(), sizeof(uint32_t) * (c.T + 1), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(c.d_kmap, km.data(), sizeof(uint32_t) * c.T, cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = configure_group(c);
   if (e == cudaSuccess) e = configure_tc(c);
   if (e == cudaSuccess) e = configure_fused(c);
@@ -313,6 +343,15 @@ int ttemb_core_layout(ttemb_t h, int table, int core, int64_t* offset_floats, in
   const TableMeta& m = c.meta[table];
   int32_t s[4];
   int64_t off;
+  if (m.dense) {   // hybrid: core 0 = W[M][N], cores 1, 2 empty
+    off = core == 0 ? (int64_t)m.c1_off : 0;
+    if (core == 0) { s[0] = (int32_t)m.M; s[1] = c.N; s[2] = 1; s[3] = 1; }
+    else if (core == 1) { s[0] = 0; s[1] = c.R; s[2] = c.n2; s[3] = c.R; }
+    else { s[0] = 0; s[1] = c.R; s[2] = c.n3; s[3] = 1; }
+    if (offset_floats) *offset_floats = off;
+    if (shape) memcpy(shape, s, sizeof(s));
+    return TTEMB_OK;
+  }
   if (core == 0) { off = m.c1_off; s[0] = m.m1; s[1] = c.n1; s[2] = c.R; s[3] = 1; }
   else if (core == 1) { off = m.c2_off; s[0] = m.m2; s[1] = c.R; s[2] = c.n2; s[3] = c.R; }
   else { off = m.c3_off; s[0] = m.m3; s[1] = c.R; s[2] = c.n3; s[3] = 1; }

@@ -239,6 +239,30 @@ cudaError_t run_group_bwd(Ctx& c, float lr, cudaStream_t s);
 int64_t agg_chunks(int64_t nnz) { return (nnz + AGG_CS - 1) / AGG_CS; }
 int64_t dc1_chunks(int64_t P) { return 1; }
 
+// Hybrid placement: dense-table rows [Utt, U) take their aggregated gradient G_u
+// directly: dW[row] = G_u (written to the gradient buffer), or -- fused, one replica -- the
+// row is updated in place (each unique row is owned by one thread per column: no races).
+__global__ void __launch_bounds__(256)
+k_dense_bwd(float* __restrict__ cores, float* __restrict__ state, float* __restrict__ grads,
+            const TableMeta* __restrict__ meta, const uint64_t* __restrict__ kbase,
+            const uint32_t* __restrict__ kmap, int T, const uint32_t* __restrict__ ukey,
+            const uint32_t* __restrict__ counts, int N, const float* __restrict__ gbuf, int fused,
+            float lr, float eps, int opt) {
+  const uint32_t U = counts[kCntU], u0 = tt_rows(counts);
+  const int64_t total = (int64_t)(U - u0) * N;
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t u = u0 + (uint32_t)(e / N);
+    const int col = (int)(e % N);
+    const uint32_t key = __ldg(ukey + u);
+    const int it = table_of_key(kbase, T, key);
+    const TableMeta& m = meta[__ldg(kmap + it)];
+    const size_t dst = m.c1_off + (size_t)(key - __ldg(kbase + it)) * N + col;
+    const float g = gbuf[(size_t)u * N + col];
+    if (fused) apply_update(cores + dst, state ? state + dst : nullptr, g, lr, eps, opt);
+    else grads[dst] = g;
+  }
+}
+
 cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s) {
   const PlanDev& p = c.p;
   const bool fused = (c.flags & TTEMB_FUSED_UPDATE) != 0;
@@ -271,6 +295,12 @@ cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s
       k_agg_fix<<<grid_for(c, agg_chunks(c.nnz) * 32, 256, 32), 256, 0, s>>>(
           p.skey, p.spos, p.inverse, p.seg_off, c.nnz, c.N, p.aggpart, p.gbuf);
     }
+  }
+  if (c.nnz > 0 && c.n_dense > 0) {   // hybrid placement: dense-table rows
+    StageScope sc(c, ST_BWD_ROWS, s);
+    k_dense_bwd<<<grid_for(c, (int64_t)c.U_cap * c.N, 256, 8), 256, 0, s>>>(
+        c.cores, c.state, c.grads, c.d_meta, c.d_kbase, c.d_kmap, c.T, p.ukey, p.counts, c.N, p.gbuf,
+        fused ? 1 : 0, lr, c.eps, c.opt);
   }
   BwdArgs a;
   a.cores = c.cores; a.grads = c.grads; a.state = c.state; a.meta = c.d_meta;

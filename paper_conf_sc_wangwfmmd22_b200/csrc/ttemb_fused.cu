@@ -367,7 +367,7 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 3) k_rows_fwd2(RowArgs a) {
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   float* const ringp = rw_smem + w * (RW_NSL * SLOT);
   const uint32_t ring = tc::smem_u32(ringp);
-  const uint32_t U = a.counts[kCntU];
+  const uint32_t U = tt_rows(a.counts);   // TT rows only (hybrid: dense rows follow)
   const int J12 = a.n1 * a.n2;
   const int jq = lane >> 3, rp = lane & 7;
   // per-lane P offsets inside a prefix block [n1][NC] for e = 0..3 (j12 = 4 jq + e)
@@ -515,7 +515,7 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 2) k_rows_bwd2(RowBwdArgs a) {
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   float* const ringp = rw_smem + w * (RW_NSL * SLOT);
   const uint32_t ring = tc::smem_u32(ringp);
-  const uint32_t U = a.counts[kCntU];
+  const uint32_t U = tt_rows(a.counts);   // TT rows only (hybrid: dense rows follow)
   const int J12 = a.n1 * a.n2;
   const int jq = lane >> 3, rp = lane & 7;
   int poff[4];

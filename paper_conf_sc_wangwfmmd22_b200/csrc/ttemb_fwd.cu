@@ -99,7 +99,33 @@ k_pool_single(const float* __restrict__ rows, const uint32_t* __restrict__ inver
   }
 }
 
+// Hybrid placement: the unique rows of dense tables, [Utt, U), are plain table rows:
+// rows[u] = W_t[row].  Thread = (row, column); coalesced along the row.
+__global__ void __launch_bounds__(256)
+k_dense_fwd(const float* __restrict__ cores, const TableMeta* __restrict__ meta,
+            const uint64_t* __restrict__ kbase, const uint32_t* __restrict__ kmap, int T,
+            const uint32_t* __restrict__ ukey, const uint32_t* __restrict__ counts, int N,
+            float* __restrict__ rows) {
+  const uint32_t U = counts[kCntU], u0 = tt_rows(counts);
+  const int64_t total = (int64_t)(U - u0) * N;
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t u = u0 + (uint32_t)(e / N);
+    const int col = (int)(e % N);
+    const uint32_t key = __ldg(ukey + u);
+    const int it = table_of_key(kbase, T, key);
+    const TableMeta& m = meta[__ldg(kmap + it)];
+    rows[(size_t)u * N + col] = __ldg(cores + m.c1_off + (size_t)(key - __ldg(kbase + it)) * N + col);
+  }
+}
+
 }  // namespace
+
+cudaError_t run_dense_fwd(Ctx& c, cudaStream_t s) {
+  StageScope sc(c, ST_FWD_ROWS, s);
+  k_dense_fwd<<<grid_for(c, (int64_t)c.U_cap * c.N, 256, 8), 256, 0, s>>>(
+      c.cores, c.d_meta, c.d_kbase, c.d_kmap, c.T, c.p.ukey, c.p.counts, c.N, c.p.rows);
+  return cudaGetLastError();
+}
 
 cudaError_t run_group_fwd(Ctx& c, cudaStream_t s);
 
@@ -108,6 +134,7 @@ cudaError_t run_forward_compute(Ctx& c, float* out, const int64_t* offsets, cuda
   const bool tc = tc_eligible(c);
   if (c.nnz > 0) {
     cudaError_t e = tc ? run_tc_fwd(c, out, s) : run_group_fwd(c, s);
+    if (e == cudaSuccess && c.n_dense > 0) e = run_dense_fwd(c, s);
     if (e != cudaSuccess) return e;
   }
   {

@@ -173,6 +173,8 @@ k_build_keys(const IdxT* __restrict__ indices, const int64_t* __restrict__ offse
         const uint32_t r = bt ? __ldg(bt + id) : (uint32_t)id;   // New_Batch = {index(i_j)}
         if (r >= M) {
           err |= kErrRange;
+        } else if (mt.dense) {                  // hybrid: plain table, key = row id
+          key = kb + r;
         } else {
           const uint32_t p = r / m3, i3 = r - p * m3, i1 = p / m2, i2 = p - i1 * m2;
           key = kb + (i2 * m1 + i1) * m3 + i3;
@@ -379,11 +381,15 @@ struct UniqueBody {
   uint32_t* ukey; uint32_t* seg_off; uint32_t* inverse; uint32_t* sbag; uint32_t* counts;
   uint32_t nnz;
   uint32_t every;   // TTEMB_NO_AGGREGATION: each occurrence is its own row
+  uint64_t tt_keys; // keys >= tt_keys are rows of dense (hybrid) tables
   __device__ uint32_t size() const { return nnz; }
   __device__ bool flag(uint32_t k) const { return every || k == 0 || skey[k] != skey[k - 1]; }
   __device__ void emit(uint32_t k, uint32_t slot, uint32_t f) const {
     const uint32_t u = f ? slot : slot - 1;
-    if (f) { ukey[u] = skey[k]; seg_off[u] = k; }
+    if (f) {
+      ukey[u] = skey[k]; seg_off[u] = k;
+      if (skey[k] >= tt_keys && (k == 0 || skey[k - 1] < tt_keys)) counts[kCntUtt1] = u + 1;
+    }
     const uint32_t pos = spos[k];
     inverse[pos] = u;
     sbag[k] = bag_of[pos];
@@ -391,31 +397,26 @@ struct UniqueBody {
   __device__ void finish(uint32_t U) const { counts[kCntU] = U; seg_off[U] = nnz; }
 };
 
-__device__ __forceinline__ int table_of_key(const uint64_t* kbase, int T, uint32_t key) {
-  int lo = 0, hi = T - 1;   // last t with kbase[t] <= key
-  while (lo < hi) {
-    const int mid = (lo + hi + 1) >> 1;
-    if (__ldg(kbase + mid) <= key) lo = mid; else hi = mid - 1;
-  }
-  return lo;
-}
 
 // a4: TT digits (Eq. 3) and unique prefixes (runs of (t, i2 m1 + i1)) over the unique rows
 struct PrefixBody {
-  const uint32_t* ukey; const uint64_t* kbase; const TableMeta* meta; int T;
+  const uint32_t* ukey; const uint64_t* kbase; const uint32_t* kmap; const TableMeta* meta; int T;
   uint32_t* row_pfx; uint32_t* row_i3; uint32_t* pfx_t; uint32_t* pfx_i1; uint32_t* pfx_i2;
   uint32_t* row_seg; uint32_t* counts;
   uint32_t every;   // TTEMB_NO_PREFIX_REUSE: each row is its own prefix
   __device__ uint32_t size() const { return counts[kCntU]; }
   __device__ void decode(uint32_t u, int& t, uint32_t& pq, uint32_t& i3) const {
     const uint32_t key = ukey[u];
-    t = table_of_key(kbase, T, key);
-    const uint32_t local = (uint32_t)(key - __ldg(kbase + t));
+    const int it = table_of_key(kbase, T, key);      // key ranges are in key order
+    t = (int)__ldg(kmap + it);
+    const uint32_t local = (uint32_t)(key - __ldg(kbase + it));
     const uint32_t m3 = meta[t].m3;
     pq = local / m3;                  // i2 * m1 + i1
     i3 = local - pq * m3;
   }
+  __device__ bool is_dense_row(uint32_t u) const { return counts[kCntUtt1] && u >= counts[kCntUtt1] - 1; }
   __device__ bool flag(uint32_t u) const {
+    if (is_dense_row(u)) return false;             // hybrid: dense rows have no prefix
     if (u == 0 || every) return true;
     int t0, t1; uint32_t p0, p1, x;
     decode(u, t1, p1, x);
@@ -423,6 +424,7 @@ struct PrefixBody {
     return t0 != t1 || p0 != p1;
   }
   __device__ void emit(uint32_t u, uint32_t slot, uint32_t f) const {
+    if (is_dense_row(u)) { row_pfx[u] = 0xFFFFFFFFu; row_i3[u] = 0; return; }
     int t; uint32_t pq, i3;
     decode(u, t, pq, i3);
     const uint32_t q = f ? slot : slot - 1;
@@ -434,7 +436,7 @@ struct PrefixBody {
       pfx_t[q] = (uint32_t)t; pfx_i1[q] = i1; pfx_i2[q] = i2; row_seg[q] = u;
     }
   }
-  __device__ void finish(uint32_t P) const { counts[kCntP] = P; row_seg[P] = counts[kCntU]; }
+  __device__ void finish(uint32_t P) const { counts[kCntP] = P; row_seg[P] = tt_rows(counts); }
 };
 
 // i2-groups: runs of (t, i2) over the prefixes (already in group-major order)
@@ -521,14 +523,14 @@ cudaError_t run_index_stage(Ctx& c, const void* indices, const int64_t* offsets,
   {
     StageScope sc(c, ST_UNIQUE, s);
     UniqueBody b{p.skey, p.spos, p.bag_of, p.ukey, p.seg_off, p.inverse, p.sbag, p.counts,
-                 (uint32_t)nnz, (c.flags & TTEMB_NO_AGGREGATION) ? 1u : 0u};
+                 (uint32_t)nnz, (c.flags & TTEMB_NO_AGGREGATION) ? 1u : 0u, c.tt_keys};
     const int64_t tiles = scan_tiles(nnz);
     k_scan<UniqueBody><<<(unsigned)(tiles ? tiles : 1), SC_T, 0, s>>>(b, p.sc_status, p.sc_counter + 0);
   }
   // a4: digits + prefixes, then i2-groups
   {
     StageScope sc(c, ST_PREFIX, s);
-    PrefixBody b{p.ukey, c.d_kbase, c.d_meta, c.T, p.row_pfx, p.row_i3, p.pfx_t, p.pfx_i1,
+    PrefixBody b{p.ukey, c.d_kbase, c.d_kmap, c.d_meta, c.T, p.row_pfx, p.row_i3, p.pfx_t, p.pfx_i1,
                  p.pfx_i2, p.row_seg, p.counts, (c.flags & TTEMB_NO_PREFIX_REUSE) ? 1u : 0u};
     const int64_t tiles = scan_tiles(c.U_cap);
     k_scan<PrefixBody><<<(unsigned)(tiles ? tiles : 1), SC_T, 0, s>>>(

@@ -24,7 +24,13 @@ constexpr uint32_t kErrRange = 1u;     // an id outside [0, M_t)
 constexpr uint32_t kErrOffsets = 2u;   // malformed offsets
 
 // counts[] slots (device)
-constexpr int kCntU = 0, kCntP = 1, kCntNG = 2, kCntErr = 3, kCntMulti = 4, kNumCounts = 16;
+constexpr int kCntU = 0, kCntP = 1, kCntNG = 2, kCntErr = 3, kCntMulti = 4, kCntUtt1 = 5, kNumCounts = 16;
+
+// Unique rows [0, Utt) belong to TT tables, [Utt, U) to dense (hybrid) tables: plan keys number
+// the TT tables first.  counts[kCntUtt1] = Utt + 1 when a dense row exists, else 0.
+__host__ __device__ inline uint32_t tt_rows(const uint32_t* counts) {
+  return counts[kCntUtt1] ? counts[kCntUtt1] - 1 : counts[kCntU];
+}
 
 // ---- stage ids for per-stage timing ----------------------------------------------
 enum Stage : int {
@@ -51,13 +57,23 @@ inline int env_int(const char* name, int dflt) {
   return e ? atoi(e) : dflt;
 }
 
+// Index of the key range holding `key` (kbase[0..T-1] ascending, in key order).
+__device__ __forceinline__ int table_of_key(const uint64_t* kbase, int T, uint32_t key) {
+  int lo = 0, hi = T - 1;   // last range with kbase[i] <= key
+  while (lo < hi) {
+    const int mid = (lo + hi + 1) >> 1;
+    if (__ldg(kbase + mid) <= key) lo = mid; else hi = mid - 1;
+  }
+  return lo;
+}
+
 struct TableMeta {
   uint32_t m1, m2, m3, M;      // row factors, rows (M <= 2^32-1 checked on host)
   uint64_t rowbase;            // exclusive prefix sum of M (row numbering across tables)
   uint64_t kbase;              // first plan key of the table: exclusive prefix sum of m1 m2 m3
   uint64_t c1_off, c2_off, c3_off;  // float offsets into cores / grads / state
-  uint32_t grpbase;            // first (t, i2) bucket id = sum of m2 of earlier tables
-  uint32_t pad;
+  uint32_t grpbase;            // first (t, i2) bucket id = sum of m2 of earlier TT tables
+  uint32_t dense;              // hybrid placement: plain table W[M][N] at c1_off
 };
 
 // Per-step plan pointers (all device).
@@ -111,6 +127,10 @@ struct Ctx {
   TableMeta* d_meta = nullptr;
   uint64_t* d_kbase = nullptr;       // [T+1] plan-key base of every table (+ total)
   uint32_t* d_grpbase = nullptr;     // [T+1]
+  uint32_t* d_kmap = nullptr;        // [T] user table of the i-th key range (d_kbase is in key order)
+  int n_dense = 0;                   // hybrid placement: number of dense tables
+  uint64_t tt_keys = 0;              // plan keys of the TT tables (dense keys follow)
+  size_t dense_begin = 0, dense_floats = 0;   // dense tables' region of cores / grads / state
   PlanDev p{};
   uint8_t* zero_begin = nullptr;
   size_t zero_bytes = 0;

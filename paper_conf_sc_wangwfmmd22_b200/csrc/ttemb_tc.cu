@@ -520,7 +520,7 @@ __global__ void __launch_bounds__(128) k_rows_fwd(TcArgs a) {
   __shared__ __align__(16) WarpSmem ws_all[4];
   WarpSmem& ws = ws_all[threadIdx.x >> 5];
   const int lane = threadIdx.x & 31, J12 = a.n1 * a.n2;
-  const uint32_t U = a.counts[kCntU];
+  const uint32_t U = tt_rows(a.counts);   // TT rows only (hybrid: dense rows follow)
   const int j12 = lane >> 1, rh = lane & 1;
   const int64_t nch = (U + RCH - 1) / RCH;
   for (int64_t ch = (int64_t)blockIdx.x * 4 + (threadIdx.x >> 5); ch < nch; ch += (int64_t)gridDim.x * 4) {
@@ -589,7 +589,7 @@ __global__ void __launch_bounds__(128) k_rows_bwd(TcArgs a) {
   __shared__ __align__(16) WarpSmem ws_all[4];
   WarpSmem& ws = ws_all[threadIdx.x >> 5];
   const int lane = threadIdx.x & 31, J12 = a.n1 * a.n2;
-  const uint32_t U = a.counts[kCntU];
+  const uint32_t U = tt_rows(a.counts);   // TT rows only (hybrid: dense rows follow)
   const int j12 = lane >> 1, rh = lane & 1;
   const int64_t nch = (U + RCH - 1) / RCH;
   for (int64_t ch = (int64_t)blockIdx.x * 4 + (threadIdx.x >> 5); ch < nch; ch += (int64_t)gridDim.x * 4) {

@@ -120,3 +120,16 @@ def test_ablation_flags_accepted_and_size_the_workspace():
     cfg.flags = 1 << 7
     v = [C.c_size_t() for _ in range(4)]
     assert L.load().ttemb_query_sizes(C.byref(cfg), *[C.byref(x) for x in v]) == L.TTEMB_ERR_INVALID_ARG
+
+
+def test_hybrid_tables_sizes_and_layout_validation():
+    """Hybrid placement (P:310): a dense table's factors are ignored and it occupies M x dim floats;
+    the core / grad buffers grow by exactly the dense tables' size (16-byte padded blocks)."""
+    c = W.config("c2")
+    h = W.hybrid(c)
+    cfg_tt, k1 = _cfg()
+    cfg_h, k2 = tt.make_config(h.table_rows, [(0, 0, 0) if d else f for d, f in zip(h.dense, h.row_factors)],
+                               h.col_factors, h.rank, h.batch, h.batch * h.num_tables, dense=h.dense)
+    core_h = tt.ttemb_query_sizes(cfg_h)[0]
+    assert W.core_bytes(h) <= core_h <= W.core_bytes(h) + 16 * 3 * h.num_tables
+    assert core_h != tt.ttemb_query_sizes(cfg_tt)[0]

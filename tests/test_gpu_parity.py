@@ -23,6 +23,7 @@ DEV = torch.device("cuda", 0)
 
 
 def gpu_emb(cfg, B, nnz, **kw):
+    kw.setdefault("dense", getattr(cfg, "dense", ()))
     emb = tt.TTEmbeddingBag(cfg.table_rows, cfg.row_factors, cfg.col_factors, cfg.rank,
                             max(B, 1), max(nnz, 1), **kw)
     return emb
@@ -458,3 +459,71 @@ def test_weights_with_mean_rejected_by_the_abi():
     with pytest.raises(tt.TTEmbError):
         emb.forward(torch.as_tensor(idx, device=DEV), torch.as_tensor(off, device=DEV), cfg.batch,
                     per_sample_weights=torch.ones(len(idx), device=DEV))
+
+
+HYBRID = {
+    "small-ffma": lambda: W.hybrid(W.small_config([37, 300, 5, 1000], [(3, 4, 4), (7, 7, 7), (1, 2, 3), (10, 10, 10)],
+                                                  (2, 3, 2), 4, 24, 1, 1.05), threshold=100),
+    "tc-r64": lambda: W.hybrid(W.small_config([20000, 300, 5000, 40], [(28, 28, 26), (7, 7, 7), (18, 18, 16), (4, 4, 3)],
+                                              (4, 4, 4), 64, 96, 1, 1.05), threshold=1000),
+    "c4-hybrid-b1024": lambda: W.hybrid(W.config("c4")),
+}
+
+
+@pytest.mark.parametrize("case", list(HYBRID))
+def test_hybrid_placement(case):
+    """Hybrid placement (TTEMB table.dense): small tables are plain EmbeddingBag tables in the
+    same call.  Plan (TT-first keys, dense rows without prefix), forward, dW / dC_k vs the oracle;
+    variable bag lengths."""
+    cfg = HYBRID[case]()
+    B = 1024 if case.startswith("c4") else None
+    idx, off, B = make_inputs(cfg, "var", seed=17, batch=B)
+    cores = W.make_cores(cfg, seed=17)
+    go = W.make_grad_out(cfg, B, seed=17)
+    emb = gpu_emb(cfg, B, len(idx))
+    emb.load_cores(cores)
+    out = run_forward(emb, idx, off, B)
+    emb.backward(torch.as_tensor(go, device=DEV))
+    assert emb.check() == 0
+    orc = Oracle.from_config(cfg)
+    check_plan(emb, orc, idx, off, B)
+    assert_companion(out.cpu().numpy(), orc.forward(cores, idx, off, B),
+                     orc.forward(cores, idx, off, B, absolute=True), 1e-5, "forward")
+    g = orc.backward(cores, idx, off, B, go)
+    ga = orc.backward(cores, idx, off, B, go, absolute=True)
+    for t, mine in enumerate(emb.grad_views()):
+        for k in range(3):
+            if g[t][k].size:
+                assert_companion(mine[k].cpu().numpy(), g[t][k], ga[t][k], 1e-4, f"dC{k+1} t{t}")
+
+
+@pytest.mark.parametrize("opt", ["sgd", "adagrad"])
+def test_hybrid_fused_update(opt):
+    """Dense rows are updated in place by the backward (fused, one replica) exactly like the
+    unfused backward + ttemb_update; TT cores as before."""
+    cfg = HYBRID["tc-r64"]()
+    idx, off = W.make_batch(cfg, seed=19)
+    B = cfg.batch
+    cores = W.make_cores(cfg, seed=19)
+    go = W.make_grad_out(cfg, B, seed=19)
+    orc = Oracle.from_config(cfg)
+    g = orc.backward(cores, idx, off, B, go)
+    ga = orc.backward(cores, idx, off, B, go, absolute=True)
+    lr = 0.05
+    for fused in (True, False):
+        emb = gpu_emb(cfg, B, len(idx), optimizer=opt, fused_update=fused)
+        emb.load_cores(cores)
+        run_forward(emb, idx, off, B)
+        emb.backward(torch.as_tensor(go, device=DEV), lr=lr)
+        if not fused:
+            emb.update(lr)
+        torch.cuda.synchronize()
+        for t, (cv, sv) in enumerate(zip(emb.core_views(), emb.state_views() or [None] * cfg.num_tables)):
+            for k in range(3):
+                if not cores[t][k].size:
+                    continue
+                ref_p, ref_s = Oracle.update(opt, lr, cores[t][k], g[t][k], None)
+                assert_update_close(cv[k].cpu().numpy(), ref_p, cores[t][k], g[t][k], ga[t][k], lr,
+                                    opt, got_s=None if sv is None else sv[k].cpu().numpy(),
+                                    ref_s=ref_s, s_old=np.zeros_like(cores[t][k]),
+                                    what=f"{opt} fused={fused} t{t} C{k+1}")
