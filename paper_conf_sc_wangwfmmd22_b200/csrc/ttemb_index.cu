@@ -15,6 +15,9 @@
 //      as two more single-pass scans, so one CTA owns each C2 slice (replaces Alg. 1's
 //      flag array).
 // Everything here is integer work and bit-exact against oracle/ttemb_oracle.c.
+#include <algorithm>
+#include <stdlib.h>
+
 #include "ttemb_internal.cuh"
 
 namespace ttemb {
@@ -151,23 +154,35 @@ k_build_keys(const IdxT* __restrict__ indices, const int64_t* __restrict__ offse
   __syncthreads();
   const int64_t nbags = (int64_t)T * B;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  const int lane = threadIdx.x & 31;
   uint32_t err = 0, multi = 0;
-  for (int64_t b = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; b < nbags; b += stride) {
-    int64_t s = __ldg(offsets + b), e = __ldg(offsets + b + 1);
+  // whole warps iterate together (the digit histogram below is warp-aggregated)
+  for (int64_t b0 = (int64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31); b0 < nbags; b0 += stride) {
+    const int64_t b = b0 + lane;
+    const bool bval = b < nbags;
+    int64_t s = bval ? __ldg(offsets + b) : 0, e = bval ? __ldg(offsets + b + 1) : 0;
     if (s < 0 || e > nnz || e < s) { err |= kErrOffsets; s = 0; e = 0; }
     if (b == 0 && s != 0) err |= kErrOffsets;
     if (b == nbags - 1 && e != nnz) err |= kErrOffsets;
-    if (e - s != 1) multi = 1u;
-    const int t = (int)(b / B);
+    if (bval && e - s != 1) multi = 1u;
+    const int t = bval ? (int)(b / B) : 0;
     const int64_t bb = b - (int64_t)t * B;
     const TableMeta& mt = meta[t];
     const uint32_t kb = (uint32_t)mt.kbase, M = mt.M, m1 = mt.m1, m2 = mt.m2, m3 = mt.m3;
     const uint32_t bo = (uint32_t)(bb * T + t);
     const uint32_t* bt = bij ? bij + mt.rowbase : nullptr;   // table t's bijection
     const float wmean = e > s ? 1.0f / (float)(e - s) : 0.f; // nn.EmbeddingBag mode="mean"
-    for (int64_t j = s; j < e; ++j) {
+    const int64_t len = e - s;
+    int64_t rounds = len;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) rounds = max(rounds, __shfl_xor_sync(0xffffffffu, rounds, o));
+    for (int64_t r = 0; r < rounds; ++r) {
+      const int64_t j = s + r;
+      const bool act = r < len;
+      uint32_t key = 0xFFFFFFFFu;
+      if (act) {
       const int64_t id = (int64_t)indices[j];
-      uint32_t key = kb;
+      key = kb;
       if (id < 0 || (uint64_t)id >= M) err |= kErrRange;
       else {
         const uint32_t r = bt ? __ldg(bt + id) : (uint32_t)id;   // New_Batch = {index(i_j)}
@@ -183,7 +198,14 @@ k_build_keys(const IdxT* __restrict__ indices, const int64_t* __restrict__ offse
       keys[j] = key;
       bag_of[j] = bo;
       if (wpos) wpos[j] = psw ? __ldg(psw + j) : wmean;
-      for (int p = 0; p < passes; ++p) atomicAdd(&sh[p][(key >> (8 * p)) & 255u], 1u);
+      }
+      // digit histograms: one shared-memory atomic per distinct digit per warp (Zipf-hot keys
+      // share their high digits, so per-key atomics would serialise)
+      for (int p = 0; p < passes; ++p) {
+        const uint32_t d = act ? ((key >> (8 * p)) & 255u) : 256u;
+        const uint32_t peers = __match_any_sync(0xffffffffu, d);
+        if (d < 256 && (__ffs(peers) - 1) == lane) atomicAdd(&sh[p][d], __popc(peers));
+      }
     }
   }
   if (nbags == 0 && nnz != 0 && blockIdx.x == 0 && threadIdx.x == 0) err |= kErrOffsets;
@@ -198,8 +220,11 @@ k_build_keys(const IdxT* __restrict__ indices, const int64_t* __restrict__ offse
 
 // ------------------------------------------------------------------------------------
 // a2: onesweep LSD radix sort, 8-bit digits
+#ifndef TTEMB_RS_IPT
+#define TTEMB_RS_IPT 8    // keys per thread (tile = 256 x RS_IPT; 8 beats 16 and 4 at C4)
+#endif
 // ------------------------------------------------------------------------------------
-constexpr int RS_T = 256, RS_IPT = 16, RS_WARPS = RS_T / 32, RS_TILE = RS_T * RS_IPT;
+constexpr int RS_T = 256, RS_IPT = TTEMB_RS_IPT, RS_WARPS = RS_T / 32, RS_TILE = RS_T * RS_IPT;
 
 // Digit histograms of all passes in one read of the keys.
 __global__ void __launch_bounds__(256)
@@ -454,6 +479,145 @@ struct GroupBody {
   __device__ void finish(uint32_t NG) const { counts[kCntNG] = NG; grp_off[NG] = counts[kCntP]; }
 };
 
+// a3 + a4 in ONE pass over the sorted occurrences (replaces the three scans above on the default
+// path): position k starts a unique row (key change), a unique prefix (change of (t, i2 m1 + i1)
+// on a TT row) and an i2-group (change of (t, i2)).  Three flag ballots, three warp-count
+// scans and three decoupled look-backs (warps 0-2 in parallel) give every position its row
+// slot u, prefix slot q and group slot g; the emits write the same arrays the three scans did.
+struct PlanScanArgs {
+  const uint32_t *skey, *spos, *bag_of;
+  const uint64_t* kbase; const uint32_t* kmap; const TableMeta* meta; int T;
+  uint32_t *ukey, *seg_off, *inverse, *sbag, *counts;
+  uint32_t *row_pfx, *row_i3, *pfx_t, *pfx_i1, *pfx_i2, *row_seg;
+  uint32_t *grp_pfx, *grp_off, *grp_t, *grp_i2;
+  uint32_t nnz, every_row, every_pfx;
+  uint64_t tt_keys;
+};
+
+struct KeyInfo { uint32_t t, pq, i3, dense; };
+
+__device__ __forceinline__ KeyInfo decode_key(const PlanScanArgs& a, uint32_t key) {
+  KeyInfo r;
+  const int it = table_of_key(a.kbase, a.T, key);
+  r.t = __ldg(a.kmap + it);
+  const uint32_t local = (uint32_t)(key - __ldg(a.kbase + it));
+  r.dense = key >= a.tt_keys ? 1u : 0u;
+  const uint32_t m3 = r.dense ? 1u : a.meta[r.t].m3;
+  r.pq = local / m3;
+  r.i3 = local - r.pq * m3;
+  return r;
+}
+
+__global__ void __launch_bounds__(SC_T) k_plan_scan(PlanScanArgs a, uint32_t* status, uint32_t* counter) {
+  __shared__ uint32_t s_wc[3][SC_IPT * 8];
+  __shared__ uint32_t s_tile, s_base[3], s_total[3];
+  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  if (tid == 0) s_tile = atomicAdd(counter, 1u);
+  __syncthreads();
+  const uint32_t n = a.nnz;
+  const uint32_t tile = s_tile, base = tile * SC_TILE;
+  if (n == 0) {
+    if (tile == 0 && tid == 0) {
+      a.counts[kCntU] = 0; a.seg_off[0] = 0; a.counts[kCntP] = 0; a.row_seg[0] = 0;
+      a.counts[kCntNG] = 0; a.grp_off[0] = 0;
+    }
+    return;
+  }
+  if (base >= n) return;
+  uint32_t bal[3][SC_IPT];
+  KeyInfo ki[SC_IPT];
+#pragma unroll
+  for (int k = 0; k < SC_IPT; ++k) {
+    const uint32_t i = base + k * SC_T + tid;
+    bool fr = false, fp = false, fg = false;
+    ki[k] = KeyInfo{0, 0, 0, 1};
+    if (i < n) {
+      const uint32_t key = a.skey[i];
+      ki[k] = decode_key(a, key);
+      const bool newkey = i == 0 || a.skey[i - 1] != key;
+      fr = a.every_row || newkey;
+      if (fr && !ki[k].dense) {
+        if (i == 0) {
+          fp = fg = true;
+        } else {
+          const KeyInfo pv = newkey ? decode_key(a, a.skey[i - 1]) : ki[k];
+          const bool newgrp = pv.dense || pv.t != ki[k].t || pv.pq / a.meta[pv.t].m1 != ki[k].pq / a.meta[ki[k].t].m1;
+          fp = a.every_pfx || newgrp || pv.pq != ki[k].pq;
+          fg = newgrp;
+        }
+      }
+    }
+    bal[0][k] = __ballot_sync(FULL, fr);
+    bal[1][k] = __ballot_sync(FULL, fp);
+    bal[2][k] = __ballot_sync(FULL, fg);
+    if (lane == 0) {
+      s_wc[0][k * 8 + w] = __popc(bal[0][k]);
+      s_wc[1][k * 8 + w] = __popc(bal[1][k]);
+      s_wc[2][k * 8 + w] = __popc(bal[2][k]);
+    }
+  }
+  __syncthreads();
+  if (w < 3) {   // exclusive scan of the 64 warp counts (k-major) of flag w, then its look-back
+    const uint32_t x0 = s_wc[w][2 * lane], x1 = s_wc[w][2 * lane + 1];
+    uint32_t x = x0 + x1;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(FULL, x, o);
+      if (lane >= o) x += y;
+    }
+    const uint32_t ex = x - x0 - x1;
+    s_wc[w][2 * lane] = ex;
+    s_wc[w][2 * lane + 1] = ex + x0;
+    const uint32_t tot = __shfl_sync(FULL, x, 31);
+    const uint32_t b = lookback_warp(status + (size_t)w * gridDim.x, tile, tot);
+    if (lane == 0) { s_base[w] = b; s_total[w] = tot; }
+  }
+  __syncthreads();
+  const uint32_t lt = lanemask_lt();
+#pragma unroll
+  for (int k = 0; k < SC_IPT; ++k) {
+    const uint32_t i = base + k * SC_T + tid;
+    if (i >= n) continue;
+    // inclusive counts - 1 = this position's row / prefix / group slot
+    const uint32_t u = s_base[0] + s_wc[0][k * 8 + w] + __popc(bal[0][k] & lt) + ((bal[0][k] >> lane) & 1u) - 1u;
+    const uint32_t q = s_base[1] + s_wc[1][k * 8 + w] + __popc(bal[1][k] & lt) + ((bal[1][k] >> lane) & 1u) - 1u;
+    const uint32_t g = s_base[2] + s_wc[2][k * 8 + w] + __popc(bal[2][k] & lt) + ((bal[2][k] >> lane) & 1u) - 1u;
+    const uint32_t pos = a.spos[i];
+    a.inverse[pos] = u;
+    a.sbag[i] = __ldg(a.bag_of + pos);
+    if ((bal[0][k] >> lane) & 1u) {
+      const uint32_t key = a.skey[i];
+      a.ukey[u] = key;
+      a.seg_off[u] = i;
+      if (ki[k].dense) {
+        a.row_pfx[u] = 0xFFFFFFFFu;
+        a.row_i3[u] = 0;
+        if (i == 0 || a.skey[i - 1] < a.tt_keys) {   // first dense row: TT rows / prefixes end here
+          a.counts[kCntUtt1] = u + 1;
+          a.row_seg[q + 1] = u;
+        }
+      } else {
+        a.row_pfx[u] = q;
+        a.row_i3[u] = ki[k].i3;
+      }
+    }
+    if ((bal[1][k] >> lane) & 1u) {
+      const uint32_t m1 = a.meta[ki[k].t].m1;
+      const uint32_t i2 = ki[k].pq / m1;
+      a.pfx_t[q] = ki[k].t; a.pfx_i1[q] = ki[k].pq - i2 * m1; a.pfx_i2[q] = i2;
+      a.row_seg[q] = u;
+      a.grp_pfx[q] = q;
+      if ((bal[2][k] >> lane) & 1u) { a.grp_off[g] = q; a.grp_t[g] = ki[k].t; a.grp_i2[g] = i2; }
+    }
+  }
+  if (base + SC_TILE >= n && tid == 0) {
+    const uint32_t U = s_base[0] + s_total[0], P = s_base[1] + s_total[1], NG = s_base[2] + s_total[2];
+    a.counts[kCntU] = U; a.seg_off[U] = n;
+    a.counts[kCntP] = P; a.counts[kCntNG] = NG; a.grp_off[NG] = P;
+    if (a.skey[n - 1] < a.tt_keys) a.row_seg[P] = U;   // no dense rows (else written above)
+  }
+}
+
 // Host: full LSD sort; returns which buffer pair holds the result (0 = A, 1 = B).
 int radix_sort(Ctx& c, uint32_t* kA, uint32_t* vA, uint32_t* kB, uint32_t* vB,
                const uint32_t* n_dev, uint32_t n_static, int64_t n_max, int passes,
@@ -519,6 +683,21 @@ cudaError_t run_index_stage(Ctx& c, const void* indices, const int64_t* offsets,
                                ST_SORT_HIST, ST_SORT_PASS, s, /*have_hist=*/true);
   p.skey = which ? p.keysB : p.keysA;
   p.spos = which ? p.valsB : p.valsA;
+  if (!getenv("TTEMB_THREE_SCANS")) {   // a3 + a4 fused (default)
+    StageScope sc(c, ST_UNIQUE, s);
+    PlanScanArgs a;
+    a.skey = p.skey; a.spos = p.spos; a.bag_of = p.bag_of; a.kbase = c.d_kbase; a.kmap = c.d_kmap;
+    a.meta = c.d_meta; a.T = c.T; a.ukey = p.ukey; a.seg_off = p.seg_off; a.inverse = p.inverse;
+    a.sbag = p.sbag; a.counts = p.counts; a.row_pfx = p.row_pfx; a.row_i3 = p.row_i3; a.pfx_t = p.pfx_t;
+    a.pfx_i1 = p.pfx_i1; a.pfx_i2 = p.pfx_i2; a.row_seg = p.row_seg; a.grp_pfx = p.grp_pfx;
+    a.grp_off = p.grp_off; a.grp_t = p.grp_t; a.grp_i2 = p.grp_i2; a.nnz = (uint32_t)nnz;
+    a.every_row = (c.flags & TTEMB_NO_AGGREGATION) ? 1u : 0u;
+    a.every_pfx = (c.flags & TTEMB_NO_PREFIX_REUSE) ? 1u : 0u;
+    a.tt_keys = c.tt_keys;
+    const int64_t tiles = std::max<int64_t>(1, scan_tiles(nnz));
+    k_plan_scan<<<(unsigned)tiles, SC_T, 0, s>>>(a, p.sc_status, p.sc_counter + 0);
+    return cudaGetLastError();
+  }
   // a3
   {
     StageScope sc(c, ST_UNIQUE, s);
