@@ -1,6 +1,6 @@
 # ablation switches + the paper-design comparator on the bench workload (c4), one GPU.
 mkdir -p gpurun_out/abl
-timeout 900 python -m pytest tests -m gpu -q --timeout 300 -p no:cacheprovider -x > gpurun_out/abl/pytest_gpu.log 2>&1; tail -3 gpurun_out/abl/pytest_gpu.log
+[ -n "$ABL_TESTS" ] && timeout 900 python -m pytest tests -m gpu -q --timeout 300 -p no:cacheprovider -x > gpurun_out/abl/pytest_gpu.log 2>&1
 B="python bench.py --steps 10 --warmup 3 --no-e2e --no-cpu-baseline"
 for cfgn in ${ABL_CONFIGS:-c4 c3}; do
   timeout 300 $B --config $cfgn > gpurun_out/abl/$cfgn-base.json 2> gpurun_out/abl/$cfgn-base.err

@@ -12,7 +12,8 @@ PAPER = {"no_reuse": "1.75x lookup from reuse (Fig. 17); -10 % throughput (Fig. 
          "unfused": "1.15x backward from the fused update (Fig. 18)",
          "perm": "index reordering: 1.05x lookup, 1.06x backward, -13 % throughput",
          "perm_bij": "(runtime bijection restores part of the reordering gain)",
-         "paper": "the paper's design: Alg. 1 reuse + cuBLAS batched GEMM (P:346)"}
+         "paper": "the paper's design: Alg. 1 reuse + cuBLAS batched GEMM (P:346)",
+         "hybrid": "hybrid placement (P:310): tables <= 1M rows kept dense (speed-up, not a slowdown)"}
 lines = [f"# {tag}: optimisation breakdown on B200 (scripts/ablation.sh)", "",
          "One B200, `bench.py --steps 10 --warmup 3` (CUDA-graph replay, L2 flushed between steps); "
          "`--impl paper` = comparators/paper_design.py (torch + cuBLAS fp32, eager), 5 steps.",
@@ -27,7 +28,7 @@ for cfg in ("c4", "c3", "c2"):
     lines += [f"## {cfg} ({base['config']['workload']})", "",
               "| variant | ms/step | lookups/s | slowdown vs ours | U | P | paper's figure |",
               "|---|---|---|---|---|---|---|"]
-    for v in ("base", "no_reuse", "no_agg", "unfused", "perm", "perm_bij", "paper"):
+    for v in ("base", "no_reuse", "no_agg", "unfused", "perm", "perm_bij", "paper", "hybrid"):
         p = os.path.join(ABL, f"{cfg}-{v}.json")
         if not os.path.exists(p):
             continue
