@@ -296,12 +296,11 @@ def workload_config(cfg, B, world, args):
 # ---------------------------------------------------------------------------
 def kernels_per_step(emb_ctx, world, fused=True, cfg=None, fused_update=None):
     """Our kernel launches per step (cudaMemsetAsync excluded), matching the ncu launch list.
-    tcgen05 path: index stage = build_keys + hist_scan + kp radix passes + unique / prefix /
-    group scans; forward = prep + prefix GEMM + rows + pool (single + multi, one exits early);
+    tcgen05 path: index stage = build_keys + hist_scan + kp radix passes + the fused plan scan; forward = prep + prefix GEMM + rows + pool (single + multi, one exits early);
     backward = zero_rows + agg + dp_zero + rows_bwd + prefix GEMM bwd (+ 2 dense C1/C3 updates
     when fused, + 1 update after the all-reduce otherwise)."""
     kp, _ = emb_ctx
-    idx_stage = 1 + 1 + kp + 3
+    idx_stage = 1 + 1 + kp + 1          # build_keys, hist_scan, kp radix passes, fused plan scan
     if fused_update is None:
         fused_update = world == 1
     if fused:
