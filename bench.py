@@ -192,6 +192,8 @@ def cpu_baseline(cfg, cores, idx, off, B, go, lr, opt, target_s=15.0):
 def run_reference(args, cfg, rank, world):
     if rank != 0:
         return
+    # torchrun pins OMP_NUM_THREADS=1 per rank; rank 0 runs the oracle alone on the host cores
+    os.environ["OMP_NUM_THREADS"] = str(os.cpu_count() or 1)
     import oracle
     B = cfg.batch if args.scaling == "weak" else cfg.batch // world
     cores = W.make_cores(cfg, seed=args.seed)
@@ -372,10 +374,18 @@ def main():
     import paper_conf_sc_wangwfmmd22_b200 as tt
     from paper_conf_sc_wangwfmmd22_b200 import parallel
 
+    # one rank per GPU; on a box with fewer GPUs than ranks (a functional check of the N > 1
+    # path only) ranks share devices and the all-reduce falls back to gloo
+    ndev = torch.cuda.device_count()
+    shared = world > ndev
+    local_rank = local_rank % ndev
     torch.cuda.set_device(local_rank)
     dev = torch.device("cuda", local_rank)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if shared:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
     B = cfg.batch if args.scaling == "weak" else cfg.batch // world
     fused = world == 1 and not args.unfused
 

@@ -533,9 +533,10 @@ __global__ void __launch_bounds__(SC_T) k_plan_scan(PlanScanArgs a, uint32_t* st
     ki[k] = KeyInfo{0, 0, 0, 1};
     if (i < n) {
       const uint32_t key = a.skey[i];
-      ki[k] = decode_key(a, key);
       const bool newkey = i == 0 || a.skey[i - 1] != key;
       fr = a.every_row || newkey;
+      ki[k].dense = key >= a.tt_keys ? 1u : 0u;
+      if (fr) ki[k] = decode_key(a, key);          // digits are needed at row starts only
       if (fr && !ki[k].dense) {
         if (i == 0) {
           fp = fg = true;
