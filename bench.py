@@ -344,6 +344,8 @@ def main():
                          "history batches of the stream, applied at run time (P:269)")
     ap.add_argument("--hybrid", action="store_true",
                     help="f3: hybrid placement -- tables with <= 1M rows stay dense (P:310)")
+    ap.add_argument("--no-pipeline", dest="pipeline", action="store_false",
+                    help="no cross-step pipelining of the next batch's index stage")
     ap.add_argument("--no-graph", dest="graph", action="store_false",
                     help="launch every step eagerly instead of replaying a captured CUDA graph")
     args = ap.parse_args()
@@ -430,8 +432,43 @@ def main():
         if not fused:
             emb.update(args.lr)
 
+    # ---- cross-step pipelining (default): the index stage of batch g+1 (ttemb_plan_batch, reads no
+    #      parameters) runs on a side stream while batch g's forward compute + backward + update run;
+    #      two handles on the same cores / grads alternate so each keeps its own plan.  Every timed
+    #      step = one batch's compute + the next batch's index stage, joined at the step's end. ----
+    pipe = args.pipeline and len(dpool) % 2 == 0
+    if pipe:
+        embs = [emb, emb.sibling()]
+        side = torch.cuda.Stream(device=dev)
+        ev_go = [torch.cuda.Event() for _ in range(len(dpool))]
+        ev_planned = [torch.cuda.Event() for _ in range(len(dpool))]
+        gstate = {"g": 0}
+
+        def pstep(g):
+            cur = torch.cuda.current_stream()
+            h, nh = embs[g % 2], embs[(g + 1) % 2]
+            _, _, dg = dpool[g % len(dpool)]
+            ni, no, _ = dpool[(g + 1) % len(dpool)]
+            e_go, e_pl = ev_go[g % len(dpool)], ev_planned[g % len(dpool)]
+            e_go.record(cur)                 # nh's previous step (g-1) is queued before this point
+            h.forward_planned(out)
+            side.wait_event(e_go)
+            nh.plan_batch(ni, no, B, stream=side)
+            e_pl.record(side)
+            h.backward(dg, lr=args.lr)
+            if world > 1:
+                parallel.allreduce_grads(h.grads)
+            if not fused:
+                h.update(args.lr)
+            cur.wait_event(e_pl)
+
+        embs[0].plan_batch(dpool[0][0], dpool[0][1], B)
+
+        def step_pipe(_i):
+            pstep(gstate["g"])
+            gstate["g"] += 1
     for i in range(args.warmup):
-        step(i)
+        step_pipe(i) if pipe else step(i)
     torch.cuda.synchronize()
     assert emb.check() == 0, "device-side input error"
 
@@ -440,10 +477,11 @@ def main():
     if args.graph and world == 1:
         torch.cuda.synchronize()
         graphs = []
+        g0 = gstate["g"] if pipe else 0
         for i in range(len(dpool)):
             g = torch.cuda.CUDAGraph()
             with torch.cuda.graph(g):
-                step(i)
+                pstep(g0 + i) if pipe else step(i)
             graphs.append(g)
         for i in range(len(graphs)):
             graphs[i].replay()
@@ -453,6 +491,8 @@ def main():
     def run(i):
         if graphs is not None:
             graphs[i % len(graphs)].replay()
+        elif pipe:
+            step_pipe(i)
         else:
             step(i)
 
@@ -593,6 +633,7 @@ def main():
                 "gpu_launches": kernels_per_step(emb_passes(emb), world, fused=tc_path(cfg, args),
                                                  fused_update=fused) * args.steps,
                 "graph": bool(graphs is not None),
+                "pipeline": "next batch's index stage on a side stream" if pipe else None,
                 "clocks": clk.summary(),
                 "stages_us_per_step": {k: round(v[0] / args.steps * 1e3, 2) for k, v in stages.items() if v[1]}}
         print(json.dumps(line), flush=True)

@@ -176,6 +176,20 @@ typedef struct {
 
 int ttemb_get_plan(ttemb_t h, ttemb_plan* plan);
 
+/* The forward in two halves, so that the index stage of the NEXT batch (a1-a4: key build, sort,
+ * unique rows / prefixes / groups -- it reads no parameters) can run on another stream while the
+ * current batch's forward compute / backward / update run (cross-step pipelining).
+ * ttemb_plan_batch: the index stage for (indices, offsets[, per_sample_weights]) into this handle's
+ * workspace (same arguments and errors as ttemb_forward_weighted minus `out`); `offsets` must stay
+ * valid until ttemb_forward_planned.  ttemb_forward_planned: the contractions + pooling of the
+ * planned batch (TTEMB_ERR_STATE without a preceding ttemb_plan_batch).  ttemb_forward = both.
+ * To pipeline, create two handles on the SAME cores / state / grads buffers (each with its own
+ * workspace) and alternate them; order the streams so that a handle's plan starts after its
+ * previous backward and the forward after its plan. */
+int ttemb_plan_batch(ttemb_t h, const void* indices, const int64_t* offsets, const float* per_sample_weights,
+               int64_t nnz, int32_t batch, void* stream);
+int ttemb_forward_planned(ttemb_t h, float* out, void* stream);
+
 /* ttemb_forward with per-sample weights (nn.EmbeddingBag(mode="sum") per_sample_weights):
  * out[b][t] = sum_j w[j] W_t[idx_j]; `per_sample_weights` is a DEVICE float array [nnz]
  * aligned with `indices` (NULL = all ones, i.e. ttemb_forward).  The weights are copied into

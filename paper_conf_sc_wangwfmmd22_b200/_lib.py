@@ -31,7 +31,8 @@ SYMBOLS = ["ttemb_query_sizes", "ttemb_create", "ttemb_destroy", "ttemb_core_lay
            "ttemb_forward", "ttemb_backward", "ttemb_update", "ttemb_forward_host",
            "ttemb_backward_host", "ttemb_check", "ttemb_get_plan", "ttemb_read_counts",
            "ttemb_set_timing", "ttemb_stage_times", "ttemb_stage_name", "ttemb_status_string",
-           "ttemb_set_bijection", "ttemb_total_rows", "ttemb_forward_weighted"]
+           "ttemb_set_bijection", "ttemb_total_rows", "ttemb_forward_weighted", "ttemb_plan_batch",
+           "ttemb_forward_planned"]
 
 
 class ttemb_table(C.Structure):
@@ -97,6 +98,8 @@ def load(path: str = LIB_PATH):
     lib.ttemb_status_string.restype = C.c_char_p
     lib.ttemb_set_bijection.argtypes = [vp, vp]
     lib.ttemb_forward_weighted.argtypes = [vp, vp, vp, vp, i64, i32, vp, vp]
+    lib.ttemb_plan_batch.argtypes = [vp, vp, vp, vp, i64, i32, vp]
+    lib.ttemb_forward_planned.argtypes = [vp, vp, vp]
     lib.ttemb_total_rows.argtypes = [vp]
     for s in SYMBOLS:
         f = getattr(lib, s)

@@ -97,6 +97,15 @@ def ttemb_forward_weighted(h: int, indices: int, offsets: int, per_sample_weight
                                            int(batch), out, stream)
 
 
+def ttemb_plan_batch(h: int, indices: int, offsets: int, per_sample_weights: int, nnz: int, batch: int,
+               stream: int) -> int:
+    return L.load().ttemb_plan_batch(h, indices, offsets, per_sample_weights or None, int(nnz), int(batch), stream)
+
+
+def ttemb_forward_planned(h: int, out: int, stream: int) -> int:
+    return L.load().ttemb_forward_planned(h, out, stream)
+
+
 def ttemb_backward(h: int, grad_out: int, lr: float, stream: int) -> int:
     return L.load().ttemb_backward(h, grad_out, float(lr), stream)
 
@@ -271,6 +280,37 @@ class TTEmbeddingBag:
                                     nnz, batch, out.data_ptr() if out.numel() else None, _stream_ptr(stream))
         check(rc, "ttemb_forward")
         self.batch, self.nnz = batch, nnz
+        return out
+
+    # -- cross-step pipelining: the index stage of the next batch on another stream ----------
+    def sibling(self) -> "TTEmbeddingBag":
+        """A second handle on the SAME cores / state / grads with its own workspace (plan), for
+        running the next batch's index stage while this one computes (ttemb_plan_batch)."""
+        other = object.__new__(TTEmbeddingBag)
+        other.__dict__.update({k: v for k, v in self.__dict__.items() if k not in ("h", "workspace", "_bij")})
+        other.workspace = torch.empty_like(self.workspace)
+        other.h = ttemb_create(self._cfg, self.device.index, self.cores.data_ptr(),
+                               self.state.data_ptr() if self.state is not None else 0,
+                               self.grads.data_ptr(), other.workspace.data_ptr())
+        if getattr(self, "_bij", None) is not None:
+            other.set_bijection(self._bij)
+        return other
+
+    def plan_batch(self, indices: torch.Tensor, offsets: torch.Tensor, batch: int, stream=None,
+                   per_sample_weights: Optional[torch.Tensor] = None) -> None:
+        """Index stage only (ttemb_plan_batch); `offsets` must stay alive until forward_planned.
+        (`plan()` returns a copy of the last plan's arrays.)"""
+        nnz = indices.numel()
+        psw = per_sample_weights.data_ptr() if (per_sample_weights is not None and nnz) else 0
+        check(ttemb_plan_batch(self.h, indices.data_ptr() if nnz else None, offsets.data_ptr(), psw, nnz, batch,
+                         _stream_ptr(stream)), "ttemb_plan_batch")
+        self.batch, self.nnz = batch, nnz
+
+    def forward_planned(self, out: Optional[torch.Tensor] = None, stream=None) -> torch.Tensor:
+        if out is None:
+            out = torch.empty(self.batch, self.T, self.N, dtype=torch.float32, device=self.device)
+        check(ttemb_forward_planned(self.h, out.data_ptr() if out.numel() else None, _stream_ptr(stream)),
+              "ttemb_forward_planned")
         return out
 
     def backward(self, grad_out: torch.Tensor, lr: float = 0.0, stream=None) -> None:

@@ -369,25 +369,50 @@ int ttemb_forward_weighted(ttemb_t h, const void* indices, const int64_t* offset
                            const float* per_sample_weights, int64_t nnz, int32_t batch, float* out,
                            void* stream) {
   if (!h) return TTEMB_ERR_INVALID_ARG;
+  if (!out && batch > 0) return TTEMB_ERR_INVALID_ARG;
+  const int rc = ttemb_plan_batch(h, indices, offsets, per_sample_weights, nnz, batch, stream);
+  if (rc) return rc;
+  return ttemb_forward_planned(h, out, stream);
+}
+
+int ttemb_plan_batch(ttemb_t h, const void* indices, const int64_t* offsets, const float* per_sample_weights,
+               int64_t nnz, int32_t batch, void* stream) {
+  if (!h) return TTEMB_ERR_INVALID_ARG;
   Ctx& c = h->c;
   if (per_sample_weights && (c.flags & TTEMB_MEAN_POOLING)) return TTEMB_ERR_INVALID_ARG;
-  c.psw = nnz > 0 ? per_sample_weights : nullptr;
-  c.weighted = c.psw != nullptr || (c.flags & TTEMB_MEAN_POOLING) != 0;
-  if (nnz < 0 || batch < 0 || !offsets || (nnz > 0 && !indices) || (!out && batch > 0))
-    return TTEMB_ERR_INVALID_ARG;
+  if (nnz < 0 || batch < 0 || !offsets || (nnz > 0 && !indices)) return TTEMB_ERR_INVALID_ARG;
   if (nnz > c.max_nnz || batch > c.max_batch) return TTEMB_ERR_CAPACITY;
   if (batch == 0 && nnz != 0) return TTEMB_ERR_INVALID_ARG;
+  c.psw = nnz > 0 ? per_sample_weights : nullptr;
+  c.weighted = c.psw != nullptr || (c.flags & TTEMB_MEAN_POOLING) != 0;
   DeviceGuard dg(c.device);
   cudaStream_t s = (cudaStream_t)stream;
   c.nnz = nnz;
   c.B = batch;
+  c.offsets = offsets;
   c.fwd_done = false;
+  c.planned = false;
   cudaError_t e = run_index_stage(c, indices, offsets, s);
-  if (e == cudaSuccess) e = run_forward_compute(c, out, offsets, s);
+  if (e != cudaSuccess) {
+    fprintf(stderr, "ttemb_plan_batch: %s\n", cudaGetErrorString(e));
+    return TTEMB_ERR_CUDA;
+  }
+  c.planned = true;
+  return TTEMB_OK;
+}
+
+int ttemb_forward_planned(ttemb_t h, float* out, void* stream) {
+  if (!h) return TTEMB_ERR_INVALID_ARG;
+  Ctx& c = h->c;
+  if (!c.planned) return TTEMB_ERR_STATE;
+  if (!out && c.B > 0) return TTEMB_ERR_INVALID_ARG;
+  DeviceGuard dg(c.device);
+  cudaError_t e = run_forward_compute(c, out, c.offsets, (cudaStream_t)stream);
   if (e != cudaSuccess) {
     fprintf(stderr, "ttemb_forward: %s\n", cudaGetErrorString(e));
     return TTEMB_ERR_CUDA;
   }
+  c.planned = false;
   c.fwd_done = true;
   return TTEMB_OK;
 }

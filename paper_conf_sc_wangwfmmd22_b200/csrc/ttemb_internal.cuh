@@ -144,6 +144,8 @@ struct Ctx {
   int64_t nnz = 0;
   int32_t B = 0;
   bool fwd_done = false;
+  bool planned = false;              // ttemb_plan ran; ttemb_forward_planned may follow
+  const int64_t* offsets = nullptr;  // the planned batch's offsets (device; caller keeps alive)
   const float* psw = nullptr;        // per-sample weights of the current forward (device) or null
   bool weighted = false;             // this step's bags carry weights (psw or mean): p.wpos valid
 

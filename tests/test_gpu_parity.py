@@ -527,3 +527,50 @@ def test_hybrid_fused_update(opt):
                                     opt, got_s=None if sv is None else sv[k].cpu().numpy(),
                                     ref_s=ref_s, s_old=np.zeros_like(cores[t][k]),
                                     what=f"{opt} fused={fused} t{t} C{k+1}")
+
+
+@pytest.mark.parametrize("case", ["c1", "tc-r64"])
+def test_pipelined_plan_on_side_stream(case):
+    """ttemb_plan_batch / ttemb_forward_planned with two handles on the same cores (the bench's
+    cross-step pipelining): batch s+1's index stage runs on a side stream during batch s's
+    forward + fused SGD backward; three steps follow the oracle's trajectory and the plans match."""
+    if case == "c1":
+        cfg = W.small_config([1000], [(10, 10, 10)], (2, 2, 4), 8, 64, 1, 1.05)
+    else:
+        cfg = W.small_config([20000, 300], [(28, 28, 26), (7, 7, 7)], (4, 4, 4), 64, 96, 1, 1.05)
+    B = cfg.batch
+    cores = W.make_cores(cfg, seed=6)
+    emb = gpu_emb(cfg, B, B * cfg.num_tables, fused_update=True)
+    emb.load_cores(cores)
+    embs = [emb, emb.sibling()]
+    orc = Oracle.from_config(cfg)
+    lr = 0.1
+    batches = [W.make_batch(cfg, step=s, seed=6) for s in range(4)]
+    gos = [W.make_grad_out(cfg, B, step=s, seed=6) for s in range(4)]
+    dev = [(torch.as_tensor(i, device=DEV), torch.as_tensor(o, device=DEV)) for i, o in batches]
+    side = torch.cuda.Stream()
+    cur = torch.cuda.current_stream()
+    embs[0].plan_batch(dev[0][0], dev[0][1], B)
+    ref = [tuple(x.copy() for x in c) for c in cores]
+    outs = []
+    for s in range(3):
+        h, nh = embs[s % 2], embs[(s + 1) % 2]
+        go_ = cur.record_event()
+        out = h.forward_planned()
+        side.wait_event(go_)
+        nh.plan_batch(dev[s + 1][0], dev[s + 1][1], B, stream=side)
+        pl = side.record_event()
+        h.backward(torch.as_tensor(gos[s], device=DEV), lr=lr)
+        cur.wait_event(pl)
+        outs.append(out.cpu().numpy())
+        idx, off = batches[s]
+        assert_companion(outs[-1], orc.forward(ref, idx, off, B), orc.forward(ref, idx, off, B, absolute=True),
+                         1e-4, f"forward step {s}")
+        g = orc.backward(ref, idx, off, B, gos[s])
+        ref = [tuple(Oracle.update("sgd", lr, c[k], g[t][k])[0] for k in range(3)) for t, c in enumerate(ref)]
+    torch.cuda.synchronize()
+    for cv, rc in zip(emb.core_views(), ref):
+        for k in range(3):
+            np.testing.assert_allclose(cv[k].cpu().numpy(), rc[k], rtol=1e-4, atol=1e-5)
+    with pytest.raises(tt.TTEmbError):            # forward_planned needs a fresh plan
+        embs[0].forward_planned()
