@@ -41,12 +41,11 @@ constexpr uint32_t Y_B1 = 2u * YR * YT * 4;     // C1^T hi + lo (CM(r1, m)), 32 
 constexpr uint32_t Y_A2LBO = 16 * 128 + 16;    // CM(128 rows, 64 c); +16 B per core column keeps
                                                 // the column-wise dP^T extraction conflict-free
 constexpr uint32_t Y_A2 = 16 * Y_A2LBO;         // [dP_hi; dP_lo] chunk (~32 KB)
-constexpr uint32_t Y_B2LBO = 8 * 128 + 16;     // CM(64 r1, 64 c) core-column stride (+16 B: the
-                                                // row-contiguous staging map is conflict-free)
-constexpr uint32_t Y_B2 = 2u * 16 * Y_B2LBO;    // C2 chunk hi + lo (~32.5 KB)
+constexpr uint32_t Y_B2LBO = 8 * 128;          // CM(64 r1, 64 c) core-column stride
+constexpr uint32_t Y_B2 = 2u * 16 * Y_B2LBO;    // C2 chunk hi + lo (32 KB)
 constexpr uint32_t Y_STAGE = Y_A2 + Y_B2;
 constexpr int Y_NST = 3;                        // chunk stages (cp.async, two in flight)
-constexpr size_t kBwdSmem = 128 + Y_B1 + Y_NST * Y_STAGE;
+constexpr size_t kBwdSmem = 1024 + Y_B1 + Y_NST * Y_STAGE;   // base aligned to 1024 (SW128 B1)
 
 struct YArgs {
   float* cores;
@@ -82,7 +81,7 @@ __device__ __forceinline__ float lo32(float x) { return x - tc::tf32_trunc(x); }
 __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
   extern __shared__ __align__(128) char smem_raw[];
   __shared__ YCtl ctl;
-  char* const smem = smem_raw + ((128u - (tc::smem_u32(smem_raw) & 127u)) & 127u);
+  char* const smem = smem_raw + ((1024u - (tc::smem_u32(smem_raw) & 1023u)) & 1023u);
   char* const b1 = smem;                                 // C1^T hi | lo
   char* const stg = smem + Y_B1;                         // stages: [A2 | B2 hi | B2 lo]
   const int tid = threadIdx.x, w = tid >> 5, lane = tid & 31;
@@ -141,17 +140,18 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
     // 256-byte row segment (coalesced); the padded core-column strides keep the stores conflict-free
     const int cr = tid >> 4, cc4 = 4 * (tid & 15);
     auto a2_off = [&](int r) { return (uint32_t)((cc4 >> 2) * Y_A2LBO + (r >> 3) * 128 + (r & 7) * 16); };
-    auto b2_off = [&](int r) { return (uint32_t)((cc4 >> 2) * Y_B2LBO + (r >> 3) * 128 + (r & 7) * 16); };
+    // C2 chunk map: row mb, float4 columns (tid >> 6) + 4 k (conflict-free stores into CM(r1, c))
+    auto b2_off = [&](int k) { return tc::cm_off(mb, 4 * ((tid >> 6) + 4 * k), 8); };
     auto issue = [&](const Job& j, uint32_t sidx) {
       const uint32_t rows = min((uint32_t)tpp, j.q1 - j.qa) << a.n1s;
       const float* dps = a.dpbuf + (size_t)j.qa * a.n1 * NC + j.ck * 64 + cc4;
-      const float* c2 = a.cores + j.c2 + j.ck * 64 + cc4;
+      const float* c2 = a.cores + j.c2 + j.ck * 64 + (size_t)mb * NC;
       const uint32_t a2 = tc::smem_u32(stg + (sidx % Y_NST) * Y_STAGE), b2 = a2 + Y_A2;
 #pragma unroll
       for (int k = 0; k < 4; ++k) {
         const int r = cr + 16 * k;
         tc::cp_async16_z(a2 + a2_off(r), dps + (size_t)(r < (int)rows ? r : 0) * NC, r < (int)rows);
-        tc::cp_async16(b2 + b2_off(r), c2 + (size_t)r * NC);
+        tc::cp_async16(b2 + b2_off(k), c2 + 4 * ((tid >> 6) + 4 * k));
       }
     };
     uint32_t ui = 0, si = 0, sp = 0;          // tile counter, issued / processed chunk counters
@@ -203,16 +203,15 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
         tc::mbar_wait(&ctl.a1_free, (ui & 1) ^ 1);      // previous tile's dC2 GEMM done
         YTA(1);
         tc::fence_after();
+        // C1^T as the MN-major (N = r1 contiguous) SWIZZLE_128B_BASE32B operand: the C1 row
+        // pieces are stored as they were loaded, one 16-byte store each (hi and lo)
 #pragma unroll
         for (int k = 0; k < 4; ++k) {
           const int r0 = 4 * ((tid >> 6) + 4 * k);
-          const float v[4] = {cv[k].x, cv[k].y, cv[k].z, cv[k].w};
-#pragma unroll
-          for (int i = 0; i < 4; ++i) {
-            const uint32_t off = tc::cm_off(r0 + i, mb, YR / 8);
-            *reinterpret_cast<float*>(b1 + off) = v[i];
-            *reinterpret_cast<float*>(b1 + Y_B1 / 2 + off) = lo32(v[i]);
-          }
+          const uint32_t off = tc::mn32_off(r0, mb, YR);
+          const float4 v = cv[k];
+          *reinterpret_cast<float4*>(b1 + off) = v;
+          *reinterpret_cast<float4*>(b1 + Y_B1 / 2 + off) = make_float4(lo32(v.x), lo32(v.y), lo32(v.z), lo32(v.w));
         }
       }
       // chunk P landed (one newer chunk may still be in flight)
@@ -229,14 +228,14 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
         for (int k = 0; k < 4; ++k) {
           const int r = cr + 16 * k;
           p[k] = *reinterpret_cast<const float4*>(a2 + a2_off(r));
-          q[k] = *reinterpret_cast<const float4*>(b2h + b2_off(r));
+          q[k] = *reinterpret_cast<const float4*>(b2h + b2_off(k));
         }
 #pragma unroll
         for (int k = 0; k < 4; ++k) {
           const int r = cr + 16 * k;
           *reinterpret_cast<float4*>(a2 + a2_off(64 + r)) =
               make_float4(lo32(p[k].x), lo32(p[k].y), lo32(p[k].z), lo32(p[k].w));
-          *reinterpret_cast<float4*>(b2l + b2_off(r)) =
+          *reinterpret_cast<float4*>(b2l + b2_off(k)) =
               make_float4(lo32(q[k].x), lo32(q[k].y), lo32(q[k].z), lo32(q[k].w));
         }
       }
@@ -337,15 +336,15 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
       if (fl & 1u) tc::mbar_wait(&ctl.d1_free, (gs & 1) ^ 1);
       tc::fence_after();
       if (lane == 0) {
-        const uint32_t id = tc::idesc_tf32(128, 64, false, false);
+        const uint32_t id = tc::idesc_tf32(128, 64, false, true);    // B = C1^T MN-major
         const uint32_t bh = tc::smem_u32(b1), bl = bh + Y_B1 / 2;
         for (int blk = 0; blk < a.nblk; ++blk) {
           const uint32_t d = tm + 256 + blk * 64;
 #pragma unroll
           for (int kk = 0; kk < YT / 8; ++kk) {
-            const uint32_t o = kk * 2 * (YR / 8) * 128;
-            const uint64_t dbh = tc::sdesc(bh + o, (YR / 8) * 128, 128);
-            const uint64_t dbl = tc::sdesc(bl + o, (YR / 8) * 128, 128);
+            const uint32_t sbo = (YR / 32) * 512, o = kk * 2 * sbo;   // MN-major, K groups of 4 outermost
+            const uint64_t dbh = tc::sdesc_l(bh + o, 512, sbo, 1);
+            const uint64_t dbl = tc::sdesc_l(bl + o, 512, sbo, 1);
             const uint32_t ah = tm + blk * 64 + kk * 8, al = tm + 128 + blk * 64 + kk * 8;
             if (a.exp & 32) continue;
             tc::mma_tf32_ts(d, ah, dbh, id, ((fl & 1u) && kk == 0) ? 0u : 1u);
