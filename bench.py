@@ -307,7 +307,7 @@ def kernels_per_step(emb_ctx, world, fused=True, cfg=None, fused_update=None):
         fused_update = world == 1
     if fused:
         fwd = 4
-        bwd = 5 + (2 if fused_update else 1)
+        bwd = 5 + 1                     # + k_update_zero (fused) or k_update after the all-reduce
     else:
         fwd = 2
         bwd = 2 + 1 + 1 + (1 if world == 1 else 1)

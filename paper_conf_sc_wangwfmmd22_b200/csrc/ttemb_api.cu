@@ -320,6 +320,8 @@ int ttemb_create(const ttemb_config* cfg, int device, void* cores, void* state, 
   if (e == cudaSuccess) e = configure_tc(c);
   if (e == cudaSuccess) e = configure_fused(c);
   if (e == cudaSuccess) e = configure_bwdtc(c);
+  // fused backward keeps the C1 / C3 gradient accumulators zero between steps (k_update_zero)
+  if (e == cudaSuccess) e = cudaMemset(c.grads, 0, sizeof(float) * c.core_floats);
   if (e != cudaSuccess) {
     fprintf(stderr, "ttemb_create: %s\n", cudaGetErrorString(e));
     delete h;

@@ -232,6 +232,23 @@ k_update(float* __restrict__ cores, float* __restrict__ state, const float* __re
   }
 }
 
+// Fused update of the C1 and C3 regions (one launch over both): apply, then clear the gradient
+// accumulator, so the next backward starts from zero without a memset (the buffer is zeroed once
+// by ttemb_create).
+__global__ void __launch_bounds__(256)
+k_update_zero(float* __restrict__ cores, float* __restrict__ state, float* __restrict__ grads, size_t n1,
+              size_t begin2, size_t n2, float lr, float eps, int opt) {
+  const size_t n = n1 + n2;
+  for (size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
+    const size_t e = i < n1 ? i : begin2 + (i - n1);
+    const float g = grads[e];
+    if (g != 0.f) {
+      apply_update(cores + e, state ? state + e : nullptr, g, lr, eps, opt);
+      grads[e] = 0.f;
+    }
+  }
+}
+
 }  // namespace
 
 cudaError_t run_group_bwd(Ctx& c, float lr, cudaStream_t s);
@@ -269,8 +286,7 @@ cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s
   {
     StageScope sc(c, ST_BWD_ZERO, s);
     if (fused) {
-      cudaMemsetAsync(c.grads, 0, sizeof(float) * c.c1_floats, s);
-      cudaMemsetAsync(c.grads + c.c3_begin, 0, sizeof(float) * c.c3_floats, s);
+      // the C1 / C3 accumulators were cleared by the previous fused update (k_update_zero)
     } else {
       cudaMemsetAsync(c.grads, 0, sizeof(float) * c.core_floats, s);
     }
@@ -322,10 +338,8 @@ cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s
   }
   if (fused) {   // C2 was updated inside the group kernel; C1 and C3 densely here
     StageScope sc(c, ST_UPD_C3, s);
-    k_update<<<grid_for(c, (int64_t)c.c3_floats, 256, 32), 256, 0, s>>>(
-        c.cores, c.state, c.grads, c.c3_begin, c.c3_floats, lr, c.eps, c.opt);
-    k_update<<<grid_for(c, (int64_t)c.c1_floats, 256, 32), 256, 0, s>>>(
-        c.cores, c.state, c.grads, 0, c.c1_floats, lr, c.eps, c.opt);
+    k_update_zero<<<grid_for(c, (int64_t)(c.c1_floats + c.c3_floats), 256, 32), 256, 0, s>>>(
+        c.cores, c.state, c.grads, c.c1_floats, c.c3_begin, c.c3_floats, lr, c.eps, c.opt);
   }
   return cudaGetLastError();
 }
