@@ -280,6 +280,17 @@ k_dense_bwd(float* __restrict__ cores, float* __restrict__ state, float* __restr
   }
 }
 
+bool agg_scatter_path(const Ctx& c) { return c.N % 4 == 0 && c.N <= 128 && (128 % c.N) == 0; }
+
+// Plan-dependent zeroing for the coming backward (G rows for the scatter aggregation, dP rows for
+// the row kernel): reads no parameters, so it runs with the index stage (pipelined side stream).
+cudaError_t run_plan_tail(Ctx& c, cudaStream_t s) {
+  if (c.nnz > 0 && agg_scatter_path(c))
+    k_zero_rows<<<grid_for(c, c.U_cap * c.N / 4, 256, 8), 256, 0, s>>>(c.p.gbuf, c.p.counts, c.N);
+  if (c.nnz > 0 && fused_eligible(c)) return run_dp_zero(c, s);
+  return cudaGetLastError();
+}
+
 cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s) {
   const PlanDev& p = c.p;
   const bool fused = (c.flags & TTEMB_FUSED_UPDATE) != 0;
@@ -293,8 +304,8 @@ cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s
   }
   if (c.nnz > 0) {
     StageScope sc(c, ST_AGG, s);
-    if (c.N % 4 == 0 && c.N <= 128 && (128 % c.N) == 0) {
-      k_zero_rows<<<grid_for(c, c.U_cap * c.N / 4, 256, 8), 256, 0, s>>>(p.gbuf, p.counts, c.N);
+    if (agg_scatter_path(c)) {
+      // (G was zeroed at the end of the index stage: run_plan_tail)
       k_agg_scatter<<<grid_for(c, cdiv(c.nnz, 32), 8, 32), 256, 0, s>>>(grad_out, p.sbag, p.spos, p.inverse,
                                                                          c.nnz, c.N, p.gbuf,
                                                                          c.weighted ? p.wpos : nullptr);

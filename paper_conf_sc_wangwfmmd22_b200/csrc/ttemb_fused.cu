@@ -729,13 +729,25 @@ cudaError_t run_fused_fwd(Ctx& c, float* out, cudaStream_t s) {
 }
 
 // Backward row stage (dP stash + dC3) for the fused-eligible shapes.
-cudaError_t run_rows_bwd2(Ctx& c, cudaStream_t s) {
+// Zero the dP rows the backward row kernel accumulates with reductions (plan-dependent, reads
+// no parameters: runs at the end of the index stage, i.e. on the pipelined side stream).
+cudaError_t run_dp_zero(Ctx& c, cudaStream_t s) {
   const PlanDev& p = c.p;
   RowBwdArgs r;
   r.cores = c.cores; r.grads = c.grads; r.meta = c.d_meta; r.counts = p.counts; r.row_pfx = p.row_pfx;
   r.row_i3 = p.row_i3; r.pfx_t = p.pfx_t; r.row_seg = p.row_seg; r.pbuf = p.pbuf; r.gbuf = p.gbuf;
   r.dpbuf = p.dpbuf; r.n1 = c.n1; r.n2 = c.n2; r.N = c.N; r.NC = c.NC;
   k_dp_zero2<<<grid_for(c, c.P_cap, 8, 8), 256, 0, s>>>(r);
+  return cudaGetLastError();
+}
+
+cudaError_t run_rows_bwd2(Ctx& c, cudaStream_t s) {
+  const PlanDev& p = c.p;
+  RowBwdArgs r;
+  r.cores = c.cores; r.grads = c.grads; r.meta = c.d_meta; r.counts = p.counts; r.row_pfx = p.row_pfx;
+  r.row_i3 = p.row_i3; r.pfx_t = p.pfx_t; r.row_seg = p.row_seg; r.pbuf = p.pbuf; r.gbuf = p.gbuf;
+  r.dpbuf = p.dpbuf; r.n1 = c.n1; r.n2 = c.n2; r.N = c.N; r.NC = c.NC;
+  // (the dP rows of chunk-straddling prefixes were zeroed at the end of the index stage)
   const int grid = grid_for(c, cdiv(c.U_cap, RW_RCH), RW_WARPS, 2);
   if (c.n3 == 4) k_rows_bwd2<4><<<grid, RW_WARPS * 32, rows_bwd_smem(4), s>>>(r);
   else k_rows_bwd2<8><<<grid, RW_WARPS * 32, rows_bwd_smem(8), s>>>(r);

@@ -697,7 +697,7 @@ cudaError_t run_index_stage(Ctx& c, const void* indices, const int64_t* offsets,
     a.tt_keys = c.tt_keys;
     const int64_t tiles = std::max<int64_t>(1, scan_tiles(nnz));
     k_plan_scan<<<(unsigned)tiles, SC_T, 0, s>>>(a, p.sc_status, p.sc_counter + 0);
-    return cudaGetLastError();
+    return run_plan_tail(c, s);
   }
   // a3
   {
@@ -723,7 +723,7 @@ cudaError_t run_index_stage(Ctx& c, const void* indices, const int64_t* offsets,
     k_scan<GroupBody><<<(unsigned)(tiles ? tiles : 1), SC_T, 0, s>>>(
         b, p.sc_status + 2 * c.sc_tiles, p.sc_counter + 2);
   }
-  return cudaGetLastError();
+  return run_plan_tail(c, s);
 }
 
 }  // namespace ttemb

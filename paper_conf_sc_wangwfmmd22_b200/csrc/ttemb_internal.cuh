@@ -176,6 +176,8 @@ bool tc_eligible(const Ctx& c);
 cudaError_t run_tc_fwd(Ctx& c, float* out, cudaStream_t s);
 cudaError_t run_tc_bwd(Ctx& c, float lr, cudaStream_t s);
 bool fused_eligible(const Ctx& c);
+cudaError_t run_dp_zero(Ctx& c, cudaStream_t s);
+cudaError_t run_plan_tail(Ctx& c, cudaStream_t s);
 cudaError_t configure_fused(Ctx& c);
 cudaError_t run_fused_fwd(Ctx& c, float* out, cudaStream_t s);
 cudaError_t run_rows_bwd2(Ctx& c, cudaStream_t s);
