@@ -298,20 +298,15 @@ def workload_config(cfg, B, world, args):
 # ---------------------------------------------------------------------------
 def kernels_per_step(emb_ctx, world, fused=True, cfg=None, fused_update=None):
     """Our kernel launches per step (cudaMemsetAsync excluded), matching the ncu launch list.
-    tcgen05 path: index stage = build_keys + hist_scan + kp radix passes + the fused plan scan; forward = prep + prefix GEMM + rows + pool (single + multi, one exits early);
-    backward = zero_rows + agg + dp_zero + rows_bwd + prefix GEMM bwd (+ 2 dense C1/C3 updates
-    when fused, + 1 update after the all-reduce otherwise)."""
+    tcgen05 path: index stage = build_keys + hist_scan + kp radix passes + plan scan + the
+    plan-dependent zeroing (zero_rows, dp_zero2); forward = gather-table prep + prefix GEMM + rows
+    + two pool launches (one-id copy / bag sums; the one not needed exits); backward = agg + rows_bwd + prefix GEMM bwd + one update (k_update_zero
+    when fused, k_update after the all-reduce otherwise).  FFMA path: build_keys + hist_scan + kp
+    passes + plan scan + zero_rows; group fwd + pool; agg + group bwd + dc1 + update."""
     kp, _ = emb_ctx
-    idx_stage = 1 + 1 + kp + 1          # build_keys, hist_scan, kp radix passes, fused plan scan
-    if fused_update is None:
-        fused_update = world == 1
     if fused:
-        fwd = 4
-        bwd = 5 + 1                     # + k_update_zero (fused) or k_update after the all-reduce
-    else:
-        fwd = 2
-        bwd = 2 + 1 + 1 + (1 if world == 1 else 1)
-    return idx_stage + fwd + bwd
+        return (1 + 1 + kp + 1 + 2) + 5 + 4    # fwd = prep + prefix + rows + two pool launches
+    return (1 + 1 + kp + 1 + 1) + 3 + 4
 
 
 def main():
