@@ -200,6 +200,8 @@ size_t carve(Ctx& c, uint8_t* base) {
   p.grp_pfx = k.take<uint32_t>(P); p.grp_off = k.take<uint32_t>(NG + 1);
   p.grp_t = k.take<uint32_t>(NG); p.grp_i2 = k.take<uint32_t>(NG);
   p.grp_arow = k.take<uint32_t>(P);
+  p.chunk_off = k.take<uint32_t>(NG + 1);
+  p.split_list = k.take<uint32_t>(NG);
   p.grp_c2 = k.take<unsigned long long>(NG);
   // --- float intermediates ---
   p.dabuf = k.take<float>((size_t)P * c.n1 * c.R);

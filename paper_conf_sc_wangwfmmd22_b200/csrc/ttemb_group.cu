@@ -35,7 +35,8 @@ struct GroupArgs {
   float* rows;          // forward output  [U][N]
   const float* gbuf;    // backward input  [U][N]
   float* dabuf;         // backward output [P][n1][R]
-  uint32_t* work;       // dynamic group counter
+  uint32_t* work;       // dynamic unit counter
+  const uint32_t *chunk_off, *split_list;
   int n1, n2, n3, N, R, NC, CW, CWs, CWp, MT, PPT;
   float lr, eps;
   int opt, fused;
@@ -55,6 +56,80 @@ __device__ __forceinline__ void red_add_v4(float* addr, float a, float b, float 
   asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(addr), "f"(a), "f"(b),
                "f"(c), "f"(d)
                : "memory");
+}
+
+// Work unit k -> (group g, prefixes [q0, q1), #units of g); false when k is past the last unit.
+__device__ __forceinline__ bool claim_unit(const GroupArgs& a, uint32_t k, uint32_t& g, uint32_t& q0,
+                                           uint32_t& q1, uint32_t& nch) {
+  const uint32_t NG = a.counts[kCntNG];
+  if (k >= a.counts[kCntNCh]) return false;
+  uint32_t lo = 0, hi = NG - 1;                 // last g with chunk_off[g] <= k
+  while (lo < hi) {
+    const uint32_t mid = (lo + hi + 1) >> 1;
+    if (a.chunk_off[mid] <= k) lo = mid; else hi = mid - 1;
+  }
+  g = lo;
+  nch = a.chunk_off[g + 1] - a.chunk_off[g];
+  const uint32_t gq0 = a.grp_off[g], gq1 = a.grp_off[g + 1];
+  q0 = gq0 + (k - a.chunk_off[g]) * kGroupChunk;
+  q1 = min(gq1, q0 + kGroupChunk);
+  return true;
+}
+
+// Units of every group (one block): chunk_off = exclusive scan of ceil(#prefixes / kGroupChunk),
+// and the list of split groups (more than one unit).
+__global__ void __launch_bounds__(1024) k_group_chunks(uint32_t* counts, const uint32_t* __restrict__ grp_off,
+                                                       uint32_t* chunk_off, uint32_t* split_list) {
+  __shared__ uint32_t s_w[32], s_carry;
+  const uint32_t NG = counts[kCntNG];
+  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  if (tid == 0) s_carry = 0;
+  __syncthreads();
+  for (uint32_t base = 0; base < NG; base += 1024) {
+    const uint32_t g = base + tid;
+    uint32_t n = 0;
+    if (g < NG) {
+      n = (grp_off[g + 1] - grp_off[g] + kGroupChunk - 1) / kGroupChunk;
+      if (n > 1) split_list[atomicAdd(counts + kCntNSplit, 1u)] = g;
+    }
+    uint32_t x = n;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+      if (lane >= o) x += y;
+    }
+    if (lane == 31) s_w[w] = x;
+    __syncthreads();
+    if (w == 0) {
+      uint32_t v = s_w[lane];
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, v, o);
+        if (lane >= o) v += y;
+      }
+      s_w[lane] = v;
+    }
+    __syncthreads();
+    const uint32_t excl = s_carry + (w ? s_w[w - 1] : 0u) + x - n;
+    if (g < NG) chunk_off[g] = excl;
+    __syncthreads();
+    if (tid == 0) s_carry += s_w[31];
+    __syncthreads();
+  }
+  if (tid == 0) { chunk_off[NG] = s_carry; counts[kCntNCh] = s_carry; }
+}
+
+// Fused update of split groups' C2 slices from their accumulated dC2 (then cleared).
+__global__ void __launch_bounds__(256) k_split_update(GroupArgs a) {
+  const uint32_t ns = a.counts[kCntNSplit];
+  const size_t per = (size_t)a.R * a.NC, total = (size_t)ns * per;
+  for (size_t e = (size_t)blockIdx.x * blockDim.x + threadIdx.x; e < total; e += (size_t)gridDim.x * blockDim.x) {
+    const uint32_t g = a.split_list[e / per];
+    const size_t idx = a.meta[a.grp_t[g]].c2_off + (size_t)a.grp_i2[g] * per + e % per;
+    const float gr = a.grads[idx];
+    upd(a.cores + idx, a.state + idx, gr, a.lr, a.eps, a.opt);
+    a.grads[idx] = 0.f;
+  }
 }
 
 // Shared-memory plan of one CTA (floats unless noted).
@@ -274,16 +349,14 @@ template <int MN1, int MN3, bool VEC>
 __global__ void __launch_bounds__(256) k_group_fwd(GroupArgs a) {
   extern __shared__ __align__(16) float smem[];
   const Smem s = carve_smem(smem, a, false);
-  const uint32_t NG = a.counts[kCntNG];
   const int tid = threadIdx.x;
   for (;;) {
     __syncthreads();
     if (tid == 0) s.misc[0] = atomicAdd(a.work, 1u);
     __syncthreads();
-    const uint32_t g = s.misc[0];
-    if (g >= NG) break;
+    uint32_t g, q0, q1, nch;
+    if (!claim_unit(a, s.misc[0], g, q0, q1, nch)) break;
     const uint32_t t = a.grp_t[g], i2 = a.grp_i2[g];
-    const uint32_t q0 = a.grp_off[g], q1 = a.grp_off[g + 1];
     const TableMeta tm = a.meta[t];
     const float* C2s = a.cores + tm.c2_off + (size_t)i2 * a.R * a.NC;
     const float* C1t = a.cores + tm.c1_off;
@@ -521,17 +594,15 @@ template <int MN1, int MN3, bool VEC>
 __global__ void __launch_bounds__(256) k_group_bwd(GroupArgs a) {
   extern __shared__ __align__(16) float smem[];
   const Smem s = carve_smem(smem, a, true);
-  const uint32_t NG = a.counts[kCntNG];
   const int tid = threadIdx.x;
   const int ty2 = tid >> 4, tx2 = tid & 15;
   for (;;) {
     __syncthreads();
     if (tid == 0) s.misc[0] = atomicAdd(a.work, 1u);
     __syncthreads();
-    const uint32_t g = s.misc[0];
-    if (g >= NG) break;
+    uint32_t g, q0, q1, nch;
+    if (!claim_unit(a, s.misc[0], g, q0, q1, nch)) break;
     const uint32_t t = a.grp_t[g], i2 = a.grp_i2[g];
-    const uint32_t q0 = a.grp_off[g], q1 = a.grp_off[g + 1];
     const TableMeta tm = a.meta[t];
     const size_t c2o = tm.c2_off + (size_t)i2 * a.R * a.NC;
     const float* C1t = a.cores + tm.c1_off;
@@ -568,7 +639,8 @@ __global__ void __launch_bounds__(256) k_group_bwd(GroupArgs a) {
           const int c = tx2 + 16 * j;
           if (c >= cw) continue;
           const size_t idx = c2o + (size_t)r1 * a.NC + c0 + c;
-          if (a.fused) upd(a.cores + idx, a.state + idx, acc2[i][j], a.lr, a.eps, a.opt);
+          if (nch > 1) atomicAdd(a.grads + idx, acc2[i][j]);   // split group: partial dC2
+          else if (a.fused) upd(a.cores + idx, a.state + idx, acc2[i][j], a.lr, a.eps, a.opt);
           else a.grads[idx] = acc2[i][j];
         }
       }
@@ -638,6 +710,7 @@ GroupArgs make_args(Ctx& c, float lr, uint32_t* work) {
   a.counts = p.counts; a.grp_off = p.grp_off; a.grp_t = p.grp_t; a.grp_i2 = p.grp_i2;
   a.grp_pfx = p.grp_pfx; a.pfx_i1 = p.pfx_i1; a.row_seg = p.row_seg; a.row_i3 = p.row_i3;
   a.rows = p.rows; a.gbuf = p.gbuf; a.dabuf = p.dabuf; a.work = work;
+  a.chunk_off = p.chunk_off; a.split_list = p.split_list;
   a.n1 = c.n1; a.n2 = c.n2; a.n3 = c.n3; a.N = c.N; a.R = c.R; a.NC = c.NC;
   a.CW = sh.CW; a.CWs = sh.CW | 1; a.CWp = (sh.CW + 3) & ~3; a.MT = sh.MT; a.PPT = sh.PPT;
   a.lr = lr; a.eps = c.eps; a.opt = c.opt; a.fused = (c.flags & TTEMB_FUSED_UPDATE) ? 1 : 0;
@@ -663,6 +736,7 @@ cudaError_t run_group_fwd(Ctx& c, cudaStream_t s) {
   const Shape sh = shape_of(c);
   GroupArgs a = make_args(c, 0.f, c.p.work + 0);
   StageScope sc(c, ST_FWD_PREFIX, s);
+  k_group_chunks<<<1, 1024, 0, s>>>(c.p.counts, c.p.grp_off, c.p.chunk_off, c.p.split_list);
   const size_t bytes = group_smem_bytes(c, false);
   const int per_sm = bytes > 110 * 1024 ? 1 : 2;
   const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(c.NG_cap, (int64_t)c.sm_count * per_sm));
@@ -680,6 +754,8 @@ cudaError_t run_group_bwd(Ctx& c, float lr, cudaStream_t s) {
   const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(c.NG_cap, (int64_t)c.sm_count * per_sm));
   if (sh.vec) dispatch_launch<true>(sh.mn1, sh.mn3, true, grid, bytes, a, s);
   else dispatch_launch<false>(sh.mn1, sh.mn3, true, grid, bytes, a, s);
+  if (a.fused)   // split groups: their C2 slices were reduced into the (zero) gradient buffer
+    k_split_update<<<c.sm_count * 8, 256, 0, s>>>(a);
   return cudaGetLastError();
 }
 

@@ -24,7 +24,12 @@ constexpr uint32_t kErrRange = 1u;     // an id outside [0, M_t)
 constexpr uint32_t kErrOffsets = 2u;   // malformed offsets
 
 // counts[] slots (device)
-constexpr int kCntU = 0, kCntP = 1, kCntNG = 2, kCntErr = 3, kCntMulti = 4, kCntUtt1 = 5, kNumCounts = 16;
+constexpr int kCntU = 0, kCntP = 1, kCntNG = 2, kCntErr = 3, kCntMulti = 4, kCntUtt1 = 5,
+              kCntNCh = 6, kCntNSplit = 7, kNumCounts = 16;
+
+// FFMA group kernels: an i2-group is processed in units of at most kGroupChunk prefixes, so a
+// Zipf-hot group is spread over many CTAs (dC2 partials of split groups meet by reductions).
+constexpr uint32_t kGroupChunk = 128;
 
 // Unique rows [0, Utt) belong to TT tables, [Utt, U) to dense (hybrid) tables: plan keys number
 // the TT tables first.  counts[kCntUtt1] = Utt + 1 when a dense row exists, else 0.
@@ -96,6 +101,7 @@ struct PlanDev {
   float* wpos;                                 // [nnz] bag weight of every position (weighted/mean bags)
   float *pbuf, *dpbuf;                         // tensor-core path: P and dL/dP per prefix
   uint32_t* grp_arow;                          // [P]  C1 row (float offset / R) of sorted prefix q, j1 = 0
+  uint32_t *chunk_off, *split_list;            // FFMA path: [NG+1] first unit of group g; [NG] split groups
   unsigned long long* grp_c2;                  // [NG] float offset of the C2 slice of group g
 };
 

@@ -574,3 +574,43 @@ def test_pipelined_plan_on_side_stream(case):
             np.testing.assert_allclose(cv[k].cpu().numpy(), rc[k], rtol=1e-4, atol=1e-5)
     with pytest.raises(tt.TTEmbError):            # forward_planned needs a fresh plan
         embs[0].forward_planned()
+
+
+@pytest.mark.parametrize("opt", ["sgd", "adagrad"])
+def test_ffma_split_groups_fused_and_unfused(opt):
+    """FFMA path with Zipf-hot i2-groups of more than kGroupChunk (128) prefixes: a group is split
+    over several CTAs, its dC2 partials meet by reductions and (fused) a separate pass updates the
+    slice.  Gradients (unfused) and updated cores (fused) vs the oracle."""
+    cfg = W.small_config([200000], [(2000, 10, 10)], (2, 2, 4), 16, 2048, 4, 0.9)
+    idx, off = W.make_batch(cfg, seed=23)
+    B = cfg.batch
+    cores = W.make_cores(cfg, seed=23)
+    go = W.make_grad_out(cfg, B, seed=23)
+    orc = Oracle.from_config(cfg)
+    plan = orc.plan(idx, off, B)
+    sizes = np.diff(plan["grp_off"])
+    assert sizes.max() > 128, sizes.max()          # the case must contain split groups
+    g = orc.backward(cores, idx, off, B, go)
+    ga = orc.backward(cores, idx, off, B, go, absolute=True)
+    lr = 0.05
+    for fused in (False, True):
+        emb = gpu_emb(cfg, B, len(idx), optimizer=opt, fused_update=fused)
+        emb.load_cores(cores)
+        run_forward(emb, idx, off, B)
+        emb.backward(torch.as_tensor(go, device=DEV), lr=lr)
+        if not fused:
+            for k in range(3):
+                assert_companion(emb.grad_views()[0][k].cpu().numpy(), g[0][k], ga[0][k], 1e-4, f"dC{k+1}")
+            emb.update(lr)
+        torch.cuda.synchronize()
+        sv = emb.state_views()
+        for k in range(3):
+            ref_p, ref_s = Oracle.update(opt, lr, cores[0][k], g[0][k], None)
+            assert_update_close(emb.core_views()[0][k].cpu().numpy(), ref_p, cores[0][k], g[0][k], ga[0][k], lr,
+                                opt, got_s=None if sv is None else sv[0][k].cpu().numpy(), ref_s=ref_s,
+                                s_old=np.zeros_like(cores[0][k]), what=f"{opt} fused={fused} C{k+1}")
+        # a second step must start from cleared split-group accumulators
+        if fused:
+            run_forward(emb, idx, off, B)
+            emb.backward(torch.as_tensor(go, device=DEV), lr=lr)
+            assert emb.check() == 0
