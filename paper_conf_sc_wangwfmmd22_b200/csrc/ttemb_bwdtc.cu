@@ -430,32 +430,19 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
             tc::tmem_ld32(tc::taddr(tm + 256 + blk * 64 + 32 * h, 32 * Q, 0), v);
             if (c < NC && !(a.exp & 1)) {
               const size_t base = so + (size_t)(32 * h) * NC + c;
-              if (!a.fused) {
+              if (!a.fused || a.opt != TTEMB_SGD) {
+                // unfused, or fused Adagrad: dC2 to the gradient buffer (plain coalesced stores);
+                // Adagrad's read-modify-write of C2 and its state runs after the kernel as a
+                // bandwidth-bound pass over the touched slices (k_c2_update_zero)
 #pragma unroll
                 for (int i = 0; i < 32; ++i) a.grads[base + (size_t)i * NC] = v[i];
-              } else if (a.opt == TTEMB_SGD) {
+              } else {
                 // C2 -= lr dC2 as fire-and-forget reductions (each warp instruction covers 32
                 // consecutive floats): no read of the old slice, no load latency on this path
 #pragma unroll
                 for (int i = 0; i < 32; ++i)
                   asm volatile("red.global.add.f32 [%0], %1;" ::"l"(a.cores + base + (size_t)i * NC),
                                "f"(-a.lr * v[i]) : "memory");
-              } else {
-#pragma unroll
-                for (int h2 = 0; h2 < 32; h2 += 16) {
-                  float old[16], st[16];
-#pragma unroll
-                  for (int i = 0; i < 16; ++i) {
-                    old[i] = a.cores[base + (size_t)(h2 + i) * NC];
-                    st[i] = a.state[base + (size_t)(h2 + i) * NC];
-                  }
-#pragma unroll
-                  for (int i = 0; i < 16; ++i) {
-                    const float gr = v[h2 + i], sn = st[i] + gr * gr;
-                    a.state[base + (size_t)(h2 + i) * NC] = sn;
-                    a.cores[base + (size_t)(h2 + i) * NC] = old[i] - a.lr * gr / (sqrtf(sn) + a.eps);
-                  }
-                }
               }
             }
           }
@@ -486,6 +473,27 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
 
 }  // namespace
 
+// Fused Adagrad for the C2 slices the prefix-backward kernel wrote to the gradient buffer:
+// s += g^2, C2 -= lr g / (sqrt(s) + eps), g = 0 (keeps the fused-mode accumulators zero).
+__global__ void __launch_bounds__(256)
+k_c2_update_zero(float* __restrict__ cores, float* __restrict__ state, float* __restrict__ grads,
+                 const unsigned long long* __restrict__ grp_c2, const uint32_t* __restrict__ counts,
+                 uint32_t slice, float lr, float eps) {
+  const size_t n4 = (size_t)counts[kCntNG] * (slice / 4);
+  for (size_t e = (size_t)blockIdx.x * blockDim.x + threadIdx.x; e < n4; e += (size_t)gridDim.x * blockDim.x) {
+    const size_t gi = e / (slice / 4), o = grp_c2[gi] + 4 * (e % (slice / 4));
+    float4 g = *reinterpret_cast<float4*>(grads + o);
+    float4 p = *reinterpret_cast<float4*>(cores + o);
+    float4 st = *reinterpret_cast<float4*>(state + o);
+    st.x += g.x * g.x; st.y += g.y * g.y; st.z += g.z * g.z; st.w += g.w * g.w;
+    p.x -= lr * g.x / (sqrtf(st.x) + eps); p.y -= lr * g.y / (sqrtf(st.y) + eps);
+    p.z -= lr * g.z / (sqrtf(st.z) + eps); p.w -= lr * g.w / (sqrtf(st.w) + eps);
+    *reinterpret_cast<float4*>(state + o) = st;
+    *reinterpret_cast<float4*>(cores + o) = p;
+    *reinterpret_cast<float4*>(grads + o) = make_float4(0.f, 0.f, 0.f, 0.f);
+  }
+}
+
 cudaError_t configure_bwdtc(Ctx& c) {
   if (!fused_eligible(c)) return cudaSuccess;
   return cudaFuncSetAttribute(k_prefix_bwd, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBwdSmem);
@@ -514,6 +522,9 @@ cudaError_t run_prefix_bwd(Ctx& c, float lr, cudaStream_t s) {
     a.trace = trace;
   }
   k_prefix_bwd<<<grid, Y_THREADS, kBwdSmem, s>>>(a);
+  if (a.fused && a.opt != TTEMB_SGD)
+    k_c2_update_zero<<<c.sm_count * 8, 256, 0, s>>>(c.cores, c.state, c.grads, p.grp_c2, p.counts,
+                                                    (uint32_t)(YR * c.NC), lr, c.eps);
   if (a.trace) {
     std::vector<unsigned long long> hb(32 * grid);
     cudaMemcpyAsync(hb.data(), trace, hb.size() * 8, cudaMemcpyDeviceToHost, s);
