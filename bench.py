@@ -357,9 +357,8 @@ def main():
         args.scaling = "strong" if args.config == "c5" else "weak"
 
     if args.impl == "reference":
-        if world > 1:
-            import torch.distributed as dist
-            dist.init_process_group("gloo")
+        # rank 0 alone times the oracle; no process group (and no torch import, whose OpenMP
+        # runtime would pin the oracle to torchrun's OMP_NUM_THREADS=1)
         run_reference(args, cfg, rank, world)
         return
     if args.impl == "paper":

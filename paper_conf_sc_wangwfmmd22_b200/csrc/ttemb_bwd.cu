@@ -1,15 +1,13 @@
-// ttemb_bwd.cu -- backward and update, sm_100a.
+// ttemb_bwd.cu -- backward driver, aggregation and updates, sm_100a.
 //
-//   a8  in-advance aggregation G_u = sum_{positions of row u} grad_out[bag]
-//       as a fixed-chunk segmented reduction over the sorted occurrence list (no atomics,
-//       deterministic; long Zipf segments are split across chunks and re-joined)
-//   a9  per prefix p: dP_p = sum_{u in p} G_u . C3[i3]^T, dC3[i3] += P_p^T G_u   (Eq. 6 read
-//       as left^T . dL/de . right^T; dP aggregated per prefix = exact algebra)
-//   a10 per i2-group g: dC2[i2] = A_g^T . dP_g  (reduced inside the CTA, no atomics),
-//       dA_g = dP_g . C2[i2]^T  (per-prefix dC1 partials)
-//   a11 dC1[t][i1] = sum of the partials of the contiguous (t, i1) prefix run
-//   a12 SGD / Adagrad; with TTEMB_FUSED_UPDATE the C2 slices are updated by the group
-//       CTA that owns them and C1 by the run reduction ("fused TT core update")
+//   a8  in-advance aggregation G_u = sum_{positions of row u} w_j grad_out[bag]:
+//       k_agg_scatter (warp per 32 sorted occurrences, vector reductions) or the deterministic
+//       fixed-chunk segmented reduction k_agg + k_agg_fix (other dims)
+//   a9-a11 in the tensor-core kernels (ttemb_fused.cu / ttemb_bwdtc.cu) or the FFMA group
+//       kernels (ttemb_group.cu; k_dc1 reduces their per-prefix dC1 partials)
+//   a12 SGD / Adagrad: fused on one replica (C2 by its owning CTA, C1 + C3 by k_update_zero,
+//       dense tables by k_dense_bwd; "fused TT core update"), else k_update after
+//       the caller's gradient all-reduce
 #include <type_traits>
 
 #include "ttemb_internal.cuh"

@@ -5,16 +5,19 @@
 //   dC2[i2]^T[c][r1] += sum_m dP[m][c] . C1[i1_m][j1_m][r1]      (Eq. 6 read as left^T . dL/de
 //                       . right^T; the left factor of C2 is the C1 slice)
 //       M = 128 c per block, N = 64 r1, K = 64 m: A = dP^T held in TENSOR MEMORY (lane = c,
-//       column = m, written by the loader threads), B = C1^T rows in shared memory;
+//       column = m, written by the loader threads), B = C1^T as an MN-major
+//       SWIZZLE_128B_BASE32B operand in shared memory (the C1 row pieces stored as loaded);
 //       accumulated in TMEM over all tiles of the group (no atomics, no partial buffers).
 //   dA[m][r1] = sum_c dP[m][c] . C2[i2][r1][c]                  (the C1 gradient partials)
 //       M = 128 = the tile's dP rows stacked as [dP_hi; dP_lo], N = 64 r1, K = c in chunks of
 //       64 staged in shared memory (double-buffered); two MMAs per K step (B = C2_hi, C2_lo)
 //       give A_hi B_hi + A_lo B_hi + A_hi B_lo, i.e. 3xTF32 with two M = 128 instructions.
 //       The epilogue adds dA straight into the C1 gradient (red.global.add.v4, L2-resident).
-// At the group's last tile the dC2 accumulator is drained and, with TTEMB_FUSED_UPDATE, the
-// C2 slice is updated in place (SGD / Adagrad, the paper's fused TT core update);
-// the slice has no other reader in this kernel once its last tile's MMAs completed.
+// At the group's last tile the dC2 accumulator is drained: with TTEMB_FUSED_UPDATE and SGD the
+// C2 slice is updated in place by reductions straight from TMEM (the paper's fused TT core
+// update; the slice has no other reader once its last tile's MMAs completed); for
+// Adagrad (read-modify-write of the slice and its state) or unfused, dC2 is stored and fused
+// Adagrad finishes in k_c2_update_zero.
 // fp32 accuracy: 3xTF32 (hi = raw fp32, read by the tensor core with truncation; lo =
 // x - trunc_tf32(x)); scripts/tc_probe3.cu measures the TMEM-A form.
 //
@@ -511,12 +514,12 @@ cudaError_t run_prefix_bwd(Ctx& c, float lr, cudaStream_t s) {
   a.NC = c.NC; a.nblk = (c.NC + 127) / 128; a.tpp = YT / c.n1; a.nchunk = (c.NC + 63) / 64;
   a.lr = lr; a.eps = c.eps; a.opt = c.opt; a.fused = (c.flags & TTEMB_FUSED_UPDATE) ? 1 : 0;
   a.exp = exp_bits();
-  a.pf = env_int("TTEMB_PF_BWD", 0);
+  a.pf = knobs().pf_bwd;
   StageScope sc(c, ST_BWD_PREFIX, s);
   const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(c.NG_cap, (int64_t)c.sm_count));
   static unsigned long long* trace = nullptr;
   a.trace = nullptr;
-  if (getenv("TTEMB_TRACE")) {
+  if (knobs().trace) {
     if (!trace) cudaMalloc(&trace, sizeof(unsigned long long) * 32 * grid);
     cudaMemsetAsync(trace, 0, sizeof(unsigned long long) * 32 * grid, s);
     a.trace = trace;

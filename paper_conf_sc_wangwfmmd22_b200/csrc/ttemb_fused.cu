@@ -653,7 +653,7 @@ size_t rows_bwd_smem(int n3) { return (size_t)RW_WARPS * RW_NSL * (XR * n3 + 32 
 }  // namespace
 
 bool fused_eligible(const Ctx& c) {
-  return !(c.flags & TTEMB_FP32_CORES) && !getenv("TTEMB_OLD_FWD") && c.R == XR && c.NC <= 256 &&
+  return !(c.flags & TTEMB_FP32_CORES) && !knobs().old_fwd && c.R == XR && c.NC <= 256 &&
          (c.n3 == 4 || c.n3 == 8) && (c.n1 == 1 || c.n1 == 2 || c.n1 == 4 || c.n1 == 8) && c.n1 * c.n2 <= 16;
 }
 
@@ -678,7 +678,7 @@ cudaError_t run_fused_fwd(Ctx& c, float* out, cudaStream_t s) {
   a.grp_i2 = p.grp_i2; a.grp_pfx = p.grp_pfx; a.pfx_i1 = p.pfx_i1; a.pfx_t = p.pfx_t; a.row_seg = p.row_seg;
   a.row_i3 = p.row_i3; a.row_pfx = p.row_pfx; a.grp_arow = p.grp_arow; a.grp_c2 = p.grp_c2; a.rows = p.rows; a.pbuf = p.pbuf;
   a.work = p.work + 0;
-  a.dbg = getenv("TTEMB_DBG") ? atoi(getenv("TTEMB_DBG")) : 0;
+  a.dbg = knobs().dbg;
   a.n1 = c.n1; a.n1s = c.n1 == 1 ? 0 : c.n1 == 2 ? 1 : c.n1 == 4 ? 2 : 3;
   a.n2 = c.n2; a.n3 = c.n3; a.N = c.N; a.NC = c.NC; a.nblk = (c.NC + 127) / 128; a.tpp = XT / c.n1;
   {
@@ -687,7 +687,7 @@ cudaError_t run_fused_fwd(Ctx& c, float* out, cudaStream_t s) {
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(c.NG_cap, (int64_t)c.sm_count));
     static unsigned long long* trace = nullptr;
     a.trace = nullptr;
-    if (getenv("TTEMB_TRACE")) {
+    if (knobs().trace) {
       if (!trace) cudaMalloc(&trace, sizeof(unsigned long long) * 32 * grid);
       cudaMemsetAsync(trace, 0, sizeof(unsigned long long) * 32 * grid, s);
       a.trace = trace;

@@ -1,14 +1,11 @@
-// ttemb_fwd.cu -- forward contractions and pooling, sm_100a.
+// ttemb_fwd.cu -- forward driver, pooling and the dense (hybrid) rows (SURVEY 8(a) row a7,
+// 8(f3)), sm_100a.
 //
-//   a5 prefix contraction, one CTA per i2-group g = (t, i2):
-//        P_g = A_g . C2[i2]     A_g = the C1[i1] slices of the group's prefixes stacked
-//        ((Q n1) x R), C2[i2] viewed as (R x n2 R); the result rows are the Reuse buffer
-//        entries P_p[j1][j2][r2] = sum_r1 C1[i1,j1,r1] C2[i2,r1,j2,r2]
-//      C2[i2] is staged in shared memory once per group (column chunks of <= 128).
-//   a6 row contraction E_u = P_p (n1 n2 x R) . C3[i3] (R x n3)  (Eq. 2, P:164 step 3)
-//   a7 sum pooling out[b][t] = sum_{j in bag} E_{inverse[j]}     (Eq. 4, P:164 step 4)
-// FP32 FFMA on CUDA cores (tensor cores only where ncu shows the rank-R
-// contraction is the bottleneck).
+//   a5 + a6 run in the tensor-core kernels (ttemb_fused.cu, R = 64) or the FFMA group kernels
+//   (ttemb_group.cu); this file dispatches them, copies the rows of dense (hybrid) tables
+//   (k_dense_fwd) and pools:
+//   a7 out[b][t] = sum_{j in bag} w_j E_{inverse[j]}   (Eq. 4, P:164 step 4; w_j = 1, the
+//      per-sample weight or 1/|bag| for nn.EmbeddingBag "mean", P:48 / P:306)
 #include <type_traits>
 
 #include "ttemb_internal.cuh"

@@ -684,7 +684,7 @@ cudaError_t run_index_stage(Ctx& c, const void* indices, const int64_t* offsets,
                                ST_SORT_HIST, ST_SORT_PASS, s, /*have_hist=*/true);
   p.skey = which ? p.keysB : p.keysA;
   p.spos = which ? p.valsB : p.valsA;
-  if (!getenv("TTEMB_THREE_SCANS")) {   // a3 + a4 fused (default)
+  if (!knobs().three_scans) {   // a3 + a4 fused (default)
     StageScope sc(c, ST_UNIQUE, s);
     PlanScanArgs a;
     a.skey = p.skey; a.spos = p.spos; a.bag_of = p.bag_of; a.kbase = c.d_kbase; a.kmap = c.d_kmap;

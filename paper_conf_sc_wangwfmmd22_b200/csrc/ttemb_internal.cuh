@@ -45,22 +45,26 @@ enum Stage : int {
   ST_COUNT
 };
 
-// TTEMB_EXP environment bits: switch parts of a kernel off for timing experiments (results
-// are invalid; never set in tests / bench runs that report numbers).
-inline int exp_bits() {
-  static int v = -1;
-  if (v < 0) {
-    const char* e = getenv("TTEMB_EXP");
-    v = e ? atoi(e) : 0;
-  }
-  return v;
+// Debug / experiment knobs from the environment, read ONCE per process (never on the launch
+// path): TTEMB_EXP bits switch parts of k_prefix_bwd off (timing experiments, results invalid),
+// TTEMB_DBG likewise for the forward kernels, TTEMB_TRACE enables role timers (trace builds),
+// TTEMB_THREE_SCANS / TTEMB_OLD_FWD select the older index scans / forward kernels, TTEMB_PF_BWD
+// sets an L2 prefetch distance in k_prefix_bwd.
+struct Knobs {
+  int exp = 0, dbg = 0, trace = 0, three_scans = 0, old_fwd = 0, pf_bwd = 0;
+};
+inline const Knobs& knobs() {
+  static const Knobs k = [] {
+    auto num = [](const char* n) { const char* e = getenv(n); return e ? atoi(e) : 0; };
+    Knobs r;
+    r.exp = num("TTEMB_EXP"); r.dbg = num("TTEMB_DBG"); r.trace = getenv("TTEMB_TRACE") ? 1 : 0;
+    r.three_scans = getenv("TTEMB_THREE_SCANS") ? 1 : 0; r.old_fwd = getenv("TTEMB_OLD_FWD") ? 1 : 0;
+    r.pf_bwd = num("TTEMB_PF_BWD");
+    return r;
+  }();
+  return k;
 }
-
-// Tuning knob from the environment (default when unset).
-inline int env_int(const char* name, int dflt) {
-  const char* e = getenv(name);
-  return e ? atoi(e) : dflt;
-}
+inline int exp_bits() { return knobs().exp; }
 
 // Index of the key range holding `key` (kbase[0..T-1] ascending, in key order).
 __device__ __forceinline__ int table_of_key(const uint64_t* kbase, int T, uint32_t key) {

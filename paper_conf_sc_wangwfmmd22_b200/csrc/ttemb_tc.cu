@@ -930,7 +930,7 @@ TcArgs make_tc_args(Ctx& c, float lr, uint32_t* work, float* out) {
   a.grp_arow = p.grp_arow; a.grp_c2 = p.grp_c2;
   a.pbuf = p.pbuf; a.dpbuf = p.dpbuf; a.rows = p.rows; a.gbuf = p.gbuf; a.dabuf = p.dabuf;
   a.out = out; a.work = work; a.trace = nullptr;
-  a.dbg = getenv("TTEMB_DBG") ? atoi(getenv("TTEMB_DBG")) : 0;
+  a.dbg = knobs().dbg;
   a.n1 = c.n1; a.n2 = c.n2; a.n3 = c.n3; a.N = c.N; a.NC = c.NC;
   a.n1s = c.n1 == 1 ? 0 : c.n1 == 2 ? 1 : c.n1 == 4 ? 2 : 3;
   a.f_nmb = (c.NC + 127) / 128;
@@ -970,7 +970,7 @@ cudaError_t run_tc_fwd(Ctx& c, float* out, cudaStream_t s) {
     StageScope sc(c, ST_FWD_PREFIX, s);
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(c.NG_cap, (int64_t)c.sm_count));
     static unsigned long long* trace = nullptr;
-    if (getenv("TTEMB_TRACE")) {
+    if (knobs().trace) {
       if (!trace) cudaMalloc(&trace, sizeof(unsigned long long) * 16 * grid);
       cudaMemsetAsync(trace, 0, sizeof(unsigned long long) * 16 * grid, s);
       a.trace = trace;
