@@ -233,7 +233,10 @@ class TTEmbeddingBag:
 
     # -- parameters --------------------------------------------------------
     def _views(self, buf: torch.Tensor):
+        """Per table (C1, C2, C3) views at the configured rank; a zero-padded storage rank
+        (ttemb_config.rank doc) is sliced away, so the views are strided then."""
         out = []
+        R = self.rank
         for t in range(self.T):
             vs = []
             for k in range(3):
@@ -242,7 +245,15 @@ class TTEmbeddingBag:
                 if self.dense[t] and k == 0:
                     shp = shape[:2]            # hybrid: the plain table W[M][N]
                 n = int(np.prod(shp))
-                vs.append(buf[off:off + n].view(*shp))
+                v = buf[off:off + n].view(*shp)
+                if not self.dense[t]:
+                    if k == 0:
+                        v = v[:, :, :R]
+                    elif k == 1:
+                        v = v[:, :R, :, :R]
+                    else:
+                        v = v[:, :R, :]
+                vs.append(v)
             out.append(tuple(vs))
         return out
 

@@ -113,6 +113,7 @@ struct Ctx {
   // configuration
   int device = 0, sm_count = 148;
   int T = 0, n1 = 0, n2 = 0, n3 = 0, N = 0, R = 0, NC = 0;
+  int R_user = 0;                    // the configured rank (R may be the zero-padded storage rank)
   int index_bits = 64, opt = 0;
   float eps = 1e-10f;
   uint32_t flags = 0;

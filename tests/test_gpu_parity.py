@@ -147,7 +147,7 @@ def test_c4_reduced_batch(fp32_cores):
             assert_companion(mine[k].cpu().numpy(), g[t][k], ga[t][k], 1e-4, f"dC{k+1} t{t}")
 
 
-@pytest.mark.parametrize("name,rank", [("c4", None), ("c5", 64), ("c5", 128)])
+@pytest.mark.parametrize("name,rank", [("c4", None), ("c5", 64), ("c5", 128), ("c5", 32)])
 def test_full_size_sampled(name, rank):
     """Full BASELINE sizes in the bench launch configuration (fused update off so
     the gradients stay observable): plan bit-exact vs numpy, sampled bags vs the
@@ -614,3 +614,37 @@ def test_ffma_split_groups_fused_and_unfused(opt):
             run_forward(emb, idx, off, B)
             emb.backward(torch.as_tensor(go, device=DEV), lr=lr)
             assert emb.check() == 0
+
+
+def test_rank_padding_storage_is_exact():
+    """32 <= R < 64 runs on the tcgen05 path with cores stored zero-padded to rank 64
+    (ttemb_config.rank doc, R28): the padding stays exactly zero through fused SGD and
+    Adagrad steps, and the results match the oracle at the configured rank."""
+    cfg = W.small_config([20000, 300], [(28, 28, 26), (7, 7, 7)], (4, 4, 4), 40, 96, 2, 1.05)
+    idx, off = W.make_batch(cfg, seed=29)
+    B = cfg.batch
+    cores = W.make_cores(cfg, seed=29)
+    go = W.make_grad_out(cfg, B, seed=29)
+    orc = Oracle.from_config(cfg)
+    for opt in ("sgd", "adagrad"):
+        emb = gpu_emb(cfg, B, len(idx), optimizer=opt, fused_update=True)
+        assert emb.layout[0][1][1][1] == 64              # storage rank of C2
+        emb.load_cores(cores)
+        out = run_forward(emb, idx, off, B)
+        assert_companion(out.cpu().numpy(), orc.forward(cores, idx, off, B),
+                         orc.forward(cores, idx, off, B, absolute=True), 1e-5, "forward")
+        for _ in range(2):
+            run_forward(emb, idx, off, B)
+            emb.backward(torch.as_tensor(go, device=DEV), lr=0.05)
+        torch.cuda.synchronize()
+        R = cfg.rank
+        for t in range(cfg.num_tables):
+            full = []
+            for k in range(3):
+                o, shp = emb.layout[t][k]
+                shp = shp if k == 1 else shp[:3]
+                full.append(emb.cores[o:o + int(np.prod(shp))].view(*shp))
+            assert torch.count_nonzero(full[0][:, :, R:]) == 0
+            assert torch.count_nonzero(full[1][:, R:]) == 0 and torch.count_nonzero(full[1][..., R:]) == 0
+            assert torch.count_nonzero(full[2][:, R:]) == 0
+            assert torch.count_nonzero(full[1][:, :R, :, :R]) > 0
