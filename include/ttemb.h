@@ -88,7 +88,7 @@ typedef struct {
   int32_t dim;                   /* N = col_factors[0]*col_factors[1]*col_factors[2]  */
   int32_t col_factors[3];        /* (n1, n2, n3), shared by all tables                */
   int32_t rank;                  /* R1 = R2 = rank (1..128), R0 = R3 = 1; on
-                                    the tensor-core path a rank 32..63 is STORED zero-padded
+                                    the tensor-core path a rank 16..63 is STORED zero-padded
                                     to 64 (ttemb_core_layout reports the storage shapes;
                                     padding entries must be 0 and stay 0)               */
   int32_t index_bits;            /* 64 (int64 ids, PyTorch default) or 32             */

@@ -97,16 +97,21 @@ int validate(const ttemb_config* cfg) {
   return TTEMB_OK;
 }
 
+#ifndef TTEMB_PAD_MIN_RANK
+#define TTEMB_PAD_MIN_RANK 16   // c2 (R = 16) 1.56x faster padded; c1 (R = 8) is not
+#endif
+constexpr int kPadMinRank = TTEMB_PAD_MIN_RANK;   // smallest rank run zero-padded on tcgen05
+
 // Fills every size-derived field of c (no device pointers).
 void plan_sizes(const ttemb_config* cfg, Ctx& c) {
   c.T = cfg->num_tables;
   c.n1 = cfg->col_factors[0]; c.n2 = cfg->col_factors[1]; c.n3 = cfg->col_factors[2];
   c.N = cfg->dim; c.R = cfg->rank;
-  // 32 <= R < 64: store the cores zero-padded to rank 64 and run the tcgen05 path.  Exact: the
+  // kPadMinRank <= R < 64: store the cores zero-padded to rank 64 and run the tcgen05 path.  Exact: the
   // padded rows / columns of C1, C2, C3 multiply only zeros, so every padded entry of dC_k is
   // exactly 0 and SGD / Adagrad keep it 0 (R28).
   c.R_user = c.R;
-  if (!(c.flags & TTEMB_FP32_CORES) && c.R >= 32 && c.R < 64 && (c.n3 == 4 || c.n3 == 8) &&
+  if (!(cfg->flags & TTEMB_FP32_CORES) && c.R >= kPadMinRank && c.R < 64 && (c.n3 == 4 || c.n3 == 8) &&
       (c.n1 == 1 || c.n1 == 2 || c.n1 == 4 || c.n1 == 8) && c.n1 * c.n2 <= 16 && c.n2 * 64 <= 256)
     c.R = 64;
   c.NC = c.n2 * c.R;

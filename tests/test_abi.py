@@ -58,13 +58,13 @@ def _cfg(**kw):
 
 
 def test_query_sizes_consistent():
-    cfg, keep = _cfg()
+    cfg, keep = _cfg(fp32_cores=True)     # (the tensor-core path stores R = 16 zero-padded to 64)
     core, state, grad, ws = tt.ttemb_query_sizes(cfg)
     c = W.config("c2")
     assert core == grad and state == 0 and ws > 0
     # padded per-table blocks: at least the exact core bytes, at most 16 B per block more
     assert W.core_bytes(c) <= core <= W.core_bytes(c) + 16 * 3 * c.num_tables
-    cfg2, keep2 = _cfg(optimizer="adagrad")
+    cfg2, keep2 = _cfg(optimizer="adagrad", fp32_cores=True)
     assert tt.ttemb_query_sizes(cfg2)[1] == core
 
 
@@ -127,9 +127,10 @@ def test_hybrid_tables_sizes_and_layout_validation():
     the core / grad buffers grow by exactly the dense tables' size (16-byte padded blocks)."""
     c = W.config("c2")
     h = W.hybrid(c)
-    cfg_tt, k1 = _cfg()
+    cfg_tt, k1 = _cfg(fp32_cores=True)
     cfg_h, k2 = tt.make_config(h.table_rows, [(0, 0, 0) if d else f for d, f in zip(h.dense, h.row_factors)],
-                               h.col_factors, h.rank, h.batch, h.batch * h.num_tables, dense=h.dense)
+                               h.col_factors, h.rank, h.batch, h.batch * h.num_tables, dense=h.dense,
+                               fp32_cores=True)   # (unpadded rank: exact byte count)
     core_h = tt.ttemb_query_sizes(cfg_h)[0]
     assert W.core_bytes(h) <= core_h <= W.core_bytes(h) + 16 * 3 * h.num_tables
     assert core_h != tt.ttemb_query_sizes(cfg_tt)[0]
