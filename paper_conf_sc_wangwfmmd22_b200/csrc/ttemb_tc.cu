@@ -983,7 +983,7 @@ cudaError_t run_tc_fwd(Ctx& c, float* out, cudaStream_t s) {
       cudaStreamSynchronize(s);
       double m[16] = {};
       for (int b = 0; b < grid; ++b) for (int k = 0; k < 16; ++k) m[k] += (double)h[16 * b + k] / grid;
-      fprintf(stderr, "[trace fwd] tiles/CTA %.1f loader-total %.0f | loader: issue %.0f prefetch %.0f landed %.0f empty %.0f convert %.0f -"
+      fprintf(stderr, "[trace fwd] tiles/CTA %.1f loader-total %.0f | loader: issue %.0f prefetch %.0f landed %.0f empty %.0f convert %.0f other %.0f"
               " | mma: full %.0f accempty %.0f issue %.0f | epi: tinfo %.0f table %.0f accfull %.0f drain %.0f (cycles/CTA)\n",
               m[13], m[14], m[0], m[1], m[2], m[3], m[4], m[5], m[6], m[7], m[8], m[9], m[10], m[11], m[12]);
     }
