@@ -10,9 +10,31 @@
 
 #include "ttemb_internal.cuh"
 
+#ifndef TTEMB_POOL_MODE
+#define TTEMB_POOL_MODE 1     // one-hot pooling: 1 = output-ordered, 0 = position-ordered scatter
+#endif
+#ifndef TTEMB_POOL_IPT
+#define TTEMB_POOL_IPT 2      // independent float4 items per thread (output-ordered kernel)
+#endif
+#ifndef TTEMB_POOL_STCS
+#define TTEMB_POOL_STCS 1     // 1 = streaming (evict-first) stores of the pooled output
+#endif
+#ifndef TTEMB_POOL_PER_SM
+#define TTEMB_POOL_PER_SM 32  // grid cap, CTAs per SM
+#endif
+
 namespace ttemb {
 
 namespace {
+
+// the pooled output is written once and not re-read by this step: optionally streamed past L2
+__device__ __forceinline__ void pool_store(float4* p, float4 v) {
+#if TTEMB_POOL_STCS
+  __stcs(p, v);
+#else
+  *p = v;
+#endif
+}
 
 // a7: out[b][t][:] = sum over the bag's positions (index order); empty bag -> 0.
 // Thread = (bag, VW-wide column group); 4 independent items per thread are processed
@@ -92,7 +114,42 @@ k_pool_single(const float* __restrict__ rows, const uint32_t* __restrict__ inver
     }
 #pragma unroll
     for (int i = 0; i < 4; ++i)
-      if (dst[i] >= 0) reinterpret_cast<float4*>(out)[dst[i]] = v[i];
+      if (dst[i] >= 0) pool_store(reinterpret_cast<float4*>(out) + dst[i], v[i]);
+  }
+}
+
+// a7 one-hot, output-ordered: with one id per bag the validated offsets are the identity
+// (offsets[bag] = bag), so output row o = b*T + t reads position j = t*B + b directly and the
+// 109 MB (C4) output is written in address order.  Thread = (output row, float4 column).
+__global__ void __launch_bounds__(256)
+k_pool_single_out(const float* __restrict__ rows, const uint32_t* __restrict__ inverse, int64_t nnz,
+                  int T, int B, int N, float* __restrict__ out, const uint32_t* __restrict__ counts,
+                  const float* __restrict__ wpos) {
+  if (counts[kCntMulti] != 0) return;
+  const int NV = N >> 2;
+  const int64_t total = (int64_t)T * B * NV, stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t e0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e0 < total; e0 += TTEMB_POOL_IPT * stride) {
+    float4 v[TTEMB_POOL_IPT];
+#pragma unroll
+    for (int i = 0; i < TTEMB_POOL_IPT; ++i) {
+      const int64_t e = e0 + i * stride;
+      v[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+      if (e < total) {
+        const int64_t o = e / NV;
+        const int f = (int)(e - o * NV);
+        const int64_t b = o / T, t = o - b * T, j = t * B + b;
+        if (j < nnz) {
+          v[i] = __ldg(reinterpret_cast<const float4*>(rows + (size_t)__ldg(inverse + j) * N) + f);
+          if (wpos) {
+            const float w = __ldg(wpos + j);
+            v[i].x *= w; v[i].y *= w; v[i].z *= w; v[i].w *= w;
+          }
+        }
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < TTEMB_POOL_IPT; ++i)
+      if (e0 + i * stride < total) pool_store(reinterpret_cast<float4*>(out) + e0 + i * stride, v[i]);
   }
 }
 
@@ -140,11 +197,16 @@ cudaError_t run_forward_compute(Ctx& c, float* out, const int64_t* offsets, cuda
     if (total > 0) {
       if (c.N % 4 == 0) {
         // one id per bag (device flag): a position-parallel copy; otherwise the bag-parallel sum
-        if (c.nnz > 0)
-          k_pool_single<<<grid_for(c, c.nnz * c.N / 16, 256, 32), 256, 0, s>>>(p.rows, p.inverse, p.bag_of,
-                                                                              c.nnz, c.N, out, p.counts,
-                                                                              c.weighted ? p.wpos : nullptr);
-        k_pool<4><<<grid_for(c, total / 16, 256, 32), 256, 0, s>>>(p.rows, p.inverse, offsets, c.nnz,
+        if (c.nnz > 0) {
+          if (TTEMB_POOL_MODE == 1)
+            k_pool_single_out<<<grid_for(c, total / (4 * TTEMB_POOL_IPT), 256, TTEMB_POOL_PER_SM), 256, 0, s>>>(
+                p.rows, p.inverse, c.nnz, c.T, c.B, c.N, out, p.counts, c.weighted ? p.wpos : nullptr);
+          else
+            k_pool_single<<<grid_for(c, c.nnz * c.N / 16, 256, TTEMB_POOL_PER_SM), 256, 0, s>>>(
+                p.rows, p.inverse, p.bag_of, c.nnz, c.N, out, p.counts, c.weighted ? p.wpos : nullptr);
+        }
+        // the multi-hot sum exits at once on one-hot batches: one wave of CTAs, not four
+        k_pool<4><<<grid_for(c, total / 16, 256, 8), 256, 0, s>>>(p.rows, p.inverse, offsets, c.nnz,
                                                                  c.T, c.B, c.N, out, p.counts, 1,
                                                                  c.weighted ? p.wpos : nullptr);
       }

@@ -220,6 +220,9 @@ k_build_keys(const IdxT* __restrict__ indices, const int64_t* __restrict__ offse
 
 // ------------------------------------------------------------------------------------
 // a2: onesweep LSD radix sort, 8-bit digits
+#ifndef TTEMB_KEYS_PER_SM
+#define TTEMB_KEYS_PER_SM 4   // k_build_keys grid cap, CTAs per SM
+#endif
 #ifndef TTEMB_RS_IPT
 #define TTEMB_RS_IPT 8    // keys per thread (tile = 256 x RS_IPT; 8 beats 16 and 4 at C4)
 #endif
@@ -663,7 +666,8 @@ cudaError_t run_index_stage(Ctx& c, const void* indices, const int64_t* offsets,
       cudaMemsetAsync(p.bag_of, 0, sizeof(uint32_t) * nnz, s);
     }
     const int64_t bags = (int64_t)c.T * c.B;
-    const int g = grid_for(c, bags > 0 ? bags : 1, 256, 32);
+    // fewer CTAs than bags (grid-stride): each CTA flushes up to passes x 256 histogram atomics
+    const int g = grid_for(c, bags > 0 ? bags : 1, 256, TTEMB_KEYS_PER_SM);
     if (c.index_bits == 64)
       k_build_keys<int64_t><<<g, 256, 0, s>>>((const int64_t*)indices, offsets, nnz, c.B, c.T,
                                               c.d_meta, p.keysA, p.bag_of, p.counts,

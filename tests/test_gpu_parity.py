@@ -420,13 +420,15 @@ def test_bijection_out_of_range_is_reported():
 
 
 @pytest.mark.parametrize("mode,weighted", [("mean", False), ("sum", True)], ids=["mean", "weighted"])
-@pytest.mark.parametrize("case", ["multi-var-L", "tc-n1-2", "c4-b1024-var"])
+@pytest.mark.parametrize("case", ["multi-var-L", "tc-n1-2", "c4-b1024-var", "c4-b1000-one"])
 def test_mean_and_weighted_bags(case, mode, weighted):
     """nn.EmbeddingBag mode="mean" (TTEMB_MEAN_POOLING) and per-sample weights
     (ttemb_forward_weighted) vs the oracle's definition (P:48 / P:306 drop-in); variable bag
-    lengths with empty bags; the backward differentiates the weighted bags."""
+    lengths with empty bags; the backward differentiates the weighted bags.  The one-hot case
+    (B = 1000, ragged against every tile) runs the output-ordered one-hot pooling kernel."""
     if case.startswith("c4"):
-        cfg, mode_in, B = W.config("c4"), "var", 1024
+        cfg, B = W.config("c4"), int(case.split("-")[1][1:])
+        mode_in = "var" if case.endswith("var") else None
     else:
         cfg, mode_in = {c[0]: (c[1], c[2]) for c in small_cases()}[case]
         mode_in, B = "var", None
