@@ -12,6 +12,10 @@
 
 #include "ttemb_internal.cuh"
 
+#ifndef TTEMB_AGG_LDCS
+#define TTEMB_AGG_LDCS 1      // 1 = streaming loads of grad_out in the one-hot aggregation
+#endif
+
 namespace ttemb {
 
 namespace {
@@ -134,9 +138,11 @@ __global__ void __launch_bounds__(256) k_zero_rows(float* __restrict__ buf, cons
 __global__ void __launch_bounds__(256)
 k_agg_scatter(const float* __restrict__ grad_out, const uint32_t* __restrict__ sbag,
               const uint32_t* __restrict__ spos, const uint32_t* __restrict__ inverse, int64_t nnz, int N,
-              float* __restrict__ gbuf, const float* __restrict__ wpos) {
+              float* __restrict__ gbuf, const float* __restrict__ wpos, const uint32_t* __restrict__ counts) {
   const int lane = threadIdx.x & 31;
-  const int NV = N >> 2, P = 32 / NV;            // float4 columns; occurrences in flight per step
+  const int NV = N >> 2, P = 32 / NV;
+  // one id per bag: every grad_out row is read exactly once -> evict-first loads keep L2 for G
+  const bool once = TTEMB_AGG_LDCS && __ldg(counts + kCntMulti) == 0;            // float4 columns; occurrences in flight per step
   const int f = lane % NV, p = lane / NV;
   const int64_t nch = (nnz + 31) / 32;
   const int64_t nw = (int64_t)gridDim.x * (blockDim.x >> 5);
@@ -166,7 +172,8 @@ k_agg_scatter(const float* __restrict__ grad_out, const uint32_t* __restrict__ s
           acc = make_float4(0.f, 0.f, 0.f, 0.f);
           cur = u;
         }
-        const float4 v = __ldg(reinterpret_cast<const float4*>(grad_out + (size_t)bag * N) + f);
+        const float4* gp = reinterpret_cast<const float4*>(grad_out + (size_t)bag * N) + f;
+        const float4 v = once ? __ldcs(gp) : __ldg(gp);
         acc.x += w * v.x; acc.y += w * v.y; acc.z += w * v.z; acc.w += w * v.w;
       }
     }
@@ -306,7 +313,7 @@ cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s
       // (G was zeroed at the end of the index stage: run_plan_tail)
       k_agg_scatter<<<grid_for(c, cdiv(c.nnz, 32), 8, 32), 256, 0, s>>>(grad_out, p.sbag, p.spos, p.inverse,
                                                                          c.nnz, c.N, p.gbuf,
-                                                                         c.weighted ? p.wpos : nullptr);
+                                                                         c.weighted ? p.wpos : nullptr, p.counts);
     } else {
       const int64_t total = agg_chunks(c.nnz) * c.N;
       if (c.N % 4 == 0)
