@@ -68,6 +68,11 @@ __device__ __forceinline__ float tf32_trunc(float x) { return __uint_as_float(__
 __device__ __forceinline__ void cp_async16(uint32_t dst, const void* src) {
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(src) : "memory");
 }
+// 16-byte copy of data read once: L2 evict-first cache policy.
+__device__ __forceinline__ void cp_async16_ef(uint32_t dst, const void* src) {
+  asm volatile("{\n .reg .b64 pol;\n createpolicy.fractional.L2::evict_first.b64 pol, 1.0;\n"
+               " cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, pol;\n}" ::"r"(dst), "l"(src) : "memory");
+}
 // 16-byte copy that writes zeros when !valid (src-size 0).
 __device__ __forceinline__ void cp_async16_z(uint32_t dst, const void* src, bool valid) {
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(valid ? 16 : 0) : "memory");

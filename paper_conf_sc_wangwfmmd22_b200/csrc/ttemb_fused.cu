@@ -25,6 +25,10 @@
 #include "tc.cuh"
 #include "ttemb_internal.cuh"
 
+#ifndef TTEMB_G_EVICT_FIRST
+#define TTEMB_G_EVICT_FIRST 0  // 1 = L2 evict-first policy on k_rows_bwd2's reads of G
+#endif
+
 namespace ttemb {
 
 namespace {
@@ -547,8 +551,13 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 2) k_rows_bwd2(RowBwdArgs a) {
         tc::cp_async16(dst + 4u * (uint32_t)(4 * f + 4 * ((r >> 3) & 7)), src + f);
       }
       if (lane < a.N / 4)
+#if TTEMB_G_EVICT_FIRST
+        tc::cp_async16_ef(dst + 4u * (uint32_t)(C3S + 4 * lane),   // G row: read once
+                          reinterpret_cast<const float4*>(a.gbuf + (size_t)(u0 + j) * a.N) + lane);
+#else
         tc::cp_async16(dst + 4u * (uint32_t)(C3S + 4 * lane),
                        reinterpret_cast<const float4*>(a.gbuf + (size_t)(u0 + j) * a.N) + lane);
+#endif
     };
 #pragma unroll
     for (int j = 0; j < RW_NSL - 1; ++j) {
