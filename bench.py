@@ -100,40 +100,75 @@ class Clocks:
 # ---------------------------------------------------------------------------
 # algorithmic work
 # ---------------------------------------------------------------------------
-def step_work(cfg, B, nnz, counts, touched, opt):
+def step_work(cfg, B, nnz, counts, touched, opt, tc):
+    """(tensor_flops, alu_flops, bytes) of one step: the rank-R prefix contractions (fwd a5 + bwd
+    a10, 3 x 2 n1 n2 R^2 per unique prefix) on tcgen05 when `tc`, the row contractions (a6, a9:
+    3 x 2 N R per unique row) on FFMA; bytes per SURVEY 8(d)."""
     n1, n2, n3 = cfg.col_factors
     R, N, T = cfg.rank, cfg.dim, cfg.num_tables
     U, P = counts["U"], counts["P"]
     nd = touched.get("dense_rows", 0)                  # hybrid: plain rows (no TT arithmetic)
-    flops = 3 * 2 * n1 * n2 * R * R * P + 3 * 2 * N * R * (U - nd)
+    pf = 3 * 2 * n1 * n2 * R * R * P
+    rf = 3 * 2 * N * R * (U - nd)
     slice_bytes = 4 * (touched["c1"] * n1 * R + touched["c2"] * R * n2 * R + touched["c3"] * R * n3
                        + nd * N)
     passes = 3 if opt == "sgd" else 5                  # fwd read, bwd read, update write (+ state r/w)
     bytes_ = 8 * nnz + 8 * (T * B + 1) + 2 * 4 * N * T * B + passes * slice_bytes
-    return flops, bytes_
+    return (pf if tc else 0), rf + (0 if tc else pf), bytes_
 
 
 def stage_work(name, cfg, B, nnz, counts, tc=False):
-    """(flops, bytes, bound) of one launch of a stage, algorithmic.  On the tcgen05 path the
-    rank-R contractions are bound by the tensor pipe ("tensor"), else by FP32 FFMA ("alu")."""
+    """Algorithmic work of one launch of a stage: (tensor_flops, alu_flops, bytes).
+    tensor_flops are the rank-R prefix contractions when they run on tcgen05 (3xTF32), alu_flops
+    the FP32 FFMA work (row contractions; the prefix contractions on the FFMA path), bytes the
+    algorithmic HBM bytes (touched slices, ids, out / grad_out; intermediates a
+    fused design keeps on chip are not counted)."""
     n1, n2, n3 = cfg.col_factors
     R, N, T = cfg.rank, cfg.dim, cfg.num_tables
     U, P, NG = counts["U"], counts["P"], counts["NG"]
-    if name == "fwd_prefix":
-        return 2 * n1 * n2 * R * R * P, 4 * (NG * R * n2 * R + P * n1 * R), "tensor" if tc else "alu"
-    if name == "bwd_prefix":
-        return 4 * n1 * n2 * R * R * P, 4 * (2 * NG * R * n2 * R + P * n1 * R), "tensor" if tc else "alu"
+    c2 = 4 * NG * R * n2 * R
+    pf = 2 * n1 * n2 * R * R * P
+
+    def split(f):
+        return (f, 0) if tc else (0, f)
+    if name == "fwd_prefix":                      # a5 (+ a6 when fused)
+        return (*split(pf), c2 + 4 * P * n1 * R)
     if name == "fwd_rows":
-        return 2 * N * R * U, 4 * U * N, "alu"
+        return 0, 2 * N * R * U, 4 * U * N
+    if name == "fwd_fused":                       # a5 + a6 (+ a7 for one-id bags)
+        return (*split(pf), 2 * N * R * U, c2 + 4 * P * n1 * R + 4 * N * T * B)
+    if name == "bwd_prefix":                      # a10 - a12
+        return (*split(2 * pf), 2 * c2 + 4 * P * n1 * R)
     if name == "bwd_rows":
-        return 4 * N * R * U, 4 * U * N, "alu"
+        return 0, 4 * N * R * U, 4 * U * N
+    if name == "bwd_fused":                       # a9 - a12 (prefix recomputed on chip)
+        return (*split(3 * pf), 4 * N * R * U, 2 * c2 + 4 * P * n1 * R + 4 * U * N)
     if name == "pool":
-        return 0, 4 * N * T * B + 4 * N * nnz + 4 * nnz + 8 * (T * B + 1), "hbm"
+        return 0, 0, 4 * N * T * B + 4 * N * nnz + 4 * nnz + 8 * (T * B + 1)
     if name == "agg":
-        return 0, 4 * N * nnz + 8 * nnz + 4 * N * U, "hbm"
+        return 0, 0, 4 * N * nnz + 8 * nnz + 4 * N * U
     if name == "sort_pass":
-        return 0, 16 * nnz, "hbm"
-    return 0, 0, "hbm"
+        return 0, 0, 16 * nnz
+    return 0, 0, 0
+
+
+def kernel_roofline(name, work, per_launch_ms, hbm_peak, tensor_peak, alu_peak):
+    """The binding roofline of one launch: the largest of (tensor flops at the 3xTF32 peak, FFMA
+    flops at the FP32 peak, algorithmic bytes at the HBM peak); achieved = that quantity per
+    measured launch time, frac = floor time / measured time."""
+    tf, af, by = work
+    t = {"tensor": tf / (tensor_peak * 1e12), "alu": af / (alu_peak * 1e12), "hbm": by / (hbm_peak * 1e9)}
+    bound = max(t, key=t.get)
+    sec = per_launch_ms / 1e3
+    if bound == "hbm":
+        ach, peak, unit = by / sec / 1e9, hbm_peak, "GB/s"
+    elif bound == "tensor":
+        ach, peak, unit = tf / sec / 1e12, tensor_peak, "TFLOP/s"
+    else:
+        ach, peak, unit = af / sec / 1e12, alu_peak, "TFLOP/s"
+    return {"bound": bound, "kernel": name, "achieved": ach, "peak": peak, "unit": unit, "frac": ach / peak,
+            "floors_us": {k: round(v * 1e6, 2) for k, v in t.items()}, "measured_us": round(per_launch_ms * 1e3, 2),
+            "work": {"tensor_gflop": tf / 1e9, "alu_gflop": af / 1e9, "alg_mb": by / 1e6}}
 
 
 # ---------------------------------------------------------------------------
@@ -393,7 +428,7 @@ def main():
             go = W.make_grad_out(cfg, B, step=i, seed=args.seed + 1000 * rank)
         else:
             gi, goff = W.make_batch(cfg, step=i, seed=args.seed)
-            idx, off, _ = parallel.shard_bags(gi, goff, cfg.num_tables, cfg.batch, rank, world)
+            idx, off, _ = W.shard_batch(gi, goff, cfg.num_tables, cfg.batch, rank, world)
             go = W.make_grad_out(cfg, cfg.batch, step=i, seed=args.seed)[rank * B:(rank + 1) * B].copy()
         pool.append((idx, off, go))
     max_nnz = max(len(p[0]) for p in pool)
@@ -541,43 +576,36 @@ def main():
     on_tc = tc_path(cfg, args)
     sm_count = torch.cuda.get_device_properties(dev).multi_processor_count
     alu_peak = fp32_peak_tflops(sm_count, sm_max_mhz)
-    flops, bytes_ = step_work(cfg, B, nnz_last, counts, touched, args.opt)
+    tflops, aflops, bytes_ = step_work(cfg, B, nnz_last, counts, touched, args.opt, on_tc)
+    tensor_peak = bf16_peak / 2.0 / 3.0          # 3xTF32: 3 TF32 MMAs per fp32 product, TF32 = bf16 / 2
     ms_step = t_ms / args.steps
-    # dominant stage
+    # dominant kernel (stage) of the eager breakdown; its binding roofline
     dom = max(stages.items(), key=lambda kv: kv[1][0])
     dname, (dms, dn) = dom
-    f1, b1, bound = stage_work(dname, cfg, B, nnz_last, counts, tc=on_tc)
     per_launch_ms = dms / max(dn, 1)
-    if bound == "tensor":
-        # 3xTF32: each fp32 product costs 3 TF32 MMAs; TF32 dense = bf16 / 2 (nominal ratio)
-        tpk = bf16_peak / 2.0 / 3.0
-        ach = f1 / (per_launch_ms / 1e3) / 1e12
-        roof = {"bound": "tensor", "kernel": dname, "achieved": ach, "peak": tpk, "unit": "TFLOP/s",
-                "frac": ach / tpk, "traffic": None,
-                "peak_source": f"{peak_kind} bf16 {bf16_peak:.0f} TFLOP/s x 1/2 (tf32) x 1/3 (3xTF32), "
-                               "fp32-equivalent algorithmic FLOPs"}
-    elif bound == "alu":
-        ach = f1 / (per_launch_ms / 1e3) / 1e12
-        roof = {"bound": "alu", "kernel": dname, "achieved": ach, "peak": alu_peak, "unit": "TFLOP/s",
-                "frac": ach / alu_peak, "traffic": None,
-                "peak_source": f"derived: {sm_count} SM x 128 FP32 FMA/clk x 2 x {sm_max_mhz:.0f} MHz"}
-    else:
-        ach = b1 / (per_launch_ms / 1e3) / 1e9
-        roof = {"bound": "hbm", "kernel": dname, "achieved": ach, "peak": hbm_peak, "unit": "GB/s",
-                "frac": ach / hbm_peak, "traffic": None, "peak_source": f"{peak_kind} copy bandwidth"}
+    roof = kernel_roofline(dname, stage_work(dname, cfg, B, nnz_last, counts, tc=on_tc), per_launch_ms,
+                           hbm_peak, tensor_peak, alu_peak)
+    roof["peak_source"] = {"hbm": f"{peak_kind} copy bandwidth (MEASURED_PEAKS.json hbm_gbs)",
+                           "tensor": f"{peak_kind} bf16 {bf16_peak:.0f} TFLOP/s x 1/2 (tf32) x 1/3 (3xTF32)",
+                           "alu": f"derived: {sm_count} SM x 128 FP32 FMA/clk x 2 x {sm_max_mhz:.0f} MHz"}[roof["bound"]]
     roof["share_of_step"] = dms / max(stage_total_ms, 1e-9)
+    roof["traffic"] = None
     tr_path = os.path.join(ROOT, "profiles", "traffic.json")
-    if os.path.exists(tr_path):      # DRAM bytes per launch from the committed ncu --set full capture
+    if os.path.exists(tr_path):      # DRAM bytes per launch from a committed ncu --set full capture of THIS config
         tr = json.load(open(tr_path))
-        if dname in tr.get("dram_bytes_per_launch", {}):
-            roof["traffic"] = tr["dram_bytes_per_launch"][dname]
+        key = f"{cfg.name}-r{cfg.rank}/{dname}"
+        if key in tr.get("dram_bytes_per_launch", {}):
+            roof["traffic"] = tr["dram_bytes_per_launch"][key]
             roof["traffic_source"] = tr.get("source")
-            roof["alg_bytes_per_launch"] = b1
-    t_alu = flops / (alu_peak * 1e12) * 1e3
+    t_tc = tflops / (tensor_peak * 1e12) * 1e3
+    t_alu = aflops / (alu_peak * 1e12) * 1e3
     t_hbm = bytes_ / (hbm_peak * 1e9) * 1e3
-    step_roof = {"alg_gflop": flops / 1e9, "alg_mb": bytes_ / 1e6, "t_alu_ms": t_alu, "t_hbm_ms": t_hbm,
-                 "frac_hbm_roofline": t_hbm / ms_step, "frac_binding_roofline": max(t_alu, t_hbm) / ms_step,
-                 "binding": "alu" if t_alu > t_hbm else "hbm", "U": counts["U"], "P": counts["P"],
+    t_cmp = t_tc + t_alu                           # tensor and FFMA work counted serially
+    step_roof = {"alg_gflop_tensor": tflops / 1e9, "alg_gflop_alu": aflops / 1e9, "alg_mb": bytes_ / 1e6,
+                 "t_tensor_ms": t_tc, "t_alu_ms": t_alu, "t_hbm_ms": t_hbm,
+                 "frac_hbm_roofline": t_hbm / ms_step, "frac_binding_roofline": max(t_cmp, t_hbm) / ms_step,
+                 "binding": "hbm" if t_hbm >= t_cmp else ("tensor+alu" if t_tc and t_alu else "alu"),
+                 "U": counts["U"], "P": counts["P"],
                  "NG": counts["NG"], "touched_slices": touched}
 
     # ---- end-to-end through the host-buffer ABI calls ----

@@ -110,9 +110,15 @@ int ttemb_query_sizes(const ttemb_config* cfg, size_t* core_bytes, size_t* state
  * ttemb_query_sizes; 256-byte aligned): cores (parameters, initialised by the
  * caller via ttemb_core_layout), state (Adagrad accumulator, zero-initialised
  * by the caller; may be NULL for SGD), grads (dense dL/dC, same layout as
- * cores; written by ttemb_backward, read by ttemb_update; safe to all-reduce
- * in place between the two), workspace (scratch).  `device` is the CUDA
- * ordinal the buffers live on.  On success *out is a new handle. */
+ * cores, ZERO-initialised by the caller; written by ttemb_backward, read by
+ * ttemb_update; safe to all-reduce in place between the two; with
+ * TTEMB_FUSED_UPDATE the backward keeps it zero between steps), workspace
+ * (scratch).  ttemb_create enqueues no device work and never touches these
+ * buffers, so a second handle on the same cores / state / grads (cross-step
+ * pipelining, ttemb_plan_batch) may be created at any time.  `device` is the
+ * CUDA ordinal the buffers live on.  On success *out is a new handle.
+ * Errors: INVALID_ARG (null / misaligned pointers, bad factors, Adagrad with
+ * adagrad_eps <= 0), UNSUPPORTED (limits), CUDA. */
 int ttemb_create(const ttemb_config* cfg, int device, void* cores, void* state, void* grads,
                  void* workspace, ttemb_t* out);
 int ttemb_destroy(ttemb_t h);
@@ -133,7 +139,8 @@ int ttemb_forward(ttemb_t h, const void* indices, const int64_t* offsets, int64_
 /* Backward of the last forward: grad_out [batch][T][dim] float32 (device).
  * Without TTEMB_FUSED_UPDATE it overwrites the whole grads buffer with dL/dC
  * (untouched slices 0); with it, it applies the update with `lr` instead
- * (grads then holds scratch). */
+ * (grads then stays zero).  Exactly one backward per forward: a second call
+ * (or one without a forward) returns TTEMB_ERR_STATE. */
 int ttemb_backward(ttemb_t h, const float* grad_out, float lr, void* stream);
 
 /* Optimizer step from the grads buffer (after an optional all-reduce SUM).
@@ -157,11 +164,16 @@ int ttemb_check(ttemb_t h, void* stream);
 typedef struct {
   int64_t nnz;
   int32_t batch;
-  const uint32_t* counts;    /* [4] U, P, NG, error flags                              */
-  const uint32_t* skey;      /* [nnz] sorted keys, key = rowbase_t + id                */
+  const uint32_t* counts;    /* [16] U, P, NG, error flags, ... (ttemb_read_counts)    */
+  const uint32_t* skey;      /* [nnz] sorted plan keys (R29): for a TT table
+                                 key = kbase_t + (i2 m1 + i1) m3 + i3 with the digits of
+                                 Eq. 3 and kbase_t = sum of m1 m2 m3 over earlier TT
+                                 tables; dense (hybrid) tables follow all TT keys with
+                                 key = kbase_t + id.  A bijection of (t, row) for valid ids,
+                                 ordered by (t, i2, i1, i3)                                */
   const uint32_t* spos;      /* [nnz] stable argsort of the keys                       */
   const uint32_t* bag_of;    /* [nnz] output row b*T + t of position j                 */
-  const uint32_t* ukey;      /* [U] distinct keys, ascending                            */
+  const uint32_t* ukey;      /* [U] distinct plan keys, ascending                       */
   const uint32_t* seg_off;   /* [U+1] sorted-position segment of each unique row        */
   const uint32_t* inverse;   /* [nnz] unique slot of position j                         */
   const uint32_t* row_pfx;   /* [U] prefix slot of each unique row                      */
@@ -170,7 +182,9 @@ typedef struct {
   const uint32_t* pfx_i1;    /* [P] first digit                                         */
   const uint32_t* pfx_i2;    /* [P] second digit                                        */
   const uint32_t* row_seg;   /* [P+1] unique rows of each prefix                        */
-  const uint32_t* grp_pfx;   /* [P] prefixes ordered by (t, i2, i1)                     */
+  const uint32_t* grp_pfx;   /* [P] prefix slot of the q-th prefix in (t, i2, i1) order;
+                                 the identity, because the plan key already orders the
+                                 prefixes that way (kept for ABI stability)            */
   const uint32_t* grp_off;   /* [NG+1] i2-groups (one C2 slice each)                    */
   const uint32_t* grp_t;     /* [NG] */
   const uint32_t* grp_i2;    /* [NG] */

@@ -208,7 +208,7 @@ static int64_t find_key(const uint32_t* ukey, int64_t U, uint32_t key) {
 /* Plan                                                                      */
 /* ------------------------------------------------------------------------ */
 /* The plan orders distinct rows "group-major": by table t, then the C2 digit i2, then the C1
- * digit i1, then i3 (R23), i.e. by the plan key
+ * digit i1, then i3 (R29), i.e. by the plan key
  *     K(t, i) = gbase_t + (i2 * m1 + i1) * m3 + i3,   gbase_t = sum_{t' < t} m1 m2 m3,
  * with (i1, i2, i3) the digits of Eq. 3.  Rows sharing a prefix (i1, i2) (Alg. 1's
  * Buf_idx = idx / length_3) are then consecutive, and prefixes sharing a C2 slice

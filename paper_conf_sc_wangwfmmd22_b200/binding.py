@@ -368,6 +368,15 @@ class TTEmbeddingBag:
         U, P, NG, err = ttemb_read_counts(self.h, _stream_ptr(stream))
         return dict(U=U, P=P, NG=NG, err=err)
 
+    def all_counts(self, stream=None) -> Dict[str, int]:
+        """Every device counter of the last forward's plan (include/ttemb.h ttemb_plan.counts):
+        U, P, NG, error flags, multi-id-bag flag, Utt + 1, FFMA work units, split i2-groups."""
+        torch.cuda.synchronize(self.device)
+        p = ttemb_get_plan(self.h)
+        v = _copy_device_u32(p.counts, 16, self.device).cpu().numpy().view("uint32")
+        names = ("U", "P", "NG", "err", "multi", "utt1", "nchunks", "nsplit")
+        return {k: int(v[i]) for i, k in enumerate(names)}
+
     def plan(self, stream=None) -> Dict[str, torch.Tensor]:
         """Copies of the index-stage outputs of the last forward (sizes from the counts)."""
         c = self.counts(stream)

@@ -73,6 +73,11 @@ int validate(const ttemb_config* cfg) {
   if (cfg->max_nnz > (int64_t(1) << 30)) return TTEMB_ERR_UNSUPPORTED;
   if ((int64_t)cfg->num_tables * cfg->max_batch > (int64_t(1) << 31)) return TTEMB_ERR_UNSUPPORTED;
   if (cfg->optimizer != TTEMB_SGD && cfg->optimizer != TTEMB_ADAGRAD) return TTEMB_ERR_INVALID_ARG;
+  // Adagrad divides by sqrt(S) + eps; the fused C2 pass also visits zero-gradient entries, so
+  // eps = 0 would turn untouched (e.g. rank-padding) entries into 0/0
+  if (cfg->optimizer == TTEMB_ADAGRAD && !(cfg->adagrad_eps > 0.f)) return TTEMB_ERR_INVALID_ARG;
+  // pooled output / gradient element counts stay below 2^31 (32-bit element indexing)
+  if ((int64_t)cfg->num_tables * cfg->max_batch * cfg->dim >= (int64_t(1) << 31)) return TTEMB_ERR_UNSUPPORTED;
   if (cfg->flags & ~(TTEMB_FUSED_UPDATE | TTEMB_FP32_CORES | TTEMB_NO_PREFIX_REUSE | TTEMB_NO_AGGREGATION |
                      TTEMB_MEAN_POOLING))
     return TTEMB_ERR_INVALID_ARG;
@@ -335,8 +340,9 @@ int ttemb_create(const ttemb_config* cfg, int device, void* cores, void* state, 
   if (e == cudaSuccess) e = configure_tc(c);
   if (e == cudaSuccess) e = configure_fused(c);
   if (e == cudaSuccess) e = configure_bwdtc(c);
-  // fused backward keeps the C1 / C3 gradient accumulators zero between steps (k_update_zero)
-  if (e == cudaSuccess) e = cudaMemset(c.grads, 0, sizeof(float) * c.core_floats);
+  // (the caller hands in a zeroed grads buffer -- include/ttemb.h; the fused backward keeps the
+  // C1 / C3 accumulators zero between steps, so a second handle on the same buffers, created
+  // mid-training, must not and does not touch them)
   if (e != cudaSuccess) {
     fprintf(stderr, "ttemb_create: %s\n", cudaGetErrorString(e));
     delete h;
@@ -431,13 +437,16 @@ int ttemb_forward_planned(ttemb_t h, float* out, void* stream) {
   }
   c.planned = false;
   c.fwd_done = true;
+  c.bwd_done = false;
   return TTEMB_OK;
 }
 
 int ttemb_backward(ttemb_t h, const float* grad_out, float lr, void* stream) {
   if (!h) return TTEMB_ERR_INVALID_ARG;
   Ctx& c = h->c;
-  if (!c.fwd_done) return TTEMB_ERR_STATE;
+  // one backward per forward: the plan-dependent accumulators (aggregated rows, straddling dP
+  // rows) are zeroed by the index stage and consumed by the backward
+  if (!c.fwd_done || c.bwd_done) return TTEMB_ERR_STATE;
   if (!grad_out && c.B > 0) return TTEMB_ERR_INVALID_ARG;
   DeviceGuard dg(c.device);
   cudaError_t e = run_backward(c, grad_out, lr, (cudaStream_t)stream);
@@ -445,6 +454,7 @@ int ttemb_backward(ttemb_t h, const float* grad_out, float lr, void* stream) {
     fprintf(stderr, "ttemb_backward: %s\n", cudaGetErrorString(e));
     return TTEMB_ERR_CUDA;
   }
+  c.bwd_done = true;
   return TTEMB_OK;
 }
 
@@ -486,7 +496,7 @@ int ttemb_forward_host(ttemb_t h, const void* host_indices, const int64_t* host_
 int ttemb_backward_host(ttemb_t h, const float* host_grad_out, float lr, void* stream) {
   if (!h) return TTEMB_ERR_INVALID_ARG;
   Ctx& c = h->c;
-  if (!c.fwd_done) return TTEMB_ERR_STATE;
+  if (!c.fwd_done || c.bwd_done) return TTEMB_ERR_STATE;
   if (!host_grad_out && c.B > 0) return TTEMB_ERR_INVALID_ARG;
   DeviceGuard dg(c.device);
   cudaStream_t s = (cudaStream_t)stream;

@@ -140,9 +140,9 @@ k_agg_scatter(const float* __restrict__ grad_out, const uint32_t* __restrict__ s
               const uint32_t* __restrict__ spos, const uint32_t* __restrict__ inverse, int64_t nnz, int N,
               float* __restrict__ gbuf, const float* __restrict__ wpos, const uint32_t* __restrict__ counts) {
   const int lane = threadIdx.x & 31;
-  const int NV = N >> 2, P = 32 / NV;
+  const int NV = N >> 2, P = 32 / NV;   // float4 columns; occurrences in flight per step
   // one id per bag: every grad_out row is read exactly once -> evict-first loads keep L2 for G
-  const bool once = TTEMB_AGG_LDCS && __ldg(counts + kCntMulti) == 0;            // float4 columns; occurrences in flight per step
+  const bool once = TTEMB_AGG_LDCS && __ldg(counts + kCntMulti) == 0;
   const int f = lane % NV, p = lane / NV;
   const int64_t nch = (nnz + 31) / 32;
   const int64_t nw = (int64_t)gridDim.x * (blockDim.x >> 5);

@@ -662,9 +662,11 @@ size_t rows_bwd_smem(int n3) { return (size_t)RW_WARPS * RW_NSL * (XR * n3 + 32 
 }  // namespace
 
 bool fused_eligible(const Ctx& c) {
-  return !(c.flags & TTEMB_FP32_CORES) && !knobs().old_fwd && c.R == XR && c.NC <= 256 &&
+  return !(c.flags & TTEMB_FP32_CORES) && c.R == XR && c.NC <= 256 &&
          (c.n3 == 4 || c.n3 == 8) && (c.n1 == 1 || c.n1 == 2 || c.n1 == 4 || c.n1 == 8) && c.n1 * c.n2 <= 16;
 }
+bool tc_eligible(const Ctx& c) { return fused_eligible(c); }
+cudaError_t configure_tc(Ctx&) { return cudaSuccess; }
 
 cudaError_t configure_fused(Ctx& c) {
   if (!fused_eligible(c)) return cudaSuccess;
@@ -761,6 +763,20 @@ cudaError_t run_rows_bwd2(Ctx& c, cudaStream_t s) {
   if (c.n3 == 4) k_rows_bwd2<4><<<grid, RW_WARPS * 32, rows_bwd_smem(4), s>>>(r);
   else k_rows_bwd2<8><<<grid, RW_WARPS * 32, rows_bwd_smem(8), s>>>(r);
   return cudaGetLastError();
+}
+
+// Forward contractions on tcgen05: P (k_prefix_fwd) then rows (k_rows_fwd2).
+cudaError_t run_tc_fwd(Ctx& c, float* out, cudaStream_t s) { return run_fused_fwd(c, out, s); }
+
+// Backward contractions: dP / dC3 row stage, then the prefix GEMMs (dC2, dA) with the fused update.
+cudaError_t run_tc_bwd(Ctx& c, float lr, cudaStream_t s) {
+  cudaError_t e;
+  {
+    StageScope sc(c, ST_BWD_ROWS, s);
+    e = run_rows_bwd2(c, s);
+  }
+  if (e == cudaSuccess) e = run_prefix_bwd(c, lr, s);
+  return e;
 }
 
 }  // namespace ttemb

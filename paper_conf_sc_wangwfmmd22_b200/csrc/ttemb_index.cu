@@ -343,147 +343,11 @@ k_radix_pass(const uint32_t* __restrict__ kin, const uint32_t* __restrict__ vin,
 }
 
 // ------------------------------------------------------------------------------------
-// Single-pass scan skeleton: flags -> exclusive slots, with decoupled look-back.
-// Body provides size(), flag(i), emit(i, slot, flag), finish(total).
+// Plan scan tiles: 256 threads x 8 occurrences (SC_IPT * 8 == 64 warp counts).
 // ------------------------------------------------------------------------------------
 constexpr int SC_T = 256, SC_IPT = 8, SC_TILE = SC_T * SC_IPT;   // SC_IPT * 8 == 64 warp counts
 
-template <class Body>
-__global__ void __launch_bounds__(SC_T) k_scan(Body body, uint32_t* status, uint32_t* counter) {
-  __shared__ uint32_t s_wc[SC_IPT * 8];
-  __shared__ uint32_t s_tile, s_base, s_total;
-  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
-  if (tid == 0) s_tile = atomicAdd(counter, 1u);
-  __syncthreads();
-  const uint32_t n = body.size();
-  const uint32_t tile = s_tile, base = tile * SC_TILE;
-  if (n == 0) {
-    if (tile == 0 && tid == 0) body.finish(0);
-    return;
-  }
-  if (base >= n) return;
-  uint32_t ball[SC_IPT];
-#pragma unroll
-  for (int k = 0; k < SC_IPT; ++k) {
-    const uint32_t i = base + k * SC_T + tid;
-    const bool f = (i < n) && body.flag(i);
-    ball[k] = __ballot_sync(FULL, f);
-    if (lane == 0) s_wc[k * 8 + w] = __popc(ball[k]);
-  }
-  __syncthreads();
-  if (w == 0) {   // exclusive scan of the 64 warp counts, k-major
-    const uint32_t a = s_wc[2 * lane], b = s_wc[2 * lane + 1];
-    uint32_t x = a + b;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const uint32_t y = __shfl_up_sync(FULL, x, o);
-      if (lane >= o) x += y;
-    }
-    const uint32_t ex = x - a - b;
-    s_wc[2 * lane] = ex;
-    s_wc[2 * lane + 1] = ex + a;
-    if (lane == 31) s_total = x;
-  }
-  __syncthreads();
-  if (w == 0) {
-    const uint32_t b = lookback_warp(status, tile, s_total);
-    if (lane == 0) s_base = b;
-  }
-  __syncthreads();
-  const uint32_t lt = lanemask_lt();
-#pragma unroll
-  for (int k = 0; k < SC_IPT; ++k) {
-    const uint32_t i = base + k * SC_T + tid;
-    if (i < n) {
-      const uint32_t f = (ball[k] >> lane) & 1u;
-      const uint32_t slot = s_base + s_wc[k * 8 + w] + __popc(ball[k] & lt);
-      body.emit(i, slot, f);
-    }
-  }
-  if (base + SC_TILE >= n && tid == 0) body.finish(s_base + s_total);
-}
-
-// a3: unique rows / segments / inverse over the sorted keys
-struct UniqueBody {
-  const uint32_t* skey; const uint32_t* spos; const uint32_t* bag_of;
-  uint32_t* ukey; uint32_t* seg_off; uint32_t* inverse; uint32_t* sbag; uint32_t* counts;
-  uint32_t nnz;
-  uint32_t every;   // TTEMB_NO_AGGREGATION: each occurrence is its own row
-  uint64_t tt_keys; // keys >= tt_keys are rows of dense (hybrid) tables
-  __device__ uint32_t size() const { return nnz; }
-  __device__ bool flag(uint32_t k) const { return every || k == 0 || skey[k] != skey[k - 1]; }
-  __device__ void emit(uint32_t k, uint32_t slot, uint32_t f) const {
-    const uint32_t u = f ? slot : slot - 1;
-    if (f) {
-      ukey[u] = skey[k]; seg_off[u] = k;
-      if (skey[k] >= tt_keys && (k == 0 || skey[k - 1] < tt_keys)) counts[kCntUtt1] = u + 1;
-    }
-    const uint32_t pos = spos[k];
-    inverse[pos] = u;
-    sbag[k] = bag_of[pos];
-  }
-  __device__ void finish(uint32_t U) const { counts[kCntU] = U; seg_off[U] = nnz; }
-};
-
-
-// a4: TT digits (Eq. 3) and unique prefixes (runs of (t, i2 m1 + i1)) over the unique rows
-struct PrefixBody {
-  const uint32_t* ukey; const uint64_t* kbase; const uint32_t* kmap; const TableMeta* meta; int T;
-  uint32_t* row_pfx; uint32_t* row_i3; uint32_t* pfx_t; uint32_t* pfx_i1; uint32_t* pfx_i2;
-  uint32_t* row_seg; uint32_t* counts;
-  uint32_t every;   // TTEMB_NO_PREFIX_REUSE: each row is its own prefix
-  __device__ uint32_t size() const { return counts[kCntU]; }
-  __device__ void decode(uint32_t u, int& t, uint32_t& pq, uint32_t& i3) const {
-    const uint32_t key = ukey[u];
-    const int it = table_of_key(kbase, T, key);      // key ranges are in key order
-    t = (int)__ldg(kmap + it);
-    const uint32_t local = (uint32_t)(key - __ldg(kbase + it));
-    const uint32_t m3 = meta[t].m3;
-    pq = local / m3;                  // i2 * m1 + i1
-    i3 = local - pq * m3;
-  }
-  __device__ bool is_dense_row(uint32_t u) const { return counts[kCntUtt1] && u >= counts[kCntUtt1] - 1; }
-  __device__ bool flag(uint32_t u) const {
-    if (is_dense_row(u)) return false;             // hybrid: dense rows have no prefix
-    if (u == 0 || every) return true;
-    int t0, t1; uint32_t p0, p1, x;
-    decode(u, t1, p1, x);
-    decode(u - 1, t0, p0, x);
-    return t0 != t1 || p0 != p1;
-  }
-  __device__ void emit(uint32_t u, uint32_t slot, uint32_t f) const {
-    if (is_dense_row(u)) { row_pfx[u] = 0xFFFFFFFFu; row_i3[u] = 0; return; }
-    int t; uint32_t pq, i3;
-    decode(u, t, pq, i3);
-    const uint32_t q = f ? slot : slot - 1;
-    row_pfx[u] = q;
-    row_i3[u] = i3;
-    if (f) {
-      const uint32_t m1 = meta[t].m1;
-      const uint32_t i2 = pq / m1, i1 = pq - i2 * m1;
-      pfx_t[q] = (uint32_t)t; pfx_i1[q] = i1; pfx_i2[q] = i2; row_seg[q] = u;
-    }
-  }
-  __device__ void finish(uint32_t P) const { counts[kCntP] = P; row_seg[P] = tt_rows(counts); }
-};
-
-// i2-groups: runs of (t, i2) over the prefixes (already in group-major order)
-struct GroupBody {
-  const uint32_t* pfx_t; const uint32_t* pfx_i2;
-  uint32_t* grp_pfx; uint32_t* grp_off; uint32_t* grp_t; uint32_t* grp_i2; uint32_t* counts;
-  __device__ uint32_t size() const { return counts[kCntP]; }
-  __device__ bool flag(uint32_t q) const {
-    return q == 0 || pfx_t[q] != pfx_t[q - 1] || pfx_i2[q] != pfx_i2[q - 1];
-  }
-  __device__ void emit(uint32_t q, uint32_t slot, uint32_t f) const {
-    grp_pfx[q] = q;
-    if (f) { grp_off[slot] = q; grp_t[slot] = pfx_t[q]; grp_i2[slot] = pfx_i2[q]; }
-  }
-  __device__ void finish(uint32_t NG) const { counts[kCntNG] = NG; grp_off[NG] = counts[kCntP]; }
-};
-
-// a3 + a4 in ONE pass over the sorted occurrences (replaces the three scans above on the default
-// path): position k starts a unique row (key change), a unique prefix (change of (t, i2 m1 + i1)
+// a3 + a4 in ONE pass over the sorted occurrences: position k starts a unique row (key change), a unique prefix (change of (t, i2 m1 + i1)
 // on a TT row) and an i2-group (change of (t, i2)).  Three flag ballots, three warp-count
 // scans and three decoupled look-backs (warps 0-2 in parallel) give every position its row
 // slot u, prefix slot q and group slot g; the emits write the same arrays the three scans did.
@@ -688,7 +552,7 @@ cudaError_t run_index_stage(Ctx& c, const void* indices, const int64_t* offsets,
                                ST_SORT_HIST, ST_SORT_PASS, s, /*have_hist=*/true);
   p.skey = which ? p.keysB : p.keysA;
   p.spos = which ? p.valsB : p.valsA;
-  if (!knobs().three_scans) {   // a3 + a4 fused (default)
+  {   // a3 + a4 in one scan
     StageScope sc(c, ST_UNIQUE, s);
     PlanScanArgs a;
     a.skey = p.skey; a.spos = p.spos; a.bag_of = p.bag_of; a.kbase = c.d_kbase; a.kmap = c.d_kmap;
@@ -701,31 +565,6 @@ cudaError_t run_index_stage(Ctx& c, const void* indices, const int64_t* offsets,
     a.tt_keys = c.tt_keys;
     const int64_t tiles = std::max<int64_t>(1, scan_tiles(nnz));
     k_plan_scan<<<(unsigned)tiles, SC_T, 0, s>>>(a, p.sc_status, p.sc_counter + 0);
-    return run_plan_tail(c, s);
-  }
-  // a3
-  {
-    StageScope sc(c, ST_UNIQUE, s);
-    UniqueBody b{p.skey, p.spos, p.bag_of, p.ukey, p.seg_off, p.inverse, p.sbag, p.counts,
-                 (uint32_t)nnz, (c.flags & TTEMB_NO_AGGREGATION) ? 1u : 0u, c.tt_keys};
-    const int64_t tiles = scan_tiles(nnz);
-    k_scan<UniqueBody><<<(unsigned)(tiles ? tiles : 1), SC_T, 0, s>>>(b, p.sc_status, p.sc_counter + 0);
-  }
-  // a4: digits + prefixes, then i2-groups
-  {
-    StageScope sc(c, ST_PREFIX, s);
-    PrefixBody b{p.ukey, c.d_kbase, c.d_kmap, c.d_meta, c.T, p.row_pfx, p.row_i3, p.pfx_t, p.pfx_i1,
-                 p.pfx_i2, p.row_seg, p.counts, (c.flags & TTEMB_NO_PREFIX_REUSE) ? 1u : 0u};
-    const int64_t tiles = scan_tiles(c.U_cap);
-    k_scan<PrefixBody><<<(unsigned)(tiles ? tiles : 1), SC_T, 0, s>>>(
-        b, p.sc_status + c.sc_tiles, p.sc_counter + 1);
-  }
-  {
-    StageScope sc(c, ST_GROUPS, s);
-    GroupBody b{p.pfx_t, p.pfx_i2, p.grp_pfx, p.grp_off, p.grp_t, p.grp_i2, p.counts};
-    const int64_t tiles = scan_tiles(c.P_cap);
-    k_scan<GroupBody><<<(unsigned)(tiles ? tiles : 1), SC_T, 0, s>>>(
-        b, p.sc_status + 2 * c.sc_tiles, p.sc_counter + 2);
   }
   return run_plan_tail(c, s);
 }

@@ -48,17 +48,15 @@ enum Stage : int {
 // Debug / experiment knobs from the environment, read ONCE per process (never on the launch
 // path): TTEMB_EXP bits switch parts of k_prefix_bwd off (timing experiments, results invalid),
 // TTEMB_DBG likewise for the forward kernels, TTEMB_TRACE enables role timers (trace builds),
-// TTEMB_THREE_SCANS / TTEMB_OLD_FWD select the older index scans / forward kernels, TTEMB_PF_BWD
-// sets an L2 prefetch distance in k_prefix_bwd.
+// TTEMB_PF_BWD sets an L2 prefetch distance in k_prefix_bwd.
 struct Knobs {
-  int exp = 0, dbg = 0, trace = 0, three_scans = 0, old_fwd = 0, pf_bwd = 0;
+  int exp = 0, dbg = 0, trace = 0, pf_bwd = 0;
 };
 inline const Knobs& knobs() {
   static const Knobs k = [] {
     auto num = [](const char* n) { const char* e = getenv(n); return e ? atoi(e) : 0; };
     Knobs r;
     r.exp = num("TTEMB_EXP"); r.dbg = num("TTEMB_DBG"); r.trace = getenv("TTEMB_TRACE") ? 1 : 0;
-    r.three_scans = getenv("TTEMB_THREE_SCANS") ? 1 : 0; r.old_fwd = getenv("TTEMB_OLD_FWD") ? 1 : 0;
     r.pf_bwd = num("TTEMB_PF_BWD");
     return r;
   }();
@@ -155,6 +153,7 @@ struct Ctx {
   int64_t nnz = 0;
   int32_t B = 0;
   bool fwd_done = false;
+  bool bwd_done = false;             // the last forward's backward ran (one backward per forward)
   bool planned = false;              // ttemb_plan ran; ttemb_forward_planned may follow
   const int64_t* offsets = nullptr;  // the planned batch's offsets (device; caller keeps alive)
   const float* psw = nullptr;        // per-sample weights of the current forward (device) or null

@@ -40,8 +40,14 @@ def assert_update_close(got_p, ref_p, p_old, g_ref, g_abs, lr, opt, tol=1e-4, go
         s = s0 + g * g
         # d/dg [g / sqrt(s0 + g^2)] = s0 / (s0+g^2)^1.5 <= 1/sqrt(s0+g^2); ill-conditioned
         # where |g| ~ dg and s0 ~ 0: allow the full step there.
-        sens = np.where(s > (10 * dg) ** 2, 1.0 / np.sqrt(np.maximum(s, 1e-300)), np.inf)
-        bound = np.minimum(lr * dg * sens * 2, 2 * lr) + ulp
+        # An untouched element (g_abs = 0, so dg = 0) must stay put up to rounding: its bound is
+        # the ulp term alone (without the mask, 0 * inf = NaN would make it unfailable).
+        touched = dg > 0
+        with np.errstate(divide="ignore", invalid="ignore", over="ignore"):
+            sens = np.where(s > (10 * dg) ** 2, 1.0 / np.sqrt(np.maximum(s, 1e-300)), np.inf)
+            step = np.where(touched, np.minimum(lr * dg * sens * 2, 2 * lr), 0.0)
+        bound = step + ulp
+        assert not np.isnan(bound).any(), what
         if got_s is not None:
             gs = np.asarray(got_s, np.float64).ravel()
             rs = np.asarray(ref_s, np.float64).ravel()
@@ -57,7 +63,7 @@ def assert_update_close(got_p, ref_p, p_old, g_ref, g_abs, lr, opt, tol=1e-4, go
 
 
 def plan_key(cfg, idx, off, B):
-    """Group-major plan key of every position (R23): kbase_t + (i2 m1 + i1) m3 + i3,
+    """Group-major plan key of every position (R29): kbase_t + (i2 m1 + i1) m3 + i3,
     digits (i1, i2, i3) of Eq. 3 via numpy.unravel_index per table."""
     T = cfg.num_tables
     mf = np.array(cfg.row_factors, np.int64)

@@ -76,6 +76,8 @@ def test_query_sizes_consistent():
     (dict(row_factors=[(1, 1, 1)] * 20), L.TTEMB_ERR_INVALID_ARG),     # prod < M
     (dict(max_nnz=(1 << 30) + 1), L.TTEMB_ERR_UNSUPPORTED),
     (dict(table_rows=[0] + list(W.config("c2").table_rows[1:])), L.TTEMB_ERR_INVALID_ARG),
+    (dict(optimizer="adagrad", adagrad_eps=0.0), L.TTEMB_ERR_INVALID_ARG),   # 0/0 on padding
+    (dict(max_batch=1 << 23), L.TTEMB_ERR_UNSUPPORTED),                    # T B dim >= 2^31 elements
 ])
 def test_query_sizes_rejects(kw, code):
     cfg, keep = _cfg(**kw)

@@ -1,6 +1,6 @@
 """Multi-process host logic of the data-parallel path on CPU (gloo, world size 2).
 
-Each rank takes its shard with `parallel.shard_bags`, computes its core gradients (the CPU
+Each rank takes its shard with `synth.workload.shard_batch`, computes its core gradients (the CPU
 oracle stands in for the GPU kernels here: no GPU on this box), and the gradients are summed
 with `parallel.allreduce_grads` (the same call bench.py uses with NCCL).  The result must
 equal the full-batch gradients (R16: SUM, no 1/B), and SGD replicas must stay identical.
@@ -40,7 +40,7 @@ def _worker(rank, world, port, result_path):
         idx, off = W.make_batch(cfg, seed=2)
         cores = W.make_cores(cfg, seed=2)
         go = W.make_grad_out(cfg, cfg.batch, seed=2)
-        li, lo, bl = parallel.shard_bags(idx, off, cfg.num_tables, cfg.batch, rank, world)
+        li, lo, bl = W.shard_batch(idx, off, cfg.num_tables, cfg.batch, rank, world)
         orc = Oracle.from_config(cfg)
         g = orc.backward(cores, li, lo, bl, go[rank * bl:(rank + 1) * bl])
         flat = torch.cat([torch.from_numpy(x).reshape(-1) for tg in g for x in tg])
@@ -75,7 +75,7 @@ def test_shard_bags_partition():
     cfg = _cfg()
     lens = np.random.default_rng(0).integers(0, 5, size=cfg.num_tables * cfg.batch)
     idx, off = W.make_batch(cfg, seed=1, lengths=lens)
-    pieces = [parallel.shard_bags(idx, off, cfg.num_tables, cfg.batch, r, 4) for r in range(4)]
+    pieces = [W.shard_batch(idx, off, cfg.num_tables, cfg.batch, r, 4) for r in range(4)]
     assert sum(len(p[0]) for p in pieces) == len(idx)
     for r, (i, o, bl) in enumerate(pieces):
         assert bl == 4 and o[0] == 0 and o[-1] == len(i)
@@ -84,4 +84,4 @@ def test_shard_bags_partition():
                 gb = t * cfg.batch + r * bl + b
                 np.testing.assert_array_equal(i[o[t * bl + b]:o[t * bl + b + 1]], idx[off[gb]:off[gb + 1]])
     with pytest.raises(ValueError):
-        parallel.shard_bags(idx, off, cfg.num_tables, cfg.batch, 0, 3)
+        W.shard_batch(idx, off, cfg.num_tables, cfg.batch, 0, 3)

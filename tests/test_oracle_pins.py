@@ -174,7 +174,7 @@ def test_plan_matches_numpy(name, seed):
     orc = Oracle.from_config(cfg)
     plan = orc.plan(idx, off, B)
     T = cfg.num_tables
-    # group-major plan key (R23): digits by numpy, re-ravelled in (i2, i1, i3) order
+    # group-major plan key (R29): digits by numpy, re-ravelled in (i2, i1, i3) order
     mf = np.array(cfg.row_factors, np.int64)
     span = mf.prod(axis=1)
     gbase = np.concatenate([[0], np.cumsum(span)[:-1]]).astype(np.int64)
@@ -209,6 +209,36 @@ def test_plan_matches_numpy(name, seed):
     np.testing.assert_array_equal(plan["grp_off"], np.concatenate([gfirst, [plan["P"]]]))
     np.testing.assert_array_equal(plan["grp_t"], gu[:, 0])
     np.testing.assert_array_equal(plan["grp_i2"], gu[:, 1])
+
+
+@pytest.mark.parametrize("name,seed", [("c2", 3), ("c3", 4)])
+def test_plan_key_is_a_bijection_of_table_row(name, seed):
+    """DESIGN.md R29: the plan's distinct keys, mapped back to (table, row) by inverting the key
+    K = kbase_t + (i2 m1 + i1) m3 + i3 and re-composing row = (i1 m2 + i2) m3 + i3 (Eq. 3), are
+    exactly the distinct (t, row) pairs of the batch: np.unique(rowbase_t + id) (SURVEY 8(c)'s
+    plan definition), and ukey is ascending in (t, i2, i1, i3) order."""
+    cfg = W.config(name)
+    B = min(cfg.batch, 1024)
+    idx, off = W.make_batch(cfg, seed=seed, batch=B)
+    plan = Oracle.from_config(cfg).plan(idx, off, B)
+    T = cfg.num_tables
+    mf = np.array(cfg.row_factors, np.int64)
+    rows = np.array(cfg.table_rows, np.int64)
+    kbase = np.concatenate([[0], np.cumsum(mf.prod(axis=1))])
+    rowbase = np.concatenate([[0], np.cumsum(rows)])
+    uk = plan["ukey"].astype(np.int64)
+    t = np.searchsorted(kbase, uk, side="right") - 1
+    local = uk - kbase[t]
+    i3 = local % mf[t, 2]
+    i1 = (local // mf[t, 2]) % mf[t, 0]
+    i2 = (local // mf[t, 2]) // mf[t, 0]
+    row = (i1 * mf[t, 1] + i2) * mf[t, 2] + i3
+    assert (row < rows[t]).all()
+    tab = np.repeat(np.arange(T * B), np.diff(off)) // B
+    want = np.unique(rowbase[tab] + np.asarray(idx, np.int64))
+    np.testing.assert_array_equal(np.sort(rowbase[t] + row), want)
+    order = np.lexsort((i3, i1, i2, t))
+    np.testing.assert_array_equal(order, np.arange(len(uk)))
 
 
 def test_plan_empty_batch():
