@@ -9,9 +9,13 @@
 //       SWIZZLE_128B_BASE32B operand in shared memory (the C1 row pieces stored as loaded);
 //       accumulated in TMEM over all tiles of the group (no atomics, no partial buffers).
 //   dA[m][r1] = sum_c dP[m][c] . C2[i2][r1][c]                  (the C1 gradient partials)
-//       M = 128 = the tile's dP rows stacked as [dP_hi; dP_lo], N = 64 r1, K = c in chunks of
-//       64 staged in shared memory (double-buffered); two MMAs per K step (B = C2_hi, C2_lo)
-//       give A_hi B_hi + A_lo B_hi + A_hi B_lo, i.e. 3xTF32 with two M = 128 instructions.
+//       M = 128 = the tile's dP rows stacked as [dP_hi; dP_lo] IN TENSOR MEMORY (lanes 0-63 hi,
+//       64-127 lo, column = c of the current 64-c chunk), N = 64 r1, K = c; B = the C2 chunk
+//       (hi, lo) in shared memory; two MMAs per K step accumulate dP_hi C2_hi + dP_hi C2_lo in
+//       lanes m and dP_lo C2_hi + dP_lo C2_lo in lanes 64 + m (3xTF32 plus the lo.lo term); the
+//       epilogue sums the two lane halves.  With A in TMEM the tensor core reads only the 2 KB
+//       B operand from shared memory per MMA (SS mode read 6 KB and shared the bandwidth with
+//       the loaders).
 //       The epilogue adds dA straight into the C1 gradient (red.global.add.v4, L2-resident).
 // At the group's last tile the dC2 accumulator is drained: with TTEMB_FUSED_UPDATE and SGD the
 // C2 slice is updated in place by reductions straight from TMEM (the paper's fused TT core
@@ -21,7 +25,8 @@
 // fp32 accuracy: 3xTF32 (hi = raw fp32, read by the tensor core with truncation; lo =
 // x - trunc_tf32(x)); scripts/tc_probe3.cu measures the TMEM-A form.
 //
-// Warp roles (416 threads): 0-7 loaders (cp.async chunk staging, lo split, dP^T -> TMEM),
+// Warp roles (416 threads): 0-7 loaders (cp.async chunk staging, C2 lo split, dP and dP^T ->
+// TMEM with the lo parts computed in registers),
 // 8 MMA issuer, 9-12 epilogue (dA -> dC1 reductions, dC2 -> gradient / fused update).
 #include <stdio.h>
 #include <stdlib.h>
@@ -41,13 +46,14 @@ constexpr int Y_LW = 8, Y_EW = 4;
 constexpr int Y_THREADS = (Y_LW + 1 + Y_EW) * 32;
 constexpr int Y_MMA_W = Y_LW;
 constexpr uint32_t Y_B1 = 2u * YR * YT * 4;     // C1^T hi + lo (CM(r1, m)), 32 KB
-constexpr uint32_t Y_A2LBO = 16 * 128 + 16;    // CM(128 rows, 64 c); +16 B per core column keeps
-                                                // the column-wise dP^T extraction conflict-free
-constexpr uint32_t Y_A2 = 16 * Y_A2LBO;         // [dP_hi; dP_lo] chunk (~32 KB)
+constexpr int Y_A2S = 68;                       // dP chunk staging row stride (floats): 64 c + 4
+constexpr uint32_t Y_A2 = YT * Y_A2S * 4;       // dP chunk, row-major (17 KB): conflict-free row
+                                                // (16-byte) and column (4-byte) reads
 constexpr uint32_t Y_B2LBO = 8 * 128;          // CM(64 r1, 64 c) core-column stride
 constexpr uint32_t Y_B2 = 2u * 16 * Y_B2LBO;    // C2 chunk hi + lo (32 KB)
 constexpr uint32_t Y_STAGE = Y_A2 + Y_B2;
 constexpr int Y_NST = 3;                        // chunk stages (cp.async, two in flight)
+constexpr int Y_GI = 64;                        // groups per CTA whose metadata is staged in shared memory
 constexpr size_t kBwdSmem = 1024 + Y_B1 + Y_NST * Y_STAGE;   // base aligned to 1024 (SW128 B1)
 
 struct YArgs {
@@ -73,10 +79,15 @@ struct YCtl {
   uint64_t s_full[Y_NST], s_free[Y_NST];  // K-chunk stages
   uint64_t d1_full, d1_free;              // dC2 accumulator (per group)
   uint64_t d2_full, d2_free;              // dA accumulator (per tile)
+  uint64_t p_free;                        // dP chunk A operand in TMEM (per chunk)
   uint64_t u_full[4], u_empty[4];
   uint32_t ring[4][4];                    // group, first prefix, #prefixes, flags (1 first, 2 last, 4 done)
   uint32_t claim[2];
   uint32_t tmem;
+  // this CTA's groups (static round robin) loaded once, in parallel, at kernel start: first /
+  // last prefix and C2 slice offset, so no group boundary waits on a global-memory round trip
+  uint32_t gq0[Y_GI], gq1[Y_GI];
+  unsigned long long gc2[Y_GI];
 };
 
 __device__ __forceinline__ float lo32(float x) { return x - tc::tf32_trunc(x); }
@@ -97,10 +108,15 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
     tc::mbar_init(&ctl.d1_free, Y_EW * 32);
     tc::mbar_init(&ctl.d2_full, 1);
     tc::mbar_init(&ctl.d2_free, Y_EW * 32);
+    tc::mbar_init(&ctl.p_free, 1);
     for (int s = 0; s < 4; ++s) { tc::mbar_init(&ctl.u_full[s], 1); tc::mbar_init(&ctl.u_empty[s], 1 + Y_EW); }
     tc::fence_mbar_init();
   }
   if (w == Y_MMA_W) tc::tmem_alloc(&ctl.tmem, 512);
+  for (int i = tid; i < Y_GI; i += blockDim.x) {
+    const uint32_t g = blockIdx.x + (uint32_t)i * gridDim.x;
+    if (g < NG) { ctl.gq0[i] = a.grp_off[g]; ctl.gq1[i] = a.grp_off[g + 1]; ctl.gc2[i] = a.grp_c2[g]; }
+  }
   tc::fence_before();
   __syncthreads();
   tc::fence_after();
@@ -116,7 +132,8 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
 #define YTA(k) do { } while (0)
 #endif
   // TMEM columns: [0,128) dP^T hi (64 per c-block), [128,256) lo, [256,384) dC2^T (64 per
-  // c-block), [384,448) dA pass B = C2_hi, [448,512) dA pass B = C2_lo.
+  // c-block), [384,448) dA (lanes m: dP_hi rows, 64 + m: dP_lo rows), [448,512) the current
+  // chunk's [dP_hi; dP_lo] (dA A operand).
   const int tpp = a.tpp, NC = a.NC;
 
   if (w < Y_LW) {
@@ -128,9 +145,13 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
     // chunk's TMEM lane quarters extract dP^T (hi, lo) from A2 into TMEM for the dC2 GEMM.
     struct Job { uint32_t g, q0, q1, qa; int ck; unsigned long long c2; };
     const uint32_t G0 = blockIdx.x, GS = gridDim.x;
-    auto start = [&](Job& j, uint32_t g) {   // group metadata loaded once (three independent loads)
+    auto start = [&](Job& j, uint32_t g) {   // group metadata (staged in shared memory)
       j.g = g; j.ck = 0;
-      if (g < NG) { j.q0 = j.qa = a.grp_off[g]; j.q1 = a.grp_off[g + 1]; j.c2 = a.grp_c2[g]; }
+      if (g < NG) {
+        const uint32_t k = (g - G0) / GS;
+        if (k < (uint32_t)Y_GI) { j.q0 = j.qa = ctl.gq0[k]; j.q1 = ctl.gq1[k]; j.c2 = ctl.gc2[k]; }
+        else { j.q0 = j.qa = a.grp_off[g]; j.q1 = a.grp_off[g + 1]; j.c2 = a.grp_c2[g]; }
+      }
     };
     auto advance = [&](Job& j) {
       if (++j.ck < a.nchunk) return;
@@ -142,7 +163,7 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
     // chunk copy map: rows (tid >> 4) + 16 k, float4 column 4 (tid & 15): every half-warp reads one
     // 256-byte row segment (coalesced); the padded core-column strides keep the stores conflict-free
     const int cr = tid >> 4, cc4 = 4 * (tid & 15);
-    auto a2_off = [&](int r) { return (uint32_t)((cc4 >> 2) * Y_A2LBO + (r >> 3) * 128 + (r & 7) * 16); };
+    auto a2_off = [&](int r) { return (uint32_t)((r * Y_A2S + cc4) * 4); };
     // C2 chunk map: row mb, float4 columns (tid >> 6) + 4 k (conflict-free stores into CM(r1, c))
     auto b2_off = [&](int k) { return tc::cm_off(mb, 4 * ((tid >> 6) + 4 * k), 8); };
     auto issue = [&](const Job& j, uint32_t sidx) {
@@ -225,45 +246,55 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
       char* a2 = stg + sidx * Y_STAGE;
       char* b2h = a2 + Y_A2;
       char* b2l = b2h + Y_B2 / 2;
-      if (!(a.exp & 4)) {
-        float4 p[4], q[4];
+      if (!(a.exp & 4)) {   // the C2 chunk's lo part (the dP lo parts are made in registers below)
+        float4 q[4];
 #pragma unroll
-        for (int k = 0; k < 4; ++k) {
-          const int r = cr + 16 * k;
-          p[k] = *reinterpret_cast<const float4*>(a2 + a2_off(r));
-          q[k] = *reinterpret_cast<const float4*>(b2h + b2_off(k));
-        }
+        for (int k = 0; k < 4; ++k) q[k] = *reinterpret_cast<const float4*>(b2h + b2_off(k));
 #pragma unroll
-        for (int k = 0; k < 4; ++k) {
-          const int r = cr + 16 * k;
-          *reinterpret_cast<float4*>(a2 + a2_off(64 + r)) =
-              make_float4(lo32(p[k].x), lo32(p[k].y), lo32(p[k].z), lo32(p[k].w));
+        for (int k = 0; k < 4; ++k)
           *reinterpret_cast<float4*>(b2l + b2_off(k)) =
               make_float4(lo32(q[k].x), lo32(q[k].y), lo32(q[k].z), lo32(q[k].w));
-        }
       }
       YTA(4);
       tc::named_sync(1, Y_LW * 32);                     // whole chunk (hi and lo) visible
       YTA(5);
-      {   // dP^T of this chunk -> TMEM: chunk ck covers c-block ck / 2, lane quarters 2 (ck & 1) + {0, 1}
+      const float* a2f = reinterpret_cast<const float*>(a2);
+      {   // dP^T of this chunk -> TMEM [0, 256) (dC2 A operand): chunk ck covers c-block ck / 2,
+          // lane quarters 2 (ck & 1) + {0, 1}; thread = column, 32 tile rows; lo in registers
         const int blk = P.ck >> 1, Q = w & 3;
         if ((Q >> 1) == (P.ck & 1) && blk < a.nblk && !(a.exp & 8)) {
           const int cc = 32 * (Q & 1) + lane;             // column inside the chunk
           const int m0 = 32 * (w >> 2);                    // warps 0-3: rows 0..31, 4-7: 32..63
-          float xh[32], xl[32];
+          float x[32];
 #pragma unroll
-          for (int i = 0; i < 32; ++i) {
-            const int m = m0 + i;
-            const uint32_t base = (uint32_t)((cc >> 2) * Y_A2LBO + (m & 7) * 16 + (cc & 3) * 4);
-            xh[i] = *reinterpret_cast<const float*>(a2 + base + (m >> 3) * 128);
-            xl[i] = *reinterpret_cast<const float*>(a2 + base + ((64 + m) >> 3) * 128);
-          }
-          tc::tmem_st32(tc::taddr(tm + blk * 64 + m0, 32 * Q, 0), xh);
-          tc::tmem_st32(tc::taddr(tm + 128 + blk * 64 + m0, 32 * Q, 0), xl);
-          tc::tmem_wait_st();
+          for (int i = 0; i < 32; ++i) x[i] = a2f[(m0 + i) * Y_A2S + cc];
+          tc::tmem_st32(tc::taddr(tm + blk * 64 + m0, 32 * Q, 0), x);
+#pragma unroll
+          for (int i = 0; i < 32; ++i) x[i] = lo32(x[i]);
+          tc::tmem_st32(tc::taddr(tm + 128 + blk * 64 + m0, 32 * Q, 0), x);
         }
       }
       YTA(6);
+      // dP of this chunk -> TMEM [448, 512) (dA A operand, M = 128): lanes 0-63 dP_hi rows,
+      // 64-127 dP_lo rows; warp (Q, h): rows 32 (Q & 1) + lane, columns 32 h .. 32 h + 31.
+      // Single-buffered: wait until the previous chunk's dA MMAs have read it.
+      tc::mbar_wait(&ctl.p_free, (sp & 1) ^ 1);
+      tc::fence_after();
+      if (!(a.exp & 8)) {
+        const int Q = w & 3, h = w >> 2, m = 32 * (Q & 1) + lane;
+        float x[32];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+          const float4 v = *reinterpret_cast<const float4*>(a2f + m * Y_A2S + 32 * h + 4 * k);
+          x[4 * k] = v.x; x[4 * k + 1] = v.y; x[4 * k + 2] = v.z; x[4 * k + 3] = v.w;
+        }
+        if (Q >= 2) {
+#pragma unroll
+          for (int i = 0; i < 32; ++i) x[i] = lo32(x[i]);
+        }
+        tc::tmem_st32(tc::taddr(tm + 448 + 32 * h, 32 * Q, 0), x);
+      }
+      tc::tmem_wait_st();
       tc::fence_async_smem();
       tc::fence_before();
       tc::mbar_arrive(&ctl.s_full[sidx]);
@@ -314,19 +345,19 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
         tc::fence_after();
         if (lane == 0) {
           const uint32_t id = tc::idesc_tf32(128, 64, false, false);
-          const uint32_t a2 = tc::smem_u32(stg + s * Y_STAGE), b2h = a2 + Y_A2, b2l = b2h + Y_B2 / 2;
+          const uint32_t b2h = tc::smem_u32(stg + s * Y_STAGE) + Y_A2, b2l = b2h + Y_B2 / 2;
 #pragma unroll
           for (int kk = 0; kk < 8; ++kk) {
-            const uint64_t da = tc::sdesc(a2 + kk * 2 * Y_A2LBO, Y_A2LBO, 128);
             const uint64_t dbh = tc::sdesc(b2h + kk * 2 * Y_B2LBO, Y_B2LBO, 128);
             const uint64_t dbl = tc::sdesc(b2l + kk * 2 * Y_B2LBO, Y_B2LBO, 128);
             const uint32_t acc = (ck > 0 || kk > 0) ? 1u : 0u;
             if (!(a.exp & 32)) {
-              tc::mma_tf32(tm + 384, da, dbh, id, acc);
-              tc::mma_tf32(tm + 448, da, dbl, id, acc);
+              tc::mma_tf32_ts(tm + 384, tm + 448 + kk * 8, dbh, id, acc);
+              tc::mma_tf32_ts(tm + 384, tm + 448 + kk * 8, dbl, id, 1u);
             }
           }
           tc::commit(&ctl.s_free[s]);
+          tc::commit(&ctl.p_free);
           if (ck + 1 == a.nchunk) tc::commit(&ctl.d2_full);
         }
         __syncwarp();
@@ -394,20 +425,13 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
       tc::fence_after();
       {
         const int m = (Q & 1) * 32 + lane;               // tile row of this lane
-        float v[32], x[32];
+        float v[32];
         float* dst = nullptr;
-        if (m < rows) {
-          const uint32_t q = qa + (m >> a.n1s);
-          const uint32_t t = a.pfx_t[q];
-          dst = a.grads + a.meta[t].c1_off + ((size_t)(a.pfx_i1[q] << a.n1s) + (m & ((1 << a.n1s) - 1))) * YR;
-        }
+        if (m < rows)   // grp_arow = C1 row of (prefix, j1 = 0): one load, no pfx_t -> meta chain
+          dst = a.grads + ((size_t)__ldg(a.grp_arow + qa + (m >> a.n1s)) + (m & ((1 << a.n1s) - 1))) * YR;
         for (int h = 0; h < 2; ++h) {
+          // lanes m: dP_hi (C2_hi + C2_lo); lanes 64 + m: dP_lo (C2_hi + C2_lo); both reduce into dC1
           tc::tmem_ld32(tc::taddr(tm + 384 + 32 * h, 32 * Q, 0), v);
-          if (Q < 2) {
-            tc::tmem_ld32(tc::taddr(tm + 448 + 32 * h, 32 * Q, 0), x);
-#pragma unroll
-            for (int i = 0; i < 32; ++i) v[i] += x[i];
-          }
           if (dst && !(a.exp & 2)) {
 #pragma unroll
             for (int i = 0; i < 32; i += 4)
