@@ -152,6 +152,37 @@ def stage_work(name, cfg, B, nnz, counts, tc=False):
     return 0, 0, 0
 
 
+def plan_work(cfg, idx, off, B):
+    """Algorithmic FLOPs of one batch from its unique rows / prefixes (numpy)."""
+    n1, n2, n3 = cfg.col_factors
+    R, N, T = cfg.rank, cfg.dim, cfg.num_tables
+    tab = np.repeat(np.arange(T * B), np.diff(off)) // B
+    U = P = 0
+    for t in range(T):
+        ids = np.unique(np.asarray(idx)[tab == t])
+        if getattr(cfg, "dense", ()) and cfg.dense[t]:
+            continue
+        m3 = cfg.row_factors[t][2]
+        U += len(ids)
+        P += len(np.unique(ids // m3))
+    return 3 * 2 * n1 * n2 * R * R * P + 3 * 2 * N * R * U
+
+
+def scaling_cap(cfg, world, args):
+    """SURVEY 8(e) work model: per-GPU dedup shrinks slower than 1/G, so with a fixed global
+    batch (strong scaling) the best possible efficiency is W(1) / (G max_g W_g) with W the
+    algorithmic FLOPs of a batch; with a fixed per-GPU batch (weak scaling) the work per GPU does
+    not change (cap 1, minus the gradient exchange)."""
+    if world == 1 or args.scaling == "weak":
+        return {"kind": args.scaling, "cap": 1.0, "model": "per-GPU work fixed"}
+    gi, goff = W.make_batch(cfg, step=0, seed=args.seed)
+    w1 = plan_work(cfg, gi, goff, cfg.batch)
+    shards = [W.shard_batch(gi, goff, cfg.num_tables, cfg.batch, r, world) for r in range(world)]
+    wg = max(plan_work(cfg, i, o, b) for i, o, b in shards)
+    return {"kind": "strong", "cap": w1 / (world * wg), "model": "alg FLOPs of the global batch / (G x max shard)",
+            "gflop_global": w1 / 1e9, "gflop_max_shard": wg / 1e9}
+
+
 def kernel_roofline(name, work, per_launch_ms, hbm_peak, tensor_peak, alu_peak):
     """The binding roofline of one launch: the largest of (tensor flops at the 3xTF32 peak, FFMA
     flops at the FP32 peak, algorithmic bytes at the HBM peak); achieved = that quantity per
@@ -320,7 +351,8 @@ def workload_config(cfg, B, world, args):
             "ids": f"zipf{cfg.zipf_s}-{cfg.id_map}" if cfg.zipf_s else f"uniform-{cfg.id_map}",
             "optimizer": args.opt,
             "update": ("fused" if world == 1 and not getattr(args, "unfused", False)
-                       else "allreduce+update" if world > 1 else "unfused"),
+                       else ("bucketed all-reduce + update" if getattr(args, "grad_sync", "allreduce") == "allreduce"
+                             else "reduce-scatter + sharded update + all-gather") if world > 1 else "unfused"),
             "parallelism": f"dp{world}", "l2": "flushed between timed steps (untimed 512 MiB write)",
             **({"bijection": f"frequency order (Alg. 2 l.1-4), {args.bijection} history batches"}
                if getattr(args, "bijection", 0) else {}),
@@ -378,6 +410,9 @@ def main():
                     help="no cross-step pipelining of the next batch's index stage")
     ap.add_argument("--no-graph", dest="graph", action="store_false",
                     help="launch every step eagerly instead of replaying a captured CUDA graph")
+    ap.add_argument("--grad-sync", default="allreduce", choices=["allreduce", "rs_ag"],
+                    help="N > 1: bucketed all-reduce overlapped with the backward, or reduce-scatter -> "
+                         "sharded update -> all-gather (SURVEY 8(e))")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
@@ -452,14 +487,14 @@ def main():
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
     stream = torch.cuda.current_stream()
 
+    sync = parallel.GradSync(emb, mode=args.grad_sync) if not fused else None
+
     def step(i):
         di, do, dg = dpool[i % len(dpool)]
         emb.forward(di, do, B, out=out)
         emb.backward(dg, lr=args.lr)
-        if world > 1:
-            parallel.allreduce_grads(emb.grads)
-        if not fused:
-            emb.update(args.lr)
+        if sync is not None:
+            sync.exchange_and_update(args.lr)
 
     # ---- cross-step pipelining (default): the index stage of batch g+1 (ttemb_plan_batch, reads no
     #      parameters) runs on a side stream while batch g's forward compute + backward + update run;
@@ -468,6 +503,8 @@ def main():
     pipe = args.pipeline and len(dpool) % 2 == 0
     if pipe:
         embs = [emb, emb.sibling()]
+        hsync = [sync, parallel.GradSync(embs[1], mode=args.grad_sync, comm_stream=sync.comm)] \
+            if sync is not None else None
         side = torch.cuda.Stream(device=dev)
         ev_go = [torch.cuda.Event() for _ in range(len(dpool))]
         ev_planned = [torch.cuda.Event() for _ in range(len(dpool))]
@@ -485,10 +522,8 @@ def main():
             nh.plan_batch(ni, no, B, stream=side)
             e_pl.record(side)
             h.backward(dg, lr=args.lr)
-            if world > 1:
-                parallel.allreduce_grads(h.grads)
-            if not fused:
-                h.update(args.lr)
+            if sync is not None:
+                hsync[g % 2].exchange_and_update(args.lr)
             cur.wait_event(e_pl)
 
         embs[0].plan_batch(dpool[0][0], dpool[0][1], B)
@@ -503,7 +538,8 @@ def main():
 
     # ---- optional CUDA graphs: one captured step per pool batch (same kernels, no launch gaps) ----
     graphs = None
-    if args.graph and world == 1:
+    # CUDA graphs: NCCL collectives are capturable; the gloo fallback (ranks sharing a GPU) is not
+    if args.graph and (world == 1 or not shared):
         torch.cuda.synchronize()
         graphs = []
         g0 = gstate["g"] if pipe else 0
@@ -655,6 +691,7 @@ def main():
                 "gpu_launches": kernels_per_step(emb_passes(emb), world, fused=tc_path(cfg, args),
                                                  fused_update=fused) * args.steps,
                 "graph": bool(graphs is not None),
+                **({"scaling_cap": scaling_cap(cfg, world, args)} if world > 1 else {}),
                 "pipeline": "next batch's index stage on a side stream" if pipe else None,
                 "clocks": clk.summary(),
                 "stages_us_per_step": {k: round(v[0] / args.steps * 1e3, 2) for k, v in stages.items() if v[1]}}

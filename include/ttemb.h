@@ -147,6 +147,26 @@ int ttemb_backward(ttemb_t h, const float* grad_out, float lr, void* stream);
  * TTEMB_ERR_STATE when the handle was created with TTEMB_FUSED_UPDATE. */
 int ttemb_update(ttemb_t h, float lr, void* stream);
 
+/* Data-parallel plumbing ("the only communication is the
+ * gradient all-reduce").
+ * ttemb_grad_buckets: the gradient buffer as contiguous float ranges in the order the
+ * (unfused) backward finalises them, so a caller can start the all-reduce of a bucket while the
+ * backward is still computing the next: bucket 0 = the dense (hybrid) tables (final after the
+ * aggregation), bucket 1 = every C3 core (final after the row stage), bucket 2 = every C1 and
+ * C2 core (final at the end of the backward).  Writes up to max_buckets (begin, count) pairs
+ * (float offsets into grads; count 0 = empty bucket) and returns the number of buckets (3).
+ * ttemb_set_bucket_events: `events` is an array of n (<= 3) cudaEvent_t (host handles, owned by
+ * the caller; NULL / n = 0 switches it off); every later unfused ttemb_backward records event i
+ * on its stream as soon as bucket i is final (the tcgen05 path records them at those points,
+ * the FFMA path after its last gradient kernel).  Capturable in a CUDA graph.
+ * ttemb_update_range: the optimizer step restricted to the float range [begin, begin + count)
+ * of cores / state / grads (a rank's shard after a reduce-scatter: sharded update, then the
+ * caller all-gathers the cores).  TTEMB_ERR_STATE with TTEMB_FUSED_UPDATE, INVALID_ARG for a
+ * range outside the buffers. */
+int ttemb_grad_buckets(ttemb_t h, int64_t* begin, int64_t* count, int max_buckets);
+int ttemb_set_bucket_events(ttemb_t h, void* const* events, int n);
+int ttemb_update_range(ttemb_t h, float lr, int64_t begin, int64_t count, void* stream);
+
 /* Host-buffer variants (end-to-end path): copy the inputs from host memory
  * into the workspace staging area, run the step, and copy `out` back to the
  * host, all on `stream`.  Pinned host memory keeps the copies asynchronous. */

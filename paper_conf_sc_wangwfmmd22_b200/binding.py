@@ -171,6 +171,9 @@ def ttemb_status_string(code: int) -> str:
 # ---------------------------------------------------------------------------
 # Convenience owner
 # ---------------------------------------------------------------------------
+FLAT_ALIGN = 1024
+
+
 class TTEmbeddingBag:
     """Table-batched TT-EmbeddingBag (sum pooling) on one CUDA device.
 
@@ -203,9 +206,14 @@ class TTEmbeddingBag:
         cb, sb, gb, wb = ttemb_query_sizes(self._cfg)
         self.sizes = dict(core_bytes=cb, state_bytes=sb, grad_bytes=gb, workspace_bytes=wb)
         f32 = torch.float32
-        self.cores = torch.zeros(cb // 4, dtype=f32, device=self.device)
-        self.grads = torch.zeros(gb // 4, dtype=f32, device=self.device)
-        self.state = torch.zeros(sb // 4, dtype=f32, device=self.device) if sb else None
+        # flat buffers padded to a multiple of FLAT_ALIGN floats, so a data-parallel group of up
+        # to FLAT_ALIGN / 4 ranks can reduce-scatter / all-gather them in equal 16-byte-aligned
+        # shards (the library only touches the first core_bytes; the padding stays 0)
+        nfl = -(-(cb // 4) // FLAT_ALIGN) * FLAT_ALIGN
+        self.n_floats = cb // 4
+        self.cores = torch.zeros(nfl, dtype=f32, device=self.device)
+        self.grads = torch.zeros(nfl, dtype=f32, device=self.device)
+        self.state = torch.zeros(nfl, dtype=f32, device=self.device) if sb else None
         self.workspace = torch.empty(max(wb, 256), dtype=torch.uint8, device=self.device)
         self.h = ttemb_create(self._cfg, device, self.cores.data_ptr(),
                               self.state.data_ptr() if self.state is not None else 0,
@@ -332,6 +340,33 @@ class TTEmbeddingBag:
 
     def update(self, lr: float, stream=None) -> None:
         check(ttemb_update(self.h, lr, _stream_ptr(stream)), "ttemb_update")
+
+    def update_range(self, lr: float, begin: int, count: int, stream=None) -> None:
+        """Optimizer step on floats [begin, begin + count) of the flat buffers (clipped to the
+        library's part; the padding has no parameters)."""
+        end = min(begin + count, self.n_floats)
+        if end > begin:
+            check(L.load().ttemb_update_range(self.h, lr, begin, end - begin, _stream_ptr(stream)),
+                  "ttemb_update_range")
+
+    def grad_buckets(self):
+        """[(begin, count)] float ranges of the gradient buffer in the order the unfused backward
+        finalises them (dense tables, C3 cores, C1 + C2 cores)."""
+        b = (C.c_int64 * 3)()
+        n = (C.c_int64 * 3)()
+        k = L.load().ttemb_grad_buckets(self.h, b, n, 3)
+        if k < 0:
+            check(k, "ttemb_grad_buckets")
+        return [(int(b[i]), int(n[i])) for i in range(k)]
+
+    def set_bucket_events(self, events) -> None:
+        """torch.cuda.Event objects (one per bucket) the backward records as buckets finish, or
+        None.  The events are kept alive by this object."""
+        self._bucket_events = list(events) if events else []
+        for e in self._bucket_events:
+            e.record(torch.cuda.current_stream(self.device))   # materialise the CUDA event handle
+        arr = (C.c_void_p * 3)(*[e.cuda_event for e in self._bucket_events])
+        check(L.load().ttemb_set_bucket_events(self.h, arr, len(self._bucket_events)), "ttemb_set_bucket_events")
 
     def forward_host(self, indices: torch.Tensor, offsets: torch.Tensor, batch: int,
                      out: torch.Tensor, stream=None) -> None:

@@ -466,6 +466,32 @@ int ttemb_update(ttemb_t h, float lr, void* stream) {
   return map_cuda(run_update(c, lr, (cudaStream_t)stream));
 }
 
+int ttemb_update_range(ttemb_t h, float lr, int64_t begin, int64_t count, void* stream) {
+  if (!h) return TTEMB_ERR_INVALID_ARG;
+  Ctx& c = h->c;
+  if (c.flags & TTEMB_FUSED_UPDATE) return TTEMB_ERR_STATE;
+  if (begin < 0 || count < 0 || (uint64_t)(begin + count) > (uint64_t)c.core_floats) return TTEMB_ERR_INVALID_ARG;
+  if (count == 0) return TTEMB_OK;
+  DeviceGuard dg(c.device);
+  return map_cuda(run_update_range(c, lr, (size_t)begin, (size_t)count, (cudaStream_t)stream));
+}
+
+int ttemb_grad_buckets(ttemb_t h, int64_t* begin, int64_t* count, int max_buckets) {
+  if (!h || max_buckets < 0 || (max_buckets > 0 && (!begin || !count))) return TTEMB_ERR_INVALID_ARG;
+  const Ctx& c = h->c;
+  const int64_t b[3] = {(int64_t)c.dense_begin, (int64_t)c.c3_begin, 0};
+  const int64_t n[3] = {(int64_t)c.dense_floats, (int64_t)c.c3_floats, (int64_t)c.c3_begin};
+  for (int i = 0; i < 3 && i < max_buckets; ++i) { begin[i] = b[i]; count[i] = n[i]; }
+  return 3;
+}
+
+int ttemb_set_bucket_events(ttemb_t h, void* const* events, int n) {
+  if (!h || n < 0 || n > 3 || (n > 0 && !events)) return TTEMB_ERR_INVALID_ARG;
+  Ctx& c = h->c;
+  for (int i = 0; i < 3; ++i) c.bucket_ev[i] = i < n ? (cudaEvent_t)events[i] : nullptr;
+  return TTEMB_OK;
+}
+
 int ttemb_forward_host(ttemb_t h, const void* host_indices, const int64_t* host_offsets,
                        int64_t nnz, int32_t batch, float* host_out, void* stream) {
   if (!h) return TTEMB_ERR_INVALID_ARG;

@@ -334,6 +334,7 @@ cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s
         c.cores, c.state, c.grads, c.d_meta, c.d_kbase, c.d_kmap, c.T, p.ukey, p.counts, c.N, p.gbuf,
         fused ? 1 : 0, lr, c.eps, c.opt);
   }
+  if (!fused) c.mark_bucket(0, s);      // the dense tables' gradients are final
   BwdArgs a;
   a.cores = c.cores; a.grads = c.grads; a.state = c.state; a.meta = c.d_meta;
   a.counts = p.counts; a.grp_off = p.grp_off; a.grp_t = p.grp_t; a.grp_i2 = p.grp_i2;
@@ -352,11 +353,22 @@ cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s
         k_dc1_scalar<<<grid_for(c, c.P_cap * c.n1 * c.R, 256, 32), 256, 0, s>>>(a);
     }
   }
+  if (!fused) {   // (the tcgen05 path marked the C3 bucket after its row stage)
+    if (!tc_eligible(c) || c.nnz == 0) c.mark_bucket(1, s);
+    c.mark_bucket(2, s);
+  }
   if (fused) {   // C2 was updated inside the group kernel; C1 and C3 densely here
     StageScope sc(c, ST_UPD_C3, s);
     k_update_zero<<<grid_for(c, (int64_t)(c.c1_floats + c.c3_floats), 256, 32), 256, 0, s>>>(
         c.cores, c.state, c.grads, c.c1_floats, c.c3_begin, c.c3_floats, lr, c.eps, c.opt);
   }
+  return cudaGetLastError();
+}
+
+cudaError_t run_update_range(Ctx& c, float lr, size_t begin, size_t count, cudaStream_t s) {
+  StageScope sc(c, ST_UPDATE, s);
+  k_update<<<grid_for(c, (int64_t)count, 256, 32), 256, 0, s>>>(c.cores, c.state, c.grads, begin, count, lr,
+                                                                c.eps, c.opt);
   return cudaGetLastError();
 }
 

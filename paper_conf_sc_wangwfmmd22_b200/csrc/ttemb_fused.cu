@@ -775,6 +775,7 @@ cudaError_t run_tc_bwd(Ctx& c, float lr, cudaStream_t s) {
     StageScope sc(c, ST_BWD_ROWS, s);
     e = run_rows_bwd2(c, s);
   }
+  if (!(c.flags & TTEMB_FUSED_UPDATE)) c.mark_bucket(1, s);   // every C3 gradient is final
   if (e == cudaSuccess) e = run_prefix_bwd(c, lr, s);
   return e;
 }

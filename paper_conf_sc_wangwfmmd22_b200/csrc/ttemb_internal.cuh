@@ -159,6 +159,12 @@ struct Ctx {
   const float* psw = nullptr;        // per-sample weights of the current forward (device) or null
   bool weighted = false;             // this step's bags carry weights (psw or mean): p.wpos valid
 
+  // data-parallel gradient buckets (ttemb_set_bucket_events): event i recorded when bucket i is final
+  cudaEvent_t bucket_ev[3] = {nullptr, nullptr, nullptr};
+  void mark_bucket(int i, cudaStream_t s) const {
+    if (bucket_ev[i]) cudaEventRecord(bucket_ev[i], s);
+  }
+
   // timing
   bool timing = false;
   std::vector<cudaEvent_t> ev_pool;
@@ -180,6 +186,7 @@ cudaError_t run_index_stage(Ctx& c, const void* indices, const int64_t* offsets,
 cudaError_t run_forward_compute(Ctx& c, float* out, const int64_t* offsets, cudaStream_t s);
 cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s);
 cudaError_t run_update(Ctx& c, float lr, cudaStream_t s);
+cudaError_t run_update_range(Ctx& c, float lr, size_t begin, size_t count, cudaStream_t s);
 cudaError_t configure_group(Ctx& c);
 cudaError_t configure_tc(Ctx& c);
 bool tc_eligible(const Ctx& c);
