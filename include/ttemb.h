@@ -167,6 +167,15 @@ int ttemb_grad_buckets(ttemb_t h, int64_t* begin, int64_t* count, int max_bucket
 int ttemb_set_bucket_events(ttemb_t h, void* const* events, int n);
 int ttemb_update_range(ttemb_t h, float lr, int64_t begin, int64_t count, void* stream);
 
+/* Offline index-bijection generator (Sec. IV-C), host code: modularity-based
+ * community detection (Louvain method, the paper's refs [34], [35]) of an undirected weighted
+ * graph with n vertices and m edges (u[e], v[e], w[e] > 0; every edge listed once).  Writes a
+ * community label per vertex (0 .. C-1, numbered by first vertex) into labels[n] (host memory,
+ * caller-owned).  Deterministic.  INVALID_ARG for null pointers or vertex ids outside [0, n).
+ * Used by paper_conf_sc_wangwfmmd22_b200/reorder.py to build the index bijection that
+ * ttemb_set_bijection applies at run time. */
+int ttemb_louvain(int64_t n, int64_t m, const int64_t* u, const int64_t* v, const double* w, int64_t* labels);
+
 /* Host-buffer variants (end-to-end path): copy the inputs from host memory
  * into the workspace staging area, run the step, and copy `out` back to the
  * host, all on `stream`.  Pinned host memory keeps the copies asynchronous. */

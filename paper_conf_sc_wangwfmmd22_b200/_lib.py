@@ -32,7 +32,7 @@ SYMBOLS = ["ttemb_query_sizes", "ttemb_create", "ttemb_destroy", "ttemb_core_lay
            "ttemb_backward_host", "ttemb_check", "ttemb_get_plan", "ttemb_read_counts",
            "ttemb_set_timing", "ttemb_stage_times", "ttemb_stage_name", "ttemb_status_string",
            "ttemb_set_bijection", "ttemb_total_rows", "ttemb_forward_weighted", "ttemb_plan_batch",
-           "ttemb_forward_planned", "ttemb_update_range", "ttemb_grad_buckets", "ttemb_set_bucket_events"]
+           "ttemb_forward_planned", "ttemb_update_range", "ttemb_grad_buckets", "ttemb_set_bucket_events", "ttemb_louvain"]
 
 
 class ttemb_table(C.Structure):
@@ -104,6 +104,7 @@ def load(path: str = LIB_PATH):
     lib.ttemb_update_range.argtypes = [vp, f32, i64, i64, vp]
     lib.ttemb_grad_buckets.argtypes = [vp, C.POINTER(i64), C.POINTER(i64), C.c_int]
     lib.ttemb_set_bucket_events.argtypes = [vp, C.POINTER(vp), C.c_int]
+    lib.ttemb_louvain.argtypes = [i64, i64, C.POINTER(i64), C.POINTER(i64), C.POINTER(C.c_double), C.POINTER(i64)]
     for s in SYMBOLS:
         f = getattr(lib, s)
         if s not in ("ttemb_stage_name", "ttemb_status_string", "ttemb_total_rows"):

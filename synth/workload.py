@@ -213,6 +213,37 @@ def make_batch(cfg: TTConfig, step: int = 0, seed: int = 0, batch: Optional[int]
     return indices, offsets
 
 
+def make_session_batch(cfg: TTConfig, step: int = 0, seed: int = 0, batch: Optional[int] = None,
+                       topics: int = 8, topic_frac: float = 0.5, topic_size: int = 4096
+                       ) -> Tuple[np.ndarray, np.ndarray]:
+    """A stream with LOCAL information (a batch reflects the user behaviour of one
+    period): batch `step` belongs to session topic k = step % topics; each id is, with
+    probability topic_frac, uniform over topic k's fixed id set (topic_size ids of the table,
+    disjoint across topics, scattered by the table's raw-id permutation), else a Zipf(s) id
+    through the same permutation.  Used to measure the community part of the paper's index
+    bijection (Alg. 2 + modularity communities); id generation only."""
+    B = cfg.batch if batch is None else int(batch)
+    T = cfg.num_tables
+    lengths = np.full(T * B, cfg.pooling, dtype=np.int64)
+    offsets = np.zeros(T * B + 1, dtype=np.int64)
+    np.cumsum(lengths, out=offsets[1:])
+    k = step % topics
+    parts = []
+    for t in range(T):
+        m = cfg.table_rows[t]
+        n_t = int(offsets[(t + 1) * B] - offsets[t * B])
+        g = rng("session", cfg.name, seed, step, t)
+        perm = _perm(m, f"{cfg.name}/{t}")
+        ts = min(topic_size, max(1, m // (topics + 1)))
+        ranks = zipf_ids(g, m, cfg.zipf_s, n_t, "identity")
+        topic = g.random(n_t) < topic_frac
+        # topic k's ids: ranks [m - (k + 1) ts, m - k ts) (the cold tail), permuted like every id
+        ranks[topic] = m - (k + 1) * ts + g.integers(0, ts, size=int(topic.sum()))
+        parts.append(perm[ranks])
+    indices = np.concatenate(parts) if parts else np.zeros(0, dtype=np.int64)
+    return indices, offsets
+
+
 def shard_batch(indices: np.ndarray, offsets: np.ndarray, num_tables: int, batch: int,
                 rank: int, world: int) -> Tuple[np.ndarray, np.ndarray, int]:
     """Rank `rank` of `world` takes samples [rank*B/G, (rank+1)*B/G) of every table
