@@ -703,8 +703,9 @@ def main():
 def tc_path(cfg, args):
     """The tcgen05 path (R = 64, n2 R <= 256, n3 in {4, 8}, n1 a power of two <= 8)."""
     n1, n2, n3 = cfg.col_factors
-    return (not args.fp32_cores) and 16 <= cfg.rank <= 64 and n3 in (4, 8) and n1 in (1, 2, 4, 8) \
-        and n1 * n2 <= 16 and n2 * 64 <= 256          # ranks 16..63 run zero-padded to 64
+    R = 64 if 16 <= cfg.rank <= 64 else cfg.rank       # ranks 16..63 run zero-padded to 64
+    return (not args.fp32_cores) and R in (64, 128) and n3 in (4, 8) and n1 in (1, 2, 4, 8) \
+        and n1 * n2 <= 16 and n2 * R <= 4 * R
 
 
 def emb_passes(emb):

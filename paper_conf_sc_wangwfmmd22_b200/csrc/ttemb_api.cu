@@ -570,7 +570,7 @@ int ttemb_get_plan(ttemb_t h, ttemb_plan* plan) {
   plan->row_pfx = p.row_pfx; plan->row_i3 = p.row_i3; plan->pfx_t = p.pfx_t;
   plan->pfx_i1 = p.pfx_i1; plan->pfx_i2 = p.pfx_i2; plan->row_seg = p.row_seg;
   plan->grp_pfx = p.grp_pfx; plan->grp_off = p.grp_off; plan->grp_t = p.grp_t;
-  plan->grp_i2 = p.grp_i2; plan->rows = p.rows;
+  plan->grp_i2 = p.grp_i2; plan->rows = (knobs().dbg & 1024) ? p.pbuf : p.rows;   // debug: the P stash
   return TTEMB_OK;
 }
 

@@ -41,20 +41,34 @@ namespace ttemb {
 
 namespace {
 
-constexpr int YR = 64, YT = 64;                 // rank; tile rows (prefix, j1)
+constexpr int YT = 64;                          // tile rows (prefix, j1)
 constexpr int Y_LW = 8, Y_EW = 4;
 constexpr int Y_THREADS = (Y_LW + 1 + Y_EW) * 32;
 constexpr int Y_MMA_W = Y_LW;
-constexpr uint32_t Y_B1 = 2u * YR * YT * 4;     // C1^T hi + lo (CM(r1, m)), 32 KB
-constexpr int Y_A2S = 68;                       // dP chunk staging row stride (floats): 64 c + 4
-constexpr uint32_t Y_A2 = YT * Y_A2S * 4;       // dP chunk, row-major (17 KB): conflict-free row
-                                                // (16-byte) and column (4-byte) reads
-constexpr uint32_t Y_B2LBO = 8 * 128;          // CM(64 r1, 64 c) core-column stride
-constexpr uint32_t Y_B2 = 2u * 16 * Y_B2LBO;    // C2 chunk hi + lo (32 KB)
-constexpr uint32_t Y_STAGE = Y_A2 + Y_B2;
 constexpr int Y_NST = 3;                        // chunk stages (cp.async, two in flight)
-constexpr int Y_GI = 64;                        // groups per CTA whose metadata is staged in shared memory
-constexpr size_t kBwdSmem = 1024 + Y_B1 + Y_NST * Y_STAGE;   // base aligned to 1024 (SW128 B1)
+constexpr int Y_GI = 64;                        // work units per CTA whose metadata is staged in shared memory
+
+// Shape of the kernel for rank KR: a work unit is (i2-group, BPU c-blocks of 128); K-chunks of
+// CK columns of c.  R = 64: one unit per group (both c-blocks), 64-column chunks.  R = 128: one
+// unit per c-block (the dC2 / dA accumulators are N = 128 wide), 32-column chunks (the C2 chunk
+// [CK][KR] hi + lo then fits three stages).
+template <int KR> struct YShape {
+  static constexpr int BPU = KR == 64 ? 2 : 1;
+  static constexpr int CK = KR == 64 ? 64 : 32;
+  static constexpr int A2S = CK + 4;                                    // dP staging row stride (floats)
+  static constexpr uint32_t A2 = YT * A2S * 4;                          // dP chunk staging
+  static constexpr uint32_t B2LBO = (KR / 8) * 128;                     // CM(KR r1, CK c) core-column stride
+  static constexpr uint32_t B2 = 2u * (CK / 4) * B2LBO;                 // C2 chunk hi + lo
+  static constexpr uint32_t STAGE = A2 + B2;
+  static constexpr uint32_t B1 = 2u * KR * YT * 4;                      // C1^T hi + lo (MN-major)
+  static constexpr size_t SMEM = 1024 + B1 + Y_NST * STAGE;
+  // TMEM columns
+  static constexpr uint32_t T_DPT = 0;                                  // dP^T hi [64 BPU), lo [64 BPU, 128 BPU)
+  static constexpr uint32_t T_DC2 = 128 * BPU;                          // dC2^T, KR per c-block
+  static constexpr uint32_t T_DA = T_DC2 + KR * BPU;                    // dA (N = KR)
+  static constexpr uint32_t T_CH = T_DA + KR;                           // [dP_hi; dP_lo] chunk, CK cols
+  static_assert(T_CH + CK <= 512, "TMEM budget");
+};
 
 struct YArgs {
   float* cores;
@@ -66,7 +80,7 @@ struct YArgs {
   const unsigned long long* grp_c2;       // [NG] float offset of the group's C2 slice
   const float* dpbuf;                     // [P][n1][NC]
   uint32_t* work;
-  int n1, n1s, NC, nblk, tpp, nchunk;
+  int n1, n1s, NC, nblk, tpp, nchunk, R;
   float lr, eps;
   int opt, fused;
   unsigned long long* trace;              // TTEMB_TRACE: 32 cycle counters per CTA (timing only)
@@ -81,25 +95,31 @@ struct YCtl {
   uint64_t d2_full, d2_free;              // dA accumulator (per tile)
   uint64_t p_free;                        // dP chunk A operand in TMEM (per chunk)
   uint64_t u_full[4], u_empty[4];
-  uint32_t ring[4][4];                    // group, first prefix, #prefixes, flags (1 first, 2 last, 4 done)
+  uint32_t ring[4][5];                    // group, first prefix, #prefixes, flags (1 first, 2 last, 4 done), unit block
   uint32_t claim[2];
   uint32_t tmem;
-  // this CTA's groups (static round robin) loaded once, in parallel, at kernel start: first /
-  // last prefix and C2 slice offset, so no group boundary waits on a global-memory round trip
+  // this CTA's work units (static round robin) loaded once, in parallel, at kernel start: first /
+  // last prefix and C2 slice offset of the unit's group, so no unit boundary waits on a
+  // global-memory round trip
   uint32_t gq0[Y_GI], gq1[Y_GI];
   unsigned long long gc2[Y_GI];
 };
 
 __device__ __forceinline__ float lo32(float x) { return x - tc::tf32_trunc(x); }
 
+template <int KR>
 __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
+  using S = YShape<KR>;
+  constexpr int BPU = S::BPU, CK = S::CK, A2S = S::A2S;
   extern __shared__ __align__(128) char smem_raw[];
   __shared__ YCtl ctl;
   char* const smem = smem_raw + ((1024u - (tc::smem_u32(smem_raw) & 1023u)) & 1023u);
   char* const b1 = smem;                                 // C1^T hi | lo
-  char* const stg = smem + Y_B1;                         // stages: [A2 | B2 hi | B2 lo]
+  char* const stg = smem + S::B1;                        // stages: [A2 | B2 hi | B2 lo]
   const int tid = threadIdx.x, w = tid >> 5, lane = tid & 31;
   const uint32_t NG = a.counts[kCntNG];
+  const uint32_t UPG = (uint32_t)(a.nblk + BPU - 1) / BPU;   // work units per group
+  const uint32_t NU = NG * UPG;
   if (tid == 0) {
     tc::mbar_init(&ctl.a1_full, Y_LW * 32);
     tc::mbar_init(&ctl.a1_free, 1);
@@ -114,8 +134,11 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
   }
   if (w == Y_MMA_W) tc::tmem_alloc(&ctl.tmem, 512);
   for (int i = tid; i < Y_GI; i += blockDim.x) {
-    const uint32_t g = blockIdx.x + (uint32_t)i * gridDim.x;
-    if (g < NG) { ctl.gq0[i] = a.grp_off[g]; ctl.gq1[i] = a.grp_off[g + 1]; ctl.gc2[i] = a.grp_c2[g]; }
+    const uint32_t u = blockIdx.x + (uint32_t)i * gridDim.x;
+    if (u < NU) {
+      const uint32_t g = u / UPG;
+      ctl.gq0[i] = a.grp_off[g]; ctl.gq1[i] = a.grp_off[g + 1]; ctl.gc2[i] = a.grp_c2[g];
+    }
   }
   tc::fence_before();
   __syncthreads();
@@ -131,24 +154,24 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
 #define YT0() do { } while (0)
 #define YTA(k) do { } while (0)
 #endif
-  // TMEM columns: [0,128) dP^T hi (64 per c-block), [128,256) lo, [256,384) dC2^T (64 per
-  // c-block), [384,448) dA (lanes m: dP_hi rows, 64 + m: dP_lo rows), [448,512) the current
-  // chunk's [dP_hi; dP_lo] (dA A operand).
+  // TMEM columns (YShape): dP^T hi / lo of the unit's c-blocks (lane = c, column = m), the dC2^T
+  // accumulators (lane = c, column = r1), dA (lanes m: dP_hi rows, 64 + m: dP_lo rows; column =
+  // r1) and the current chunk's [dP_hi; dP_lo] (dA A operand, column = c of the chunk).
   const int tpp = a.tpp, NC = a.NC;
 
   if (w < Y_LW) {
     // ------------------------------- loaders -------------------------------
-    // Jobs = (group, tile, K-chunk) in a static round-robin group order, so the issue side can
-    // run two chunks ahead across tile and group boundaries.  A chunk is copied with cp.async
-    // straight into its MMA layout (dP rows -> A2 rows 0..63, C2 rows -> B2 hi); each thread
-    // then writes the lo parts of the 16-byte pieces it copied, and the warps owning the
-    // chunk's TMEM lane quarters extract dP^T (hi, lo) from A2 into TMEM for the dC2 GEMM.
-    struct Job { uint32_t g, q0, q1, qa; int ck; unsigned long long c2; };
+    // Jobs = (unit, tile, K-chunk) in a static round-robin unit order, so the issue side can run
+    // two chunks ahead across tile and unit boundaries.  A chunk's dP rows are copied with
+    // cp.async into a row-major staging buffer, its C2 rows straight into the B operand's
+    // core-matrix layout (hi); each thread writes the lo parts of the C2 pieces it copied, and
+    // dP (lanes m) and dP^T (lanes c) go to tensor memory with their lo parts made in registers.
+    struct Job { uint32_t u, q0, q1, qa; int ck; unsigned long long c2; };
     const uint32_t G0 = blockIdx.x, GS = gridDim.x;
-    auto start = [&](Job& j, uint32_t g) {   // group metadata (staged in shared memory)
-      j.g = g; j.ck = 0;
-      if (g < NG) {
-        const uint32_t k = (g - G0) / GS;
+    auto start = [&](Job& j, uint32_t u) {   // unit metadata (staged in shared memory)
+      j.u = u; j.ck = 0;
+      if (u < NU) {
+        const uint32_t k = (u - G0) / GS, g = u / UPG;
         if (k < (uint32_t)Y_GI) { j.q0 = j.qa = ctl.gq0[k]; j.q1 = ctl.gq1[k]; j.c2 = ctl.gc2[k]; }
         else { j.q0 = j.qa = a.grp_off[g]; j.q1 = a.grp_off[g + 1]; j.c2 = a.grp_c2[g]; }
       }
@@ -157,26 +180,31 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
       if (++j.ck < a.nchunk) return;
       j.ck = 0;
       j.qa += tpp;
-      if (j.qa >= j.q1) start(j, j.g + GS);
+      if (j.qa >= j.q1) start(j, j.u + GS);
     };
     const int mb = tid & 63;                  // C1^T staging map: row mb, float4 columns (tid >> 6) + 4 k
-    // chunk copy map: rows (tid >> 4) + 16 k, float4 column 4 (tid & 15): every half-warp reads one
-    // 256-byte row segment (coalesced); the padded core-column strides keep the stores conflict-free
-    const int cr = tid >> 4, cc4 = 4 * (tid & 15);
-    auto a2_off = [&](int r) { return (uint32_t)((r * Y_A2S + cc4) * 4); };
-    // C2 chunk map: row mb, float4 columns (tid >> 6) + 4 k (conflict-free stores into CM(r1, c))
-    auto b2_off = [&](int k) { return tc::cm_off(mb, 4 * ((tid >> 6) + 4 * k), 8); };
+    // dP chunk copy map: rows (tid / (CK/4)) + (256 / (CK/4)) k, float4 column cc4: every row
+    // segment is read by consecutive threads (coalesced)
+    constexpr int F4 = CK / 4, RPP = 256 / F4;
+    const int cr = tid / F4, cc4 = 4 * (tid % F4);
+    auto a2_off = [&](int r) { return (uint32_t)((r * A2S + cc4) * 4); };
+    // C2 chunk map: row (r1) tid % KR, float4 columns (tid / KR) + (256 / KR) k
+    constexpr int C2F = KR * CK / 4 / 256;    // float4 per thread
+    const int br = tid % KR, bc = tid / KR;
+    auto b2_off = [&](int k) { return tc::cm_off(br, 4 * (bc + (256 / KR) * k), KR / 8); };
     auto issue = [&](const Job& j, uint32_t sidx) {
       const uint32_t rows = min((uint32_t)tpp, j.q1 - j.qa) << a.n1s;
-      const float* dps = a.dpbuf + (size_t)j.qa * a.n1 * NC + j.ck * 64 + cc4;
-      const float* c2 = a.cores + j.c2 + j.ck * 64 + (size_t)mb * NC;
-      const uint32_t a2 = tc::smem_u32(stg + (sidx % Y_NST) * Y_STAGE), b2 = a2 + Y_A2;
+      const int c0 = (int)(j.u % UPG) * BPU * 128 + j.ck * CK;   // first slice column of the chunk
+      const float* dps = a.dpbuf + (size_t)j.qa * a.n1 * NC + c0 + cc4;
+      const float* c2 = a.cores + j.c2 + c0 + (size_t)br * NC;
+      const uint32_t a2 = tc::smem_u32(stg + (sidx % Y_NST) * S::STAGE), b2 = a2 + S::A2;
 #pragma unroll
-      for (int k = 0; k < 4; ++k) {
-        const int r = cr + 16 * k;
+      for (int k = 0; k < YT / RPP; ++k) {
+        const int r = cr + RPP * k;
         tc::cp_async16_z(a2 + a2_off(r), dps + (size_t)(r < (int)rows ? r : 0) * NC, r < (int)rows);
-        tc::cp_async16(b2 + b2_off(k), c2 + 4 * ((tid >> 6) + 4 * k));
       }
+#pragma unroll
+      for (int k = 0; k < C2F; ++k) tc::cp_async16(b2 + b2_off(k), c2 + 4 * (bc + (256 / KR) * k));
     };
     uint32_t ui = 0, si = 0, sp = 0;          // tile counter, issued / processed chunk counters
     Job P, I;
@@ -184,18 +212,19 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
     I = P;
     // C1 rows of a tile (row mb of the tile, float4 columns (tid >> 6) + 4 k), loaded one tile
     // ahead (NT = the next tile of the processing job) so their latency overlaps a whole tile.
-    float4 cvn[4];
+    constexpr int C1F = KR / 16;
+    float4 cvn[C1F];
     auto load_c1 = [&](const Job& j, float4* cv) {
-      const uint32_t np = j.g < NG ? min((uint32_t)tpp, j.q1 - j.qa) : 0u;
+      const uint32_t np = j.u < NU ? min((uint32_t)tpp, j.q1 - j.qa) : 0u;
       const bool ok = mb < (int)(np << a.n1s) && !(a.exp & 16);
-      const uint32_t arow = ok ? a.grp_arow[j.qa + (mb >> a.n1s)] + (mb & ((1 << a.n1s) - 1)) : 0u;
-      const float4* src = reinterpret_cast<const float4*>(a.cores + (size_t)arow * YR);
+      const float4* src = reinterpret_cast<const float4*>(
+          a.cores + (size_t)(ok ? a.grp_arow[j.qa + (mb >> a.n1s)] + (mb & ((1 << a.n1s) - 1)) : 0u) * KR);
 #pragma unroll
-      for (int k = 0; k < 4; ++k) cv[k] = ok ? __ldg(src + (tid >> 6) + 4 * k) : make_float4(0.f, 0.f, 0.f, 0.f);
+      for (int k = 0; k < C1F; ++k) cv[k] = ok ? __ldg(src + (tid >> 6) + 4 * k) : make_float4(0.f, 0.f, 0.f, 0.f);
     };
     load_c1(P, cvn);
     for (int d = 0; d < Y_NST - 1; ++d) {
-      if (I.g < NG) {
+      if (I.u < NU) {
         tc::mbar_wait(&ctl.s_free[si % Y_NST], ((si / Y_NST) & 1) ^ 1);
         issue(I, si);
         advance(I);
@@ -203,24 +232,25 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
       }
       tc::cp_commit();
     }
-    while (P.g < NG) {
+    while (P.u < NU) {
       YT0();
       const uint32_t np = min((uint32_t)tpp, P.q1 - P.qa);
       if (P.ck == 0) {
         const uint32_t fl = (P.qa == P.q0 ? 1u : 0u) | (P.qa + tpp >= P.q1 ? 2u : 0u);
         if (tid == 0) {
           tc::mbar_wait(&ctl.u_empty[ui & 3], ((ui >> 2) & 1) ^ 1);
-          ctl.ring[ui & 3][0] = P.g; ctl.ring[ui & 3][1] = P.qa; ctl.ring[ui & 3][2] = np; ctl.ring[ui & 3][3] = fl;
+          ctl.ring[ui & 3][0] = P.u / UPG; ctl.ring[ui & 3][1] = P.qa; ctl.ring[ui & 3][2] = np;
+          ctl.ring[ui & 3][3] = fl; ctl.ring[ui & 3][4] = P.u % UPG;
           tc::mbar_arrive(&ctl.u_full[ui & 3]);
         }
-        // C1^T -> B1 = CM(r1, m) hi | lo (element (r1, m) = C1 row m, column r1); zero past the tile
-        float4 cv[4];
+        // C1^T -> B1 (element (r1, m) = C1 row m, column r1); zero past the tile
+        float4 cv[C1F];
 #pragma unroll
-        for (int k = 0; k < 4; ++k) cv[k] = cvn[k];
+        for (int k = 0; k < C1F; ++k) cv[k] = cvn[k];
         {   // prefetch the next tile's C1 rows
           Job NT = P;
           NT.qa += tpp;
-          if (NT.qa >= NT.q1) start(NT, NT.g + GS);
+          if (NT.qa >= NT.q1) start(NT, NT.u + GS);
           load_c1(NT, cvn);
         }
         YTA(0);
@@ -230,12 +260,12 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
         // C1^T as the MN-major (N = r1 contiguous) SWIZZLE_128B_BASE32B operand: the C1 row
         // pieces are stored as they were loaded, one 16-byte store each (hi and lo)
 #pragma unroll
-        for (int k = 0; k < 4; ++k) {
+        for (int k = 0; k < C1F; ++k) {
           const int r0 = 4 * ((tid >> 6) + 4 * k);
-          const uint32_t off = tc::mn32_off(r0, mb, YR);
+          const uint32_t off = tc::mn32_off(r0, mb, KR);
           const float4 v = cv[k];
           *reinterpret_cast<float4*>(b1 + off) = v;
-          *reinterpret_cast<float4*>(b1 + Y_B1 / 2 + off) = make_float4(lo32(v.x), lo32(v.y), lo32(v.z), lo32(v.w));
+          *reinterpret_cast<float4*>(b1 + S::B1 / 2 + off) = make_float4(lo32(v.x), lo32(v.y), lo32(v.z), lo32(v.w));
         }
       }
       // chunk P landed (one newer chunk may still be in flight)
@@ -243,15 +273,15 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
       tc::cp_wait<Y_NST - 2>();
       YTA(3);
       const uint32_t sidx = sp % Y_NST;
-      char* a2 = stg + sidx * Y_STAGE;
-      char* b2h = a2 + Y_A2;
-      char* b2l = b2h + Y_B2 / 2;
+      char* a2 = stg + sidx * S::STAGE;
+      char* b2h = a2 + S::A2;
+      char* b2l = b2h + S::B2 / 2;
       if (!(a.exp & 4)) {   // the C2 chunk's lo part (the dP lo parts are made in registers below)
-        float4 q[4];
+        float4 q[C2F];
 #pragma unroll
-        for (int k = 0; k < 4; ++k) q[k] = *reinterpret_cast<const float4*>(b2h + b2_off(k));
+        for (int k = 0; k < C2F; ++k) q[k] = *reinterpret_cast<const float4*>(b2h + b2_off(k));
 #pragma unroll
-        for (int k = 0; k < 4; ++k)
+        for (int k = 0; k < C2F; ++k)
           *reinterpret_cast<float4*>(b2l + b2_off(k)) =
               make_float4(lo32(q[k].x), lo32(q[k].y), lo32(q[k].z), lo32(q[k].w));
       }
@@ -259,40 +289,45 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
       tc::named_sync(1, Y_LW * 32);                     // whole chunk (hi and lo) visible
       YTA(5);
       const float* a2f = reinterpret_cast<const float*>(a2);
-      {   // dP^T of this chunk -> TMEM [0, 256) (dC2 A operand): chunk ck covers c-block ck / 2,
-          // lane quarters 2 (ck & 1) + {0, 1}; thread = column, 32 tile rows; lo in registers
-        const int blk = P.ck >> 1, Q = w & 3;
-        if ((Q >> 1) == (P.ck & 1) && blk < a.nblk && !(a.exp & 8)) {
-          const int cc = 32 * (Q & 1) + lane;             // column inside the chunk
-          const int m0 = 32 * (w >> 2);                    // warps 0-3: rows 0..31, 4-7: 32..63
+      {   // dP^T of this chunk -> TMEM (dC2 A operand): thread = column, 32 tile rows; lo in
+          // registers.  R = 64: chunk ck covers c-block ck / 2, lane quarters 2 (ck & 1) + {0, 1};
+          // R = 128: the unit's block, lane quarter ck & 3.
+        const int Q = w & 3;
+        const int blk = BPU == 2 ? (P.ck >> 1) : 0;
+        const bool mine = BPU == 2 ? ((Q >> 1) == (P.ck & 1) && blk < a.nblk) : (Q == (P.ck & 3));
+        if (mine && !(a.exp & 8)) {
+          const int cc = BPU == 2 ? 32 * (Q & 1) + lane : lane;   // column inside the chunk
+          const int m0 = 32 * (w >> 2);                           // warps 0-3: rows 0..31, 4-7: 32..63
           float x[32];
 #pragma unroll
-          for (int i = 0; i < 32; ++i) x[i] = a2f[(m0 + i) * Y_A2S + cc];
-          tc::tmem_st32(tc::taddr(tm + blk * 64 + m0, 32 * Q, 0), x);
+          for (int i = 0; i < 32; ++i) x[i] = a2f[(m0 + i) * A2S + cc];
+          tc::tmem_st32(tc::taddr(tm + S::T_DPT + blk * 64 + m0, 32 * Q, 0), x);
 #pragma unroll
           for (int i = 0; i < 32; ++i) x[i] = lo32(x[i]);
-          tc::tmem_st32(tc::taddr(tm + 128 + blk * 64 + m0, 32 * Q, 0), x);
+          tc::tmem_st32(tc::taddr(tm + S::T_DPT + 64 * BPU + blk * 64 + m0, 32 * Q, 0), x);
         }
       }
       YTA(6);
-      // dP of this chunk -> TMEM [448, 512) (dA A operand, M = 128): lanes 0-63 dP_hi rows,
-      // 64-127 dP_lo rows; warp (Q, h): rows 32 (Q & 1) + lane, columns 32 h .. 32 h + 31.
+      // dP of this chunk -> TMEM (dA A operand, M = 128): lanes 0-63 dP_hi rows, 64-127 dP_lo
+      // rows; warp (Q, h): rows 32 (Q & 1) + lane, columns 32 h .. 32 h + 31 of the chunk.
       // Single-buffered: wait until the previous chunk's dA MMAs have read it.
       tc::mbar_wait(&ctl.p_free, (sp & 1) ^ 1);
       tc::fence_after();
-      if (!(a.exp & 8)) {
+      {
         const int Q = w & 3, h = w >> 2, m = 32 * (Q & 1) + lane;
-        float x[32];
+        if (!(a.exp & 8) && 32 * h < CK) {
+          float x[32];
 #pragma unroll
-        for (int k = 0; k < 8; ++k) {
-          const float4 v = *reinterpret_cast<const float4*>(a2f + m * Y_A2S + 32 * h + 4 * k);
-          x[4 * k] = v.x; x[4 * k + 1] = v.y; x[4 * k + 2] = v.z; x[4 * k + 3] = v.w;
-        }
-        if (Q >= 2) {
+          for (int k = 0; k < 8; ++k) {
+            const float4 v = *reinterpret_cast<const float4*>(a2f + m * A2S + 32 * h + 4 * k);
+            x[4 * k] = v.x; x[4 * k + 1] = v.y; x[4 * k + 2] = v.z; x[4 * k + 3] = v.w;
+          }
+          if (Q >= 2) {
 #pragma unroll
-          for (int i = 0; i < 32; ++i) x[i] = lo32(x[i]);
+            for (int i = 0; i < 32; ++i) x[i] = lo32(x[i]);
+          }
+          tc::tmem_st32(tc::taddr(tm + S::T_CH + 32 * h, 32 * Q, 0), x);
         }
-        tc::tmem_st32(tc::taddr(tm + 448 + 32 * h, 32 * Q, 0), x);
       }
       tc::tmem_wait_st();
       tc::fence_async_smem();
@@ -305,7 +340,7 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
       ++sp;
       advance(P);
       // refill: the chunk two ahead
-      if (I.g < NG) {
+      if (I.u < NU) {
         YTA(7);
         tc::mbar_wait(&ctl.s_free[si % Y_NST], ((si / Y_NST) & 1) ^ 1);
         YTA(8);
@@ -329,11 +364,11 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
       YT0();
       tc::mbar_wait(&ctl.u_full[ui & 3], (ui >> 2) & 1);
       YTA(10);
-      const uint32_t fl = ctl.ring[ui & 3][3];
+      const uint32_t fl = ctl.ring[ui & 3][3], ub = ctl.ring[ui & 3][4];
       __syncwarp();
       if (lane == 0) tc::mbar_arrive(&ctl.u_empty[ui & 3]);
       if (fl & 4u) break;
-      // dA = [dP_hi; dP_lo] . C2_{hi,lo}^T over the K chunks (as they land)
+      // dA = [dP_hi; dP_lo] . C2_{hi,lo}^T over the K chunks (as they land); N = KR
       tc::mbar_wait(&ctl.d2_free, (ui & 1) ^ 1);
       YTA(11);
       tc::fence_after();
@@ -344,16 +379,16 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
         YTA(12);
         tc::fence_after();
         if (lane == 0) {
-          const uint32_t id = tc::idesc_tf32(128, 64, false, false);
-          const uint32_t b2h = tc::smem_u32(stg + s * Y_STAGE) + Y_A2, b2l = b2h + Y_B2 / 2;
+          const uint32_t id = tc::idesc_tf32(128, KR, false, false);
+          const uint32_t b2h = tc::smem_u32(stg + s * S::STAGE) + S::A2, b2l = b2h + S::B2 / 2;
 #pragma unroll
-          for (int kk = 0; kk < 8; ++kk) {
-            const uint64_t dbh = tc::sdesc(b2h + kk * 2 * Y_B2LBO, Y_B2LBO, 128);
-            const uint64_t dbl = tc::sdesc(b2l + kk * 2 * Y_B2LBO, Y_B2LBO, 128);
+          for (int kk = 0; kk < CK / 8; ++kk) {
+            const uint64_t dbh = tc::sdesc(b2h + kk * 2 * S::B2LBO, S::B2LBO, 128);
+            const uint64_t dbl = tc::sdesc(b2l + kk * 2 * S::B2LBO, S::B2LBO, 128);
             const uint32_t acc = (ck > 0 || kk > 0) ? 1u : 0u;
             if (!(a.exp & 32)) {
-              tc::mma_tf32_ts(tm + 384, tm + 448 + kk * 8, dbh, id, acc);
-              tc::mma_tf32_ts(tm + 384, tm + 448 + kk * 8, dbl, id, 1u);
+              tc::mma_tf32_ts(tm + S::T_DA, tm + S::T_CH + kk * 8, dbh, id, acc);
+              tc::mma_tf32_ts(tm + S::T_DA, tm + S::T_CH + kk * 8, dbl, id, 1u);
             }
           }
           tc::commit(&ctl.s_free[s]);
@@ -362,7 +397,7 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
         }
         __syncwarp();
       }
-      // dC2^T += dP^T . C1  (K = 64 tile rows), after the whole tile's dP^T reached TMEM
+      // dC2^T += dP^T . C1  (K = 64 tile rows, N = KR), after the whole tile's dP^T reached TMEM
       YTA(13);
       tc::mbar_wait(&ctl.a1_full, ui & 1);
       YTA(14);
@@ -370,16 +405,16 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
       if (fl & 1u) tc::mbar_wait(&ctl.d1_free, (gs & 1) ^ 1);
       tc::fence_after();
       if (lane == 0) {
-        const uint32_t id = tc::idesc_tf32(128, 64, false, true);    // B = C1^T MN-major
-        const uint32_t bh = tc::smem_u32(b1), bl = bh + Y_B1 / 2;
-        for (int blk = 0; blk < a.nblk; ++blk) {
-          const uint32_t d = tm + 256 + blk * 64;
+        const uint32_t id = tc::idesc_tf32(128, KR, false, true);    // B = C1^T MN-major
+        const uint32_t bh = tc::smem_u32(b1), bl = bh + S::B1 / 2;
+        for (int blk = 0; blk < BPU && (int)ub * BPU + blk < a.nblk; ++blk) {
+          const uint32_t d = tm + S::T_DC2 + blk * KR;
 #pragma unroll
           for (int kk = 0; kk < YT / 8; ++kk) {
-            const uint32_t sbo = (YR / 32) * 512, o = kk * 2 * sbo;   // MN-major, K groups of 4 outermost
+            const uint32_t sbo = (KR / 32) * 512, o = kk * 2 * sbo;   // MN-major, K groups of 4 outermost
             const uint64_t dbh = tc::sdesc_l(bh + o, 512, sbo, 1);
             const uint64_t dbl = tc::sdesc_l(bl + o, 512, sbo, 1);
-            const uint32_t ah = tm + blk * 64 + kk * 8, al = tm + 128 + blk * 64 + kk * 8;
+            const uint32_t ah = tm + S::T_DPT + blk * 64 + kk * 8, al = ah + 64 * BPU;
             if (a.exp & 32) continue;
             tc::mma_tf32_ts(d, ah, dbh, id, ((fl & 1u) && kk == 0) ? 0u : 1u);
             tc::mma_tf32_ts(d, ah, dbl, id, 1u);
@@ -402,23 +437,11 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
       tc::mbar_wait(&ctl.u_full[ui & 3], (ui >> 2) & 1);
       YTA(20);
       const uint32_t g = ctl.ring[ui & 3][0], qa = ctl.ring[ui & 3][1];
-      const uint32_t np = ctl.ring[ui & 3][2], fl = ctl.ring[ui & 3][3];
+      const uint32_t np = ctl.ring[ui & 3][2], fl = ctl.ring[ui & 3][3], ub = ctl.ring[ui & 3][4];
       __syncwarp();
       if (fl & 4u) break;
       const int rows = (int)np << a.n1s;
-      // L2 prefetch of the group PF groups ahead in this CTA's order (dP rows of all its tiles +
-      // its C2 slice: two contiguous ranges), so the loaders' cp.async chunks hit L2.
-      if ((fl & 1u) && w == Y_LW + 1 && lane == 0 && a.pf > 0) {
-        const uint32_t gn = g + (uint32_t)a.pf * gridDim.x;
-        if (gn < NG) {
-          const uint32_t q0 = a.grp_off[gn], q1 = a.grp_off[gn + 1];
-          const size_t fl0 = (size_t)q0 * a.n1 * NC, nfl = (size_t)(q1 - q0) * a.n1 * NC;
-          for (size_t o = 0; o < nfl; o += 16384)
-            tc::bulk_prefetch_l2(a.dpbuf + fl0 + o, (uint32_t)(min((size_t)16384, nfl - o) * 4));
-          tc::bulk_prefetch_l2(a.cores + a.grp_c2[gn], (uint32_t)(YR * NC * 4));
-        }
-      }
-      // dA: lanes 0..63 hold dP_hi rows (both passes), lanes 64..127 dP_lo rows (pass C2_hi)
+      // dA: lanes m hold dP_hi (C2_hi + C2_lo), lanes 64 + m dP_lo (C2_hi + C2_lo); both add into dC1
       YTA(25);
       tc::mbar_wait(&ctl.d2_full, ui & 1);
       YTA(21);
@@ -427,11 +450,10 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
         const int m = (Q & 1) * 32 + lane;               // tile row of this lane
         float v[32];
         float* dst = nullptr;
-        if (m < rows)   // grp_arow = C1 row of (prefix, j1 = 0): one load, no pfx_t -> meta chain
-          dst = a.grads + ((size_t)__ldg(a.grp_arow + qa + (m >> a.n1s)) + (m & ((1 << a.n1s) - 1))) * YR;
-        for (int h = 0; h < 2; ++h) {
-          // lanes m: dP_hi (C2_hi + C2_lo); lanes 64 + m: dP_lo (C2_hi + C2_lo); both reduce into dC1
-          tc::tmem_ld32(tc::taddr(tm + 384 + 32 * h, 32 * Q, 0), v);
+        if (m < rows)   // grp_arow = C1 row of (prefix, j1 = 0): one load
+          dst = a.grads + ((size_t)__ldg(a.grp_arow + qa + (m >> a.n1s)) + (m & ((1 << a.n1s) - 1))) * KR;
+        for (int h = 0; h < KR / 32; ++h) {
+          tc::tmem_ld32(tc::taddr(tm + S::T_DA + 32 * h, 32 * Q, 0), v);
           if (dst && !(a.exp & 2)) {
 #pragma unroll
             for (int i = 0; i < 32; i += 4)
@@ -445,16 +467,16 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
       tc::mbar_arrive(&ctl.d2_free);
       YTA(22);
       if (fl & 2u) {
-        // group complete: dC2^T [c][r1] -> gradient or fused C2 update (this CTA owns the slice)
+        // unit complete: dC2^T [c][r1] -> gradient or fused C2 update (this CTA owns the columns)
         tc::mbar_wait(&ctl.d1_full, gs & 1);
         YTA(23);
         tc::fence_after();
         const unsigned long long so = a.grp_c2[g];
-        for (int blk = 0; blk < a.nblk; ++blk) {
-          const int c = blk * 128 + Q * 32 + lane;
-          for (int h = 0; h < 2; ++h) {
+        for (int blk = 0; blk < BPU; ++blk) {
+          const int c = ((int)ub * BPU + blk) * 128 + Q * 32 + lane;
+          for (int h = 0; h < KR / 32; ++h) {
             float v[32];
-            tc::tmem_ld32(tc::taddr(tm + 256 + blk * 64 + 32 * h, 32 * Q, 0), v);
+            tc::tmem_ld32(tc::taddr(tm + S::T_DC2 + blk * KR + 32 * h, 32 * Q, 0), v);
             if (c < NC && !(a.exp & 1)) {
               const size_t base = so + (size_t)(32 * h) * NC + c;
               if (!a.fused || a.opt != TTEMB_SGD) {
@@ -523,7 +545,11 @@ k_c2_update_zero(float* __restrict__ cores, float* __restrict__ state, float* __
 
 cudaError_t configure_bwdtc(Ctx& c) {
   if (!fused_eligible(c)) return cudaSuccess;
-  return cudaFuncSetAttribute(k_prefix_bwd, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBwdSmem);
+  cudaError_t e = cudaFuncSetAttribute(k_prefix_bwd<64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)YShape<64>::SMEM);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(k_prefix_bwd<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)YShape<128>::SMEM);
+  return e;
 }
 
 // dC2 (fused update) and dC1 partials from the dP stash; requires run_fused_fwd's per-step
@@ -535,12 +561,16 @@ cudaError_t run_prefix_bwd(Ctx& c, float lr, cudaStream_t s) {
   a.grp_off = p.grp_off; a.grp_t = p.grp_t; a.pfx_i1 = p.pfx_i1; a.pfx_t = p.pfx_t; a.grp_arow = p.grp_arow;
   a.grp_c2 = p.grp_c2; a.dpbuf = p.dpbuf; a.work = p.work + 2;
   a.n1 = c.n1; a.n1s = c.n1 == 1 ? 0 : c.n1 == 2 ? 1 : c.n1 == 4 ? 2 : 3;
-  a.NC = c.NC; a.nblk = (c.NC + 127) / 128; a.tpp = YT / c.n1; a.nchunk = (c.NC + 63) / 64;
+  a.NC = c.NC; a.nblk = (c.NC + 127) / 128; a.tpp = YT / c.n1; a.R = c.R;
+  // K-chunks per work unit: R = 64 the whole slice in 64-column chunks, R = 128 one c-block in
+  // 32-column chunks
+  a.nchunk = c.R == 64 ? (c.NC + 63) / 64 : 128 / YShape<128>::CK;
   a.lr = lr; a.eps = c.eps; a.opt = c.opt; a.fused = (c.flags & TTEMB_FUSED_UPDATE) ? 1 : 0;
   a.exp = exp_bits();
   a.pf = knobs().pf_bwd;
   StageScope sc(c, ST_BWD_PREFIX, s);
-  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(c.NG_cap, (int64_t)c.sm_count));
+  const int64_t units = c.NG_cap * (c.R == 64 ? 1 : (c.NC + 127) / 128);
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(units, (int64_t)c.sm_count));
   static unsigned long long* trace = nullptr;
   a.trace = nullptr;
   if (knobs().trace) {
@@ -548,10 +578,11 @@ cudaError_t run_prefix_bwd(Ctx& c, float lr, cudaStream_t s) {
     cudaMemsetAsync(trace, 0, sizeof(unsigned long long) * 32 * grid, s);
     a.trace = trace;
   }
-  k_prefix_bwd<<<grid, Y_THREADS, kBwdSmem, s>>>(a);
+  if (c.R == 64) k_prefix_bwd<64><<<grid, Y_THREADS, YShape<64>::SMEM, s>>>(a);
+  else k_prefix_bwd<128><<<grid, Y_THREADS, YShape<128>::SMEM, s>>>(a);
   if (a.fused && a.opt != TTEMB_SGD)
     k_c2_update_zero<<<c.sm_count * 8, 256, 0, s>>>(c.cores, c.state, c.grads, p.grp_c2, p.counts,
-                                                    (uint32_t)(YR * c.NC), lr, c.eps);
+                                                    (uint32_t)(c.R * c.NC), lr, c.eps);
   if (a.trace) {
     std::vector<unsigned long long> hb(32 * grid);
     cudaMemcpyAsync(hb.data(), trace, hb.size() * 8, cudaMemcpyDeviceToHost, s);

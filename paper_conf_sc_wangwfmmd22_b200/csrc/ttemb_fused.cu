@@ -54,7 +54,7 @@ struct XArgs {
   uint32_t* work;
   int dbg;                            // TTEMB_DBG bit mask (timing experiments only; results invalid)
   unsigned long long* trace;          // optional per-CTA role timers (TTEMB_TRACE): 32 slots per CTA
-  int n1, n1s, n2, n3, N, NC, nblk, tpp;
+  int n1, n1s, n2, n3, N, NC, nblk, tpp, R;
 };
 
 // TTEMB_TRACE instrumentation: clock64 intervals accumulated per role leader.
@@ -72,7 +72,7 @@ struct XCtl {
   uint64_t raw_full, a_full, a_free;
   uint64_t b_full[2], b_free[2], d_full[2], d_free[2];
   uint64_t u_full[4], u_empty[4];
-  uint32_t ring[4][8];                // group, first prefix, #prefixes, flags (1 first, 2 last, 4 done), u0, u1
+  uint32_t ring[4][8];                // group, first prefix, #prefixes, flags (1 first, 2 last, 4 done), unit block
   uint32_t claim[2];
   uint32_t tmem;
 };
@@ -82,15 +82,23 @@ __global__ void k_fused_prep(XArgs a) {
   for (uint32_t q = blockIdx.x * blockDim.x + threadIdx.x; q < max(P, NG); q += gridDim.x * blockDim.x) {
     if (q < P) {
       const uint32_t p = a.grp_pfx[q];
-      a.grp_arow[q] = (uint32_t)(a.meta[a.pfx_t[p]].c1_off / XR) + (a.pfx_i1[p] << a.n1s);
+      a.grp_arow[q] = (uint32_t)(a.meta[a.pfx_t[p]].c1_off / a.R) + (a.pfx_i1[p] << a.n1s);
     }
-    if (q < NG) a.grp_c2[q] = a.meta[a.grp_t[q]].c2_off + (unsigned long long)a.grp_i2[q] * XR * a.NC;
+    if (q < NG) a.grp_c2[q] = a.meta[a.grp_t[q]].c2_off + (unsigned long long)a.grp_i2[q] * a.R * a.NC;
   }
 }
 
 __device__ __forceinline__ float tf32_lo(float x) { return x - tc::tf32_trunc(x); }
 
+// Work unit = (i2-group, c-range of BPU 128-wide c-blocks): at R = 64 one unit covers the group's
+// whole C2 slice (C2^T of both c-blocks fills TMEM columns [0, 256)); at R = 128 (K = 128) one
+// c-block's C2^T hi + lo already takes 256 columns, so a group is split into NC / 128 units and
+// the C1 rows of a tile are staged once per unit.
+template <int KR>
 __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
+  constexpr int BPU = KR == 64 ? 2 : 1;            // c-blocks per work unit
+  constexpr uint32_t BSLOT = 2u * XT * KR * 4;    // one B slot: C1 tile hi + lo (K = KR)
+  constexpr uint32_t BHALF = XT * KR * 4;
   extern __shared__ __align__(128) char smem_raw[];
   __shared__ XCtl ctl;
   char* const smem = smem_raw + ((128u - (tc::smem_u32(smem_raw) & 127u)) & 127u);
@@ -98,7 +106,11 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
   char* const bbuf = smem + X_RAW_BYTES;
   const int tid = threadIdx.x, w = tid >> 5, lane = tid & 31;
   const uint32_t NG = a.counts[kCntNG];
-  const uint32_t raw_bytes = (uint32_t)XR * a.NC * 4u;
+  const uint32_t UPG = (uint32_t)(a.nblk + BPU - 1) / BPU;   // units per group
+  const uint32_t NU = NG * UPG;
+  // raw staging: R = 64 the whole C2 slice [KR][NC] (contiguous); R = 128 the unit's block,
+  // KR rows of 128 columns (row stride RS)
+  const int RS = BPU == 2 ? a.NC : 128;
   if (tid == 0) {
     tc::mbar_init(&ctl.raw_full, 1);
     tc::mbar_init(&ctl.a_full, X_LW * 32);
@@ -117,7 +129,7 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
   __syncthreads();
   tc::fence_after();
   const uint32_t tm = ctl.tmem;
-  // TMEM columns: [0,128) C2^T hi (64 per c-block), [128,256) lo, [256,512) D[2] (128 each:
+  // TMEM columns: [0,128) C2^T hi (KR per c-block), [128,256) lo, [256,512) D[2] (128 each:
   // 64 per c-block).
   const int tpp = a.tpp;
   unsigned long long trc[10] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
@@ -126,39 +138,54 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
 
   if (w < X_LW) {
     // ------------------------------- loaders -------------------------------
-    const int blk = w >> 2, Q = w & 3;
-    const int c = blk * 128 + Q * 32 + lane;
-    const bool cval = c < a.NC;
-    const bool bact = blk < a.nblk;
+    // thread = C2^T row (column c of the slice) x 64 r1 values: R = 64 warps 0-3 / 4-7 take the
+    // two c-blocks, R = 128 they take r1 [0, 64) / [64, 128) of the unit's block
+    const int wb = w >> 2, Q = w & 3;
+    const int blk = BPU == 2 ? wb : 0, r0 = BPU == 2 ? 0 : 64 * wb;
+    const int cl = blk * 128 + Q * 32 + lane;      // column inside the staged raw block
     float xa[32], xb[32];
     uint32_t ui = 0, gs = 0, rawk = 0;
-    auto load_raw = [&]() {          // regs <- raw (this thread's column c, all r1)
+    bool cval = false;
+    auto col_valid = [&](uint32_t u) { return ((int)(u % UPG) * BPU * 128 + cl) < a.NC; };
+    auto load_raw = [&]() {          // regs <- raw (this thread's column, 64 r1)
 #pragma unroll
       for (int r = 0; r < 32; ++r) {
-        xa[r] = cval ? raw[r * a.NC + c] : 0.f;
-        xb[r] = cval ? raw[(r + 32) * a.NC + c] : 0.f;
+        xa[r] = cval ? raw[(r0 + r) * RS + cl] : 0.f;
+        xb[r] = cval ? raw[(r0 + r + 32) * RS + cl] : 0.f;
       }
     };
-    auto issue_raw = [&](uint32_t g) {
-      tc::mbar_arrive_tx(&ctl.raw_full, raw_bytes);
-      tc::bulk_g2s(tc::smem_u32(raw), a.cores + a.grp_c2[g], raw_bytes, &ctl.raw_full);
+    auto issue_raw = [&](uint32_t u) {   // thread 0: the unit's C2 columns -> raw
+      const uint32_t g = u / UPG, ub = u % UPG;
+      const float* src = a.cores + a.grp_c2[g];
+      if (BPU == 2) {
+        const uint32_t bytes = (uint32_t)KR * a.NC * 4u;
+        tc::mbar_arrive_tx(&ctl.raw_full, bytes);
+        tc::bulk_g2s(tc::smem_u32(raw), src, bytes, &ctl.raw_full);
+      } else {
+        const int c0 = (int)ub * 128, nc = min(128, a.NC - c0);
+        tc::mbar_arrive_tx(&ctl.raw_full, (uint32_t)(KR * nc * 4));
+        for (int r = 0; r < KR; ++r)
+          tc::bulk_g2s(tc::smem_u32(raw + r * 128), src + (size_t)r * a.NC + c0, (uint32_t)(nc * 4), &ctl.raw_full);
+      }
     };
     if (tid == 0) {
       ctl.claim[0] = atomicAdd(a.work, 1u);
       ctl.claim[1] = atomicAdd(a.work, 1u);
-      if (ctl.claim[0] < NG) issue_raw(ctl.claim[0]);
+      if (ctl.claim[0] < NU) issue_raw(ctl.claim[0]);
     }
     tc::named_sync(1, X_LW * 32);
     uint32_t cur = ctl.claim[0], nxt = ctl.claim[1];
-    if (cur < NG) {
+    if (cur < NU) {
       tc::mbar_wait(&ctl.raw_full, rawk & 1);
       ++rawk;
+      cval = col_valid(cur);
       load_raw();
     }
     tc::named_sync(1, X_LW * 32);
-    if (tid == 0 && nxt < NG) issue_raw(nxt);
-    while (cur < NG) {
-      const uint32_t q0 = a.grp_off[cur], q1 = a.grp_off[cur + 1];
+    if (tid == 0 && nxt < NU) issue_raw(nxt);
+    while (cur < NU) {
+      const uint32_t g = cur / UPG, ub = cur % UPG;
+      const uint32_t q0 = a.grp_off[g], q1 = a.grp_off[g + 1];
       for (uint32_t qa = q0; qa < q1; qa += tpp, ++ui) {
         const uint32_t np = min((uint32_t)tpp, q1 - qa);
         const int rows = (int)np << a.n1s;
@@ -166,32 +193,32 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
         XT0();
         if (tid == 0) {
           tc::mbar_wait(&ctl.u_empty[ui & 3], ((ui >> 2) & 1) ^ 1);
-          ctl.ring[ui & 3][0] = cur; ctl.ring[ui & 3][1] = qa; ctl.ring[ui & 3][2] = np; ctl.ring[ui & 3][3] = fl;
-          ctl.ring[ui & 3][4] = a.row_seg[qa]; ctl.ring[ui & 3][5] = a.row_seg[qa + np];
+          ctl.ring[ui & 3][0] = g; ctl.ring[ui & 3][1] = qa; ctl.ring[ui & 3][2] = np; ctl.ring[ui & 3][3] = fl;
+          ctl.ring[ui & 3][4] = ub;
           tc::mbar_arrive(&ctl.u_full[ui & 3]);
         }
-        // C1 rows of the tile -> registers (B = CM(m, r1), m = tid & 63, 4 float4 of r1)
+        // C1 rows of the tile -> registers (B = CM(m, r1), m = tid & 63, KR / 16 float4 of r1)
         const int m = tid & 63;
-        float4 bv[4];
+        float4 bv[KR / 16];
         {
           const bool ok = m < rows;
           const uint32_t arow = ok ? a.grp_arow[qa + (m >> a.n1s)] + (m & ((1 << a.n1s) - 1)) : 0u;
-          const float4* src = reinterpret_cast<const float4*>(a.cores + (size_t)arow * XR);
+          const float4* src = reinterpret_cast<const float4*>(a.cores + (size_t)arow * KR);
 #pragma unroll
-          for (int k = 0; k < 4; ++k) bv[k] = ok ? __ldg(src + (tid >> 6) + 4 * k) : make_float4(0.f, 0.f, 0.f, 0.f);
+          for (int k = 0; k < KR / 16; ++k) bv[k] = ok ? __ldg(src + (tid >> 6) + 4 * k) : make_float4(0.f, 0.f, 0.f, 0.f);
         }
         XTA(0);
-        if (fl & 1u) {   // the group's C2^T -> TMEM (hi = raw fp32, lo = x - trunc_tf32(x))
+        if (fl & 1u) {   // the unit's C2^T -> TMEM (hi = raw fp32, lo = x - trunc_tf32(x))
           tc::mbar_wait(&ctl.a_free, (gs & 1) ^ 1);
           XTA(1);
           tc::fence_after();
-          if (bact) {
-            tc::tmem_st32(tc::taddr(tm + blk * 64, 32 * Q, 0), xa);
-            tc::tmem_st32(tc::taddr(tm + blk * 64 + 32, 32 * Q, 0), xb);
+          if (BPU == 1 || blk < a.nblk) {
+            tc::tmem_st32(tc::taddr(tm + blk * KR + r0, 32 * Q, 0), xa);
+            tc::tmem_st32(tc::taddr(tm + blk * KR + r0 + 32, 32 * Q, 0), xb);
 #pragma unroll
             for (int r = 0; r < 32; ++r) { xa[r] = tf32_lo(xa[r]); xb[r] = tf32_lo(xb[r]); }
-            tc::tmem_st32(tc::taddr(tm + 128 + blk * 64, 32 * Q, 0), xa);
-            tc::tmem_st32(tc::taddr(tm + 128 + blk * 64 + 32, 32 * Q, 0), xb);
+            tc::tmem_st32(tc::taddr(tm + 128 + blk * KR + r0, 32 * Q, 0), xa);
+            tc::tmem_st32(tc::taddr(tm + 128 + blk * KR + r0 + 32, 32 * Q, 0), xb);
             tc::tmem_wait_st();
           }
           tc::fence_before();
@@ -202,10 +229,10 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
           const uint32_t s = ui & 1;
           tc::mbar_wait(&ctl.b_free[s], ((ui >> 1) & 1) ^ 1);
           XTA(3);
-          char* bh = bbuf + s * XB_SLOT;
-          char* bl = bh + XB_HALF;
+          char* bh = bbuf + s * BSLOT;
+          char* bl = bh + BHALF;
 #pragma unroll
-          for (int k = 0; k < 4; ++k) {
+          for (int k = 0; k < KR / 16; ++k) {
             const uint32_t off = tc::cm_off(m, 4 * ((tid >> 6) + 4 * k), XT / 8);
             const float4 v = bv[k];
             *reinterpret_cast<float4*>(bh + off) = v;
@@ -217,18 +244,19 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
         }
       }
       XT0();
-      // next group: registers <- raw (nxt); raw <- the group after (claimed now)
+      // next unit: registers <- raw (nxt); raw <- the unit after (claimed now)
       if (tid == 0) ctl.claim[gs & 1] = atomicAdd(a.work, 1u);
-      if (nxt < NG) {
+      if (nxt < NU) {
         tc::mbar_wait(&ctl.raw_full, rawk & 1);
         ++rawk;
         XTA(5);
+        cval = col_valid(nxt);
         load_raw();
       }
       tc::named_sync(1, X_LW * 32);
       XTA(6);
       const uint32_t nn = ctl.claim[gs & 1];
-      if (tid == 0 && nn < NG) issue_raw(nn);
+      if (tid == 0 && nn < NU) issue_raw(nn);
       ++gs;
       cur = nxt;
       nxt = nn;
@@ -245,7 +273,7 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
       XT0();
       tc::mbar_wait(&ctl.u_full[ui & 3], (ui >> 2) & 1);
       XTA(0);
-      const uint32_t np = ctl.ring[ui & 3][2], fl = ctl.ring[ui & 3][3];
+      const uint32_t np = ctl.ring[ui & 3][2], fl = ctl.ring[ui & 3][3], ub = ctl.ring[ui & 3][4];
       __syncwarp();
       if (lane == 0) tc::mbar_arrive(&ctl.u_empty[ui & 3]);
       if (fl & 4u) break;
@@ -261,15 +289,15 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
       tc::fence_after();
       if (lane == 0) {
         const uint32_t id = tc::idesc_tf32(128, n16, false, false);
-        const uint32_t bh = tc::smem_u32(bbuf + s * XB_SLOT), bl = bh + XB_HALF;
-        for (int blk = 0; blk < a.nblk; ++blk) {
+        const uint32_t bh = tc::smem_u32(bbuf + s * BSLOT), bl = bh + BHALF;
+        for (int blk = 0; blk < BPU && (int)ub * BPU + blk < a.nblk; ++blk) {
           const uint32_t d = tm + 256 + s * 128 + blk * 64;
 #pragma unroll
-          for (int kk = 0; kk < XR / 8; ++kk) {
+          for (int kk = 0; kk < KR / 8; ++kk) {
             const uint32_t o = kk * 2 * (XT / 8) * 128;
             const uint64_t dbh = tc::sdesc(bh + o, (XT / 8) * 128, 128);
             const uint64_t dbl = tc::sdesc(bl + o, (XT / 8) * 128, 128);
-            const uint32_t ah = tm + blk * 64 + kk * 8, al = tm + 128 + blk * 64 + kk * 8;
+            const uint32_t ah = tm + blk * KR + kk * 8, al = tm + 128 + blk * KR + kk * 8;
             tc::mma_tf32_ts(d, ah, dbh, id, kk > 0 ? 1u : 0u);
             tc::mma_tf32_ts(d, ah, dbl, id, 1u);
             tc::mma_tf32_ts(d, al, dbh, id, 1u);
@@ -286,14 +314,15 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
     }
   } else {
     // ------------------------- epilogue: TMEM -> P stash -------------------------
-    // warp w drains lane quarter Q = w % 4 of every c-block: thread = column c, 32 tile rows
-    // per tcgen05.ld; pbuf[(q n1 + j1)][c] rows of one tile are contiguous (group-major plan)
+    // warp w drains lane quarter Q = w % 4 of every c-block of the unit: thread = column c, 32
+    // tile rows per tcgen05.ld; pbuf[(q n1 + j1)][c] rows of one tile are contiguous
     const int Q = w & 3;
     for (uint32_t ui = 0;; ++ui) {
       XT0();
       tc::mbar_wait(&ctl.u_full[ui & 3], (ui >> 2) & 1);
       XTA(0);
       const uint32_t qa = ctl.ring[ui & 3][1], np = ctl.ring[ui & 3][2], fl = ctl.ring[ui & 3][3];
+      const uint32_t ub = ctl.ring[ui & 3][4];
       __syncwarp();
       if (fl & 4u) break;
       const int rows = (int)np << a.n1s;
@@ -302,8 +331,8 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
       XTA(1);
       tc::fence_after();
       float* dst = a.pbuf + (size_t)qa * a.n1 * a.NC;
-      for (int blk = 0; blk < a.nblk; ++blk) {
-        const int c = blk * 128 + Q * 32 + lane;
+      for (int blk = 0; blk < BPU; ++blk) {
+        const int c = ((int)ub * BPU + blk) * 128 + Q * 32 + lane;
         for (int j0 = 0; j0 < rows; j0 += 32) {
           float v[32];
           tc::tmem_ld32(tc::taddr(tm + 256 + s * 128 + blk * 64 + j0, 32 * Q, 0), v);
@@ -338,7 +367,7 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
   if (w == X_MMA_W) tc::tmem_dealloc(tm, 512);
 }
 
-constexpr size_t kPrefixSmem = 128 + X_RAW_BYTES + 2 * XB_SLOT;
+template <int KR> constexpr size_t prefix_smem() { return 128 + X_RAW_BYTES + 2 * (2u * XT * KR * 4); }
 
 // ------------------------------------------------------------------------------------
 // Row contraction a6 (Eq. 2, Fig. 5(b) step 3): E_u = P_q (n1 n2 x R) . C3[i3_u] (R x n3)
@@ -363,10 +392,11 @@ struct RowArgs {
   int n1, n1s, n2, N, NC;
 };
 
-template <int N3>
-__global__ void __launch_bounds__(RW_WARPS * 32, 3) k_rows_fwd2(RowArgs a) {
-  constexpr int SLOT = XR * N3 + 32;
-  constexpr int C3L = XR * N3 / 4 / 32;
+template <int N3, int RPL>   // RPL = R / 8: r values per lane (8 at R = 64, 16 at R = 128)
+__global__ void __launch_bounds__(RW_WARPS * 32, RPL == 8 ? 3 : 2) k_rows_fwd2(RowArgs a) {
+  constexpr int KR = 8 * RPL;
+  constexpr int SLOT = KR * N3 + KR / 2;       // + 4 floats of skew per 8 rows of r
+  constexpr int C3L = KR * N3 / 4 / 32;
   extern __shared__ __align__(16) float rw_smem[];
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   float* const ringp = rw_smem + w * (RW_NSL * SLOT);
@@ -379,7 +409,7 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 3) k_rows_fwd2(RowArgs a) {
 #pragma unroll
   for (int e = 0; e < 4; ++e) {
     const int j12 = 4 * jq + e, j1 = j12 / a.n2, j2 = j12 - j1 * a.n2;
-    poff[e] = j12 < J12 ? j1 * a.NC + j2 * XR + 8 * rp : -1;
+    poff[e] = j12 < J12 ? j1 * a.NC + j2 * KR + RPL * rp : -1;
   }
   const int64_t nch = ((int64_t)U + RW_RCH - 1) / RW_RCH;
   const int64_t gw = (int64_t)blockIdx.x * RW_WARPS + w, nw = (int64_t)gridDim.x * RW_WARPS;
@@ -390,7 +420,7 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 3) k_rows_fwd2(RowArgs a) {
     unsigned long long o3l = 0;
     if (lane < nr) {
       ql = __ldg(a.row_pfx + u0 + lane);
-      o3l = a.meta[__ldg(a.pfx_t + ql)].c3_off + (unsigned long long)__ldg(a.row_i3 + u0 + lane) * XR * N3;
+      o3l = a.meta[__ldg(a.pfx_t + ql)].c3_off + (unsigned long long)__ldg(a.row_i3 + u0 + lane) * KR * N3;
     }
     auto issue = [&](int j) {
       const unsigned long long o3 = __shfl_sync(0xffffffffu, o3l, j);
@@ -399,7 +429,7 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 3) k_rows_fwd2(RowArgs a) {
 #pragma unroll
       for (int i = 0; i < C3L; ++i) {
         const int f = lane + 32 * i, r = f / (N3 / 4);
-        tc::cp_async16(dst + 4u * (uint32_t)(4 * f + 4 * ((r >> 3) & 7)), src + f);
+        tc::cp_async16(dst + 4u * (uint32_t)(4 * f + 4 * (r >> 3)), src + f);
       }
     };
 #pragma unroll
@@ -408,21 +438,19 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 3) k_rows_fwd2(RowArgs a) {
       tc::cp_commit();
     }
     uint32_t curq = 0xffffffffu;
-    float pr[4][8];
+    float pr[4][RPL];
     for (int j = 0; j < nr; ++j) {
       const uint32_t q = __shfl_sync(0xffffffffu, ql, j);
       if (q != curq) {
         const float* pq = a.pbuf + (size_t)q * a.n1 * a.NC;
 #pragma unroll
-        for (int e = 0; e < 4; ++e) {
-          float4 x0 = make_float4(0.f, 0.f, 0.f, 0.f), x1 = x0;
-          if (poff[e] >= 0) {
-            x0 = __ldg(reinterpret_cast<const float4*>(pq + poff[e]));
-            x1 = __ldg(reinterpret_cast<const float4*>(pq + poff[e] + 4));
+        for (int e = 0; e < 4; ++e)
+#pragma unroll
+          for (int h = 0; h < RPL; h += 4) {
+            const float4 x0 = poff[e] >= 0 ? __ldg(reinterpret_cast<const float4*>(pq + poff[e] + h))
+                                           : make_float4(0.f, 0.f, 0.f, 0.f);
+            pr[e][h] = x0.x; pr[e][h + 1] = x0.y; pr[e][h + 2] = x0.z; pr[e][h + 3] = x0.w;
           }
-          pr[e][0] = x0.x; pr[e][1] = x0.y; pr[e][2] = x0.z; pr[e][3] = x0.w;
-          pr[e][4] = x1.x; pr[e][5] = x1.y; pr[e][6] = x1.z; pr[e][7] = x1.w;
-        }
         curq = q;
       }
       tc::cp_wait<RW_NSL - 2>();
@@ -430,13 +458,15 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 3) k_rows_fwd2(RowArgs a) {
       float acc[4 * N3];
 #pragma unroll
       for (int i = 0; i < 4 * N3; ++i) acc[i] = 0.f;
-      const float* c3 = ringp + (j % RW_NSL) * SLOT + (8 * rp) * N3 + 4 * rp;
+      const float* slot3 = ringp + (j % RW_NSL) * SLOT;
 #pragma unroll
-      for (int x = 0; x < 8; ++x) {
+      for (int x = 0; x < RPL; ++x) {
+        const int r = RPL * rp + x;
+        const float* c3 = slot3 + r * N3 + 4 * (r >> 3);   // the ring's per-8-row skew
         float cv[N3];
 #pragma unroll
         for (int b = 0; b < N3; b += 4) {
-          const float4 t4 = *reinterpret_cast<const float4*>(c3 + x * N3 + b);
+          const float4 t4 = *reinterpret_cast<const float4*>(c3 + b);
           cv[b] = t4.x; cv[b + 1] = t4.y; cv[b + 2] = t4.z; cv[b + 3] = t4.w;
         }
 #pragma unroll
@@ -470,7 +500,7 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 3) k_rows_fwd2(RowArgs a) {
   }
 }
 
-size_t rows_smem(int n3) { return (size_t)RW_WARPS * RW_NSL * (XR * n3 + 32) * 4; }
+size_t rows_smem(int n3, int R) { return (size_t)RW_WARPS * RW_NSL * (R * n3 + R / 2) * 4; }
 
 // ------------------------------------------------------------------------------------
 // Row backward a9 (Eq. 6 read as left^T . dL/de . right^T), same lane map and
@@ -490,7 +520,7 @@ struct RowBwdArgs {
   const float* pbuf;          // [P][n1][NC]
   const float* gbuf;          // [U][N]
   float* dpbuf;               // [P][n1][NC]
-  int n1, n2, N, NC;
+  int n1, n2, N, NC, R;
 };
 
 __global__ void __launch_bounds__(256) k_dp_zero2(RowBwdArgs a) {
@@ -522,22 +552,31 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 2) k_rows_bwd2(RowBwdArgs a) {
   const uint32_t U = tt_rows(a.counts);   // TT rows only (hybrid: dense rows follow)
   const int J12 = a.n1 * a.n2;
   const int jq = lane >> 3, rp = lane & 7;
-  int poff[4];
+  // R = 128: a work item is (16 rows, one 64-wide slice of r), the lane map of R = 64 per slice:
+  // dP_q[j12][r] and dC3[i3][r][j3] of a slice are independent of the other slice
+  const int nsl = a.R / XR;
+  int poff0[4];
 #pragma unroll
   for (int e = 0; e < 4; ++e) {
     const int j12 = 4 * jq + e, j1 = j12 / a.n2, j2 = j12 - j1 * a.n2;
-    poff[e] = j12 < J12 ? j1 * a.NC + j2 * XR + 8 * rp : -1;
+    poff0[e] = j12 < J12 ? j1 * a.NC + j2 * a.R + 8 * rp : -1;
   }
   const int64_t nch = ((int64_t)U + RW_RCH - 1) / RW_RCH;
   const int64_t gw = (int64_t)blockIdx.x * RW_WARPS + w, nw = (int64_t)gridDim.x * RW_WARPS;
-  for (int64_t ch = gw; ch < nch; ch += nw) {
+  for (int64_t it = gw; it < nch * nsl; it += nw) {
+    const int64_t ch = it / nsl;
+    const int rb = XR * (int)(it - ch * nsl);     // first r of the slice
+    int poff[4];
+#pragma unroll
+    for (int e = 0; e < 4; ++e) poff[e] = poff0[e] >= 0 ? poff0[e] + rb : -1;
     const uint32_t u0 = (uint32_t)ch * RW_RCH;
     const int nr = (int)min((uint32_t)RW_RCH, U - u0);
     uint32_t ql = 0;
     unsigned long long o3l = 0;
     if (lane < nr) {
       ql = __ldg(a.row_pfx + u0 + lane);
-      o3l = a.meta[__ldg(a.pfx_t + ql)].c3_off + (unsigned long long)__ldg(a.row_i3 + u0 + lane) * XR * N3;
+      o3l = a.meta[__ldg(a.pfx_t + ql)].c3_off + (unsigned long long)__ldg(a.row_i3 + u0 + lane) * a.R * N3 +
+            (unsigned long long)rb * N3;
     }
     const uint32_t prevq = u0 > 0 ? __ldg(a.row_pfx + u0 - 1) : 0xffffffffu;
     const uint32_t nextq = u0 + nr < U ? __ldg(a.row_pfx + u0 + nr) : 0xffffffffu;
@@ -657,12 +696,13 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 2) k_rows_bwd2(RowBwdArgs a) {
   }
 }
 
-size_t rows_bwd_smem(int n3) { return (size_t)RW_WARPS * RW_NSL * (XR * n3 + 32 + 16 * n3) * 4; }
+size_t rows_bwd_smem(int n3) { return (size_t)RW_WARPS * RW_NSL * (XR * n3 + 32 + 16 * n3) * 4; }   // per 64-r slice
 
 }  // namespace
 
 bool fused_eligible(const Ctx& c) {
-  return !(c.flags & TTEMB_FP32_CORES) && c.R == XR && c.NC <= 256 &&
+  // R = 64 (and ranks 16..63 stored padded to 64) with n2 R <= 256; R = 128 with n2 R <= 512
+  return !(c.flags & TTEMB_FP32_CORES) && (c.R == 64 || c.R == 128) && c.NC <= 4 * c.R &&
          (c.n3 == 4 || c.n3 == 8) && (c.n1 == 1 || c.n1 == 2 || c.n1 == 4 || c.n1 == 8) && c.n1 * c.n2 <= 16;
 }
 bool tc_eligible(const Ctx& c) { return fused_eligible(c); }
@@ -670,15 +710,18 @@ cudaError_t configure_tc(Ctx&) { return cudaSuccess; }
 
 cudaError_t configure_fused(Ctx& c) {
   if (!fused_eligible(c)) return cudaSuccess;
-  cudaError_t e = cudaFuncSetAttribute(k_prefix_fwd, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kPrefixSmem);
-  if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(k_rows_fwd2<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)rows_smem(4));
-  if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(k_rows_fwd2<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)rows_smem(8));
-  if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(k_rows_bwd2<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)rows_bwd_smem(4));
-  if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(k_rows_bwd2<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)rows_bwd_smem(8));
+  cudaError_t e = cudaSuccess;
+  auto set = [&](const void* f, size_t bytes) {
+    if (e == cudaSuccess) e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
+  };
+  set((const void*)k_prefix_fwd<64>, prefix_smem<64>());
+  set((const void*)k_prefix_fwd<128>, prefix_smem<128>());
+  set((const void*)k_rows_fwd2<4, 8>, rows_smem(4, 64));
+  set((const void*)k_rows_fwd2<8, 8>, rows_smem(8, 64));
+  set((const void*)k_rows_fwd2<4, 16>, rows_smem(4, 128));
+  set((const void*)k_rows_fwd2<8, 16>, rows_smem(8, 128));
+  set((const void*)k_rows_bwd2<4>, rows_bwd_smem(4));
+  set((const void*)k_rows_bwd2<8>, rows_bwd_smem(8));
   return e;
 }
 
@@ -691,7 +734,7 @@ cudaError_t run_fused_fwd(Ctx& c, float* out, cudaStream_t s) {
   a.work = p.work + 0;
   a.dbg = knobs().dbg;
   a.n1 = c.n1; a.n1s = c.n1 == 1 ? 0 : c.n1 == 2 ? 1 : c.n1 == 4 ? 2 : 3;
-  a.n2 = c.n2; a.n3 = c.n3; a.N = c.N; a.NC = c.NC; a.nblk = (c.NC + 127) / 128; a.tpp = XT / c.n1;
+  a.n2 = c.n2; a.n3 = c.n3; a.N = c.N; a.NC = c.NC; a.nblk = (c.NC + 127) / 128; a.tpp = XT / c.n1; a.R = c.R;
   {
     StageScope sc(c, ST_FWD_PREFIX, s);
     k_fused_prep<<<grid_for(c, std::max(c.P_cap, c.NG_cap), 256, 4), 256, 0, s>>>(a);
@@ -703,7 +746,8 @@ cudaError_t run_fused_fwd(Ctx& c, float* out, cudaStream_t s) {
       cudaMemsetAsync(trace, 0, sizeof(unsigned long long) * 32 * grid, s);
       a.trace = trace;
     }
-    k_prefix_fwd<<<grid, X_THREADS, kPrefixSmem, s>>>(a);
+    if (c.R == 64) k_prefix_fwd<64><<<grid, X_THREADS, prefix_smem<64>(), s>>>(a);
+    else k_prefix_fwd<128><<<grid, X_THREADS, prefix_smem<128>(), s>>>(a);
     if (a.trace) {
       std::vector<unsigned long long> hb(32 * grid);
       cudaMemcpyAsync(hb.data(), trace, hb.size() * 8, cudaMemcpyDeviceToHost, s);
@@ -733,8 +777,13 @@ cudaError_t run_fused_fwd(Ctx& c, float* out, cudaStream_t s) {
     r.pfx_t = p.pfx_t; r.pbuf = p.pbuf; r.rows = p.rows; r.seg_off = p.seg_off; r.sbag = p.sbag; r.out = out;
     r.n1 = c.n1; r.n1s = a.n1s; r.n2 = c.n2; r.N = c.N; r.NC = c.NC;
     const int grid = grid_for(c, cdiv(c.U_cap, RW_RCH), RW_WARPS, 4);
-    if (c.n3 == 4) k_rows_fwd2<4><<<grid, RW_WARPS * 32, rows_smem(4), s>>>(r);
-    else k_rows_fwd2<8><<<grid, RW_WARPS * 32, rows_smem(8), s>>>(r);
+    if (c.R == 64) {
+      if (c.n3 == 4) k_rows_fwd2<4, 8><<<grid, RW_WARPS * 32, rows_smem(4, 64), s>>>(r);
+      else k_rows_fwd2<8, 8><<<grid, RW_WARPS * 32, rows_smem(8, 64), s>>>(r);
+    } else {
+      if (c.n3 == 4) k_rows_fwd2<4, 16><<<grid, RW_WARPS * 32, rows_smem(4, 128), s>>>(r);
+      else k_rows_fwd2<8, 16><<<grid, RW_WARPS * 32, rows_smem(8, 128), s>>>(r);
+    }
   }
   return cudaGetLastError();
 }
@@ -747,7 +796,7 @@ cudaError_t run_dp_zero(Ctx& c, cudaStream_t s) {
   RowBwdArgs r;
   r.cores = c.cores; r.grads = c.grads; r.meta = c.d_meta; r.counts = p.counts; r.row_pfx = p.row_pfx;
   r.row_i3 = p.row_i3; r.pfx_t = p.pfx_t; r.row_seg = p.row_seg; r.pbuf = p.pbuf; r.gbuf = p.gbuf;
-  r.dpbuf = p.dpbuf; r.n1 = c.n1; r.n2 = c.n2; r.N = c.N; r.NC = c.NC;
+  r.dpbuf = p.dpbuf; r.n1 = c.n1; r.n2 = c.n2; r.N = c.N; r.NC = c.NC; r.R = c.R;
   k_dp_zero2<<<grid_for(c, c.P_cap, 8, 8), 256, 0, s>>>(r);
   return cudaGetLastError();
 }
@@ -757,9 +806,9 @@ cudaError_t run_rows_bwd2(Ctx& c, cudaStream_t s) {
   RowBwdArgs r;
   r.cores = c.cores; r.grads = c.grads; r.meta = c.d_meta; r.counts = p.counts; r.row_pfx = p.row_pfx;
   r.row_i3 = p.row_i3; r.pfx_t = p.pfx_t; r.row_seg = p.row_seg; r.pbuf = p.pbuf; r.gbuf = p.gbuf;
-  r.dpbuf = p.dpbuf; r.n1 = c.n1; r.n2 = c.n2; r.N = c.N; r.NC = c.NC;
+  r.dpbuf = p.dpbuf; r.n1 = c.n1; r.n2 = c.n2; r.N = c.N; r.NC = c.NC; r.R = c.R;
   // (the dP rows of chunk-straddling prefixes were zeroed at the end of the index stage)
-  const int grid = grid_for(c, cdiv(c.U_cap, RW_RCH), RW_WARPS, 2);
+  const int grid = grid_for(c, cdiv(c.U_cap, RW_RCH) * (c.R / XR), RW_WARPS, 2);
   if (c.n3 == 4) k_rows_bwd2<4><<<grid, RW_WARPS * 32, rows_bwd_smem(4), s>>>(r);
   else k_rows_bwd2<8><<<grid, RW_WARPS * 32, rows_bwd_smem(8), s>>>(r);
   return cudaGetLastError();
