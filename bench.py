@@ -703,9 +703,10 @@ def main():
 def tc_path(cfg, args):
     """The tcgen05 path (R = 64, n2 R <= 256, n3 in {4, 8}, n1 a power of two <= 8)."""
     n1, n2, n3 = cfg.col_factors
-    R = 64 if 16 <= cfg.rank <= 64 else cfg.rank       # ranks 16..63 run zero-padded to 64
-    return (not args.fp32_cores) and R in (64, 128) and n3 in (4, 8) and n1 in (1, 2, 4, 8) \
-        and n1 * n2 <= 16 and n2 * R <= 4 * R
+    # ranks 16..31 / 33..63 run zero-padded to 32 / 64 (DESIGN.md R28); 32, 64, 128 natively
+    R = 32 if 16 <= cfg.rank <= 32 else 64 if 32 < cfg.rank <= 64 else cfg.rank
+    return (not args.fp32_cores) and R in (32, 64, 128) and n3 in (4, 8) and n1 in (1, 2, 4, 8) \
+        and n1 * n2 <= 16 and n2 * R <= (512 if R == 128 else 256)
 
 
 def emb_passes(emb):

@@ -87,10 +87,11 @@ typedef struct {
   int32_t num_cores;             /* must be 3 (the paper's design)         */
   int32_t dim;                   /* N = col_factors[0]*col_factors[1]*col_factors[2]  */
   int32_t col_factors[3];        /* (n1, n2, n3), shared by all tables                */
-  int32_t rank;                  /* R1 = R2 = rank (1..128), R0 = R3 = 1; on
-                                    the tensor-core path a rank 16..63 is STORED zero-padded
-                                    to 64 (ttemb_core_layout reports the storage shapes;
-                                    padding entries must be 0 and stay 0)               */
+  int32_t rank;                  /* R1 = R2 = rank (1..128), R0 = R3 = 1; the
+                                    tensor-core path runs R = 32, 64, 128 natively and STORES
+                                    a rank 16..31 / 33..63 zero-padded to 32 / 64
+                                    (ttemb_core_layout reports the storage shapes; padding
+                                    entries must be 0 and stay 0)                         */
   int32_t index_bits;            /* 64 (int64 ids, PyTorch default) or 32             */
   int32_t max_batch;             /* B capacity (workspace sizing)                     */
   int64_t max_nnz;               /* nnz capacity, <= 2^30                             */

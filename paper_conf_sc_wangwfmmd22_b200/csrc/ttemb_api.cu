@@ -112,13 +112,16 @@ void plan_sizes(const ttemb_config* cfg, Ctx& c) {
   c.T = cfg->num_tables;
   c.n1 = cfg->col_factors[0]; c.n2 = cfg->col_factors[1]; c.n3 = cfg->col_factors[2];
   c.N = cfg->dim; c.R = cfg->rank;
-  // kPadMinRank <= R < 64: store the cores zero-padded to rank 64 and run the tcgen05 path.  Exact: the
-  // padded rows / columns of C1, C2, C3 multiply only zeros, so every padded entry of dC_k is
-  // exactly 0 and SGD / Adagrad keep it 0 (R28).
+  // kPadMinRank <= R < 32 / 32 < R < 64: store the cores zero-padded to rank 32 / 64 and run the
+  // tcgen05 path (native kernels exist for R = 32, 64, 128).  Exact: the padded rows / columns of
+  // C1, C2, C3 multiply only zeros, so every padded entry of dC_k is exactly 0 and SGD / Adagrad
+  // keep it 0 (R28).
   c.R_user = c.R;
-  if (!(cfg->flags & TTEMB_FP32_CORES) && c.R >= kPadMinRank && c.R < 64 && (c.n3 == 4 || c.n3 == 8) &&
-      (c.n1 == 1 || c.n1 == 2 || c.n1 == 4 || c.n1 == 8) && c.n1 * c.n2 <= 16 && c.n2 * 64 <= 256)
-    c.R = 64;
+  if (!(cfg->flags & TTEMB_FP32_CORES) && c.R >= kPadMinRank && c.R < 64 && c.R != 32 && (c.n3 == 4 || c.n3 == 8) &&
+      (c.n1 == 1 || c.n1 == 2 || c.n1 == 4 || c.n1 == 8) && c.n1 * c.n2 <= 16) {
+    const int padded = c.R < 32 ? 32 : 64;
+    if (c.n2 * padded <= 256) c.R = padded;
+  }
   c.NC = c.n2 * c.R;
   c.index_bits = cfg->index_bits; c.opt = cfg->optimizer;
   c.eps = cfg->adagrad_eps; c.flags = cfg->flags;

@@ -53,8 +53,8 @@ constexpr int Y_GI = 64;                        // work units per CTA whose meta
 // unit per c-block (the dC2 / dA accumulators are N = 128 wide), 32-column chunks (the C2 chunk
 // [CK][KR] hi + lo then fits three stages).
 template <int KR> struct YShape {
-  static constexpr int BPU = KR == 64 ? 2 : 1;
-  static constexpr int CK = KR == 64 ? 64 : 32;
+  static constexpr int BPU = KR <= 64 ? 2 : 1;
+  static constexpr int CK = KR <= 64 ? 64 : 32;
   static constexpr int A2S = CK + 4;                                    // dP staging row stride (floats)
   static constexpr uint32_t A2 = YT * A2S * 4;                          // dP chunk staging
   static constexpr uint32_t B2LBO = (KR / 8) * 128;                     // CM(KR r1, CK c) core-column stride
@@ -548,6 +548,8 @@ cudaError_t configure_bwdtc(Ctx& c) {
   cudaError_t e = cudaFuncSetAttribute(k_prefix_bwd<64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)YShape<64>::SMEM);
   if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(k_prefix_bwd<32>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)YShape<32>::SMEM);
+  if (e == cudaSuccess)
     e = cudaFuncSetAttribute(k_prefix_bwd<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)YShape<128>::SMEM);
   return e;
 }
@@ -564,12 +566,12 @@ cudaError_t run_prefix_bwd(Ctx& c, float lr, cudaStream_t s) {
   a.NC = c.NC; a.nblk = (c.NC + 127) / 128; a.tpp = YT / c.n1; a.R = c.R;
   // K-chunks per work unit: R = 64 the whole slice in 64-column chunks, R = 128 one c-block in
   // 32-column chunks
-  a.nchunk = c.R == 64 ? (c.NC + 63) / 64 : 128 / YShape<128>::CK;
+  a.nchunk = c.R <= 64 ? (c.NC + 63) / 64 : 128 / YShape<128>::CK;
   a.lr = lr; a.eps = c.eps; a.opt = c.opt; a.fused = (c.flags & TTEMB_FUSED_UPDATE) ? 1 : 0;
   a.exp = exp_bits();
   a.pf = knobs().pf_bwd;
   StageScope sc(c, ST_BWD_PREFIX, s);
-  const int64_t units = c.NG_cap * (c.R == 64 ? 1 : (c.NC + 127) / 128);
+  const int64_t units = c.NG_cap * (c.R <= 64 ? 1 : (c.NC + 127) / 128);
   const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(units, (int64_t)c.sm_count));
   static unsigned long long* trace = nullptr;
   a.trace = nullptr;
@@ -578,7 +580,8 @@ cudaError_t run_prefix_bwd(Ctx& c, float lr, cudaStream_t s) {
     cudaMemsetAsync(trace, 0, sizeof(unsigned long long) * 32 * grid, s);
     a.trace = trace;
   }
-  if (c.R == 64) k_prefix_bwd<64><<<grid, Y_THREADS, YShape<64>::SMEM, s>>>(a);
+  if (c.R == 32) k_prefix_bwd<32><<<grid, Y_THREADS, YShape<32>::SMEM, s>>>(a);
+  else if (c.R == 64) k_prefix_bwd<64><<<grid, Y_THREADS, YShape<64>::SMEM, s>>>(a);
   else k_prefix_bwd<128><<<grid, Y_THREADS, YShape<128>::SMEM, s>>>(a);
   if (a.fused && a.opt != TTEMB_SGD)
     k_c2_update_zero<<<c.sm_count * 8, 256, 0, s>>>(c.cores, c.state, c.grads, p.grp_c2, p.counts,

@@ -38,9 +38,6 @@ constexpr int XT = 64;                         // tile rows (prefix, j1) = MMA N
 constexpr int X_LW = 8, X_RW = 4;   // loaders, epilogue warps
 constexpr int X_THREADS = (X_LW + 1 + X_RW) * 32;
 constexpr int X_MMA_W = X_LW, X_ROW_W0 = X_LW + 1;
-constexpr int XPSTR = 256;                     // P_s row stride (floats); columns XOR-swizzled
-constexpr uint32_t XB_SLOT = 2u * XT * XR * 4; // one B slot: hi + lo CM matrices (32 KB)
-constexpr uint32_t XB_HALF = XT * XR * 4;
 constexpr uint32_t X_RAW_BYTES = 65536;        // R x NC fp32, NC <= 256
 
 struct XArgs {
@@ -96,7 +93,7 @@ __device__ __forceinline__ float tf32_lo(float x) { return x - tc::tf32_trunc(x)
 // the C1 rows of a tile are staged once per unit.
 template <int KR>
 __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
-  constexpr int BPU = KR == 64 ? 2 : 1;            // c-blocks per work unit
+  constexpr int BPU = KR <= 64 ? 2 : 1;            // c-blocks per work unit
   constexpr uint32_t BSLOT = 2u * XT * KR * 4;    // one B slot: C1 tile hi + lo (K = KR)
   constexpr uint32_t BHALF = XT * KR * 4;
   extern __shared__ __align__(128) char smem_raw[];
@@ -151,7 +148,7 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
 #pragma unroll
       for (int r = 0; r < 32; ++r) {
         xa[r] = cval ? raw[(r0 + r) * RS + cl] : 0.f;
-        xb[r] = cval ? raw[(r0 + r + 32) * RS + cl] : 0.f;
+        xb[r] = (cval && KR > 32) ? raw[(r0 + r + 32) * RS + cl] : 0.f;
       }
     };
     auto issue_raw = [&](uint32_t u) {   // thread 0: the unit's C2 columns -> raw
@@ -214,11 +211,11 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
           tc::fence_after();
           if (BPU == 1 || blk < a.nblk) {
             tc::tmem_st32(tc::taddr(tm + blk * KR + r0, 32 * Q, 0), xa);
-            tc::tmem_st32(tc::taddr(tm + blk * KR + r0 + 32, 32 * Q, 0), xb);
+            if (KR > 32) tc::tmem_st32(tc::taddr(tm + blk * KR + r0 + 32, 32 * Q, 0), xb);
 #pragma unroll
             for (int r = 0; r < 32; ++r) { xa[r] = tf32_lo(xa[r]); xb[r] = tf32_lo(xb[r]); }
             tc::tmem_st32(tc::taddr(tm + 128 + blk * KR + r0, 32 * Q, 0), xa);
-            tc::tmem_st32(tc::taddr(tm + 128 + blk * KR + r0 + 32, 32 * Q, 0), xb);
+            if (KR > 32) tc::tmem_st32(tc::taddr(tm + 128 + blk * KR + r0 + 32, 32 * Q, 0), xb);
             tc::tmem_wait_st();
           }
           tc::fence_before();
@@ -540,11 +537,12 @@ __device__ __forceinline__ void red_v4(float* addr, float4 v) {
                : "memory");
 }
 
-template <int N3>
+template <int N3, int RPL>   // RPL = r values per lane: 4 (R = 32) or 8 (R = 64; R = 128 in two slices)
 __global__ void __launch_bounds__(RW_WARPS * 32, 2) k_rows_bwd2(RowBwdArgs a) {
-  constexpr int C3S = XR * N3 + 32;             // skewed C3 part of a slot
+  constexpr int SW = 8 * RPL;                   // r width of a work item (a slice of R)
+  constexpr int C3S = SW * N3 + SW / 2;         // skewed C3 part of a slot (+ 4 floats per 8 rows)
   constexpr int SLOT = C3S + 16 * N3;           // + G_u (N <= 16 n3)
-  constexpr int C3L = XR * N3 / 4 / 32;
+  constexpr int C3L = SW * N3 / 4 / 32;
   extern __shared__ __align__(16) float rw_smem[];
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   float* const ringp = rw_smem + w * (RW_NSL * SLOT);
@@ -554,18 +552,18 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 2) k_rows_bwd2(RowBwdArgs a) {
   const int jq = lane >> 3, rp = lane & 7;
   // R = 128: a work item is (16 rows, one 64-wide slice of r), the lane map of R = 64 per slice:
   // dP_q[j12][r] and dC3[i3][r][j3] of a slice are independent of the other slice
-  const int nsl = a.R / XR;
+  const int nsl = a.R / SW;
   int poff0[4];
 #pragma unroll
   for (int e = 0; e < 4; ++e) {
     const int j12 = 4 * jq + e, j1 = j12 / a.n2, j2 = j12 - j1 * a.n2;
-    poff0[e] = j12 < J12 ? j1 * a.NC + j2 * a.R + 8 * rp : -1;
+    poff0[e] = j12 < J12 ? j1 * a.NC + j2 * a.R + RPL * rp : -1;
   }
   const int64_t nch = ((int64_t)U + RW_RCH - 1) / RW_RCH;
   const int64_t gw = (int64_t)blockIdx.x * RW_WARPS + w, nw = (int64_t)gridDim.x * RW_WARPS;
   for (int64_t it = gw; it < nch * nsl; it += nw) {
     const int64_t ch = it / nsl;
-    const int rb = XR * (int)(it - ch * nsl);     // first r of the slice
+    const int rb = SW * (int)(it - ch * nsl);     // first r of the slice
     int poff[4];
 #pragma unroll
     for (int e = 0; e < 4; ++e) poff[e] = poff0[e] >= 0 ? poff0[e] + rb : -1;
@@ -587,7 +585,7 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 2) k_rows_bwd2(RowBwdArgs a) {
 #pragma unroll
       for (int i = 0; i < C3L; ++i) {
         const int f = lane + 32 * i, r = f / (N3 / 4);
-        tc::cp_async16(dst + 4u * (uint32_t)(4 * f + 4 * ((r >> 3) & 7)), src + f);
+        tc::cp_async16(dst + 4u * (uint32_t)(4 * f + 4 * (r >> 3)), src + f);
       }
       if (lane < a.N / 4)
 #if TTEMB_G_EVICT_FIRST
@@ -604,19 +602,18 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 2) k_rows_bwd2(RowBwdArgs a) {
       tc::cp_commit();
     }
     uint32_t curq = 0xffffffffu;
-    float pr[4][8], dp[4][8];
+    float pr[4][RPL], dp[4][RPL];
     auto flush = [&]() {
       const bool red = curq == prevq || curq == nextq;
       float* d = a.dpbuf + (size_t)curq * a.n1 * a.NC;
 #pragma unroll
       for (int e = 0; e < 4; ++e) {
         if (poff[e] < 0) continue;
-        const float4 v0 = make_float4(dp[e][0], dp[e][1], dp[e][2], dp[e][3]);
-        const float4 v1 = make_float4(dp[e][4], dp[e][5], dp[e][6], dp[e][7]);
-        if (red) { red_v4(d + poff[e], v0); red_v4(d + poff[e] + 4, v1); }
-        else {
-          *reinterpret_cast<float4*>(d + poff[e]) = v0;
-          *reinterpret_cast<float4*>(d + poff[e] + 4) = v1;
+#pragma unroll
+        for (int h = 0; h < RPL; h += 4) {
+          const float4 v = make_float4(dp[e][h], dp[e][h + 1], dp[e][h + 2], dp[e][h + 3]);
+          if (red) red_v4(d + poff[e] + h, v);
+          else *reinterpret_cast<float4*>(d + poff[e] + h) = v;
         }
       }
     };
@@ -627,15 +624,14 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 2) k_rows_bwd2(RowBwdArgs a) {
         const float* pq = a.pbuf + (size_t)q * a.n1 * a.NC;
 #pragma unroll
         for (int e = 0; e < 4; ++e) {
-          float4 x0 = make_float4(0.f, 0.f, 0.f, 0.f), x1 = x0;
-          if (poff[e] >= 0) {
-            x0 = __ldg(reinterpret_cast<const float4*>(pq + poff[e]));
-            x1 = __ldg(reinterpret_cast<const float4*>(pq + poff[e] + 4));
-          }
-          pr[e][0] = x0.x; pr[e][1] = x0.y; pr[e][2] = x0.z; pr[e][3] = x0.w;
-          pr[e][4] = x1.x; pr[e][5] = x1.y; pr[e][6] = x1.z; pr[e][7] = x1.w;
 #pragma unroll
-          for (int x = 0; x < 8; ++x) dp[e][x] = 0.f;
+          for (int h = 0; h < RPL; h += 4) {
+            const float4 x0 = poff[e] >= 0 ? __ldg(reinterpret_cast<const float4*>(pq + poff[e] + h))
+                                           : make_float4(0.f, 0.f, 0.f, 0.f);
+            pr[e][h] = x0.x; pr[e][h + 1] = x0.y; pr[e][h + 2] = x0.z; pr[e][h + 3] = x0.w;
+          }
+#pragma unroll
+          for (int x = 0; x < RPL; ++x) dp[e][x] = 0.f;
         }
         curq = q;
       }
@@ -650,14 +646,15 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 2) k_rows_bwd2(RowBwdArgs a) {
           const float4 t4 = *reinterpret_cast<const float4*>(slot + C3S + (4 * jq + e) * N3 + b);
           g[e][b] = t4.x; g[e][b + 1] = t4.y; g[e][b + 2] = t4.z; g[e][b + 3] = t4.w;
         }
-      float dc[8 * N3];
-      const float* c3 = slot + (8 * rp) * N3 + 4 * rp;
+      float dc[RPL * N3];
 #pragma unroll
-      for (int x = 0; x < 8; ++x) {
+      for (int x = 0; x < RPL; ++x) {
+        const int r = RPL * rp + x;
+        const float* c3 = slot + r * N3 + 4 * (r >> 3);   // the ring's per-8-row skew
         float cv[N3];
 #pragma unroll
         for (int b = 0; b < N3; b += 4) {
-          const float4 t4 = *reinterpret_cast<const float4*>(c3 + x * N3 + b);
+          const float4 t4 = *reinterpret_cast<const float4*>(c3 + b);
           cv[b] = t4.x; cv[b + 1] = t4.y; cv[b + 2] = t4.z; cv[b + 3] = t4.w;
         }
 #pragma unroll
@@ -673,10 +670,10 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 2) k_rows_bwd2(RowBwdArgs a) {
       __syncwarp();
       if (j + RW_NSL - 1 < nr) issue(j + RW_NSL - 1);
       tc::cp_commit();
-      // dC3: reduce over jq (lane bits 4, 3); lane keeps r = 8 rp + 2 jq + {0, 1}, all j3
+      // dC3: reduce over jq (lane bits 4, 3); lane keeps r = RPL rp + (RPL / 4) jq + {0 .. RPL/4 - 1}, all j3
 #pragma unroll
       for (int lv = 0; lv < 2; ++lv) {
-        const int mask = 16 >> lv, half = (8 * N3) >> (lv + 1);
+        const int mask = 16 >> lv, half = (RPL * N3) >> (lv + 1);
         const bool hi = (lane & mask) != 0;
 #pragma unroll
         for (int i = 0; i < half; ++i) {
@@ -686,9 +683,9 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 2) k_rows_bwd2(RowBwdArgs a) {
         }
       }
       const unsigned long long o3 = __shfl_sync(0xffffffffu, o3l, j);
-      float* d3 = a.grads + o3 + (size_t)(8 * rp + 2 * jq) * N3;
+      float* d3 = a.grads + o3 + (size_t)(RPL * rp + (RPL / 4) * jq) * N3;
 #pragma unroll
-      for (int i = 0; i < 2 * N3; i += 4) red_v4(d3 + i, make_float4(dc[i], dc[i + 1], dc[i + 2], dc[i + 3]));
+      for (int i = 0; i < (RPL / 4) * N3; i += 4) red_v4(d3 + i, make_float4(dc[i], dc[i + 1], dc[i + 2], dc[i + 3]));
     }
     if (curq != 0xffffffffu) flush();
     tc::cp_wait<0>();
@@ -696,13 +693,14 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 2) k_rows_bwd2(RowBwdArgs a) {
   }
 }
 
-size_t rows_bwd_smem(int n3) { return (size_t)RW_WARPS * RW_NSL * (XR * n3 + 32 + 16 * n3) * 4; }   // per 64-r slice
+size_t rows_bwd_smem(int n3, int sw) { return (size_t)RW_WARPS * RW_NSL * (sw * n3 + sw / 2 + 16 * n3) * 4; }   // per sw-wide r slice
 
 }  // namespace
 
 bool fused_eligible(const Ctx& c) {
   // R = 64 (and ranks 16..63 stored padded to 64) with n2 R <= 256; R = 128 with n2 R <= 512
-  return !(c.flags & TTEMB_FP32_CORES) && (c.R == 64 || c.R == 128) && c.NC <= 4 * c.R &&
+  return !(c.flags & TTEMB_FP32_CORES) && (c.R == 32 || c.R == 64 || c.R == 128) &&
+         c.NC <= (c.R == 128 ? 512 : 256) &&
          (c.n3 == 4 || c.n3 == 8) && (c.n1 == 1 || c.n1 == 2 || c.n1 == 4 || c.n1 == 8) && c.n1 * c.n2 <= 16;
 }
 bool tc_eligible(const Ctx& c) { return fused_eligible(c); }
@@ -714,14 +712,19 @@ cudaError_t configure_fused(Ctx& c) {
   auto set = [&](const void* f, size_t bytes) {
     if (e == cudaSuccess) e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
   };
+  set((const void*)k_prefix_fwd<32>, prefix_smem<32>());
   set((const void*)k_prefix_fwd<64>, prefix_smem<64>());
   set((const void*)k_prefix_fwd<128>, prefix_smem<128>());
   set((const void*)k_rows_fwd2<4, 8>, rows_smem(4, 64));
   set((const void*)k_rows_fwd2<8, 8>, rows_smem(8, 64));
+  set((const void*)k_rows_fwd2<4, 4>, rows_smem(4, 32));
+  set((const void*)k_rows_fwd2<8, 4>, rows_smem(8, 32));
   set((const void*)k_rows_fwd2<4, 16>, rows_smem(4, 128));
   set((const void*)k_rows_fwd2<8, 16>, rows_smem(8, 128));
-  set((const void*)k_rows_bwd2<4>, rows_bwd_smem(4));
-  set((const void*)k_rows_bwd2<8>, rows_bwd_smem(8));
+  set((const void*)k_rows_bwd2<4, 4>, rows_bwd_smem(4, 32));
+  set((const void*)k_rows_bwd2<8, 4>, rows_bwd_smem(8, 32));
+  set((const void*)k_rows_bwd2<4, 8>, rows_bwd_smem(4, 64));
+  set((const void*)k_rows_bwd2<8, 8>, rows_bwd_smem(8, 64));
   return e;
 }
 
@@ -746,7 +749,8 @@ cudaError_t run_fused_fwd(Ctx& c, float* out, cudaStream_t s) {
       cudaMemsetAsync(trace, 0, sizeof(unsigned long long) * 32 * grid, s);
       a.trace = trace;
     }
-    if (c.R == 64) k_prefix_fwd<64><<<grid, X_THREADS, prefix_smem<64>(), s>>>(a);
+    if (c.R == 32) k_prefix_fwd<32><<<grid, X_THREADS, prefix_smem<32>(), s>>>(a);
+    else if (c.R == 64) k_prefix_fwd<64><<<grid, X_THREADS, prefix_smem<64>(), s>>>(a);
     else k_prefix_fwd<128><<<grid, X_THREADS, prefix_smem<128>(), s>>>(a);
     if (a.trace) {
       std::vector<unsigned long long> hb(32 * grid);
@@ -777,7 +781,10 @@ cudaError_t run_fused_fwd(Ctx& c, float* out, cudaStream_t s) {
     r.pfx_t = p.pfx_t; r.pbuf = p.pbuf; r.rows = p.rows; r.seg_off = p.seg_off; r.sbag = p.sbag; r.out = out;
     r.n1 = c.n1; r.n1s = a.n1s; r.n2 = c.n2; r.N = c.N; r.NC = c.NC;
     const int grid = grid_for(c, cdiv(c.U_cap, RW_RCH), RW_WARPS, 4);
-    if (c.R == 64) {
+    if (c.R == 32) {
+      if (c.n3 == 4) k_rows_fwd2<4, 4><<<grid, RW_WARPS * 32, rows_smem(4, 32), s>>>(r);
+      else k_rows_fwd2<8, 4><<<grid, RW_WARPS * 32, rows_smem(8, 32), s>>>(r);
+    } else if (c.R == 64) {
       if (c.n3 == 4) k_rows_fwd2<4, 8><<<grid, RW_WARPS * 32, rows_smem(4, 64), s>>>(r);
       else k_rows_fwd2<8, 8><<<grid, RW_WARPS * 32, rows_smem(8, 64), s>>>(r);
     } else {
@@ -808,9 +815,14 @@ cudaError_t run_rows_bwd2(Ctx& c, cudaStream_t s) {
   r.row_i3 = p.row_i3; r.pfx_t = p.pfx_t; r.row_seg = p.row_seg; r.pbuf = p.pbuf; r.gbuf = p.gbuf;
   r.dpbuf = p.dpbuf; r.n1 = c.n1; r.n2 = c.n2; r.N = c.N; r.NC = c.NC; r.R = c.R;
   // (the dP rows of chunk-straddling prefixes were zeroed at the end of the index stage)
-  const int grid = grid_for(c, cdiv(c.U_cap, RW_RCH) * (c.R / XR), RW_WARPS, 2);
-  if (c.n3 == 4) k_rows_bwd2<4><<<grid, RW_WARPS * 32, rows_bwd_smem(4), s>>>(r);
-  else k_rows_bwd2<8><<<grid, RW_WARPS * 32, rows_bwd_smem(8), s>>>(r);
+  const int grid = grid_for(c, cdiv(c.U_cap, RW_RCH) * std::max(1, c.R / XR), RW_WARPS, 2);
+  if (c.R == 32) {
+    if (c.n3 == 4) k_rows_bwd2<4, 4><<<grid, RW_WARPS * 32, rows_bwd_smem(4, 32), s>>>(r);
+    else k_rows_bwd2<8, 4><<<grid, RW_WARPS * 32, rows_bwd_smem(8, 32), s>>>(r);
+  } else {
+    if (c.n3 == 4) k_rows_bwd2<4, 8><<<grid, RW_WARPS * 32, rows_bwd_smem(4, 64), s>>>(r);
+    else k_rows_bwd2<8, 8><<<grid, RW_WARPS * 32, rows_bwd_smem(8, 64), s>>>(r);
+  }
   return cudaGetLastError();
 }
 

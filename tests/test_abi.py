@@ -58,7 +58,7 @@ def _cfg(**kw):
 
 
 def test_query_sizes_consistent():
-    cfg, keep = _cfg(fp32_cores=True)     # (the tensor-core path stores R = 16 zero-padded to 64)
+    cfg, keep = _cfg(fp32_cores=True)     # (the tensor-core path stores R = 16 zero-padded to 32)
     core, state, grad, ws = tt.ttemb_query_sizes(cfg)
     c = W.config("c2")
     assert core == grad and state == 0 and ws > 0

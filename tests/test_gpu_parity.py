@@ -714,11 +714,12 @@ def test_ffma_split_groups_fused_and_unfused(opt, rank):
                                     what=f"{opt} step 2 C{k+1}")
 
 
-def test_rank_padding_storage_is_exact():
-    """32 <= R < 64 runs on the tcgen05 path with cores stored zero-padded to rank 64
-    (ttemb_config.rank doc, R28): the padding stays exactly zero through fused SGD and
-    Adagrad steps, and the results match the oracle at the configured rank."""
-    cfg = W.small_config([20000, 300], [(28, 28, 26), (7, 7, 7)], (4, 4, 4), 40, 96, 2, 1.05)
+@pytest.mark.parametrize("rank,storage", [(40, 64), (20, 32)])
+def test_rank_padding_storage_is_exact(rank, storage):
+    """16 <= R < 32 and 32 < R < 64 run on the tcgen05 path with cores stored zero-padded to rank
+    32 / 64 (ttemb_config.rank doc, R28): the padding stays exactly zero through fused
+    SGD and Adagrad steps, and the results match the oracle at the configured rank."""
+    cfg = W.small_config([20000, 300], [(28, 28, 26), (7, 7, 7)], (4, 4, 4), rank, 96, 2, 1.05)
     idx, off = W.make_batch(cfg, seed=29)
     B = cfg.batch
     cores = W.make_cores(cfg, seed=29)
@@ -726,7 +727,7 @@ def test_rank_padding_storage_is_exact():
     orc = Oracle.from_config(cfg)
     for opt in ("sgd", "adagrad"):
         emb = gpu_emb(cfg, B, len(idx), optimizer=opt, fused_update=True)
-        assert emb.layout[0][1][1][1] == 64              # storage rank of C2
+        assert emb.layout[0][1][1][1] == storage         # storage rank of C2
         emb.load_cores(cores)
         out = run_forward(emb, idx, off, B)
         assert_companion(out.cpu().numpy(), orc.forward(cores, idx, off, B),
