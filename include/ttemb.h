@@ -177,6 +177,68 @@ int ttemb_update_range(ttemb_t h, float lr, int64_t begin, int64_t count, void* 
  * ttemb_set_bijection applies at run time. */
 int ttemb_louvain(int64_t n, int64_t m, const int64_t* u, const int64_t* v, const double* w, int64_t* labels);
 
+/* ---- Host-memory tier (PAPER §V) ----------------------------------
+ * Tables too large for HBM stay in host memory (float32 [n_rows][dim], caller-owned); a CPU
+ * parameter server pre-fetches the rows of the next batches and applies the gradients
+ * the GPU worker pushes back; the GPU embedding cache below keeps rows that recent batches
+ * updated, so a batch pre-fetched before those updates reached host memory is synchronised
+ * (the read-after-write conflict).  A batch's host rows travel as a block
+ * rows[U][dim] with ids[U] = the distinct global host-row numbers (unique within the batch).
+ *
+ * ttemb_ht_cache: caller-allocated device buffers (the "index table" and the cached rows):
+ *   index[n_rows]        int32, cache slot of a host row or -1
+ *   rows[capacity][dim]  float32 cached rows;  lc[capacity] int32 life cycles (0 = free slot)
+ *   owner[capacity]      int64 host row of a slot;  free_list[capacity] int32;  top[2] int32
+ *                        (free-list size, overflow flag).
+ * Capacity: at most `life` batches' rows are live, so life * max(U) slots always suffice; an
+ * insert that finds no free slot sets the overflow flag (ttemb_ht_cache_stats) and that row is
+ * not cached (later reads of it may then be stale).
+ * All device calls are asynchronous on `stream` (cudaStream_t, NULL = legacy default) and return
+ * TTEMB_ERR_INVALID_ARG (null pointers, negative sizes) before enqueuing anything. */
+typedef struct {
+  int32_t* index;
+  float* rows;
+  int32_t* lc;
+  int64_t* owner;
+  int32_t* free_list;
+  int32_t* top;
+  int64_t n_rows;
+  int32_t capacity;
+  int32_t dim;
+} ttemb_ht_cache;
+
+/* Empty cache: index = -1, every slot free. */
+int ttemb_ht_cache_init(const ttemb_ht_cache* c, void* stream);
+/* Step 1 of P:290 / P:298: rows[u] = the cached row of ids[u] where one exists (device ids[n],
+ * rows[n][dim]); other rows keep the pre-fetched values. */
+int ttemb_ht_sync(const ttemb_ht_cache* c, const int64_t* ids, int64_t n, float* rows, void* stream);
+/* Sum pooling over the block: bag (t,b) = positions offsets[t*batch+b] .. offsets[t*batch+b+1]
+ * (int64, table-major like ttemb_forward), ridx[j] = block row of position j (int32);
+ * out[b][t][:] = sum of rows[ridx[j]] in position order (float32, written in full). */
+int ttemb_ht_pool(const float* rows, const int32_t* ridx, const int64_t* offsets, int32_t num_tables,
+                  int32_t batch, int32_t dim, float* out, void* stream);
+/* Row gradients of L = sum(out * grad_out): g[u] = sum over k in [occ_ptr[u], occ_ptr[u+1]) of
+ * grad_out[b][t] with bag occ_bag[k] = t*batch + b (the positions of row u, in position order). */
+int ttemb_ht_grad(const float* grad_out, const int64_t* occ_ptr, const int32_t* occ_bag, int64_t n,
+                  int32_t num_tables, int32_t batch, int32_t dim, float* g, void* stream);
+/* One pull from the gradient queue: every live entry's LC decreases by 1; an entry that
+ * reaches 0 is evicted (index entry -1, slot freed). */
+int ttemb_ht_tick(const ttemb_ht_cache* c, void* stream);
+/* SGD on the block, rows[u] = rows[u] - rn(lr * g[u]) (two roundings, the server's arithmetic),
+ * then, for life > 0, insert / refresh each row in the cache with LC = life ("the
+ * maximum length of the Requests Queue").  life = 0 updates without caching. */
+int ttemb_ht_update_push(const ttemb_ht_cache* c, float* rows, const float* g, const int64_t* ids, int64_t n,
+                         float lr, int32_t life, void* stream);
+/* Live entries and the overflow flag (synchronises `stream`). */
+int ttemb_ht_cache_stats(const ttemb_ht_cache* c, int32_t* live, int32_t* overflow, void* stream);
+/* Parameter-server side, host memory, `nthreads` worker threads (<= 0: up to 16):
+ * gather out[u] = table[ids[u]] (the pre-fetch) and apply table[ids[u]] -= rn(lr * g[u]).
+ * TTEMB_ERR_INDEX_RANGE (nothing written) for an id outside [0, n_rows); ids must be distinct. */
+int ttemb_ht_host_gather(const float* table, int64_t n_rows, int32_t dim, const int64_t* ids, int64_t n,
+                         float* out, int32_t nthreads);
+int ttemb_ht_host_sgd(float* table, int64_t n_rows, int32_t dim, const int64_t* ids, int64_t n, const float* g,
+                      float lr, int32_t nthreads);
+
 /* Host-buffer variants (end-to-end path): copy the inputs from host memory
  * into the workspace staging area, run the step, and copy `out` back to the
  * host, all on `stream`.  Pinned host memory keeps the copies asynchronous. */

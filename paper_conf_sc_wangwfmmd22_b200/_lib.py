@@ -32,7 +32,15 @@ SYMBOLS = ["ttemb_query_sizes", "ttemb_create", "ttemb_destroy", "ttemb_core_lay
            "ttemb_backward_host", "ttemb_check", "ttemb_get_plan", "ttemb_read_counts",
            "ttemb_set_timing", "ttemb_stage_times", "ttemb_stage_name", "ttemb_status_string",
            "ttemb_set_bijection", "ttemb_total_rows", "ttemb_forward_weighted", "ttemb_plan_batch",
-           "ttemb_forward_planned", "ttemb_update_range", "ttemb_grad_buckets", "ttemb_set_bucket_events", "ttemb_louvain"]
+           "ttemb_forward_planned", "ttemb_update_range", "ttemb_grad_buckets", "ttemb_set_bucket_events", "ttemb_louvain",
+           "ttemb_ht_cache_init", "ttemb_ht_sync", "ttemb_ht_pool", "ttemb_ht_grad", "ttemb_ht_tick",
+           "ttemb_ht_update_push", "ttemb_ht_cache_stats", "ttemb_ht_host_gather", "ttemb_ht_host_sgd"]
+
+
+class ttemb_ht_cache(C.Structure):
+    _fields_ = [("index", C.c_void_p), ("rows", C.c_void_p), ("lc", C.c_void_p), ("owner", C.c_void_p),
+                ("free_list", C.c_void_p), ("top", C.c_void_p), ("n_rows", C.c_int64),
+                ("capacity", C.c_int32), ("dim", C.c_int32)]
 
 
 class ttemb_table(C.Structure):
@@ -105,6 +113,16 @@ def load(path: str = LIB_PATH):
     lib.ttemb_grad_buckets.argtypes = [vp, C.POINTER(i64), C.POINTER(i64), C.c_int]
     lib.ttemb_set_bucket_events.argtypes = [vp, C.POINTER(vp), C.c_int]
     lib.ttemb_louvain.argtypes = [i64, i64, C.POINTER(i64), C.POINTER(i64), C.POINTER(C.c_double), C.POINTER(i64)]
+    hc = C.POINTER(ttemb_ht_cache)
+    lib.ttemb_ht_cache_init.argtypes = [hc, vp]
+    lib.ttemb_ht_sync.argtypes = [hc, vp, i64, vp, vp]
+    lib.ttemb_ht_pool.argtypes = [vp, vp, vp, i32, i32, i32, vp, vp]
+    lib.ttemb_ht_grad.argtypes = [vp, vp, vp, i64, i32, i32, i32, vp, vp]
+    lib.ttemb_ht_tick.argtypes = [hc, vp]
+    lib.ttemb_ht_update_push.argtypes = [hc, vp, vp, vp, i64, f32, i32, vp]
+    lib.ttemb_ht_cache_stats.argtypes = [hc, C.POINTER(i32), C.POINTER(i32), vp]
+    lib.ttemb_ht_host_gather.argtypes = [vp, i64, i32, vp, i64, vp, i32]
+    lib.ttemb_ht_host_sgd.argtypes = [vp, i64, i32, vp, i64, vp, f32, i32]
     for s in SYMBOLS:
         f = getattr(lib, s)
         if s not in ("ttemb_stage_name", "ttemb_status_string", "ttemb_total_rows"):

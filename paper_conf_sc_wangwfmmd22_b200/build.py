@@ -31,7 +31,7 @@ def _stale() -> bool:
 def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not _stale():
         return LIB
-    cmd = [NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2", "-shared",
+    cmd = [NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2,-ffp-contract=off", "-shared",
            "--expt-relaxed-constexpr", "-I", os.path.join(ROOT, "include"),
            *os.environ.get("TTEMB_NVCC_FLAGS", "").split(), "-o", LIB + ".tmp", *sources()]
     if verbose:

@@ -325,3 +325,27 @@ def small_config(table_rows: Sequence[int], row_factors: Sequence[Tuple[int, int
     """Ad-hoc config for tests (explicit factors)."""
     return _mk(name, table_rows, col_factors, rank, batch, pooling, zipf_s,
                factors=row_factors, id_map=id_map)
+
+
+def make_host_batch(table_rows: Sequence[int], batch: int, pooling: int, zipf_s: Optional[float],
+                    step: int = 0, seed: int = 0, name: str = "host") -> Tuple[np.ndarray, np.ndarray]:
+    """Ids of the host-memory tables of the pipeline (f4; P:417 keeps all but the largest table
+    in host memory): (indices int64, offsets int64 [T*B+1]), table-major, fixed bag length,
+    Zipf ids so consecutive batches share hot rows (the RAW hazard of P:296)."""
+    T = len(table_rows)
+    offsets = np.arange(T * batch + 1, dtype=np.int64) * pooling
+    parts = [zipf_ids(rng("host_ids", name, seed, step, t), int(table_rows[t]), zipf_s, batch * pooling)
+             for t in range(T)]
+    return (np.concatenate(parts) if parts else np.zeros(0, dtype=np.int64)), offsets
+
+
+def make_host_weight(table_rows: Sequence[int], dim: int, seed: int = 0) -> np.ndarray:
+    """Initial host-table parameters, float32 [sum rows][dim], U(-0.05, 0.05)."""
+    return rng("host_w", seed, dim, *[int(r) for r in table_rows]).uniform(
+        -0.05, 0.05, size=(int(sum(table_rows)), dim)).astype(np.float32)
+
+
+def make_host_grad_out(num_tables: int, batch: int, dim: int, step: int = 0, seed: int = 0) -> np.ndarray:
+    """Upstream gradient of the host-table outputs, float32 [B][T][dim], U(-1, 1)."""
+    return rng("host_go", seed, step, batch, num_tables, dim).uniform(
+        -1.0, 1.0, size=(batch, num_tables, dim)).astype(np.float32)
