@@ -89,6 +89,23 @@ __device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t
                : "memory");
 }
 
+// 2-D tiled TMA load (tensor map in kernel-parameter / constant space) into shared memory,
+// completing the box's bytes as transactions on mbar.  c0 = inner (contiguous) coordinate.
+__device__ __forceinline__ void tma_load_2d(uint32_t dst, const void* tmap, int c0, int c1, uint64_t* mbar) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];"
+      ::"r"(dst), "l"(tmap), "r"(c0), "r"(c1), "r"(smem_u32(mbar))
+      : "memory");
+}
+
+// Byte offset of fp32 element (row, c) in a tile a 2-D TMA load with CU_TENSOR_MAP_SWIZZLE_128B
+// wrote as boxes of 32 columns x `rows` rows, box b = c / 32 at b * rows * 128: the 16-byte chunk
+// (c % 32) / 4 of each 128-byte row is stored at chunk ^ (row % 8) (the K-major SWIZZLE_128B
+// operand layout: SBO = 1024, K-step(8) = +32 bytes inside a box).  Needs 1024-byte alignment.
+__device__ __forceinline__ uint32_t sw128_off(int row, int c, int rows) {
+  return (uint32_t)((c >> 5) * rows * 128 + row * 128 + ((((c & 31) >> 2) ^ (row & 7)) << 4) + (c & 3) * 4);
+}
+
 // 1-D bulk prefetch of [src, src + bytes) into L2 (TMA engine, no shared memory, no completion).
 // src and bytes must be multiples of 16.
 __device__ __forceinline__ void bulk_prefetch_l2(const void* src, uint32_t bytes) {

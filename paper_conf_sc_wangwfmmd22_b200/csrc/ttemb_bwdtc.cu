@@ -11,7 +11,8 @@
 //   dA[m][r1] = sum_c dP[m][c] . C2[i2][r1][c]                  (the C1 gradient partials)
 //       M = 128 = the tile's dP rows stacked as [dP_hi; dP_lo] IN TENSOR MEMORY (lanes 0-63 hi,
 //       64-127 lo, column = c of the current 64-c chunk), N = 64 r1, K = c; B = the C2 chunk
-//       (hi, lo) in shared memory; two MMAs per K step accumulate dP_hi C2_hi + dP_hi C2_lo in
+//       (hi, lo) in shared memory as a K-major SWIZZLE_128B operand; two MMAs per K step
+//       accumulate dP_hi C2_hi + dP_hi C2_lo in
 //       lanes m and dP_lo C2_hi + dP_lo C2_lo in lanes 64 + m (3xTF32 plus the lo.lo term); the
 //       epilogue sums the two lane halves.  With A in TMEM the tensor core reads only the 2 KB
 //       B operand from shared memory per MMA (SS mode read 6 KB and shared the bandwidth with
@@ -25,9 +26,10 @@
 // fp32 accuracy: 3xTF32 (hi = raw fp32, read by the tensor core with truncation; lo =
 // x - trunc_tf32(x)); scripts/tc_probe3.cu measures the TMEM-A form.
 //
-// Warp roles (416 threads): 0-7 loaders (cp.async chunk staging, C2 lo split, dP and dP^T ->
-// TMEM with the lo parts computed in registers),
-// 8 MMA issuer, 9-12 epilogue (dA -> dC1 reductions, dC2 -> gradient / fused update).
+// Warp roles (448 threads): 0-7 loaders (C2 lo split, dP and dP^T -> TMEM with the lo parts
+// computed in registers), 8 MMA issuer, 9-12 epilogue (dA -> dC1 reductions, dC2 -> gradient /
+// fused update), 13 TMA producer (per K-chunk: 2-D TMA loads of the tile's dP rows and the C2
+// slice rows, SWIZZLE_128B, up to Y_NST chunks ahead).
 #include <stdio.h>
 #include <stdlib.h>
 
@@ -43,9 +45,10 @@ namespace {
 
 constexpr int YT = 64;                          // tile rows (prefix, j1)
 constexpr int Y_LW = 8, Y_EW = 4;
-constexpr int Y_THREADS = (Y_LW + 1 + Y_EW) * 32;
+constexpr int Y_THREADS = (Y_LW + 1 + Y_EW + 1) * 32;
 constexpr int Y_MMA_W = Y_LW;
-constexpr int Y_NST = 3;                        // chunk stages (cp.async, two in flight)
+constexpr int Y_TMA_W = Y_LW + 1 + Y_EW;           // the TMA producer warp
+constexpr int Y_NST = 3;                        // chunk stages (TMA)
 constexpr int Y_GI = 64;                        // work units per CTA whose metadata is staged in shared memory
 
 // Shape of the kernel for rank KR: a work unit is (i2-group, BPU c-blocks of 128); K-chunks of
@@ -55,10 +58,10 @@ constexpr int Y_GI = 64;                        // work units per CTA whose meta
 template <int KR> struct YShape {
   static constexpr int BPU = KR <= 64 ? 2 : 1;
   static constexpr int CK = KR <= 64 ? 64 : 32;
-  static constexpr int A2S = CK + 4;                                    // dP staging row stride (floats)
-  static constexpr uint32_t A2 = YT * A2S * 4;                          // dP chunk staging
-  static constexpr uint32_t B2LBO = (KR / 8) * 128;                     // CM(KR r1, CK c) core-column stride
-  static constexpr uint32_t B2 = 2u * (CK / 4) * B2LBO;                 // C2 chunk hi + lo
+  // stage = [dP chunk | C2 chunk hi | C2 chunk lo], each as TMA SWIZZLE_128B boxes of 32 columns
+  // (tc::sw128_off): dP rows m = 64 per box, C2 rows r1 = KR per box (the K-major B operand)
+  static constexpr uint32_t A2 = YT * CK * 4;                           // dP chunk
+  static constexpr uint32_t B2 = 2u * KR * CK * 4;                      // C2 chunk hi + lo
   static constexpr uint32_t STAGE = A2 + B2;
   static constexpr uint32_t B1 = 2u * KR * YT * 4;                      // C1^T hi + lo (MN-major)
   static constexpr size_t SMEM = 1024 + B1 + Y_NST * STAGE;
@@ -78,6 +81,7 @@ struct YArgs {
   const uint32_t *counts, *grp_off, *grp_t, *pfx_i1, *pfx_t;
   const uint32_t* grp_arow;               // [P]  C1 row index (floats / R) of prefix q, j1 = 0
   const unsigned long long* grp_c2;       // [NG] float offset of the group's C2 slice
+  unsigned long long c2_begin;            // float offset of the C2 region (tm_c2 row 0)
   const float* dpbuf;                     // [P][n1][NC]
   uint32_t* work;
   int n1, n1s, NC, nblk, tpp, nchunk, R;
@@ -90,7 +94,8 @@ struct YArgs {
 
 struct YCtl {
   uint64_t a1_full, a1_free;              // dP^T in TMEM + C1^T in smem (per tile)
-  uint64_t s_full[Y_NST], s_free[Y_NST];  // K-chunk stages
+  uint64_t s_full[Y_NST], s_free[Y_NST];  // K-chunk stages (loaders done / MMAs done)
+  uint64_t s_tma[Y_NST];                  // K-chunk stage landed (TMA transactions)
   uint64_t d1_full, d1_free;              // dC2 accumulator (per group)
   uint64_t d2_full, d2_free;              // dA accumulator (per tile)
   uint64_t p_free;                        // dP chunk A operand in TMEM (per chunk)
@@ -108,9 +113,10 @@ struct YCtl {
 __device__ __forceinline__ float lo32(float x) { return x - tc::tf32_trunc(x); }
 
 template <int KR>
-__global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
+__global__ void __launch_bounds__(Y_THREADS, 1)
+k_prefix_bwd(const __grid_constant__ CUtensorMap tm_dp, const __grid_constant__ CUtensorMap tm_c2, YArgs a) {
   using S = YShape<KR>;
-  constexpr int BPU = S::BPU, CK = S::CK, A2S = S::A2S;
+  constexpr int BPU = S::BPU, CK = S::CK;
   extern __shared__ __align__(128) char smem_raw[];
   __shared__ YCtl ctl;
   char* const smem = smem_raw + ((1024u - (tc::smem_u32(smem_raw) & 1023u)) & 1023u);
@@ -123,7 +129,9 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
   if (tid == 0) {
     tc::mbar_init(&ctl.a1_full, Y_LW * 32);
     tc::mbar_init(&ctl.a1_free, 1);
-    for (int s = 0; s < Y_NST; ++s) { tc::mbar_init(&ctl.s_full[s], Y_LW * 32); tc::mbar_init(&ctl.s_free[s], 1); }
+    for (int s = 0; s < Y_NST; ++s) {
+      tc::mbar_init(&ctl.s_full[s], Y_LW * 32); tc::mbar_init(&ctl.s_free[s], 1); tc::mbar_init(&ctl.s_tma[s], 1);
+    }
     tc::mbar_init(&ctl.d1_full, 1);
     tc::mbar_init(&ctl.d1_free, Y_EW * 32);
     tc::mbar_init(&ctl.d2_full, 1);
@@ -159,57 +167,36 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
   // r1) and the current chunk's [dP_hi; dP_lo] (dA A operand, column = c of the chunk).
   const int tpp = a.tpp, NC = a.NC;
 
+  // Jobs = (unit, tile, K-chunk) in a static round-robin unit order (loaders, TMA producer)
+  struct Job { uint32_t u, q0, q1, qa; int ck, crow; unsigned long long c2; };
+  const uint32_t G0 = blockIdx.x, GS = gridDim.x;
+  auto start = [&](Job& j, uint32_t u) {   // unit metadata (staged in shared memory)
+    j.u = u; j.ck = 0;
+    if (u < NU) {
+      const uint32_t k = (u - G0) / GS, g = u / UPG;
+      if (k < (uint32_t)Y_GI) { j.q0 = j.qa = ctl.gq0[k]; j.q1 = ctl.gq1[k]; j.c2 = ctl.gc2[k]; }
+      else { j.q0 = j.qa = a.grp_off[g]; j.q1 = a.grp_off[g + 1]; j.c2 = a.grp_c2[g]; }
+      j.crow = (int)((j.c2 - a.c2_begin) / (unsigned long long)NC);   // C2 region row of r1 = 0
+    }
+  };
+  auto advance = [&](Job& j) {
+    if (++j.ck < a.nchunk) return;
+    j.ck = 0;
+    j.qa += tpp;
+    if (j.qa >= j.q1) start(j, j.u + GS);
+  };
   if (w < Y_LW) {
     // ------------------------------- loaders -------------------------------
-    // Jobs = (unit, tile, K-chunk) in a static round-robin unit order, so the issue side can run
-    // two chunks ahead across tile and unit boundaries.  A chunk's dP rows are copied with
-    // cp.async into a row-major staging buffer, its C2 rows straight into the B operand's
-    // core-matrix layout (hi); each thread writes the lo parts of the C2 pieces it copied, and
-    // dP (lanes m) and dP^T (lanes c) go to tensor memory with their lo parts made in registers.
-    struct Job { uint32_t u, q0, q1, qa; int ck; unsigned long long c2; };
-    const uint32_t G0 = blockIdx.x, GS = gridDim.x;
-    auto start = [&](Job& j, uint32_t u) {   // unit metadata (staged in shared memory)
-      j.u = u; j.ck = 0;
-      if (u < NU) {
-        const uint32_t k = (u - G0) / GS, g = u / UPG;
-        if (k < (uint32_t)Y_GI) { j.q0 = j.qa = ctl.gq0[k]; j.q1 = ctl.gq1[k]; j.c2 = ctl.gc2[k]; }
-        else { j.q0 = j.qa = a.grp_off[g]; j.q1 = a.grp_off[g + 1]; j.c2 = a.grp_c2[g]; }
-      }
-    };
-    auto advance = [&](Job& j) {
-      if (++j.ck < a.nchunk) return;
-      j.ck = 0;
-      j.qa += tpp;
-      if (j.qa >= j.q1) start(j, j.u + GS);
-    };
+    // Per K-chunk the TMA producer has landed the tile's 64 dP rows (rows past the tile belong to
+    // the next group or lie past the stash; they are masked to zero here) and the KR rows of the
+    // C2 slice in the B operand's K-major SWIZZLE_128B layout (hi); each thread writes the lo parts
+    // of its share of the C2 chunk, and dP (lanes m) and dP^T (lanes c) go to tensor memory with
+    // their lo parts made in registers.
     const int mb = tid & 63;                  // C1^T staging map: row mb, float4 columns (tid >> 6) + 4 k
-    // dP chunk copy map: rows (tid / (CK/4)) + (256 / (CK/4)) k, float4 column cc4: every row
-    // segment is read by consecutive threads (coalesced)
-    constexpr int F4 = CK / 4, RPP = 256 / F4;
-    const int cr = tid / F4, cc4 = 4 * (tid % F4);
-    auto a2_off = [&](int r) { return (uint32_t)((r * A2S + cc4) * 4); };
-    // C2 chunk map: row (r1) tid % KR, float4 columns (tid / KR) + (256 / KR) k
-    constexpr int C2F = KR * CK / 4 / 256;    // float4 per thread
-    const int br = tid % KR, bc = tid / KR;
-    auto b2_off = [&](int k) { return tc::cm_off(br, 4 * (bc + (256 / KR) * k), KR / 8); };
-    auto issue = [&](const Job& j, uint32_t sidx) {
-      const uint32_t rows = min((uint32_t)tpp, j.q1 - j.qa) << a.n1s;
-      const int c0 = (int)(j.u % UPG) * BPU * 128 + j.ck * CK;   // first slice column of the chunk
-      const float* dps = a.dpbuf + (size_t)j.qa * a.n1 * NC + c0 + cc4;
-      const float* c2 = a.cores + j.c2 + c0 + (size_t)br * NC;
-      const uint32_t a2 = tc::smem_u32(stg + (sidx % Y_NST) * S::STAGE), b2 = a2 + S::A2;
-#pragma unroll
-      for (int k = 0; k < YT / RPP; ++k) {
-        const int r = cr + RPP * k;
-        tc::cp_async16_z(a2 + a2_off(r), dps + (size_t)(r < (int)rows ? r : 0) * NC, r < (int)rows);
-      }
-#pragma unroll
-      for (int k = 0; k < C2F; ++k) tc::cp_async16(b2 + b2_off(k), c2 + 4 * (bc + (256 / KR) * k));
-    };
-    uint32_t ui = 0, si = 0, sp = 0;          // tile counter, issued / processed chunk counters
-    Job P, I;
+    constexpr int C2F = KR * CK / 4 / 256;    // float4 of the C2 chunk per thread (lo split)
+    uint32_t ui = 0, sp = 0;                  // tile counter, processed chunk counter
+    Job P;
     start(P, G0);
-    I = P;
     // C1 rows of a tile (row mb of the tile, float4 columns (tid >> 6) + 4 k), loaded one tile
     // ahead (NT = the next tile of the processing job) so their latency overlaps a whole tile.
     constexpr int C1F = KR / 16;
@@ -223,18 +210,10 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
       for (int k = 0; k < C1F; ++k) cv[k] = ok ? __ldg(src + (tid >> 6) + 4 * k) : make_float4(0.f, 0.f, 0.f, 0.f);
     };
     load_c1(P, cvn);
-    for (int d = 0; d < Y_NST - 1; ++d) {
-      if (I.u < NU) {
-        tc::mbar_wait(&ctl.s_free[si % Y_NST], ((si / Y_NST) & 1) ^ 1);
-        issue(I, si);
-        advance(I);
-        ++si;
-      }
-      tc::cp_commit();
-    }
     while (P.u < NU) {
       YT0();
       const uint32_t np = min((uint32_t)tpp, P.q1 - P.qa);
+      const int rows = (int)(np << a.n1s);              // valid dP rows of the tile
       if (P.ck == 0) {
         const uint32_t fl = (P.qa == P.q0 ? 1u : 0u) | (P.qa + tpp >= P.q1 ? 2u : 0u);
         if (tid == 0) {
@@ -268,27 +247,26 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
           *reinterpret_cast<float4*>(b1 + S::B1 / 2 + off) = make_float4(lo32(v.x), lo32(v.y), lo32(v.z), lo32(v.w));
         }
       }
-      // chunk P landed (one newer chunk may still be in flight)
+      // chunk P landed
       YTA(2);
-      tc::cp_wait<Y_NST - 2>();
-      YTA(3);
       const uint32_t sidx = sp % Y_NST;
+      tc::mbar_wait(&ctl.s_tma[sidx], (sp / Y_NST) & 1);
+      YTA(3);
       char* a2 = stg + sidx * S::STAGE;
       char* b2h = a2 + S::A2;
       char* b2l = b2h + S::B2 / 2;
-      if (!(a.exp & 4)) {   // the C2 chunk's lo part (the dP lo parts are made in registers below)
+      if (!(a.exp & 4)) {   // the C2 chunk's lo part (elementwise: same swizzled positions)
         float4 q[C2F];
 #pragma unroll
-        for (int k = 0; k < C2F; ++k) q[k] = *reinterpret_cast<const float4*>(b2h + b2_off(k));
+        for (int k = 0; k < C2F; ++k) q[k] = reinterpret_cast<const float4*>(b2h)[tid + 256 * k];
 #pragma unroll
         for (int k = 0; k < C2F; ++k)
-          *reinterpret_cast<float4*>(b2l + b2_off(k)) =
+          reinterpret_cast<float4*>(b2l)[tid + 256 * k] =
               make_float4(lo32(q[k].x), lo32(q[k].y), lo32(q[k].z), lo32(q[k].w));
       }
       YTA(4);
       tc::named_sync(1, Y_LW * 32);                     // whole chunk (hi and lo) visible
       YTA(5);
-      const float* a2f = reinterpret_cast<const float*>(a2);
       {   // dP^T of this chunk -> TMEM (dC2 A operand): thread = column, 32 tile rows; lo in
           // registers.  R = 64: chunk ck covers c-block ck / 2, lane quarters 2 (ck & 1) + {0, 1};
           // R = 128: the unit's block, lane quarter ck & 3.
@@ -300,7 +278,10 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
           const int m0 = 32 * (w >> 2);                           // warps 0-3: rows 0..31, 4-7: 32..63
           float x[32];
 #pragma unroll
-          for (int i = 0; i < 32; ++i) x[i] = a2f[(m0 + i) * A2S + cc];
+          for (int i = 0; i < 32; ++i) {
+            const float v = *reinterpret_cast<const float*>(a2 + tc::sw128_off(m0 + i, cc, YT));
+            x[i] = m0 + i < rows ? v : 0.f;
+          }
           tc::tmem_st32(tc::taddr(tm + S::T_DPT + blk * 64 + m0, 32 * Q, 0), x);
 #pragma unroll
           for (int i = 0; i < 32; ++i) x[i] = lo32(x[i]);
@@ -317,9 +298,11 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
         const int Q = w & 3, h = w >> 2, m = 32 * (Q & 1) + lane;
         if (!(a.exp & 8) && 32 * h < CK) {
           float x[32];
+          const bool ok = m < rows;
 #pragma unroll
           for (int k = 0; k < 8; ++k) {
-            const float4 v = *reinterpret_cast<const float4*>(a2f + m * A2S + 32 * h + 4 * k);
+            float4 v = *reinterpret_cast<const float4*>(a2 + tc::sw128_off(m, 32 * h + 4 * k, YT));
+            if (!ok) v = make_float4(0.f, 0.f, 0.f, 0.f);
             x[4 * k] = v.x; x[4 * k + 1] = v.y; x[4 * k + 2] = v.z; x[4 * k + 3] = v.w;
           }
           if (Q >= 2) {
@@ -339,19 +322,7 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
       }
       ++sp;
       advance(P);
-      // refill: the chunk two ahead
-      if (I.u < NU) {
-        YTA(7);
-        tc::mbar_wait(&ctl.s_free[si % Y_NST], ((si / Y_NST) & 1) ^ 1);
-        YTA(8);
-        issue(I, si);
-        YTA(9);
-        advance(I);
-        ++si;
-      }
-      tc::cp_commit();
     }
-    tc::cp_wait<0>();
     if (tid == 0) {
       tc::mbar_wait(&ctl.u_empty[ui & 3], ((ui >> 2) & 1) ^ 1);
       ctl.ring[ui & 3][3] = 4u;
@@ -383,8 +354,10 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
           const uint32_t b2h = tc::smem_u32(stg + s * S::STAGE) + S::A2, b2l = b2h + S::B2 / 2;
 #pragma unroll
           for (int kk = 0; kk < CK / 8; ++kk) {
-            const uint64_t dbh = tc::sdesc(b2h + kk * 2 * S::B2LBO, S::B2LBO, 128);
-            const uint64_t dbl = tc::sdesc(b2l + kk * 2 * S::B2LBO, S::B2LBO, 128);
+            // K-major SWIZZLE_128B: 8 K-columns = 32 bytes inside a 32-column box, boxes KR rows apart
+            const uint32_t o = (kk >> 2) * KR * 128 + (kk & 3) * 32;
+            const uint64_t dbh = tc::sdesc_l(b2h + o, 16, 1024, 2);
+            const uint64_t dbl = tc::sdesc_l(b2l + o, 16, 1024, 2);
             const uint32_t acc = (ck > 0 || kk > 0) ? 1u : 0u;
             if (!(a.exp & 32)) {
               tc::mma_tf32_ts(tm + S::T_DA, tm + S::T_CH + kk * 8, dbh, id, acc);
@@ -428,7 +401,7 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
       YTA(16);
       if (fl & 2u) ++gs;
     }
-  } else {
+  } else if (w < Y_TMA_W) {
     // ------------------------------- epilogue -------------------------------
     const int Q = w & 3;
     uint32_t gs = 0;
@@ -503,6 +476,32 @@ __global__ void __launch_bounds__(Y_THREADS, 1) k_prefix_bwd(YArgs a) {
       }
       if (lane == 0) tc::mbar_arrive(&ctl.u_empty[ui & 3]);
     }
+  } else {
+    // ------------------------------- TMA producer -------------------------------
+    auto issue = [&](const Job& j, uint32_t sidx) {
+      const int c0 = (int)(j.u % UPG) * BPU * 128 + j.ck * CK;   // first slice column of the chunk
+      const uint32_t st = sidx % Y_NST;
+      const uint32_t a2 = tc::smem_u32(stg + st * S::STAGE), b2 = a2 + S::A2;
+      const int prow = (int)(j.qa << a.n1s);                      // dP stash row of tile row 0
+      tc::mbar_arrive_tx(&ctl.s_tma[st], S::A2 + S::B2 / 2);
+#pragma unroll
+      for (int h = 0; h < CK / 32; ++h) {
+        tc::tma_load_2d(a2 + h * YT * 128, &tm_dp, c0 + 32 * h, prow, &ctl.s_tma[st]);
+        tc::tma_load_2d(b2 + h * KR * 128, &tm_c2, c0 + 32 * h, j.crow, &ctl.s_tma[st]);
+      }
+    };
+    if (lane == 0) {
+      asm volatile("prefetch.tensormap [%0];" ::"l"(&tm_dp) : "memory");
+      asm volatile("prefetch.tensormap [%0];" ::"l"(&tm_c2) : "memory");
+      Job I;
+      start(I, G0);
+      for (uint32_t si = 0; I.u < NU; ++si) {
+        tc::mbar_wait(&ctl.s_free[si % Y_NST], ((si / Y_NST) & 1) ^ 1);
+        issue(I, si);
+        advance(I);
+      }
+    }
+    __syncwarp();
   }
   tc::fence_before();
   __syncthreads();
@@ -554,14 +553,46 @@ cudaError_t configure_bwdtc(Ctx& c) {
   return e;
 }
 
+namespace {
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                  const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+// fp32 matrix [rows][cols] (row stride cols), boxes of 32 columns x box_rows rows, SWIZZLE_128B,
+// out-of-range elements read as zero
+bool encode_rows(CUtensorMap* m, const float* base, uint64_t cols, uint64_t rows, uint32_t box_rows) {
+  static EncodeTiledFn enc = nullptr;
+  if (!enc) {
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", (void**)&enc, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+      enc = nullptr;
+    if (!enc) return false;
+  }
+  cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)std::max<uint64_t>(rows, 1)};
+  cuuint64_t strides[1] = {(cuuint64_t)cols * 4};
+  cuuint32_t box[2] = {32, box_rows}, es[2] = {1, 1};
+  return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(base), dims, strides, box, es,
+             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+}  // namespace
+
 // dC2 (fused update) and dC1 partials from the dP stash; requires run_fused_fwd's per-step
 // tables (grp_arow, grp_c2).
 cudaError_t run_prefix_bwd(Ctx& c, float lr, cudaStream_t s) {
   const PlanDev& p = c.p;
+  if (!c.tm_bwd_ready) {   // dP stash [P_cap n1][NC]; C2 region [sum m2 R][NC] (contiguous, NC-aligned)
+    if (!encode_rows(&c.tm_dp, p.dpbuf, (uint64_t)c.NC, (uint64_t)c.P_cap * c.n1, YT) ||
+        !encode_rows(&c.tm_c2, c.cores + c.c1_floats, (uint64_t)c.NC, (c.c3_begin - c.c1_floats) / c.NC,
+                     (uint32_t)c.R))
+      return cudaErrorInvalidValue;
+    c.tm_bwd_ready = true;
+  }
   YArgs a;
   a.cores = c.cores; a.grads = c.grads; a.state = c.state; a.meta = c.d_meta; a.counts = p.counts;
   a.grp_off = p.grp_off; a.grp_t = p.grp_t; a.pfx_i1 = p.pfx_i1; a.pfx_t = p.pfx_t; a.grp_arow = p.grp_arow;
-  a.grp_c2 = p.grp_c2; a.dpbuf = p.dpbuf; a.work = p.work + 2;
+  a.grp_c2 = p.grp_c2; a.dpbuf = p.dpbuf; a.work = p.work + 2; a.c2_begin = c.c1_floats;
   a.n1 = c.n1; a.n1s = c.n1 == 1 ? 0 : c.n1 == 2 ? 1 : c.n1 == 4 ? 2 : 3;
   a.NC = c.NC; a.nblk = (c.NC + 127) / 128; a.tpp = YT / c.n1; a.R = c.R;
   // K-chunks per work unit: R = 64 the whole slice in 64-column chunks, R = 128 one c-block in
@@ -580,9 +611,9 @@ cudaError_t run_prefix_bwd(Ctx& c, float lr, cudaStream_t s) {
     cudaMemsetAsync(trace, 0, sizeof(unsigned long long) * 32 * grid, s);
     a.trace = trace;
   }
-  if (c.R == 32) k_prefix_bwd<32><<<grid, Y_THREADS, YShape<32>::SMEM, s>>>(a);
-  else if (c.R == 64) k_prefix_bwd<64><<<grid, Y_THREADS, YShape<64>::SMEM, s>>>(a);
-  else k_prefix_bwd<128><<<grid, Y_THREADS, YShape<128>::SMEM, s>>>(a);
+  if (c.R == 32) k_prefix_bwd<32><<<grid, Y_THREADS, YShape<32>::SMEM, s>>>(c.tm_dp, c.tm_c2, a);
+  else if (c.R == 64) k_prefix_bwd<64><<<grid, Y_THREADS, YShape<64>::SMEM, s>>>(c.tm_dp, c.tm_c2, a);
+  else k_prefix_bwd<128><<<grid, Y_THREADS, YShape<128>::SMEM, s>>>(c.tm_dp, c.tm_c2, a);
   if (a.fused && a.opt != TTEMB_SGD)
     k_c2_update_zero<<<c.sm_count * 8, 256, 0, s>>>(c.cores, c.state, c.grads, p.grp_c2, p.counts,
                                                     (uint32_t)(c.R * c.NC), lr, c.eps);

@@ -9,6 +9,7 @@
 //   zeroed scan/sort state, and host staging buffers.
 #pragma once
 
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
 #include <stdlib.h>
@@ -164,6 +165,11 @@ struct Ctx {
   void mark_bucket(int i, cudaStream_t s) const {
     if (bucket_ev[i]) cudaEventRecord(bucket_ev[i], s);
   }
+
+  // TMA tensor maps of the prefix-backward kernel (dP stash, C2 region), encoded on first use
+  // (the buffers never move)
+  CUtensorMap tm_dp{}, tm_c2{};
+  bool tm_bwd_ready = false;
 
   // timing
   bool timing = false;
