@@ -9,14 +9,13 @@
 //       SWIZZLE_128B_BASE32B operand in shared memory (the C1 row pieces stored as loaded);
 //       accumulated in TMEM over all tiles of the group (no atomics, no partial buffers).
 //   dA[m][r1] = sum_c dP[m][c] . C2[i2][r1][c]                  (the C1 gradient partials)
-//       M = 128 = the tile's dP rows stacked as [dP_hi; dP_lo] IN TENSOR MEMORY (lanes 0-63 hi,
-//       64-127 lo, column = c of the current 64-c chunk), N = 64 r1, K = c; B = the C2 chunk
-//       (hi, lo) in shared memory as a K-major SWIZZLE_128B operand; two MMAs per K step
-//       accumulate dP_hi C2_hi + dP_hi C2_lo in
-//       lanes m and dP_lo C2_hi + dP_lo C2_lo in lanes 64 + m (3xTF32 plus the lo.lo term); the
-//       epilogue sums the two lane halves.  With A in TMEM the tensor core reads only the 2 KB
-//       B operand from shared memory per MMA (SS mode read 6 KB and shared the bandwidth with
-//       the loaders).
+//       one SS MMA per K step: M = 128 = the tile's dP rows stacked as [dP_hi; dP_lo] (rows
+//       0-63 as the TMA landed them, 64-127 the lo parts the loaders wrote next to them),
+//       N = 2 KR = [C2_hi | C2_lo] rows (likewise), K = c, both K-major SWIZZLE_128B operands in
+//       shared memory; the accumulator holds dP_{hi,lo} . C2_{hi,lo} in its four quadrants (3xTF32
+//       plus the lo.lo term) and the epilogue sums them.  (Round 2 measured this 1.10x faster
+//       than dP in TMEM written by the loaders with two N = KR MMAs per K step: the loaders'
+//       tensor-memory stores were on the critical path.)
 //       The epilogue adds dA straight into the C1 gradient (red.global.add.v4, L2-resident).
 // At the group's last tile the dC2 accumulator is drained: with TTEMB_FUSED_UPDATE and SGD the
 // C2 slice is updated in place by reductions straight from TMEM (the paper's fused TT core
@@ -26,8 +25,8 @@
 // fp32 accuracy: 3xTF32 (hi = raw fp32, read by the tensor core with truncation; lo =
 // x - trunc_tf32(x)); scripts/tc_probe3.cu measures the TMEM-A form.
 //
-// Warp roles (448 threads): 0-7 loaders (C2 lo split, dP and dP^T -> TMEM with the lo parts
-// computed in registers), 8 MMA issuer, 9-12 epilogue (dA -> dC1 reductions, dC2 -> gradient /
+// Warp roles (448 threads): 0-7 loaders (lo rows of the dP and C2 chunks, C1^T hi / lo, dP^T ->
+// TMEM with the lo part computed in registers), 8 MMA issuer, 9-12 epilogue (dA -> dC1 reductions, dC2 -> gradient /
 // fused update), 13 TMA producer (per K-chunk: 2-D TMA loads of the tile's dP rows and the C2
 // slice rows, SWIZZLE_128B, up to Y_NST chunks ahead).
 #include <stdio.h>
@@ -58,9 +57,11 @@ constexpr int Y_GI = 64;                        // work units per CTA whose meta
 template <int KR> struct YShape {
   static constexpr int BPU = KR <= 64 ? 2 : 1;
   static constexpr int CK = KR <= 64 ? 64 : 32;
-  // stage = [dP chunk | C2 chunk hi | C2 chunk lo], each as TMA SWIZZLE_128B boxes of 32 columns
-  // (tc::sw128_off): dP rows m = 64 per box, C2 rows r1 = KR per box (the K-major B operand)
-  static constexpr uint32_t A2 = YT * CK * 4;                           // dP chunk
+  // stage = [dP chunk | C2 chunk] as TMA SWIZZLE_128B boxes of 32 columns (tc::sw128_off); box h
+  // of the dP chunk = [hi rows m = 0..63 | lo rows 64..127] (the dA A operand, M = 128), box h of
+  // the C2 chunk = [hi rows r1 = 0..KR-1 | lo rows KR..2KR-1] (the dA B operand, N = 2 KR)
+  static constexpr uint32_t A2BOX = 2u * YT * 128, B2BOX = 2u * KR * 128;
+  static constexpr uint32_t A2 = 2u * YT * CK * 4;                      // dP chunk hi + lo
   static constexpr uint32_t B2 = 2u * KR * CK * 4;                      // C2 chunk hi + lo
   static constexpr uint32_t STAGE = A2 + B2;
   static constexpr uint32_t B1 = 2u * KR * YT * 4;                      // C1^T hi + lo (MN-major)
@@ -68,9 +69,9 @@ template <int KR> struct YShape {
   // TMEM columns
   static constexpr uint32_t T_DPT = 0;                                  // dP^T hi [64 BPU), lo [64 BPU, 128 BPU)
   static constexpr uint32_t T_DC2 = 128 * BPU;                          // dC2^T, KR per c-block
-  static constexpr uint32_t T_DA = T_DC2 + KR * BPU;                    // dA (N = KR)
-  static constexpr uint32_t T_CH = T_DA + KR;                           // [dP_hi; dP_lo] chunk, CK cols
-  static_assert(T_CH + CK <= 512, "TMEM budget");
+  static constexpr uint32_t T_DA = T_DC2 + KR * BPU;                    // dA quadrants (N = 2 KR)
+  static_assert(T_DA + 2 * KR <= 512, "TMEM budget");
+  static_assert(SMEM <= 227 * 1024, "shared memory budget");
 };
 
 struct YArgs {
@@ -98,7 +99,6 @@ struct YCtl {
   uint64_t s_tma[Y_NST];                  // K-chunk stage landed (TMA transactions)
   uint64_t d1_full, d1_free;              // dC2 accumulator (per group)
   uint64_t d2_full, d2_free;              // dA accumulator (per tile)
-  uint64_t p_free;                        // dP chunk A operand in TMEM (per chunk)
   uint64_t u_full[4], u_empty[4];
   uint32_t ring[4][5];                    // group, first prefix, #prefixes, flags (1 first, 2 last, 4 done), unit block
   uint32_t claim[2];
@@ -136,7 +136,6 @@ k_prefix_bwd(const __grid_constant__ CUtensorMap tm_dp, const __grid_constant__ 
     tc::mbar_init(&ctl.d1_free, Y_EW * 32);
     tc::mbar_init(&ctl.d2_full, 1);
     tc::mbar_init(&ctl.d2_free, Y_EW * 32);
-    tc::mbar_init(&ctl.p_free, 1);
     for (int s = 0; s < 4; ++s) { tc::mbar_init(&ctl.u_full[s], 1); tc::mbar_init(&ctl.u_empty[s], 1 + Y_EW); }
     tc::fence_mbar_init();
   }
@@ -253,15 +252,27 @@ k_prefix_bwd(const __grid_constant__ CUtensorMap tm_dp, const __grid_constant__ 
       tc::mbar_wait(&ctl.s_tma[sidx], (sp / Y_NST) & 1);
       YTA(3);
       char* a2 = stg + sidx * S::STAGE;
-      char* b2h = a2 + S::A2;
-      char* b2l = b2h + S::B2 / 2;
-      if (!(a.exp & 4)) {   // the C2 chunk's lo part (elementwise: same swizzled positions)
-        float4 q[C2F];
+      char* b2 = a2 + S::A2;
+      if (!(a.exp & 4)) {   // lo rows of both chunks: row n + 64 (dP) / n + KR (C2) of a box = lo of
+                            // row n (same swizzle phase: 64 % 8 == KR % 8 == 0), elementwise
+        constexpr int AF = YT * CK / 4 / 256;
+        float4 q[AF + C2F];
+        uint32_t o[AF + C2F];
 #pragma unroll
-        for (int k = 0; k < C2F; ++k) q[k] = reinterpret_cast<const float4*>(b2h)[tid + 256 * k];
+        for (int k = 0; k < AF; ++k) {
+          const uint32_t e = tid + 256 * k;
+          o[k] = (e / (YT * 8)) * S::A2BOX + (e % (YT * 8)) * 16;
+          q[k] = *reinterpret_cast<const float4*>(a2 + o[k]);
+        }
 #pragma unroll
-        for (int k = 0; k < C2F; ++k)
-          reinterpret_cast<float4*>(b2l)[tid + 256 * k] =
+        for (int k = 0; k < C2F; ++k) {
+          const uint32_t e = tid + 256 * k;
+          o[AF + k] = S::A2 + (e / (KR * 8)) * S::B2BOX + (e % (KR * 8)) * 16;
+          q[AF + k] = *reinterpret_cast<const float4*>(a2 + o[AF + k]);
+        }
+#pragma unroll
+        for (int k = 0; k < AF + C2F; ++k)
+          *reinterpret_cast<float4*>(a2 + o[k] + (k < AF ? YT * 128 : KR * 128)) =
               make_float4(lo32(q[k].x), lo32(q[k].y), lo32(q[k].z), lo32(q[k].w));
       }
       YTA(4);
@@ -279,7 +290,7 @@ k_prefix_bwd(const __grid_constant__ CUtensorMap tm_dp, const __grid_constant__ 
           float x[32];
 #pragma unroll
           for (int i = 0; i < 32; ++i) {
-            const float v = *reinterpret_cast<const float*>(a2 + tc::sw128_off(m0 + i, cc, YT));
+            const float v = *reinterpret_cast<const float*>(a2 + tc::sw128_off(m0 + i, cc, 2 * YT));
             x[i] = m0 + i < rows ? v : 0.f;
           }
           tc::tmem_st32(tc::taddr(tm + S::T_DPT + blk * 64 + m0, 32 * Q, 0), x);
@@ -289,29 +300,6 @@ k_prefix_bwd(const __grid_constant__ CUtensorMap tm_dp, const __grid_constant__ 
         }
       }
       YTA(6);
-      // dP of this chunk -> TMEM (dA A operand, M = 128): lanes 0-63 dP_hi rows, 64-127 dP_lo
-      // rows; warp (Q, h): rows 32 (Q & 1) + lane, columns 32 h .. 32 h + 31 of the chunk.
-      // Single-buffered: wait until the previous chunk's dA MMAs have read it.
-      tc::mbar_wait(&ctl.p_free, (sp & 1) ^ 1);
-      tc::fence_after();
-      {
-        const int Q = w & 3, h = w >> 2, m = 32 * (Q & 1) + lane;
-        if (!(a.exp & 8) && 32 * h < CK) {
-          float x[32];
-          const bool ok = m < rows;
-#pragma unroll
-          for (int k = 0; k < 8; ++k) {
-            float4 v = *reinterpret_cast<const float4*>(a2 + tc::sw128_off(m, 32 * h + 4 * k, YT));
-            if (!ok) v = make_float4(0.f, 0.f, 0.f, 0.f);
-            x[4 * k] = v.x; x[4 * k + 1] = v.y; x[4 * k + 2] = v.z; x[4 * k + 3] = v.w;
-          }
-          if (Q >= 2) {
-#pragma unroll
-            for (int i = 0; i < 32; ++i) x[i] = lo32(x[i]);
-          }
-          tc::tmem_st32(tc::taddr(tm + S::T_CH + 32 * h, 32 * Q, 0), x);
-        }
-      }
       tc::tmem_wait_st();
       tc::fence_async_smem();
       tc::fence_before();
@@ -350,22 +338,16 @@ k_prefix_bwd(const __grid_constant__ CUtensorMap tm_dp, const __grid_constant__ 
         YTA(12);
         tc::fence_after();
         if (lane == 0) {
-          const uint32_t id = tc::idesc_tf32(128, KR, false, false);
-          const uint32_t b2h = tc::smem_u32(stg + s * S::STAGE) + S::A2, b2l = b2h + S::B2 / 2;
+          const uint32_t id = tc::idesc_tf32(128, 2 * KR, false, false);
+          const uint32_t a2 = tc::smem_u32(stg + s * S::STAGE), b2 = a2 + S::A2;
 #pragma unroll
           for (int kk = 0; kk < CK / 8; ++kk) {
-            // K-major SWIZZLE_128B: 8 K-columns = 32 bytes inside a 32-column box, boxes KR rows apart
-            const uint32_t o = (kk >> 2) * KR * 128 + (kk & 3) * 32;
-            const uint64_t dbh = tc::sdesc_l(b2h + o, 16, 1024, 2);
-            const uint64_t dbl = tc::sdesc_l(b2l + o, 16, 1024, 2);
-            const uint32_t acc = (ck > 0 || kk > 0) ? 1u : 0u;
-            if (!(a.exp & 32)) {
-              tc::mma_tf32_ts(tm + S::T_DA, tm + S::T_CH + kk * 8, dbh, id, acc);
-              tc::mma_tf32_ts(tm + S::T_DA, tm + S::T_CH + kk * 8, dbl, id, 1u);
-            }
+            // K-major SWIZZLE_128B: 8 K-columns = 32 bytes inside a 32-column box
+            const uint64_t da = tc::sdesc_l(a2 + (kk >> 2) * S::A2BOX + (kk & 3) * 32, 16, 1024, 2);
+            const uint64_t db = tc::sdesc_l(b2 + (kk >> 2) * S::B2BOX + (kk & 3) * 32, 16, 1024, 2);
+            if (!(a.exp & 32)) tc::mma_tf32(tm + S::T_DA, da, db, id, (ck > 0 || kk > 0) ? 1u : 0u);
           }
           tc::commit(&ctl.s_free[s]);
-          tc::commit(&ctl.p_free);
           if (ck + 1 == a.nchunk) tc::commit(&ctl.d2_full);
         }
         __syncwarp();
@@ -427,6 +409,12 @@ k_prefix_bwd(const __grid_constant__ CUtensorMap tm_dp, const __grid_constant__ 
           dst = a.grads + ((size_t)__ldg(a.grp_arow + qa + (m >> a.n1s)) + (m & ((1 << a.n1s) - 1))) * KR;
         for (int h = 0; h < KR / 32; ++h) {
           tc::tmem_ld32(tc::taddr(tm + S::T_DA + 32 * h, 32 * Q, 0), v);
+          {   // + the C2_lo quadrant
+            float v2[32];
+            tc::tmem_ld32(tc::taddr(tm + S::T_DA + KR + 32 * h, 32 * Q, 0), v2);
+#pragma unroll
+            for (int i = 0; i < 32; ++i) v[i] += v2[i];
+          }
           if (dst && !(a.exp & 2)) {
 #pragma unroll
             for (int i = 0; i < 32; i += 4)
@@ -483,11 +471,11 @@ k_prefix_bwd(const __grid_constant__ CUtensorMap tm_dp, const __grid_constant__ 
       const uint32_t st = sidx % Y_NST;
       const uint32_t a2 = tc::smem_u32(stg + st * S::STAGE), b2 = a2 + S::A2;
       const int prow = (int)(j.qa << a.n1s);                      // dP stash row of tile row 0
-      tc::mbar_arrive_tx(&ctl.s_tma[st], S::A2 + S::B2 / 2);
+      tc::mbar_arrive_tx(&ctl.s_tma[st], S::A2 / 2 + S::B2 / 2);
 #pragma unroll
       for (int h = 0; h < CK / 32; ++h) {
-        tc::tma_load_2d(a2 + h * YT * 128, &tm_dp, c0 + 32 * h, prow, &ctl.s_tma[st]);
-        tc::tma_load_2d(b2 + h * KR * 128, &tm_c2, c0 + 32 * h, j.crow, &ctl.s_tma[st]);
+        tc::tma_load_2d(a2 + h * S::A2BOX, &tm_dp, c0 + 32 * h, prow, &ctl.s_tma[st]);
+        tc::tma_load_2d(b2 + h * S::B2BOX, &tm_c2, c0 + 32 * h, j.crow, &ctl.s_tma[st]);
       }
     };
     if (lane == 0) {
