@@ -644,33 +644,40 @@ def main():
                  "U": counts["U"], "P": counts["P"],
                  "NG": counts["NG"], "touched_slices": touched}
 
-    # ---- end-to-end through the host-buffer ABI calls ----
+    # ---- end-to-end from pinned host memory: every step copies its inputs in and its pooled ----
+    # ---- output back; HostStepPipeline overlaps step k+1's input copy and step k-1's output ----
+    # ---- copy with step k's kernels (two staging slots)                                      ----
     e2e = None
     if not args.no_e2e and world == 1:
         hpool = [(torch.as_tensor(i).pin_memory(), torch.as_tensor(o).pin_memory(),
                   torch.as_tensor(g).pin_memory()) for i, o, g in pool]
-        hout = torch.empty(B, cfg.num_tables, cfg.dim).pin_memory()
+        houts = [torch.empty(B, cfg.num_tables, cfg.dim).pin_memory() for _ in range(2)]
+        pipe = tt.HostStepPipeline(emb, max(p[0].numel() for p in hpool), B, depth=2)
 
         def hstep(i):
             hi, ho, hg = hpool[i % len(hpool)]
-            emb.forward_host(hi, ho, B, hout)
-            emb.backward_host(hg, lr=args.lr)
+            return pipe.step(hi, ho, hg, houts[i % 2], lr=args.lr)
 
-        for i in range(args.warmup):
-            hstep(i)
-        torch.cuda.synchronize()
-        hev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-        for i in range(args.steps):
-            flush.fill_(i & 0xff)
-            hev[i][0].record(stream)
-            hstep(i)
-            hev[i][1].record(stream)
-        torch.cuda.synchronize()
-        te = sum(a.elapsed_time(b) for a, b in hev)
+        with torch.cuda.stream(stream):
+            for i in range(args.warmup):
+                hstep(i)
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(pipe.h2d)                    # before the first input copy
+            last = 0
+            for i in range(args.steps):
+                flush.fill_(i & 0xff)
+                last = hstep(i)
+            e1.record(pipe.d2h)                    # after the last output copy
+            pipe.wait(last)
+            torch.cuda.synchronize()
+        te = e0.elapsed_time(e1)
         h2d = sum(p[0].size * 8 + p[1].size * 8 + p[2].size * 4 for p in pool) / len(pool)
         e2e = {"value": look_step * args.steps / (te / 1e3), "unit": UNIT, "h2d_bytes_per_step": int(h2d),
-               "d2h_bytes_per_step": int(hout.numel() * 4), "ms_per_step": te / args.steps,
-               "path": "ttemb_forward_host + ttemb_backward_host (pinned host buffers)"}
+               "d2h_bytes_per_step": int(houts[0].numel() * 4), "ms_per_step": te / args.steps,
+               "path": "HostStepPipeline: pinned host ids / offsets / grad_out -> device, "
+                       "ttemb_forward + ttemb_backward, pooled output -> pinned host; copies of "
+                       "neighbouring steps overlapped with compute (2 staging slots)"}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:

@@ -428,6 +428,36 @@ class TTEmbeddingBag:
         out.update(U=U, P=P, NG=NG)
         return out
 
+    # -- checkpoint / resume ---------------------------------------------------------------
+    def _signature(self) -> Dict:
+        return {"table_rows": list(self.table_rows), "row_factors": [list(f) for f in self.row_factors],
+                "col_factors": list(self.col_factors), "rank": self.rank, "optimizer": self.optimizer,
+                "dense": list(self.dense), "n_floats": self.n_floats}
+
+    def state_dict(self) -> Dict:
+        """Parameters and optimizer state as host tensors (a checkpoint): the flat core buffer
+        (all tables, storage layout of ttemb_core_layout), the Adagrad accumulators if any, and
+        the configuration they belong to.  Call between steps (the gradient buffer is not
+        saved: it is zero after an update / a fused backward)."""
+        torch.cuda.synchronize(self.device)
+        sd = {"format": "ttemb-v1", "config": self._signature(),
+              "cores": self.cores[:self.n_floats].detach().cpu().clone()}
+        if self.state is not None:
+            sd["state"] = self.state[:self.n_floats].detach().cpu().clone()
+        return sd
+
+    def load_state_dict(self, sd: Dict) -> None:
+        """Restore a state_dict() of an identically configured instance (bitwise)."""
+        if sd.get("format") != "ttemb-v1" or sd.get("config") != self._signature():
+            raise ValueError("checkpoint does not match this TTEmbeddingBag's configuration")
+        if (self.state is None) != ("state" not in sd):
+            raise ValueError("checkpoint optimizer state does not match")
+        self.cores[:self.n_floats].copy_(sd["cores"].to(self.device))
+        if self.state is not None:
+            self.state[:self.n_floats].copy_(sd["state"].to(self.device))
+        self.grads.zero_()
+        torch.cuda.synchronize(self.device)
+
     def set_timing(self, enable: bool) -> None:
         ttemb_set_timing(self.h, enable)
 
@@ -453,3 +483,60 @@ def _copy_device_f32(ptr: int, n: int, device) -> torch.Tensor:
     if n <= 0:
         return torch.empty(0, dtype=torch.float32, device=device)
     return torch.as_tensor(_DevArray(ptr, n, "<f4"), device=device).clone()
+
+
+class HostStepPipeline:
+    """End-to-end training steps from pinned host memory with the copies overlapped.
+
+    step(k): the inputs of step k (ids, offsets, grad_out; pinned host tensors) are copied to a
+    device staging slot on an H2D stream while the previous step computes; forward + backward
+    (the library's kernels) run on the compute stream once the slot has landed; the pooled
+    output is copied back to the caller's pinned host tensor on a D2H stream while the next step
+    computes.  `depth` slots rotate; a slot is refilled only after its last step's compute and
+    output copy finished (events), so nothing is overwritten in flight.  Host tensors must not be
+    modified until `wait(k)` returned for the step that uses them.
+    """
+
+    def __init__(self, emb: "TTEmbeddingBag", max_nnz: int, batch: int, depth: int = 2):
+        self.emb, self.depth, self.B = emb, int(depth), int(batch)
+        dev = emb.device
+        it = torch.int64 if emb.index_bits == 64 else torch.int32
+        self.h2d = torch.cuda.Stream(device=dev)
+        self.d2h = torch.cuda.Stream(device=dev)
+        self.idx = [torch.empty(max(max_nnz, 1), dtype=it, device=dev) for _ in range(depth)]
+        self.off = [torch.empty(emb.T * batch + 1, dtype=torch.int64, device=dev) for _ in range(depth)]
+        self.grad = [torch.empty(batch, emb.T, emb.N, dtype=torch.float32, device=dev) for _ in range(depth)]
+        self.out = [torch.empty(batch, emb.T, emb.N, dtype=torch.float32, device=dev) for _ in range(depth)]
+        self.ev_in = [torch.cuda.Event() for _ in range(depth)]
+        self.ev_comp = [torch.cuda.Event() for _ in range(depth)]
+        self.ev_out = [torch.cuda.Event() for _ in range(depth)]
+        self.k = 0
+
+    def step(self, h_idx: torch.Tensor, h_off: torch.Tensor, h_grad: torch.Tensor, h_out: torch.Tensor,
+             lr: float) -> int:
+        """Enqueue one training step; returns its step number (for wait)."""
+        k, s = self.k, self.k % self.depth
+        comp = torch.cuda.current_stream(self.emb.device)
+        nnz = h_idx.numel()
+        if k >= self.depth:
+            self.h2d.wait_event(self.ev_comp[s])          # the slot's inputs were consumed
+            comp.wait_event(self.ev_out[s])               # the slot's output was copied out
+        with torch.cuda.stream(self.h2d):
+            self.idx[s][:nnz].copy_(h_idx, non_blocking=True)
+            self.off[s].copy_(h_off, non_blocking=True)
+            self.grad[s].copy_(h_grad, non_blocking=True)
+            self.ev_in[s].record(self.h2d)
+        comp.wait_event(self.ev_in[s])
+        self.emb.forward(self.idx[s][:nnz], self.off[s], self.B, out=self.out[s], stream=comp)
+        self.emb.backward(self.grad[s], lr=lr, stream=comp)
+        self.ev_comp[s].record(comp)
+        self.d2h.wait_event(self.ev_comp[s])
+        with torch.cuda.stream(self.d2h):
+            h_out.copy_(self.out[s], non_blocking=True)
+            self.ev_out[s].record(self.d2h)
+        self.k += 1
+        return k
+
+    def wait(self, k: int) -> None:
+        """Block until step k's output reached host memory."""
+        self.ev_out[k % self.depth].synchronize()

@@ -121,24 +121,27 @@ k_pool_single(const float* __restrict__ rows, const uint32_t* __restrict__ inver
 // a7 one-hot, output-ordered: with one id per bag the validated offsets are the identity
 // (offsets[bag] = bag), so output row o = b*T + t reads position j = t*B + b directly and the
 // 109 MB (C4) output is written in address order.  Thread = (output row, float4 column).
+// Index math in I (uint32_t whenever the float4 count fits, the common case: a 64-bit division
+// is a long software sequence and made this copy ALU-bound), float4 columns per row NV = 2^nvs.
+template <typename I>
 __global__ void __launch_bounds__(256)
 k_pool_single_out(const float* __restrict__ rows, const uint32_t* __restrict__ inverse, int64_t nnz,
-                  int T, int B, int N, float* __restrict__ out, const uint32_t* __restrict__ counts,
+                  int T, int B, int N, int nvs, float* __restrict__ out, const uint32_t* __restrict__ counts,
                   const float* __restrict__ wpos) {
   if (counts[kCntMulti] != 0) return;
-  const int NV = N >> 2;
-  const int64_t total = (int64_t)T * B * NV, stride = (int64_t)gridDim.x * blockDim.x;
-  for (int64_t e0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e0 < total; e0 += TTEMB_POOL_IPT * stride) {
+  const I NV = (I)(N >> 2), uT = (I)T, uB = (I)B;
+  const I total = (I)T * (I)B * NV, stride = (I)gridDim.x * blockDim.x;
+  for (I e0 = (I)blockIdx.x * blockDim.x + threadIdx.x; e0 < total; e0 += TTEMB_POOL_IPT * stride) {
     float4 v[TTEMB_POOL_IPT];
 #pragma unroll
     for (int i = 0; i < TTEMB_POOL_IPT; ++i) {
-      const int64_t e = e0 + i * stride;
+      const I e = e0 + (I)i * stride;
       v[i] = make_float4(0.f, 0.f, 0.f, 0.f);
       if (e < total) {
-        const int64_t o = e / NV;
-        const int f = (int)(e - o * NV);
-        const int64_t b = o / T, t = o - b * T, j = t * B + b;
-        if (j < nnz) {
+        const I o = nvs >= 0 ? (e >> nvs) : e / NV;
+        const I f = e - o * NV;
+        const I b = o / uT, t = o - b * uT, j = t * uB + b;
+        if ((int64_t)j < nnz) {
           v[i] = __ldg(reinterpret_cast<const float4*>(rows + (size_t)__ldg(inverse + j) * N) + f);
           if (wpos) {
             const float w = __ldg(wpos + j);
@@ -149,7 +152,7 @@ k_pool_single_out(const float* __restrict__ rows, const uint32_t* __restrict__ i
     }
 #pragma unroll
     for (int i = 0; i < TTEMB_POOL_IPT; ++i)
-      if (e0 + i * stride < total) pool_store(reinterpret_cast<float4*>(out) + e0 + i * stride, v[i]);
+      if (e0 + (I)i * stride < total) pool_store(reinterpret_cast<float4*>(out) + e0 + (I)i * stride, v[i]);
   }
 }
 
@@ -198,10 +201,17 @@ cudaError_t run_forward_compute(Ctx& c, float* out, const int64_t* offsets, cuda
       if (c.N % 4 == 0) {
         // one id per bag (device flag): a position-parallel copy; otherwise the bag-parallel sum
         if (c.nnz > 0) {
-          if (TTEMB_POOL_MODE == 1)
-            k_pool_single_out<<<grid_for(c, total / (4 * TTEMB_POOL_IPT), 256, TTEMB_POOL_PER_SM), 256, 0, s>>>(
-                p.rows, p.inverse, c.nnz, c.T, c.B, c.N, out, p.counts, c.weighted ? p.wpos : nullptr);
-          else
+          if (TTEMB_POOL_MODE == 1) {
+            const int grid = grid_for(c, total / (4 * TTEMB_POOL_IPT), 256, TTEMB_POOL_PER_SM);
+            const int nv = c.N / 4, nvs = (nv & (nv - 1)) == 0 ? __builtin_ctz(nv) : -1;
+            const int64_t span = total / 4 + (int64_t)TTEMB_POOL_IPT * grid * 256;   // largest index formed
+            if (span < ((int64_t)1 << 32))
+              k_pool_single_out<uint32_t><<<grid, 256, 0, s>>>(p.rows, p.inverse, c.nnz, c.T, c.B, c.N, nvs, out,
+                                                             p.counts, c.weighted ? p.wpos : nullptr);
+            else
+              k_pool_single_out<uint64_t><<<grid, 256, 0, s>>>(p.rows, p.inverse, c.nnz, c.T, c.B, c.N, nvs, out,
+                                                             p.counts, c.weighted ? p.wpos : nullptr);
+          } else
             k_pool_single<<<grid_for(c, c.nnz * c.N / 16, 256, TTEMB_POOL_PER_SM), 256, 0, s>>>(
                 p.rows, p.inverse, p.bag_of, c.nnz, c.N, out, p.counts, c.weighted ? p.wpos : nullptr);
         }

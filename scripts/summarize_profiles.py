@@ -16,6 +16,7 @@ import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 OUT = os.path.join(ROOT, "gpurun_out")
+CONFIG_KEY = "c4-terabyte-r64"                 # the workload round_profile.sh captures
 PROF = os.path.join(ROOT, "profiles")
 STAGE_OF = {"k_tc_bwd2": "bwd_prefix", "k_tc_p": "fwd_prefix", "k_rows_bwd": "bwd_rows",
             "k_rows_fwd": "fwd_rows", "k_group_bwd": "bwd_prefix", "k_group_fwd": "fwd_prefix",
@@ -123,12 +124,14 @@ def ncu_top(tag):
             base = n.split("<")[0].split("::")[-1]
             st = STAGE_OF.get(base)
             if st:
-                traffic[st] = rd + wr
+                traffic[f"{CONFIG_KEY}/{st}"] = rd + wr
         except (KeyError, ValueError):
             pass
     open(os.path.join(PROF, f"{tag}_ncu_top.md"), "w").write("\n".join(lines) + "\n")
     if traffic:
-        json.dump({"source": f"profiles/{tag}_ncu_top.md", "dram_bytes_per_launch": traffic},
+        json.dump({"source": f"profiles/{tag}_ncu_top.md", "dram_bytes_per_launch": traffic,
+                   "note": "keys are <config name>-r<rank>/<stage> (the capture is of the c4 bench step); "
+                           "a config that was not captured gets traffic null"},
                   open(os.path.join(PROF, "traffic.json"), "w"), indent=1)
 
 
