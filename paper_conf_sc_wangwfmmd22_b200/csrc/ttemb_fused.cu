@@ -698,7 +698,7 @@ size_t rows_bwd_smem(int n3, int sw) { return (size_t)RW_WARPS * RW_NSL * (sw * 
 }  // namespace
 
 bool fused_eligible(const Ctx& c) {
-  // R = 64 (and ranks 16..63 stored padded to 64) with n2 R <= 256; R = 128 with n2 R <= 512
+  // R = 32 / 64 (ranks 16..63 stored padded to 32 or 64) with n2 R <= 256; R = 128 with n2 R <= 512
   return !(c.flags & TTEMB_FP32_CORES) && (c.R == 32 || c.R == 64 || c.R == 128) &&
          c.NC <= (c.R == 128 ? 512 : 256) &&
          (c.n3 == 4 || c.n3 == 8) && (c.n1 == 1 || c.n1 == 2 || c.n1 == 4 || c.n1 == 8) && c.n1 * c.n2 <= 16;

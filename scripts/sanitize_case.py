@@ -16,8 +16,23 @@ CASES = {
     "c2-b256": (lambda: W.config("c2"), dict(batch=256)),
     "tc-r64": (lambda: W.small_config([20000, 300], [(28, 28, 26), (7, 7, 7)], (4, 4, 4), 64, 96, 2, 1.05), {}),
     "ffma-split": (lambda: W.small_config([200000], [(2000, 10, 10)], (2, 2, 4), 16, 512, 2, 0.9), dict(fp32=True)),
+    "tc-r32": (lambda: W.small_config([20000, 300], [(28, 28, 26), (7, 7, 7)], (4, 4, 4), 32, 96, 2, 1.05), {}),
+    "tc-r128": (lambda: W.small_config([20000, 300], [(28, 28, 26), (7, 7, 7)], (4, 4, 8), 128, 64, 2, 1.05), {}),
 }
 name = sys.argv[1]
+if name == "hosttier":      # f4: host-memory tier kernels (cache sync / pool / grad / tick / update-push)
+    from paper_conf_sc_wangwfmmd22_b200.hosttier import HostTierEmbedding
+    rows, B, L = [300, 50, 800], 32, 3
+    batches = [W.make_host_batch(rows, B, 3, 1.05, step=k, seed=1) for k in range(6)]
+    ht = HostTierEmbedding(rows, 16, B, len(rows) * B * 3, L, 0.05, threaded=False,
+                           weight=W.make_host_weight(rows, 16, seed=1))
+    ht.start(lambda k: batches[k], len(batches))
+    for k in range(len(batches)):
+        o = ht.forward(k)
+        ht.backward((o - 0.1).contiguous())
+    ht.finish()
+    print(name, "ok", ht.cache_stats())
+    sys.exit(0)
 mk, kw = CASES[name]
 cfg = mk()
 B = kw.get("batch", cfg.batch)

@@ -13,8 +13,8 @@ import sys
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 HEADER = """# {tag}: bench lines of every BASELINE config (one B200, `scripts/config_sweep.sh`)
 
-Parity of every config against the oracle: tests/test_gpu_parity.py (c1-c3 full batch, c4 reduced batch + full-size sampled, c5 r32/r64/r128 full-size sampled).
-tcgen05 path: c4 and c5-r64 (R = 64), c2, c3, c5-r32 (R = 16 / 32 stored zero-padded to 64, DESIGN.md R28); FFMA path: c1 (R = 8) and c5-r128 (DESIGN.md section 14 item 2).
+Parity of every config against the oracle: tests/test_gpu_parity.py (c1-c3 full batch; c4 full batch fwd + bwd + fused SGD / Adagrad; c5 r32/r64/r128 full-size sampled fwd + bwd).
+tcgen05 path: c2 (R = 16 stored zero-padded to 32, DESIGN.md R28), c3 and c5-r32 (native R = 32), c4 and c5-r64 (R = 64), c5-r128 (R = 128); FFMA path: c1 (R = 8).
 
 | workload | tables | dim | R | batch | L | opt | ms/step | lookups/s | e2e lookups/s |
 |---|---|---|---|---|---|---|---|---|---|
