@@ -89,19 +89,6 @@ __device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t
                : "memory");
 }
 
-// 1-D bulk (TMA engine) shared -> global copy in this thread's bulk group; dst, src and bytes
-// multiples of 16.  bulk_commit() closes the group, bulk_wait_read<N>() waits until at most N
-// groups still read shared memory (the source may then be overwritten).
-__device__ __forceinline__ void bulk_s2g(void* dst, uint32_t src, uint32_t bytes) {
-  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(src), "r"(bytes)
-               : "memory");
-}
-__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory"); }
-template <int N>
-__device__ __forceinline__ void bulk_wait() { asm volatile("cp.async.bulk.wait_group %0;" ::"n"(N) : "memory"); }
-
 // 2-D tiled TMA load (tensor map in kernel-parameter / constant space) into shared memory,
 // completing the box's bytes as transactions on mbar.  c0 = inner (contiguous) coordinate.
 __device__ __forceinline__ void tma_load_2d(uint32_t dst, const void* tmap, int c0, int c1, uint64_t* mbar) {

@@ -311,14 +311,9 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
     }
   } else {
     // ------------------------- epilogue: TMEM -> P stash -------------------------
-    // warp w drains lane quarter Q = w % 4 of every c-block of the unit (thread = column c, 32
-    // tile rows per tcgen05.ld) into a shared-memory staging tile [rows][SW] (conflict-free: a
-    // warp store covers 32 consecutive columns), then one thread writes each valid row of the
-    // tile to the P stash with a 1-D bulk copy (the TMA engine does the global writes; the
-    // per-element global stores made this drain the kernel's critical path)
-    const int Q = w & 3, et = tid - X_ROW_W0 * 32;
-    constexpr int SW = BPU * 128;                          // staging row width (floats)
-    float* const stg = reinterpret_cast<float*>(bbuf + 2 * BSLOT);
+    // warp w drains lane quarter Q = w % 4 of every c-block of the unit: thread = column c, 32
+    // tile rows per tcgen05.ld; pbuf[(q n1 + j1)][c] rows of one tile are contiguous
+    const int Q = w & 3;
     for (uint32_t ui = 0;; ++ui) {
       XT0();
       tc::mbar_wait(&ctl.u_full[ui & 3], (ui >> 2) & 1);
@@ -332,34 +327,26 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
       tc::mbar_wait(&ctl.d_full[s], (ui >> 1) & 1);
       XTA(1);
       tc::fence_after();
-      if (et == 0) tc::bulk_wait_read<0>();                // the previous tile's bulk stores read the staging
-      tc::named_sync(2, X_RW * 32);
+      float* dst = a.pbuf + (size_t)qa * a.n1 * a.NC;
       for (int blk = 0; blk < BPU; ++blk) {
-        const int cl = blk * 128 + Q * 32 + lane;
+        const int c = ((int)ub * BPU + blk) * 128 + Q * 32 + lane;
         for (int j0 = 0; j0 < rows; j0 += 32) {
           float v[32];
           tc::tmem_ld32(tc::taddr(tm + 256 + s * 128 + blk * 64 + j0, 32 * Q, 0), v);
           const int lim = min(32, rows - j0);
+          if (c < a.NC) {
+            float* d = dst + (size_t)j0 * a.NC + c;
 #pragma unroll
-          for (int j = 0; j < 32; ++j)
-            if (j < lim) stg[(j0 + j) * SW + cl] = v[j];
+            for (int j = 0; j < 32; ++j)
+              if (j < lim) d[(size_t)j * a.NC] = v[j];
+          }
         }
       }
       tc::fence_before();
-      tc::mbar_arrive(&ctl.d_free[s]);                     // the TMEM slot is free again
-      tc::fence_async_smem();                              // staging writes -> async proxy
-      tc::named_sync(2, X_RW * 32);
-      if (et == 0) {
-        const int c0 = (int)ub * SW, nb = min(SW, a.NC - c0) * 4;
-        float* dst = a.pbuf + (size_t)qa * a.n1 * a.NC + c0;
-        const uint32_t src = tc::smem_u32(stg);
-        for (int r = 0; r < rows; ++r) tc::bulk_s2g(dst + (size_t)r * a.NC, src + (uint32_t)(r * SW * 4), (uint32_t)nb);
-        tc::bulk_commit();
-      }
+      tc::mbar_arrive(&ctl.d_free[s]);
       XTA(2);
       if (lane == 0) tc::mbar_arrive(&ctl.u_empty[ui & 3]);
     }
-    if (et == 0) tc::bulk_wait<0>();                       // every row written before the kernel ends
   }
   if (a.trace) {
     const int role = tid == 0 ? 0 : tid == X_MMA_W * 32 ? 1 : tid == X_ROW_W0 * 32 ? 2 : -1;
@@ -377,10 +364,7 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
   if (w == X_MMA_W) tc::tmem_dealloc(tm, 512);
 }
 
-// raw C2 staging + two B slots + the epilogue's P staging tile [XT][BPU 128]
-template <int KR> constexpr size_t prefix_smem() {
-  return 128 + X_RAW_BYTES + 2 * (2u * XT * KR * 4) + (size_t)XT * (KR <= 64 ? 256 : 128) * 4;
-}
+template <int KR> constexpr size_t prefix_smem() { return 128 + X_RAW_BYTES + 2 * (2u * XT * KR * 4); }
 
 // ------------------------------------------------------------------------------------
 // Row contraction a6 (Eq. 2, Fig. 5(b) step 3): E_u = P_q (n1 n2 x R) . C3[i3_u] (R x n3)
