@@ -253,6 +253,31 @@ k_prefix_bwd(const __grid_constant__ CUtensorMap tm_dp, const __grid_constant__ 
       YTA(3);
       char* a2 = stg + sidx * S::STAGE;
       char* b2 = a2 + S::A2;
+      // dP^T first (it reads only the TMA-landed hi rows), so its tensor-memory stores complete
+      // while the lo rows are written; no loader-wide barrier: every thread fences its own
+      // shared-memory writes and arrives on s_full itself
+      {   // dP^T of this chunk -> TMEM (dC2 A operand): thread = column, 32 tile rows; lo in
+          // registers.  R = 64: chunk ck covers c-block ck / 2, lane quarters 2 (ck & 1) + {0, 1};
+          // R = 128: the unit's block, lane quarter ck & 3.
+        const int Q = w & 3;
+        const int blk = BPU == 2 ? (P.ck >> 1) : 0;
+        const bool mine = BPU == 2 ? ((Q >> 1) == (P.ck & 1) && blk < a.nblk) : (Q == (P.ck & 3));
+        if (mine && !(a.exp & 8)) {
+          const int cc = BPU == 2 ? 32 * (Q & 1) + lane : lane;   // column inside the chunk
+          const int m0 = 32 * (w >> 2);                           // warps 0-3: rows 0..31, 4-7: 32..63
+          float x[32];
+#pragma unroll
+          for (int i = 0; i < 32; ++i) {
+            const float v = *reinterpret_cast<const float*>(a2 + tc::sw128_off(m0 + i, cc, 2 * YT));
+            x[i] = m0 + i < rows ? v : 0.f;
+          }
+          tc::tmem_st32(tc::taddr(tm + S::T_DPT + blk * 64 + m0, 32 * Q, 0), x);
+#pragma unroll
+          for (int i = 0; i < 32; ++i) x[i] = lo32(x[i]);
+          tc::tmem_st32(tc::taddr(tm + S::T_DPT + 64 * BPU + blk * 64 + m0, 32 * Q, 0), x);
+        }
+      }
+      YTA(5);
       if (!(a.exp & 4)) {   // lo rows of both chunks: row n + 64 (dP) / n + KR (C2) of a box = lo of
                             // row n (same swizzle phase: 64 % 8 == KR % 8 == 0), elementwise
         constexpr int AF = YT * CK / 4 / 256;
@@ -274,30 +299,6 @@ k_prefix_bwd(const __grid_constant__ CUtensorMap tm_dp, const __grid_constant__ 
         for (int k = 0; k < AF + C2F; ++k)
           *reinterpret_cast<float4*>(a2 + o[k] + (k < AF ? YT * 128 : KR * 128)) =
               make_float4(lo32(q[k].x), lo32(q[k].y), lo32(q[k].z), lo32(q[k].w));
-      }
-      YTA(4);
-      tc::named_sync(1, Y_LW * 32);                     // whole chunk (hi and lo) visible
-      YTA(5);
-      {   // dP^T of this chunk -> TMEM (dC2 A operand): thread = column, 32 tile rows; lo in
-          // registers.  R = 64: chunk ck covers c-block ck / 2, lane quarters 2 (ck & 1) + {0, 1};
-          // R = 128: the unit's block, lane quarter ck & 3.
-        const int Q = w & 3;
-        const int blk = BPU == 2 ? (P.ck >> 1) : 0;
-        const bool mine = BPU == 2 ? ((Q >> 1) == (P.ck & 1) && blk < a.nblk) : (Q == (P.ck & 3));
-        if (mine && !(a.exp & 8)) {
-          const int cc = BPU == 2 ? 32 * (Q & 1) + lane : lane;   // column inside the chunk
-          const int m0 = 32 * (w >> 2);                           // warps 0-3: rows 0..31, 4-7: 32..63
-          float x[32];
-#pragma unroll
-          for (int i = 0; i < 32; ++i) {
-            const float v = *reinterpret_cast<const float*>(a2 + tc::sw128_off(m0 + i, cc, 2 * YT));
-            x[i] = m0 + i < rows ? v : 0.f;
-          }
-          tc::tmem_st32(tc::taddr(tm + S::T_DPT + blk * 64 + m0, 32 * Q, 0), x);
-#pragma unroll
-          for (int i = 0; i < 32; ++i) x[i] = lo32(x[i]);
-          tc::tmem_st32(tc::taddr(tm + S::T_DPT + 64 * BPU + blk * 64 + m0, 32 * Q, 0), x);
-        }
       }
       YTA(6);
       tc::tmem_wait_st();
