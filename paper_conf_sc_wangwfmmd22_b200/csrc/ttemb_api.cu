@@ -214,7 +214,7 @@ size_t carve(Ctx& c, uint8_t* base) {
   p.keysB = k.take<uint32_t>(nnz); p.valsB = k.take<uint32_t>(nnz);
   p.bag_of = k.take<uint32_t>(nnz); p.sbag = k.take<uint32_t>(nnz); p.inverse = k.take<uint32_t>(nnz);
   p.ukey = k.take<uint32_t>(U); p.seg_off = k.take<uint32_t>(U + 1);
-  p.row_pfx = k.take<uint32_t>(U); p.row_i3 = k.take<uint32_t>(U);
+  p.row_pfx = k.take<uint32_t>(U); p.row_i3 = k.take<uint32_t>(U); p.row_c3 = k.take<uint32_t>(U);
   p.pfx_t = k.take<uint32_t>(P); p.pfx_i1 = k.take<uint32_t>(P); p.pfx_i2 = k.take<uint32_t>(P);
   p.row_seg = k.take<uint32_t>(P + 1);
   p.gkeyB = k.take<uint32_t>(P); p.gvalB = k.take<uint32_t>(P);

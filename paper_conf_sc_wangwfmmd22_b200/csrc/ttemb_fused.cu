@@ -25,10 +25,6 @@
 #include "tc.cuh"
 #include "ttemb_internal.cuh"
 
-#ifndef TTEMB_G_EVICT_FIRST
-#define TTEMB_G_EVICT_FIRST 0  // 1 = L2 evict-first policy on k_rows_bwd2's reads of G
-#endif
-
 namespace ttemb {
 
 namespace {
@@ -382,7 +378,8 @@ constexpr int RW_WARPS = 8, RW_RCH = 16, RW_NSL = 3;
 struct RowArgs {
   const float* cores;
   const TableMeta* meta;
-  const uint32_t *counts, *row_pfx, *row_i3, *pfx_t, *seg_off, *sbag;
+  const uint32_t *counts, *row_pfx, *row_c3, *pfx_t, *seg_off, *sbag;
+  unsigned long long c3_begin;   // float offset of the C3 region (row_c3 counts R n3 slices from it)
   const float* pbuf;          // [P][n1][NC]
   float* rows;                // [U][N]
   float* out;                 // [B][T][N]: written directly when every bag holds one id (a7)
@@ -417,7 +414,7 @@ __global__ void __launch_bounds__(RW_WARPS * 32, RPL == 8 ? 3 : 2) k_rows_fwd2(R
     unsigned long long o3l = 0;
     if (lane < nr) {
       ql = __ldg(a.row_pfx + u0 + lane);
-      o3l = a.meta[__ldg(a.pfx_t + ql)].c3_off + (unsigned long long)__ldg(a.row_i3 + u0 + lane) * KR * N3;
+      o3l = a.c3_begin + (unsigned long long)__ldg(a.row_c3 + u0 + lane) * KR * N3;
     }
     auto issue = [&](int j) {
       const unsigned long long o3 = __shfl_sync(0xffffffffu, o3l, j);
@@ -500,20 +497,26 @@ __global__ void __launch_bounds__(RW_WARPS * 32, RPL == 8 ? 3 : 2) k_rows_fwd2(R
 size_t rows_smem(int n3, int R) { return (size_t)RW_WARPS * RW_NSL * (R * n3 + R / 2) * 4; }
 
 // ------------------------------------------------------------------------------------
-// Row backward a9 (Eq. 6 read as left^T . dL/de . right^T), same lane map and
-// C3 ring as k_rows_fwd2, with the aggregated row gradient G_u (a8) staged next to C3:
-//   dP_q[j12][r] += sum_j3 G_u[j12][j3] C3_u[r][j3]   registers (4 j12 x 8 r per lane),
-//                                                     flushed to dpbuf at prefix changes
-//   dC3[i3_u][r][j3] += sum_j12 P_q[j12][r] G_u[j12][j3]  partial over the lane's 4 j12,
-//                    reduced over jq (2 shuffle levels), red.global.add.v4 (L2-resident)
-// dP of a prefix whose rows straddle a chunk boundary is accumulated with vector reductions
-// into rows zeroed by k_dp_zero2; prefixes inside one chunk are stored directly.
+// Row backward a9 (Eq. 6 read as left^T . dL/de . right^T).  A warp owns 16
+// consecutive unique rows (rows of one prefix are consecutive) and one SW-wide slice of r;
+// lane l owns r = rb + RL l + x (x < RL) for ALL j12 and j3, so neither product needs a
+// cross-lane reduction:
+//   dP_q[j12][r] += sum_j3 G_u[j12][j3] C3_u[r][j3]     registers (16 j12 x RL per lane),
+//                                                       flushed to dpbuf at prefix changes
+//   dC3[i3_u][r][j3] += sum_j12 P_q[j12][r] G_u[j12][j3]  (RL x n3 per lane, red.global.add.v4
+//                                                         into the L2-resident gradient)
+// The C3 slice (r-slice of the row) and G_u stream into a per-warp 3-slot shared-memory ring by
+// cp.async two rows ahead; the C3 part is stored [x][j3/4][l] in 16-byte pieces so a lane's
+// loads are conflict-free, and G_u is read as broadcasts.  dP of a prefix whose rows straddle a
+// chunk boundary is accumulated with vector reductions into rows zeroed by k_dp_zero2;
+// prefixes inside one chunk are stored directly.
 // ------------------------------------------------------------------------------------
 struct RowBwdArgs {
   const float* cores;
   float* grads;
   const TableMeta* meta;
-  const uint32_t *counts, *row_pfx, *row_i3, *pfx_t, *row_seg;
+  const uint32_t *counts, *row_pfx, *row_c3, *pfx_t, *row_seg;
+  unsigned long long c3_begin;   // float offset of the C3 region (row_c3 counts R n3 slices from it)
   const float* pbuf;          // [P][n1][NC]
   const float* gbuf;          // [U][N]
   float* dpbuf;               // [P][n1][NC]
@@ -536,65 +539,65 @@ __device__ __forceinline__ void red_v4(float* addr, float4 v) {
   asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(addr), "f"(v.x), "f"(v.y), "f"(v.z), "f"(v.w)
                : "memory");
 }
+__device__ __forceinline__ void red_v2(float* addr, float x, float y) {
+  asm volatile("red.global.add.v2.f32 [%0], {%1, %2};" ::"l"(addr), "f"(x), "f"(y) : "memory");
+}
 
-template <int N3, int RPL>   // RPL = r values per lane: 4 (R = 32) or 8 (R = 64; R = 128 in two slices)
+constexpr int RB_J12 = 16;   // n1 n2 <= 16
+
+// P_q[j12][r] sits at pbuf[(q J12 + j12) R + r] (NC = n2 R), so with R a template constant every
+// per-j12 access is an immediate offset from one base pointer.
+template <int N3, int RL, int KR, int J12T>   // RL = r per lane: 1 (R = 32) or 2 (R = 64, 128 in two
+                                              // slices); J12T = n1 n2 (0: runtime, <= 16)
 __global__ void __launch_bounds__(RW_WARPS * 32, 2) k_rows_bwd2(RowBwdArgs a) {
-  constexpr int SW = 8 * RPL;                   // r width of a work item (a slice of R)
-  constexpr int C3S = SW * N3 + SW / 2;         // skewed C3 part of a slot (+ 4 floats per 8 rows)
-  constexpr int SLOT = C3S + 16 * N3;           // + G_u (N <= 16 n3)
-  constexpr int C3L = SW * N3 / 4 / 32;
+  constexpr int SW = 32 * RL;                   // r width of a work item (a slice of R)
+  constexpr int NSL = KR / SW;                  // slices per row
+  constexpr int C3S = SW * N3;                  // C3 part of a slot
+  constexpr int SLOT = C3S + RB_J12 * N3;       // + G_u (N <= 16 n3)
+  constexpr int H4 = N3 / 4;                    // 16-byte pieces per r row
+  constexpr int C3L = RL * H4;                  // 16-byte pieces of the C3 slice per lane
+  constexpr int JM = J12T ? J12T : RB_J12;      // unrolled j12 extent
   extern __shared__ __align__(16) float rw_smem[];
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   float* const ringp = rw_smem + w * (RW_NSL * SLOT);
   const uint32_t ring = tc::smem_u32(ringp);
   const uint32_t U = tt_rows(a.counts);   // TT rows only (hybrid: dense rows follow)
-  const int J12 = a.n1 * a.n2;
-  const int jq = lane >> 3, rp = lane & 7;
-  // R = 128: a work item is (16 rows, one 64-wide slice of r), the lane map of R = 64 per slice:
-  // dP_q[j12][r] and dC3[i3][r][j3] of a slice are independent of the other slice
-  const int nsl = a.R / SW;
-  int poff0[4];
-#pragma unroll
-  for (int e = 0; e < 4; ++e) {
-    const int j12 = 4 * jq + e, j1 = j12 / a.n2, j2 = j12 - j1 * a.n2;
-    poff0[e] = j12 < J12 ? j1 * a.NC + j2 * a.R + RPL * rp : -1;
-  }
+  const int J12 = J12T ? J12T : a.n1 * a.n2;
   const int64_t nch = ((int64_t)U + RW_RCH - 1) / RW_RCH;
   const int64_t gw = (int64_t)blockIdx.x * RW_WARPS + w, nw = (int64_t)gridDim.x * RW_WARPS;
-  for (int64_t it = gw; it < nch * nsl; it += nw) {
-    const int64_t ch = it / nsl;
-    const int rb = SW * (int)(it - ch * nsl);     // first r of the slice
-    int poff[4];
-#pragma unroll
-    for (int e = 0; e < 4; ++e) poff[e] = poff0[e] >= 0 ? poff0[e] + rb : -1;
+  // work item metadata (row prefix, C3 slice) is loaded one item ahead
+  auto load_meta = [&](int64_t it, uint32_t& q, uint32_t& c3) {
+    q = 0; c3 = 0;
+    if (it < nch * NSL) {
+      const uint32_t u = (uint32_t)(NSL == 1 ? it : it / NSL) * RW_RCH + lane;
+      if (u < U) { q = __ldg(a.row_pfx + u); c3 = __ldg(a.row_c3 + u); }
+    }
+  };
+  uint32_t nql, nc3;
+  load_meta(gw, nql, nc3);
+  for (int64_t it = gw; it < nch * NSL; it += nw) {
+    const int64_t ch = NSL == 1 ? it : it / NSL;
+    const int rb = SW * (int)(it - ch * NSL);     // first r of the slice (R = 128: two slices)
+    const int rl = rb + RL * lane;                // this lane's first r
     const uint32_t u0 = (uint32_t)ch * RW_RCH;
     const int nr = (int)min((uint32_t)RW_RCH, U - u0);
-    uint32_t ql = 0;
-    unsigned long long o3l = 0;
-    if (lane < nr) {
-      ql = __ldg(a.row_pfx + u0 + lane);
-      o3l = a.meta[__ldg(a.pfx_t + ql)].c3_off + (unsigned long long)__ldg(a.row_i3 + u0 + lane) * a.R * N3 +
-            (unsigned long long)rb * N3;
-    }
+    const uint32_t ql = nql;
+    // the row's C3 slice, this work item's r-slice
+    const unsigned long long o3l = a.c3_begin + (unsigned long long)nc3 * KR * N3 + (unsigned long long)rb * N3;
+    load_meta(it + nw, nql, nc3);
     const uint32_t prevq = u0 > 0 ? __ldg(a.row_pfx + u0 - 1) : 0xffffffffu;
     const uint32_t nextq = u0 + nr < U ? __ldg(a.row_pfx + u0 + nr) : 0xffffffffu;
+    // slot layout: C3 piece (x, h) of lane l at [(x H4 + h) 32 + l] (16 bytes each: the warp's
+    // cp.async stores and a lane's loads are contiguous / conflict-free), then G_u
     auto issue = [&](int j) {
-      const unsigned long long o3 = __shfl_sync(0xffffffffu, o3l, j);
+      const unsigned long long o3 = __shfl_sync(0xffffffffu, o3l, j) + (unsigned long long)(RL * lane) * N3;
       const float4* src = reinterpret_cast<const float4*>(a.cores + o3);
-      const uint32_t dst = ring + (uint32_t)((j % RW_NSL) * SLOT * 4);
+      const uint32_t dst = ring + (uint32_t)((j % RW_NSL) * SLOT * 4) + 16u * lane;
 #pragma unroll
-      for (int i = 0; i < C3L; ++i) {
-        const int f = lane + 32 * i, r = f / (N3 / 4);
-        tc::cp_async16(dst + 4u * (uint32_t)(4 * f + 4 * (r >> 3)), src + f);
-      }
+      for (int i = 0; i < C3L; ++i) tc::cp_async16(dst + 16u * 32u * i, src + i);
       if (lane < a.N / 4)
-#if TTEMB_G_EVICT_FIRST
-        tc::cp_async16_ef(dst + 4u * (uint32_t)(C3S + 4 * lane),   // G row: read once
-                          reinterpret_cast<const float4*>(a.gbuf + (size_t)(u0 + j) * a.N) + lane);
-#else
-        tc::cp_async16(dst + 4u * (uint32_t)(C3S + 4 * lane),
+        tc::cp_async16(ring + (uint32_t)(((j % RW_NSL) * SLOT + C3S) * 4) + 16u * lane,
                        reinterpret_cast<const float4*>(a.gbuf + (size_t)(u0 + j) * a.N) + lane);
-#endif
     };
 #pragma unroll
     for (int j = 0; j < RW_NSL - 1; ++j) {
@@ -602,18 +605,20 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 2) k_rows_bwd2(RowBwdArgs a) {
       tc::cp_commit();
     }
     uint32_t curq = 0xffffffffu;
-    float pr[4][RPL], dp[4][RPL];
+    float pr[JM][RL], dp[JM][RL];
     auto flush = [&]() {
       const bool red = curq == prevq || curq == nextq;
-      float* d = a.dpbuf + (size_t)curq * a.n1 * a.NC;
+      float* d = a.dpbuf + (size_t)curq * J12 * KR + rl;
 #pragma unroll
-      for (int e = 0; e < 4; ++e) {
-        if (poff[e] < 0) continue;
-#pragma unroll
-        for (int h = 0; h < RPL; h += 4) {
-          const float4 v = make_float4(dp[e][h], dp[e][h + 1], dp[e][h + 2], dp[e][h + 3]);
-          if (red) red_v4(d + poff[e] + h, v);
-          else *reinterpret_cast<float4*>(d + poff[e] + h) = v;
+      for (int j12 = 0; j12 < JM; ++j12) {
+        if (!J12T && j12 >= J12) break;
+        float* e = d + j12 * KR;
+        if (RL == 2) {
+          if (red) red_v2(e, dp[j12][0], dp[j12][RL - 1]);
+          else *reinterpret_cast<float2*>(e) = make_float2(dp[j12][0], dp[j12][RL - 1]);
+        } else {
+          if (red) atomicAdd(e, dp[j12][0]);
+          else *e = dp[j12][0];
         }
       }
     };
@@ -621,71 +626,71 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 2) k_rows_bwd2(RowBwdArgs a) {
       const uint32_t q = __shfl_sync(0xffffffffu, ql, j);
       if (q != curq) {
         if (curq != 0xffffffffu) flush();
-        const float* pq = a.pbuf + (size_t)q * a.n1 * a.NC;
+        {   // L1 prefetch of the next prefix of the item (its P slice: 16 j12 x SW floats)
+          const unsigned later = __ballot_sync(0xffffffffu, lane > j && lane < nr && ql != q);
+          if (later) {
+            const uint32_t qn = __shfl_sync(0xffffffffu, ql, __ffs(later) - 1);
+            if ((lane >> 1) < J12)
+              asm volatile("prefetch.global.L1 [%0];" ::"l"(a.pbuf + (size_t)qn * J12 * KR + (lane >> 1) * KR + rb + 32 * (lane & 1)));
+          }
+        }
+        const float* pq = a.pbuf + (size_t)q * J12 * KR + rl;
 #pragma unroll
-        for (int e = 0; e < 4; ++e) {
+        for (int j12 = 0; j12 < JM; ++j12) {
+          if (J12T || j12 < J12) {
+            if (RL == 2) {
+              const float2 x0 = __ldg(reinterpret_cast<const float2*>(pq + j12 * KR));
+              pr[j12][0] = x0.x; pr[j12][RL - 1] = x0.y;
+            } else {
+              pr[j12][0] = __ldg(pq + j12 * KR);
+            }
+          } else {
 #pragma unroll
-          for (int h = 0; h < RPL; h += 4) {
-            const float4 x0 = poff[e] >= 0 ? __ldg(reinterpret_cast<const float4*>(pq + poff[e] + h))
-                                           : make_float4(0.f, 0.f, 0.f, 0.f);
-            pr[e][h] = x0.x; pr[e][h + 1] = x0.y; pr[e][h + 2] = x0.z; pr[e][h + 3] = x0.w;
+            for (int x = 0; x < RL; ++x) pr[j12][x] = 0.f;
           }
 #pragma unroll
-          for (int x = 0; x < RPL; ++x) dp[e][x] = 0.f;
+          for (int x = 0; x < RL; ++x) dp[j12][x] = 0.f;
         }
         curq = q;
       }
       tc::cp_wait<RW_NSL - 2>();
       __syncwarp();
       const float* slot = ringp + (j % RW_NSL) * SLOT;
-      float g[4][N3];
+      float c3[RL][N3], dc[RL][N3];
 #pragma unroll
-      for (int e = 0; e < 4; ++e)
+      for (int i = 0; i < C3L; ++i) {   // piece i = (x, h): r = rl + x, j3 = 4h .. 4h + 3
+        const int x = i / H4, h = i - x * H4;
+        const float4 t4 = *reinterpret_cast<const float4*>(slot + 4 * (i * 32 + lane));
+        c3[x][4 * h] = t4.x; c3[x][4 * h + 1] = t4.y; c3[x][4 * h + 2] = t4.z; c3[x][4 * h + 3] = t4.w;
+        dc[x][4 * h] = 0.f; dc[x][4 * h + 1] = 0.f; dc[x][4 * h + 2] = 0.f; dc[x][4 * h + 3] = 0.f;
+      }
 #pragma unroll
-        for (int b = 0; b < N3; b += 4) {
-          const float4 t4 = *reinterpret_cast<const float4*>(slot + C3S + (4 * jq + e) * N3 + b);
-          g[e][b] = t4.x; g[e][b + 1] = t4.y; g[e][b + 2] = t4.z; g[e][b + 3] = t4.w;
-        }
-      float dc[RPL * N3];
+      for (int j12 = 0; j12 < JM; ++j12) {
+        if (J12T || j12 < J12) {
+          float g[N3];
 #pragma unroll
-      for (int x = 0; x < RPL; ++x) {
-        const int r = RPL * rp + x;
-        const float* c3 = slot + r * N3 + 4 * (r >> 3);   // the ring's per-8-row skew
-        float cv[N3];
-#pragma unroll
-        for (int b = 0; b < N3; b += 4) {
-          const float4 t4 = *reinterpret_cast<const float4*>(c3 + b);
-          cv[b] = t4.x; cv[b + 1] = t4.y; cv[b + 2] = t4.z; cv[b + 3] = t4.w;
-        }
-#pragma unroll
-        for (int b = 0; b < N3; ++b) dc[x * N3 + b] = 0.f;
-#pragma unroll
-        for (int e = 0; e < 4; ++e)
-#pragma unroll
-          for (int b = 0; b < N3; ++b) {
-            dp[e][x] = fmaf(g[e][b], cv[b], dp[e][x]);
-            dc[x * N3 + b] = fmaf(pr[e][x], g[e][b], dc[x * N3 + b]);
+          for (int h = 0; h < H4; ++h) {   // broadcast read of G_u[j12][4h .. 4h + 3]
+            const float4 t4 = *reinterpret_cast<const float4*>(slot + C3S + j12 * N3 + 4 * h);
+            g[4 * h] = t4.x; g[4 * h + 1] = t4.y; g[4 * h + 2] = t4.z; g[4 * h + 3] = t4.w;
           }
+#pragma unroll
+          for (int x = 0; x < RL; ++x)
+#pragma unroll
+            for (int b = 0; b < N3; ++b) {
+              dp[j12][x] = fmaf(g[b], c3[x][b], dp[j12][x]);
+              dc[x][b] = fmaf(pr[j12][x], g[b], dc[x][b]);
+            }
+        }
       }
       __syncwarp();
       if (j + RW_NSL - 1 < nr) issue(j + RW_NSL - 1);
       tc::cp_commit();
-      // dC3: reduce over jq (lane bits 4, 3); lane keeps r = RPL rp + (RPL / 4) jq + {0 .. RPL/4 - 1}, all j3
+      // dC3[i3_u][rl + x][0 .. n3): RL n3 consecutive floats per lane
+      float* d3 = a.grads + __shfl_sync(0xffffffffu, o3l, j) + (size_t)(RL * lane) * N3;
 #pragma unroll
-      for (int lv = 0; lv < 2; ++lv) {
-        const int mask = 16 >> lv, half = (RPL * N3) >> (lv + 1);
-        const bool hi = (lane & mask) != 0;
+      for (int x = 0; x < RL; ++x)
 #pragma unroll
-        for (int i = 0; i < half; ++i) {
-          const float snd = hi ? dc[i] : dc[i + half];
-          const float kp = hi ? dc[i + half] : dc[i];
-          dc[i] = kp + __shfl_xor_sync(0xffffffffu, snd, mask);
-        }
-      }
-      const unsigned long long o3 = __shfl_sync(0xffffffffu, o3l, j);
-      float* d3 = a.grads + o3 + (size_t)(RPL * rp + (RPL / 4) * jq) * N3;
-#pragma unroll
-      for (int i = 0; i < (RPL / 4) * N3; i += 4) red_v4(d3 + i, make_float4(dc[i], dc[i + 1], dc[i + 2], dc[i + 3]));
+        for (int b = 0; b < N3; b += 4) red_v4(d3 + x * N3 + b, make_float4(dc[x][b], dc[x][b + 1], dc[x][b + 2], dc[x][b + 3]));
     }
     if (curq != 0xffffffffu) flush();
     tc::cp_wait<0>();
@@ -693,7 +698,29 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 2) k_rows_bwd2(RowBwdArgs a) {
   }
 }
 
-size_t rows_bwd_smem(int n3, int sw) { return (size_t)RW_WARPS * RW_NSL * (sw * n3 + sw / 2 + 16 * n3) * 4; }   // per sw-wide r slice
+size_t rows_bwd_smem(int n3, int sw) { return (size_t)RW_WARPS * RW_NSL * (sw * n3 + RB_J12 * n3) * 4; }   // per sw-wide r slice
+
+// (n3, R, n1 n2) -> k_rows_bwd2 instantiation (n1 n2 = 16 unrolled exactly, others predicated)
+template <int N3, int RL, int KR> const void* rows_bwd_pick(int j12) {
+  return j12 == 16 ? (const void*)k_rows_bwd2<N3, RL, KR, 16> : (const void*)k_rows_bwd2<N3, RL, KR, 0>;
+}
+const void* rows_bwd_kernel(int n3, int R, int j12) {
+  if (n3 == 4) {
+    if (R == 32) return rows_bwd_pick<4, 1, 32>(j12);
+    if (R == 64) return rows_bwd_pick<4, 2, 64>(j12);
+    if (R == 128) return rows_bwd_pick<4, 2, 128>(j12);
+  } else if (n3 == 8) {
+    if (R == 32) return rows_bwd_pick<8, 1, 32>(j12);
+    if (R == 64) return rows_bwd_pick<8, 2, 64>(j12);
+    if (R == 128) return rows_bwd_pick<8, 2, 128>(j12);
+  }
+  return nullptr;
+}
+template <class F> void for_rows_bwd(F&& f) {
+  for (int n3 : {4, 8})
+    for (int R : {32, 64, 128})
+      for (int j12 : {16, 4}) f(rows_bwd_kernel(n3, R, j12), n3, R == 32 ? 32 : 64);
+}
 
 }  // namespace
 
@@ -721,10 +748,7 @@ cudaError_t configure_fused(Ctx& c) {
   set((const void*)k_rows_fwd2<8, 4>, rows_smem(8, 32));
   set((const void*)k_rows_fwd2<4, 16>, rows_smem(4, 128));
   set((const void*)k_rows_fwd2<8, 16>, rows_smem(8, 128));
-  set((const void*)k_rows_bwd2<4, 4>, rows_bwd_smem(4, 32));
-  set((const void*)k_rows_bwd2<8, 4>, rows_bwd_smem(8, 32));
-  set((const void*)k_rows_bwd2<4, 8>, rows_bwd_smem(4, 64));
-  set((const void*)k_rows_bwd2<8, 8>, rows_bwd_smem(8, 64));
+  for_rows_bwd([&](const void* f, int n3, int sw) { set(f, rows_bwd_smem(n3, sw)); });
   return e;
 }
 
@@ -777,8 +801,8 @@ cudaError_t run_fused_fwd(Ctx& c, float* out, cudaStream_t s) {
   {
     StageScope sc(c, ST_FWD_ROWS, s);
     RowArgs r;
-    r.cores = c.cores; r.meta = c.d_meta; r.counts = p.counts; r.row_pfx = p.row_pfx; r.row_i3 = p.row_i3;
-    r.pfx_t = p.pfx_t; r.pbuf = p.pbuf; r.rows = p.rows; r.seg_off = p.seg_off; r.sbag = p.sbag; r.out = out;
+    r.cores = c.cores; r.meta = c.d_meta; r.counts = p.counts; r.row_pfx = p.row_pfx; r.row_c3 = p.row_c3;
+    r.c3_begin = c.c3_begin; r.pfx_t = p.pfx_t; r.pbuf = p.pbuf; r.rows = p.rows; r.seg_off = p.seg_off; r.sbag = p.sbag; r.out = out;
     r.n1 = c.n1; r.n1s = a.n1s; r.n2 = c.n2; r.N = c.N; r.NC = c.NC;
     const int grid = grid_for(c, cdiv(c.U_cap, RW_RCH), RW_WARPS, 4);
     if (c.R == 32) {
@@ -802,7 +826,7 @@ cudaError_t run_dp_zero(Ctx& c, cudaStream_t s) {
   const PlanDev& p = c.p;
   RowBwdArgs r;
   r.cores = c.cores; r.grads = c.grads; r.meta = c.d_meta; r.counts = p.counts; r.row_pfx = p.row_pfx;
-  r.row_i3 = p.row_i3; r.pfx_t = p.pfx_t; r.row_seg = p.row_seg; r.pbuf = p.pbuf; r.gbuf = p.gbuf;
+  r.row_c3 = p.row_c3; r.c3_begin = c.c3_begin; r.pfx_t = p.pfx_t; r.row_seg = p.row_seg; r.pbuf = p.pbuf; r.gbuf = p.gbuf;
   r.dpbuf = p.dpbuf; r.n1 = c.n1; r.n2 = c.n2; r.N = c.N; r.NC = c.NC; r.R = c.R;
   k_dp_zero2<<<grid_for(c, c.P_cap, 8, 8), 256, 0, s>>>(r);
   return cudaGetLastError();
@@ -812,18 +836,15 @@ cudaError_t run_rows_bwd2(Ctx& c, cudaStream_t s) {
   const PlanDev& p = c.p;
   RowBwdArgs r;
   r.cores = c.cores; r.grads = c.grads; r.meta = c.d_meta; r.counts = p.counts; r.row_pfx = p.row_pfx;
-  r.row_i3 = p.row_i3; r.pfx_t = p.pfx_t; r.row_seg = p.row_seg; r.pbuf = p.pbuf; r.gbuf = p.gbuf;
+  r.row_c3 = p.row_c3; r.c3_begin = c.c3_begin; r.pfx_t = p.pfx_t; r.row_seg = p.row_seg; r.pbuf = p.pbuf; r.gbuf = p.gbuf;
   r.dpbuf = p.dpbuf; r.n1 = c.n1; r.n2 = c.n2; r.N = c.N; r.NC = c.NC; r.R = c.R;
   // (the dP rows of chunk-straddling prefixes were zeroed at the end of the index stage)
-  const int grid = grid_for(c, cdiv(c.U_cap, RW_RCH) * std::max(1, c.R / XR), RW_WARPS, 2);
-  if (c.R == 32) {
-    if (c.n3 == 4) k_rows_bwd2<4, 4><<<grid, RW_WARPS * 32, rows_bwd_smem(4, 32), s>>>(r);
-    else k_rows_bwd2<8, 4><<<grid, RW_WARPS * 32, rows_bwd_smem(8, 32), s>>>(r);
-  } else {
-    if (c.n3 == 4) k_rows_bwd2<4, 8><<<grid, RW_WARPS * 32, rows_bwd_smem(4, 64), s>>>(r);
-    else k_rows_bwd2<8, 8><<<grid, RW_WARPS * 32, rows_bwd_smem(8, 64), s>>>(r);
-  }
-  return cudaGetLastError();
+  const int sw = c.R == 32 ? 32 : 64;
+  const int grid = grid_for(c, cdiv(c.U_cap, RW_RCH) * (c.R / sw), RW_WARPS, 2);
+  const void* f = rows_bwd_kernel(c.n3, c.R, c.n1 * c.n2);
+  if (!f) return cudaErrorInvalidValue;
+  void* args[] = {&r};
+  return cudaLaunchKernel(f, dim3(grid), dim3(RW_WARPS * 32), args, rows_bwd_smem(c.n3, sw), s);
 }
 
 // Forward contractions on tcgen05: P (k_prefix_fwd) then rows (k_rows_fwd2).

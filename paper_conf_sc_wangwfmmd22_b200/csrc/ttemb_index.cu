@@ -357,6 +357,8 @@ struct PlanScanArgs {
   uint32_t *ukey, *seg_off, *inverse, *sbag, *counts;
   uint32_t *row_pfx, *row_i3, *pfx_t, *pfx_i1, *pfx_i2, *row_seg;
   uint32_t *grp_pfx, *grp_off, *grp_t, *grp_i2;
+  uint32_t* row_c3;                 // [U] C3 slice index of the row (row kernels: one load per row)
+  uint64_t c3_begin, s3;            // C3 region start, floats per C3 slice (R n3)
   uint32_t nnz, every_row, every_pfx;
   uint64_t tt_keys;
 };
@@ -460,6 +462,7 @@ __global__ void __launch_bounds__(SC_T) k_plan_scan(PlanScanArgs a, uint32_t* st
       if (ki[k].dense) {
         a.row_pfx[u] = 0xFFFFFFFFu;
         a.row_i3[u] = 0;
+        a.row_c3[u] = 0;
         if (i == 0 || a.skey[i - 1] < a.tt_keys) {   // first dense row: TT rows / prefixes end here
           a.counts[kCntUtt1] = u + 1;
           a.row_seg[q + 1] = u;
@@ -467,6 +470,7 @@ __global__ void __launch_bounds__(SC_T) k_plan_scan(PlanScanArgs a, uint32_t* st
       } else {
         a.row_pfx[u] = q;
         a.row_i3[u] = ki[k].i3;
+        a.row_c3[u] = (uint32_t)((a.meta[ki[k].t].c3_off - a.c3_begin) / a.s3) + ki[k].i3;
       }
     }
     if ((bal[1][k] >> lane) & 1u) {
@@ -563,6 +567,7 @@ cudaError_t run_index_stage(Ctx& c, const void* indices, const int64_t* offsets,
     a.every_row = (c.flags & TTEMB_NO_AGGREGATION) ? 1u : 0u;
     a.every_pfx = (c.flags & TTEMB_NO_PREFIX_REUSE) ? 1u : 0u;
     a.tt_keys = c.tt_keys;
+    a.row_c3 = p.row_c3; a.c3_begin = c.c3_begin; a.s3 = (uint64_t)c.R * c.n3;
     const int64_t tiles = std::max<int64_t>(1, scan_tiles(nnz));
     k_plan_scan<<<(unsigned)tiles, SC_T, 0, s>>>(a, p.sc_status, p.sc_counter + 0);
   }

@@ -91,6 +91,7 @@ struct PlanDev {
   uint32_t *skey, *spos;                       // -> final sort-1 buffers
   uint32_t *bag_of, *sbag, *inverse;           // [nnz]
   uint32_t *ukey, *seg_off, *row_pfx, *row_i3; // [U]
+  uint32_t* row_c3;                            // [U] C3 slice of the row: (C3 float offset - c3_begin) / (R n3)
   uint32_t *pfx_t, *pfx_i1, *pfx_i2, *row_seg; // [P]
   uint32_t *gkeyA, *gvalA, *gkeyB, *gvalB;     // group sort ping-pong [P]
   uint32_t *gkey, *gval;                       // -> final sort-2 buffers

@@ -90,7 +90,7 @@ __global__ void probe(int M, int N, int K, int la, int lb, int swap, int var, co
   stage(Ahi, Alo, A, M, K, la, var);
   stage(Bhi, Blo, B, N, K, lb, var);
   if (threadIdx.x == 0) { tc::mbar_init(&mbar, 1); tc::fence_mbar_init(); }
-  if (threadIdx.x < 32) tc::tmem_alloc(&tmem_base, 256);
+  if (threadIdx.x < 32) tc::tmem_alloc(&tmem_base, 512);
   tc::fence_async_smem();
   tc::fence_before();
   __syncthreads();
@@ -127,7 +127,7 @@ __global__ void probe(int M, int N, int K, int la, int lb, int swap, int var, co
   }
   tc::fence_before();
   __syncthreads();
-  if (threadIdx.x < 32) tc::tmem_dealloc(tb, 256);
+  if (threadIdx.x < 32) tc::tmem_dealloc(tb, 512);
 }
 
 static double run_case(int M, int N, int K, int la, int lb, int swap, int var, bool* err) {
@@ -159,7 +159,7 @@ static double run_case(int M, int N, int K, int la, int lb, int swap, int var, b
 }
 
 // ---- throughput: reps x (K=64: 8 k-steps x 3 MMAs), one CTA ----
-__global__ void mma_timing(int M, int N, int la, int lb, int reps, long long* cycles) {
+__global__ void mma_timing(int M, int N, int la, int lb, int reps, long long* cycles, int nd = 1) {
   extern __shared__ __align__(1024) char smraw[];
   float* sm = reinterpret_cast<float*>(smraw);
   __shared__ uint64_t mbar;
@@ -167,7 +167,7 @@ __global__ void mma_timing(int M, int N, int la, int lb, int reps, long long* cy
   const int K = 64;
   for (int i = threadIdx.x; i < 2 * (M + N) * K; i += blockDim.x) sm[i] = 0.001f * (i % 97);
   if (threadIdx.x == 0) { tc::mbar_init(&mbar, 1); tc::fence_mbar_init(); }
-  if (threadIdx.x < 32) tc::tmem_alloc(&tmem_base, 256);
+  if (threadIdx.x < 32) tc::tmem_alloc(&tmem_base, 512);
   tc::fence_async_smem();
   tc::fence_before();
   __syncthreads();
@@ -184,9 +184,11 @@ __global__ void mma_timing(int M, int N, int la, int lb, int reps, long long* cy
       for (int kk = 0; kk < 8; ++kk) {
         const uint64_t dah = mkdesc(ah + koff(da, kk), da), dal = mkdesc(al + koff(da, kk), da);
         const uint64_t dbh = mkdesc(bh + koff(db, kk), db), dbl = mkdesc(bl + koff(db, kk), db);
-        tc::mma_tf32(tb, dah, dbh, id, (rep > 0 || kk > 0) ? 1u : 0u);
-        tc::mma_tf32(tb, dah, dbl, id, 1u);
-        tc::mma_tf32(tb, dal, dbh, id, 1u);
+        // nd independent accumulators: the 3 split MMAs of K step kk go to D[(kk % nd)]
+        const uint32_t td = tb + (uint32_t)((kk % nd) * N);
+        tc::mma_tf32(td, dah, dbh, id, (rep > 0 || kk >= nd) ? 1u : 0u);
+        tc::mma_tf32(td, dah, dbl, id, 1u);
+        tc::mma_tf32(td, dal, dbh, id, 1u);
       }
     }
     t1 = clock64();
@@ -196,7 +198,27 @@ __global__ void mma_timing(int M, int N, int la, int lb, int reps, long long* cy
   if (threadIdx.x == 0) { cycles[0] = t1 - t0; cycles[1] = clock64() - t0; }
   tc::fence_before();
   __syncthreads();
-  if (threadIdx.x < 32) tc::tmem_dealloc(tb, 256);
+  if (threadIdx.x < 32) tc::tmem_dealloc(tb, 512);
+}
+
+static int timing_nd() {
+  long long* d;
+  cudaMalloc(&d, 16);
+  const int smem = 2 * (128 + 256) * 64 * 4;
+  cudaFuncSetAttribute(mma_timing, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  for (int N : {16, 32, 64, 128})
+    for (int nd : {1, 2, 4, 8}) {
+      if (nd * N > 512) continue;
+      const int reps = 40;
+      mma_timing<<<1, 128, smem>>>(128, N, KSW128, KSW128, reps, d, nd);
+      cudaError_t e = cudaDeviceSynchronize();
+      long long h[2];
+      cudaMemcpy(h, d, 16, cudaMemcpyDeviceToHost);
+      const double n = reps * 24.0;
+      printf("M=128 N=%3d, %d independent accumulators: issue %5.1f cyc/MMA, complete %6.1f cyc/MMA (%6.0f MAC/cyc) %s\n", N, nd,
+             h[0] / n, h[1] / n, 128.0 * N * 8 / (h[1] / n), e == cudaSuccess ? "" : cudaGetErrorString(e));
+    }
+  return 0;
 }
 
 static int timing_main() {
@@ -227,6 +249,7 @@ static int timing_main() {
 }
 
 int main(int argc, char** argv) {
+  if (argc > 1 && argv[1][0] == 'n') return timing_nd();
   if (argc > 1) return timing_main();
   struct Case { int M, N, K, la, lb; };
   const Case cases[] = {
