@@ -20,6 +20,7 @@
 #include <stdlib.h>
 
 #include <algorithm>
+#include <type_traits>
 #include <vector>
 
 #include "tc.cuh"
@@ -373,6 +374,15 @@ template <int KR> constexpr size_t prefix_smem() { return 128 + X_RAW_BYTES + 2 
 // partial sums are reduced over rp by recursive halving (3 shuffle levels) and each lane
 // stores n3/2 consecutive outputs.
 // ------------------------------------------------------------------------------------
+// Packed fp32 pairs on sm_100 (FFMA2): d = a * b + c lane by lane, each an ordinary
+// round-to-nearest fp32 fma; ptxas folds a {s, s} pair into a scalar operand.
+__device__ __forceinline__ void ffma2(float2& d, float2 a, float2 b) {
+  asm("fma.rn.f32x2 %0, %1, %2, %0;"
+      : "+l"(*reinterpret_cast<unsigned long long*>(&d))
+      : "l"(*reinterpret_cast<unsigned long long*>(&a)), "l"(*reinterpret_cast<unsigned long long*>(&b)));
+}
+__device__ __forceinline__ void ffma2s(float2& d, float s, float2 b) { ffma2(d, make_float2(s, s), b); }
+
 constexpr int RW_WARPS = 8, RW_RCH = 16, RW_NSL = 3;
 
 struct RowArgs {
@@ -449,25 +459,28 @@ __global__ void __launch_bounds__(RW_WARPS * 32, RPL == 8 ? 3 : 2) k_rows_fwd2(R
       }
       tc::cp_wait<RW_NSL - 2>();
       __syncwarp();
-      float acc[4 * N3];
+      float2 acc2[2 * N3];   // (E[j12][b], E[j12][b + 1]) partial pairs: packed FFMA2, P scalar
 #pragma unroll
-      for (int i = 0; i < 4 * N3; ++i) acc[i] = 0.f;
+      for (int i = 0; i < 2 * N3; ++i) acc2[i] = make_float2(0.f, 0.f);
       const float* slot3 = ringp + (j % RW_NSL) * SLOT;
 #pragma unroll
       for (int x = 0; x < RPL; ++x) {
         const int r = RPL * rp + x;
         const float* c3 = slot3 + r * N3 + 4 * (r >> 3);   // the ring's per-8-row skew
-        float cv[N3];
+        float2 cv[N3 / 2];
 #pragma unroll
         for (int b = 0; b < N3; b += 4) {
           const float4 t4 = *reinterpret_cast<const float4*>(c3 + b);
-          cv[b] = t4.x; cv[b + 1] = t4.y; cv[b + 2] = t4.z; cv[b + 3] = t4.w;
+          cv[b / 2] = make_float2(t4.x, t4.y); cv[b / 2 + 1] = make_float2(t4.z, t4.w);
         }
 #pragma unroll
         for (int e = 0; e < 4; ++e)
 #pragma unroll
-          for (int b = 0; b < N3; ++b) acc[e * N3 + b] = fmaf(pr[e][x], cv[b], acc[e * N3 + b]);
+          for (int b2 = 0; b2 < N3 / 2; ++b2) ffma2s(acc2[e * (N3 / 2) + b2], pr[e][x], cv[b2]);
       }
+      float acc[4 * N3];
+#pragma unroll
+      for (int i = 0; i < 2 * N3; ++i) { acc[2 * i] = acc2[i].x; acc[2 * i + 1] = acc2[i].y; }
       __syncwarp();
       if (j + RW_NSL - 1 < nr) issue(j + RW_NSL - 1);
       tc::cp_commit();
@@ -521,6 +534,7 @@ struct RowBwdArgs {
   const float* gbuf;          // [U][N]
   float* dpbuf;               // [P][n1][NC]
   int n1, n2, N, NC, R;
+  int exp;                    // TTEMB_EXP bits (timing experiments only; results invalid)
 };
 
 __global__ void __launch_bounds__(256) k_dp_zero2(RowBwdArgs a) {
@@ -545,11 +559,12 @@ __device__ __forceinline__ void red_v2(float* addr, float x, float y) {
 
 constexpr int RB_J12 = 16;   // n1 n2 <= 16
 
+
 // P_q[j12][r] sits at pbuf[(q J12 + j12) R + r] (NC = n2 R), so with R a template constant every
 // per-j12 access is an immediate offset from one base pointer.
 template <int N3, int RL, int KR, int J12T>   // RL = r per lane: 1 (R = 32) or 2 (R = 64, 128 in two
                                               // slices); J12T = n1 n2 (0: runtime, <= 16)
-__global__ void __launch_bounds__(RW_WARPS * 32, 2) k_rows_bwd2(RowBwdArgs a) {
+__global__ void __launch_bounds__(RW_WARPS * 32, RL == 1 ? 3 : 2) k_rows_bwd2(RowBwdArgs a) {
   constexpr int SW = 32 * RL;                   // r width of a work item (a slice of R)
   constexpr int NSL = KR / SW;                  // slices per row
   constexpr int C3S = SW * N3;                  // C3 part of a slot
@@ -590,6 +605,7 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 2) k_rows_bwd2(RowBwdArgs a) {
     // slot layout: C3 piece (x, h) of lane l at [(x H4 + h) 32 + l] (16 bytes each: the warp's
     // cp.async stores and a lane's loads are contiguous / conflict-free), then G_u
     auto issue = [&](int j) {
+      if (a.exp & 512) return;
       const unsigned long long o3 = __shfl_sync(0xffffffffu, o3l, j) + (unsigned long long)(RL * lane) * N3;
       const float4* src = reinterpret_cast<const float4*>(a.cores + o3);
       const uint32_t dst = ring + (uint32_t)((j % RW_NSL) * SLOT * 4) + 16u * lane;
@@ -605,20 +621,23 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 2) k_rows_bwd2(RowBwdArgs a) {
       tc::cp_commit();
     }
     uint32_t curq = 0xffffffffu;
-    float pr[JM][RL], dp[JM][RL];
+    // lane's P_q[j12][rl .. rl + RL) and dP accumulators: one fp32 (RL = 1) or a packed pair
+    using PV = typename std::conditional<RL == 2, float2, float>::type;
+    PV pr[JM], dp[JM];
     auto flush = [&]() {
+      if (a.exp & 128) return;
       const bool red = curq == prevq || curq == nextq;
       float* d = a.dpbuf + (size_t)curq * J12 * KR + rl;
 #pragma unroll
       for (int j12 = 0; j12 < JM; ++j12) {
         if (!J12T && j12 >= J12) break;
         float* e = d + j12 * KR;
-        if (RL == 2) {
-          if (red) red_v2(e, dp[j12][0], dp[j12][RL - 1]);
-          else *reinterpret_cast<float2*>(e) = make_float2(dp[j12][0], dp[j12][RL - 1]);
+        if constexpr (RL == 2) {
+          if (red) red_v2(e, dp[j12].x, dp[j12].y);
+          else *reinterpret_cast<float2*>(e) = dp[j12];
         } else {
-          if (red) atomicAdd(e, dp[j12][0]);
-          else *e = dp[j12][0];
+          if (red) atomicAdd(e, dp[j12]);
+          else *e = dp[j12];
         }
       }
     };
@@ -637,49 +656,59 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 2) k_rows_bwd2(RowBwdArgs a) {
         const float* pq = a.pbuf + (size_t)q * J12 * KR + rl;
 #pragma unroll
         for (int j12 = 0; j12 < JM; ++j12) {
-          if (J12T || j12 < J12) {
-            if (RL == 2) {
-              const float2 x0 = __ldg(reinterpret_cast<const float2*>(pq + j12 * KR));
-              pr[j12][0] = x0.x; pr[j12][RL - 1] = x0.y;
-            } else {
-              pr[j12][0] = __ldg(pq + j12 * KR);
-            }
+          if constexpr (RL == 2) {
+            pr[j12] = ((J12T || j12 < J12) && !(a.exp & 256)) ? __ldg(reinterpret_cast<const float2*>(pq + j12 * KR)) : make_float2(0.f, 0.f);
+            dp[j12] = make_float2(0.f, 0.f);
           } else {
-#pragma unroll
-            for (int x = 0; x < RL; ++x) pr[j12][x] = 0.f;
+            pr[j12] = (J12T || j12 < J12) ? __ldg(pq + j12 * KR) : 0.f;
+            dp[j12] = 0.f;
           }
-#pragma unroll
-          for (int x = 0; x < RL; ++x) dp[j12][x] = 0.f;
         }
         curq = q;
       }
       tc::cp_wait<RW_NSL - 2>();
       __syncwarp();
       const float* slot = ringp + (j % RW_NSL) * SLOT;
-      float c3[RL][N3], dc[RL][N3];
+      // C3[rl + x][b] for the lane's r; c3x[b] = (C3[rl][b], C3[rl + 1][b]) pairs the lane's two r
+      float c3[RL][N3];
+      float2 dc[RL][N3 / 2];
 #pragma unroll
       for (int i = 0; i < C3L; ++i) {   // piece i = (x, h): r = rl + x, j3 = 4h .. 4h + 3
         const int x = i / H4, h = i - x * H4;
         const float4 t4 = *reinterpret_cast<const float4*>(slot + 4 * (i * 32 + lane));
         c3[x][4 * h] = t4.x; c3[x][4 * h + 1] = t4.y; c3[x][4 * h + 2] = t4.z; c3[x][4 * h + 3] = t4.w;
-        dc[x][4 * h] = 0.f; dc[x][4 * h + 1] = 0.f; dc[x][4 * h + 2] = 0.f; dc[x][4 * h + 3] = 0.f;
+        dc[x][2 * h] = make_float2(0.f, 0.f); dc[x][2 * h + 1] = make_float2(0.f, 0.f);
       }
 #pragma unroll
       for (int j12 = 0; j12 < JM; ++j12) {
         if (J12T || j12 < J12) {
-          float g[N3];
+          float2 g[N3 / 2];
 #pragma unroll
           for (int h = 0; h < H4; ++h) {   // broadcast read of G_u[j12][4h .. 4h + 3]
             const float4 t4 = *reinterpret_cast<const float4*>(slot + C3S + j12 * N3 + 4 * h);
-            g[4 * h] = t4.x; g[4 * h + 1] = t4.y; g[4 * h + 2] = t4.z; g[4 * h + 3] = t4.w;
+            g[2 * h] = make_float2(t4.x, t4.y); g[2 * h + 1] = make_float2(t4.z, t4.w);
+          }
+          // dP: scalar FFMA (a packed form would need (C3[rl][b], C3[rl + 1][b]) pairs, which cost
+          // more register moves than they save); dC3: packed pairs (FFMA2) of G[j12][b], G[j12][b + 1]
+#pragma unroll
+          for (int b = 0; b < N3; ++b) {   // dP[j12][rl + x] += G[j12][b] C3[rl + x][b]
+            const float gb = (b & 1) ? g[b >> 1].y : g[b >> 1].x;
+            if constexpr (RL == 2) {
+              dp[j12].x = fmaf(gb, c3[0][b], dp[j12].x);
+              dp[j12].y = fmaf(gb, c3[1][b], dp[j12].y);
+            } else {
+              dp[j12] = fmaf(gb, c3[0][b], dp[j12]);
+            }
           }
 #pragma unroll
-          for (int x = 0; x < RL; ++x)
-#pragma unroll
-            for (int b = 0; b < N3; ++b) {
-              dp[j12][x] = fmaf(g[b], c3[x][b], dp[j12][x]);
-              dc[x][b] = fmaf(pr[j12][x], g[b], dc[x][b]);
+          for (int b2 = 0; b2 < N3 / 2; ++b2) {   // dC3[rl + x][2 b2 .. 2 b2 + 1] += P[j12][rl + x] G[j12][2 b2 ..]
+            if constexpr (RL == 2) {
+              ffma2s(dc[0][b2], pr[j12].x, g[b2]);
+              ffma2s(dc[1][b2], pr[j12].y, g[b2]);
+            } else {
+              ffma2s(dc[0][b2], pr[j12], g[b2]);
             }
+          }
         }
       }
       __syncwarp();
@@ -687,10 +716,12 @@ __global__ void __launch_bounds__(RW_WARPS * 32, 2) k_rows_bwd2(RowBwdArgs a) {
       tc::cp_commit();
       // dC3[i3_u][rl + x][0 .. n3): RL n3 consecutive floats per lane
       float* d3 = a.grads + __shfl_sync(0xffffffffu, o3l, j) + (size_t)(RL * lane) * N3;
+      if (!(a.exp & 64))
 #pragma unroll
       for (int x = 0; x < RL; ++x)
 #pragma unroll
-        for (int b = 0; b < N3; b += 4) red_v4(d3 + x * N3 + b, make_float4(dc[x][b], dc[x][b + 1], dc[x][b + 2], dc[x][b + 3]));
+        for (int b2 = 0; b2 < N3 / 2; b2 += 2)
+          red_v4(d3 + x * N3 + 2 * b2, make_float4(dc[x][b2].x, dc[x][b2].y, dc[x][b2 + 1].x, dc[x][b2 + 1].y));
     }
     if (curq != 0xffffffffu) flush();
     tc::cp_wait<0>();
@@ -716,7 +747,22 @@ const void* rows_bwd_kernel(int n3, int R, int j12) {
   }
   return nullptr;
 }
+const void* rows_bwd_kernel_rl1(int n3, int R, int j12) {
+  if (n3 == 4) {
+    if (R == 32) return rows_bwd_pick<4, 1, 32>(j12);
+    if (R == 64) return rows_bwd_pick<4, 1, 64>(j12);
+    if (R == 128) return rows_bwd_pick<4, 1, 128>(j12);
+  } else if (n3 == 8) {
+    if (R == 32) return rows_bwd_pick<8, 1, 32>(j12);
+    if (R == 64) return rows_bwd_pick<8, 1, 64>(j12);
+    if (R == 128) return rows_bwd_pick<8, 1, 128>(j12);
+  }
+  return nullptr;
+}
 template <class F> void for_rows_bwd(F&& f) {
+  for (int n3 : {4, 8})
+    for (int R : {32, 64, 128})
+      for (int j12 : {16, 4}) f(rows_bwd_kernel_rl1(n3, R, j12), n3, 32);
   for (int n3 : {4, 8})
     for (int R : {32, 64, 128})
       for (int j12 : {16, 4}) f(rows_bwd_kernel(n3, R, j12), n3, R == 32 ? 32 : 64);
@@ -838,10 +884,14 @@ cudaError_t run_rows_bwd2(Ctx& c, cudaStream_t s) {
   r.cores = c.cores; r.grads = c.grads; r.meta = c.d_meta; r.counts = p.counts; r.row_pfx = p.row_pfx;
   r.row_c3 = p.row_c3; r.c3_begin = c.c3_begin; r.pfx_t = p.pfx_t; r.row_seg = p.row_seg; r.pbuf = p.pbuf; r.gbuf = p.gbuf;
   r.dpbuf = p.dpbuf; r.n1 = c.n1; r.n2 = c.n2; r.N = c.N; r.NC = c.NC; r.R = c.R;
+  r.exp = exp_bits();
   // (the dP rows of chunk-straddling prefixes were zeroed at the end of the index stage)
-  const int sw = c.R == 32 ? 32 : 64;
-  const int grid = grid_for(c, cdiv(c.U_cap, RW_RCH) * (c.R / sw), RW_WARPS, 2);
-  const void* f = rows_bwd_kernel(c.n3, c.R, c.n1 * c.n2);
+  // 32-wide r slices (RL = 1, 24 warps / SM) by default: at c4 88 us vs 98.7 us for 64-wide
+  // slices (RL = 2, 16 warps / SM; TTEMB_EXP bit 2048 selects them for comparison)
+  const bool narrow = c.R == 32 || !(exp_bits() & 2048);
+  const int sw = narrow ? 32 : 64;
+  const int grid = grid_for(c, cdiv(c.U_cap, RW_RCH) * (c.R / sw), RW_WARPS, narrow ? 3 : 2);
+  const void* f = narrow ? rows_bwd_kernel_rl1(c.n3, c.R, c.n1 * c.n2) : rows_bwd_kernel(c.n3, c.R, c.n1 * c.n2);
   if (!f) return cudaErrorInvalidValue;
   void* args[] = {&r};
   return cudaLaunchKernel(f, dim3(grid), dim3(RW_WARPS * 32), args, rows_bwd_smem(c.n3, sw), s);
