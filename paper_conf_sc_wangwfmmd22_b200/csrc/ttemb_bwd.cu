@@ -21,6 +21,7 @@ namespace ttemb {
 namespace {
 
 constexpr int AGG_CS = 32;   // sorted positions per aggregation chunk
+constexpr int AGG_B = 8;     // grad_out rows per lane group loaded ahead in k_agg_scatter
 
 __device__ __forceinline__ void apply_update(float* param, float* state, float g, float lr,
                                              float eps, int opt) {
@@ -159,22 +160,35 @@ k_agg_scatter(const float* __restrict__ grad_out, const uint32_t* __restrict__ s
     }
     float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
     uint32_t cur = 0xffffffffu;
-    for (int i0 = 0; i0 < cnt; i0 += P) {
-      const int i = i0 + p;
-      const uint32_t bag = __shfl_sync(0xffffffffu, bl, i & 31);
-      const uint32_t u = __shfl_sync(0xffffffffu, ul, i & 31);
-      const float w = __shfl_sync(0xffffffffu, wl, i & 31);
-      if (i < cnt) {
-        if (u != cur) {
-          if (cur != 0xffffffffu)
-            asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(gbuf + (size_t)cur * N + 4 * f),
-                         "f"(acc.x), "f"(acc.y), "f"(acc.z), "f"(acc.w) : "memory");
-          acc = make_float4(0.f, 0.f, 0.f, 0.f);
-          cur = u;
+    // AGG_B occurrences of this lane group are loaded before any is added (AGG_B loads in flight
+    // per lane instead of one dependent load per step)
+    for (int i0 = 0; i0 < cnt; i0 += AGG_B * P) {
+      float4 v[AGG_B];
+#pragma unroll
+      for (int t = 0; t < AGG_B; ++t) {
+        const int i = i0 + t * P + p;
+        const uint32_t bag = __shfl_sync(0xffffffffu, bl, i & 31);
+        v[t] = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (i < cnt) {
+          const float4* gp = reinterpret_cast<const float4*>(grad_out + (size_t)bag * N) + f;
+          v[t] = once ? __ldcs(gp) : __ldg(gp);
         }
-        const float4* gp = reinterpret_cast<const float4*>(grad_out + (size_t)bag * N) + f;
-        const float4 v = once ? __ldcs(gp) : __ldg(gp);
-        acc.x += w * v.x; acc.y += w * v.y; acc.z += w * v.z; acc.w += w * v.w;
+      }
+#pragma unroll
+      for (int t = 0; t < AGG_B; ++t) {
+        const int i = i0 + t * P + p;
+        const uint32_t u = __shfl_sync(0xffffffffu, ul, i & 31);
+        const float w = __shfl_sync(0xffffffffu, wl, i & 31);
+        if (i < cnt) {
+          if (u != cur) {
+            if (cur != 0xffffffffu)
+              asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(gbuf + (size_t)cur * N + 4 * f),
+                           "f"(acc.x), "f"(acc.y), "f"(acc.z), "f"(acc.w) : "memory");
+            acc = make_float4(0.f, 0.f, 0.f, 0.f);
+            cur = u;
+          }
+          acc.x += w * v[t].x; acc.y += w * v[t].y; acc.z += w * v[t].z; acc.w += w * v[t].w;
+        }
       }
     }
     if (cur != 0xffffffffu)
@@ -251,6 +265,25 @@ k_update_zero(float* __restrict__ cores, float* __restrict__ state, float* __res
       apply_update(cores + e, state ? state + e : nullptr, g, lr, eps, opt);
       grads[e] = 0.f;
     }
+  }
+}
+
+// k_update_zero on float4 (both regions are multiples of 4 floats): the mostly-zero gradient is
+// streamed once and the parameters / state are read only for float4 groups that carry a gradient;
+// per element the same arithmetic as k_update_zero.
+__global__ void __launch_bounds__(256)
+k_update_zero4(float* __restrict__ cores, float* __restrict__ state, float* __restrict__ grads, size_t n1,
+               size_t begin2, size_t n2, float lr, float eps, int opt) {
+  const size_t n = (n1 + n2) / 4;
+  for (size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
+    const size_t e = 4 * i < n1 ? 4 * i : begin2 + (4 * i - n1);
+    const float4 g = *reinterpret_cast<const float4*>(grads + e);
+    if (g.x == 0.f && g.y == 0.f && g.z == 0.f && g.w == 0.f) continue;
+    const float gv[4] = {g.x, g.y, g.z, g.w};
+#pragma unroll
+    for (int k = 0; k < 4; ++k)
+      if (gv[k] != 0.f) apply_update(cores + e + k, state ? state + e + k : nullptr, gv[k], lr, eps, opt);
+    *reinterpret_cast<float4*>(grads + e) = make_float4(0.f, 0.f, 0.f, 0.f);
   }
 }
 
@@ -359,8 +392,12 @@ cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s
   }
   if (fused) {   // C2 was updated inside the group kernel; C1 and C3 densely here
     StageScope sc(c, ST_UPD_C3, s);
-    k_update_zero<<<grid_for(c, (int64_t)(c.c1_floats + c.c3_floats), 256, 32), 256, 0, s>>>(
-        c.cores, c.state, c.grads, c.c1_floats, c.c3_begin, c.c3_floats, lr, c.eps, c.opt);
+    if (c.c1_floats % 4 == 0 && c.c3_begin % 4 == 0 && c.c3_floats % 4 == 0)
+      k_update_zero4<<<grid_for(c, (int64_t)(c.c1_floats + c.c3_floats) / 4, 256, 8), 256, 0, s>>>(
+          c.cores, c.state, c.grads, c.c1_floats, c.c3_begin, c.c3_floats, lr, c.eps, c.opt);
+    else
+      k_update_zero<<<grid_for(c, (int64_t)(c.c1_floats + c.c3_floats), 256, 32), 256, 0, s>>>(
+          c.cores, c.state, c.grads, c.c1_floats, c.c3_begin, c.c3_floats, lr, c.eps, c.opt);
   }
   return cudaGetLastError();
 }
