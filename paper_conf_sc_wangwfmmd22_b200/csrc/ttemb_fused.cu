@@ -88,8 +88,9 @@ __device__ __forceinline__ float tf32_lo(float x) { return x - tc::tf32_trunc(x)
 // whole C2 slice (C2^T of both c-blocks fills TMEM columns [0, 256)); at R = 128 (K = 128) one
 // c-block's C2^T hi + lo already takes 256 columns, so a group is split into NC / 128 units and
 // the C1 rows of a tile are staged once per unit.
-template <int KR>
+template <int KR, int NC_T>   // NC_T = n2 R when fixed at compile time (immediate store offsets), else 0
 __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
+  const int NCT = NC_T ? NC_T : a.NC;
   constexpr int BPU = KR <= 64 ? 2 : 1;            // c-blocks per work unit
   constexpr uint32_t BSLOT = 2u * XT * KR * 4;    // one B slot: C1 tile hi + lo (K = KR)
   constexpr uint32_t BHALF = XT * KR * 4;
@@ -199,7 +200,7 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
           const uint32_t arow = ok ? a.grp_arow[qa + (m >> a.n1s)] + (m & ((1 << a.n1s) - 1)) : 0u;
           const float4* src = reinterpret_cast<const float4*>(a.cores + (size_t)arow * KR);
 #pragma unroll
-          for (int k = 0; k < KR / 16; ++k) bv[k] = ok ? __ldg(src + (tid >> 6) + 4 * k) : make_float4(0.f, 0.f, 0.f, 0.f);
+          for (int k = 0; k < KR / 16; ++k) bv[k] = (ok && !(a.dbg & 2)) ? __ldg(src + (tid >> 6) + 4 * k) : make_float4(0.f, 0.f, 0.f, 0.f);
         }
         XTA(0);
         if (fl & 1u) {   // the unit's C2^T -> TMEM (hi = raw fp32, lo = x - trunc_tf32(x))
@@ -292,7 +293,9 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
             const uint64_t dbh = tc::sdesc(bh + o, (XT / 8) * 128, 128);
             const uint64_t dbl = tc::sdesc(bl + o, (XT / 8) * 128, 128);
             const uint32_t ah = tm + blk * KR + kk * 8, al = tm + 128 + blk * KR + kk * 8;
+            if (a.dbg & 4) continue;
             tc::mma_tf32_ts(d, ah, dbh, id, kk > 0 ? 1u : 0u);
+            if (a.dbg & 8) continue;
             tc::mma_tf32_ts(d, ah, dbl, id, 1u);
             tc::mma_tf32_ts(d, al, dbh, id, 1u);
           }
@@ -331,11 +334,16 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
           float v[32];
           tc::tmem_ld32(tc::taddr(tm + 256 + s * 128 + blk * 64 + j0, 32 * Q, 0), v);
           const int lim = min(32, rows - j0);
-          if (c < a.NC) {
+          if (c < a.NC && !(a.dbg & 1)) {
             float* d = dst + (size_t)j0 * a.NC + c;
+            if (lim == 32) {   // full 32-row chunk: no per-element predicates / branches
 #pragma unroll
-            for (int j = 0; j < 32; ++j)
-              if (j < lim) d[(size_t)j * a.NC] = v[j];
+              for (int j = 0; j < 32; ++j) d[(size_t)j * NCT] = v[j];
+            } else {
+#pragma unroll
+              for (int j = 0; j < 32; ++j)
+                if (j < lim) d[(size_t)j * NCT] = v[j];
+            }
           }
         }
       }
@@ -785,9 +793,12 @@ cudaError_t configure_fused(Ctx& c) {
   auto set = [&](const void* f, size_t bytes) {
     if (e == cudaSuccess) e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
   };
-  set((const void*)k_prefix_fwd<32>, prefix_smem<32>());
-  set((const void*)k_prefix_fwd<64>, prefix_smem<64>());
-  set((const void*)k_prefix_fwd<128>, prefix_smem<128>());
+  set((const void*)k_prefix_fwd<32, 0>, prefix_smem<32>());
+  set((const void*)k_prefix_fwd<64, 0>, prefix_smem<64>());
+  set((const void*)k_prefix_fwd<128, 0>, prefix_smem<128>());
+  set((const void*)k_prefix_fwd<32, 128>, prefix_smem<32>());
+  set((const void*)k_prefix_fwd<64, 256>, prefix_smem<64>());
+  set((const void*)k_prefix_fwd<128, 512>, prefix_smem<128>());
   set((const void*)k_rows_fwd2<4, 8>, rows_smem(4, 64));
   set((const void*)k_rows_fwd2<8, 8>, rows_smem(8, 64));
   set((const void*)k_rows_fwd2<4, 4>, rows_smem(4, 32));
@@ -819,9 +830,17 @@ cudaError_t run_fused_fwd(Ctx& c, float* out, cudaStream_t s) {
       cudaMemsetAsync(trace, 0, sizeof(unsigned long long) * 32 * grid, s);
       a.trace = trace;
     }
-    if (c.R == 32) k_prefix_fwd<32><<<grid, X_THREADS, prefix_smem<32>(), s>>>(a);
-    else if (c.R == 64) k_prefix_fwd<64><<<grid, X_THREADS, prefix_smem<64>(), s>>>(a);
-    else k_prefix_fwd<128><<<grid, X_THREADS, prefix_smem<128>(), s>>>(a);
+    const bool n2_4 = c.n2 == 4;   // the c4 / c5 shapes: NC = 4 R as a compile-time constant
+    if (c.R == 32) {
+      if (n2_4) k_prefix_fwd<32, 128><<<grid, X_THREADS, prefix_smem<32>(), s>>>(a);
+      else k_prefix_fwd<32, 0><<<grid, X_THREADS, prefix_smem<32>(), s>>>(a);
+    } else if (c.R == 64) {
+      if (n2_4) k_prefix_fwd<64, 256><<<grid, X_THREADS, prefix_smem<64>(), s>>>(a);
+      else k_prefix_fwd<64, 0><<<grid, X_THREADS, prefix_smem<64>(), s>>>(a);
+    } else {
+      if (n2_4) k_prefix_fwd<128, 512><<<grid, X_THREADS, prefix_smem<128>(), s>>>(a);
+      else k_prefix_fwd<128, 0><<<grid, X_THREADS, prefix_smem<128>(), s>>>(a);
+    }
     if (a.trace) {
       std::vector<unsigned long long> hb(32 * grid);
       cudaMemcpyAsync(hb.data(), trace, hb.size() * 8, cudaMemcpyDeviceToHost, s);
