@@ -392,6 +392,7 @@ def main():
     ap.add_argument("--lr", type=float, default=0.01)
     ap.add_argument("--seed", type=int, default=0)
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--e2e-depth", type=int, default=2, help="HostStepPipeline staging slots for the e2e leg")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--stages", action="store_true", help="print per-stage times to stderr")
     ap.add_argument("--fp32-cores", action="store_true", help="force the FFMA contraction path (no tcgen05)")
@@ -651,12 +652,13 @@ def main():
     if not args.no_e2e and world == 1:
         hpool = [(torch.as_tensor(i).pin_memory(), torch.as_tensor(o).pin_memory(),
                   torch.as_tensor(g).pin_memory()) for i, o, g in pool]
-        houts = [torch.empty(B, cfg.num_tables, cfg.dim).pin_memory() for _ in range(2)]
-        pipe = tt.HostStepPipeline(emb, max(p[0].numel() for p in hpool), B, depth=2)
+        depth = args.e2e_depth
+        houts = [torch.empty(B, cfg.num_tables, cfg.dim).pin_memory() for _ in range(depth)]
+        pipe = tt.HostStepPipeline(emb, max(p[0].numel() for p in hpool), B, depth=depth)
 
         def hstep(i):
             hi, ho, hg = hpool[i % len(hpool)]
-            return pipe.step(hi, ho, hg, houts[i % 2], lr=args.lr)
+            return pipe.step(hi, ho, hg, houts[i % depth], lr=args.lr)
 
         with torch.cuda.stream(stream):
             for i in range(args.warmup):
@@ -677,7 +679,7 @@ def main():
                "d2h_bytes_per_step": int(houts[0].numel() * 4), "ms_per_step": te / args.steps,
                "path": "HostStepPipeline: pinned host ids / offsets / grad_out -> device, "
                        "ttemb_forward + ttemb_backward, pooled output -> pinned host; copies of "
-                       "neighbouring steps overlapped with compute (2 staging slots)"}
+                       f"neighbouring steps overlapped with compute ({depth} staging slots)"}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
