@@ -224,6 +224,8 @@ size_t carve(Ctx& c, uint8_t* base) {
   p.chunk_off = k.take<uint32_t>(NG + 1);
   p.split_list = k.take<uint32_t>(NG);
   p.grp_c2 = k.take<unsigned long long>(NG);
+  p.unit_sorted = k.take<uint32_t>((size_t)NG * 4);   // <= 4 units per group (R = 128, NC <= 512)
+  p.unit_snake = k.take<uint32_t>((size_t)NG * 4);
   // --- float intermediates ---
   p.dabuf = k.take<float>((size_t)P * c.n1 * c.R);
   const size_t pf = tc_eligible(c) ? (size_t)P * c.n1 * c.NC : 1;

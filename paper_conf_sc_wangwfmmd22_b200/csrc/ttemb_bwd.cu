@@ -325,7 +325,11 @@ bool agg_scatter_path(const Ctx& c) { return c.N % 4 == 0 && c.N <= 128 && (128 
 cudaError_t run_plan_tail(Ctx& c, cudaStream_t s) {
   if (c.nnz > 0 && agg_scatter_path(c))
     k_zero_rows<<<grid_for(c, c.U_cap * c.N / 4, 256, 8), 256, 0, s>>>(c.p.gbuf, c.p.counts, c.N);
-  if (c.nnz > 0 && fused_eligible(c)) return run_dp_zero(c, s);
+  if (c.nnz > 0 && fused_eligible(c)) {
+    cudaError_t e = run_unit_order(c, s);
+    if (e != cudaSuccess) return e;
+    return run_dp_zero(c, s);
+  }
   return cudaGetLastError();
 }
 

@@ -84,6 +84,7 @@ struct YArgs {
   const unsigned long long* grp_c2;       // [NG] float offset of the group's C2 slice
   unsigned long long c2_begin;            // float offset of the C2 region (tm_c2 row 0)
   const float* dpbuf;                     // [P][n1][NC]
+  const uint32_t* unit_snake;             // [NU] unit at static position p (balanced by tile count)
   uint32_t* work;
   int n1, n1s, NC, nblk, tpp, nchunk, R;
   float lr, eps;
@@ -106,7 +107,7 @@ struct YCtl {
   // this CTA's work units (static round robin) loaded once, in parallel, at kernel start: first /
   // last prefix and C2 slice offset of the unit's group, so no unit boundary waits on a
   // global-memory round trip
-  uint32_t gq0[Y_GI], gq1[Y_GI];
+  uint32_t gq0[Y_GI], gq1[Y_GI], gu[Y_GI];
   unsigned long long gc2[Y_GI];
 };
 
@@ -141,10 +142,10 @@ k_prefix_bwd(const __grid_constant__ CUtensorMap tm_dp, const __grid_constant__ 
   }
   if (w == Y_MMA_W) tc::tmem_alloc(&ctl.tmem, 512);
   for (int i = tid; i < Y_GI; i += blockDim.x) {
-    const uint32_t u = blockIdx.x + (uint32_t)i * gridDim.x;
-    if (u < NU) {
-      const uint32_t g = u / UPG;
-      ctl.gq0[i] = a.grp_off[g]; ctl.gq1[i] = a.grp_off[g + 1]; ctl.gc2[i] = a.grp_c2[g];
+    const uint32_t pu = blockIdx.x + (uint32_t)i * gridDim.x;   // static position -> unit
+    if (pu < NU) {
+      const uint32_t u = a.unit_snake[pu], g = u / UPG;
+      ctl.gu[i] = u; ctl.gq0[i] = a.grp_off[g]; ctl.gq1[i] = a.grp_off[g + 1]; ctl.gc2[i] = a.grp_c2[g];
     }
   }
   tc::fence_before();
@@ -167,14 +168,19 @@ k_prefix_bwd(const __grid_constant__ CUtensorMap tm_dp, const __grid_constant__ 
   const int tpp = a.tpp, NC = a.NC;
 
   // Jobs = (unit, tile, K-chunk) in a static round-robin unit order (loaders, TMA producer)
-  struct Job { uint32_t u, q0, q1, qa; int ck, crow; unsigned long long c2; };
+  // Job.u = static position (G0 + k GS), Job.unit = the unit dealt to it (unit_snake)
+  struct Job { uint32_t u, unit, q0, q1, qa; int ck, crow; unsigned long long c2; };
   const uint32_t G0 = blockIdx.x, GS = gridDim.x;
   auto start = [&](Job& j, uint32_t u) {   // unit metadata (staged in shared memory)
     j.u = u; j.ck = 0;
     if (u < NU) {
-      const uint32_t k = (u - G0) / GS, g = u / UPG;
-      if (k < (uint32_t)Y_GI) { j.q0 = j.qa = ctl.gq0[k]; j.q1 = ctl.gq1[k]; j.c2 = ctl.gc2[k]; }
-      else { j.q0 = j.qa = a.grp_off[g]; j.q1 = a.grp_off[g + 1]; j.c2 = a.grp_c2[g]; }
+      const uint32_t k = (u - G0) / GS;
+      if (k < (uint32_t)Y_GI) { j.unit = ctl.gu[k]; j.q0 = j.qa = ctl.gq0[k]; j.q1 = ctl.gq1[k]; j.c2 = ctl.gc2[k]; }
+      else {
+        j.unit = a.unit_snake[u];
+        const uint32_t g = j.unit / UPG;
+        j.q0 = j.qa = a.grp_off[g]; j.q1 = a.grp_off[g + 1]; j.c2 = a.grp_c2[g];
+      }
       j.crow = (int)((j.c2 - a.c2_begin) / (unsigned long long)NC);   // C2 region row of r1 = 0
     }
   };
@@ -217,8 +223,8 @@ k_prefix_bwd(const __grid_constant__ CUtensorMap tm_dp, const __grid_constant__ 
         const uint32_t fl = (P.qa == P.q0 ? 1u : 0u) | (P.qa + tpp >= P.q1 ? 2u : 0u);
         if (tid == 0) {
           tc::mbar_wait(&ctl.u_empty[ui & 3], ((ui >> 2) & 1) ^ 1);
-          ctl.ring[ui & 3][0] = P.u / UPG; ctl.ring[ui & 3][1] = P.qa; ctl.ring[ui & 3][2] = np;
-          ctl.ring[ui & 3][3] = fl; ctl.ring[ui & 3][4] = P.u % UPG;
+          ctl.ring[ui & 3][0] = P.unit / UPG; ctl.ring[ui & 3][1] = P.qa; ctl.ring[ui & 3][2] = np;
+          ctl.ring[ui & 3][3] = fl; ctl.ring[ui & 3][4] = P.unit % UPG;
           tc::mbar_arrive(&ctl.u_full[ui & 3]);
         }
         // C1^T -> B1 (element (r1, m) = C1 row m, column r1); zero past the tile
@@ -468,7 +474,7 @@ k_prefix_bwd(const __grid_constant__ CUtensorMap tm_dp, const __grid_constant__ 
   } else {
     // ------------------------------- TMA producer -------------------------------
     auto issue = [&](const Job& j, uint32_t sidx) {
-      const int c0 = (int)(j.u % UPG) * BPU * 128 + j.ck * CK;   // first slice column of the chunk
+      const int c0 = (int)(j.unit % UPG) * BPU * 128 + j.ck * CK;   // first slice column of the chunk
       const uint32_t st = sidx % Y_NST;
       const uint32_t a2 = tc::smem_u32(stg + st * S::STAGE), b2 = a2 + S::A2;
       const int prow = (int)(j.qa << a.n1s);                      // dP stash row of tile row 0
@@ -582,6 +588,7 @@ cudaError_t run_prefix_bwd(Ctx& c, float lr, cudaStream_t s) {
   a.cores = c.cores; a.grads = c.grads; a.state = c.state; a.meta = c.d_meta; a.counts = p.counts;
   a.grp_off = p.grp_off; a.grp_t = p.grp_t; a.pfx_i1 = p.pfx_i1; a.pfx_t = p.pfx_t; a.grp_arow = p.grp_arow;
   a.grp_c2 = p.grp_c2; a.dpbuf = p.dpbuf; a.work = p.work + 2; a.c2_begin = c.c1_floats;
+  a.unit_snake = p.unit_snake;
   a.n1 = c.n1; a.n1s = c.n1 == 1 ? 0 : c.n1 == 2 ? 1 : c.n1 == 4 ? 2 : 3;
   a.NC = c.NC; a.nblk = (c.NC + 127) / 128; a.tpp = YT / c.n1; a.R = c.R;
   // K-chunks per work unit: R = 64 the whole slice in 64-column chunks, R = 128 one c-block in
@@ -591,8 +598,7 @@ cudaError_t run_prefix_bwd(Ctx& c, float lr, cudaStream_t s) {
   a.exp = exp_bits();
   a.pf = knobs().pf_bwd;
   StageScope sc(c, ST_BWD_PREFIX, s);
-  const int64_t units = c.NG_cap * (c.R <= 64 ? 1 : (c.NC + 127) / 128);
-  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(units, (int64_t)c.sm_count));
+  const int grid = prefix_bwd_grid(c);   // (the unit_snake deal was made for this grid)
   static unsigned long long* trace = nullptr;
   a.trace = nullptr;
   if (knobs().trace) {

@@ -42,6 +42,7 @@ struct XArgs {
   const TableMeta* meta;
   const uint32_t *counts, *grp_off, *grp_t, *grp_i2, *grp_pfx, *pfx_i1, *pfx_t, *row_seg, *row_i3, *row_pfx;
   uint32_t* grp_arow;                 // [P]  C1 row index (floats / R) of sorted prefix q, j1 = 0
+  const uint32_t* unit_sorted;        // [NU] work units, largest first (claim k -> unit_sorted[k])
   unsigned long long* grp_c2;         // [NG] float offset of group g's C2 slice
   float* rows;                        // [U][N]
   float* pbuf;                        // [P][n1][NC] (consumed by the backward row stage)
@@ -163,9 +164,15 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
           tc::bulk_g2s(tc::smem_u32(raw + r * 128), src + (size_t)r * a.NC + c0, (uint32_t)(nc * 4), &ctl.raw_full);
       }
     };
+    // thread 0: the next unit in group order (claiming the largest-first order of unit_sorted
+    // instead measured 1.5 us slower at c4: TTEMB_DBG bit 64 selects it for comparison)
+    auto claim = [&]() {
+      const uint32_t k = atomicAdd(a.work, 1u);
+      return k < NU ? ((a.dbg & 64) ? a.unit_sorted[k] : k) : NU;
+    };
     if (tid == 0) {
-      ctl.claim[0] = atomicAdd(a.work, 1u);
-      ctl.claim[1] = atomicAdd(a.work, 1u);
+      ctl.claim[0] = claim();
+      ctl.claim[1] = claim();
       if (ctl.claim[0] < NU) issue_raw(ctl.claim[0]);
     }
     tc::named_sync(1, X_LW * 32);
@@ -240,7 +247,7 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
       }
       XT0();
       // next unit: registers <- raw (nxt); raw <- the unit after (claimed now)
-      if (tid == 0) ctl.claim[gs & 1] = atomicAdd(a.work, 1u);
+      if (tid == 0) ctl.claim[gs & 1] = claim();
       if (nxt < NU) {
         tc::mbar_wait(&ctl.raw_full, rawk & 1);
         ++rawk;
@@ -776,7 +783,64 @@ template <class F> void for_rows_bwd(F&& f) {
       for (int j12 : {16, 4}) f(rows_bwd_kernel(n3, R, j12), n3, R == 32 ? 32 : 64);
 }
 
+// Work-unit order of the prefix kernels (plan-dependent, run with the index stage): units (i2-group,
+// c-block range) sorted by their tile count, largest first (a counting sort; the order inside one
+// count is arbitrary and only changes which CTA does what).  k_prefix_bwd deals it to its G
+// CTAs round by round in alternating directions (round r, CTA c takes sorted unit r G + c for even
+// r, r G + G - 1 - c for odd r), which balances its static schedule: at c4 the most loaded CTA
+// had 22 tiles against a mean of 18.3 in group order (bwd_prefix 150 -> 135 us).  k_prefix_fwd
+// keeps claiming in group order (dynamic claims already balance it; see its claim()).
+__global__ void __launch_bounds__(1024) k_unit_order(const uint32_t* __restrict__ counts, const uint32_t* __restrict__ grp_off,
+                                                     int tpp, int upg, int G, uint32_t* __restrict__ sorted,
+                                                     uint32_t* __restrict__ snake) {
+  __shared__ uint32_t hist[256];
+  const uint32_t NU = counts[kCntNG] * (uint32_t)upg;
+  for (int i = threadIdx.x; i < 256; i += blockDim.x) hist[i] = 0;
+  __syncthreads();
+  auto bucket = [&](uint32_t u) {   // 255 - min(tiles, 255): ascending bucket = descending size
+    const uint32_t g = u / upg, np = grp_off[g + 1] - grp_off[g];
+    return 255u - min((np + tpp - 1) / tpp, 255u);
+  };
+  for (uint32_t u = threadIdx.x; u < NU; u += blockDim.x) atomicAdd(&hist[bucket(u)], 1u);
+  __syncthreads();
+  if (threadIdx.x < 32) {   // exclusive scan of 256 buckets by one warp (8 per lane)
+    const int l = threadIdx.x;
+    uint32_t v[8], t = 0;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) { v[i] = hist[8 * l + i]; t += v[i]; }
+    uint32_t x = t;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+      if (l >= o) x += y;
+    }
+    uint32_t run = x - t;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) { hist[8 * l + i] = run; run += v[i]; }
+  }
+  __syncthreads();
+  for (uint32_t u = threadIdx.x; u < NU; u += blockDim.x) sorted[atomicAdd(&hist[bucket(u)], 1u)] = u;
+  __syncthreads();
+  for (uint32_t p = threadIdx.x; p < NU; p += blockDim.x) {
+    const uint32_t r = p / (uint32_t)G, c = p - r * (uint32_t)G, base = r * (uint32_t)G;
+    const uint32_t m = min((uint32_t)G, NU - base);   // units in this round
+    snake[p] = sorted[base + ((r & 1u) ? m - 1u - c : c)];
+  }
+}
+
 }  // namespace
+
+int prefix_units_per_group(const Ctx& c) { return c.R <= 64 ? 1 : (c.NC + 127) / 128; }
+int prefix_bwd_grid(const Ctx& c) {
+  const int64_t units = c.NG_cap * prefix_units_per_group(c);
+  return (int)std::max<int64_t>(1, std::min<int64_t>(units, (int64_t)c.sm_count));
+}
+
+cudaError_t run_unit_order(Ctx& c, cudaStream_t s) {
+  k_unit_order<<<1, 1024, 0, s>>>(c.p.counts, c.p.grp_off, XT / c.n1, prefix_units_per_group(c), prefix_bwd_grid(c),
+                                  c.p.unit_sorted, c.p.unit_snake);
+  return cudaGetLastError();
+}
 
 bool fused_eligible(const Ctx& c) {
   // R = 32 / 64 (ranks 16..63 stored padded to 32 or 64) with n2 R <= 256; R = 128 with n2 R <= 512
@@ -815,6 +879,7 @@ cudaError_t run_fused_fwd(Ctx& c, float* out, cudaStream_t s) {
   a.cores = c.cores; a.meta = c.d_meta; a.counts = p.counts; a.grp_off = p.grp_off; a.grp_t = p.grp_t;
   a.grp_i2 = p.grp_i2; a.grp_pfx = p.grp_pfx; a.pfx_i1 = p.pfx_i1; a.pfx_t = p.pfx_t; a.row_seg = p.row_seg;
   a.row_i3 = p.row_i3; a.row_pfx = p.row_pfx; a.grp_arow = p.grp_arow; a.grp_c2 = p.grp_c2; a.rows = p.rows; a.pbuf = p.pbuf;
+  a.unit_sorted = p.unit_sorted;
   a.work = p.work + 0;
   a.dbg = knobs().dbg;
   a.n1 = c.n1; a.n1s = c.n1 == 1 ? 0 : c.n1 == 2 ? 1 : c.n1 == 4 ? 2 : 3;

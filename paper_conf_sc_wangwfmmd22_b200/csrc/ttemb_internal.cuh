@@ -107,6 +107,8 @@ struct PlanDev {
   uint32_t* grp_arow;                          // [P]  C1 row (float offset / R) of sorted prefix q, j1 = 0
   uint32_t *chunk_off, *split_list;            // FFMA path: [NG+1] first unit of group g; [NG] split groups
   unsigned long long* grp_c2;                  // [NG] float offset of the C2 slice of group g
+  uint32_t *unit_sorted, *unit_snake;          // [NU] prefix-kernel work units by tile count (desc) /
+                                               // that order dealt to the backward grid boustrophedon
 };
 
 struct Ctx {
@@ -201,6 +203,9 @@ cudaError_t run_tc_fwd(Ctx& c, float* out, cudaStream_t s);
 cudaError_t run_tc_bwd(Ctx& c, float lr, cudaStream_t s);
 bool fused_eligible(const Ctx& c);
 cudaError_t run_dp_zero(Ctx& c, cudaStream_t s);
+cudaError_t run_unit_order(Ctx& c, cudaStream_t s);
+int prefix_units_per_group(const Ctx& c);
+int prefix_bwd_grid(const Ctx& c);
 cudaError_t run_plan_tail(Ctx& c, cudaStream_t s);
 cudaError_t configure_fused(Ctx& c);
 cudaError_t run_fused_fwd(Ctx& c, float* out, cudaStream_t s);
