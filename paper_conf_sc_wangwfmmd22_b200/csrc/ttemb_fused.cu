@@ -970,9 +970,10 @@ cudaError_t run_rows_bwd2(Ctx& c, cudaStream_t s) {
   r.dpbuf = p.dpbuf; r.n1 = c.n1; r.n2 = c.n2; r.N = c.N; r.NC = c.NC; r.R = c.R;
   r.exp = exp_bits();
   // (the dP rows of chunk-straddling prefixes were zeroed at the end of the index stage)
-  // 32-wide r slices (RL = 1, 24 warps / SM) by default: at c4 88 us vs 98.7 us for 64-wide
-  // slices (RL = 2, 16 warps / SM; TTEMB_EXP bit 2048 selects them for comparison)
-  const bool narrow = c.R == 32 || !(exp_bits() & 2048);
+  // 32-wide r slices (RL = 1, 24 warps / SM) for n3 = 4: at c4 88 us vs 98.7 us for 64-wide slices
+  // (RL = 2, 16 warps / SM); 64-wide for n3 = 8 (c5 R = 64: 3.83 vs 3.99 ms, R = 128: 7.61 vs
+  // 7.94 ms); TTEMB_EXP bit 2048 flips the choice for comparison
+  const bool narrow = c.R == 32 || ((c.n3 == 4) != ((exp_bits() & 2048) != 0));
   const int sw = narrow ? 32 : 64;
   const int grid = grid_for(c, cdiv(c.U_cap, RW_RCH) * (c.R / sw), RW_WARPS, narrow ? 3 : 2);
   const void* f = narrow ? rows_bwd_kernel_rl1(c.n3, c.R, c.n1 * c.n2) : rows_bwd_kernel(c.n3, c.R, c.n1 * c.n2);
