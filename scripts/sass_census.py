@@ -5,7 +5,7 @@
 
 Counts the opcodes that prove which hardware paths a kernel uses (B200_PROFILING.md):
 UTCHMMA / UTCQMMA (tcgen05.mma), LDTM / STTM (TMEM ld / st), UTMALDG (tensor-map TMA load),
-UBLKCP (1-D bulk copy), LDGSTS (Ampere cp.async), FFMA, REDG (global reductions), SHFL.
+UBLKCP (1-D bulk copy), LDGSTS (Ampere cp.async), FFMA, FFMA2 (packed fp32 pairs), REDG, SHFL.
 """
 from __future__ import annotations
 
@@ -19,7 +19,7 @@ import sys
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 LIB = os.path.join(ROOT, "paper_conf_sc_wangwfmmd22_b200", "libttemb.so")
 OPS = ["UTCHMMA", "UTCQMMA", "UTCBAR", "LDTM", "STTM", "UTMALDG", "UTMASTG", "UBLKCP", "LDGSTS", "SYNCS",
-       "FFMA", "REDG", "ATOMG", "SHFL", "LDS", "STS", "LDG", "STG"]
+       "FFMA", "FFMA2", "REDG", "ATOMG", "SHFL", "LDS", "STS", "LDG", "STG"]
 
 
 def demangle(name: str) -> str:
