@@ -140,6 +140,7 @@ __global__ void __launch_bounds__(256)
 k_agg_scatter(const float* __restrict__ grad_out, const uint32_t* __restrict__ sbag,
               const uint32_t* __restrict__ spos, const uint32_t* __restrict__ inverse, int64_t nnz, int N,
               float* __restrict__ gbuf, const float* __restrict__ wpos, const uint32_t* __restrict__ counts) {
+  pdl_wait();
   const int lane = threadIdx.x & 31;
   const int NV = N >> 2, P = 32 / NV;   // float4 columns; occurrences in flight per step
   // one id per bag: every grad_out row is read exactly once -> evict-first loads keep L2 for G
@@ -274,6 +275,8 @@ k_update_zero(float* __restrict__ cores, float* __restrict__ state, float* __res
 __global__ void __launch_bounds__(256)
 k_update_zero4(float* __restrict__ cores, float* __restrict__ state, float* __restrict__ grads, size_t n1,
                size_t begin2, size_t n2, float lr, float eps, int opt) {
+  pdl_wait();
+  pdl_trigger();
   const size_t n = (n1 + n2) / 4;
   for (size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
     const size_t e = 4 * i < n1 ? 4 * i : begin2 + (4 * i - n1);
@@ -348,9 +351,9 @@ cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s
     StageScope sc(c, ST_AGG, s);
     if (agg_scatter_path(c)) {
       // (G was zeroed at the end of the index stage: run_plan_tail)
-      k_agg_scatter<<<grid_for(c, cdiv(c.nnz, 32), 8, 32), 256, 0, s>>>(grad_out, p.sbag, p.spos, p.inverse,
-                                                                         c.nnz, c.N, p.gbuf,
-                                                                         c.weighted ? p.wpos : nullptr, p.counts);
+      launch_pdl(k_agg_scatter, dim3(grid_for(c, cdiv(c.nnz, 32), 8, 32)), dim3(256), 0, s, grad_out,
+                 (const uint32_t*)p.sbag, (const uint32_t*)p.spos, (const uint32_t*)p.inverse, (int64_t)c.nnz, c.N,
+                 p.gbuf, (const float*)(c.weighted ? p.wpos : nullptr), (const uint32_t*)p.counts);
     } else {
       const int64_t total = agg_chunks(c.nnz) * c.N;
       if (c.N % 4 == 0)
@@ -397,8 +400,8 @@ cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s
   if (fused) {   // C2 was updated inside the group kernel; C1 and C3 densely here
     StageScope sc(c, ST_UPD_C3, s);
     if (c.c1_floats % 4 == 0 && c.c3_begin % 4 == 0 && c.c3_floats % 4 == 0)
-      k_update_zero4<<<grid_for(c, (int64_t)(c.c1_floats + c.c3_floats) / 4, 256, 8), 256, 0, s>>>(
-          c.cores, c.state, c.grads, c.c1_floats, c.c3_begin, c.c3_floats, lr, c.eps, c.opt);
+      launch_pdl(k_update_zero4, dim3(grid_for(c, (int64_t)(c.c1_floats + c.c3_floats) / 4, 256, 8)), dim3(256), 0, s,
+                 c.cores, c.state, c.grads, (size_t)c.c1_floats, (size_t)c.c3_begin, (size_t)c.c3_floats, lr, c.eps, c.opt);
     else
       k_update_zero<<<grid_for(c, (int64_t)(c.c1_floats + c.c3_floats), 256, 32), 256, 0, s>>>(
           c.cores, c.state, c.grads, c.c1_floats, c.c3_begin, c.c3_floats, lr, c.eps, c.opt);

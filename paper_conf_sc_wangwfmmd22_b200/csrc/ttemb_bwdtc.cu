@@ -116,6 +116,8 @@ __device__ __forceinline__ float lo32(float x) { return x - tc::tf32_trunc(x); }
 template <int KR>
 __global__ void __launch_bounds__(Y_THREADS, 1)
 k_prefix_bwd(const __grid_constant__ CUtensorMap tm_dp, const __grid_constant__ CUtensorMap tm_c2, YArgs a) {
+  pdl_wait();
+  pdl_trigger();
   using S = YShape<KR>;
   constexpr int BPU = S::BPU, CK = S::CK;
   extern __shared__ __align__(128) char smem_raw[];
@@ -606,9 +608,9 @@ cudaError_t run_prefix_bwd(Ctx& c, float lr, cudaStream_t s) {
     cudaMemsetAsync(trace, 0, sizeof(unsigned long long) * 32 * grid, s);
     a.trace = trace;
   }
-  if (c.R == 32) k_prefix_bwd<32><<<grid, Y_THREADS, YShape<32>::SMEM, s>>>(c.tm_dp, c.tm_c2, a);
-  else if (c.R == 64) k_prefix_bwd<64><<<grid, Y_THREADS, YShape<64>::SMEM, s>>>(c.tm_dp, c.tm_c2, a);
-  else k_prefix_bwd<128><<<grid, Y_THREADS, YShape<128>::SMEM, s>>>(c.tm_dp, c.tm_c2, a);
+  if (c.R == 32) launch_pdl(k_prefix_bwd<32>, dim3(grid), dim3(Y_THREADS), YShape<32>::SMEM, s, c.tm_dp, c.tm_c2, a);
+  else if (c.R == 64) launch_pdl(k_prefix_bwd<64>, dim3(grid), dim3(Y_THREADS), YShape<64>::SMEM, s, c.tm_dp, c.tm_c2, a);
+  else launch_pdl(k_prefix_bwd<128>, dim3(grid), dim3(Y_THREADS), YShape<128>::SMEM, s, c.tm_dp, c.tm_c2, a);
   if (a.fused && a.opt != TTEMB_SGD)
     k_c2_update_zero<<<c.sm_count * 8, 256, 0, s>>>(c.cores, c.state, c.grads, p.grp_c2, p.counts,
                                                     (uint32_t)(c.R * c.NC), lr, c.eps);

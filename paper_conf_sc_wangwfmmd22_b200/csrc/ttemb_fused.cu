@@ -73,6 +73,7 @@ struct XCtl {
 };
 
 __global__ void k_fused_prep(XArgs a) {
+  pdl_wait();
   const uint32_t P = a.counts[kCntP], NG = a.counts[kCntNG];
   for (uint32_t q = blockIdx.x * blockDim.x + threadIdx.x; q < max(P, NG); q += gridDim.x * blockDim.x) {
     if (q < P) {
@@ -91,6 +92,8 @@ __device__ __forceinline__ float tf32_lo(float x) { return x - tc::tf32_trunc(x)
 // the C1 rows of a tile are staged once per unit.
 template <int KR, int NC_T>   // NC_T = n2 R when fixed at compile time (immediate store offsets), else 0
 __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
+  pdl_wait();
+  pdl_trigger();
   const int NCT = NC_T ? NC_T : a.NC;
   constexpr int BPU = KR <= 64 ? 2 : 1;            // c-blocks per work unit
   constexpr uint32_t BSLOT = 2u * XT * KR * 4;    // one B slot: C1 tile hi + lo (K = KR)
@@ -413,6 +416,8 @@ struct RowArgs {
 
 template <int N3, int RPL>   // RPL = R / 8: r values per lane (8 at R = 64, 16 at R = 128)
 __global__ void __launch_bounds__(RW_WARPS * 32, RPL == 8 ? 3 : 2) k_rows_fwd2(RowArgs a) {
+  pdl_wait();
+  pdl_trigger();
   constexpr int KR = 8 * RPL;
   constexpr int SLOT = KR * N3 + KR / 2;       // + 4 floats of skew per 8 rows of r
   constexpr int C3L = KR * N3 / 4 / 32;
@@ -580,6 +585,8 @@ constexpr int RB_J12 = 16;   // n1 n2 <= 16
 template <int N3, int RL, int KR, int J12T>   // RL = r per lane: 1 (R = 32) or 2 (R = 64, 128 in two
                                               // slices); J12T = n1 n2 (0: runtime, <= 16)
 __global__ void __launch_bounds__(RW_WARPS * 32, RL == 1 ? 3 : 2) k_rows_bwd2(RowBwdArgs a) {
+  pdl_wait();
+  pdl_trigger();
   constexpr int SW = 32 * RL;                   // r width of a work item (a slice of R)
   constexpr int NSL = KR / SW;                  // slices per row
   constexpr int C3S = SW * N3;                  // C3 part of a slot
@@ -886,7 +893,7 @@ cudaError_t run_fused_fwd(Ctx& c, float* out, cudaStream_t s) {
   a.n2 = c.n2; a.n3 = c.n3; a.N = c.N; a.NC = c.NC; a.nblk = (c.NC + 127) / 128; a.tpp = XT / c.n1; a.R = c.R;
   {
     StageScope sc(c, ST_FWD_PREFIX, s);
-    k_fused_prep<<<grid_for(c, std::max(c.P_cap, c.NG_cap), 256, 4), 256, 0, s>>>(a);
+    launch_pdl(k_fused_prep, dim3(grid_for(c, std::max(c.P_cap, c.NG_cap), 256, 4)), dim3(256), 0, s, a);
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(c.NG_cap, (int64_t)c.sm_count));
     static unsigned long long* trace = nullptr;
     a.trace = nullptr;
@@ -897,14 +904,14 @@ cudaError_t run_fused_fwd(Ctx& c, float* out, cudaStream_t s) {
     }
     const bool n2_4 = c.n2 == 4;   // the c4 / c5 shapes: NC = 4 R as a compile-time constant
     if (c.R == 32) {
-      if (n2_4) k_prefix_fwd<32, 128><<<grid, X_THREADS, prefix_smem<32>(), s>>>(a);
-      else k_prefix_fwd<32, 0><<<grid, X_THREADS, prefix_smem<32>(), s>>>(a);
+      if (n2_4) launch_pdl(k_prefix_fwd<32, 128>, dim3(grid), dim3(X_THREADS), prefix_smem<32>(), s, a);
+      else launch_pdl(k_prefix_fwd<32, 0>, dim3(grid), dim3(X_THREADS), prefix_smem<32>(), s, a);
     } else if (c.R == 64) {
-      if (n2_4) k_prefix_fwd<64, 256><<<grid, X_THREADS, prefix_smem<64>(), s>>>(a);
-      else k_prefix_fwd<64, 0><<<grid, X_THREADS, prefix_smem<64>(), s>>>(a);
+      if (n2_4) launch_pdl(k_prefix_fwd<64, 256>, dim3(grid), dim3(X_THREADS), prefix_smem<64>(), s, a);
+      else launch_pdl(k_prefix_fwd<64, 0>, dim3(grid), dim3(X_THREADS), prefix_smem<64>(), s, a);
     } else {
-      if (n2_4) k_prefix_fwd<128, 512><<<grid, X_THREADS, prefix_smem<128>(), s>>>(a);
-      else k_prefix_fwd<128, 0><<<grid, X_THREADS, prefix_smem<128>(), s>>>(a);
+      if (n2_4) launch_pdl(k_prefix_fwd<128, 512>, dim3(grid), dim3(X_THREADS), prefix_smem<128>(), s, a);
+      else launch_pdl(k_prefix_fwd<128, 0>, dim3(grid), dim3(X_THREADS), prefix_smem<128>(), s, a);
     }
     if (a.trace) {
       std::vector<unsigned long long> hb(32 * grid);
@@ -935,15 +942,16 @@ cudaError_t run_fused_fwd(Ctx& c, float* out, cudaStream_t s) {
     r.c3_begin = c.c3_begin; r.pfx_t = p.pfx_t; r.pbuf = p.pbuf; r.rows = p.rows; r.seg_off = p.seg_off; r.sbag = p.sbag; r.out = out;
     r.n1 = c.n1; r.n1s = a.n1s; r.n2 = c.n2; r.N = c.N; r.NC = c.NC;
     const int grid = grid_for(c, cdiv(c.U_cap, RW_RCH), RW_WARPS, 4);
+    const dim3 g(grid), b(RW_WARPS * 32);
     if (c.R == 32) {
-      if (c.n3 == 4) k_rows_fwd2<4, 4><<<grid, RW_WARPS * 32, rows_smem(4, 32), s>>>(r);
-      else k_rows_fwd2<8, 4><<<grid, RW_WARPS * 32, rows_smem(8, 32), s>>>(r);
+      if (c.n3 == 4) launch_pdl(k_rows_fwd2<4, 4>, g, b, rows_smem(4, 32), s, r);
+      else launch_pdl(k_rows_fwd2<8, 4>, g, b, rows_smem(8, 32), s, r);
     } else if (c.R == 64) {
-      if (c.n3 == 4) k_rows_fwd2<4, 8><<<grid, RW_WARPS * 32, rows_smem(4, 64), s>>>(r);
-      else k_rows_fwd2<8, 8><<<grid, RW_WARPS * 32, rows_smem(8, 64), s>>>(r);
+      if (c.n3 == 4) launch_pdl(k_rows_fwd2<4, 8>, g, b, rows_smem(4, 64), s, r);
+      else launch_pdl(k_rows_fwd2<8, 8>, g, b, rows_smem(8, 64), s, r);
     } else {
-      if (c.n3 == 4) k_rows_fwd2<4, 16><<<grid, RW_WARPS * 32, rows_smem(4, 128), s>>>(r);
-      else k_rows_fwd2<8, 16><<<grid, RW_WARPS * 32, rows_smem(8, 128), s>>>(r);
+      if (c.n3 == 4) launch_pdl(k_rows_fwd2<4, 16>, g, b, rows_smem(4, 128), s, r);
+      else launch_pdl(k_rows_fwd2<8, 16>, g, b, rows_smem(8, 128), s, r);
     }
   }
   return cudaGetLastError();
@@ -979,7 +987,7 @@ cudaError_t run_rows_bwd2(Ctx& c, cudaStream_t s) {
   const void* f = narrow ? rows_bwd_kernel_rl1(c.n3, c.R, c.n1 * c.n2) : rows_bwd_kernel(c.n3, c.R, c.n1 * c.n2);
   if (!f) return cudaErrorInvalidValue;
   void* args[] = {&r};
-  return cudaLaunchKernel(f, dim3(grid), dim3(RW_WARPS * 32), args, rows_bwd_smem(c.n3, sw), s);
+  return launch_pdl_ptr(f, dim3(grid), dim3(RW_WARPS * 32), rows_bwd_smem(c.n3, sw), s, args);
 }
 
 // Forward contractions on tcgen05: P (k_prefix_fwd) then rows (k_rows_fwd2).

@@ -44,6 +44,7 @@ __global__ void __launch_bounds__(256)
 k_pool(const float* __restrict__ rows, const uint32_t* __restrict__ inverse,
        const int64_t* __restrict__ offsets, int64_t nnz, int T, int B, int N, float* __restrict__ out,
        const uint32_t* __restrict__ counts, int skip_single, const float* __restrict__ wpos) {
+  pdl_wait();
   if (skip_single && counts[kCntMulti] == 0) return;   // one id per bag: written directly
   using V = typename std::conditional<VW == 4, float4, float>::type;
   const uint32_t NV = (uint32_t)(N / VW);
@@ -128,6 +129,7 @@ __global__ void __launch_bounds__(256)
 k_pool_single_out(const float* __restrict__ rows, const uint32_t* __restrict__ inverse, int64_t nnz,
                   int T, int B, int N, int nvs, float* __restrict__ out, const uint32_t* __restrict__ counts,
                   const float* __restrict__ wpos) {
+  pdl_wait();
   if (counts[kCntMulti] != 0) return;
   const I NV = (I)(N >> 2), uT = (I)T, uB = (I)B;
   const I total = (I)T * (I)B * NV, stride = (I)gridDim.x * blockDim.x;
@@ -205,20 +207,21 @@ cudaError_t run_forward_compute(Ctx& c, float* out, const int64_t* offsets, cuda
             const int grid = grid_for(c, total / (4 * TTEMB_POOL_IPT), 256, TTEMB_POOL_PER_SM);
             const int nv = c.N / 4, nvs = (nv & (nv - 1)) == 0 ? __builtin_ctz(nv) : -1;
             const int64_t span = total / 4 + (int64_t)TTEMB_POOL_IPT * grid * 256;   // largest index formed
+            const float* wp = c.weighted ? p.wpos : nullptr;
             if (span < ((int64_t)1 << 32))
-              k_pool_single_out<uint32_t><<<grid, 256, 0, s>>>(p.rows, p.inverse, c.nnz, c.T, c.B, c.N, nvs, out,
-                                                             p.counts, c.weighted ? p.wpos : nullptr);
+              launch_pdl(k_pool_single_out<uint32_t>, dim3(grid), dim3(256), 0, s, (const float*)p.rows,
+                         (const uint32_t*)p.inverse, (int64_t)c.nnz, c.T, c.B, c.N, nvs, out, (const uint32_t*)p.counts, wp);
             else
-              k_pool_single_out<uint64_t><<<grid, 256, 0, s>>>(p.rows, p.inverse, c.nnz, c.T, c.B, c.N, nvs, out,
-                                                             p.counts, c.weighted ? p.wpos : nullptr);
+              launch_pdl(k_pool_single_out<uint64_t>, dim3(grid), dim3(256), 0, s, (const float*)p.rows,
+                         (const uint32_t*)p.inverse, (int64_t)c.nnz, c.T, c.B, c.N, nvs, out, (const uint32_t*)p.counts, wp);
           } else
             k_pool_single<<<grid_for(c, c.nnz * c.N / 16, 256, TTEMB_POOL_PER_SM), 256, 0, s>>>(
                 p.rows, p.inverse, p.bag_of, c.nnz, c.N, out, p.counts, c.weighted ? p.wpos : nullptr);
         }
         // the multi-hot sum exits at once on one-hot batches: one wave of CTAs, not four
-        k_pool<4><<<grid_for(c, total / 16, 256, 8), 256, 0, s>>>(p.rows, p.inverse, offsets, c.nnz,
-                                                                 c.T, c.B, c.N, out, p.counts, 1,
-                                                                 c.weighted ? p.wpos : nullptr);
+        launch_pdl(k_pool<4>, dim3(grid_for(c, total / 16, 256, 8)), dim3(256), 0, s, (const float*)p.rows,
+                   (const uint32_t*)p.inverse, offsets, (int64_t)c.nnz, c.T, c.B, c.N, out, (const uint32_t*)p.counts, 1,
+                   (const float*)(c.weighted ? p.wpos : nullptr));
       }
       else
         k_pool<1><<<grid_for(c, total / 4, 256, 32), 256, 0, s>>>(p.rows, p.inverse, offsets, c.nnz, c.T,

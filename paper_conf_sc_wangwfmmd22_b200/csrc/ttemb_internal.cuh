@@ -215,6 +215,43 @@ cudaError_t run_prefix_bwd(Ctx& c, float lr, cudaStream_t s);
 
 // ---- small helpers -------------------------------------------------------------------
 static inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+// Programmatic dependent launch along the step's main chain (forward: prefix -> rows -> pooling;
+// backward: aggregation -> rows -> prefix -> update).  A kernel launched with launch_pdl may be
+// scheduled while its predecessor on the stream is still draining; it calls pdl_wait() before
+// its first access to anything the predecessor wrote (every such kernel does so on entry), so
+// results are those of plain stream order.  The successor is released when the predecessor's CTAs
+// exit (implicit trigger): c4 step 433 -> 430 us in an interleaved A/B.  Triggering on entry
+// (pdl_trigger, built only with TTEMB_PDL_EARLY_TRIGGER) measured 483 us: early successor CTAs
+// took SMs from the predecessors' later waves and from the pipelined index stage.  TTEMB_EXP bit
+// 32768 launches without the attribute (plain stream order) for comparison.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() {
+#ifdef TTEMB_PDL_EARLY_TRIGGER
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+#endif
+}
+
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s,
+                              Args&&... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid; cfg.blockDim = block; cfg.dynamicSmemBytes = smem; cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = (exp_bits() & 32768) ? 0 : 1;
+  cfg.attrs = at; cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kernel, static_cast<KArgs>(args)...);
+}
+inline cudaError_t launch_pdl_ptr(const void* kernel, dim3 grid, dim3 block, size_t smem, cudaStream_t s, void** args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid; cfg.blockDim = block; cfg.dynamicSmemBytes = smem; cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = (exp_bits() & 32768) ? 0 : 1;
+  cfg.attrs = at; cfg.numAttrs = 1;
+  return cudaLaunchKernelExC(&cfg, kernel, args);
+}
 static inline int grid_for(const Ctx& c, int64_t items, int threads, int per_sm = 32) {
   int64_t g = cdiv(items, threads);
   int64_t cap = (int64_t)c.sm_count * per_sm;
