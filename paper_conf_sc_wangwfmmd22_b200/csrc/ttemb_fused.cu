@@ -415,7 +415,7 @@ struct RowArgs {
 };
 
 template <int N3, int RPL>   // RPL = R / 8: r values per lane (8 at R = 64, 16 at R = 128)
-__global__ void __launch_bounds__(RW_WARPS * 32, RPL == 8 ? 3 : 2) k_rows_fwd2(RowArgs a) {
+__global__ void __launch_bounds__(RW_WARPS * 32, (RPL == 8 && N3 == 4) ? 3 : 2) k_rows_fwd2(RowArgs a) {
   pdl_wait();
   pdl_trigger();
   constexpr int KR = 8 * RPL;
