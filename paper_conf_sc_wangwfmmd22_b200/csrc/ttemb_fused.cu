@@ -401,6 +401,9 @@ __device__ __forceinline__ void ffma2(float2& d, float2 a, float2 b) {
 }
 __device__ __forceinline__ void ffma2s(float2& d, float s, float2 b) { ffma2(d, make_float2(s, s), b); }
 
+#ifndef TTEMB_FWD_ROWS_BLOCKS
+#define TTEMB_FWD_ROWS_BLOCKS 3   // k_rows_fwd2 CTAs per SM at n3 = 4, R = 64 (register cap 85)
+#endif
 constexpr int RW_WARPS = 8, RW_RCH = 16, RW_NSL = 3;
 
 struct RowArgs {
@@ -415,7 +418,7 @@ struct RowArgs {
 };
 
 template <int N3, int RPL>   // RPL = R / 8: r values per lane (8 at R = 64, 16 at R = 128)
-__global__ void __launch_bounds__(RW_WARPS * 32, (RPL == 8 && N3 == 4) ? 3 : 2) k_rows_fwd2(RowArgs a) {
+__global__ void __launch_bounds__(RW_WARPS * 32, (RPL == 8 && N3 == 4) ? TTEMB_FWD_ROWS_BLOCKS : 2) k_rows_fwd2(RowArgs a) {
   pdl_wait();
   pdl_trigger();
   constexpr int KR = 8 * RPL;
