@@ -22,6 +22,11 @@ import time
 
 import numpy as np
 
+if int(os.environ.get("WORLD_SIZE", "1")) > 1:
+    # N > 1: the step graph interleaves NCCL kernels with ours; launch the main chain in plain
+    # stream order there (PDL next to NCCL kernels was not validated on a multi-GPU box)
+    os.environ.setdefault("TTEMB_NO_PDL", "1")
+
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 

@@ -49,16 +49,18 @@ enum Stage : int {
 // Debug / experiment knobs from the environment, read ONCE per process (never on the launch
 // path): TTEMB_EXP bits switch parts of k_prefix_bwd off (timing experiments, results invalid),
 // TTEMB_DBG likewise for the forward kernels, TTEMB_TRACE enables role timers (trace builds),
-// TTEMB_PF_BWD sets an L2 prefetch distance in k_prefix_bwd.
+// TTEMB_PF_BWD sets an L2 prefetch distance in k_prefix_bwd; TTEMB_NO_PDL=1 launches the main
+// chain without programmatic dependent launch (bench.py sets it for N > 1, where the step graph
+// interleaves NCCL kernels and no multi-GPU box was available to validate PDL next to them).
 struct Knobs {
-  int exp = 0, dbg = 0, trace = 0, pf_bwd = 0;
+  int exp = 0, dbg = 0, trace = 0, pf_bwd = 0, no_pdl = 0;
 };
 inline const Knobs& knobs() {
   static const Knobs k = [] {
     auto num = [](const char* n) { const char* e = getenv(n); return e ? atoi(e) : 0; };
     Knobs r;
     r.exp = num("TTEMB_EXP"); r.dbg = num("TTEMB_DBG"); r.trace = getenv("TTEMB_TRACE") ? 1 : 0;
-    r.pf_bwd = num("TTEMB_PF_BWD");
+    r.pf_bwd = num("TTEMB_PF_BWD"); r.no_pdl = num("TTEMB_NO_PDL");
     return r;
   }();
   return k;
@@ -239,7 +241,7 @@ inline cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, s
   cfg.gridDim = grid; cfg.blockDim = block; cfg.dynamicSmemBytes = smem; cfg.stream = s;
   cudaLaunchAttribute at[1];
   at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-  at[0].val.programmaticStreamSerializationAllowed = (exp_bits() & 32768) ? 0 : 1;
+  at[0].val.programmaticStreamSerializationAllowed = ((exp_bits() & 32768) || knobs().no_pdl) ? 0 : 1;
   cfg.attrs = at; cfg.numAttrs = 1;
   return cudaLaunchKernelEx(&cfg, kernel, static_cast<KArgs>(args)...);
 }
@@ -248,7 +250,7 @@ inline cudaError_t launch_pdl_ptr(const void* kernel, dim3 grid, dim3 block, siz
   cfg.gridDim = grid; cfg.blockDim = block; cfg.dynamicSmemBytes = smem; cfg.stream = s;
   cudaLaunchAttribute at[1];
   at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-  at[0].val.programmaticStreamSerializationAllowed = (exp_bits() & 32768) ? 0 : 1;
+  at[0].val.programmaticStreamSerializationAllowed = ((exp_bits() & 32768) || knobs().no_pdl) ? 0 : 1;
   cfg.attrs = at; cfg.numAttrs = 1;
   return cudaLaunchKernelExC(&cfg, kernel, args);
 }
