@@ -188,9 +188,22 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
     }
     tc::named_sync(1, X_LW * 32);
     if (tid == 0 && nxt < NU) issue_raw(nxt);
+    // The C1 row of this thread's B row in the NEXT tile (its grp_arow entry, loaded one tile ahead)
+    // is prefetched into L1 at the end of the current tile, and the next unit's group bounds are
+    // loaded one unit ahead, so a tile's C1 loads neither wait on grp_arow nor on DRAM.
+    const int m = tid & 63;
+    const uint32_t jm = (uint32_t)(m & ((1 << a.n1s) - 1));
+    auto arow_of = [&](uint32_t qa, uint32_t q1) {   // C1 row of B row m of the tile at qa, or ~0
+      const uint32_t np = qa < q1 ? min((uint32_t)tpp, q1 - qa) : 0u;
+      return m < (int)(np << a.n1s) ? a.grp_arow[qa + (m >> a.n1s)] + jm : 0xffffffffu;
+    };
+    uint32_t q0n = 0, q1n = 0;
+    if (nxt < NU) { q0n = a.grp_off[nxt / UPG]; q1n = a.grp_off[nxt / UPG + 1]; }
+    uint32_t q0 = 0, q1 = 0;
+    if (cur < NU) { q0 = a.grp_off[cur / UPG]; q1 = a.grp_off[cur / UPG + 1]; }
+    uint32_t arow_n = arow_of(q0, q1);
     while (cur < NU) {
       const uint32_t g = cur / UPG, ub = cur % UPG;
-      const uint32_t q0 = a.grp_off[g], q1 = a.grp_off[g + 1];
       for (uint32_t qa = q0; qa < q1; qa += tpp, ++ui) {
         const uint32_t np = min((uint32_t)tpp, q1 - qa);
         const int rows = (int)np << a.n1s;
@@ -203,14 +216,16 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
           tc::mbar_arrive(&ctl.u_full[ui & 3]);
         }
         // C1 rows of the tile -> registers (B = CM(m, r1), m = tid & 63, KR / 16 float4 of r1)
-        const int m = tid & 63;
         float4 bv[KR / 16];
         {
-          const bool ok = m < rows;
-          const uint32_t arow = ok ? a.grp_arow[qa + (m >> a.n1s)] + (m & ((1 << a.n1s) - 1)) : 0u;
-          const float4* src = reinterpret_cast<const float4*>(a.cores + (size_t)arow * KR);
+          const uint32_t arow = arow_n;
+          const bool ok = arow != 0xffffffffu;
+          const float4* src = reinterpret_cast<const float4*>(a.cores + (size_t)(ok ? arow : 0u) * KR);
 #pragma unroll
           for (int k = 0; k < KR / 16; ++k) bv[k] = (ok && !(a.dbg & 2)) ? __ldg(src + (tid >> 6) + 4 * k) : make_float4(0.f, 0.f, 0.f, 0.f);
+          (void)rows;
+          // the next tile's grp_arow entry (this group's next tile, else the next unit's first)
+          arow_n = qa + tpp < q1 ? arow_of(qa + tpp, q1) : (nxt < NU ? arow_of(q0n, q1n) : 0xffffffffu);
         }
         XTA(0);
         if (fl & 1u) {   // the unit's C2^T -> TMEM (hi = raw fp32, lo = x - trunc_tf32(x))
@@ -247,6 +262,11 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
           tc::mbar_arrive(&ctl.b_full[s]);
           XTA(4);
         }
+        if (arow_n != 0xffffffffu && !(a.dbg & 256)) {   // next tile's C1 row lines -> L1
+          const float* pf = a.cores + (size_t)arow_n * KR + 4 * (tid >> 6);
+#pragma unroll
+          for (int k = 0; k < KR / 16; k += 2) asm volatile("prefetch.global.L1 [%0];" ::"l"(pf + 16 * k));
+        }
       }
       XT0();
       // next unit: registers <- raw (nxt); raw <- the unit after (claimed now)
@@ -265,6 +285,8 @@ __global__ void __launch_bounds__(X_THREADS, 1) k_prefix_fwd(XArgs a) {
       ++gs;
       cur = nxt;
       nxt = nn;
+      q0 = q0n; q1 = q1n;
+      if (nn < NU) { q0n = a.grp_off[nn / UPG]; q1n = a.grp_off[nn / UPG + 1]; }
     }
     if (tid == 0) {
       tc::mbar_wait(&ctl.u_empty[ui & 3], ((ui >> 2) & 1) ^ 1);
