@@ -75,7 +75,7 @@ class Clocks:
                     self.rows.append([x.strip() for x in out.split(",")])
             except Exception:
                 pass
-            self._stop.wait(0.2)
+            self._stop.wait(0.05)
 
     def __enter__(self):
         self._th = threading.Thread(target=self._run, daemon=True)
@@ -384,7 +384,7 @@ def kernels_per_step(emb_ctx, world, fused=True, cfg=None, fused_update=None):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--config", default="c4")
     ap.add_argument("--rank", type=int, default=None, help="TT rank for c5 (32/64/128)")
