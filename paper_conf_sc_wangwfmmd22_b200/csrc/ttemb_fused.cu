@@ -426,7 +426,13 @@ __device__ __forceinline__ void ffma2s(float2& d, float s, float2 b) { ffma2(d, 
 #ifndef TTEMB_FWD_ROWS_BLOCKS
 #define TTEMB_FWD_ROWS_BLOCKS 3   // k_rows_fwd2 CTAs per SM at n3 = 4, R = 64 (register cap 85)
 #endif
-constexpr int RW_WARPS = 8, RW_RCH = 16, RW_NSL = 3;
+#ifndef TTEMB_RF_NSL
+#define TTEMB_RF_NSL 3   // ring slots of k_rows_fwd2 (rows in flight + 1)
+#endif
+#ifndef TTEMB_RB_NSL
+#define TTEMB_RB_NSL 3   // ring slots of k_rows_bwd2
+#endif
+constexpr int RW_WARPS = 8, RW_RCH = 16, RW_NSL = TTEMB_RF_NSL, RB_NSL = TTEMB_RB_NSL;
 
 struct RowArgs {
   const float* cores;
@@ -621,7 +627,7 @@ __global__ void __launch_bounds__(RW_WARPS * 32, RL == 1 ? 3 : 2) k_rows_bwd2(Ro
   constexpr int JM = J12T ? J12T : RB_J12;      // unrolled j12 extent
   extern __shared__ __align__(16) float rw_smem[];
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  float* const ringp = rw_smem + w * (RW_NSL * SLOT);
+  float* const ringp = rw_smem + w * (RB_NSL * SLOT);
   const uint32_t ring = tc::smem_u32(ringp);
   const uint32_t U = tt_rows(a.counts);   // TT rows only (hybrid: dense rows follow)
   const int J12 = J12T ? J12T : a.n1 * a.n2;
@@ -655,15 +661,15 @@ __global__ void __launch_bounds__(RW_WARPS * 32, RL == 1 ? 3 : 2) k_rows_bwd2(Ro
       if (a.exp & 512) return;
       const unsigned long long o3 = __shfl_sync(0xffffffffu, o3l, j) + (unsigned long long)(RL * lane) * N3;
       const float4* src = reinterpret_cast<const float4*>(a.cores + o3);
-      const uint32_t dst = ring + (uint32_t)((j % RW_NSL) * SLOT * 4) + 16u * lane;
+      const uint32_t dst = ring + (uint32_t)((j % RB_NSL) * SLOT * 4) + 16u * lane;
 #pragma unroll
       for (int i = 0; i < C3L; ++i) tc::cp_async16(dst + 16u * 32u * i, src + i);
       if (lane < a.N / 4)
-        tc::cp_async16(ring + (uint32_t)(((j % RW_NSL) * SLOT + C3S) * 4) + 16u * lane,
+        tc::cp_async16(ring + (uint32_t)(((j % RB_NSL) * SLOT + C3S) * 4) + 16u * lane,
                        reinterpret_cast<const float4*>(a.gbuf + (size_t)(u0 + j) * a.N) + lane);
     };
 #pragma unroll
-    for (int j = 0; j < RW_NSL - 1; ++j) {
+    for (int j = 0; j < RB_NSL - 1; ++j) {
       if (j < nr) issue(j);
       tc::cp_commit();
     }
@@ -713,9 +719,9 @@ __global__ void __launch_bounds__(RW_WARPS * 32, RL == 1 ? 3 : 2) k_rows_bwd2(Ro
         }
         curq = q;
       }
-      tc::cp_wait<RW_NSL - 2>();
+      tc::cp_wait<RB_NSL - 2>();
       __syncwarp();
-      const float* slot = ringp + (j % RW_NSL) * SLOT;
+      const float* slot = ringp + (j % RB_NSL) * SLOT;
       // C3[rl + x][b] for the lane's r; c3x[b] = (C3[rl][b], C3[rl + 1][b]) pairs the lane's two r
       float c3[RL][N3];
       float2 dc[RL][N3 / 2];
@@ -759,7 +765,7 @@ __global__ void __launch_bounds__(RW_WARPS * 32, RL == 1 ? 3 : 2) k_rows_bwd2(Ro
         }
       }
       __syncwarp();
-      if (j + RW_NSL - 1 < nr) issue(j + RW_NSL - 1);
+      if (j + RB_NSL - 1 < nr) issue(j + RB_NSL - 1);
       tc::cp_commit();
       // dC3[i3_u][rl + x][0 .. n3): RL n3 consecutive floats per lane
       float* d3 = a.grads + __shfl_sync(0xffffffffu, o3l, j) + (size_t)(RL * lane) * N3;
@@ -776,7 +782,7 @@ __global__ void __launch_bounds__(RW_WARPS * 32, RL == 1 ? 3 : 2) k_rows_bwd2(Ro
   }
 }
 
-size_t rows_bwd_smem(int n3, int sw) { return (size_t)RW_WARPS * RW_NSL * (sw * n3 + RB_J12 * n3) * 4; }   // per sw-wide r slice
+size_t rows_bwd_smem(int n3, int sw) { return (size_t)RW_WARPS * RB_NSL * (sw * n3 + RB_J12 * n3) * 4; }   // per sw-wide r slice
 
 // (n3, R, n1 n2) -> k_rows_bwd2 instantiation (n1 n2 = 16 unrolled exactly, others predicated)
 template <int N3, int RL, int KR> const void* rows_bwd_pick(int j12) {
