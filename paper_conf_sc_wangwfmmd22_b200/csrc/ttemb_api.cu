@@ -231,6 +231,10 @@ size_t carve(Ctx& c, uint8_t* base) {
   const size_t pf = tc_eligible(c) ? (size_t)P * c.n1 * c.NC : 1;
   p.pbuf = k.take<float>(pf);
   p.dpbuf = k.take<float>(pf);
+  // dC2 per group for the fused Adagrad pass (overwritten every step, so the C2 part of the
+  // gradient buffer stays zero and needs no clearing); only the tensor-core path with Adagrad
+  p.dc2buf = k.take<float>(tc_eligible(c) && c.opt == TTEMB_ADAGRAD && (c.flags & TTEMB_FUSED_UPDATE)
+                               ? (size_t)NG * c.R * c.NC : 1);
   p.wpos = k.take<float>(nnz);
   p.rows = k.take<float>((size_t)U * c.N);
   p.gbuf = k.take<float>((size_t)U * c.N);

@@ -21,7 +21,7 @@
 // C2 slice is updated in place by reductions straight from TMEM (the paper's fused TT core
 // update; the slice has no other reader once its last tile's MMAs completed); for
 // Adagrad (read-modify-write of the slice and its state) or unfused, dC2 is stored and fused
-// Adagrad finishes in k_c2_update_zero.
+// Adagrad writes dC2 to a per-group scratch and finishes in k_c2_update.
 // fp32 accuracy: 3xTF32 (hi = raw fp32, read by the tensor core with truncation; lo =
 // x - trunc_tf32(x)); scripts/tc_probe3.cu measures the TMEM-A form.
 //
@@ -84,6 +84,7 @@ struct YArgs {
   const unsigned long long* grp_c2;       // [NG] float offset of the group's C2 slice
   unsigned long long c2_begin;            // float offset of the C2 region (tm_c2 row 0)
   const float* dpbuf;                     // [P][n1][NC]
+  float* dc2buf;                          // fused Adagrad: dC2 of group g at g R NC (slice layout)
   const uint32_t* unit_snake;             // [NU] unit at static position p (balanced by tile count)
   uint32_t* work;
   int n1, n1s, NC, nblk, tpp, nchunk, R;
@@ -449,12 +450,17 @@ k_prefix_bwd(const __grid_constant__ CUtensorMap tm_dp, const __grid_constant__ 
             tc::tmem_ld32(tc::taddr(tm + S::T_DC2 + blk * KR + 32 * h, 32 * Q, 0), v);
             if (c < NC && !(a.exp & 1)) {
               const size_t base = so + (size_t)(32 * h) * NC + c;
-              if (!a.fused || a.opt != TTEMB_SGD) {
-                // unfused, or fused Adagrad: dC2 to the gradient buffer (plain coalesced stores);
-                // Adagrad's read-modify-write of C2 and its state runs after the kernel as a
-                // bandwidth-bound pass over the touched slices (k_c2_update_zero)
+              if (!a.fused) {
+                // unfused: dC2 to the gradient buffer (plain coalesced stores)
 #pragma unroll
                 for (int i = 0; i < 32; ++i) a.grads[base + (size_t)i * NC] = v[i];
+              } else if (a.opt != TTEMB_SGD) {
+                // fused Adagrad: dC2 to the per-group scratch (same slice layout); the read-modify-
+                // write of C2 and its state runs after the kernel as a bandwidth-bound pass over the
+                // touched slices (k_c2_update), which never has to clear it
+                float* d = a.dc2buf + (size_t)g * KR * NC + (base - so);
+#pragma unroll
+                for (int i = 0; i < 32; ++i) d[(size_t)i * NC] = v[i];
               } else {
                 // C2 -= lr dC2 as fire-and-forget reductions (each warp instruction covers 32
                 // consecutive floats): no read of the old slice, no load latency on this path
@@ -518,16 +524,16 @@ k_prefix_bwd(const __grid_constant__ CUtensorMap tm_dp, const __grid_constant__ 
 
 }  // namespace
 
-// Fused Adagrad for the C2 slices the prefix-backward kernel wrote to the gradient buffer:
-// s += g^2, C2 -= lr g / (sqrt(s) + eps), g = 0 (keeps the fused-mode accumulators zero).
+// Fused Adagrad for the C2 slices, from the dC2 the prefix-backward kernel wrote to the per-group
+// scratch: s += g^2, C2 -= lr g / (sqrt(s) + eps).
 __global__ void __launch_bounds__(256)
-k_c2_update_zero(float* __restrict__ cores, float* __restrict__ state, float* __restrict__ grads,
-                 const unsigned long long* __restrict__ grp_c2, const uint32_t* __restrict__ counts,
-                 uint32_t slice, float lr, float eps) {
+k_c2_update(float* __restrict__ cores, float* __restrict__ state, const float* __restrict__ dc2,
+            const unsigned long long* __restrict__ grp_c2, const uint32_t* __restrict__ counts,
+            uint32_t slice, float lr, float eps) {
   const size_t n4 = (size_t)counts[kCntNG] * (slice / 4);
   for (size_t e = (size_t)blockIdx.x * blockDim.x + threadIdx.x; e < n4; e += (size_t)gridDim.x * blockDim.x) {
     const size_t gi = e / (slice / 4), o = grp_c2[gi] + 4 * (e % (slice / 4));
-    float4 g = *reinterpret_cast<float4*>(grads + o);
+    const float4 g = __ldcs(reinterpret_cast<const float4*>(dc2) + e);
     float4 p = *reinterpret_cast<float4*>(cores + o);
     float4 st = *reinterpret_cast<float4*>(state + o);
     st.x += g.x * g.x; st.y += g.y * g.y; st.z += g.z * g.z; st.w += g.w * g.w;
@@ -535,7 +541,6 @@ k_c2_update_zero(float* __restrict__ cores, float* __restrict__ state, float* __
     p.z -= lr * g.z / (sqrtf(st.z) + eps); p.w -= lr * g.w / (sqrtf(st.w) + eps);
     *reinterpret_cast<float4*>(state + o) = st;
     *reinterpret_cast<float4*>(cores + o) = p;
-    *reinterpret_cast<float4*>(grads + o) = make_float4(0.f, 0.f, 0.f, 0.f);
   }
 }
 
@@ -589,7 +594,7 @@ cudaError_t run_prefix_bwd(Ctx& c, float lr, cudaStream_t s) {
   YArgs a;
   a.cores = c.cores; a.grads = c.grads; a.state = c.state; a.meta = c.d_meta; a.counts = p.counts;
   a.grp_off = p.grp_off; a.grp_t = p.grp_t; a.pfx_i1 = p.pfx_i1; a.pfx_t = p.pfx_t; a.grp_arow = p.grp_arow;
-  a.grp_c2 = p.grp_c2; a.dpbuf = p.dpbuf; a.work = p.work + 2; a.c2_begin = c.c1_floats;
+  a.grp_c2 = p.grp_c2; a.dpbuf = p.dpbuf; a.work = p.work + 2; a.c2_begin = c.c1_floats; a.dc2buf = p.dc2buf;
   a.unit_snake = p.unit_snake;
   a.n1 = c.n1; a.n1s = c.n1 == 1 ? 0 : c.n1 == 2 ? 1 : c.n1 == 4 ? 2 : 3;
   a.NC = c.NC; a.nblk = (c.NC + 127) / 128; a.tpp = YT / c.n1; a.R = c.R;
@@ -612,8 +617,8 @@ cudaError_t run_prefix_bwd(Ctx& c, float lr, cudaStream_t s) {
   else if (c.R == 64) launch_pdl(k_prefix_bwd<64>, dim3(grid), dim3(Y_THREADS), YShape<64>::SMEM, s, c.tm_dp, c.tm_c2, a);
   else launch_pdl(k_prefix_bwd<128>, dim3(grid), dim3(Y_THREADS), YShape<128>::SMEM, s, c.tm_dp, c.tm_c2, a);
   if (a.fused && a.opt != TTEMB_SGD)
-    k_c2_update_zero<<<c.sm_count * 8, 256, 0, s>>>(c.cores, c.state, c.grads, p.grp_c2, p.counts,
-                                                    (uint32_t)(c.R * c.NC), lr, c.eps);
+    k_c2_update<<<c.sm_count * 8, 256, 0, s>>>(c.cores, c.state, p.dc2buf, p.grp_c2, p.counts,
+                                               (uint32_t)(c.R * c.NC), lr, c.eps);
   if (a.trace) {
     std::vector<unsigned long long> hb(32 * grid);
     cudaMemcpyAsync(hb.data(), trace, hb.size() * 8, cudaMemcpyDeviceToHost, s);

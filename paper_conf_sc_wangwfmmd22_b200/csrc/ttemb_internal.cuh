@@ -106,6 +106,7 @@ struct PlanDev {
   float *rows, *gbuf, *dabuf, *aggpart;
   float* wpos;                                 // [nnz] bag weight of every position (weighted/mean bags)
   float *pbuf, *dpbuf;                         // tensor-core path: P and dL/dP per prefix
+  float* dc2buf;                               // fused Adagrad (tensor-core path): dC2 per group [NG][R NC]
   uint32_t* grp_arow;                          // [P]  C1 row (float offset / R) of sorted prefix q, j1 = 0
   uint32_t *chunk_off, *split_list;            // FFMA path: [NG+1] first unit of group g; [NG] split groups
   unsigned long long* grp_c2;                  // [NG] float offset of the C2 slice of group g
