@@ -359,6 +359,38 @@ def test_deterministic_forward_and_plan():
         assert torch.equal(p1[k], p2[k])
 
 
+def test_pdl_launch_order_does_not_change_results(tmp_path):
+    """The main chain is launched with programmatic dependent launch; with it switched off
+    (TTEMB_NO_PDL=1, read once per process, hence the subprocesses) the forward output -- which
+    has no atomics, so it is deterministic -- is bitwise equal (c4 shapes, B = 1024)."""
+    import os
+    import subprocess
+    import sys
+    code = (
+        "import sys, numpy as np, torch\n"
+        "sys.path.insert(0, {root!r})\n"
+        "import paper_conf_sc_wangwfmmd22_b200 as tt\n"
+        "from synth import workload as W\n"
+        "cfg = W.config('c4'); B = 1024\n"
+        "idx, off = W.make_batch(cfg, seed=3, batch=B)\n"
+        "emb = tt.TTEmbeddingBag(cfg.table_rows, cfg.row_factors, cfg.col_factors, cfg.rank, B, len(idx))\n"
+        "emb.load_cores(W.make_cores(cfg, seed=3))\n"
+        "d = torch.device('cuda', 0)\n"
+        "out = emb.forward(torch.as_tensor(idx, device=d), torch.as_tensor(off, device=d), B)\n"
+        "np.save({out!r}, out.cpu().numpy())\n"
+    )
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    res = []
+    for flag in ("0", "1"):
+        f = str(tmp_path / f"out{flag}.npy")
+        env = dict(os.environ, TTEMB_NO_PDL=flag)
+        r = subprocess.run([sys.executable, "-c", code.format(root=root, out=f)], env=env, cwd=root,
+                           capture_output=True, text=True, timeout=300)
+        assert r.returncode == 0, r.stderr[-2000:]
+        res.append(np.load(f))
+    np.testing.assert_array_equal(res[0], res[1])
+
+
 def test_edge_cases_empty_and_range_errors():
     cfg = W.small_config([100, 50], [(5, 5, 4), (4, 4, 4)], (2, 2, 2), 4, 8, 1)
     cores = W.make_cores(cfg, seed=0)
