@@ -30,7 +30,6 @@ namespace ttemb {
 
 namespace {
 
-constexpr int XR = 64;                         // TT rank = K of the prefix GEMM
 constexpr int XT = 64;                         // tile rows (prefix, j1) = MMA N (max)
 constexpr int X_LW = 8, X_RW = 4;   // loaders, epilogue warps
 constexpr int X_THREADS = (X_LW + 1 + X_RW) * 32;
