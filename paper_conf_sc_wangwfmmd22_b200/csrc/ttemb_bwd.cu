@@ -21,7 +21,10 @@ namespace ttemb {
 namespace {
 
 constexpr int AGG_CS = 32;   // sorted positions per aggregation chunk
-constexpr int AGG_B = 8;     // grad_out rows per lane group loaded ahead in k_agg_scatter
+#ifndef TTEMB_AGG_B
+#define TTEMB_AGG_B 8
+#endif
+constexpr int AGG_B = TTEMB_AGG_B;   // grad_out rows per lane group loaded ahead in k_agg_scatter
 
 __device__ __forceinline__ void apply_update(float* param, float* state, float g, float lr,
                                              float eps, int opt) {
