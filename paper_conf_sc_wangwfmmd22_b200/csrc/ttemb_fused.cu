@@ -422,6 +422,9 @@ __device__ __forceinline__ void ffma2(float2& d, float2 a, float2 b) {
 }
 __device__ __forceinline__ void ffma2s(float2& d, float s, float2 b) { ffma2(d, make_float2(s, s), b); }
 
+#ifndef TTEMB_FWD_ROWS_GRID
+#define TTEMB_FWD_ROWS_GRID 4     // k_rows_fwd2 grid cap, CTAs per SM
+#endif
 #ifndef TTEMB_FWD_ROWS_BLOCKS
 #define TTEMB_FWD_ROWS_BLOCKS 3   // k_rows_fwd2 CTAs per SM at n3 = 4, R = 64 (register cap 85)
 #endif
@@ -971,7 +974,7 @@ cudaError_t run_fused_fwd(Ctx& c, float* out, cudaStream_t s) {
     r.cores = c.cores; r.meta = c.d_meta; r.counts = p.counts; r.row_pfx = p.row_pfx; r.row_c3 = p.row_c3;
     r.c3_begin = c.c3_begin; r.pfx_t = p.pfx_t; r.pbuf = p.pbuf; r.rows = p.rows; r.seg_off = p.seg_off; r.sbag = p.sbag; r.out = out;
     r.n1 = c.n1; r.n1s = a.n1s; r.n2 = c.n2; r.N = c.N; r.NC = c.NC;
-    const int grid = grid_for(c, cdiv(c.U_cap, RW_RCH), RW_WARPS, 4);
+    const int grid = grid_for(c, cdiv(c.U_cap, RW_RCH), RW_WARPS, TTEMB_FWD_ROWS_GRID);
     const dim3 g(grid), b(RW_WARPS * 32);
     if (c.R == 32) {
       if (c.n3 == 4) launch_pdl(k_rows_fwd2<4, 4>, g, b, rows_smem(4, 32), s, r);
