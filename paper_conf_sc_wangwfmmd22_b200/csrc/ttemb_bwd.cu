@@ -21,6 +21,12 @@ namespace ttemb {
 namespace {
 
 constexpr int AGG_CS = 32;   // sorted positions per aggregation chunk
+#ifndef TTEMB_UPD_GRID
+#define TTEMB_UPD_GRID 8    // fused C1 / C3 update grid cap, CTAs per SM
+#endif
+#ifndef TTEMB_AGG_GRID
+#define TTEMB_AGG_GRID 32   // k_agg_scatter grid cap, CTAs per SM
+#endif
 #ifndef TTEMB_AGG_B
 #define TTEMB_AGG_B 8
 #endif
@@ -354,7 +360,7 @@ cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s
     StageScope sc(c, ST_AGG, s);
     if (agg_scatter_path(c)) {
       // (G was zeroed at the end of the index stage: run_plan_tail)
-      launch_pdl(k_agg_scatter, dim3(grid_for(c, cdiv(c.nnz, 32), 8, 32)), dim3(256), 0, s, grad_out,
+      launch_pdl(k_agg_scatter, dim3(grid_for(c, cdiv(c.nnz, 32), 8, TTEMB_AGG_GRID)), dim3(256), 0, s, grad_out,
                  (const uint32_t*)p.sbag, (const uint32_t*)p.spos, (const uint32_t*)p.inverse, (int64_t)c.nnz, c.N,
                  p.gbuf, (const float*)(c.weighted ? p.wpos : nullptr), (const uint32_t*)p.counts);
     } else {
@@ -403,7 +409,7 @@ cudaError_t run_backward(Ctx& c, const float* grad_out, float lr, cudaStream_t s
   if (fused) {   // C2 was updated inside the group kernel; C1 and C3 densely here
     StageScope sc(c, ST_UPD_C3, s);
     if (c.c1_floats % 4 == 0 && c.c3_begin % 4 == 0 && c.c3_floats % 4 == 0)
-      launch_pdl(k_update_zero4, dim3(grid_for(c, (int64_t)(c.c1_floats + c.c3_floats) / 4, 256, 8)), dim3(256), 0, s,
+      launch_pdl(k_update_zero4, dim3(grid_for(c, (int64_t)(c.c1_floats + c.c3_floats) / 4, 256, TTEMB_UPD_GRID)), dim3(256), 0, s,
                  c.cores, c.state, c.grads, (size_t)c.c1_floats, (size_t)c.c3_begin, (size_t)c.c3_floats, lr, c.eps, c.opt);
     else
       k_update_zero<<<grid_for(c, (int64_t)(c.c1_floats + c.c3_floats), 256, 32), 256, 0, s>>>(
